@@ -1,0 +1,502 @@
+/*
+ * abft_oracle.c -- CPU ORACLE (test infrastructure only; see abft_oracle.h).
+ *
+ * Plain, slow, obviously correct.  No blocking, fusion or reordering beyond
+ * what the paper (or a DESIGN.md reading) states.  Shares nothing with
+ * paper_conf_dsn_schollbkw16_b200/csrc/.
+ *
+ * Build: gcc -std=c99 -O2 -ffp-contract=off -fno-fast-math -shared -fPIC -lm
+ */
+#include "abft_oracle.h"
+
+#include <math.h>
+#include <stdlib.h>
+#include <string.h>
+
+/* ------------------------------------------------------------------------ */
+/* R2: canonical pairwise summation PW.                                      */
+/* PW(v_0..v_{n-1}) is the balanced binary tree over the list padded to the  */
+/* next power of two, where padding slots are ABSENT (a node with one absent */
+/* child is its other child, unchanged).  PW of an empty list is +0.0.       */
+/* The paper fixes no order for its inner products ("reductions", */
+/* P:164); this reading makes every result bit-reproducible.                 */
+/* ------------------------------------------------------------------------ */
+static int pw_node(const double *v, const unsigned char *present, int64_t n, int64_t lo,
+                   int64_t size, double *out) {
+  if (lo >= n) return 0; /* absent */
+  if (size == 1) {
+    if (present && !present[lo]) return 0;
+    *out = v[lo];
+    return 1;
+  }
+  double l = 0.0, r = 0.0;
+  int hl = pw_node(v, present, n, lo, size / 2, &l);
+  int hr = pw_node(v, present, n, lo + size / 2, size / 2, &r);
+  if (hl && hr) {
+    *out = l + r;
+    return 1;
+  }
+  if (hl) {
+    *out = l;
+    return 1;
+  }
+  if (hr) {
+    *out = r;
+    return 1;
+  }
+  return 0;
+}
+
+double or_pw_slots(const double *v, const unsigned char *present, int64_t n) {
+  int64_t size = 1;
+  double out = 0.0;
+  while (size < n) size *= 2;
+  if (!pw_node(v, present, n, 0, size, &out)) return 0.0; /* empty sum */
+  return out;
+}
+
+double or_pw(const double *v, int64_t n) { return or_pw_slots(v, NULL, n); }
+
+/* ------------------------------------------------------------------------ */
+/* SpMV (Fig. 1 step 1): y_i = sum_j a_ij * x_j, summed by PW over the */
+/* row's entries in CSR order (R3).                                          */
+/* ------------------------------------------------------------------------ */
+double or_row_dot(const or_csr *A, int64_t i, const double *x) {
+  int64_t b = A->row_ptr[i], e = A->row_ptr[i + 1];
+  double *p = (double *)malloc(sizeof(double) * (size_t)(e > b ? e - b : 1));
+  for (int64_t q = b; q < e; ++q) p[q - b] = A->val[q] * x[A->col[q]];
+  double r = or_pw(p, e - b);
+  free(p);
+  return r;
+}
+
+void or_spmv(const or_csr *A, const double *x, double *y) {
+  for (int64_t i = 0; i < A->n; ++i) y[i] = or_row_dot(A, i, x);
+}
+
+/* ------------------------------------------------------------------------ */
+/* Encoding, structure (Fig. 2; Fig. 3 step 1): row k of C */
+/* holds the columns of row block A_k that contain at least one element     */
+/* (structural, R5), ascending.  Blocks are rows k*bs .. min((k+1)*bs,N)-1  */
+/* (P:80, 0-based per R4).                                                    */
+/* ------------------------------------------------------------------------ */
+static int cmp_i32(const void *a, const void *b) {
+  int32_t x = *(const int32_t *)a, y = *(const int32_t *)b;
+  return (x > y) - (x < y);
+}
+
+int64_t or_encode_structure(const or_csr *A, int32_t bs, int32_t *c_row_ptr, int32_t *c_col) {
+  int64_t n = A->n, nb = (n + bs - 1) / bs;
+  int64_t *seen = (int64_t *)malloc(sizeof(int64_t) * (size_t)(n > 0 ? n : 1));
+  int32_t *tmp = (int32_t *)malloc(sizeof(int32_t) * (size_t)(n > 0 ? n : 1));
+  for (int64_t j = 0; j < n; ++j) seen[j] = -1;
+  int64_t total = 0;
+  c_row_ptr[0] = 0;
+  for (int64_t k = 0; k < nb; ++k) {
+    int64_t cnt = 0;
+    for (int64_t i = k * bs; i < (k + 1) * bs && i < n; ++i)
+      for (int64_t q = A->row_ptr[i]; q < A->row_ptr[i + 1]; ++q) {
+        int32_t j = A->col[q];
+        if (seen[j] != k) {
+          seen[j] = k;
+          tmp[cnt++] = j;
+        }
+      }
+    qsort(tmp, (size_t)cnt, sizeof(int32_t), cmp_i32);
+    if (c_col) memcpy(c_col + total, tmp, sizeof(int32_t) * (size_t)cnt);
+    total += cnt;
+    c_row_ptr[k + 1] = (int32_t)total;
+  }
+  free(seen);
+  free(tmp);
+  return total;
+}
+
+/* Find a_ij in row i (binary search over the ascending columns); 1 if present. */
+static int find_entry(const or_csr *A, int64_t i, int32_t j, double *out) {
+  int64_t lo = A->row_ptr[i], hi = A->row_ptr[i + 1];
+  while (lo < hi) {
+    int64_t mid = lo + (hi - lo) / 2;
+    if (A->col[mid] < j)
+      lo = mid + 1;
+    else
+      hi = mid;
+  }
+  if (lo < A->row_ptr[i + 1] && A->col[lo] == j) {
+    *out = A->val[lo];
+    return 1;
+  }
+  return 0;
+}
+
+/* Encoding, values: c_k = w_k^T A_k with w_k = (1..1)  */
+/* (R1), i.e. c_kj = sum over the b_s row slots of block k of a_ij,   */
+/* summed by PW over the slots, absent where row i has no entry j or i >= N */
+/* (R4').                                                                     */
+void or_encode_values(const or_csr *A, int32_t bs, const int32_t *c_row_ptr,
+                      const int32_t *c_col, double *c_val) {
+  int64_t n = A->n, nb = (n + bs - 1) / bs;
+  double *slot = (double *)malloc(sizeof(double) * (size_t)bs);
+  unsigned char *pres = (unsigned char *)malloc((size_t)bs);
+  for (int64_t k = 0; k < nb; ++k)
+    for (int64_t q = c_row_ptr[k]; q < c_row_ptr[k + 1]; ++q) {
+      for (int32_t s = 0; s < bs; ++s) {
+        int64_t i = k * bs + s;
+        pres[s] = 0;
+        slot[s] = 0.0;
+        if (i < n) pres[s] = (unsigned char)find_entry(A, i, c_col[q], &slot[s]);
+      }
+      c_val[q] = or_pw_slots(slot, pres, bs);
+    }
+  free(slot);
+  free(pres);
+}
+
+/* Encoding, bound constants: the sparse bound                   */
+/*   tau_k(beta) = ((n_k + 2 b_s - 2) * sum_{i in k} ||a_i||_2                 */
+/*                  + n_k * ||c_k||_2) * eps_M * beta,   eps_M = 2^-53 */
+/* is split into K_k (everything but beta, computed once per matrix) and    */
+/* tau_k = K_k * beta (R7, R11).  The row sum runs over the b_s slots with  */
+/* absent slots past N (R3'); ||.||_2 = sqrt(PW of squares) (R6).            */
+void or_encode_bound(const or_csr *A, int32_t bs, const int32_t *c_row_ptr,
+                     const double *c_val, double *K, double *row_norm, double *S_out,
+                     double *c_norm) {
+  int64_t n = A->n, nb = (n + bs - 1) / bs;
+  double *rn = (double *)malloc(sizeof(double) * (size_t)(n > 0 ? n : 1));
+  for (int64_t i = 0; i < n; ++i) {
+    int64_t b = A->row_ptr[i], e = A->row_ptr[i + 1];
+    double *sq = (double *)malloc(sizeof(double) * (size_t)(e > b ? e - b : 1));
+    for (int64_t q = b; q < e; ++q) sq[q - b] = A->val[q] * A->val[q];
+    rn[i] = sqrt(or_pw(sq, e - b));
+    free(sq);
+    if (row_norm) row_norm[i] = rn[i];
+  }
+  double *slot = (double *)malloc(sizeof(double) * (size_t)bs);
+  unsigned char *pres = (unsigned char *)malloc((size_t)bs);
+  const double eps_m = ldexp(1.0, -53);
+  for (int64_t k = 0; k < nb; ++k) {
+    for (int32_t s = 0; s < bs; ++s) {
+      int64_t i = k * bs + s;
+      pres[s] = (unsigned char)(i < n);
+      slot[s] = i < n ? rn[i] : 0.0;
+    }
+    double S = or_pw_slots(slot, pres, bs);
+    int64_t cb = c_row_ptr[k], ce = c_row_ptr[k + 1];
+    double *sq = (double *)malloc(sizeof(double) * (size_t)(ce > cb ? ce - cb : 1));
+    for (int64_t q = cb; q < ce; ++q) sq[q - cb] = c_val[q] * c_val[q];
+    double cn = sqrt(or_pw(sq, ce - cb));
+    free(sq);
+    double n_k = (double)(ce - cb);
+    double m_k = n_k + 2.0 * (double)bs - 2.0;
+    K[k] = (m_k * S + n_k * cn) * eps_m;
+    if (S_out) S_out[k] = S;
+    if (c_norm) c_norm[k] = cn;
+  }
+  free(slot);
+  free(pres);
+  free(rn);
+}
+
+/* ------------------------------------------------------------------------ */
+/* Fault model.                                                               */
+/* Philox4x32-10 (Salmon et al., SC'11), the counter-based generator both    */
+/* sides implement independently (task rule ③).                              */
+/* ------------------------------------------------------------------------ */
+void or_philox4x32_10(const uint32_t ctr[4], const uint32_t key[2], uint32_t out[4]) {
+  uint32_t c0 = ctr[0], c1 = ctr[1], c2 = ctr[2], c3 = ctr[3];
+  uint32_t k0 = key[0], k1 = key[1];
+  for (int r = 0; r < 10; ++r) {
+    uint64_t p0 = (uint64_t)0xD2511F53u * c0;
+    uint64_t p1 = (uint64_t)0xCD9E8D57u * c2;
+    uint32_t hi0 = (uint32_t)(p0 >> 32), lo0 = (uint32_t)p0;
+    uint32_t hi1 = (uint32_t)(p1 >> 32), lo1 = (uint32_t)p1;
+    uint32_t n0 = hi1 ^ c1 ^ k0;
+    uint32_t n1 = lo1;
+    uint32_t n2 = hi0 ^ c3 ^ k1;
+    uint32_t n3 = lo0;
+    c0 = n0;
+    c1 = n1;
+    c2 = n2;
+    c3 = n3;
+    k0 += 0x9E3779B9u;
+    k1 += 0xBB67AE85u;
+  }
+  out[0] = c0;
+  out[1] = c1;
+  out[2] = c2;
+  out[3] = c3;
+}
+
+/* Burst length: "randomly chosen from a normal distribution with    */
+/* mean = 3 and variance = 2", read as L = max(1, round(3 + sqrt(2) Z)) (R12).*/
+/* T[l] = floor(2^32 * P(L <= l)), P(L <= l) = Phi((l + 0.5 - 3)/sqrt 2)     */
+/*      = erfc(-(l - 2.5)/2) / 2 for l = 1..63; T[64] = 2^32; T[0] = 0.       */
+void or_burst_table(uint64_t T[65]) {
+  T[0] = 0;
+  for (int l = 1; l < 64; ++l) {
+    double p = 0.5 * erfc(-((double)l - 2.5) / 2.0);
+    T[l] = (uint64_t)floor(ldexp(p, 32));
+  }
+  T[64] = (uint64_t)1 << 32;
+}
+
+static uint64_t burst_from_words(uint32_t w_start, uint32_t w_len) {
+  static uint64_t T[65];
+  static int init = 0;
+  if (!init) {
+    or_burst_table(T);
+    init = 1;
+  }
+  int start = (int)(w_start & 63u);
+  int len = 1;
+  while (len < 64 && (uint64_t)w_len >= T[len]) ++len;
+  int hi = start + len - 1;
+  if (hi > 63) hi = 63;
+  uint64_t m = 0;
+  for (int b = start; b <= hi; ++b) m |= (uint64_t)1 << b;
+  return m;
+}
+
+/* The XOR mask for the value produced for (round, target, index).
+ * List mode: XOR of all plan entries that match.  Rate mode (R13):
+ * each produced value is faulty with probability p = min(1, lambda * ops),
+ * decided by Philox(ctr = {index lo, index hi, call, round<<8 | target},
+ * key = {seed lo, seed hi}): faulty iff out[0] < floor(p * 2^32); then
+ * burst start = out[1] & 63 and length from out[2] via T (R12). */
+uint64_t or_fault_mask(const or_inject *inj, int32_t round, int32_t target, int64_t index,
+                       int64_t ops) {
+  if (!inj || inj->mode == OR_INJ_NONE) return 0;
+  if (inj->mode == OR_INJ_LIST) {
+    uint64_t m = 0;
+    for (int64_t e = 0; e < inj->n_list; ++e)
+      if (inj->list_round[e] == round && inj->list_target[e] == target &&
+          inj->list_index[e] == index)
+        m ^= inj->list_mask[e];
+    return m;
+  }
+  if (!(inj->targets & (1u << target))) return 0;
+  double p = inj->lambda * (double)ops;
+  uint64_t thr = p >= 1.0 ? ((uint64_t)1 << 32) : (uint64_t)(p * 4294967296.0);
+  uint32_t ctr[4] = {(uint32_t)(uint64_t)index, (uint32_t)((uint64_t)index >> 32),
+                     (uint32_t)inj->call, ((uint32_t)round << 8) | (uint32_t)target};
+  uint32_t key[2] = {(uint32_t)inj->seed, (uint32_t)(inj->seed >> 32)};
+  uint32_t w[4];
+  or_philox4x32_10(ctr, key, w);
+  if ((uint64_t)w[0] >= thr) return 0;
+  return burst_from_words(w[1], w[2]);
+}
+
+static double xor_double(double v, uint64_t m) {
+  uint64_t u;
+  memcpy(&u, &v, 8);
+  u ^= m;
+  memcpy(&v, &u, 8);
+  return v;
+}
+
+/* ------------------------------------------------------------------------ */
+/* Protected SpMV, Fig. 1:                                          */
+/*  1. y = A x  and  t1 = C x                                                 */
+/*  2. beta = ||x||_2  and  t2_k = w_k^T y_k                                  */
+/*  3. s = t1 - t2                                                            */
+/*  4. flag k iff NOT(|s_k| <= tau_k)   (pass condition R5'/Q5)       */
+/*  5. recompute only the flagged blocks, re-verify (R11')     */
+/* Faults are applied to the produced value before it is used.  */
+/* ------------------------------------------------------------------------ */
+static double block_t1(const int32_t *c_row_ptr, const int32_t *c_col, const double *c_val,
+                       int64_t k, const double *x) {
+  int64_t b = c_row_ptr[k], e = c_row_ptr[k + 1];
+  double *p = (double *)malloc(sizeof(double) * (size_t)(e > b ? e - b : 1));
+  for (int64_t q = b; q < e; ++q) p[q - b] = c_val[q] * x[c_col[q]];
+  double r = or_pw(p, e - b);
+  free(p);
+  return r;
+}
+
+static double block_t2(const double *y, int64_t n, int32_t bs, int64_t k, double *slot,
+                       unsigned char *pres) {
+  for (int32_t s = 0; s < bs; ++s) {
+    int64_t i = k * bs + s;
+    pres[s] = (unsigned char)(i < n);
+    slot[s] = i < n ? y[i] : 0.0;
+  }
+  return or_pw_slots(slot, pres, bs);
+}
+
+static int64_t rows_in_block(int64_t n, int32_t bs, int64_t k) {
+  int64_t e = (k + 1) * bs < n ? (k + 1) * bs : n;
+  return e - k * bs;
+}
+
+/* Compute y rows, t1_k, t2_k and the decision for block k in `round`. */
+static int check_block(const or_csr *A, int32_t bs, const int32_t *c_row_ptr,
+                       const int32_t *c_col, const double *c_val, const double *K,
+                       const double *x, double beta, const or_inject *inj, int32_t round,
+                       int64_t k, double *y, double *t1, double *t2, double *s, double *slot,
+                       unsigned char *pres) {
+  int64_t n = A->n;
+  for (int64_t i = k * bs; i < (k + 1) * bs && i < n; ++i) {
+    double v = or_row_dot(A, i, x);
+    int64_t ops = 2 * (int64_t)(A->row_ptr[i + 1] - A->row_ptr[i]);
+    y[i] = xor_double(v, or_fault_mask(inj, round, OR_T_Y, i, ops));
+  }
+  double a = block_t1(c_row_ptr, c_col, c_val, k, x);
+  a = xor_double(a, or_fault_mask(inj, round, OR_T_T1, k,
+                                  2 * (int64_t)(c_row_ptr[k + 1] - c_row_ptr[k])));
+  double b = block_t2(y, n, bs, k, slot, pres);
+  b = xor_double(b, or_fault_mask(inj, round, OR_T_T2, k, rows_in_block(n, bs, k)));
+  double syn = a - b;
+  double tau = K[k] * beta;
+  if (t1) t1[k] = a;
+  if (t2) t2[k] = b;
+  if (s) s[k] = syn;
+  return !(fabs(syn) <= tau);
+}
+
+int or_abft_spmv(const or_csr *A, int32_t bs, const int32_t *c_row_ptr, const int32_t *c_col,
+                 const double *c_val, const double *K, const double *x, const or_inject *inj,
+                 int32_t max_rounds, double *y, double *y_pre, double *t1, double *t2,
+                 double *s, double *beta_out, int32_t *flag_counts, int32_t *flags) {
+  int64_t n = A->n, nb = (n + bs - 1) / bs;
+  /* step 2: beta = ||x||_2 = sqrt(PW(x_i^2)) (R10) */
+  double *sq = (double *)malloc(sizeof(double) * (size_t)(n > 0 ? n : 1));
+  for (int64_t i = 0; i < n; ++i) sq[i] = x[i] * x[i];
+  double beta = sqrt(or_pw(sq, n));
+  free(sq);
+  if (beta_out) *beta_out = beta;
+  double *slot = (double *)malloc(sizeof(double) * (size_t)bs);
+  unsigned char *pres = (unsigned char *)malloc((size_t)bs);
+  /* steps 1-4 over all blocks (round 0) */
+  int32_t cnt = 0;
+  for (int64_t k = 0; k < nb; ++k)
+    if (check_block(A, bs, c_row_ptr, c_col, c_val, K, x, beta, inj, 0, k, y, t1, t2, s, slot,
+                    pres))
+      flags[cnt++] = (int32_t)k;
+  flag_counts[0] = cnt;
+  if (y_pre) memcpy(y_pre, y, sizeof(double) * (size_t)n);
+  /* step 5: partial recomputation of flagged blocks, re-verified each round */
+  int rc = 0;
+  for (int32_t r = 1; r <= max_rounds; ++r) {
+    const int32_t *prev = flags + (int64_t)(r - 1) * nb;
+    int32_t *next = flags + (int64_t)r * nb;
+    int32_t nn = 0;
+    for (int32_t q = 0; q < flag_counts[r - 1]; ++q) {
+      int64_t k = prev[q];
+      if (check_block(A, bs, c_row_ptr, c_col, c_val, K, x, beta, inj, r, k, y, t1, t2, s, slot,
+                      pres))
+        next[nn++] = (int32_t)k;
+    }
+    flag_counts[r] = nn;
+  }
+  if (max_rounds > 0 && flag_counts[max_rounds] > 0) rc = -6;
+  free(slot);
+  free(pres);
+  return rc;
+}
+
+/* ------------------------------------------------------------------------ */
+/* Jacobi-preconditioned CG (Saad, Alg. 9.1) using the protected */
+/* SpMV for every product with A.  Stop when ||r||_2 <= tol * ||b||_2 (R16)  */
+/* or after max_iter iterations (10 N by default).  M = diag(A) and  */
+/* z = r / d elementwise (R21).  Updates follow R15.                         */
+/* ------------------------------------------------------------------------ */
+static double dot_pw(const double *a, const double *b, int64_t n, double *tmp) {
+  for (int64_t i = 0; i < n; ++i) tmp[i] = a[i] * b[i];
+  return or_pw(tmp, n);
+}
+
+int or_pcg(const or_csr *A, int32_t bs, const int32_t *c_row_ptr, const int32_t *c_col,
+           const double *c_val, const double *K, const double *b, double *x,
+           const double *diag, double tol, int64_t max_iter, const or_inject *inj_in,
+           int32_t max_rounds, int32_t check, double *res_hist, int64_t *stats) {
+  int64_t n = A->n, nb = (n + bs - 1) / bs;
+  if (max_iter <= 0) max_iter = 10 * n;
+  size_t vb = sizeof(double) * (size_t)(n > 0 ? n : 1);
+  double *r = (double *)malloc(vb), *z = (double *)malloc(vb), *p = (double *)malloc(vb);
+  double *q = (double *)malloc(vb), *tmp = (double *)malloc(vb), *d = (double *)malloc(vb);
+  int32_t *fc = (int32_t *)malloc(sizeof(int32_t) * (size_t)(max_rounds + 1));
+  int32_t *fl = (int32_t *)malloc(sizeof(int32_t) * (size_t)((max_rounds + 1) * nb + 1));
+  or_inject inj;
+  memset(&inj, 0, sizeof inj);
+  if (inj_in) inj = *inj_in;
+  uint64_t call0 = inj.call;
+  int64_t calls = 0;
+  for (int i = 0; i < 5; ++i) stats[i] = 0;
+  for (int64_t i = 0; i < n; ++i) {
+    if (diag) {
+      d[i] = diag[i];
+    } else {
+      double v = 0.0;
+      if (!find_entry(A, i, (int32_t)i, &v)) v = 0.0;
+      d[i] = v;
+    }
+  }
+  int rc = 0;
+  /* protected SpMV wrapper: y = A v, counting flags and recomputations */
+#define PROTECTED_SPMV(vin, yout)                                                          \
+  do {                                                                                     \
+    inj.call = call0 + (uint64_t)calls;                                                    \
+    if (check) {                                                                           \
+      int st = or_abft_spmv(A, bs, c_row_ptr, c_col, c_val, K, vin, &inj, max_rounds, yout, \
+                            NULL, NULL, NULL, NULL, NULL, fc, fl);                         \
+      stats[2] += fc[0];                                                                   \
+      for (int32_t rr = 0; rr < max_rounds; ++rr) stats[3] += fc[rr];                      \
+      if (st) stats[4] += 1;                                                               \
+    } else {                                                                               \
+      for (int64_t i_ = 0; i_ < n; ++i_) {                                                 \
+        double v_ = or_row_dot(A, i_, vin);                                                \
+        yout[i_] = xor_double(v_, or_fault_mask(&inj, 0, OR_T_Y, i_,                       \
+                                                2 * (int64_t)(A->row_ptr[i_ + 1] -          \
+                                                              A->row_ptr[i_])));            \
+      }                                                                                    \
+    }                                                                                      \
+    calls++;                                                                               \
+  } while (0)
+
+  PROTECTED_SPMV(x, q); /* q = A x0 */
+  for (int64_t i = 0; i < n; ++i) r[i] = b[i] - q[i];
+  for (int64_t i = 0; i < n; ++i) z[i] = r[i] / d[i];
+  for (int64_t i = 0; i < n; ++i) p[i] = z[i];
+  double rho = dot_pw(r, z, n, tmp);
+  double bnorm = sqrt(dot_pw(b, b, n, tmp));
+  double thr = tol * bnorm;
+  double res = sqrt(dot_pw(r, r, n, tmp));
+  res_hist[0] = res;
+  int64_t it = 0;
+  while (!(res <= thr) && it < max_iter) {
+    if (res != res) {
+      rc = -7;
+      break;
+    }
+    PROTECTED_SPMV(p, q);
+    double pq = dot_pw(p, q, n, tmp);
+    if (!(pq > 0.0)) {
+      rc = -7;
+      break;
+    }
+    double alpha = rho / pq;
+    for (int64_t i = 0; i < n; ++i) x[i] = x[i] + alpha * p[i];
+    for (int64_t i = 0; i < n; ++i) r[i] = r[i] - alpha * q[i];
+    for (int64_t i = 0; i < n; ++i) z[i] = r[i] / d[i];
+    double rho_new = dot_pw(r, z, n, tmp);
+    res = sqrt(dot_pw(r, r, n, tmp));
+    ++it;
+    res_hist[it] = res;
+    double beta = rho_new / rho;
+    rho = rho_new;
+    for (int64_t i = 0; i < n; ++i) p[i] = z[i] + beta * p[i];
+  }
+#undef PROTECTED_SPMV
+  if (rc == 0 && !(res <= thr)) rc = -5;
+  stats[0] = it;
+  stats[1] = calls;
+  free(r);
+  free(z);
+  free(p);
+  free(q);
+  free(tmp);
+  free(d);
+  free(fc);
+  free(fl);
+  return rc;
+}

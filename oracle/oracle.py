@@ -1,0 +1,266 @@
+"""ctypes wrapper around liboracle.so -- TEST INFRASTRUCTURE ONLY.
+
+Only tests/, __graft_entry__.smoke() and bench.py's cpu_baseline /
+--impl reference legs may import this module.  It never imports the product
+package's CUDA code, and the product package never imports it.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+import subprocess
+from dataclasses import dataclass
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_HERE, "abft_oracle.c")
+_LIB = os.path.join(_HERE, "liboracle.so")
+
+CFLAGS = ["-std=c99", "-O2", "-ffp-contract=off", "-fno-fast-math", "-fno-builtin",
+          "-Wall", "-shared", "-fPIC"]
+
+
+def build(force: bool = False) -> str:
+    """Compile liboracle.so (gcc, no FMA contraction)."""
+    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < max(
+            os.path.getmtime(_SRC), os.path.getmtime(os.path.join(_HERE, "abft_oracle.h"))):
+        subprocess.check_call(["gcc", *CFLAGS, "-o", _LIB, _SRC, "-lm"])
+    return _LIB
+
+
+_lib = None
+
+
+class _Csr(C.Structure):
+    _fields_ = [("n", C.c_int64), ("row_ptr", C.c_void_p), ("col", C.c_void_p),
+                ("val", C.c_void_p)]
+
+
+class _Inj(C.Structure):
+    _fields_ = [("mode", C.c_int32), ("seed", C.c_uint64), ("call", C.c_uint64),
+                ("lambda_", C.c_double), ("targets", C.c_uint32), ("n_list", C.c_int64),
+                ("list_round", C.c_void_p), ("list_target", C.c_void_p),
+                ("list_index", C.c_void_p), ("list_mask", C.c_void_p)]
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        _lib = C.CDLL(build())
+        L = _lib
+        P, i64, i32, d = C.c_void_p, C.c_int64, C.c_int32, C.c_double
+        L.or_pw.restype = d
+        L.or_pw.argtypes = [P, i64]
+        L.or_pw_slots.restype = d
+        L.or_pw_slots.argtypes = [P, P, i64]
+        L.or_spmv.argtypes = [P, P, P]
+        L.or_encode_structure.restype = i64
+        L.or_encode_structure.argtypes = [P, i32, P, P]
+        L.or_encode_values.argtypes = [P, i32, P, P, P]
+        L.or_encode_bound.argtypes = [P, i32, P, P, P, P, P, P]
+        L.or_philox4x32_10.argtypes = [P, P, P]
+        L.or_burst_table.argtypes = [P]
+        L.or_fault_mask.restype = C.c_uint64
+        L.or_fault_mask.argtypes = [P, i32, i32, i64, i64]
+        L.or_abft_spmv.restype = C.c_int
+        L.or_abft_spmv.argtypes = [P, i32, P, P, P, P, P, P, i32, P, P, P, P, P, P, P, P]
+        L.or_pcg.restype = C.c_int
+        L.or_pcg.argtypes = [P, i32, P, P, P, P, P, P, P, d, i64, P, i32, i32, P, P]
+    return _lib
+
+
+def _p(a):
+    return None if a is None else a.ctypes.data_as(C.c_void_p)
+
+
+class _CsrRef:
+    """Keeps the numpy arrays alive while the C struct points into them."""
+
+    def __init__(self, A):
+        self.rp = np.ascontiguousarray(A.row_ptr, dtype=np.int32)
+        self.col = np.ascontiguousarray(A.col, dtype=np.int32)
+        self.val = np.ascontiguousarray(A.val, dtype=np.float64)
+        self.s = _Csr(int(self.rp.shape[0] - 1), _p(self.rp).value, _p(self.col).value,
+                      _p(self.val).value)
+
+    def ref(self):
+        return C.byref(self.s)
+
+
+class Inject:
+    """Fault injection spec shared by oracle calls (mirrors abft_inject_t)."""
+
+    NONE, LIST, RATE = 0, 1, 2
+
+    def __init__(self, mode=0, seed=0, call=0, lam=0.0, targets=0b001, plan=None):
+        self.mode, self.seed, self.call, self.lam, self.targets = mode, seed, call, lam, targets
+        self.plan = plan
+
+    @staticmethod
+    def from_plan(plan):
+        return Inject(mode=Inject.LIST, plan=plan)
+
+    @staticmethod
+    def rate(seed, lam, targets=0b111, call=0):
+        return Inject(mode=Inject.RATE, seed=seed, call=call, lam=lam, targets=targets)
+
+    def _struct(self):
+        s = _Inj()
+        s.mode, s.seed, s.call, s.lambda_, s.targets = (self.mode, self.seed, self.call,
+                                                        self.lam, self.targets)
+        if self.mode == Inject.LIST and self.plan is not None and len(self.plan):
+            self._keep = (np.ascontiguousarray(self.plan.round, np.int32),
+                          np.ascontiguousarray(self.plan.target, np.int32),
+                          np.ascontiguousarray(self.plan.index, np.int64),
+                          np.ascontiguousarray(self.plan.mask, np.uint64))
+            s.n_list = len(self.plan)
+            s.list_round, s.list_target, s.list_index, s.list_mask = [
+                _p(a).value for a in self._keep]
+        else:
+            s.n_list = 0
+        return s
+
+
+def pw(v, present=None) -> float:
+    v = np.ascontiguousarray(v, dtype=np.float64)
+    if present is None:
+        return lib().or_pw(_p(v), v.shape[0])
+    pr = np.ascontiguousarray(present, dtype=np.uint8)
+    return lib().or_pw_slots(_p(v), _p(pr), v.shape[0])
+
+
+def spmv(A, x) -> np.ndarray:
+    r = _CsrRef(A)
+    x = np.ascontiguousarray(x, dtype=np.float64)
+    y = np.empty(A.n)
+    lib().or_spmv(r.ref(), _p(x), _p(y))
+    return y
+
+
+@dataclass
+class Encoded:
+    bs: int
+    row_ptr: np.ndarray  # C row_ptr int32[nb+1]
+    col: np.ndarray      # C col int32[nnz(C)]
+    val: np.ndarray      # C val f64[nnz(C)]
+    K: np.ndarray        # f64[nb]
+    row_norm: np.ndarray
+    S: np.ndarray
+    c_norm: np.ndarray
+
+    @property
+    def nb(self):
+        return int(self.row_ptr.shape[0] - 1)
+
+    @property
+    def n_k(self):
+        return np.diff(self.row_ptr.astype(np.int64))
+
+
+def encode(A, bs: int = 32) -> Encoded:
+    r = _CsrRef(A)
+    nb = (A.n + bs - 1) // bs
+    c_rp = np.zeros(nb + 1, dtype=np.int32)
+    L = lib()
+    tot = L.or_encode_structure(r.ref(), bs, _p(c_rp), None)
+    c_col = np.empty(max(tot, 1), dtype=np.int32)
+    L.or_encode_structure(r.ref(), bs, _p(c_rp), _p(c_col))
+    c_val = np.empty(max(tot, 1))
+    L.or_encode_values(r.ref(), bs, _p(c_rp), _p(c_col), _p(c_val))
+    K = np.empty(nb)
+    rn = np.empty(A.n)
+    S = np.empty(nb)
+    cn = np.empty(nb)
+    L.or_encode_bound(r.ref(), bs, _p(c_rp), _p(c_val), _p(K), _p(rn), _p(S), _p(cn))
+    return Encoded(bs, c_rp, c_col[:tot], c_val[:tot], K, rn, S, cn)
+
+
+def philox4x32_10(ctr, key):
+    c = np.ascontiguousarray(ctr, dtype=np.uint32)
+    k = np.ascontiguousarray(key, dtype=np.uint32)
+    o = np.empty(4, dtype=np.uint32)
+    lib().or_philox4x32_10(_p(c), _p(k), _p(o))
+    return o
+
+
+def burst_table() -> np.ndarray:
+    t = np.empty(65, dtype=np.uint64)
+    lib().or_burst_table(_p(t))
+    return t
+
+
+def fault_mask(inj: Inject, round_: int, target: int, index: int, ops: int) -> int:
+    s = inj._struct()
+    return int(lib().or_fault_mask(C.byref(s), round_, target, index, ops))
+
+
+@dataclass
+class SpmvResult:
+    status: int
+    y: np.ndarray
+    y_pre: np.ndarray
+    t1: np.ndarray
+    t2: np.ndarray
+    s: np.ndarray
+    beta: float
+    flags: list  # per round: sorted np.int32 array
+
+    @property
+    def flagged(self):
+        return self.flags[0]
+
+    def recomputed(self):
+        """Blocks recomputed in each correction round r = 1..R (= flags[r-1])."""
+        return self.flags[:-1]
+
+
+def abft_spmv(A, enc: Encoded, x, inj: Inject | None = None, max_rounds: int = 4) -> SpmvResult:
+    r = _CsrRef(A)
+    x = np.ascontiguousarray(x, dtype=np.float64)
+    nb = enc.nb
+    y = np.empty(A.n)
+    y_pre = np.empty(A.n)
+    t1 = np.empty(nb)
+    t2 = np.empty(nb)
+    s = np.empty(nb)
+    beta = C.c_double(0.0)
+    fc = np.zeros(max_rounds + 1, dtype=np.int32)
+    fl = np.zeros((max_rounds + 1) * max(nb, 1), dtype=np.int32)
+    ist = inj._struct() if inj is not None else None
+    st = lib().or_abft_spmv(r.ref(), enc.bs, _p(enc.row_ptr), _p(enc.col), _p(enc.val),
+                            _p(enc.K), _p(x), C.byref(ist) if ist is not None else None,
+                            max_rounds, _p(y), _p(y_pre), _p(t1), _p(t2), _p(s),
+                            C.byref(beta), _p(fc), _p(fl))
+    flags = [fl[q * nb: q * nb + fc[q]].copy() for q in range(max_rounds + 1)]
+    return SpmvResult(st, y, y_pre, t1, t2, s, beta.value, flags)
+
+
+@dataclass
+class PcgResult:
+    status: int
+    x: np.ndarray
+    res_hist: np.ndarray
+    iters: int
+    spmv_calls: int
+    flagged_blocks: int
+    recomputed_blocks: int
+    uncorrected_calls: int
+
+
+def pcg(A, enc: Encoded, b, x0, diag=None, tol=1e-6, max_iter=0, inj: Inject | None = None,
+        max_rounds=4, check=True) -> PcgResult:
+    r = _CsrRef(A)
+    b = np.ascontiguousarray(b, dtype=np.float64)
+    x = np.array(x0, dtype=np.float64, copy=True)
+    mi = max_iter if max_iter > 0 else 10 * A.n
+    hist = np.zeros(mi + 1)
+    stats = np.zeros(5, dtype=np.int64)
+    d = None if diag is None else np.ascontiguousarray(diag, dtype=np.float64)
+    ist = inj._struct() if inj is not None else None
+    st = lib().or_pcg(r.ref(), enc.bs, _p(enc.row_ptr), _p(enc.col), _p(enc.val), _p(enc.K),
+                      _p(b), _p(x), _p(d), tol, mi, C.byref(ist) if ist is not None else None,
+                      max_rounds, 1 if check else 0, _p(hist), _p(stats))
+    it = int(stats[0])
+    return PcgResult(st, x, hist[: it + 1].copy(), it, int(stats[1]), int(stats[2]),
+                     int(stats[3]), int(stats[4]))

@@ -1,0 +1,491 @@
+"""Pins for the CPU oracle (oracle/abft_oracle.c) against what PAPER.md and
+the mathematics fix -- never against the oracle itself or the CUDA path.
+
+Each test names the passage / property it pins.  These run without a GPU.
+"""
+import json
+import math
+import os
+from fractions import Fraction
+
+import numpy as np
+import pytest
+
+from paper_conf_dsn_schollbkw16_b200 import inputs as G
+
+GOLD = os.path.join(os.path.dirname(__file__), "golden")
+EPS = 2.0 ** -53
+U = 2.0 ** -53  # unit roundoff
+
+
+def csr_from_dense(D):
+    D = np.asarray(D, dtype=np.float64)
+    rows, cols = np.nonzero(D)
+    counts = np.bincount(rows, minlength=D.shape[0])
+    rp = np.concatenate([[0], np.cumsum(counts)])
+    return G.CSR(rp, cols, D[rows, cols])
+
+
+def exact_sum(vals):
+    return sum((Fraction(float(v)) for v in vals), Fraction(0))
+
+
+# --------------------------------------------------------------------------
+# R2: canonical pairwise summation -- pinned by hand-computed
+# cases whose result differs under every other grouping.
+# --------------------------------------------------------------------------
+class TestPairwise:
+    def test_tree_grouping_power_of_two(self, O):
+        # ((1 + u) + (u + u)) = 1 + 2u exactly; a left fold gives 1.0
+        assert O.pw([1.0, U, U, U]) == 1.0 + 2 * U
+
+    def test_absent_padding_three(self, O):
+        # n = 3 -> (v0 + v1) + v2 = (1 + u) + u = 1.0 ; v0 + (v1 + v2) = 1 + 2u
+        assert O.pw([1.0, U, U]) == 1.0
+
+    def test_five_elements(self, O):
+        # ((v0+v1)+(v2+v3)) + v4 with v4 alone in the right subtree
+        # ((1 + u) + (u + u)) + (-1) = (1 + 2u) - 1 = 2u; a left fold gives 0
+        assert O.pw([1.0, U, U, U, -1.0]) == 2 * U
+
+    def test_empty_and_signed_zero(self, O):
+        assert O.pw([]) == 0.0 and math.copysign(1, O.pw([])) == 1.0
+        assert math.copysign(1, O.pw([-0.0])) == -1.0
+        assert math.copysign(1, O.pw([-0.0, -0.0, -0.0])) == -1.0
+
+    def test_slots_absent_differs_from_compacted(self, O):
+        # slots [1, absent, u, u]: 1 + (u + u) = 1 + 2u; the compacted list
+        # [1, u, u] gives 1.0 -- absent slots keep their tree position.
+        v = np.array([1.0, 123.0, U, U])
+        assert O.pw(v, [1, 0, 1, 1]) == 1.0 + 2 * U
+        assert O.pw(v, [0, 0, 0, 0]) == 0.0
+
+    def test_integers_exact(self, O):
+        rng = np.random.default_rng(0)
+        for n in [1, 2, 3, 7, 31, 32, 33, 1000]:
+            v = rng.integers(-1000, 1000, n).astype(float)
+            assert O.pw(v) == float(sum(int(a) for a in v))
+
+    def test_error_bound(self, O):
+        # |PW - exact| <= gamma_{ceil(log2 n)} * sum|v|  (Higham, Thm 4.1 / pairwise)
+        rng = np.random.default_rng(1)
+        for n in [10, 100, 1000, 4097]:
+            v = rng.standard_normal(n) * 10.0 ** rng.integers(-5, 5, n)
+            d = math.ceil(math.log2(n))
+            g = d * U / (1 - d * U)
+            err = abs(Fraction(O.pw(v)) - exact_sum(v))
+            assert float(err) <= g * float(np.abs(v).sum())
+
+
+# --------------------------------------------------------------------------
+# SpMV: brute force against dense products on tiny inputs.
+# --------------------------------------------------------------------------
+class TestSpmv:
+    def test_integer_exact(self, O):
+        for seed in range(5):
+            A = G.random_csr(37, 0.2, seed, integer=True, empty_rows=0.1)
+            x = np.random.default_rng(seed).integers(-9, 10, 37).astype(float)
+            y = O.spmv(A, x)
+            assert np.array_equal(y, A.to_dense().astype(np.int64) @ x.astype(np.int64))
+
+    def test_float_within_bound(self, O):
+        A = G.random_csr(50, 0.3, 3)
+        x = G.uniform_vector(50, 42)
+        y = O.spmv(A, x)
+        D = A.to_dense()
+        for i in range(50):
+            prods = [Fraction(float(D[i, j])) * Fraction(float(x[j])) for j in range(50) if D[i, j] != 0]
+            n = max(len(prods), 1)
+            g = (math.ceil(math.log2(n)) + 1) * U / (1 - 8 * U) if n > 1 else U
+            bound = g * sum(abs(float(p)) for p in prods)
+            assert abs(float(Fraction(y[i]) - sum(prods, Fraction(0)))) <= bound + 1e-300
+
+    def test_empty_row_is_plus_zero(self, O):
+        A = csr_from_dense([[0, 0], [1, 2]])
+        y = O.spmv(A, np.array([-1.0, 1.0]))
+        assert y[0] == 0.0 and math.copysign(1, y[0]) == 1.0 and y[1] == 1.0
+
+
+# --------------------------------------------------------------------------
+# Encoding
+# --------------------------------------------------------------------------
+def brute_structure(A, bs):
+    D = A.to_dense() != 0
+    # structural: use the CSR pattern, not numerical nonzeros
+    P = np.zeros((A.n, A.n), dtype=bool)
+    rows = np.repeat(np.arange(A.n), A.row_lengths())
+    P[rows, A.col] = True
+    del D
+    nb = (A.n + bs - 1) // bs
+    return [sorted(set(np.nonzero(P[k * bs:(k + 1) * bs].any(axis=0))[0].tolist())) for k in range(nb)]
+
+
+class TestEncode:
+    @pytest.mark.parametrize("n,bs", [(20, 5), (37, 4), (33, 32), (64, 1), (65, 8), (10, 10), (10, 64)])
+    def test_structure_fig2_rule(self, O, n, bs):
+        # Fig. 2 rule: a column appears in row k of C iff it holds >= 1
+        # element of A_k.  Brute force with Python sets.
+        A = G.random_csr(n, 0.15, n * 7 + bs, empty_rows=0.1)
+        enc = O.encode(A, bs)
+        exp = brute_structure(A, bs)
+        assert enc.nb == len(exp)
+        for k, cols in enumerate(exp):
+            assert enc.col[enc.row_ptr[k]:enc.row_ptr[k + 1]].tolist() == cols
+        assert np.array_equal(enc.n_k, [len(c) for c in exp])
+
+    def test_explicit_zero_is_structural(self, O):
+        # R5 (Q2): a stored 0.0 still counts as an element of A_k.
+        A = G.CSR([0, 2, 3], [0, 1, 1], [1.0, 0.0, 2.0])
+        enc = O.encode(A, 2)
+        assert enc.col.tolist() == [0, 1] and enc.val.tolist() == [1.0, 2.0]
+
+    @pytest.mark.parametrize("bs", [1, 2, 3, 8, 32])
+    def test_values_integer_column_sums(self, O, bs):
+        # c_k = w_k^T A_k with w = ones: dense column sums.
+        A = G.random_csr(45, 0.2, bs, integer=True)
+        enc = O.encode(A, bs)
+        D = A.to_dense()
+        for k in range(enc.nb):
+            cs = D[k * bs:(k + 1) * bs].sum(axis=0)
+            cols = enc.col[enc.row_ptr[k]:enc.row_ptr[k + 1]]
+            assert np.array_equal(enc.val[enc.row_ptr[k]:enc.row_ptr[k + 1]], cs[cols])
+
+    def test_bs1_c_equals_a(self, O):
+        # "For block size 1, the checksum matrix C is equal to A."
+        A = G.random_csr(40, 0.2, 11)
+        enc = O.encode(A, 1)
+        assert np.array_equal(enc.row_ptr, A.row_ptr)
+        assert np.array_equal(enc.col, A.col)
+        assert np.array_equal(enc.val, A.val)
+
+    def test_laplacian_checksum_values(self, O):
+        # Column sums of a 5-pt / 7-pt / 27-pt Laplacian row block are small
+        # integers (diag + neighbours).  With the grid's x extent a multiple of
+        # b_s = 32 (as in every BASELINE config) a block is a piece of one
+        # x-line, so the sums are {-1,2,3} / {-1,4,5} / {-3,-2,-1,24,25}.
+        for A, allowed in [(G.laplacian_2d_5pt(64, 8), {-1.0, 2.0, 3.0}),
+                           (G.laplacian_3d_7pt(32, 4, 4), {-1.0, 4.0, 5.0}),
+                           (G.stencil_3d_27pt(32, 4, 4), {-3.0, -2.0, -1.0, 24.0, 25.0})]:
+            enc = O.encode(A, 32)
+            assert set(np.unique(enc.val).tolist()) <= allowed
+            D = A.to_dense()
+            for k in range(enc.nb):
+                cs = D[32 * k:32 * (k + 1)].sum(axis=0)
+                cols = enc.col[enc.row_ptr[k]:enc.row_ptr[k + 1]]
+                assert np.array_equal(enc.val[enc.row_ptr[k]:enc.row_ptr[k + 1]], cs[cols])
+
+    def test_bound_bs1_closed_form(self, O):
+        # b_s = 1: c_k = a_k, so tau_k = ((n_k + 0) ||a_k|| + n_k ||a_k||) eps beta
+        #        = 2 n_k ||a_k|| eps beta  (P:158 with b_s = 1, C = A from P:248).
+        # Rows with Pythagorean norms make the closed form exact.
+        A = csr_from_dense([[3, 4, 0, 0], [0, 0, 5, 12], [8, 0, 15, 0], [0, 0, 0, 7]])
+        enc = O.encode(A, 1)
+        norms = [5.0, 13.0, 17.0, 7.0]
+        nk = [2, 2, 2, 1]
+        assert enc.K.tolist() == [2 * n * r * EPS for n, r in zip(nk, norms)]
+
+    def test_bound_bsN_reduces_to_dense_bound(self, O):
+        # b_s = N with every column non-empty: one block; P:158 becomes the
+        # dense bound of [35] with m = N rows and n columns:
+        #   ((n + 2m - 2) sum_i ||a_i|| + n ||c||) eps_M.
+        A = csr_from_dense([[3, 4, 0], [0, 0, 5], [0, 0, 0]])  # col sums (3,4,5), ||c|| = 5*sqrt2
+        enc = O.encode(A, 3)
+        m, n = 3, 3
+        sum_norms = 5.0 + 5.0 + 0.0
+        c = math.sqrt(50.0)
+        assert enc.K.shape == (1,)
+        assert enc.K[0] == ((n + 2 * m - 2) * sum_norms + n * c) * EPS
+
+    def test_bound_coefficient_uses_nk_not_n(self, O):
+        # the sparse bound uses the number of NON-EMPTY columns n_k of
+        # A_k, not N.  Block 0 touches 2 of 6 columns; b_s = 2.
+        D = np.zeros((6, 6))
+        D[0, 0] = 3
+        D[0, 1] = 4
+        D[1, 1] = 5
+        D[1, 0] = 12  # ||a_0|| = 5, ||a_1|| = 13; c_0 = (15, 9)
+        D[2:, 2:] = np.eye(4)
+        A = csr_from_dense(D)
+        enc = O.encode(A, 2)
+        c0 = math.sqrt(15.0 ** 2 + 9.0 ** 2)
+        assert enc.n_k.tolist() == [2, 2, 2]
+        assert enc.K[0] == ((2 + 2 * 2 - 2) * 18.0 + 2 * c0) * EPS
+
+    def test_ragged_last_block(self, O):
+        # R3 (Q3): the last block holds only the existing rows; b_s stays literal.
+        A = G.laplacian_2d_5pt(5)  # N = 25, b_s = 8 -> last block has 1 row
+        enc = O.encode(A, 8)
+        assert enc.nb == 4
+        r = 24
+        nk = enc.n_k[3]
+        rn = math.sqrt(16 + 1 + 1)
+        c = enc.val[enc.row_ptr[3]:enc.row_ptr[4]]
+        assert c.tolist() == [-1.0, -1.0, 4.0]
+        assert enc.K[3] == ((nk + 2 * 8 - 2) * rn + nk * math.sqrt(18.0)) * EPS
+        del r
+
+
+# --------------------------------------------------------------------------
+# Detection, correction
+# --------------------------------------------------------------------------
+class TestWorkedExample:
+    def test_golden_6x6(self, O):
+        g = json.load(open(os.path.join(GOLD, "worked_example_6x6.json")))
+        A = csr_from_dense(g["A_dense"])
+        bs = g["block_size"]
+        x = np.array(g["x"], dtype=float)
+        enc = O.encode(A, bs)
+        Cd = np.zeros((enc.nb, A.n))
+        for k in range(enc.nb):
+            for q in range(enc.row_ptr[k], enc.row_ptr[k + 1]):
+                Cd[k, enc.col[q]] = enc.val[q]
+        assert Cd.tolist() == g["C_dense"]
+        assert enc.n_k.tolist() == g["n_k"]
+        ok = O.abft_spmv(A, enc, x)
+        assert ok.y.tolist() == g["y_fault_free"]
+        assert ok.t1.tolist() == g["t1"] and ok.t2.tolist() == g["t2_fault_free"]
+        assert ok.flagged.size == 0
+        plan = G.FaultPlan([0], [G.TARGET_Y], [g["fault"]["element_1based"] - 1], [g["fault"]["mask"]])
+        r = O.abft_spmv(A, enc, x, O.Inject.from_plan(plan), max_rounds=1)
+        assert r.y_pre.tolist() == g["y_faulty"]
+        assert (r.t1 - g["t1"]).tolist() == [0, 0, 0]
+        assert (np.array(g["t1"]) - np.array(g["t2_faulty"])).tolist() == g["syndrome_faulty"]
+        assert (r.flagged + 1).tolist() == g["flagged_blocks_1based"]
+        rows = [i + 1 for k in r.flagged for i in range(k * bs, (k + 1) * bs)]
+        assert rows == g["recomputed_rows_1based"]
+        assert r.y.tolist() == g["y_fault_free"] and r.status == 0
+        assert r.flags[1].size == 0
+
+
+class TestDetection:
+    def test_invariant_eq2_integers(self, O):
+        # eq. (2): with integer A, x and all partial sums < 2^53 the
+        # invariant holds exactly: t1 == t2, s == 0, for every b_s.
+        for bs in [1, 2, 5, 32]:
+            A = G.random_csr(70, 0.1, bs, integer=True, empty_rows=0.05)
+            x = np.random.default_rng(bs).integers(-50, 50, 70).astype(float)
+            enc = O.encode(A, bs)
+            r = O.abft_spmv(A, enc, x)
+            assert np.array_equal(r.t1, r.t2) and np.all(r.s == 0.0)
+            assert r.flagged.size == 0
+
+    @pytest.mark.parametrize("mat", ["lap2d", "lap3d", "st27", "rand", "rmat"])
+    def test_no_false_positives(self, O, mat):
+        # tau is an upper bound on rounding differences:
+        # error-free runs flag nothing.
+        A = {"lap2d": lambda: G.laplacian_2d_5pt(64), "lap3d": lambda: G.laplacian_3d_7pt(12),
+             "st27": lambda: G.stencil_3d_27pt(10), "rand": lambda: G.random_csr(300, 0.05, 5),
+             "rmat": lambda: G.rmat(10, 8, 3)}[mat]()
+        enc = O.encode(A, 32)
+        for seed in range(3):
+            x = G.uniform_vector(A.n, 100 + seed)
+            r = O.abft_spmv(A, enc, x)
+            assert r.flagged.size == 0
+            tau = enc.K * r.beta
+            assert np.all(np.abs(r.s) <= tau)
+
+    def test_beta_is_two_norm(self, O):
+        x = G.uniform_vector(1000, 9)
+        A = G.laplacian_2d_5pt(10)
+        x = x[:A.n]
+        r = O.abft_spmv(A, O.encode(A, 32), x)
+        exact = float(exact_sum([Fraction(v) * Fraction(v) for v in x]))
+        assert abs(r.beta - math.sqrt(exact)) <= 1e-15 * r.beta
+
+    def test_large_faults_localized(self, O):
+        # A fault with |delta| >= 2 tau_k must be flagged and localized to its
+        # own block only; correction restores y exactly.
+        A = G.laplacian_3d_7pt(10)
+        enc = O.encode(A, 32)
+        x = G.uniform_vector(A.n, 7)
+        clean = O.spmv(A, x)
+        base = O.abft_spmv(A, enc, x)
+        hit = 0
+        for seed in range(300):
+            plan = G.single_fault_plan(A.n, seed)
+            r = O.abft_spmv(A, enc, x, O.Inject.from_plan(plan), max_rounds=2)
+            i = int(plan.index[0])
+            k = i // 32
+            delta = abs(r.y_pre[i] - clean[i]) if np.isfinite(r.y_pre[i]) else np.inf
+            tau = enc.K[k] * base.beta
+            if delta >= 2 * tau:
+                hit += 1
+                assert r.flagged.tolist() == [k]
+            else:
+                assert set(r.flagged.tolist()) <= {k}
+            assert r.status == 0
+            if r.flagged.size:  # detected -> the recomputation restores y exactly
+                assert r.y.view(np.uint64).tolist() == clean.view(np.uint64).tolist()
+            else:  # undetected -> only element i differs, by less than 2 tau
+                d = np.nonzero(r.y != clean)[0]
+                assert d.tolist() in ([], [i]) and delta < 2 * tau
+        assert hit > 200
+
+    def test_checksum_target_faults(self, O):
+        # P:196 "Bit flips were also injected into operations that perform
+        # error detection": a big fault in t1_k or t2_k flags block k; the
+        # recomputation then clears it.
+        A = G.laplacian_2d_5pt(32)
+        enc = O.encode(A, 32)
+        x = G.uniform_vector(A.n, 3)
+        for tgt in (G.TARGET_T1, G.TARGET_T2):
+            plan = G.FaultPlan([0], [tgt], [5], [1 << 62])
+            r = O.abft_spmv(A, enc, x, O.Inject.from_plan(plan), max_rounds=1)
+            assert r.flagged.tolist() == [5] and r.flags[1].size == 0 and r.status == 0
+
+    def test_uncorrectable_reports(self, O):
+        # A fault re-injected in every round is never cleared -> -6 (R11').
+        A = G.laplacian_2d_5pt(16)
+        enc = O.encode(A, 32)
+        x = G.uniform_vector(A.n, 3)
+        plan = G.FaultPlan([0, 1, 2], [0, 0, 0], [40, 40, 40], [1 << 60] * 3)
+        r = O.abft_spmv(A, enc, x, O.Inject.from_plan(plan), max_rounds=2)
+        assert r.status == -6 and r.flags[2].tolist() == [1]
+
+    def test_nan_flags(self, O):
+        # R5' (Q5): flag iff NOT(|s| <= tau) also flags NaN syndromes.
+        A = G.laplacian_2d_5pt(8)
+        enc = O.encode(A, 32)
+        x = G.uniform_vector(A.n, 1)
+        plan = G.FaultPlan([0], [0], [3], [0x7FF8000000000000])  # exponent -> NaN/Inf
+        r = O.abft_spmv(A, enc, x, O.Inject.from_plan(plan), max_rounds=0)
+        assert r.flagged.tolist() == [0]
+
+    def test_zero_x_and_empty_blocks(self, O):
+        # x = 0 -> beta = 0, tau = 0; s = 0 exactly so nothing is flagged.
+        # An all-empty block has tau_k = 0 and s_k = 0 -> not flagged.
+        A = G.random_csr(96, 0.1, 2)
+        A2 = G.CSR(np.concatenate([A.row_ptr[:33], np.full(32, A.row_ptr[32]),
+                                   A.row_ptr[65:] - (A.row_ptr[64] - A.row_ptr[32])]),
+                   np.concatenate([A.col[:A.row_ptr[32]], A.col[A.row_ptr[64]:]]),
+                   np.concatenate([A.val[:A.row_ptr[32]], A.val[A.row_ptr[64]:]]))
+        enc = O.encode(A2, 32)
+        assert enc.n_k[1] == 0 and enc.K[1] == 0.0
+        r = O.abft_spmv(A2, enc, np.zeros(96))
+        assert r.beta == 0.0 and r.flagged.size == 0
+        r = O.abft_spmv(A2, enc, G.uniform_vector(96, 5))
+        assert r.flagged.size == 0 and r.t1[1] == 0.0 and r.t2[1] == 0.0
+
+
+# --------------------------------------------------------------------------
+# Fault model
+# --------------------------------------------------------------------------
+class TestFaultModel:
+    def test_philox_known_answers(self, O):
+        # Random123 published known-answer vectors for philox4x32-10.
+        kat = [([0, 0, 0, 0], [0, 0], [0x6627e8d5, 0xe169c58d, 0xbc57ac4c, 0x9b00dbd8]),
+               ([0xffffffff] * 4, [0xffffffff] * 2, [0x408f276d, 0x41c83b0e, 0xa20bc7c6, 0x6d5451fd]),
+               ([0x243f6a88, 0x85a308d3, 0x13198a2e, 0x03707344], [0xa4093822, 0x299f31d0],
+                [0xd16cfe09, 0x94fdcceb, 0x5001e420, 0x24126ea1])]
+        for c, k, o in kat:
+            assert O.philox4x32_10(c, k).tolist() == o
+
+    def test_burst_table_distribution(self, O):
+        # burst length ~ Normal(mean 3, variance 2), read as
+        # L = max(1, round(3 + sqrt2 Z)).  Compare the table's pmf with a
+        # Monte-Carlo draw from numpy's normal generator.
+        T = O.burst_table().astype(np.float64)
+        assert T[0] == 0 and T[64] == 2 ** 32 and np.all(np.diff(T) >= 0)
+        pmf = np.diff(T) / 2 ** 32  # P(L = l), l = 1..64
+        z = np.random.default_rng(0).normal(3.0, math.sqrt(2.0), 2_000_000)
+        L = np.maximum(1, np.rint(z)).astype(int)
+        emp = np.bincount(L, minlength=65)[1:65] / L.size
+        assert np.max(np.abs(emp - pmf)) < 2e-3
+        mean = float((np.arange(1, 65) * pmf).sum())
+        assert abs(mean - L.mean()) < 5e-3
+
+    def test_rate_mode_frequency(self, O):
+        # lambda = probability that an arithmetic op returns an
+        # erroneous result -> a value produced by `ops` ops is faulty with
+        # probability ~ lambda * ops.  Binomial check.
+        inj = O.Inject.rate(seed=123, lam=1e-3, targets=0b111)
+        hits = sum(O.fault_mask(inj, 0, 0, i, 14) != 0 for i in range(40000))
+        p = 14e-3
+        assert abs(hits - 40000 * p) < 5 * math.sqrt(40000 * p * (1 - p))
+        inj0 = O.Inject.rate(seed=123, lam=0.0)
+        assert all(O.fault_mask(inj0, 0, 0, i, 14) == 0 for i in range(1000))
+        inj1 = O.Inject.rate(seed=123, lam=1.0)
+        assert all(O.fault_mask(inj1, 0, 0, i, 14) != 0 for i in range(1000))
+
+    def test_rate_mode_masks_are_bursts(self, O):
+        inj = O.Inject.rate(seed=5, lam=1.0)
+        for i in range(2000):
+            m = O.fault_mask(inj, 1, 2, i, 1)
+            assert m != 0
+            lo = (m & -m).bit_length() - 1
+            run = m >> lo
+            assert run & (run + 1) == 0  # contiguous ones
+
+    def test_rate_targets_mask(self, O):
+        inj = O.Inject.rate(seed=5, lam=1.0, targets=0b010)
+        assert O.fault_mask(inj, 0, 0, 3, 1) == 0 and O.fault_mask(inj, 0, 1, 3, 1) != 0
+
+
+# --------------------------------------------------------------------------
+# PCG against SciPy's CG (an independent library routine)
+# --------------------------------------------------------------------------
+class TestPcg:
+    def test_matches_scipy_cg(self, O):
+        import scipy.sparse as sp
+        import scipy.sparse.linalg as spla
+        A = G.laplacian_3d_7pt(10)
+        enc = O.encode(A, 32)
+        xs = G.uniform_vector(A.n, 43)
+        b = O.spmv(A, xs)
+        x0 = G.uniform_vector(A.n, 44)
+        r = O.pcg(A, enc, b, x0, tol=1e-6)
+        assert r.status == 0
+        S = sp.csr_matrix((A.val, A.col, A.row_ptr), shape=(A.n, A.n))
+        d = S.diagonal()
+        M = spla.LinearOperator(S.shape, matvec=lambda v: v / d)
+        xs_hist = []
+        xsc, info = spla.cg(S, b, x0=x0.copy(), rtol=1e-6, atol=0.0, M=M,
+                            callback=lambda xk: xs_hist.append(xk.copy()), maxiter=10 * A.n)
+        assert info == 0
+        assert r.iters == len(xs_hist)
+        # residual histories agree (true residual of SciPy's iterates vs the
+        # oracle's recursive residual) to well within 1e-10 * ||b||
+        bn = np.linalg.norm(b)
+        true_res = [np.linalg.norm(b - S @ xk) for xk in xs_hist]
+        assert np.max(np.abs(np.array(true_res) - r.res_hist[1:])) < 1e-10 * bn
+        assert np.linalg.norm(r.x - xsc) <= 1e-9 * np.linalg.norm(xsc)
+        assert np.linalg.norm(r.x - xs) <= 1e-4 * np.linalg.norm(xs)
+
+    def test_constant_diagonal_equals_cg(self, O):
+        # Jacobi with a constant diagonal is plain CG up to scaling: the
+        # iteration count equals SciPy's unpreconditioned CG.
+        import scipy.sparse as sp
+        import scipy.sparse.linalg as spla
+        A = G.laplacian_2d_5pt(24)
+        enc = O.encode(A, 32)
+        b = O.spmv(A, G.uniform_vector(A.n, 1))
+        x0 = np.zeros(A.n)
+        r = O.pcg(A, enc, b, x0, tol=1e-8)
+        S = sp.csr_matrix((A.val, A.col, A.row_ptr), shape=(A.n, A.n))
+        cnt = []
+        spla.cg(S, b, x0=x0.copy(), rtol=1e-8, atol=0.0, callback=lambda xk: cnt.append(1))
+        assert r.status == 0 and r.iters == len(cnt)
+
+    def test_faulty_pcg_still_converges(self, O):
+        # With faults in the protected SpMV at a high rate the solver still
+        # converges because flagged blocks are recomputed.
+        A = G.laplacian_3d_7pt(8)
+        enc = O.encode(A, 32)
+        xs = G.uniform_vector(A.n, 43)
+        b = O.spmv(A, xs)
+        x0 = G.uniform_vector(A.n, 44)
+        clean = O.pcg(A, enc, b, x0, tol=1e-6)
+        r = O.pcg(A, enc, b, x0, tol=1e-6, inj=O.Inject.rate(seed=9, lam=1e-4))
+        assert r.status == 0 and r.flagged_blocks > 0 and r.recomputed_blocks >= r.flagged_blocks
+        assert abs(r.iters - clean.iters) <= 3
+        assert r.uncorrected_calls == 0
+
+    def test_unprotected_faulty_pcg_differs(self, O):
+        A = G.laplacian_3d_7pt(8)
+        enc = O.encode(A, 32)
+        b = O.spmv(A, G.uniform_vector(A.n, 43))
+        x0 = G.uniform_vector(A.n, 44)
+        clean = O.pcg(A, enc, b, x0, tol=1e-6)
+        r = O.pcg(A, enc, b, x0, tol=1e-6, inj=O.Inject.rate(seed=9, lam=1e-4), check=False)
+        assert not np.array_equal(r.res_hist[: min(len(r.res_hist), len(clean.res_hist))],
+                                  clean.res_hist[: min(len(r.res_hist), len(clean.res_hist))])
