@@ -1,0 +1,356 @@
+#!/usr/bin/env python
+"""bench.py -- ABFT-SpMV (Schoell et al., DSN 2016) on B200.
+
+One step = one protected SpMV through the C ABI (abft_spmv with
+ABFT_CHECK | ABFT_AUTOCORRECT): the fused multiply + detect kernel (steps 1-4
+of Fig. 1, with the in-kernel finalize) plus the correction launches (step 5),
+over the BASELINE.json configs[1] workload (3-D 7-point Laplacian 128^3, FP64,
+synthetic) unless --workload says otherwise.
+
+Prints ONE JSON line (rank 0).  `value` = whole-job ABFT-SpMV throughput in
+GB/s of algorithmic bytes, inputs resident in HBM.
+`--impl reference` times the CPU oracle instead (the reference arm).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = ("ABFT-SpMV GB/s & % of HBM peak; FT overhead % vs plain SpMV; "
+          "coverage vs error rate")
+
+WORKLOADS = {
+    "7pt128": ("3-D 7-point Laplacian 128^3 FP64 ABFT-SpMV (BASELINE configs[1])",
+               lambda G: G.laplacian_3d_7pt(128)),
+    "5pt64": ("2-D 5-point Laplacian 64x64 FP64 ABFT-SpMV (BASELINE configs[0])",
+              lambda G: G.laplacian_2d_5pt(64)),
+    "27pt256": ("3-D 27-point stencil 256^3 FP64 ABFT-SpMV (BASELINE configs[3], 1 GPU)",
+                lambda G: G.stencil_3d_27pt(256)),
+    "27pt128": ("3-D 27-point stencil 128^3 FP64 ABFT-SpMV", lambda G: G.stencil_3d_27pt(128)),
+    "rmat20": ("R-MAT scale 20, edge factor 16, permuted, FP64 ABFT-SpMV",
+               lambda G: G.rmat(20, 16, 1)),
+}
+
+
+def load_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            p = json.load(f)
+        return float(p["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md: 6.65 TB/s)"
+
+
+def algorithmic_bytes(n, nnz, nb, nnz_c, check=True):
+    """A (CSR: 8+4 B per nnz + row_ptr), x read once, y written once; with
+    the check: C (CSR) + K.  DESIGN.md "Measurement"."""
+    b = 12 * nnz + 4 * (n + 1) + 16 * n
+    if check:
+        b += 12 * nnz_c + 4 * (nb + 1) + 8 * nb
+    return b
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.proc = None
+        self.f = None
+
+    def start(self):
+        try:
+            self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}",
+                 "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=self.f, stderr=subprocess.DEVNULL)
+        except Exception:
+            self.proc = None
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        self.f.flush()
+        rows = [ln.strip().split(", ") for ln in open(self.f.name) if ln.strip()]
+        os.unlink(self.f.name)
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for r in rows:
+            try:
+                sm.append(float(r[1]))
+                mx = float(r[2])
+                for nm, v in zip(names, r[5:9]):
+                    if v.strip().lower() == "active":
+                        reasons.add(nm)
+            except Exception:
+                continue
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": mx,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def dist_init():
+    import torch
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        import torch.distributed as dist
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    elif torch.cuda.is_available():
+        torch.cuda.set_device(local)
+    return world, rank, local
+
+
+def barrier(world):
+    if world > 1:
+        import torch.distributed as dist
+        dist.barrier()
+
+
+def max_over_ranks(v, world):
+    if world == 1:
+        return v
+    import torch
+    import torch.distributed as dist
+    t = torch.tensor([v], dtype=torch.float64, device="cuda")
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
+def timed(fn, steps, world):
+    """Device time per step (ms) over `steps` calls: CUDA events on the
+    current stream, barrier + synchronize on both sides, max over ranks."""
+    import torch
+    barrier(world)
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for _ in range(steps):
+        fn()
+    e1.record()
+    torch.cuda.synchronize()
+    barrier(world)
+    return max_over_ranks(e0.elapsed_time(e1) / steps, world)
+
+
+def oracle_baseline(A, x, seconds=12.0, check=True):
+    """The CPU oracle as it stands on this host (single thread), timed on
+    bounded repetitions of the same workload."""
+    from oracle import oracle as O
+    enc = O.encode(A, 32)
+    O.abft_spmv(A, enc, x)  # warm
+    t0 = time.perf_counter()
+    reps = 0
+    while True:
+        O.abft_spmv(A, enc, x)
+        reps += 1
+        if time.perf_counter() - t0 > seconds:
+            break
+    dt = (time.perf_counter() - t0) / reps
+    return enc, dt, reps
+
+
+def run_reference(args):
+    """--impl reference: the CPU oracle (oracle/liboracle.so), rank 0 only."""
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    from oracle import oracle as O
+    from paper_conf_dsn_schollbkw16_b200 import inputs as G
+    desc, gen = WORKLOADS[args.workload]
+    A = gen(G)
+    x = G.uniform_vector(A.n, 42)
+    enc = O.encode(A, 32)
+    nbytes = algorithmic_bytes(A.n, A.nnz, enc.nb, int(enc.col.size))
+    for _ in range(args.warmup):
+        O.abft_spmv(A, enc, x)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        O.abft_spmv(A, enc, x)
+    dt = (time.perf_counter() - t0) / max(args.steps, 1)
+    gbs = nbytes / dt / 1e9
+    line = {
+        "impl": "reference", "metric": METRIC, "value": round(gbs, 4), "unit": "GB/s",
+        "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": round(dt * 1e3, 3), "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": desc, "n": A.n, "nnz": A.nnz, "block_size": 32},
+        "cpu_baseline": {"value": round(gbs, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
+                         "sample": f"{args.steps} full protected SpMVs of the workload (oracle, 1 thread)"},
+        "e2e": {"value": round(gbs, 4), "unit": "GB/s", "h2d_bytes_per_step": 0,
+                "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def run_ours(args):
+    import numpy as np
+    import torch
+
+    from paper_conf_dsn_schollbkw16_b200 import AUTOCORRECT, CHECK, NOCHECK, Inject, encode
+    from paper_conf_dsn_schollbkw16_b200 import inputs as G
+
+    world, rank, local = dist_init()
+    desc, gen = WORKLOADS[args.workload]
+    A = gen(G)
+    h = encode(A, args.block_size, args.max_rounds)
+    n, nnz, nb = A.n, A.nnz, h.nb
+    nnz_c = int(h.checksum_matrix()[1].size)
+    xh = G.uniform_vector(n, 42 + rank)
+    x = torch.from_numpy(xh).cuda()
+    y = torch.empty_like(x)
+    inj = Inject.rate(seed=1234 + rank, lam=args.lam) if args.lam > 0 else None
+    prot_mode = CHECK | AUTOCORRECT
+
+    def step():
+        h.spmv(x, y, inject=inj, mode=prot_mode)
+
+    def plain():
+        h.spmv(x, y, inject=inj, mode=NOCHECK)
+
+    def fused_only():
+        h.spmv(x, y, inject=inj, mode=CHECK)
+
+    for _ in range(max(args.warmup, 3)):
+        step()
+        plain()
+        fused_only()
+    torch.cuda.synchronize()
+
+    clocks = ClockSampler(torch.cuda.current_device())
+    clocks.start()
+    # pre-roll (untimed) so the clock samples cover a loaded GPU
+    t_end = time.perf_counter() + 1.0
+    while time.perf_counter() < t_end:
+        for _ in range(50):
+            step()
+        torch.cuda.synchronize()
+    ms = timed(step, args.steps, world)
+    ms_plain = timed(plain, args.steps, world)
+    ms_fused = timed(fused_only, args.steps, world)
+    clk = clocks.stop()
+
+    nbytes = algorithmic_bytes(n, nnz, nb, nnz_c, True)
+    nbytes_plain = algorithmic_bytes(n, nnz, nb, nnz_c, False)
+    value = world * nbytes / (ms * 1e-3) / 1e9
+    fused_gbs = nbytes / (ms_fused * 1e-3) / 1e9
+    plain_gbs = nbytes_plain / (ms_plain * 1e-3) / 1e9
+    peak, peak_src = load_peaks()
+
+    # end-to-end through the public C ABI with host buffers (pinned)
+    xp = torch.from_numpy(xh).pin_memory()
+    yp = torch.empty(n, dtype=torch.float64).pin_memory()
+    xn, yn = xp.numpy(), yp.numpy()
+    k_e2e = max(3, min(args.steps, 200))
+    for _ in range(2):
+        h.spmv_host(xn, yn, prot_mode)
+    barrier(world)
+    t0 = time.perf_counter()
+    for _ in range(k_e2e):
+        h.spmv_host(xn, yn, prot_mode)
+    dt_e2e = max_over_ranks((time.perf_counter() - t0) / k_e2e, world)
+    e2e_gbs = world * nbytes / dt_e2e / 1e9
+
+    # measured ncu traffic for the fused kernel, if a capture was committed
+    traffic = None
+    tpath = os.path.join(ROOT, "profiles", f"traffic_{args.workload}.json")
+    if os.path.exists(tpath):
+        try:
+            traffic = json.load(open(tpath)).get("dram_bytes_per_launch")
+        except Exception:
+            traffic = None
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        _, dt_cpu, reps = oracle_baseline(A, xh, seconds=args.cpu_seconds)
+        cpu = {"value": round(nbytes / dt_cpu / 1e9, 4), "unit": "GB/s", "cores": 1,
+               "kind": "oracle",
+               "sample": f"{reps} full protected SpMVs of the same workload "
+                         f"({dt_cpu * 1e3:.1f} ms each, single thread)"}
+
+    if rank == 0:
+        line = {
+            "metric": METRIC,
+            "value": round(value, 2),
+            "unit": "GB/s",
+            "n_gpus": world,
+            "steps": args.steps,
+            "warmup": args.warmup,
+            "ms_per_step": round(ms, 5),
+            "higher_is_better": True,
+            "scaling": "weak",
+            "vs_baseline": None,
+            "dtype": "f64",
+            "data": "synthetic",
+            "config": {
+                "workload": desc, "n": n, "nnz": nnz, "nnz_c": nnz_c, "block_size": args.block_size,
+                "lambda": args.lam, "parallelism": f"replicas{world}" if world > 1 else "single",
+                "l2": "no flush: working set "
+                      f"{nbytes / 1e6:.0f} MB per step > 126 MB L2 (A, C streamed evict-first)",
+                "step": "abft_spmv(CHECK|AUTOCORRECT): fused multiply+detect+finalize, "
+                        f"{args.max_rounds} correction launches",
+                "bytes_per_step": nbytes,
+            },
+            "ft_overhead_pct": round((ms / ms_plain - 1) * 100, 2),
+            "plain_spmv_gbs": round(plain_gbs, 2),
+            "plain_ms": round(ms_plain, 5),
+            "roofline": {"bound": "hbm", "kernel": "k_fused<CHECK>",
+                         "achieved": round(fused_gbs, 2), "peak": peak, "unit": "GB/s",
+                         "frac": round(fused_gbs / peak, 4), "traffic": traffic,
+                         "peak_source": peak_src, "launch_ms": round(ms_fused, 5),
+                         "algorithmic_bytes_per_launch": nbytes},
+            "cpu_baseline": cpu,
+            "e2e": {"value": round(e2e_gbs, 3), "unit": "GB/s", "h2d_bytes_per_step": 8 * n,
+                    "d2h_bytes_per_step": 8 * n + 4, "ms_per_step": round(dt_e2e * 1e3, 4)},
+            "gpu_launches": args.steps * (1 + args.max_rounds),
+            "clocks": clk,
+        }
+        print(json.dumps(line), flush=True)
+    h.close()
+    if world > 1:
+        import torch.distributed as dist
+        dist.destroy_process_group()
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=10)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--workload", default="7pt128", choices=sorted(WORKLOADS))
+    ap.add_argument("--block-size", type=int, default=32)
+    ap.add_argument("--max-rounds", type=int, default=4)
+    ap.add_argument("--lam", type=float, default=0.0, help="rate-mode fault rate per op")
+    ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_ours(args)
+
+
+if __name__ == "__main__":
+    main()

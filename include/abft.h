@@ -1,0 +1,196 @@
+/*
+ * abft.h -- C ABI of the B200-native ABFT-SpMV library (libabft.so).
+ *
+ * Method: Schoell, Braun, Kochte, Wunderlich, "Efficient Algorithm-Based Fault
+ * Tolerance for Sparse Matrix Operations", DSN 2016 (PAPER.md; P:<n> = line).
+ *
+ *   abft_encode  -- build the sparse checksum matrix C and the bound constants
+ *                   once per matrix (SIII-B/C/D, P:94, P:108, P:128-130,
+ *                   P:156-160, Fig. 2/3).
+ *   abft_spmv    -- y = A x with detection and implicit localization in the
+ *                   same pass (Fig. 1 steps 1-4).
+ *   abft_correct -- partial recomputation of the flagged blocks only
+ *                   (Fig. 1 step 5), re-verified each round.
+ *   abft_pcg     -- Jacobi-preconditioned CG whose every SpMV is protected
+ *                   (SVI-A; success within 10 N iterations).
+ *
+ * Conventions (all entry points):
+ *  - Pointers are DEVICE pointers unless marked (host).  FP64 values, int32
+ *    indices, row-major CSR with columns ascending within each row and no
+ *    duplicates (square matrices in CSR).
+ *  - `stream` is a cudaStream_t passed as void* (NULL = legacy default
+ *    stream).  abft_spmv / abft_correct are stream-ordered and asynchronous:
+ *    they never synchronise with the host.  abft_encode synchronises once (to
+ *    size C); abft_pcg and abft_spmv_host synchronise before returning.
+ *  - No exception crosses the boundary.  Host-detectable argument errors
+ *    return ABFT_EINVAL immediately; CUDA errors return ABFT_ECUDA.
+ *  - Numerics: IEEE binary64, round-to-nearest, no FMA contraction; every
+ *    sum uses the canonical pairwise order PW of DESIGN.md (R2), so results
+ *    are bit-reproducible and bit-identical to the CPU oracle.
+ *  - A handle is not thread-safe; use it from one stream at a time.
+ */
+#ifndef ABFT_H
+#define ABFT_H
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  ABFT_OK = 0,
+  ABFT_EINVAL = -1,        /* bad argument (host-detected) */
+  ABFT_ECUDA = -2,         /* CUDA runtime error (see abft_last_cuda_error) */
+  ABFT_ENOMEM = -3,        /* device allocation failed */
+  ABFT_ENOTSUP = -4,       /* unsupported configuration (e.g. block_size > 32) */
+  ABFT_ENOCONV = -5,       /* PCG: not converged within max_iter */
+  ABFT_EUNCORRECTED = -6,  /* blocks still flagged after max_rounds recomputations */
+  ABFT_EBREAKDOWN = -7     /* PCG: p.q <= 0 or NaN residual */
+} abft_status;
+
+/* Square CSR matrix, DEVICE arrays. row_ptr[n+1], col_idx[nnz], val[nnz].
+ * The caller owns the arrays; they must outlive the handle (correction and
+ * PCG re-read A; it is never copied). */
+typedef struct {
+  int64_t n;
+  int64_t nnz;
+  const int32_t *row_ptr;
+  const int32_t *col_idx;
+  const double *val;
+} abft_csr_t;
+
+typedef struct abft_ctx *abft_handle_t;
+
+/* Fault injection (PAPER.md SIV-A, and the rate model of P:284).
+ * Test/experiment harness only; mode NONE (or inj == NULL) selects kernels
+ * compiled without any injection code.
+ *  LIST: entry e XORs list_mask[e] into the value produced for element
+ *        list_index[e] of target list_target[e] (0 = y row, 1 = t1 block,
+ *        2 = t2 block) in round list_round[e] (0 = main pass, r >= 1 = r-th
+ *        correction round).  The list arrays are HOST arrays, copied.
+ *  RATE: every produced value is faulty with probability
+ *        p = min(1, lambda * ops) (ops: 2*len(row) for y_i, 2*n_k for t1_k,
+ *        rows-in-block for t2_k), decided by Philox4x32-10 with counter
+ *        {index lo, index hi, call, round<<8 | target} and key {seed lo, seed
+ *        hi}: faulty iff word0 < floor(p * 2^32); the burst starts at bit
+ *        (word1 & 63) and its length is drawn from word2 through the table of
+ *        abft_burst_table (R12/R13). */
+enum { ABFT_INJ_NONE = 0, ABFT_INJ_LIST = 1, ABFT_INJ_RATE = 2 };
+enum { ABFT_TARGET_Y = 0, ABFT_TARGET_T1 = 1, ABFT_TARGET_T2 = 2 };
+typedef struct {
+  uint32_t mode;
+  uint64_t seed;
+  uint64_t call;       /* SpMV call index (rate mode counter word 2) */
+  double lambda;       /* rate mode: fault probability per arithmetic op */
+  uint32_t targets;    /* rate mode: bit t => target t receives faults */
+  int64_t n_list;      /* list mode */
+  const int32_t *list_round;   /* (host) */
+  const int32_t *list_target;  /* (host) */
+  const int64_t *list_index;   /* (host) */
+  const uint64_t *list_mask;   /* (host) */
+} abft_inject_t;
+
+/* abft_spmv mode bits */
+enum {
+  ABFT_NOCHECK = 0,          /* plain y = A x (the unprotected baseline) */
+  ABFT_CHECK = 1,            /* steps 1-4: y, t1, t2, s, beta, tau, flags */
+  ABFT_AUTOCORRECT = 2,      /* + step 5: up to max_rounds correction rounds */
+  ABFT_DEBUG_CHECKSUMS = 4   /* also store t1, t2 per block (abft_debug_checksums) */
+};
+
+/* Build C (CSR: nb rows, ascending columns = the non-empty columns of A_k,
+ * values = column sums of A_k) and K_k = ((n_k + 2 b_s - 2)
+ * * sum_{i in k} ||a_i||_2 + n_k ||c_k||_2) * 2^-53 (eps_M of P:154),
+ * so that tau_k = K_k * ||x||_2.  block_size: power of two in [1, 32]
+ * (default 32 = the paper's choice); otherwise ABFT_ENOTSUP.
+ * max_rounds: correction rounds for ABFT_AUTOCORRECT / abft_pcg (>= 1, <= 16;
+ * 0 -> 4).  flags: reserved, pass 0.  Synchronises `stream` once.
+ * On success *out owns C, K and all scratch (device). */
+abft_status abft_encode(const abft_csr_t *A, int32_t block_size, int32_t max_rounds,
+                        uint32_t flags, void *stream, abft_handle_t *out);
+
+/* Protected SpMV y = A x (steps 1-4), optionally with correction
+ * (mode | ABFT_AUTOCORRECT, step 5).  x and y: device [n], must not alias.
+ * x_norm: nullable DEVICE scalar holding ||x||_2 if the caller already has it
+ * (PW-exact value required for oracle parity); NULL -> computed in-pass.
+ * inj: nullable (no injection).  Flagged blocks stay on the device
+ * (abft_flags); nothing is copied to the host. */
+abft_status abft_spmv(abft_handle_t h, const double *x, double *y, const double *x_norm,
+                      const abft_inject_t *inj, uint32_t mode, void *stream);
+
+/* Step 5 alone: rounds r = 1..max_rounds recompute the rows of
+ * the blocks flagged in round r-1, recompute t1/t2 and re-check; blocks that
+ * still fail form round r's list.  Uses beta of the last abft_spmv. */
+abft_status abft_correct(abft_handle_t h, const double *x, double *y, int32_t max_rounds,
+                         const abft_inject_t *inj, void *stream);
+
+/* Device pointers to round `round`'s flagged-block list (unordered set of
+ * 0-based block indices) and its length (device int32).  Round 0 = detection;
+ * round r = blocks still failing after correction round r.  Valid until the
+ * next call on the handle.  round in [0, max_rounds]. */
+abft_status abft_flags(abft_handle_t h, int32_t round, const int32_t **flagged,
+                       const int32_t **n_flagged);
+
+/* Device pointer to beta = ||x||_2 of the last abft_spmv (device double). */
+abft_status abft_beta(abft_handle_t h, const double **beta);
+
+/* Device pointers to the encoded checksum matrix and bound constants. */
+abft_status abft_checksum_matrix(abft_handle_t h, const int32_t **c_row_ptr,
+                                 const int32_t **c_col, const double **c_val, const double **K,
+                                 int64_t *nnz_c, int64_t *nb);
+
+/* Device pointers to t1 / t2 of the last abft_spmv run with
+ * ABFT_DEBUG_CHECKSUMS (values after injection, before correction). */
+abft_status abft_debug_checksums(abft_handle_t h, const double **t1, const double **t2);
+
+/* End-to-end call with HOST buffers: copies x (host, pinned recommended) to
+ * the device, runs abft_spmv(mode), copies y back to y_host and the round-0
+ * flag count to *n_flagged_host (nullable), then synchronises `stream`. */
+abft_status abft_spmv_host(abft_handle_t h, const double *x_host, double *y_host,
+                           int32_t *n_flagged_host, uint32_t mode, void *stream);
+
+/* PCG statistics (host struct). */
+typedef struct {
+  int64_t iters;
+  int64_t spmv_calls;
+  int64_t flagged_blocks;    /* sum over SpMV calls of round-0 flags */
+  int64_t recomputed_blocks; /* sum over calls and rounds of recomputed blocks */
+  int64_t uncorrected_calls; /* calls that ended with blocks still flagged */
+  int32_t converged;
+  double final_residual;     /* ||r||_2 of the recursive residual */
+} abft_pcg_stats_t;
+
+/* Jacobi-PCG (Saad Alg. 9.1) for SPD A: solves A x = b from the
+ * initial guess in x (overwritten with the solution).  diag: nullable device
+ * [n] (NULL -> the diagonal of A).  Stops when ||r||_2 <= tol * ||b||_2
+ * (R16) or after max_iter iterations (<= 0 -> 10 N).
+ * check != 0 protects every SpMV (detect + correct); check == 0 runs the
+ * unprotected baseline with the same kernels.  inj: nullable; its `call`
+ * is the index of the first SpMV (call + j for the j-th).  res_hist:
+ * nullable device [max_iter + 1] of ||r_j||_2.  stats: nullable (host).
+ * Synchronises the stream.  Returns ABFT_OK, ABFT_ENOCONV or ABFT_EBREAKDOWN. */
+abft_status abft_pcg(abft_handle_t h, const double *b, double *x, const double *diag,
+                     double tol, int64_t max_iter, const abft_inject_t *inj, int32_t check,
+                     double *res_hist, abft_pcg_stats_t *stats, void *stream);
+
+abft_status abft_destroy(abft_handle_t h);
+
+/* Plumbing for bindings: cudaMemcpyAsync(dst, src, bytes, cudaMemcpyDefault)
+ * on `stream`, then synchronise it.  Used to read the device-resident results
+ * above (flags, counts, C, K, beta) without a second CUDA binding. */
+abft_status abft_memcpy(void *dst, const void *src, int64_t bytes, void *stream);
+
+/* Host helpers (no GPU needed). */
+const char *abft_status_string(abft_status st);
+const char *abft_last_cuda_error(void);
+/* The burst-length table the device injector uses: T[l] = floor(2^32 *
+ * P(L <= l)), L = max(1, round(3 + sqrt(2) Z)) (R12),
+ * computed on the host with the C library's erfc. */
+void abft_burst_table(uint64_t T[65]);
+/* Library version string. */
+const char *abft_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* ABFT_H */

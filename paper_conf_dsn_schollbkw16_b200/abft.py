@@ -1,0 +1,298 @@
+"""Thin Python binding of libabft.so (include/abft.h): argument marshalling
+only.  Every step of the path runs in the library's CUDA kernels; there is no
+CPU fallback -- if libabft.so is missing or no CUDA device is present, every
+call raises.
+
+PyTorch provides device memory and the current stream (plumbing only).
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+from dataclasses import dataclass
+
+import numpy as np
+
+from . import _build
+
+_LIB = None
+
+OK, EINVAL, ECUDA, ENOMEM, ENOTSUP, ENOCONV, EUNCORRECTED, EBREAKDOWN = 0, -1, -2, -3, -4, -5, -6, -7
+NOCHECK, CHECK, AUTOCORRECT, DEBUG_CHECKSUMS = 0, 1, 2, 4
+INJ_NONE, INJ_LIST, INJ_RATE = 0, 1, 2
+
+SYMBOLS = [
+    "abft_encode", "abft_spmv", "abft_correct", "abft_flags", "abft_beta",
+    "abft_checksum_matrix", "abft_debug_checksums", "abft_spmv_host", "abft_pcg",
+    "abft_destroy", "abft_memcpy", "abft_status_string", "abft_last_cuda_error",
+    "abft_burst_table", "abft_version",
+]
+
+
+class AbftError(RuntimeError):
+    def __init__(self, status, where):
+        self.status = status
+        msg = lib().abft_status_string(status).decode()
+        if status == ECUDA:
+            msg += ": " + lib().abft_last_cuda_error().decode()
+        super().__init__(f"{where}: {msg} ({status})")
+
+
+class _Csr(C.Structure):
+    _fields_ = [("n", C.c_int64), ("nnz", C.c_int64), ("row_ptr", C.c_void_p),
+                ("col_idx", C.c_void_p), ("val", C.c_void_p)]
+
+
+class _Inj(C.Structure):
+    _fields_ = [("mode", C.c_uint32), ("seed", C.c_uint64), ("call", C.c_uint64),
+                ("lambda_", C.c_double), ("targets", C.c_uint32), ("n_list", C.c_int64),
+                ("list_round", C.c_void_p), ("list_target", C.c_void_p),
+                ("list_index", C.c_void_p), ("list_mask", C.c_void_p)]
+
+
+class PcgStats(C.Structure):
+    _fields_ = [("iters", C.c_int64), ("spmv_calls", C.c_int64), ("flagged_blocks", C.c_int64),
+                ("recomputed_blocks", C.c_int64), ("uncorrected_calls", C.c_int64),
+                ("converged", C.c_int32), ("final_residual", C.c_double)]
+
+    def as_dict(self):
+        return {f: getattr(self, f) for f, _ in self._fields_}
+
+
+def lib_path() -> str:
+    return _build.LIB
+
+
+def lib():
+    """Load libabft.so (raises if it has not been built -- no fallback)."""
+    global _LIB
+    if _LIB is None:
+        path = lib_path()
+        if not os.path.exists(path):
+            raise RuntimeError(f"libabft.so not built at {path}; run __graft_entry__.build()")
+        L = C.CDLL(path)
+        P, i32, i64, u32, d = C.c_void_p, C.c_int32, C.c_int64, C.c_uint32, C.c_double
+        st = C.c_int
+        L.abft_encode.restype = st
+        L.abft_encode.argtypes = [P, i32, i32, u32, P, C.POINTER(P)]
+        L.abft_spmv.restype = st
+        L.abft_spmv.argtypes = [P, P, P, P, P, u32, P]
+        L.abft_correct.restype = st
+        L.abft_correct.argtypes = [P, P, P, i32, P, P]
+        L.abft_flags.restype = st
+        L.abft_flags.argtypes = [P, i32, C.POINTER(P), C.POINTER(P)]
+        L.abft_beta.restype = st
+        L.abft_beta.argtypes = [P, C.POINTER(P)]
+        L.abft_checksum_matrix.restype = st
+        L.abft_checksum_matrix.argtypes = [P, C.POINTER(P), C.POINTER(P), C.POINTER(P),
+                                           C.POINTER(P), C.POINTER(i64), C.POINTER(i64)]
+        L.abft_debug_checksums.restype = st
+        L.abft_debug_checksums.argtypes = [P, C.POINTER(P), C.POINTER(P)]
+        L.abft_spmv_host.restype = st
+        L.abft_spmv_host.argtypes = [P, P, P, P, u32, P]
+        L.abft_pcg.restype = st
+        L.abft_pcg.argtypes = [P, P, P, P, d, i64, P, i32, P, C.POINTER(PcgStats), P]
+        L.abft_destroy.restype = st
+        L.abft_destroy.argtypes = [P]
+        L.abft_memcpy.restype = st
+        L.abft_memcpy.argtypes = [P, P, i64, P]
+        L.abft_status_string.restype = C.c_char_p
+        L.abft_status_string.argtypes = [st]
+        L.abft_last_cuda_error.restype = C.c_char_p
+        L.abft_burst_table.argtypes = [P]
+        L.abft_version.restype = C.c_char_p
+        _LIB = L
+    return _LIB
+
+
+def _check(status, where):
+    if status != OK:
+        raise AbftError(status, where)
+
+
+def _stream(stream=None):
+    import torch
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return C.c_void_p(s.cuda_stream)
+
+
+def _ptr(t):
+    return None if t is None else C.c_void_p(t.data_ptr())
+
+
+def burst_table() -> np.ndarray:
+    t = np.zeros(65, dtype=np.uint64)
+    lib().abft_burst_table(t.ctypes.data_as(C.c_void_p))
+    return t
+
+
+class Inject:
+    """Fault injection spec (abft_inject_t).  LIST plans are FaultPlan objects
+    from `inputs`; RATE mode uses the device-side Philox injector."""
+
+    def __init__(self, mode=INJ_NONE, seed=0, call=0, lam=0.0, targets=0b111, plan=None):
+        self.mode, self.seed, self.call, self.lam, self.targets, self.plan = (
+            mode, seed, call, lam, targets, plan)
+
+    @staticmethod
+    def from_plan(plan):
+        return Inject(mode=INJ_LIST, plan=plan)
+
+    @staticmethod
+    def rate(seed, lam, targets=0b111, call=0):
+        return Inject(mode=INJ_RATE, seed=seed, call=call, lam=lam, targets=targets)
+
+    def struct(self):
+        s = _Inj()
+        s.mode, s.seed, s.call, s.lambda_, s.targets = (self.mode, self.seed, self.call,
+                                                        self.lam, self.targets)
+        s.n_list = 0
+        if self.mode == INJ_LIST and self.plan is not None and len(self.plan):
+            self._keep = (np.ascontiguousarray(self.plan.round, np.int32),
+                          np.ascontiguousarray(self.plan.target, np.int32),
+                          np.ascontiguousarray(self.plan.index, np.int64),
+                          np.ascontiguousarray(self.plan.mask, np.uint64))
+            s.n_list = len(self.plan)
+            (s.list_round, s.list_target, s.list_index, s.list_mask) = [
+                a.ctypes.data for a in self._keep]
+        return s
+
+
+@dataclass
+class CsrDevice:
+    """CSR matrix resident on the device (torch tensors)."""
+    n: int
+    row_ptr: object
+    col: object
+    val: object
+
+    @property
+    def nnz(self):
+        return int(self.col.numel())
+
+    @staticmethod
+    def from_host(A, device="cuda"):
+        import torch
+        return CsrDevice(A.n, torch.from_numpy(np.ascontiguousarray(A.row_ptr)).to(device),
+                         torch.from_numpy(np.ascontiguousarray(A.col)).to(device),
+                         torch.from_numpy(np.ascontiguousarray(A.val)).to(device))
+
+
+class Handle:
+    """abft_handle_t: owns C, K and scratch; keeps A alive (the library
+    re-reads it in correction and PCG)."""
+
+    def __init__(self, A: CsrDevice, block_size: int = 32, max_rounds: int = 4, stream=None):
+        self.A = A
+        self.n = A.n
+        self.block_size = block_size
+        self.nb = (A.n + block_size - 1) // block_size
+        self.max_rounds = max_rounds if max_rounds > 0 else 4
+        csr = _Csr(A.n, A.nnz, A.row_ptr.data_ptr(), A.col.data_ptr() if A.nnz else 0,
+                   A.val.data_ptr() if A.nnz else 0)
+        h = C.c_void_p()
+        _check(lib().abft_encode(C.byref(csr), block_size, max_rounds, 0, _stream(stream),
+                                 C.byref(h)), "abft_encode")
+        self._h = h
+
+    def close(self):
+        if getattr(self, "_h", None) and self._h.value:
+            lib().abft_destroy(self._h)
+            self._h = C.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    # -- hot path --------------------------------------------------------
+    def spmv(self, x, y=None, x_norm=None, inject: Inject | None = None, mode=CHECK, stream=None):
+        import torch
+        if y is None:
+            y = torch.empty_like(x)
+        inj = inject.struct() if inject is not None else None
+        _check(lib().abft_spmv(self._h, _ptr(x), _ptr(y), _ptr(x_norm),
+                               C.byref(inj) if inj is not None else None, mode, _stream(stream)),
+               "abft_spmv")
+        return y
+
+    def correct(self, x, y, max_rounds=0, inject: Inject | None = None, stream=None):
+        inj = inject.struct() if inject is not None else None
+        _check(lib().abft_correct(self._h, _ptr(x), _ptr(y), max_rounds,
+                                  C.byref(inj) if inj is not None else None, _stream(stream)),
+               "abft_correct")
+        return y
+
+    def spmv_host(self, x_host: np.ndarray, y_host: np.ndarray, mode=CHECK | AUTOCORRECT,
+                  stream=None) -> int:
+        nf = C.c_int32(0)
+        _check(lib().abft_spmv_host(self._h, x_host.ctypes.data_as(C.c_void_p),
+                                    y_host.ctypes.data_as(C.c_void_p), C.byref(nf), mode,
+                                    _stream(stream)), "abft_spmv_host")
+        return nf.value
+
+    # -- results (device-resident; copied out on request) ----------------
+    def _d2h(self, ptr, count, dtype, stream=None):
+        out = np.empty(count, dtype=dtype)
+        if count:
+            _check(lib().abft_memcpy(out.ctypes.data_as(C.c_void_p), ptr, out.nbytes,
+                                     _stream(stream)), "abft_memcpy")
+        return out
+
+    def flags(self, round_: int = 0, stream=None) -> np.ndarray:
+        """Sorted flagged-block indices of round `round_` (copied to host)."""
+        f, nf = C.c_void_p(), C.c_void_p()
+        _check(lib().abft_flags(self._h, round_, C.byref(f), C.byref(nf)), "abft_flags")
+        cnt = int(self._d2h(nf, 1, np.int32, stream)[0])
+        return np.sort(self._d2h(f, cnt, np.int32, stream))
+
+    def all_flags(self, stream=None):
+        return [self.flags(r, stream) for r in range(self.max_rounds + 1)]
+
+    def flag_count_ptr(self, round_: int = 0) -> int:
+        f, nf = C.c_void_p(), C.c_void_p()
+        _check(lib().abft_flags(self._h, round_, C.byref(f), C.byref(nf)), "abft_flags")
+        return nf.value
+
+    def beta(self, stream=None) -> float:
+        b = C.c_void_p()
+        _check(lib().abft_beta(self._h, C.byref(b)), "abft_beta")
+        return float(self._d2h(b, 1, np.float64, stream)[0])
+
+    def checksum_matrix(self, stream=None):
+        rp, col, val, K = C.c_void_p(), C.c_void_p(), C.c_void_p(), C.c_void_p()
+        nnz_c, nb = C.c_int64(), C.c_int64()
+        _check(lib().abft_checksum_matrix(self._h, C.byref(rp), C.byref(col), C.byref(val),
+                                          C.byref(K), C.byref(nnz_c), C.byref(nb)),
+               "abft_checksum_matrix")
+        return (self._d2h(rp, nb.value + 1, np.int32, stream),
+                self._d2h(col, nnz_c.value, np.int32, stream),
+                self._d2h(val, nnz_c.value, np.float64, stream),
+                self._d2h(K, nb.value, np.float64, stream))
+
+    def debug_checksums(self, stream=None):
+        t1, t2 = C.c_void_p(), C.c_void_p()
+        _check(lib().abft_debug_checksums(self._h, C.byref(t1), C.byref(t2)),
+               "abft_debug_checksums")
+        return (self._d2h(t1, self.nb, np.float64, stream),
+                self._d2h(t2, self.nb, np.float64, stream))
+
+    # -- PCG ----------------------------------------------------------------
+    def pcg(self, b, x, diag=None, tol=1e-6, max_iter=0, inject: Inject | None = None,
+            check=True, res_hist=None, stream=None):
+        st = PcgStats()
+        inj = inject.struct() if inject is not None else None
+        status = lib().abft_pcg(self._h, _ptr(b), _ptr(x), _ptr(diag), tol, max_iter,
+                                C.byref(inj) if inj is not None else None, 1 if check else 0,
+                                _ptr(res_hist), C.byref(st), _stream(stream))
+        if status not in (OK, ENOCONV, EBREAKDOWN):
+            _check(status, "abft_pcg")
+        return status, st.as_dict()
+
+
+def encode(A, block_size: int = 32, max_rounds: int = 4, stream=None) -> Handle:
+    """Encode a CSR matrix (host `inputs.CSR` or a `CsrDevice`)."""
+    if not isinstance(A, CsrDevice):
+        A = CsrDevice.from_host(A)
+    return Handle(A, block_size, max_rounds, stream)

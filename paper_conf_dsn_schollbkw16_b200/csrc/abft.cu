@@ -1,0 +1,459 @@
+// abft.cu -- libabft.so: the C ABI of include/abft.h over the sm_100a kernels.
+// Single translation unit (kernels are header-only templates).
+#include <algorithm>
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <vector>
+
+#include "../../include/abft.h"
+#include "abft_device.cuh"
+#include "kernels_encode.cuh"
+#include "kernels_pcg.cuh"
+#include "kernels_spmv.cuh"
+
+using namespace abft;
+
+namespace {
+
+thread_local char g_cuda_err[256] = "";
+
+abft_status cuda_fail(cudaError_t e, const char *where) {
+  snprintf(g_cuda_err, sizeof g_cuda_err, "%s: %s", where, cudaGetErrorString(e));
+  return ABFT_ECUDA;
+}
+
+#define CK(call)                                          \
+  do {                                                    \
+    cudaError_t e_ = (call);                              \
+    if (e_ != cudaSuccess) return cuda_fail(e_, #call);   \
+  } while (0)
+
+#define CKM(call)                                                              \
+  do {                                                                         \
+    cudaError_t e_ = (call);                                                   \
+    if (e_ == cudaErrorMemoryAllocation) {                                     \
+      cudaGetLastError();                                                      \
+      return ABFT_ENOMEM;                                                      \
+    }                                                                          \
+    if (e_ != cudaSuccess) return cuda_fail(e_, #call);                        \
+  } while (0)
+
+void host_burst_table(uint64_t T[65]) {
+  T[0] = 0;
+  for (int l = 1; l < 64; ++l) {
+    const double p = 0.5 * std::erfc(-((double)l - 2.5) / 2.0);
+    T[l] = (uint64_t)std::floor(std::ldexp(p, 32));
+  }
+  T[64] = (uint64_t)1 << 32;
+}
+
+int g_table_device = -1;  // device the burst table was uploaded to
+
+}  // namespace
+
+struct abft_ctx {
+  int64_t n = 0, nnz = 0, nb = 0;
+  int32_t bs = 32, log2bs = 5, max_rounds = 4;
+  const int32_t *rp = nullptr, *ci = nullptr;
+  const double *va = nullptr;
+  int32_t *c_rp = nullptr, *c_col = nullptr;
+  double *c_val = nullptr, *K = nullptr;
+  int64_t nnz_c = 0;
+  int32_t max_seg = 0;
+  int cap = 0;  // staging capacity in products per warp (0: fallback only)
+  int64_t ncta = 0;
+  // scratch
+  double *partials = nullptr;
+  unsigned *done = nullptr;
+  int32_t *n_cand = nullptr, *cand = nullptr;
+  double *cand_s = nullptr;
+  int32_t *flags = nullptr, *n_flags = nullptr;
+  double *beta = nullptr;
+  double *dbg_t1 = nullptr, *dbg_t2 = nullptr;
+  uint64_t *inj_keys = nullptr, *inj_masks = nullptr;
+  int64_t inj_cap = 0;
+  double *hx = nullptr, *hy = nullptr;  // device staging for abft_spmv_host
+  // PCG scratch
+  double *pcg = nullptr;   // r, z, p, q, d : 5 n
+  double *pcg_part = nullptr;
+  double *pcg_sc = nullptr;
+  int64_t *pcg_it = nullptr;
+  int32_t *pcg_state = nullptr;
+  int64_t pcg_n = 0;
+  std::vector<void *> owned;
+  int device = 0;
+  int num_sms = 148;
+};
+
+namespace {
+
+template <typename T>
+abft_status dalloc(abft_ctx *h, T **p, size_t count) {
+  void *q = nullptr;
+  cudaError_t e = cudaMalloc(&q, std::max<size_t>(count, 1) * sizeof(T));
+  if (e == cudaErrorMemoryAllocation) {
+    cudaGetLastError();
+    return ABFT_ENOMEM;
+  }
+  if (e != cudaSuccess) return cuda_fail(e, "cudaMalloc");
+  h->owned.push_back(q);
+  *p = static_cast<T *>(q);
+  return ABFT_OK;
+}
+
+#define TRY(expr)                         \
+  do {                                    \
+    abft_status s_ = (expr);              \
+    if (s_ != ABFT_OK) return s_;         \
+  } while (0)
+
+SpmvArgs make_args(const abft_ctx *h, const double *x, double *y, const double *x_norm) {
+  SpmvArgs a;
+  memset(&a, 0, sizeof a);
+  a.n = h->n;
+  a.bs = h->bs;
+  a.log2bs = h->log2bs;
+  a.nb = h->nb;
+  a.rp = h->rp;
+  a.ci = h->ci;
+  a.va = h->va;
+  a.crp = h->c_rp;
+  a.ccol = h->c_col;
+  a.cval = h->c_val;
+  a.K = h->K;
+  a.x = x;
+  a.y = y;
+  a.x_norm = x_norm;
+  a.partials = h->partials;
+  a.done = h->done;
+  a.n_cand = h->n_cand;
+  a.cand = h->cand;
+  a.cand_s = h->cand_s;
+  a.flags = h->flags;
+  a.n_flags = h->n_flags;
+  a.max_rounds = h->max_rounds;
+  a.beta = h->beta;
+  return a;
+}
+
+// Upload a list-mode fault plan (sorted keys) and fill the device descriptor.
+abft_status prepare_inject(abft_ctx *h, const abft_inject_t *inj, cudaStream_t s, InjDev *d) {
+  memset(d, 0, sizeof *d);
+  if (!inj || inj->mode == ABFT_INJ_NONE) return ABFT_OK;
+  if (inj->mode == ABFT_INJ_RATE) {
+    if (!(inj->lambda >= 0.0)) return ABFT_EINVAL;
+    d->mode = 2;
+    d->key0 = (uint32_t)inj->seed;
+    d->key1 = (uint32_t)(inj->seed >> 32);
+    d->call = (uint32_t)inj->call;
+    d->lambda = inj->lambda;
+    d->targets = inj->targets;
+    return ABFT_OK;
+  }
+  if (inj->mode != ABFT_INJ_LIST) return ABFT_EINVAL;
+  if (inj->n_list < 0 || inj->n_list > (1 << 30)) return ABFT_EINVAL;
+  d->mode = 1;
+  d->n_list = (int32_t)inj->n_list;
+  if (inj->n_list == 0) return ABFT_OK;
+  if (!inj->list_round || !inj->list_target || !inj->list_index || !inj->list_mask)
+    return ABFT_EINVAL;
+  std::vector<std::pair<uint64_t, uint64_t>> kv((size_t)inj->n_list);
+  for (int64_t e = 0; e < inj->n_list; ++e) {
+    const int32_t r = inj->list_round[e], t = inj->list_target[e];
+    const int64_t idx = inj->list_index[e];
+    if (r < 0 || r > 31 || t < 0 || t > 2 || idx < 0 || idx >= ((int64_t)1 << 56))
+      return ABFT_EINVAL;
+    kv[(size_t)e] = {((uint64_t)r << 58) | ((uint64_t)t << 56) | (uint64_t)idx, inj->list_mask[e]};
+  }
+  std::sort(kv.begin(), kv.end(),
+            [](const auto &p, const auto &q) { return p.first < q.first; });
+  if (inj->n_list > h->inj_cap) {
+    int64_t cap = std::max<int64_t>(inj->n_list, 1024);
+    TRY(dalloc(h, &h->inj_keys, (size_t)cap));
+    TRY(dalloc(h, &h->inj_masks, (size_t)cap));
+    h->inj_cap = cap;
+  }
+  std::vector<uint64_t> keys(kv.size()), masks(kv.size());
+  for (size_t e = 0; e < kv.size(); ++e) {
+    keys[e] = kv[e].first;
+    masks[e] = kv[e].second;
+  }
+  CK(cudaMemcpyAsync(h->inj_keys, keys.data(), keys.size() * 8, cudaMemcpyHostToDevice, s));
+  CK(cudaMemcpyAsync(h->inj_masks, masks.data(), masks.size() * 8, cudaMemcpyHostToDevice, s));
+  CK(cudaStreamSynchronize(s));  // host vectors die at return
+  d->keys = h->inj_keys;
+  d->masks = h->inj_masks;
+  return ABFT_OK;
+}
+
+template <bool CHECK, bool INJECT>
+abft_status launch_fused_t(const abft_ctx *h, const SpmvArgs &a, cudaStream_t s) {
+  const unsigned grid = (unsigned)h->ncta;
+  if (h->cap == 1024) {
+    const size_t smem = (size_t)kWarps * 1024 * sizeof(double);
+    k_fused<CHECK, INJECT, 1024><<<grid, kThreads, smem, s>>>(a);
+  } else if (h->cap == 256) {
+    const size_t smem = (size_t)kWarps * 256 * sizeof(double);
+    k_fused<CHECK, INJECT, 256><<<grid, kThreads, smem, s>>>(a);
+  } else {
+    return ABFT_EINVAL;
+  }
+  CK(cudaGetLastError());
+  return ABFT_OK;
+}
+
+abft_status launch_fused(const abft_ctx *h, const SpmvArgs &a, bool check, cudaStream_t s) {
+  const bool inj = a.inj.mode != 0;
+  if (check) return inj ? launch_fused_t<true, true>(h, a, s) : launch_fused_t<true, false>(h, a, s);
+  return inj ? launch_fused_t<false, true>(h, a, s) : launch_fused_t<false, false>(h, a, s);
+}
+
+abft_status launch_correct(const abft_ctx *h, const SpmvArgs &a, int rounds, cudaStream_t s) {
+  const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>(h->num_sms * 4, (h->nb + 7) / 8));
+  for (int r = 1; r <= rounds; ++r) {
+    if (a.inj.mode != 0)
+      k_correct<true><<<grid, 256, 0, s>>>(a, r);
+    else
+      k_correct<false><<<grid, 256, 0, s>>>(a, r);
+    CK(cudaGetLastError());
+  }
+  return ABFT_OK;
+}
+
+template <typename K>
+abft_status set_smem(K kern, size_t bytes) {
+  CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes));
+  return ABFT_OK;
+}
+
+abft_status init_kernels() {
+  const size_t b1024 = (size_t)kWarps * 1024 * sizeof(double);
+  TRY(set_smem(k_fused<true, true, 1024>, b1024));
+  TRY(set_smem(k_fused<true, false, 1024>, b1024));
+  TRY(set_smem(k_fused<false, true, 1024>, b1024));
+  TRY(set_smem(k_fused<false, false, 1024>, b1024));
+  return ABFT_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+const char *abft_version(void) { return "abft-b200 0.1 (sm_100a)"; }
+
+const char *abft_last_cuda_error(void) { return g_cuda_err; }
+
+const char *abft_status_string(abft_status st) {
+  switch (st) {
+    case ABFT_OK: return "ok";
+    case ABFT_EINVAL: return "invalid argument";
+    case ABFT_ECUDA: return "CUDA error";
+    case ABFT_ENOMEM: return "out of device memory";
+    case ABFT_ENOTSUP: return "unsupported configuration";
+    case ABFT_ENOCONV: return "PCG did not converge";
+    case ABFT_EUNCORRECTED: return "blocks remain flagged after correction";
+    case ABFT_EBREAKDOWN: return "PCG breakdown";
+  }
+  return "unknown status";
+}
+
+void abft_burst_table(uint64_t T[65]) { host_burst_table(T); }
+
+abft_status abft_destroy(abft_handle_t h) {
+  if (!h) return ABFT_EINVAL;
+  for (void *p : h->owned) cudaFree(p);
+  delete h;
+  return ABFT_OK;
+}
+
+abft_status abft_encode(const abft_csr_t *A, int32_t block_size, int32_t max_rounds,
+                        uint32_t flags, void *stream, abft_handle_t *out) {
+  if (!A || !out || flags != 0) return ABFT_EINVAL;
+  *out = nullptr;
+  if (A->n <= 0 || A->n >= ((int64_t)1 << 31) - 64 || A->nnz < 0 || A->nnz >= ((int64_t)1 << 31))
+    return ABFT_EINVAL;
+  if (!A->row_ptr || (A->nnz > 0 && (!A->col_idx || !A->val))) return ABFT_EINVAL;
+  if (block_size <= 0 || (block_size & (block_size - 1)) != 0) return ABFT_EINVAL;
+  if (block_size > 32) return ABFT_ENOTSUP;
+  if (max_rounds == 0) max_rounds = 4;
+  if (max_rounds < 1 || max_rounds > 16) return ABFT_EINVAL;
+  cudaStream_t s = (cudaStream_t)stream;
+  abft_ctx *h = new abft_ctx();
+  auto fail = [&](abft_status st) {
+    abft_destroy(h);
+    return st;
+  };
+  CK(cudaGetDevice(&h->device));
+  CK(cudaDeviceGetAttribute(&h->num_sms, cudaDevAttrMultiProcessorCount, h->device));
+  if (g_table_device != h->device) {
+    uint64_t T[65];
+    host_burst_table(T);
+    CK(cudaMemcpyToSymbol(c_burst_T, T, sizeof T));
+    abft_status st = init_kernels();
+    if (st != ABFT_OK) return fail(st);
+    g_table_device = h->device;
+  }
+  h->n = A->n;
+  h->nnz = A->nnz;
+  h->bs = block_size;
+  h->log2bs = 0;
+  while ((1 << h->log2bs) < block_size) ++h->log2bs;
+  h->nb = (h->n + block_size - 1) / block_size;
+  h->max_rounds = max_rounds;
+  h->rp = A->row_ptr;
+  h->ci = A->col_idx;
+  h->va = A->val;
+  h->ncta = (h->n + kThreads - 1) / kThreads;
+
+  abft_status st;
+  int32_t *counts = nullptr, *totals = nullptr, *max_seg = nullptr;
+  const int64_t nscan = (h->nb + 1023) / 1024;
+  if ((st = dalloc(h, &h->c_rp, (size_t)h->nb + 1)) || (st = dalloc(h, &counts, (size_t)h->nb)) ||
+      (st = dalloc(h, &totals, (size_t)nscan)) || (st = dalloc(h, &max_seg, 1)) ||
+      (st = dalloc(h, &h->K, (size_t)h->nb)))
+    return fail(st);
+  cudaError_t e;
+  if ((e = cudaMemsetAsync(max_seg, 0, sizeof(int32_t), s)) != cudaSuccess)
+    return fail(cuda_fail(e, "memset"));
+  EncodeArgs ea;
+  memset(&ea, 0, sizeof ea);
+  ea.n = h->n;
+  ea.bs = h->bs;
+  ea.nb = h->nb;
+  ea.rp = h->rp;
+  ea.ci = h->ci;
+  ea.va = h->va;
+  ea.counts = counts;
+  ea.crp = h->c_rp;
+  ea.K = h->K;
+  ea.max_seg = max_seg;
+  const unsigned egrid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((h->nb + 7) / 8, 65535));
+  k_encode<false><<<egrid, 256, 0, s>>>(ea);
+  k_scan_local<<<(unsigned)nscan, 1024, 0, s>>>(counts, h->c_rp, h->nb, totals);
+  k_scan_totals<<<1, 1024, 0, s>>>(totals, nscan, h->c_rp + h->nb);
+  k_scan_add<<<(unsigned)nscan, 1024, 0, s>>>(h->c_rp, h->nb, totals);
+  if ((e = cudaGetLastError()) != cudaSuccess) return fail(cuda_fail(e, "encode count"));
+  int32_t host_tot[2];
+  if ((e = cudaMemcpyAsync(&host_tot[0], h->c_rp + h->nb, 4, cudaMemcpyDeviceToHost, s)) ||
+      (e = cudaMemcpyAsync(&host_tot[1], max_seg, 4, cudaMemcpyDeviceToHost, s)) ||
+      (e = cudaStreamSynchronize(s)))
+    return fail(cuda_fail(e, "encode sync"));
+  h->nnz_c = host_tot[0];
+  h->max_seg = host_tot[1];
+  h->cap = h->max_seg <= 256 ? 256 : (h->max_seg <= 1024 ? 1024 : 1024);
+  if ((st = dalloc(h, &h->c_col, (size_t)h->nnz_c)) || (st = dalloc(h, &h->c_val, (size_t)h->nnz_c)))
+    return fail(st);
+  ea.ccol = h->c_col;
+  ea.cval = h->c_val;
+  k_encode<true><<<egrid, 256, 0, s>>>(ea);
+  if ((e = cudaGetLastError()) != cudaSuccess) return fail(cuda_fail(e, "encode fill"));
+
+  // per-call scratch
+  if ((st = dalloc(h, &h->partials, (size_t)h->ncta)) || (st = dalloc(h, &h->done, 1)) ||
+      (st = dalloc(h, &h->n_cand, 1)) || (st = dalloc(h, &h->cand, (size_t)h->nb)) ||
+      (st = dalloc(h, &h->cand_s, (size_t)h->nb)) ||
+      (st = dalloc(h, &h->flags, (size_t)(h->max_rounds + 1) * h->nb)) ||
+      (st = dalloc(h, &h->n_flags, (size_t)h->max_rounds + 1)) || (st = dalloc(h, &h->beta, 1)) ||
+      (st = dalloc(h, &h->dbg_t1, (size_t)h->nb)) || (st = dalloc(h, &h->dbg_t2, (size_t)h->nb)))
+    return fail(st);
+  if ((e = cudaMemsetAsync(h->done, 0, sizeof(unsigned), s)) ||
+      (e = cudaMemsetAsync(h->n_cand, 0, sizeof(int32_t), s)) ||
+      (e = cudaMemsetAsync(h->n_flags, 0, sizeof(int32_t) * (h->max_rounds + 1), s)) ||
+      (e = cudaMemsetAsync(h->beta, 0, sizeof(double), s)) || (e = cudaStreamSynchronize(s)))
+    return fail(cuda_fail(e, "scratch init"));
+  *out = h;
+  return ABFT_OK;
+}
+
+abft_status abft_spmv(abft_handle_t h, const double *x, double *y, const double *x_norm,
+                      const abft_inject_t *inj, uint32_t mode, void *stream) {
+  if (!h || !x || !y || x == y) return ABFT_EINVAL;
+  if (mode & ~7u) return ABFT_EINVAL;
+  cudaStream_t s = (cudaStream_t)stream;
+  SpmvArgs a = make_args(h, x, y, x_norm);
+  TRY(prepare_inject(h, inj, s, &a.inj));
+  const bool check = (mode & ABFT_CHECK) || (mode & ABFT_AUTOCORRECT);
+  if (check && (mode & ABFT_DEBUG_CHECKSUMS)) {
+    a.dbg_t1 = h->dbg_t1;
+    a.dbg_t2 = h->dbg_t2;
+  }
+  TRY(launch_fused(h, a, check, s));
+  if (mode & ABFT_AUTOCORRECT) TRY(launch_correct(h, a, h->max_rounds, s));
+  return ABFT_OK;
+}
+
+abft_status abft_correct(abft_handle_t h, const double *x, double *y, int32_t max_rounds,
+                         const abft_inject_t *inj, void *stream) {
+  if (!h || !x || !y) return ABFT_EINVAL;
+  if (max_rounds <= 0) max_rounds = h->max_rounds;
+  if (max_rounds > h->max_rounds) return ABFT_EINVAL;
+  cudaStream_t s = (cudaStream_t)stream;
+  SpmvArgs a = make_args(h, x, y, nullptr);
+  TRY(prepare_inject(h, inj, s, &a.inj));
+  return launch_correct(h, a, max_rounds, s);
+}
+
+abft_status abft_flags(abft_handle_t h, int32_t round, const int32_t **flagged,
+                       const int32_t **n_flagged) {
+  if (!h || round < 0 || round > h->max_rounds) return ABFT_EINVAL;
+  if (flagged) *flagged = h->flags + (int64_t)round * h->nb;
+  if (n_flagged) *n_flagged = h->n_flags + round;
+  return ABFT_OK;
+}
+
+abft_status abft_beta(abft_handle_t h, const double **beta) {
+  if (!h || !beta) return ABFT_EINVAL;
+  *beta = h->beta;
+  return ABFT_OK;
+}
+
+abft_status abft_checksum_matrix(abft_handle_t h, const int32_t **c_row_ptr, const int32_t **c_col,
+                                 const double **c_val, const double **K, int64_t *nnz_c,
+                                 int64_t *nb) {
+  if (!h) return ABFT_EINVAL;
+  if (c_row_ptr) *c_row_ptr = h->c_rp;
+  if (c_col) *c_col = h->c_col;
+  if (c_val) *c_val = h->c_val;
+  if (K) *K = h->K;
+  if (nnz_c) *nnz_c = h->nnz_c;
+  if (nb) *nb = h->nb;
+  return ABFT_OK;
+}
+
+abft_status abft_debug_checksums(abft_handle_t h, const double **t1, const double **t2) {
+  if (!h) return ABFT_EINVAL;
+  if (t1) *t1 = h->dbg_t1;
+  if (t2) *t2 = h->dbg_t2;
+  return ABFT_OK;
+}
+
+abft_status abft_spmv_host(abft_handle_t h, const double *x_host, double *y_host,
+                           int32_t *n_flagged_host, uint32_t mode, void *stream) {
+  if (!h || !x_host || !y_host) return ABFT_EINVAL;
+  cudaStream_t s = (cudaStream_t)stream;
+  if (!h->hx) {
+    TRY(dalloc(h, &h->hx, (size_t)h->n));
+    TRY(dalloc(h, &h->hy, (size_t)h->n));
+  }
+  CK(cudaMemcpyAsync(h->hx, x_host, sizeof(double) * h->n, cudaMemcpyHostToDevice, s));
+  TRY(abft_spmv(h, h->hx, h->hy, nullptr, nullptr, mode, stream));
+  CK(cudaMemcpyAsync(y_host, h->hy, sizeof(double) * h->n, cudaMemcpyDeviceToHost, s));
+  if (n_flagged_host)
+    CK(cudaMemcpyAsync(n_flagged_host, h->n_flags, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  return ABFT_OK;
+}
+
+abft_status abft_memcpy(void *dst, const void *src, int64_t bytes, void *stream) {
+  if (bytes < 0 || (bytes > 0 && (!dst || !src))) return ABFT_EINVAL;
+  if (bytes == 0) return ABFT_OK;
+  cudaStream_t s = (cudaStream_t)stream;
+  CK(cudaMemcpyAsync(dst, src, (size_t)bytes, cudaMemcpyDefault, s));
+  CK(cudaStreamSynchronize(s));
+  return ABFT_OK;
+}
+
+}  // extern "C"
+
+#include "abft_pcg_api.inc"

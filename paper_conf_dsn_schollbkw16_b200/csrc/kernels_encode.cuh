@@ -1,0 +1,176 @@
+// kernels_encode.cuh -- checksum-matrix construction, once per matrix
+// (SIII-D, Fig. 3; structure P:128-130; values P:94, P:108;
+// bound constants P:156-160).  Not on the per-call path.
+//
+// One warp per row block k; lane l walks row k*b_s + l (columns ascending).
+// Each step takes the warp minimum of the lanes' current column heads: that
+// is the next column of C's row k (a b_s-way merge with de-duplication, so
+// C's columns come out ascending).  Lanes whose head equals it
+// contribute a_ij to the column sum, reduced over the b_s row slots by the
+// butterfly (PW over slots, absent where the row lacks the column).
+#pragma once
+#include "abft_device.cuh"
+
+namespace abft {
+
+struct EncodeArgs {
+  int64_t n;
+  int32_t bs;
+  int64_t nb;
+  const int32_t *__restrict__ rp;
+  const int32_t *__restrict__ ci;
+  const double *__restrict__ va;
+  int32_t *counts;   // [nb] (count pass)
+  int32_t *crp;      // [nb+1] (fill pass)
+  int32_t *ccol;
+  double *cval;
+  double *K;
+  int32_t *max_seg;  // max nnz over 32-row groups (device scalar, atomicMax)
+};
+
+template <bool FILL>
+__global__ void __launch_bounds__(256) k_encode(const EncodeArgs a) {
+  const int lane = threadIdx.x & 31;
+  const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  constexpr int kEnd = 0x7fffffff;
+  for (int64_t k = gw; k < a.nb; k += nw) {
+    const int64_t i = k * a.bs + lane;
+    const bool valid = lane < a.bs && i < a.n;
+    int32_t p = 0, e = 0;
+    if (valid) {
+      p = __ldg(a.rp + i);
+      e = __ldg(a.rp + i + 1);
+    }
+    int head = p < e ? __ldg(a.ci + p) : kEnd;
+    int32_t cnt = 0;
+    int32_t pos = FILL ? a.crp[k] : 0;
+    PwSeq csq;  // ||c_k||^2 over the ascending columns (lane 0)
+    while (true) {
+      const int mcol = warp_min_i(head);
+      if (mcol == kEnd) break;
+      if (FILL) {
+        const double v = (head == mcol) ? __ldg(a.va + p) : kAbsent;
+        const double c = bfly32(v);   // c_kj = PW over the b_s row slots
+        if (lane == 0) {
+          a.ccol[pos] = mcol;
+          a.cval[pos] = c;
+          csq.push(dmul(c, c));
+        }
+        ++pos;
+      }
+      ++cnt;
+      if (head == mcol) {
+        ++p;
+        head = p < e ? __ldg(a.ci + p) : kEnd;
+      }
+    }
+    if (!FILL) {
+      if (lane == 0) a.counts[k] = cnt;
+    } else {
+      // ||a_i||_2 = sqrt(PW(a_ij^2)) over the row (R6); S_k over the slots.
+      double rn = kAbsent;
+      if (valid) {
+        PwSeq rsq;
+        const int32_t b0 = __ldg(a.rp + i), e0 = __ldg(a.rp + i + 1);
+        for (int32_t q = b0; q < e0; ++q) {
+          const double v = __ldg(a.va + q);
+          rsq.push(dmul(v, v));
+        }
+        rn = e0 > b0 ? __dsqrt_rn(rsq.finish()) : 0.0;
+      }
+      const double S = bfly32(rn);
+      if (lane == 0) {
+        const double cn = cnt > 0 ? __dsqrt_rn(csq.finish()) : 0.0;
+        const double nk = (double)cnt;
+        const double mk = (double)(cnt + 2 * a.bs - 2);   // n_k + 2 b_s - 2
+        a.K[k] = dmul(dadd(dmul(mk, S), dmul(nk, cn)), 0x1p-53);  // eps_M = 2^-53
+      }
+    }
+  }
+  if (!FILL) {
+    // segment size of each 32-row group (selects the staging capacity)
+    const int64_t ng = (a.n + 31) / 32;
+    for (int64_t g = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; g < ng;
+         g += (int64_t)gridDim.x * blockDim.x) {
+      const int32_t s = __ldg(a.rp + min(a.n, g * 32 + 32)) - __ldg(a.rp + g * 32);
+      atomicMax(a.max_seg, s);
+    }
+  }
+}
+
+// Exclusive scan of counts[0..nb) into crp[0..nb], crp[nb] = total.
+// Three phases: per-CTA scan (1024 elements), scan of CTA totals (one CTA,
+// sequential chunks), add offsets.
+__global__ void __launch_bounds__(1024) k_scan_local(const int32_t *in, int32_t *out, int64_t n,
+                                                      int32_t *totals) {
+  __shared__ int32_t s_w[32];
+  const int64_t g = (int64_t)blockIdx.x * 1024 + threadIdx.x;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  int32_t v = g < n ? in[g] : 0;
+  int32_t inc = v;
+#pragma unroll
+  for (int m = 1; m < 32; m <<= 1) {
+    int32_t t = __shfl_up_sync(kFull, inc, m);
+    if (lane >= m) inc += t;
+  }
+  if (lane == 31) s_w[warp] = inc;
+  __syncthreads();
+  if (warp == 0) {
+    int32_t w = s_w[lane];
+#pragma unroll
+    for (int m = 1; m < 32; m <<= 1) {
+      int32_t t = __shfl_up_sync(kFull, w, m);
+      if (lane >= m) w += t;
+    }
+    s_w[lane] = w;
+  }
+  __syncthreads();
+  const int32_t off = warp > 0 ? s_w[warp - 1] : 0;
+  if (g < n) out[g] = off + inc - v;
+  if (threadIdx.x == 1023) totals[blockIdx.x] = off + inc;
+}
+
+__global__ void __launch_bounds__(1024) k_scan_totals(int32_t *totals, int64_t nt,
+                                                       int32_t *out_last) {
+  __shared__ int32_t s_w[32];
+  __shared__ int32_t s_carry;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  if (threadIdx.x == 0) s_carry = 0;
+  __syncthreads();
+  for (int64_t base = 0; base < nt; base += 1024) {
+    const int64_t g = base + threadIdx.x;
+    int32_t v = g < nt ? totals[g] : 0;
+    int32_t inc = v;
+#pragma unroll
+    for (int m = 1; m < 32; m <<= 1) {
+      int32_t t = __shfl_up_sync(kFull, inc, m);
+      if (lane >= m) inc += t;
+    }
+    if (lane == 31) s_w[warp] = inc;
+    __syncthreads();
+    if (warp == 0) {
+      int32_t w = s_w[lane];
+#pragma unroll
+      for (int m = 1; m < 32; m <<= 1) {
+        int32_t t = __shfl_up_sync(kFull, w, m);
+        if (lane >= m) w += t;
+      }
+      s_w[lane] = w;
+    }
+    __syncthreads();
+    const int32_t off = (warp > 0 ? s_w[warp - 1] : 0) + s_carry;
+    if (g < nt) totals[g] = off + inc - v;  // exclusive
+    __syncthreads();
+    if (threadIdx.x == 1023) s_carry = off + inc;
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) *out_last = s_carry;
+}
+
+__global__ void k_scan_add(int32_t *out, int64_t n, const int32_t *totals) {
+  const int64_t g = (int64_t)blockIdx.x * 1024 + threadIdx.x;
+  if (g < n) out[g] += totals[blockIdx.x];
+}
+
+}  // namespace abft

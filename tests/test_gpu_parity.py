@@ -1,0 +1,307 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle on
+the same seeded inputs and the same fault plans.
+
+Bar (BASELINE.json north_star): flagged-block sets and corrected-block
+indices bit-exact; corrected y within 1e-12 relative (we require -- and get --
+bit-exact y, t1, t2, beta, C and K because both sides follow the same PW
+order, R2); PCG residual histories within 1e-10 relative (again we
+assert bit-exact and keep the 1e-10 check as the stated bar).
+"""
+import numpy as np
+import pytest
+
+from paper_conf_dsn_schollbkw16_b200 import inputs as G
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def torch_cuda():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.fail("CUDA device required for -m gpu tests")
+    from paper_conf_dsn_schollbkw16_b200 import _build
+    _build.build()
+    return torch
+
+
+def bits(a):
+    return np.ascontiguousarray(a, dtype=np.float64).view(np.uint64)
+
+
+def assert_bits_equal(a, b, what):
+    a, b = bits(a), bits(b)
+    if not np.array_equal(a, b):
+        bad = np.nonzero(a != b)[0]
+        raise AssertionError(f"{what}: {bad.size} mismatches, first at {bad[:5].tolist()}: "
+                             f"{a.view(np.float64)[bad[:3]]} vs {b.view(np.float64)[bad[:3]]}")
+
+
+def oracle_inject(O, plan=None, rate=None):
+    if plan is not None:
+        return O.Inject.from_plan(plan)
+    if rate is not None:
+        return O.Inject.rate(**rate)
+    return None
+
+
+def gpu_inject(plan=None, rate=None):
+    from paper_conf_dsn_schollbkw16_b200 import Inject
+    if plan is not None:
+        return Inject.from_plan(plan)
+    if rate is not None:
+        return Inject.rate(**rate)
+    return None
+
+
+class Case:
+    """Encode A on both sides once; run protected SpMVs on both."""
+
+    def __init__(self, O, torch, A, bs=32, max_rounds=4):
+        from paper_conf_dsn_schollbkw16_b200 import encode
+        self.O, self.torch, self.A, self.bs = O, torch, A, bs
+        self.enc = O.encode(A, bs)
+        self.h = encode(A, bs, max_rounds)
+        self.max_rounds = max_rounds
+
+    def check_encoding(self):
+        rp, col, val, K = self.h.checksum_matrix()
+        assert np.array_equal(rp, self.enc.row_ptr)
+        assert np.array_equal(col, self.enc.col)
+        assert_bits_equal(val, self.enc.val, "C values")
+        assert_bits_equal(K, self.enc.K, "K")
+
+    def run(self, x, plan=None, rate=None, x_norm=False):
+        from paper_conf_dsn_schollbkw16_b200 import CHECK, DEBUG_CHECKSUMS
+        torch = self.torch
+        ref = self.O.abft_spmv(self.A, self.enc, x, oracle_inject(self.O, plan, rate),
+                               self.max_rounds)
+        xd = torch.from_numpy(x).cuda()
+        xn = torch.tensor([ref.beta], dtype=torch.float64, device="cuda") if x_norm else None
+        inj = gpu_inject(plan, rate)
+        y = self.h.spmv(xd, x_norm=xn, inject=inj, mode=CHECK | DEBUG_CHECKSUMS)
+        torch.cuda.synchronize()
+        assert_bits_equal(y.cpu().numpy(), ref.y_pre, "y (pre-correction)")
+        t1, t2 = self.h.debug_checksums()
+        # the oracle's t1/t2 hold the last round's values for recomputed blocks
+        keep = np.ones(self.enc.nb, dtype=bool)
+        for f in ref.flags[:-1]:
+            keep[f] = False
+        assert_bits_equal(t1[keep], ref.t1[keep], "t1")
+        assert_bits_equal(t2[keep], ref.t2[keep], "t2")
+        assert self.h.beta() == ref.beta
+        assert np.array_equal(self.h.flags(0), ref.flags[0]), (self.h.flags(0), ref.flags[0])
+        self.h.correct(xd, y, self.max_rounds, inject=inj)
+        torch.cuda.synchronize()
+        for r in range(1, self.max_rounds + 1):
+            assert np.array_equal(self.h.flags(r), ref.flags[r]), (r, self.h.flags(r), ref.flags[r])
+        assert_bits_equal(y.cpu().numpy(), ref.y, "y (corrected)")
+        return ref
+
+
+MATRICES = {
+    "lap2d_64": lambda: G.laplacian_2d_5pt(64),           # BASELINE configs[0]
+    "lap3d_16": lambda: G.laplacian_3d_7pt(16),
+    "lap3d_ragged": lambda: G.laplacian_3d_7pt(13, 11, 7),  # 1001 rows: ragged tail
+    "st27_11": lambda: G.stencil_3d_27pt(11),               # 27-pt, 1331 rows
+    "rand_empty": lambda: G.random_csr(1000, 0.01, 3, empty_rows=0.2),
+    "rand_dense": lambda: G.random_csr(300, 0.3, 4),        # rows > 32: warp fallback
+    "rmat11": lambda: G.rmat(11, 16, 5),                    # power law, long rows
+    "rmat11_natural": lambda: G.rmat(11, 8, 6, permute=False),  # empty blocks
+    "tiny1": lambda: G.CSR([0, 1], [0], [2.5]),
+    "tiny33": lambda: G.random_csr(33, 0.2, 9),
+    "all_empty": lambda: G.CSR(np.zeros(101, np.int32), np.zeros(0, np.int32), np.zeros(0)),
+}
+
+
+@pytest.mark.parametrize("name", sorted(MATRICES))
+def test_encode_and_spmv_error_free(O, torch_cuda, name):
+    A = MATRICES[name]()
+    c = Case(O, torch_cuda, A)
+    c.check_encoding()
+    for seed in (42, 43):
+        ref = c.run(G.uniform_vector(A.n, seed))
+        assert ref.flagged.size == 0
+
+
+@pytest.mark.parametrize("bs", [1, 2, 4, 8, 16])
+@pytest.mark.parametrize("name", ["lap3d_ragged", "rmat11", "rand_dense"])
+def test_block_sizes(O, torch_cuda, name, bs):
+    A = MATRICES[name]()
+    c = Case(O, torch_cuda, A, bs=bs)
+    c.check_encoding()
+    c.run(G.uniform_vector(A.n, 7))
+    plan = G.FaultPlan([0, 0, 0], [0, 1, 2], [A.n // 2, 1, c.enc.nb - 1], [1 << 62, 1 << 61, 1 << 60])
+    ref = c.run(G.uniform_vector(A.n, 8), plan=plan)
+    assert ref.flagged.size >= 1
+
+
+def test_single_bit_flips_config0(O, torch_cuda):
+    # BASELINE configs[0]: 64x64 5-pt, one seeded burst per run.
+    A = MATRICES["lap2d_64"]()
+    c = Case(O, torch_cuda, A)
+    x = G.uniform_vector(A.n, 42)
+    detected = 0
+    for seed in range(60):
+        plan = G.single_fault_plan(A.n, seed)
+        ref = c.run(x, plan=plan)
+        detected += ref.flagged.size
+    assert detected > 30
+
+
+@pytest.mark.parametrize("target", [0, 1, 2])
+def test_checksum_and_result_targets(O, torch_cuda, target):
+    A = MATRICES["st27_11"]()
+    c = Case(O, torch_cuda, A)
+    n_el = A.n if target == 0 else c.enc.nb
+    rng = np.random.default_rng(target)
+    idx = rng.choice(n_el, 12, replace=False)
+    plan = G.FaultPlan(np.zeros(12), np.full(12, target), idx,
+                       [G.burst_mask(int(s), 3) for s in rng.integers(40, 61, 12)])
+    ref = c.run(G.uniform_vector(A.n, 5), plan=plan)
+    assert ref.flagged.size > 0
+
+
+def test_faults_in_correction_rounds(O, torch_cuda):
+    # faults injected into the recomputation itself (rounds 1, 2): the block
+    # stays flagged for those rounds; round 4 exhausts -> uncorrected set.
+    A = MATRICES["lap3d_16"]()
+    c = Case(O, torch_cuda, A)
+    k = 17
+    i = k * 32 + 3
+    plan = G.FaultPlan([0, 1, 2, 1, 2, 3, 4], [0, 0, 2, 0, 1, 0, 0],
+                       [i, i, k, 100 * 32, k, i, i],
+                       [1 << 62, 1 << 62, 1 << 62, 1 << 62, 1 << 55, 1 << 62, 1 << 62])
+    ref = c.run(G.uniform_vector(A.n, 3), plan=plan)
+    assert ref.flags[4].tolist() == [k] and ref.status == -6
+
+
+@pytest.mark.parametrize("lam", [1e-6, 1e-4, 1e-2])
+def test_rate_mode(O, torch_cuda, lam):
+    # P:284 rate model through the device-side Philox injector.
+    A = MATRICES["lap3d_16"]()
+    c = Case(O, torch_cuda, A)
+    for call in range(3):
+        c.run(G.uniform_vector(A.n, 11 + call), rate=dict(seed=99, lam=lam, targets=0b111, call=call))
+
+
+def test_rate_mode_rmat_bs8(O, torch_cuda):
+    A = MATRICES["rmat11"]()
+    c = Case(O, torch_cuda, A, bs=8)
+    c.run(G.uniform_vector(A.n, 1), rate=dict(seed=5, lam=1e-3, targets=0b111, call=7))
+
+
+def test_x_norm_given(O, torch_cuda):
+    A = MATRICES["lap3d_16"]()
+    c = Case(O, torch_cuda, A)
+    plan = G.single_fault_plan(A.n, 3)
+    c.run(G.uniform_vector(A.n, 42), plan=plan, x_norm=True)
+
+
+def test_nan_and_zero(O, torch_cuda):
+    A = MATRICES["lap3d_ragged"]()
+    c = Case(O, torch_cuda, A)
+    c.run(np.zeros(A.n))
+    plan = G.FaultPlan([0], [0], [A.n - 1], [0x7FF8000000000000])
+    ref = c.run(G.uniform_vector(A.n, 1), plan=plan)
+    assert ref.flagged.tolist() == [(A.n - 1) // 32]
+
+
+def test_repeated_calls_reset_state(O, torch_cuda):
+    from paper_conf_dsn_schollbkw16_b200 import CHECK
+    A = MATRICES["lap2d_64"]()
+    c = Case(O, torch_cuda, A)
+    x = torch_cuda.from_numpy(G.uniform_vector(A.n, 1)).cuda()
+    inj = gpu_inject(plan=G.FaultPlan([0], [0], [5], [1 << 62]))
+    c.h.spmv(x, inject=inj, mode=CHECK)
+    assert c.h.flags(0).tolist() == [0]
+    for _ in range(5):
+        c.h.spmv(x, mode=CHECK)
+    assert c.h.flags(0).size == 0
+
+
+def test_spmv_host_entry(O, torch_cuda):
+    from paper_conf_dsn_schollbkw16_b200 import AUTOCORRECT, CHECK
+    A = MATRICES["st27_11"]()
+    c = Case(O, torch_cuda, A)
+    x = G.uniform_vector(A.n, 4)
+    y = np.empty(A.n)
+    nf = c.h.spmv_host(x, y, CHECK | AUTOCORRECT)
+    assert nf == 0
+    assert_bits_equal(y, O.spmv(A, x), "y via host entry")
+
+
+def test_nocheck_baseline(O, torch_cuda):
+    from paper_conf_dsn_schollbkw16_b200 import NOCHECK
+    A = MATRICES["rmat11"]()
+    c = Case(O, torch_cuda, A)
+    x = G.uniform_vector(A.n, 4)
+    y = c.h.spmv(torch_cuda.from_numpy(x).cuda(), mode=NOCHECK)
+    assert_bits_equal(y.cpu().numpy(), O.spmv(A, x), "plain y")
+
+
+# --------------------------------------------------------------------------
+# Full size: BASELINE configs[1] (3-D 7-pt 128^3), the bench workload, in the
+# launch configuration bench.py times.
+# --------------------------------------------------------------------------
+def test_full_size_config1(O, torch_cuda):
+    A = G.laplacian_3d_7pt(128)
+    c = Case(O, torch_cuda, A)
+    c.check_encoding()
+    ref = c.run(G.uniform_vector(A.n, 42))
+    assert ref.flagged.size == 0
+    rng = np.random.default_rng(0)
+    idx = rng.choice(A.n, 64, replace=False)
+    plan = G.FaultPlan(np.zeros(64), np.zeros(64), idx,
+                       [G.burst_mask(int(s), 4) for s in rng.integers(0, 64, 64)])
+    c.run(G.uniform_vector(A.n, 43), plan=plan)
+    c.run(G.uniform_vector(A.n, 44), rate=dict(seed=1, lam=1e-5, targets=0b111, call=3))
+
+
+# --------------------------------------------------------------------------
+# PCG
+# --------------------------------------------------------------------------
+def _pcg_case(O, torch, A, inj_kw=None, check=True, max_iter=0):
+    from paper_conf_dsn_schollbkw16_b200 import encode
+    enc = O.encode(A, 32)
+    xs = G.uniform_vector(A.n, 43)
+    b = O.spmv(A, xs)
+    x0 = G.uniform_vector(A.n, 44)
+    oinj = O.Inject.rate(**inj_kw) if inj_kw else None
+    ref = O.pcg(A, enc, b, x0, tol=1e-6, inj=oinj, check=check, max_iter=max_iter)
+    h = encode(A, 32)
+    bd = torch.from_numpy(b).cuda()
+    xd = torch.from_numpy(x0.copy()).cuda()
+    mi = max_iter if max_iter > 0 else 10 * A.n
+    hist = torch.zeros(mi + 1, dtype=torch.float64, device="cuda")
+    status, st = h.pcg(bd, xd, tol=1e-6, inject=gpu_inject(rate=inj_kw) if inj_kw else None,
+                       check=check, res_hist=hist, max_iter=max_iter)
+    torch.cuda.synchronize()
+    return ref, status, st, xd.cpu().numpy(), hist.cpu().numpy()[: st["iters"] + 1]
+
+
+@pytest.mark.parametrize("inj", [None, dict(seed=3, lam=1e-4, targets=0b111)])
+def test_pcg_parity(O, torch_cuda, inj):
+    A = G.laplacian_3d_7pt(16)
+    ref, status, st, x, hist = _pcg_case(O, torch_cuda, A, inj)
+    assert status == ref.status == 0
+    assert st["iters"] == ref.iters and st["spmv_calls"] == ref.spmv_calls
+    assert st["flagged_blocks"] == ref.flagged_blocks
+    assert st["recomputed_blocks"] == ref.recomputed_blocks
+    assert st["uncorrected_calls"] == ref.uncorrected_calls
+    assert np.max(np.abs(hist - ref.res_hist) / np.abs(ref.res_hist)) <= 1e-10
+    assert_bits_equal(hist, ref.res_hist, "residual history")
+    assert_bits_equal(x, ref.x, "solution")
+    if inj:
+        assert st["flagged_blocks"] > 0
+
+
+def test_pcg_unprotected_and_maxiter(O, torch_cuda):
+    A = G.laplacian_3d_7pt(12)
+    ref, status, st, x, hist = _pcg_case(O, torch_cuda, A, dict(seed=3, lam=1e-5), check=False)
+    assert status == ref.status and st["iters"] == ref.iters
+    assert_bits_equal(hist, ref.res_hist, "unprotected history")
+    ref, status, st, x, hist = _pcg_case(O, torch_cuda, A, None, max_iter=7)
+    assert status == ref.status == -5 and st["iters"] == ref.iters == 7
+    assert_bits_equal(hist, ref.res_hist, "truncated history")
+    assert_bits_equal(x, ref.x, "truncated solution")
