@@ -131,8 +131,11 @@ abft_status abft_correct(abft_handle_t h, const double *x, double *y, int32_t ma
 abft_status abft_flags(abft_handle_t h, int32_t round, const int32_t **flagged,
                        const int32_t **n_flagged);
 
-/* Device pointer to beta = ||x||_2 of the last abft_spmv (device double). */
-abft_status abft_beta(abft_handle_t h, const double **beta);
+/* Device pointer to beta = ||x||_2 of the last abft_spmv (device
+ * double).  The fused kernel completes beta only when a block needs it (a
+ * detection candidate) or x_norm was given; otherwise this call enqueues the
+ * PW reduction of the per-group partial sums on `stream` first. */
+abft_status abft_beta(abft_handle_t h, void *stream, const double **beta);
 
 /* Device pointers to the encoded checksum matrix and bound constants. */
 abft_status abft_checksum_matrix(abft_handle_t h, const int32_t **c_row_ptr,

@@ -60,7 +60,8 @@ class PcgStats(C.Structure):
 
 
 def lib_path() -> str:
-    return _build.LIB
+    # ABFT_LIB: alternative build of the same library (tuning experiments)
+    return os.environ.get("ABFT_LIB", _build.LIB)
 
 
 def lib():
@@ -82,7 +83,7 @@ def lib():
         L.abft_flags.restype = st
         L.abft_flags.argtypes = [P, i32, C.POINTER(P), C.POINTER(P)]
         L.abft_beta.restype = st
-        L.abft_beta.argtypes = [P, C.POINTER(P)]
+        L.abft_beta.argtypes = [P, P, C.POINTER(P)]
         L.abft_checksum_matrix.restype = st
         L.abft_checksum_matrix.argtypes = [P, C.POINTER(P), C.POINTER(P), C.POINTER(P),
                                            C.POINTER(P), C.POINTER(i64), C.POINTER(i64)]
@@ -257,7 +258,7 @@ class Handle:
 
     def beta(self, stream=None) -> float:
         b = C.c_void_p()
-        _check(lib().abft_beta(self._h, C.byref(b)), "abft_beta")
+        _check(lib().abft_beta(self._h, _stream(stream), C.byref(b)), "abft_beta")
         return float(self._d2h(b, 1, np.float64, stream)[0])
 
     def checksum_matrix(self, stream=None):

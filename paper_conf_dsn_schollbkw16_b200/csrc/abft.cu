@@ -3,6 +3,7 @@
 #include <algorithm>
 #include <cmath>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <vector>
 
@@ -29,14 +30,10 @@ abft_status cuda_fail(cudaError_t e, const char *where) {
     if (e_ != cudaSuccess) return cuda_fail(e_, #call);   \
   } while (0)
 
-#define CKM(call)                                                              \
-  do {                                                                         \
-    cudaError_t e_ = (call);                                                   \
-    if (e_ == cudaErrorMemoryAllocation) {                                     \
-      cudaGetLastError();                                                      \
-      return ABFT_ENOMEM;                                                      \
-    }                                                                          \
-    if (e_ != cudaSuccess) return cuda_fail(e_, #call);                        \
+#define TRY(expr)                         \
+  do {                                    \
+    abft_status s_ = (expr);              \
+    if (s_ != ABFT_OK) return s_;         \
   } while (0)
 
 void host_burst_table(uint64_t T[65]) {
@@ -48,39 +45,52 @@ void host_burst_table(uint64_t T[65]) {
   T[64] = (uint64_t)1 << 32;
 }
 
-int g_table_device = -1;  // device the burst table was uploaded to
+int g_init_device = -1;  // device the burst table / kernel attributes were set up on
+
+constexpr int kCapALimit = 1024;  // larger group segments take k_general
+constexpr int kCapCLimit = 1024;
+constexpr int kStageWarps = kLeanWarps;
+
+uint32_t align16(uint32_t v) { return (v + 15u) & ~15u; }
 
 }  // namespace
 
 struct abft_ctx {
-  int64_t n = 0, nnz = 0, nb = 0;
+  int64_t n = 0, nnz = 0, nb = 0, ngroups = 0;
   int32_t bs = 32, log2bs = 5, max_rounds = 4;
   const int32_t *rp = nullptr, *ci = nullptr;
   const double *va = nullptr;
   int32_t *c_rp = nullptr, *c_col = nullptr;
   double *c_val = nullptr, *K = nullptr;
   int64_t nnz_c = 0;
-  int32_t max_seg = 0;
-  int cap = 0;  // staging capacity in products per warp (0: fallback only)
-  int64_t ncta = 0;
+  int32_t max_seg_a = 0, max_seg_c = 0;
+  StageCfg stage{};
+  bool lean = false;        // k_lean usable (b_s = 32, 16-B aligned A)
+  size_t fused_smem = 0;
+  int fused_grid = 1;       // k_lean grid (persistent, one wave)
+  int32_t *glist = nullptr; // groups k_lean does not take
+  int64_t n_glist = 0;
+  int correct_grid = 1;
   // scratch
-  double *partials = nullptr;
+  double *gsum = nullptr;
   unsigned *done = nullptr;
   int32_t *n_cand = nullptr, *cand = nullptr;
   double *cand_s = nullptr;
   int32_t *flags = nullptr, *n_flags = nullptr;
   double *beta = nullptr;
+  int32_t *beta_valid = nullptr;
+  unsigned *gbar = nullptr;
   double *dbg_t1 = nullptr, *dbg_t2 = nullptr;
   uint64_t *inj_keys = nullptr, *inj_masks = nullptr;
   int64_t inj_cap = 0;
   double *hx = nullptr, *hy = nullptr;  // device staging for abft_spmv_host
   // PCG scratch
-  double *pcg = nullptr;   // r, z, p, q, d : 5 n
+  double *pcg = nullptr;  // r, z, p, q, d : 5 n
   double *pcg_part = nullptr;
   double *pcg_sc = nullptr;
-  int64_t *pcg_it = nullptr;
   int32_t *pcg_state = nullptr;
   int64_t pcg_n = 0;
+  int64_t ncta256 = 0;  // ceil(n / 256): PCG vector-kernel grid
   std::vector<void *> owned;
   int device = 0;
   int num_sms = 148;
@@ -102,19 +112,17 @@ abft_status dalloc(abft_ctx *h, T **p, size_t count) {
   return ABFT_OK;
 }
 
-#define TRY(expr)                         \
-  do {                                    \
-    abft_status s_ = (expr);              \
-    if (s_ != ABFT_OK) return s_;         \
-  } while (0)
+bool aligned16(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
 
 SpmvArgs make_args(const abft_ctx *h, const double *x, double *y, const double *x_norm) {
   SpmvArgs a;
   memset(&a, 0, sizeof a);
   a.n = h->n;
+  a.nnz = h->nnz;
   a.bs = h->bs;
   a.log2bs = h->log2bs;
   a.nb = h->nb;
+  a.ngroups = h->ngroups;
   a.rp = h->rp;
   a.ci = h->ci;
   a.va = h->va;
@@ -125,7 +133,7 @@ SpmvArgs make_args(const abft_ctx *h, const double *x, double *y, const double *
   a.x = x;
   a.y = y;
   a.x_norm = x_norm;
-  a.partials = h->partials;
+  a.gsum = h->gsum;
   a.done = h->done;
   a.n_cand = h->n_cand;
   a.cand = h->cand;
@@ -134,6 +142,9 @@ SpmvArgs make_args(const abft_ctx *h, const double *x, double *y, const double *
   a.n_flags = h->n_flags;
   a.max_rounds = h->max_rounds;
   a.beta = h->beta;
+  a.beta_valid = h->beta_valid;
+  a.gbar = h->gbar;
+  a.sc = h->stage;
   return a;
 }
 
@@ -187,18 +198,21 @@ abft_status prepare_inject(abft_ctx *h, const abft_inject_t *inj, cudaStream_t s
   return ABFT_OK;
 }
 
+int general_grid(const abft_ctx *h, int64_t groups) {
+  return (int)std::max<int64_t>(1, std::min<int64_t>((int64_t)h->num_sms * 8, (groups + 7) / 8));
+}
+
 template <bool CHECK, bool INJECT>
-abft_status launch_fused_t(const abft_ctx *h, const SpmvArgs &a, cudaStream_t s) {
-  const unsigned grid = (unsigned)h->ncta;
-  if (h->cap == 1024) {
-    const size_t smem = (size_t)kWarps * 1024 * sizeof(double);
-    k_fused<CHECK, INJECT, 1024><<<grid, kThreads, smem, s>>>(a);
-  } else if (h->cap == 256) {
-    const size_t smem = (size_t)kWarps * 256 * sizeof(double);
-    k_fused<CHECK, INJECT, 256><<<grid, kThreads, smem, s>>>(a);
-  } else {
-    return ABFT_EINVAL;
-  }
+abft_status launch_fused_t(const abft_ctx *h, SpmvArgs a, cudaStream_t s) {
+  // k_lean needs 16-B aligned operands for its bulk copies (x per call)
+  const bool lean = h->lean && aligned16(a.x);
+  const int64_t ngen = lean ? h->n_glist : h->ngroups;
+  a.glist = lean ? h->glist : nullptr;
+  a.n_glist = ngen;
+  const int ggrid = ngen > 0 ? general_grid(h, ngen) : 0;
+  a.ticket_total = (unsigned)((lean ? h->fused_grid : 0) + ggrid);
+  if (lean) k_lean<CHECK, INJECT><<<h->fused_grid, h->stage.warps * 32, h->fused_smem, s>>>(a);
+  if (ggrid) k_general<CHECK, INJECT><<<ggrid, 256, 0, s>>>(a);
   CK(cudaGetLastError());
   return ABFT_OK;
 }
@@ -209,30 +223,122 @@ abft_status launch_fused(const abft_ctx *h, const SpmvArgs &a, bool check, cudaS
   return inj ? launch_fused_t<false, true>(h, a, s) : launch_fused_t<false, false>(h, a, s);
 }
 
+// One launch for all correction rounds, as a programmatic dependent launch so
+// its launch latency overlaps the fused kernel (it waits on griddepcontrol).
 abft_status launch_correct(const abft_ctx *h, const SpmvArgs &a, int rounds, cudaStream_t s) {
-  const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>(h->num_sms * 4, (h->nb + 7) / 8));
-  for (int r = 1; r <= rounds; ++r) {
-    if (a.inj.mode != 0)
-      k_correct<true><<<grid, 256, 0, s>>>(a, r);
-    else
-      k_correct<false><<<grid, 256, 0, s>>>(a, r);
-    CK(cudaGetLastError());
+  cudaLaunchConfig_t cfg;
+  memset(&cfg, 0, sizeof cfg);
+  cfg.gridDim = dim3((unsigned)h->correct_grid);
+  cfg.blockDim = dim3(256);
+  cfg.dynamicSmemBytes = 0;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  if (a.inj.mode != 0)
+    CK(cudaLaunchKernelEx(&cfg, k_correct<true>, a, rounds));
+  else
+    CK(cudaLaunchKernelEx(&cfg, k_correct<false>, a, rounds));
+  return ABFT_OK;
+}
+
+size_t g_dyn_smem_limit = 0;  // opt-in shared memory per block minus static smem
+
+template <typename Kern>
+abft_status set_smem_attrs(Kern kern, int optin) {
+  cudaFuncAttributes fa;
+  CK(cudaFuncGetAttributes(&fa, kern));
+  const size_t lim = (size_t)optin - fa.sharedSizeBytes;
+  g_dyn_smem_limit = g_dyn_smem_limit ? std::min(g_dyn_smem_limit, lim) : lim;
+  CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)lim));
+  int carve = cudaSharedmemCarveoutMaxShared;
+  if (const char *e = getenv("ABFT_CARVEOUT")) carve = atoi(e);  // tuning sweeps only
+  CK(cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, carve));
+  return ABFT_OK;
+}
+
+abft_status init_device_once(int device) {
+  if (g_init_device == device) return ABFT_OK;
+  uint64_t T[65];
+  host_burst_table(T);
+  CK(cudaMemcpyToSymbol(c_burst_T, T, sizeof T));
+  int optin = 0;
+  CK(cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, device));
+  g_dyn_smem_limit = 0;
+  TRY(set_smem_attrs(k_lean<true, true>, optin));
+  TRY(set_smem_attrs(k_lean<true, false>, optin));
+  TRY(set_smem_attrs(k_lean<false, true>, optin));
+  TRY(set_smem_attrs(k_lean<false, false>, optin));
+  g_init_device = device;
+  return ABFT_OK;
+}
+
+// Stage layout and grid of k_lean, and the list of groups it does not take
+// (DESIGN.md "Kernels").  Synchronises the stream once (list length).
+abft_status plan_fused(abft_ctx *h, cudaStream_t s) {
+  StageCfg &c = h->stage;
+  memset(&c, 0, sizeof c);
+  h->correct_grid = h->num_sms;  // one CTA per SM: co-resident for the grid barrier
+  h->lean = h->bs == 32 && aligned16(h->rp) && aligned16(h->ci) && aligned16(h->va);
+  h->n_glist = h->ngroups;
+  if (!h->lean) return ABFT_OK;
+  c.capA = std::min(h->max_seg_a, kCapALimit);
+  c.capC = std::min(h->max_seg_c, kCapCLimit);
+  c.nstage = 2;  // double buffering (measured best)
+  int warps = kStageWarps;
+  // tuning overrides (benchmark sweeps only)
+  if (const char *e = getenv("ABFT_WARPS")) warps = std::max(1, std::min(kLeanWarps, atoi(e)));
+  for (;;) {
+    uint32_t o = 0;
+    c.off_rp = o;
+    o += 144;
+    c.off_x = o;
+    o += 256;
+    c.off_av = o;
+    o += align16((uint32_t)(c.capA + 2) * 8);
+    c.off_ac = o;
+    o += align16((uint32_t)(c.capA + 6) * 4);
+    c.off_cv = o;
+    o += align16((uint32_t)(c.capC + 2) * 8);
+    c.off_cc = o;
+    o += align16((uint32_t)(c.capC + 6) * 4);
+    c.off_cp = o;  // padded C products (one gap per 8)
+    o += align16((uint32_t)(c.capC + c.capC / 8 + 8) * 8);
+    c.stage_bytes = align16(o);
+    c.bar_bytes = 128;
+    h->fused_smem = c.bar_bytes + (size_t)warps * c.nstage * c.stage_bytes;
+    if (h->fused_smem <= g_dyn_smem_limit / 2 || (warps == 1 && h->fused_smem <= g_dyn_smem_limit))
+      break;
+    if (warps > 1) {
+      warps /= 2;
+    } else {
+      c.capA /= 2;
+      c.capC /= 2;
+    }
   }
-  return ABFT_OK;
-}
-
-template <typename K>
-abft_status set_smem(K kern, size_t bytes) {
-  CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes));
-  return ABFT_OK;
-}
-
-abft_status init_kernels() {
-  const size_t b1024 = (size_t)kWarps * 1024 * sizeof(double);
-  TRY(set_smem(k_fused<true, true, 1024>, b1024));
-  TRY(set_smem(k_fused<true, false, 1024>, b1024));
-  TRY(set_smem(k_fused<false, true, 1024>, b1024));
-  TRY(set_smem(k_fused<false, false, 1024>, b1024));
+  c.warps = warps;
+  int per_sm = 0;
+  CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_lean<true, false>, warps * 32,
+                                                   h->fused_smem));
+  per_sm = std::max(per_sm, 1);
+  if (const char *e = getenv("ABFT_CTAS_PER_SM")) per_sm = std::max(1, std::min(per_sm, atoi(e)));
+  const int64_t need = (h->ngroups + warps - 1) / warps;  // >= 1 group per warp
+  h->fused_grid = (int)std::max<int64_t>(1, std::min<int64_t>((int64_t)h->num_sms * per_sm, need));
+  // groups k_lean does not take
+  int32_t *count = nullptr;
+  TRY(dalloc(h, &h->glist, (size_t)h->ngroups));
+  TRY(dalloc(h, &count, 1));
+  CK(cudaMemsetAsync(count, 0, sizeof(int32_t), s));
+  SpmvArgs a = make_args(h, nullptr, nullptr, nullptr);
+  k_glist<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>((h->ngroups + 255) / 256, 4096)), 256,
+            0, s>>>(a, h->glist, count);
+  CK(cudaGetLastError());
+  int32_t cnt = 0;
+  CK(cudaMemcpyAsync(&cnt, count, sizeof cnt, cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  h->n_glist = cnt;
   return ABFT_OK;
 }
 
@@ -240,7 +346,7 @@ abft_status init_kernels() {
 
 extern "C" {
 
-const char *abft_version(void) { return "abft-b200 0.1 (sm_100a)"; }
+const char *abft_version(void) { return "abft-b200 0.2 (sm_100a)"; }
 
 const char *abft_last_cuda_error(void) { return g_cuda_err; }
 
@@ -279,42 +385,40 @@ abft_status abft_encode(const abft_csr_t *A, int32_t block_size, int32_t max_rou
   if (max_rounds == 0) max_rounds = 4;
   if (max_rounds < 1 || max_rounds > 16) return ABFT_EINVAL;
   cudaStream_t s = (cudaStream_t)stream;
+  int device = 0, num_sms = 0;
+  CK(cudaGetDevice(&device));
+  CK(cudaDeviceGetAttribute(&num_sms, cudaDevAttrMultiProcessorCount, device));
+  TRY(init_device_once(device));
+
   abft_ctx *h = new abft_ctx();
   auto fail = [&](abft_status st) {
     abft_destroy(h);
     return st;
   };
-  CK(cudaGetDevice(&h->device));
-  CK(cudaDeviceGetAttribute(&h->num_sms, cudaDevAttrMultiProcessorCount, h->device));
-  if (g_table_device != h->device) {
-    uint64_t T[65];
-    host_burst_table(T);
-    CK(cudaMemcpyToSymbol(c_burst_T, T, sizeof T));
-    abft_status st = init_kernels();
-    if (st != ABFT_OK) return fail(st);
-    g_table_device = h->device;
-  }
+  h->device = device;
+  h->num_sms = num_sms;
   h->n = A->n;
   h->nnz = A->nnz;
   h->bs = block_size;
   h->log2bs = 0;
   while ((1 << h->log2bs) < block_size) ++h->log2bs;
   h->nb = (h->n + block_size - 1) / block_size;
+  h->ngroups = (h->n + 31) / 32;
   h->max_rounds = max_rounds;
   h->rp = A->row_ptr;
   h->ci = A->col_idx;
   h->va = A->val;
-  h->ncta = (h->n + kThreads - 1) / kThreads;
+  h->ncta256 = (h->n + 255) / 256;
 
   abft_status st;
-  int32_t *counts = nullptr, *totals = nullptr, *max_seg = nullptr;
+  int32_t *counts = nullptr, *totals = nullptr, *stats = nullptr;
   const int64_t nscan = (h->nb + 1023) / 1024;
   if ((st = dalloc(h, &h->c_rp, (size_t)h->nb + 1)) || (st = dalloc(h, &counts, (size_t)h->nb)) ||
-      (st = dalloc(h, &totals, (size_t)nscan)) || (st = dalloc(h, &max_seg, 1)) ||
+      (st = dalloc(h, &totals, (size_t)nscan)) || (st = dalloc(h, &stats, 2)) ||
       (st = dalloc(h, &h->K, (size_t)h->nb)))
     return fail(st);
   cudaError_t e;
-  if ((e = cudaMemsetAsync(max_seg, 0, sizeof(int32_t), s)) != cudaSuccess)
+  if ((e = cudaMemsetAsync(stats, 0, 2 * sizeof(int32_t), s)) != cudaSuccess)
     return fail(cuda_fail(e, "memset"));
   EncodeArgs ea;
   memset(&ea, 0, sizeof ea);
@@ -327,41 +431,51 @@ abft_status abft_encode(const abft_csr_t *A, int32_t block_size, int32_t max_rou
   ea.counts = counts;
   ea.crp = h->c_rp;
   ea.K = h->K;
-  ea.max_seg = max_seg;
   const unsigned egrid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((h->nb + 7) / 8, 65535));
   k_encode<false><<<egrid, 256, 0, s>>>(ea);
   k_scan_local<<<(unsigned)nscan, 1024, 0, s>>>(counts, h->c_rp, h->nb, totals);
   k_scan_totals<<<1, 1024, 0, s>>>(totals, nscan, h->c_rp + h->nb);
   k_scan_add<<<(unsigned)nscan, 1024, 0, s>>>(h->c_rp, h->nb, totals);
+  k_group_stats<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>((h->ngroups + 255) / 256, 4096)),
+                  256, 0, s>>>(h->n, h->log2bs, h->nb, h->rp, h->c_rp, stats);
   if ((e = cudaGetLastError()) != cudaSuccess) return fail(cuda_fail(e, "encode count"));
-  int32_t host_tot[2];
+  int32_t host_tot[3];
   if ((e = cudaMemcpyAsync(&host_tot[0], h->c_rp + h->nb, 4, cudaMemcpyDeviceToHost, s)) ||
-      (e = cudaMemcpyAsync(&host_tot[1], max_seg, 4, cudaMemcpyDeviceToHost, s)) ||
+      (e = cudaMemcpyAsync(&host_tot[1], stats, 8, cudaMemcpyDeviceToHost, s)) ||
       (e = cudaStreamSynchronize(s)))
     return fail(cuda_fail(e, "encode sync"));
   h->nnz_c = host_tot[0];
-  h->max_seg = host_tot[1];
-  h->cap = h->max_seg <= 256 ? 256 : (h->max_seg <= 1024 ? 1024 : 1024);
-  if ((st = dalloc(h, &h->c_col, (size_t)h->nnz_c)) || (st = dalloc(h, &h->c_val, (size_t)h->nnz_c)))
+  h->max_seg_a = host_tot[1];
+  h->max_seg_c = host_tot[2];
+  // C arrays padded by 8 elements: bulk copies may round a segment up to 16 B
+  if ((st = dalloc(h, &h->c_col, (size_t)h->nnz_c + 8)) ||
+      (st = dalloc(h, &h->c_val, (size_t)h->nnz_c + 8)))
     return fail(st);
   ea.ccol = h->c_col;
   ea.cval = h->c_val;
   k_encode<true><<<egrid, 256, 0, s>>>(ea);
   if ((e = cudaGetLastError()) != cudaSuccess) return fail(cuda_fail(e, "encode fill"));
+  if ((e = cudaMemsetAsync(h->c_col + h->nnz_c, 0, 8 * sizeof(int32_t), s)) ||
+      (e = cudaMemsetAsync(h->c_val + h->nnz_c, 0, 8 * sizeof(double), s)))
+    return fail(cuda_fail(e, "pad"));
 
   // per-call scratch
-  if ((st = dalloc(h, &h->partials, (size_t)h->ncta)) || (st = dalloc(h, &h->done, 1)) ||
+  if ((st = dalloc(h, &h->gsum, (size_t)h->ngroups)) || (st = dalloc(h, &h->done, 1)) ||
       (st = dalloc(h, &h->n_cand, 1)) || (st = dalloc(h, &h->cand, (size_t)h->nb)) ||
       (st = dalloc(h, &h->cand_s, (size_t)h->nb)) ||
       (st = dalloc(h, &h->flags, (size_t)(h->max_rounds + 1) * h->nb)) ||
       (st = dalloc(h, &h->n_flags, (size_t)h->max_rounds + 1)) || (st = dalloc(h, &h->beta, 1)) ||
+      (st = dalloc(h, &h->beta_valid, 1)) || (st = dalloc(h, &h->gbar, 2)) ||
       (st = dalloc(h, &h->dbg_t1, (size_t)h->nb)) || (st = dalloc(h, &h->dbg_t2, (size_t)h->nb)))
     return fail(st);
   if ((e = cudaMemsetAsync(h->done, 0, sizeof(unsigned), s)) ||
       (e = cudaMemsetAsync(h->n_cand, 0, sizeof(int32_t), s)) ||
       (e = cudaMemsetAsync(h->n_flags, 0, sizeof(int32_t) * (h->max_rounds + 1), s)) ||
-      (e = cudaMemsetAsync(h->beta, 0, sizeof(double), s)) || (e = cudaStreamSynchronize(s)))
+      (e = cudaMemsetAsync(h->beta, 0, sizeof(double), s)) ||
+      (e = cudaMemsetAsync(h->beta_valid, 0, sizeof(int32_t), s)) ||
+      (e = cudaMemsetAsync(h->gbar, 0, 2 * sizeof(unsigned), s)) || (e = cudaStreamSynchronize(s)))
     return fail(cuda_fail(e, "scratch init"));
+  if ((st = plan_fused(h, s)) != ABFT_OK) return fail(st);
   *out = h;
   return ABFT_OK;
 }
@@ -402,8 +516,11 @@ abft_status abft_flags(abft_handle_t h, int32_t round, const int32_t **flagged,
   return ABFT_OK;
 }
 
-abft_status abft_beta(abft_handle_t h, const double **beta) {
+abft_status abft_beta(abft_handle_t h, void *stream, const double **beta) {
   if (!h || !beta) return ABFT_EINVAL;
+  SpmvArgs a = make_args(h, h->beta, h->beta + 1, nullptr);
+  k_beta<<<1, 1024, 0, (cudaStream_t)stream>>>(a);  // no-op when already valid
+  CK(cudaGetLastError());
   *beta = h->beta;
   return ABFT_OK;
 }

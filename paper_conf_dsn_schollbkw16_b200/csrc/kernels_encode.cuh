@@ -25,8 +25,28 @@ struct EncodeArgs {
   int32_t *ccol;
   double *cval;
   double *K;
-  int32_t *max_seg;  // max nnz over 32-row groups (device scalar, atomicMax)
 };
+
+// Largest A and C segment over the 32-row groups (sizes the staging buffers).
+__global__ void k_group_stats(int64_t n, int32_t log2bs, int64_t nb,
+                              const int32_t *__restrict__ rp, const int32_t *__restrict__ crp,
+                              int32_t *out /* [2]: max A seg, max C seg */) {
+  const int64_t ng = (n + 31) / 32;
+  int32_t ma = 0, mc = 0;
+  for (int64_t g = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; g < ng;
+       g += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t r0 = g * 32, r1 = min64(r0 + 32, n);
+    ma = max(ma, rp[r1] - rp[r0]);
+    const int64_t kb = r0 >> log2bs, ke = ((r1 - 1) >> log2bs) + 1;
+    mc = max(mc, crp[min64(ke, nb)] - crp[kb]);
+  }
+  ma = warp_max_i(ma);
+  mc = warp_max_i(mc);
+  if ((threadIdx.x & 31) == 0) {
+    atomicMax(out, ma);
+    atomicMax(out + 1, mc);
+  }
+}
 
 template <bool FILL>
 __global__ void __launch_bounds__(256) k_encode(const EncodeArgs a) {
@@ -86,15 +106,6 @@ __global__ void __launch_bounds__(256) k_encode(const EncodeArgs a) {
         const double mk = (double)(cnt + 2 * a.bs - 2);   // n_k + 2 b_s - 2
         a.K[k] = dmul(dadd(dmul(mk, S), dmul(nk, cn)), 0x1p-53);  // eps_M = 2^-53
       }
-    }
-  }
-  if (!FILL) {
-    // segment size of each 32-row group (selects the staging capacity)
-    const int64_t ng = (a.n + 31) / 32;
-    for (int64_t g = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; g < ng;
-         g += (int64_t)gridDim.x * blockDim.x) {
-      const int32_t s = __ldg(a.rp + min(a.n, g * 32 + 32)) - __ldg(a.rp + g * 32);
-      atomicMax(a.max_seg, s);
     }
   }
 }

@@ -1,40 +1,58 @@
 // kernels_spmv.cuh -- the hot path: fused multiply + detect (Fig. 1 steps
-// 1-4) with in-kernel finalize, and the correction relaunch (step 5,
-// P:76).  See DESIGN.md "Kernels".
+// 1-4) with an in-kernel finalize, and the correction pass (step 5,
+// P:76).  DESIGN.md "Kernels" has the derivations.
 //
-// Mapping.  One warp owns a group of 32 consecutive rows (= 32 / b_s row
-// blocks); a CTA of kWarps warps owns an aligned range of 32*kWarps rows.
-//  * A's segment of the group is streamed with coalesced, warp-strided loads
-//    (evict-first in L2), multiplied by the gathered x (read-only path, L2
-//    resident), and the products are staged in shared memory; lane l then
-//    reduces row r0+l with an in-register PW tree of P = 2^ceil(log2 maxlen)
-//    leaves read from shared memory.  Groups whose segment exceeds the
-//    staging capacity or whose longest row exceeds 32 fall back to one
-//    warp-cooperative reduction per row.
-//  * t2_k = PW over the b_s slots of y (xor butterfly over b_s lanes).
-//  * t1_k = c_k . x: C's row is streamed warp-strided; each 32-element chunk
-//    is reduced by a butterfly, chunks by an in-register tree (== PW).
-//  * s_k = t1_k - t2_k is compared with K_k * beta_local, beta_local = the
-//    norm of the CTA's aligned slice of x.  Monotone rounding makes
-//    beta_local <= beta exactly (R12'), so |s| <= K beta_local
-//    proves the block clean; only the rest become candidates.
-//  * The CTA's x^2 subtree goes to `partials`; the last CTA to finish (atomic
-//    ticket) completes beta = sqrt(PW(partials)), confirms the candidates
-//    against tau_k = K_k beta and writes the flagged list + count: steps 2-4
-//    finish without a second launch and without a host round trip.
+// Work unit: a GROUP of 32 consecutive rows (= 32/b_s row blocks).
+//
+// k_lean (b_s = 32, the paper's block size): a persistent grid; each warp owns
+// a contiguous range of groups and runs a software pipeline over them: one
+// lane issues TMA 1-D bulk copies (cp.async.bulk + mbarrier transaction
+// counts, L2 evict-first) of the next group's row pointers, x slice, A
+// segment (values + columns) and C segment into a shared-memory stage while
+// the warp computes the current group from the other stage.  Per group:
+//  * phase 1: every staged a_ij and c_kj becomes a product with the gathered
+//    x_j, in place (lane-strided, up to 16 x gathers in flight per lane: one
+//    L2 round trip per group);
+//  * y_i: lane l reduces row 32g+l from shared memory with an in-register PW
+//    tree of P = 2^ceil(log2 maxlen) leaves (rows > 32: the warp reduces it);
+//  * t2 = PW over the 32 slots of y (xor butterfly);
+//  * t1 = PW over C's row: butterfly per 32-chunk, tree over chunks (== PW);
+//  * s = t1 - t2 is compared with K_k * beta_g, beta_g = the norm of the
+//    group's own x slice -- an aligned node of the PW tree of ||x||^2, so
+//    beta_g <= beta exactly (monotone rounding, R12).  |s| <= K
+//    beta_g proves the block clean; anything else becomes a candidate;
+//  * the group's x^2 subtree goes to gsum[g].
+// k_general: every group k_lean cannot take (b_s < 32, the ragged last group,
+// segments beyond the staging capacity, unaligned operands) -- one warp per
+// group, operands read directly from global memory.
+// Both kernels share one completion ticket: the last CTA to finish confirms
+// the candidates against tau_k = K_k beta with beta = sqrt(PW(gsum)) --
+// computed only when a candidate exists (or taken from x_norm) -- and writes
+// the flagged-block list.
 #pragma once
 #include "abft_device.cuh"
+#include "bulk.cuh"
 
 namespace abft {
 
-constexpr int kWarps = 8;            // warps per CTA in the fused kernel
-constexpr int kThreads = kWarps * 32;
+constexpr int kLeanWarps = 4;  // warps per CTA of k_lean (<= 4)
+
+struct StageCfg {
+  int32_t capA, capC;     // staged capacity (elements) of a group's A / C segment
+  int32_t nstage;         // stages per warp (prefetch distance nstage-1)
+  int32_t warps;          // warps per CTA
+  uint32_t stage_bytes;   // bytes per stage
+  uint32_t bar_bytes;     // mbarrier region at the start of dynamic smem
+  uint32_t off_rp, off_x, off_av, off_ac, off_cv, off_cc, off_cp;
+};
 
 struct SpmvArgs {
   int64_t n;
+  int64_t nnz;
   int32_t bs;        // block size, power of two <= 32
   int32_t log2bs;
   int64_t nb;
+  int64_t ngroups;
   const int32_t *__restrict__ rp;
   const int32_t *__restrict__ ci;
   const double *__restrict__ va;
@@ -45,8 +63,9 @@ struct SpmvArgs {
   const double *__restrict__ x;
   double *__restrict__ y;
   const double *x_norm;   // nullable device scalar
-  double *partials;       // [gridDim.x]
-  unsigned *done;         // ticket counter (reset by the last CTA)
+  double *gsum;           // [ngroups] x^2 subtree of each group
+  unsigned *done;         // completion ticket (reset by the last CTA)
+  unsigned ticket_total;  // CTAs of all kernels of this call
   int32_t *n_cand;        // candidate count (reset by the last CTA)
   int32_t *cand;          // [nb]
   double *cand_s;         // [nb]
@@ -54,8 +73,13 @@ struct SpmvArgs {
   int32_t *n_flags;       // [max_rounds+1]
   int32_t max_rounds;
   double *beta;           // device scalar out
+  int32_t *beta_valid;    // 1 when *beta holds ||x|| of the last call
+  unsigned *gbar;         // [2] grid barrier of the correction pass
+  const int32_t *glist;   // k_general: groups to process (nullptr: all groups)
+  int64_t n_glist;
   double *dbg_t1, *dbg_t2;  // nullable
-  const int32_t *skip;      // nullable device flag: != 0 -> kernel is a no-op (PCG)
+  const int32_t *skip;      // nullable device flag: != 0 -> kernels are no-ops (PCG)
+  StageCfg sc;
   InjDev inj;
 };
 
@@ -63,26 +87,41 @@ __device__ __forceinline__ bool skip_call(const SpmvArgs &a) {
   return a.skip && *(volatile const int32_t *)a.skip != 0;
 }
 
-// PW over the products val[b+e] * x[col[b+e]], e in [0, cnt), cnt <= 256,
-// computed by the whole warp: lane l holds chunk elements u*32 + l; each
-// 32-chunk is reduced by the butterfly, the 8 chunk sums by a tree.
-__device__ __forceinline__ double warp_dot256(const double *__restrict__ val,
-                                              const int32_t *__restrict__ col, int64_t b,
-                                              int cnt, const double *__restrict__ x, int lane) {
+// ---------------------------------------------------------------------------
+// Operand accessors and PW reductions over them.
+// ---------------------------------------------------------------------------
+struct GlobalSrc {  // streamed (L1 no-allocate, L2 evict-first)
+  const double *v;
+  const int32_t *c;
+  __device__ __forceinline__ double val(int64_t e) const { return ld_stream(v + e); }
+  __device__ __forceinline__ int32_t col(int64_t e) const { return ld_stream(c + e); }
+};
+struct LdgSrc {  // L1-cached (correction pass)
+  const double *v;
+  const int32_t *c;
+  __device__ __forceinline__ double val(int64_t e) const { return __ldg(v + e); }
+  __device__ __forceinline__ int32_t col(int64_t e) const { return __ldg(c + e); }
+};
+
+// PW over products of elements [b, b+cnt), cnt <= 256, whole warp: lane l
+// holds elements u*32 + l; each 32-chunk by the butterfly, chunks by a tree.
+template <class Src>
+__device__ __forceinline__ double warp_dot256(const Src &s, int64_t b, int cnt,
+                                              const double *__restrict__ x, int lane) {
   double v[8];
   int c[8];
 #pragma unroll
   for (int u = 0; u < 8; ++u) {
-    int e = u * 32 + lane;
-    if (u * 32 < cnt && e < cnt) {
-      v[u] = ld_stream(val + b + e);
-      c[u] = ld_stream(col + b + e);
+    const int e = u * 32 + lane;
+    if (e < cnt) {
+      v[u] = s.val(b + e);
+      c[u] = s.col(b + e);
     }
   }
 #pragma unroll
   for (int u = 0; u < 8; ++u) {
-    int e = u * 32 + lane;
-    if (u * 32 < cnt && e < cnt) v[u] = dmul(v[u], ld_x(x + c[u])); else v[u] = kAbsent;
+    const int e = u * 32 + lane;
+    v[u] = e < cnt ? dmul(v[u], ld_x(x + c[u])) : kAbsent;
   }
 #pragma unroll
   for (int u = 0; u < 8; ++u)
@@ -91,321 +130,612 @@ __device__ __forceinline__ double warp_dot256(const double *__restrict__ val,
 }
 
 // PW over an arbitrary-length dot product, whole warp; +0.0 when empty.
-__device__ __noinline__ double warp_dot(const double *__restrict__ val,
-                                        const int32_t *__restrict__ col, int64_t b, int64_t n,
-                                        const double *__restrict__ x, int lane) {
+template <class Src>
+__device__ __forceinline__ double warp_dot(const Src &s, int64_t b, int64_t n,
+                                           const double *__restrict__ x, int lane) {
   if (n <= 0) return 0.0;
-  if (n <= 256) return warp_dot256(val, col, b, (int)n, x, lane);
+  if (n <= 256) return warp_dot256(s, b, (int)n, x, lane);
   PwSeq acc;  // binary counter over aligned 256-chunks (== PW)
   for (int64_t o = 0; o < n; o += 256)
-    acc.push(warp_dot256(val, col, b + o, (int)min64(256, n - o), x, lane));
+    acc.push(warp_dot256(s, b + o, (int)min64(256, n - o), x, lane));
   return acc.finish();
 }
 
-// Lane-private PW dot over a short row (len <= P) with direct loads.
-template <int P>
-__device__ __forceinline__ double lane_dot_direct(const double *__restrict__ val,
-                                                  const int32_t *__restrict__ col, int64_t b,
-                                                  int len, const double *__restrict__ x) {
+// Lane-private PW dot over a short row (len <= P <= 8).
+template <int P, class Src>
+__device__ __forceinline__ double lane_dot8(const Src &s, int64_t b, int len,
+                                            const double *__restrict__ x) {
   double v[P];
   int c[P];
 #pragma unroll
   for (int j = 0; j < P; ++j)
     if (j < len) {
-      v[j] = __ldg(val + b + j);
-      c[j] = __ldg(col + b + j);
+      v[j] = s.val(b + j);
+      c[j] = s.col(b + j);
     }
 #pragma unroll
   for (int j = 0; j < P; ++j) v[j] = j < len ? dmul(v[j], ld_x(x + c[j])) : kAbsent;
   return tree<P>(v);
 }
 
-__device__ __forceinline__ double lane_dot_direct_any(const double *__restrict__ val,
-                                                      const int32_t *__restrict__ col,
-                                                      int64_t b, int len, int maxlen,
-                                                      const double *__restrict__ x) {
-  if (maxlen <= 1) return lane_dot_direct<1>(val, col, b, len, x);
-  if (maxlen <= 2) return lane_dot_direct<2>(val, col, b, len, x);
-  if (maxlen <= 4) return lane_dot_direct<4>(val, col, b, len, x);
-  if (maxlen <= 8) return lane_dot_direct<8>(val, col, b, len, x);
-  if (maxlen <= 16) return lane_dot_direct<16>(val, col, b, len, x);
-  return lane_dot_direct<32>(val, col, b, len, x);
-}
-
-// Lane-private PW tree over staged products s[off .. off+len), P leaves.
-template <int P>
-__device__ __forceinline__ double lane_tree_smem(const double *s, int off, int len) {
-  double v[P];
-#pragma unroll
-  for (int j = 0; j < P; ++j) v[j] = j < len ? s[off + j] : kAbsent;
-  return tree<P>(v);
-}
-
-__device__ __forceinline__ double lane_tree_smem_any(const double *s, int off, int len,
-                                                     int maxlen) {
-  if (maxlen <= 1) return lane_tree_smem<1>(s, off, len);
-  if (maxlen <= 2) return lane_tree_smem<2>(s, off, len);
-  if (maxlen <= 4) return lane_tree_smem<4>(s, off, len);
-  if (maxlen <= 8) return lane_tree_smem<8>(s, off, len);
-  if (maxlen <= 16) return lane_tree_smem<16>(s, off, len);
-  return lane_tree_smem<32>(s, off, len);
-}
-
-// y for the 32 rows r0 .. r0+31 (lane l -> row r0+l); rows past n get len 0.
-// Returns y_i (+0.0 for empty rows); rs/len out for the caller.
-template <int CAP>
-__device__ __forceinline__ double group_rows(const SpmvArgs &a, int64_t r0, int lane,
-                                             double *s_prod, int &len_out) {
-  const int64_t n = a.n;
-  const int64_t i = r0 + lane;
-  const int32_t rs = ld_stream(a.rp + min(i, n));
-  int32_t rlast = 0;
-  if (lane == 31) rlast = ld_stream(a.rp + min(r0 + 32, n));
-  int32_t re = __shfl_down_sync(kFull, rs, 1);
-  if (lane == 31) re = rlast;
-  const int len = re - rs;
-  len_out = len;
-  const int32_t seg_b = __shfl_sync(kFull, rs, 0);
-  const int32_t seg_e = __shfl_sync(kFull, re, 31);
-  const int nseg = seg_e - seg_b;
-  const int maxlen = warp_max_i(len);
-  double yv;
-  if (nseg <= CAP && maxlen <= 32) {
-    // Stage the products of the whole segment (coalesced, warp-strided).
-    for (int base = 0; base < nseg; base += 256) {
-      double v[8];
-      int c[8];
-#pragma unroll
-      for (int u = 0; u < 8; ++u) {
-        int e = base + u * 32 + lane;
-        if (e < nseg) {
-          v[u] = ld_stream(a.va + seg_b + e);
-          c[u] = ld_stream(a.ci + seg_b + e);
-        }
-      }
-#pragma unroll
-      for (int u = 0; u < 8; ++u) {
-        int e = base + u * 32 + lane;
-        if (e < nseg) s_prod[e] = dmul(v[u], ld_x(a.x + c[u]));
-      }
-    }
-    __syncwarp();
-    yv = lane_tree_smem_any(s_prod, rs - seg_b, len, maxlen);
-    __syncwarp();
+// P = 16/32: aligned 8-leaf subtrees one at a time, then a tree over them.
+template <int P, class Src>
+__device__ __forceinline__ double lane_dot(const Src &s, int64_t b, int len,
+                                           const double *__restrict__ x) {
+  if constexpr (P <= 8) {
+    return lane_dot8<P>(s, b, len, x);
   } else {
-    // Fallback: one warp-cooperative PW reduction per row.
-    yv = 0.0;
-    for (int j = 0; j < 32; ++j) {
-      const int32_t rb = __shfl_sync(kFull, rs, j);
-      const int rl = __shfl_sync(kFull, len, j);
-      if (r0 + j >= n) break;
-      const double t = warp_dot(a.va, a.ci, rb, rl, a.x, lane);
-      if (lane == j) yv = t;
-    }
+    double q[P / 8];
+#pragma unroll
+    for (int t = 0; t < P / 8; ++t)
+      q[t] = (t * 8 < len) ? lane_dot8<8>(s, b + t * 8, len - t * 8, x) : kAbsent;
+    return tree<P / 8>(q);
   }
-  if (len == 0) yv = 0.0;  // PW of an empty row is +0.0 (R2)
-  return yv;
 }
 
-template <bool CHECK, bool INJECT, int CAP>
-__global__ void __launch_bounds__(kThreads) k_fused(const SpmvArgs a) {
-  extern __shared__ double s_dyn[];  // kWarps * CAP staged products
-  __shared__ double s_red[kThreads];
-  __shared__ int s_last;
-  __shared__ int s_nflag;
-  if (skip_call(a)) return;
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int64_t n = a.n;
-  const int64_t r0 = ((int64_t)blockIdx.x * kWarps + warp) * 32;
-  const int64_t i = r0 + lane;
-  const bool valid = i < n;
+template <class Src>
+__device__ __forceinline__ double lane_dot_any(const Src &s, int64_t b, int len, int maxlen,
+                                               const double *__restrict__ x) {
+  if (maxlen <= 1) return lane_dot<1>(s, b, len, x);
+  if (maxlen <= 2) return lane_dot<2>(s, b, len, x);
+  if (maxlen <= 4) return lane_dot<4>(s, b, len, x);
+  if (maxlen <= 8) return lane_dot<8>(s, b, len, x);
+  if (maxlen <= 16) return lane_dot<16>(s, b, len, x);
+  return lane_dot<32>(s, b, len, x);
+}
 
-  double s_syn = 0.0;
-  int64_t k = 0;
-  bool leader = false;
-  if (r0 < n) {
-    int len;
-    double yv = group_rows<CAP>(a, r0, lane, s_dyn + warp * CAP, len);
-    if (INJECT && valid) yv = apply_mask(yv, fault_mask(a.inj, 0, 0, i, 2 * (int64_t)len));
-    if (valid) a.y[i] = yv;
-    if (CHECK) {
-      // step 2: t2_k = w_k^T y_k over the b_s slots; absent past n.
-      double t2 = bfly(valid ? yv : kAbsent, a.bs);
-      // step 1: t1_k = c_k . x
-      const int bl = lane >> a.log2bs;        // block slot within the warp
-      k = (r0 >> a.log2bs) + bl;
-      leader = ((lane & (a.bs - 1)) == 0) && valid;
-      double t1;
-      int nk;
-      if (a.bs == 32) {
-        const int32_t cb = ld_stream(a.crp + k), ce = ld_stream(a.crp + k + 1);
-        nk = ce - cb;
-        t1 = warp_dot(a.cval, a.ccol, cb, nk, a.x, lane);
-      } else {
-        const int nblk = 32 >> a.log2bs;
-        int32_t cb = 0, ce = 0;
-        const int64_t kl = (r0 >> a.log2bs) + lane;
-        if (lane < nblk && kl < a.nb) {
-          cb = ld_stream(a.crp + kl);
-          ce = ld_stream(a.crp + kl + 1);
-        }
-        const int nkl = ce - cb;
-        const int maxnk = warp_max_i(nkl);
-        double t1l = 0.0;
-        if (maxnk <= 32) {
-          if (lane < nblk) t1l = lane_dot_direct_any(a.cval, a.ccol, cb, nkl, maxnk, a.x);
-          if (nkl == 0) t1l = 0.0;
-        } else {
-          for (int l = 0; l < nblk; ++l) {
-            const int32_t b = __shfl_sync(kFull, cb, l);
-            const int m = __shfl_sync(kFull, nkl, l);
-            const double t = warp_dot(a.cval, a.ccol, b, m, a.x, lane);
-            if (lane == l) t1l = t;
-          }
-        }
-        t1 = __shfl_sync(kFull, t1l, bl);
-        nk = __shfl_sync(kFull, nkl, bl);
-      }
-      if (INJECT && leader) {
-        t1 = apply_mask(t1, fault_mask(a.inj, 0, 1, k, 2 * (int64_t)nk));
-        const int64_t rows = min64(a.bs, n - (k << a.log2bs));
-        t2 = apply_mask(t2, fault_mask(a.inj, 0, 2, k, rows));
-      }
-      if (leader && a.dbg_t1) {
-        a.dbg_t1[k] = t1;
-        a.dbg_t2[k] = t2;
-      }
-      s_syn = dsub(t1, t2);  // step 3
-    }
-  }
-  if (!CHECK) return;
-
-  // beta: the CTA's aligned x^2 subtree (a node of the global PW tree).
-  {
-    double sq = kAbsent;
-    if (valid) {
-      const double xv = ld_x(a.x + i);
-      sq = dmul(xv, xv);
-    }
-    sq = bfly32(sq);
-    if (lane == 0) s_red[warp] = sq;
-  }
-  __syncthreads();
-  double cta;
-  {
-    double w[kWarps];
+// Lane-private PW over P staged products at a shared address (len <= P).
+template <int P>
+__device__ __forceinline__ double lane_sum_smem(uint32_t addr, int len) {
+  if constexpr (P <= 8) {
+    double v[P];
 #pragma unroll
-    for (int q = 0; q < kWarps; ++q) w[q] = s_red[q];
-    cta = tree<kWarps>(w);
+    for (int j = 0; j < P; ++j) v[j] = j < len ? lds_f64(addr + 8u * j) : kAbsent;
+    return tree<P>(v);
+  } else {
+    double q[P / 8];
+#pragma unroll
+    for (int t = 0; t < P / 8; ++t)
+      q[t] = (t * 8 < len) ? lane_sum_smem<8>(addr + 64u * t, len - 8 * t) : kAbsent;
+    return tree<P / 8>(q);
   }
-  // step 4 pre-filter: |s| <= K * beta_local  =>  |s| <= K * beta (exact).
-  if (leader) {
-    const double beta_loc = a.x_norm ? __ldg(a.x_norm) : __dsqrt_rn(cta);
-    const double tau_loc = dmul(__ldg(a.K + k), beta_loc);
-    if (!(fabs(s_syn) <= tau_loc)) {
-      const int pos = atomicAdd(a.n_cand, 1);
-      a.cand[pos] = (int32_t)k;
-      a.cand_s[pos] = s_syn;
-      __threadfence();
+}
+
+__device__ __forceinline__ double lane_sum_smem_any(uint32_t addr, int len, int maxlen) {
+  if (maxlen <= 1) return lane_sum_smem<1>(addr, len);
+  if (maxlen <= 2) return lane_sum_smem<2>(addr, len);
+  if (maxlen <= 4) return lane_sum_smem<4>(addr, len);
+  if (maxlen <= 8) return lane_sum_smem<8>(addr, len);
+  if (maxlen <= 16) return lane_sum_smem<16>(addr, len);
+  return lane_sum_smem<32>(addr, len);
+}
+
+// Whole-warp PW over n <= 1024 staged products at addr (+0.0 when empty).
+__device__ __forceinline__ double warp_sum_smem(uint32_t addr, int n, int lane) {
+  if (n <= 0) return 0.0;
+  double q[4];
+#pragma unroll
+  for (int t = 0; t < 4; ++t) {
+    if (t * 256 < n) {
+      double v[8];
+#pragma unroll
+      for (int u = 0; u < 8; ++u) {
+        const int e = t * 256 + u * 32 + lane;
+        v[u] = e < n ? lds_f64(addr + 8u * e) : kAbsent;
+      }
+#pragma unroll
+      for (int u = 0; u < 8; ++u)
+        if (t * 256 + u * 32 < n) v[u] = bfly32(v[u]);
+      q[t] = tree<8>(v);
+    } else {
+      q[t] = kAbsent;
     }
   }
-  __syncthreads();  // all candidate writes of this CTA precede its ticket
+  return tree<4>(q);
+}
+
+// ---------------------------------------------------------------------------
+// Candidate test (step 4 pre-filter) shared by both kernels.
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ void test_block(const SpmvArgs &a, int64_t k, double s, double gs) {
+  const double beta_g = a.x_norm ? __ldg(a.x_norm) : __dsqrt_rn(gs);
+  if (!(fabs(s) <= dmul(__ldg(a.K + k), beta_g))) {
+    const int pos = atomicAdd(a.n_cand, 1);
+    a.cand[pos] = (int32_t)k;
+    a.cand_s[pos] = s;
+    __threadfence();
+  }
+}
+
+// Last CTA of the call (ticket over a.ticket_total CTAs): beta, confirm the
+// candidates against tau_k = K_k beta, write round 0's flag list.
+__device__ __forceinline__ void finalize_ticket(const SpmvArgs &a, double *s_red, int *s_flag) {
+  __syncthreads();
   if (threadIdx.x == 0) {
-    a.partials[blockIdx.x] = cta;
     __threadfence();
     const unsigned t = atomicAdd(a.done, 1u);
-    s_last = (t == gridDim.x - 1);
-    s_nflag = 0;
+    s_flag[0] = (t == a.ticket_total - 1);
+    s_flag[1] = 0;
   }
   __syncthreads();
-  if (!s_last) return;
+  if (!s_flag[0]) return;
   __threadfence();
-
-  // ---- last CTA: beta = sqrt(PW over the CTA partials), confirm candidates.
-  const int ncta = gridDim.x;
-  int m = 1;
-  while (m * kThreads < ncta) m <<= 1;
-  {
-    PwSeq acc;
-    const int b = threadIdx.x * m;
-    for (int q = b; q < min(b + m, ncta); ++q) acc.push(__ldcg(a.partials + q));
-    s_red[threadIdx.x] = acc.finish();
-  }
-  __syncthreads();
-  for (int s = 1; s < kThreads; s <<= 1) {
-    if ((threadIdx.x & (2 * s - 1)) == 0) s_red[threadIdx.x] = dadd(s_red[threadIdx.x], s_red[threadIdx.x + s]);
-    __syncthreads();
-  }
-  const double beta = a.x_norm ? __ldcg(a.x_norm) : __dsqrt_rn(s_red[0]);
+  const int nthr = blockDim.x;
   const int nc = __ldcg(a.n_cand);
-  for (int c = threadIdx.x; c < nc; c += kThreads) {
-    const int32_t kk = __ldcg(a.cand + c);
-    const double s = __ldcg(a.cand_s + c);
-    const double tau = dmul(__ldg(a.K + kk), beta);   // tau_k = K_k * beta
-    if (!(fabs(s) <= tau)) a.flags[atomicAdd(&s_nflag, 1)] = kk;
+  double beta = 0.0;
+  if (a.x_norm) {
+    beta = __ldcg(a.x_norm);
+  } else if (nc > 0) {
+    // beta = sqrt(PW over the group subtrees) (R10)
+    int64_t m = 1;
+    while (m * nthr < a.ngroups) m <<= 1;
+    PwSeq acc;
+    const int64_t b = (int64_t)threadIdx.x * m;
+    for (int64_t q = b; q < min64(b + m, a.ngroups); ++q) acc.push(__ldcg(a.gsum + q));
+    s_red[threadIdx.x] = acc.finish();
+    __syncthreads();
+    for (int st = 1; st < nthr; st <<= 1) {
+      if ((threadIdx.x & (2 * st - 1)) == 0 && threadIdx.x + st < nthr)
+        s_red[threadIdx.x] = dadd(s_red[threadIdx.x], s_red[threadIdx.x + st]);
+      __syncthreads();
+    }
+    beta = __dsqrt_rn(s_red[0]);
+  }
+  for (int q = threadIdx.x; q < nc; q += nthr) {
+    const int32_t kk = __ldcg(a.cand + q);
+    const double s = __ldcg(a.cand_s + q);
+    const double tau = dmul(__ldg(a.K + kk), beta);  // tau_k = K_k * beta
+    if (!(fabs(s) <= tau)) a.flags[atomicAdd(&s_flag[1], 1)] = kk;
   }
   __syncthreads();
   if (threadIdx.x == 0) {
     *a.beta = beta;
-    a.n_flags[0] = s_nflag;
+    *a.beta_valid = (a.x_norm || nc > 0) ? 1 : 0;
+    a.n_flags[0] = s_flag[1];
     for (int r = 1; r <= a.max_rounds; ++r) a.n_flags[r] = 0;
     *a.n_cand = 0;
     *a.done = 0u;
   }
 }
 
-// Step 5: round `round` recomputes the rows of every block in
-// round (round-1)'s list, recomputes t1/t2 and re-checks; survivors form
-// round `round`'s list.  One warp per flagged block; grid-stride.
-template <bool INJECT>
-__global__ void __launch_bounds__(256) k_correct(const SpmvArgs a, int round) {
+// ---------------------------------------------------------------------------
+// General path: one group, operands from global memory (any b_s <= 32).
+// ---------------------------------------------------------------------------
+template <bool CHECK, bool INJECT>
+__device__ __forceinline__ void group_general(const SpmvArgs &a, int64_t g, int lane) {
+  const int64_t n = a.n;
+  const int64_t r0 = g * 32;
+  const int64_t i = r0 + lane;
+  const bool valid = i < n;
+  int32_t rs = 0, re = 0;
+  double xv = 0.0;
+  if (valid) {
+    rs = __ldg(a.rp + i);
+    re = __ldg(a.rp + i + 1);
+    xv = __ldg(a.x + i);
+  }
+  const GlobalSrc As{a.va, a.ci}, Cs{a.cval, a.ccol};
+  const int len = re - rs;
+  const int maxlen = warp_max_i(len);
+  double yv = 0.0;
+  if (maxlen <= 32) {
+    if (valid) yv = lane_dot_any(As, rs, len, maxlen, a.x);
+  } else {
+    for (int j = 0; j < 32; ++j) {
+      const int32_t rb = __shfl_sync(kFull, rs, j);
+      const int rl = __shfl_sync(kFull, len, j);
+      if (r0 + j >= n) break;
+      const double t = warp_dot(As, rb, rl, a.x, lane);
+      if (lane == j) yv = t;
+    }
+  }
+  if (len == 0) yv = 0.0;  // PW of an empty row is +0.0 (R2)
+  if (INJECT && valid) yv = apply_mask(yv, fault_mask(a.inj, 0, 0, i, 2 * (int64_t)len));
+  if (valid) a.y[i] = yv;
+  if (!CHECK) return;
+
+  // step 2: t2_k = w_k^T y_k over the b_s slots; absent past n.
+  double t2 = bfly(valid ? yv : kAbsent, a.bs);
+  // step 1: t1_k = c_k . x: the 32/b_s C rows of the group,
+  // lane-per-C-row when short, warp-cooperative otherwise.
+  const int bl = lane >> a.log2bs;
+  const int64_t k = (r0 >> a.log2bs) + bl;
+  const bool leader = ((lane & (a.bs - 1)) == 0) && valid;
+  const int nblk = 32 >> a.log2bs;
+  const int64_t kl = (r0 >> a.log2bs) + lane;
+  int32_t cb = 0, ce = 0;
+  if (lane < nblk && kl < a.nb) {
+    cb = __ldg(a.crp + kl);
+    ce = __ldg(a.crp + kl + 1);
+  }
+  const int nkl = ce - cb;
+  const int maxnk = warp_max_i(nkl);
+  double t1l = 0.0;
+  if (nblk > 1 && maxnk <= 32) {
+    if (lane < nblk) t1l = lane_dot_any(Cs, cb, nkl, maxnk, a.x);
+    if (nkl == 0) t1l = 0.0;
+  } else {
+    for (int l = 0; l < nblk; ++l) {
+      const int32_t b = __shfl_sync(kFull, cb, l);
+      const int m = __shfl_sync(kFull, nkl, l);
+      const double t = warp_dot(Cs, b, m, a.x, lane);
+      if (lane == l) t1l = t;
+    }
+  }
+  double t1 = __shfl_sync(kFull, t1l, bl);
+  const int nk = __shfl_sync(kFull, nkl, bl);
+  if (INJECT && leader) {
+    t1 = apply_mask(t1, fault_mask(a.inj, 0, 1, k, 2 * (int64_t)nk));
+    t2 = apply_mask(t2, fault_mask(a.inj, 0, 2, k, min64(a.bs, n - (k << a.log2bs))));
+  }
+  if (leader && a.dbg_t1) {
+    a.dbg_t1[k] = t1;
+    a.dbg_t2[k] = t2;
+  }
+  const double gs = bfly32(valid ? dmul(xv, xv) : kAbsent);  // the group's x^2 subtree
+  if (lane == 0) a.gsum[g] = gs;
+  if (leader) test_block(a, k, dsub(t1, t2), gs);  // steps 3-4
+}
+
+template <bool CHECK, bool INJECT>
+__global__ void __launch_bounds__(256) k_general(const SpmvArgs a) {
+  __shared__ double s_red[256];
+  __shared__ int s_flag[2];
   if (skip_call(a)) return;
-  const int32_t nprev = __ldcg(a.n_flags + round - 1);
-  if (nprev == 0) return;
   const int lane = threadIdx.x & 31;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
-  const int32_t *prev = a.flags + (int64_t)(round - 1) * a.nb;
-  int32_t *next = a.flags + (int64_t)round * a.nb;
+  for (int64_t q = gw; q < a.n_glist; q += nw) {
+    const int64_t g = a.glist ? (int64_t)__ldg(a.glist + q) : q;
+    group_general<CHECK, INJECT>(a, g, lane);
+  }
+  if (CHECK) finalize_ticket(a, s_red, s_flag);
+}
+
+// ---------------------------------------------------------------------------
+// Lean path: b_s = 32, full staged group, two stages per warp.  Shared memory
+// is addressed through pointers derived from the kernel's shared array (so
+// guarded accesses compile to predicated LDS/STS, not branches).
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ bool lean_eligible(const SpmvArgs &a, int64_t g, int32_t sa,
+                                              int32_t ea, int32_t sc, int32_t ec) {
+  return (g * 32 + 32) <= a.n && (ea - sa) <= a.sc.capA && (ec - sc) <= a.sc.capC;
+}
+
+// Padded slot of C product e: one gap every 8 doubles, so lane l can read its
+// 8 consecutive products e = 8l..8l+7 without bank conflicts.
+__device__ __forceinline__ int cpad(int e) { return e + (e >> 3); }
+
+template <bool CHECK, bool INJECT>
+__device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa, int32_t ea,
+                                        int32_t sc, int32_t ec, unsigned char *st, int lane) {
+  const StageCfg &c = a.sc;
+  const int64_t i = g * 32 + lane;
+  double *pv = reinterpret_cast<double *>(st + c.off_av) + (sa & 1);          // element sa + e
+  const int32_t *pc = reinterpret_cast<const int32_t *>(st + c.off_ac) + (sa & 3);
+  const double *cv = reinterpret_cast<const double *>(st + c.off_cv) + (sc & 1);  // sc + e
+  const int32_t *cc = reinterpret_cast<const int32_t *>(st + c.off_cc) + (sc & 3);
+  double *cp = reinterpret_cast<double *>(st + c.off_cp);  // C products, padded
+  const int nA = ea - sa;
+  const int nC = CHECK ? ec - sc : 0;
+  // phase 1: a_ij x_j (in place) and c_kj x_j (padded), one gather round
+#pragma unroll 1
+  for (int base = 0; base < max(nA, nC); base += 256) {
+    double va[8], vc[8];
+    int32_t ia[8], ic[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      const int e = base + u * 32 + lane;
+      const bool ka = e < nA, kc = CHECK && e < nC;
+      va[u] = ka ? pv[e] : 0.0;
+      ia[u] = ka ? pc[e] : 0;
+      vc[u] = kc ? cv[e] : 0.0;
+      ic[u] = kc ? cc[e] : 0;
+    }
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      const int e = base + u * 32 + lane;
+      if (e < nA) va[u] = dmul(va[u], ld_x(a.x + ia[u]));
+      if (CHECK && e < nC) vc[u] = dmul(vc[u], ld_x(a.x + ic[u]));
+    }
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      const int e = base + u * 32 + lane;
+      if (e < nA) pv[e] = va[u];
+      if (CHECK && e < nC) cp[cpad(e)] = vc[u];
+    }
+  }
+  __syncwarp();
+  // y_i = PW over the row's products (lane-private tree; PW is padding
+  // independent, so P = 8 serves every row of length <= 8)
+  const int32_t rs = reinterpret_cast<const int32_t *>(st + c.off_rp)[lane];
+  int32_t re = __shfl_down_sync(kFull, rs, 1);
+  if (lane == 31) re = ea;
+  const int len = re - rs;
+  const int maxlen = warp_max_i(len);
+  const double *row = pv + (rs - sa);
+  double yv;
+  if (maxlen <= 8) {
+    double v[8];
+#pragma unroll
+    for (int j = 0; j < 8; ++j) v[j] = j < len ? row[j] : kAbsent;
+    yv = tree<8>(v);
+  } else if (maxlen <= 32) {
+    yv = lane_sum_smem_any(smem_u32(row), len, maxlen);
+  } else {
+    yv = 0.0;
+    for (int j = 0; j < 32; ++j) {
+      const int32_t rb = __shfl_sync(kFull, rs, j);
+      const int rl = __shfl_sync(kFull, len, j);
+      const double t = warp_sum_smem(smem_u32(pv + (rb - sa)), rl, lane);
+      if (lane == j) yv = t;
+    }
+  }
+  if (len == 0) yv = 0.0;  // PW of an empty row is +0.0 (R2)
+  if (INJECT) yv = apply_mask(yv, fault_mask(a.inj, 0, 0, i, 2 * (int64_t)len));
+  a.y[i] = yv;
+  if (!CHECK) return;
+
+  double t2 = bfly32(yv);  // step 2: t2_k = w_k^T y_k
+  // step 1: t1_k = c_k . x.  Lane l owns products 8l..8l+7 of
+  // each aligned 256-chunk: an 8-leaf tree in registers, then the butterfly
+  // over lanes -- exactly the PW tree of the chunk; chunks by a 4-leaf tree.
+  double q[4];
+#pragma unroll
+  for (int t = 0; t < 4; ++t) {
+    if (t * 256 < nC) {
+      double v[8];
+#pragma unroll
+      for (int u = 0; u < 8; ++u) {
+        const int e = t * 256 + lane * 8 + u;
+        v[u] = e < nC ? cp[cpad(e)] : kAbsent;
+      }
+      q[t] = bfly32(tree<8>(v));
+    } else {
+      q[t] = kAbsent;
+    }
+  }
+  double t1 = nC > 0 ? tree<4>(q) : 0.0;
+  if (INJECT && lane == 0) {
+    t1 = apply_mask(t1, fault_mask(a.inj, 0, 1, g, 2 * (int64_t)nC));
+    t2 = apply_mask(t2, fault_mask(a.inj, 0, 2, g, 32));
+  }
+  if (lane == 0 && a.dbg_t1) {
+    a.dbg_t1[g] = t1;
+    a.dbg_t2[g] = t2;
+  }
+  const double xv = reinterpret_cast<const double *>(st + c.off_x)[lane];
+  const double gs = bfly32(dmul(xv, xv));  // the group's x^2 subtree
+  if (lane == 0) {
+    a.gsum[g] = gs;
+    test_block(a, g, dsub(t1, t2), gs);  // steps 3-4
+  }
+}
+
+// Group bounds from the per-warp window: lane l holds rp[32 (wb+l)] and
+// crp[wb+l] (b_s = 32; clamped to n / nb).
+struct Window {
+  int64_t wb;
+  int32_t rpw, crpw;
+  __device__ __forceinline__ void load(const SpmvArgs &a, int64_t base, int lane) {
+    wb = base;
+    rpw = ld_stream(a.rp + min64((base + lane) * 32, a.n));
+    crpw = ld_stream(a.crp + min64(base + lane, a.nb));
+  }
+  __device__ __forceinline__ void get(int64_t g, int32_t &sa, int32_t &ea, int32_t &sc,
+                                      int32_t &ec) const {
+    const int j = (int)(g - wb);
+    sa = __shfl_sync(kFull, rpw, j);
+    ea = __shfl_sync(kFull, rpw, j + 1);
+    sc = __shfl_sync(kFull, crpw, j);
+    ec = __shfl_sync(kFull, crpw, j + 1);
+  }
+};
+
+// Issue the bulk copies of group g into stage `st` (lane 0 only).
+__device__ __forceinline__ void issue_stage(const SpmvArgs &a, int64_t g, int32_t sa, int32_t ea,
+                                            int32_t sc, int32_t ec, unsigned char *st,
+                                            uint64_t *bar, uint64_t pol) {
+  const StageCfg &c = a.sc;
+  const int64_t r0 = g * 32;
+  const int64_t nnz2 = a.nnz & ~1ll, nnz4 = a.nnz & ~3ll;
+  const int64_t sa8 = sa & ~1, ea8 = min64((ea + 1) & ~1, nnz2);
+  const int64_t sa4 = sa & ~3, ea4 = min64((ea + 3) & ~3, nnz4);
+  const int64_t sc8 = sc & ~1, ec8 = (ec + 1) & ~1;  // C is padded: no clamp
+  const int64_t sc4 = sc & ~3, ec4 = (ec + 3) & ~3;
+  const uint32_t bav = ea8 > sa8 ? (uint32_t)(ea8 - sa8) * 8 : 0;
+  const uint32_t bac = ea4 > sa4 ? (uint32_t)(ea4 - sa4) * 4 : 0;
+  const uint32_t bcv = ec8 > sc8 ? (uint32_t)(ec8 - sc8) * 8 : 0;
+  const uint32_t bcc = ec4 > sc4 ? (uint32_t)(ec4 - sc4) * 4 : 0;
+  mbar_arrive_expect_tx(bar, 128 + 256 + bav + bac + bcv + bcc);
+  bulk_g2s(st + c.off_rp, a.rp + r0, 128, bar, pol);  // rp[r0 .. r0+31]; rp[r0+32] = ea
+  bulk_g2s(st + c.off_x, a.x + r0, 256, bar, pol);
+  if (bav) bulk_g2s(st + c.off_av, a.va + sa8, bav, bar, pol);
+  if (bac) bulk_g2s(st + c.off_ac, a.ci + sa4, bac, bar, pol);
+  if (bcv) bulk_g2s(st + c.off_cv, a.cval + sc8, bcv, bar, pol);
+  if (bcc) bulk_g2s(st + c.off_cc, a.ccol + sc4, bcc, bar, pol);
+}
+
+template <bool CHECK, bool INJECT>
+__global__ void __launch_bounds__(kLeanWarps * 32, 4) k_lean(const SpmvArgs a) {
+  extern __shared__ __align__(128) unsigned char smem[];
+  __shared__ double s_red[kLeanWarps * 32];
+  __shared__ int s_flag[2];
+  if (skip_call(a)) return;
+  const StageCfg &c = a.sc;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  uint64_t *bars = reinterpret_cast<uint64_t *>(smem) + warp * 2;
+  unsigned char *wst = smem + c.bar_bytes + (size_t)warp * 2 * c.stage_bytes;
+  if (lane == 0) {
+    mbar_init(bars, 1);
+    mbar_init(bars + 1, 1);
+    fence_mbar_init();
+  }
+  __syncwarp();
+  const uint64_t pol = policy_evict_first();
+  const int64_t tw = (int64_t)gridDim.x * c.warps;
+  const int64_t gw = (int64_t)blockIdx.x * c.warps + warp;
+  const int64_t g0 = gw * a.ngroups / tw, g1 = (gw + 1) * a.ngroups / tw;
+  if (g0 >= g1) {
+    if (CHECK) finalize_ticket(a, s_red, s_flag);
+    return;
+  }
+  Window win;
+  win.load(a, g0, lane);
+  int32_t sa, ea, sc, ec;  // bounds of the current group, carried from its prefetch
+  win.get(g0, sa, ea, sc, ec);
+  bool elig = lean_eligible(a, g0, sa, ea, sc, ec);
+  if (lane == 0 && elig) issue_stage(a, g0, sa, ea, sc, ec, wst, bars, pol);
+  uint32_t phase = 0;  // bit s = parity of stage s's next completion
+  for (int64_t g = g0; g < g1; ++g) {
+    const int s = (int)(g - g0) & 1;
+    int32_t nsa = 0, nea = 0, nsc = 0, nec = 0;
+    bool nelig = false;
+    if (g + 1 < g1) {  // prefetch g + 1 into the other stage
+      if (g + 2 > win.wb + 31) win.load(a, g, lane);
+      win.get(g + 1, nsa, nea, nsc, nec);
+      nelig = lean_eligible(a, g + 1, nsa, nea, nsc, nec);
+      if (lane == 0 && nelig)
+        issue_stage(a, g + 1, nsa, nea, nsc, nec, wst + (size_t)(s ^ 1) * c.stage_bytes,
+                    bars + (s ^ 1), pol);
+    }
+    if (elig) {
+      unsigned char *st = wst + (size_t)s * c.stage_bytes;
+      mbar_wait(bars + s, (phase >> s) & 1u);
+      phase ^= 1u << s;
+      if (ea > (a.nnz & ~3ll)) {  // A elements past the arrays' last 16-B boundary
+        const int64_t nnz2 = a.nnz & ~1ll, nnz4 = a.nnz & ~3ll;
+        const int64_t e = nnz4 + lane;
+        if (lane < 3 && e >= sa && e < ea)
+          reinterpret_cast<int32_t *>(st + c.off_ac)[e - (sa & ~3)] = __ldg(a.ci + e);
+        if (lane == 3 && nnz2 < a.nnz && nnz2 >= sa && nnz2 < ea)
+          reinterpret_cast<double *>(st + c.off_av)[nnz2 - (sa & ~1)] = __ldg(a.va + nnz2);
+        __syncwarp();
+      }
+      group32<CHECK, INJECT>(a, g, sa, ea, sc, ec, st, lane);
+      __syncwarp();
+      fence_proxy_async_smem();  // generic accesses of this stage precede its next bulk write
+    }
+    sa = nsa;
+    ea = nea;
+    sc = nsc;
+    ec = nec;
+    elig = nelig;
+  }
+  if (CHECK) finalize_ticket(a, s_red, s_flag);
+}
+
+// Encode-time helper: the groups k_lean does not take (appended, unordered).
+__global__ void k_glist(const SpmvArgs a, int32_t *glist, int32_t *count) {
+  for (int64_t g = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; g < a.ngroups;
+       g += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t sa = a.rp[min64(g * 32, a.n)], ea = a.rp[min64(g * 32 + 32, a.n)];
+    const int32_t sc = a.crp[min64(g, a.nb)], ec = a.crp[min64(g + 1, a.nb)];
+    if (!lean_eligible(a, g, sa, ea, sc, ec)) glist[atomicAdd(count, 1)] = (int32_t)g;
+  }
+}
+
+// beta on demand (abft_beta): PW over the group subtrees, one CTA.
+__global__ void __launch_bounds__(1024) k_beta(const SpmvArgs a) {
+  __shared__ double s_red[1024];
+  if (*(volatile int32_t *)a.beta_valid) return;
+  int64_t m = 1;
+  while (m * 1024 < a.ngroups) m <<= 1;
+  PwSeq acc;
+  const int64_t b = (int64_t)threadIdx.x * m;
+  for (int64_t q = b; q < min64(b + m, a.ngroups); ++q) acc.push(__ldcg(a.gsum + q));
+  s_red[threadIdx.x] = acc.finish();
+  __syncthreads();
+  for (int st = 1; st < 1024; st <<= 1) {
+    if ((threadIdx.x & (2 * st - 1)) == 0)
+      s_red[threadIdx.x] = dadd(s_red[threadIdx.x], s_red[threadIdx.x + st]);
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) {
+    *a.beta = __dsqrt_rn(s_red[0]);
+    *a.beta_valid = 1;
+  }
+}
+
+// Software grid barrier (all CTAs co-resident: grid <= SM count).
+// bar[0] = arrivals, bar[1] = generation.
+__device__ __forceinline__ void grid_sync(unsigned *bar) {
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    const unsigned gen = *(volatile unsigned *)(bar + 1);
+    __threadfence();
+    if (atomicAdd(bar, 1u) == gridDim.x - 1) {
+      *(volatile unsigned *)bar = 0u;
+      __threadfence();
+      atomicAdd(bar + 1, 1u);
+    } else {
+      while (*(volatile unsigned *)(bar + 1) == gen) __nanosleep(64);
+    }
+    __threadfence();
+  }
+  __syncthreads();
+}
+
+// Step 5, all rounds in one launch: round r recomputes the rows
+// of every block in round (r-1)'s list, recomputes t1/t2 and re-checks;
+// survivors form round r's list.  One warp per flagged block, grid-stride;
+// rounds separated by a grid barrier.  Launched as a programmatic dependent
+// launch: its launch latency overlaps the fused kernels.
+template <bool INJECT>
+__global__ void __launch_bounds__(256) k_correct(const SpmvArgs a, int rounds) {
+  asm volatile("griddepcontrol.wait;" ::: "memory");
+  if (skip_call(a)) return;
+  if (__ldcg(a.n_flags) == 0) return;
+  const int lane = threadIdx.x & 31;
+  const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
   const double beta = __ldcg(a.beta);
   const int64_t n = a.n;
-  for (int64_t q = gw; q < nprev; q += nw) {
-    const int64_t k = __ldcg(prev + q);
-    const int64_t i = (k << a.log2bs) + lane;
-    const bool valid = lane < a.bs && i < n;
-    int32_t rs = 0, len = 0;
-    if (valid) {
-      rs = __ldg(a.rp + i);
-      len = __ldg(a.rp + i + 1) - rs;
-    }
-    const int maxlen = warp_max_i(len);
-    double yv = 0.0;
-    if (maxlen <= 32) {
-      if (valid) yv = lane_dot_direct_any(a.va, a.ci, rs, len, maxlen, a.x);
-    } else {
-      for (int j = 0; j < a.bs; ++j) {
-        const int32_t rb = __shfl_sync(kFull, rs, j);
-        const int rl = __shfl_sync(kFull, len, j);
-        if ((k << a.log2bs) + j >= n) break;
-        const double t = warp_dot(a.va, a.ci, rb, rl, a.x, lane);
-        if (lane == j) yv = t;
+  const LdgSrc As{a.va, a.ci}, Cs{a.cval, a.ccol};
+  for (int round = 1; round <= rounds; ++round) {
+    const int32_t nprev = __ldcg(a.n_flags + round - 1);
+    if (nprev == 0) break;  // uniform: every CTA reads it after the barrier
+    const int32_t *prev = a.flags + (int64_t)(round - 1) * a.nb;
+    int32_t *next = a.flags + (int64_t)round * a.nb;
+    for (int64_t q = gw; q < nprev; q += nw) {
+      const int64_t k = __ldcg(prev + q);
+      const int64_t i = (k << a.log2bs) + lane;
+      const bool valid = lane < a.bs && i < n;
+      int32_t rs = 0, len = 0;
+      if (valid) {
+        rs = __ldg(a.rp + i);
+        len = __ldg(a.rp + i + 1) - rs;
+      }
+      const int maxlen = warp_max_i(len);
+      double yv = 0.0;
+      if (maxlen <= 32) {
+        if (valid) yv = lane_dot_any(As, rs, len, maxlen, a.x);
+      } else {
+        for (int j = 0; j < a.bs; ++j) {
+          const int32_t rb = __shfl_sync(kFull, rs, j);
+          const int rl = __shfl_sync(kFull, len, j);
+          if ((k << a.log2bs) + j >= n) break;
+          const double t = warp_dot(As, rb, rl, a.x, lane);
+          if (lane == j) yv = t;
+        }
+      }
+      if (len == 0) yv = 0.0;
+      if (INJECT && valid) yv = apply_mask(yv, fault_mask(a.inj, round, 0, i, 2 * (int64_t)len));
+      if (valid) a.y[i] = yv;
+      double t2 = bfly32(valid ? yv : kAbsent);
+      const int32_t cb = __ldg(a.crp + k), ce = __ldg(a.crp + k + 1);
+      double t1 = warp_dot(Cs, cb, ce - cb, a.x, lane);
+      if (lane == 0) {
+        if (INJECT) {
+          t1 = apply_mask(t1, fault_mask(a.inj, round, 1, k, 2 * (int64_t)(ce - cb)));
+          t2 = apply_mask(t2, fault_mask(a.inj, round, 2, k, min64(a.bs, n - (k << a.log2bs))));
+        }
+        const double s = dsub(t1, t2);
+        if (!(fabs(s) <= dmul(__ldg(a.K + k), beta)))
+          next[atomicAdd(a.n_flags + round, 1)] = (int32_t)k;
       }
     }
-    if (len == 0) yv = 0.0;
-    if (INJECT && valid) yv = apply_mask(yv, fault_mask(a.inj, round, 0, i, 2 * (int64_t)len));
-    if (valid) a.y[i] = yv;
-    double t2 = bfly32(valid ? yv : kAbsent);
-    const int32_t cb = __ldg(a.crp + k), ce = __ldg(a.crp + k + 1);
-    double t1 = warp_dot(a.cval, a.ccol, cb, ce - cb, a.x, lane);
-    if (lane == 0) {
-      if (INJECT) {
-        t1 = apply_mask(t1, fault_mask(a.inj, round, 1, k, 2 * (int64_t)(ce - cb)));
-        const int64_t rows = min64(a.bs, n - (k << a.log2bs));
-        t2 = apply_mask(t2, fault_mask(a.inj, round, 2, k, rows));
-      }
-      const double s = dsub(t1, t2);
-      if (!(fabs(s) <= dmul(__ldg(a.K + k), beta))) next[atomicAdd(a.n_flags + round, 1)] = (int32_t)k;
-    }
+    if (round < rounds) grid_sync(a.gbar);
   }
 }
 
