@@ -297,7 +297,7 @@ abft_status plan_fused(abft_ctx *h, cudaStream_t s) {
     c.off_x = o;
     o += 256;
     c.off_av = o;
-    o += align16((uint32_t)(c.capA + 2) * 8);
+    o += align16((uint32_t)(c.capA + 6) * 8);
     c.off_ac = o;
     o += align16((uint32_t)(c.capA + 6) * 4);
     c.off_cv = o;

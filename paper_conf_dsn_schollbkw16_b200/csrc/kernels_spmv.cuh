@@ -247,6 +247,20 @@ __device__ __forceinline__ void test_block(const SpmvArgs &a, int64_t k, double 
   }
 }
 
+// Same test with a cheaper exact lower bound of beta_g: gs rounded down to
+// float, square root rounded down -- beta_lo <= sqrt(gs) <= beta, so the
+// pre-filter stays exact (a passing block provably passes against tau_k).
+__device__ __forceinline__ void test_block_lo(const SpmvArgs &a, int64_t k, double s, double gs) {
+  const double beta_lo = a.x_norm ? __ldg(a.x_norm)
+                                  : (double)__fsqrt_rd(__double2float_rd(gs));
+  if (!(fabs(s) <= dmul(__ldg(a.K + k), beta_lo))) {
+    const int pos = atomicAdd(a.n_cand, 1);
+    a.cand[pos] = (int32_t)k;
+    a.cand_s[pos] = s;
+    __threadfence();
+  }
+}
+
 // Last CTA of the call (ticket over a.ticket_total CTAs): beta, confirm the
 // candidates against tau_k = K_k beta, write round 0's flag list.
 __device__ __forceinline__ void finalize_ticket(const SpmvArgs &a, double *s_red, int *s_flag) {
@@ -411,38 +425,73 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
                                         int32_t sc, int32_t ec, unsigned char *st, int lane) {
   const StageCfg &c = a.sc;
   const int64_t i = g * 32 + lane;
-  double *pv = reinterpret_cast<double *>(st + c.off_av) + (sa & 1);          // element sa + e
-  const int32_t *pc = reinterpret_cast<const int32_t *>(st + c.off_ac) + (sa & 3);
+  // A: values and columns staged on the same 4-element grid from sa & ~3, so
+  // slot s holds element (sa & ~3) + s in both arrays; slots [0, nS) were
+  // copied (gap slots hold real neighbouring entries -- valid columns).
+  double *av = reinterpret_cast<double *>(st + c.off_av);
+  const int32_t *ac = reinterpret_cast<const int32_t *>(st + c.off_ac);
+  double *pv = av + (sa & 3);  // product of element sa + e at pv[e]
   const double *cv = reinterpret_cast<const double *>(st + c.off_cv) + (sc & 1);  // sc + e
   const int32_t *cc = reinterpret_cast<const int32_t *>(st + c.off_cc) + (sc & 3);
   double *cp = reinterpret_cast<double *>(st + c.off_cp);  // C products, padded
-  const int nA = ea - sa;
+  const int nS = ((ea + 3) & ~3) - (sa & ~3);
   const int nC = CHECK ? ec - sc : 0;
-  // phase 1: a_ij x_j (in place) and c_kj x_j (padded), one gather round
+  // phase 1a: A products in place; lane l owns slots 4l + 128u .. +3
+  // (128-bit shared loads/stores), 8 gathers in flight per lane.
 #pragma unroll 1
-  for (int base = 0; base < max(nA, nC); base += 256) {
-    double va[8], vc[8];
-    int32_t ia[8], ic[8];
+  for (int base = 0; base < nS; base += 256) {
+    double2 v[4];
+    int4 ci[2];
 #pragma unroll
-    for (int u = 0; u < 8; ++u) {
-      const int e = base + u * 32 + lane;
-      const bool ka = e < nA, kc = CHECK && e < nC;
-      va[u] = ka ? pv[e] : 0.0;
-      ia[u] = ka ? pc[e] : 0;
-      vc[u] = kc ? cv[e] : 0.0;
-      ic[u] = kc ? cc[e] : 0;
+    for (int u = 0; u < 2; ++u) {
+      const int s0 = base + u * 128 + lane * 4;
+      if (s0 < nS) {
+        v[2 * u] = *reinterpret_cast<const double2 *>(av + s0);
+        v[2 * u + 1] = *reinterpret_cast<const double2 *>(av + s0 + 2);
+        ci[u] = *reinterpret_cast<const int4 *>(ac + s0);
+      }
     }
 #pragma unroll
-    for (int u = 0; u < 8; ++u) {
-      const int e = base + u * 32 + lane;
-      if (e < nA) va[u] = dmul(va[u], ld_x(a.x + ia[u]));
-      if (CHECK && e < nC) vc[u] = dmul(vc[u], ld_x(a.x + ic[u]));
+    for (int u = 0; u < 2; ++u) {
+      const int s0 = base + u * 128 + lane * 4;
+      if (s0 < nS) {
+        v[2 * u].x = dmul(v[2 * u].x, ld_x(a.x + ci[u].x));
+        v[2 * u].y = dmul(v[2 * u].y, ld_x(a.x + ci[u].y));
+        v[2 * u + 1].x = dmul(v[2 * u + 1].x, ld_x(a.x + ci[u].z));
+        v[2 * u + 1].y = dmul(v[2 * u + 1].y, ld_x(a.x + ci[u].w));
+      }
     }
 #pragma unroll
-    for (int u = 0; u < 8; ++u) {
-      const int e = base + u * 32 + lane;
-      if (e < nA) pv[e] = va[u];
-      if (CHECK && e < nC) cp[cpad(e)] = vc[u];
+    for (int u = 0; u < 2; ++u) {
+      const int s0 = base + u * 128 + lane * 4;
+      if (s0 < nS) {
+        *reinterpret_cast<double2 *>(av + s0) = v[2 * u];
+        *reinterpret_cast<double2 *>(av + s0 + 2) = v[2 * u + 1];
+      }
+    }
+  }
+  // phase 1b: C products into the padded layout (lane-strided, 8 gathers)
+  if (CHECK) {
+#pragma unroll 1
+    for (int base = 0; base < nC; base += 256) {
+      const double *cvl = cv + base + lane;
+      const int32_t *ccl = cc + base + lane;
+      double *cpl = cp + cpad(base + lane);  // cpad(e + 32u) = cpad(e) + 36u
+      const int rc = nC - base - lane;
+      double vc[8];
+      int32_t ic[8];
+#pragma unroll
+      for (int u = 0; u < 8; ++u)
+        if (u * 32 < rc) {
+          vc[u] = cvl[u * 32];
+          ic[u] = ccl[u * 32];
+        }
+#pragma unroll
+      for (int u = 0; u < 8; ++u)
+        if (u * 32 < rc) vc[u] = dmul(vc[u], ld_x(a.x + ic[u]));
+#pragma unroll
+      for (int u = 0; u < 8; ++u)
+        if (u * 32 < rc) cpl[u * 36] = vc[u];
     }
   }
   __syncwarp();
@@ -484,12 +533,11 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
 #pragma unroll
   for (int t = 0; t < 4; ++t) {
     if (t * 256 < nC) {
+      const double *cpl = cp + t * 288 + lane * 9;  // cpad(t*256 + 8 lane + u)
+      const int rc = nC - t * 256 - lane * 8;
       double v[8];
 #pragma unroll
-      for (int u = 0; u < 8; ++u) {
-        const int e = t * 256 + lane * 8 + u;
-        v[u] = e < nC ? cp[cpad(e)] : kAbsent;
-      }
+      for (int u = 0; u < 8; ++u) v[u] = u < rc ? cpl[u] : kAbsent;
       q[t] = bfly32(tree<8>(v));
     } else {
       q[t] = kAbsent;
@@ -508,7 +556,7 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
   const double gs = bfly32(dmul(xv, xv));  // the group's x^2 subtree
   if (lane == 0) {
     a.gsum[g] = gs;
-    test_block(a, g, dsub(t1, t2), gs);  // steps 3-4
+    test_block_lo(a, g, dsub(t1, t2), gs);  // steps 3-4
   }
 }
 
@@ -538,19 +586,18 @@ __device__ __forceinline__ void issue_stage(const SpmvArgs &a, int64_t g, int32_
                                             uint64_t *bar, uint64_t pol) {
   const StageCfg &c = a.sc;
   const int64_t r0 = g * 32;
-  const int64_t nnz2 = a.nnz & ~1ll, nnz4 = a.nnz & ~3ll;
-  const int64_t sa8 = sa & ~1, ea8 = min64((ea + 1) & ~1, nnz2);
-  const int64_t sa4 = sa & ~3, ea4 = min64((ea + 3) & ~3, nnz4);
+  const int64_t nnz4 = a.nnz & ~3ll;
+  const int64_t sa4 = sa & ~3, ea4 = min64((ea + 3) & ~3, nnz4);  // A: 4-element grid
   const int64_t sc8 = sc & ~1, ec8 = (ec + 1) & ~1;  // C is padded: no clamp
   const int64_t sc4 = sc & ~3, ec4 = (ec + 3) & ~3;
-  const uint32_t bav = ea8 > sa8 ? (uint32_t)(ea8 - sa8) * 8 : 0;
+  const uint32_t bav = ea4 > sa4 ? (uint32_t)(ea4 - sa4) * 8 : 0;
   const uint32_t bac = ea4 > sa4 ? (uint32_t)(ea4 - sa4) * 4 : 0;
   const uint32_t bcv = ec8 > sc8 ? (uint32_t)(ec8 - sc8) * 8 : 0;
   const uint32_t bcc = ec4 > sc4 ? (uint32_t)(ec4 - sc4) * 4 : 0;
   mbar_arrive_expect_tx(bar, 128 + 256 + bav + bac + bcv + bcc);
   bulk_g2s(st + c.off_rp, a.rp + r0, 128, bar, pol);  // rp[r0 .. r0+31]; rp[r0+32] = ea
   bulk_g2s(st + c.off_x, a.x + r0, 256, bar, pol);
-  if (bav) bulk_g2s(st + c.off_av, a.va + sa8, bav, bar, pol);
+  if (bav) bulk_g2s(st + c.off_av, a.va + sa4, bav, bar, pol);
   if (bac) bulk_g2s(st + c.off_ac, a.ci + sa4, bac, bar, pol);
   if (bcv) bulk_g2s(st + c.off_cv, a.cval + sc8, bcv, bar, pol);
   if (bcc) bulk_g2s(st + c.off_cc, a.ccol + sc4, bcc, bar, pol);
@@ -603,13 +650,14 @@ __global__ void __launch_bounds__(kLeanWarps * 32, 4) k_lean(const SpmvArgs a) {
       unsigned char *st = wst + (size_t)s * c.stage_bytes;
       mbar_wait(bars + s, (phase >> s) & 1u);
       phase ^= 1u << s;
-      if (ea > (a.nnz & ~3ll)) {  // A elements past the arrays' last 16-B boundary
-        const int64_t nnz2 = a.nnz & ~1ll, nnz4 = a.nnz & ~3ll;
-        const int64_t e = nnz4 + lane;
-        if (lane < 3 && e >= sa && e < ea)
-          reinterpret_cast<int32_t *>(st + c.off_ac)[e - (sa & ~3)] = __ldg(a.ci + e);
-        if (lane == 3 && nnz2 < a.nnz && nnz2 >= sa && nnz2 < ea)
-          reinterpret_cast<double *>(st + c.off_av)[nnz2 - (sa & ~1)] = __ldg(a.va + nnz2);
+      if (ea > (a.nnz & ~3ll)) {  // A slots past the arrays' last 4-element boundary
+        const int64_t nnz4 = a.nnz & ~3ll;
+        const int64_t e = nnz4 + lane;  // slots of elements nnz4 .. nnz4+3
+        if (lane < 4 && e >= (sa & ~3)) {
+          const bool real = e < a.nnz;
+          reinterpret_cast<int32_t *>(st + c.off_ac)[e - (sa & ~3)] = real ? __ldg(a.ci + e) : 0;
+          reinterpret_cast<double *>(st + c.off_av)[e - (sa & ~3)] = real ? __ldg(a.va + e) : 0.0;
+        }
         __syncwarp();
       }
       group32<CHECK, INJECT>(a, g, sa, ea, sc, ec, st, lane);
