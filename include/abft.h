@@ -104,10 +104,32 @@ enum {
  * so that tau_k = K_k * ||x||_2.  block_size: power of two in [1, 32]
  * (default 32 = the paper's choice); otherwise ABFT_ENOTSUP.
  * max_rounds: correction rounds for ABFT_AUTOCORRECT / abft_pcg (>= 1, <= 16;
- * 0 -> 4).  flags: reserved, pass 0.  Synchronises `stream` once.
+ * 0 -> 4).  flags: 0, or ABFT_ENCODE_C_CSR to stream C in the paper's plain
+ * CSR form (FP64 values, int32 columns) instead of the lossless compact form
+ * the encoder picks by default (values in the narrowest type that holds every
+ * c_kj exactly -- int8 / int16 / float / double -- and columns as uint16
+ * offsets from each row's first column, when every row spans < 65536
+ * columns).  Both give bit-identical results.
+ * Synchronises `stream` (sizes C, picks the format).
  * On success *out owns C, K and all scratch (device). */
+enum { ABFT_ENCODE_C_CSR = 1 };
 abft_status abft_encode(const abft_csr_t *A, int32_t block_size, int32_t max_rounds,
                         uint32_t flags, void *stream, abft_handle_t *out);
+
+/* Encoding facts (host struct): sizes, the checksum-matrix format the fused
+ * kernel streams and its byte count, and how the groups of 32 rows split
+ * between the staged fast path and the general path. */
+enum { ABFT_CFMT_CSR = 0, ABFT_CFMT_I8 = 1, ABFT_CFMT_I16 = 2, ABFT_CFMT_F32 = 3,
+       ABFT_CFMT_F64 = 4 };
+typedef struct {
+  int64_t n, nnz, nb, nnz_c;
+  int32_t block_size, c_format;
+  int64_t c_bytes;          /* bytes of C (+ row pointers, bases) streamed per call */
+  int64_t groups, general_groups;  /* 32-row groups; those on the general path */
+  int32_t lean;             /* staged (TMA) path available */
+  int32_t max_rounds;
+} abft_info_t;
+abft_status abft_info(abft_handle_t h, abft_info_t *info);
 
 /* Protected SpMV y = A x (steps 1-4), optionally with correction
  * (mode | ABFT_AUTOCORRECT, step 5).  x and y: device [n], must not alias.

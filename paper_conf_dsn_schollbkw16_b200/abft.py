@@ -25,8 +25,10 @@ SYMBOLS = [
     "abft_encode", "abft_spmv", "abft_correct", "abft_flags", "abft_beta",
     "abft_checksum_matrix", "abft_debug_checksums", "abft_spmv_host", "abft_pcg",
     "abft_destroy", "abft_memcpy", "abft_status_string", "abft_last_cuda_error",
-    "abft_burst_table", "abft_version",
+    "abft_burst_table", "abft_version", "abft_info",
 ]
+ENCODE_C_CSR = 1
+CFMT_NAMES = {0: "csr-f64", 1: "int8+u16", 2: "int16+u16", 3: "f32+u16", 4: "f64+u16"}
 
 
 class AbftError(RuntimeError):
@@ -48,6 +50,18 @@ class _Inj(C.Structure):
                 ("lambda_", C.c_double), ("targets", C.c_uint32), ("n_list", C.c_int64),
                 ("list_round", C.c_void_p), ("list_target", C.c_void_p),
                 ("list_index", C.c_void_p), ("list_mask", C.c_void_p)]
+
+
+class Info(C.Structure):
+    _fields_ = [("n", C.c_int64), ("nnz", C.c_int64), ("nb", C.c_int64), ("nnz_c", C.c_int64),
+                ("block_size", C.c_int32), ("c_format", C.c_int32), ("c_bytes", C.c_int64),
+                ("groups", C.c_int64), ("general_groups", C.c_int64), ("lean", C.c_int32),
+                ("max_rounds", C.c_int32)]
+
+    def as_dict(self):
+        d = {f: getattr(self, f) for f, _ in self._fields_}
+        d["c_format_name"] = CFMT_NAMES.get(self.c_format, "?")
+        return d
 
 
 class PcgStats(C.Structure):
@@ -102,6 +116,8 @@ def lib():
         L.abft_last_cuda_error.restype = C.c_char_p
         L.abft_burst_table.argtypes = [P]
         L.abft_version.restype = C.c_char_p
+        L.abft_info.restype = st
+        L.abft_info.argtypes = [P, C.POINTER(Info)]
         _LIB = L
     return _LIB
 
@@ -183,7 +199,8 @@ class Handle:
     """abft_handle_t: owns C, K and scratch; keeps A alive (the library
     re-reads it in correction and PCG)."""
 
-    def __init__(self, A: CsrDevice, block_size: int = 32, max_rounds: int = 4, stream=None):
+    def __init__(self, A: CsrDevice, block_size: int = 32, max_rounds: int = 4, stream=None,
+                 c_csr: bool = False):
         self.A = A
         self.n = A.n
         self.block_size = block_size
@@ -192,9 +209,15 @@ class Handle:
         csr = _Csr(A.n, A.nnz, A.row_ptr.data_ptr(), A.col.data_ptr() if A.nnz else 0,
                    A.val.data_ptr() if A.nnz else 0)
         h = C.c_void_p()
-        _check(lib().abft_encode(C.byref(csr), block_size, max_rounds, 0, _stream(stream),
-                                 C.byref(h)), "abft_encode")
+        _check(lib().abft_encode(C.byref(csr), block_size, max_rounds,
+                                 ENCODE_C_CSR if c_csr else 0, _stream(stream), C.byref(h)),
+               "abft_encode")
         self._h = h
+
+    def info(self) -> dict:
+        inf = Info()
+        _check(lib().abft_info(self._h, C.byref(inf)), "abft_info")
+        return inf.as_dict()
 
     def close(self):
         if getattr(self, "_h", None) and self._h.value:
@@ -292,8 +315,10 @@ class Handle:
         return status, st.as_dict()
 
 
-def encode(A, block_size: int = 32, max_rounds: int = 4, stream=None) -> Handle:
-    """Encode a CSR matrix (host `inputs.CSR` or a `CsrDevice`)."""
+def encode(A, block_size: int = 32, max_rounds: int = 4, stream=None,
+           c_csr: bool = False) -> Handle:
+    """Encode a CSR matrix (host `inputs.CSR` or a `CsrDevice`).  c_csr forces
+    the paper's plain CSR checksum matrix instead of the compact form."""
     if not isinstance(A, CsrDevice):
         A = CsrDevice.from_host(A)
-    return Handle(A, block_size, max_rounds, stream)
+    return Handle(A, block_size, max_rounds, stream, c_csr)

@@ -64,6 +64,12 @@ struct abft_ctx {
   double *c_val = nullptr, *K = nullptr;
   int64_t nnz_c = 0;
   int32_t max_seg_a = 0, max_seg_c = 0;
+  int cfmt = CF_CSR;         // format of C streamed by k_lean
+  void *cval_n = nullptr;    // compact C values
+  uint16_t *ccol16 = nullptr;
+  int32_t *cbase = nullptr;
+  int32_t *crp_c = nullptr;  // compact row starts (16-element aligned)
+  int64_t nnz_cpad = 0;      // compact slots incl. row padding
   StageCfg stage{};
   bool lean = false;        // k_lean usable (b_s = 32, 16-B aligned A)
   size_t fused_smem = 0;
@@ -129,6 +135,10 @@ SpmvArgs make_args(const abft_ctx *h, const double *x, double *y, const double *
   a.crp = h->c_rp;
   a.ccol = h->c_col;
   a.cval = h->c_val;
+  a.cval_n = h->cval_n;
+  a.ccol16 = h->ccol16;
+  a.cbase = h->cbase;
+  a.crp_c = h->crp_c;
   a.K = h->K;
   a.x = x;
   a.y = y;
@@ -203,6 +213,18 @@ int general_grid(const abft_ctx *h, int64_t groups) {
 }
 
 template <bool CHECK, bool INJECT>
+void launch_lean(const abft_ctx *h, const SpmvArgs &a, cudaStream_t s) {
+  const dim3 grid(h->fused_grid), block(h->stage.warps * 32);
+  switch (h->cfmt) {
+    case CF_I8: k_lean<CHECK, INJECT, CF_I8><<<grid, block, h->fused_smem, s>>>(a); break;
+    case CF_I16: k_lean<CHECK, INJECT, CF_I16><<<grid, block, h->fused_smem, s>>>(a); break;
+    case CF_F32: k_lean<CHECK, INJECT, CF_F32><<<grid, block, h->fused_smem, s>>>(a); break;
+    case CF_F64: k_lean<CHECK, INJECT, CF_F64><<<grid, block, h->fused_smem, s>>>(a); break;
+    default: k_lean<CHECK, INJECT, CF_CSR><<<grid, block, h->fused_smem, s>>>(a); break;
+  }
+}
+
+template <bool CHECK, bool INJECT>
 abft_status launch_fused_t(const abft_ctx *h, SpmvArgs a, cudaStream_t s) {
   // k_lean needs 16-B aligned operands for its bulk copies (x per call)
   const bool lean = h->lean && aligned16(a.x);
@@ -211,7 +233,7 @@ abft_status launch_fused_t(const abft_ctx *h, SpmvArgs a, cudaStream_t s) {
   a.n_glist = ngen;
   const int ggrid = ngen > 0 ? general_grid(h, ngen) : 0;
   a.ticket_total = (unsigned)((lean ? h->fused_grid : 0) + ggrid);
-  if (lean) k_lean<CHECK, INJECT><<<h->fused_grid, h->stage.warps * 32, h->fused_smem, s>>>(a);
+  if (lean) launch_lean<CHECK, INJECT>(h, a, s);
   if (ggrid) k_general<CHECK, INJECT><<<ggrid, 256, 0, s>>>(a);
   CK(cudaGetLastError());
   return ABFT_OK;
@@ -259,6 +281,24 @@ abft_status set_smem_attrs(Kern kern, int optin) {
   return ABFT_OK;
 }
 
+template <int CF>
+abft_status set_lean_attrs(int optin) {
+  TRY(set_smem_attrs(k_lean<true, true, CF>, optin));
+  TRY(set_smem_attrs(k_lean<true, false, CF>, optin));
+  TRY(set_smem_attrs(k_lean<false, true, CF>, optin));
+  TRY(set_smem_attrs(k_lean<false, false, CF>, optin));
+  return ABFT_OK;
+}
+
+int cf_size(int cf) {
+  switch (cf) {
+    case CF_I8: return 1;
+    case CF_I16: return 2;
+    case CF_F32: return 4;
+    default: return 8;
+  }
+}
+
 abft_status init_device_once(int device) {
   if (g_init_device == device) return ABFT_OK;
   uint64_t T[65];
@@ -267,11 +307,78 @@ abft_status init_device_once(int device) {
   int optin = 0;
   CK(cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, device));
   g_dyn_smem_limit = 0;
-  TRY(set_smem_attrs(k_lean<true, true>, optin));
-  TRY(set_smem_attrs(k_lean<true, false>, optin));
-  TRY(set_smem_attrs(k_lean<false, true>, optin));
-  TRY(set_smem_attrs(k_lean<false, false>, optin));
+  TRY(set_lean_attrs<CF_CSR>(optin));
+  TRY(set_lean_attrs<CF_I8>(optin));
+  TRY(set_lean_attrs<CF_I16>(optin));
+  TRY(set_lean_attrs<CF_F32>(optin));
+  TRY(set_lean_attrs<CF_F64>(optin));
   g_init_device = device;
+  return ABFT_OK;
+}
+
+// Lossless compact C: pick the narrowest exact value
+// type and uint16 column offsets when every row spans < 65536 columns.
+abft_status build_compact_c(abft_ctx *h, cudaStream_t s) {
+  if (h->nnz_c == 0) return ABFT_OK;
+  int32_t *dev = nullptr;
+  TRY(dalloc(h, &dev, 2));
+  TRY(dalloc(h, &h->cbase, (size_t)h->nb));
+  CK(cudaMemsetAsync(dev, 0, 2 * sizeof(int32_t), s));
+  const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((h->nb + 7) / 8, 65535));
+  k_cformat_scan<<<grid, 256, 0, s>>>(h->nb, h->c_rp, h->c_col, h->c_val, dev, dev + 1, h->cbase);
+  CK(cudaGetLastError());
+  int32_t hv[2];
+  CK(cudaMemcpyAsync(hv, dev, sizeof hv, cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  const int32_t props = hv[0], span = hv[1];
+  if (span >= 65536) return ABFT_OK;  // columns do not fit uint16 offsets: keep CSR
+  const int cf = !(props & 1) ? CF_I8 : !(props & 2) ? CF_I16 : !(props & 4) ? CF_F32 : CF_F64;
+  const size_t sz = (size_t)cf_size(cf);
+  // compact row starts: exclusive scan of the 16-element padded row lengths
+  int32_t *plen = nullptr, *totals = nullptr;
+  const int64_t nscan = (h->nb + 1023) / 1024;
+  TRY(dalloc(h, &plen, (size_t)h->nb));
+  TRY(dalloc(h, &totals, (size_t)nscan));
+  TRY(dalloc(h, &h->crp_c, (size_t)h->nb + 1));
+  k_cformat_padlen<<<grid, 256, 0, s>>>(h->nb, h->c_rp, plen);
+  k_scan_local<<<(unsigned)nscan, 1024, 0, s>>>(plen, h->crp_c, h->nb, totals);
+  k_scan_totals<<<1, 1024, 0, s>>>(totals, nscan, h->crp_c + h->nb);
+  k_scan_add<<<(unsigned)nscan, 1024, 0, s>>>(h->crp_c, h->nb, totals);
+  CK(cudaGetLastError());
+  int32_t npad = 0;
+  CK(cudaMemcpyAsync(&npad, h->crp_c + h->nb, sizeof npad, cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  h->nnz_cpad = npad;
+  char *cv = nullptr;
+  TRY(dalloc(h, &cv, (size_t)npad * sz + 64));
+  TRY(dalloc(h, &h->ccol16, (size_t)npad + 32));
+  CK(cudaMemsetAsync(cv, 0, (size_t)npad * sz + 64, s));
+  CK(cudaMemsetAsync(h->ccol16, 0, ((size_t)npad + 32) * 2, s));
+  switch (cf) {
+    case CF_I8:
+      k_cformat_fill<int8_t><<<grid, 256, 0, s>>>(h->nb, h->c_rp, h->crp_c, h->c_col, h->c_val,
+                                                  h->cbase, reinterpret_cast<int8_t *>(cv),
+                                                  h->ccol16);
+      break;
+    case CF_I16:
+      k_cformat_fill<int16_t><<<grid, 256, 0, s>>>(h->nb, h->c_rp, h->crp_c, h->c_col, h->c_val,
+                                                   h->cbase, reinterpret_cast<int16_t *>(cv),
+                                                   h->ccol16);
+      break;
+    case CF_F32:
+      k_cformat_fill<float><<<grid, 256, 0, s>>>(h->nb, h->c_rp, h->crp_c, h->c_col, h->c_val,
+                                                 h->cbase, reinterpret_cast<float *>(cv),
+                                                 h->ccol16);
+      break;
+    default:
+      k_cformat_fill<double><<<grid, 256, 0, s>>>(h->nb, h->c_rp, h->crp_c, h->c_col, h->c_val,
+                                                  h->cbase, reinterpret_cast<double *>(cv),
+                                                  h->ccol16);
+      break;
+  }
+  CK(cudaGetLastError());
+  h->cval_n = cv;
+  h->cfmt = cf;
   return ABFT_OK;
 }
 
@@ -301,11 +408,18 @@ abft_status plan_fused(abft_ctx *h, cudaStream_t s) {
     c.off_ac = o;
     o += align16((uint32_t)(c.capA + 6) * 4);
     c.off_cv = o;
-    o += align16((uint32_t)(c.capC + 2) * 8);
-    c.off_cc = o;
-    o += align16((uint32_t)(c.capC + 6) * 4);
-    c.off_cp = o;  // padded C products (one gap per 8)
-    o += align16((uint32_t)(c.capC + c.capC / 8 + 8) * 8);
+    if (h->cfmt == CF_CSR) {
+      o += align16((uint32_t)(c.capC + 2) * 8);
+      c.off_cc = o;
+      o += align16((uint32_t)(c.capC + 6) * 4);
+    } else {  // compact: a 16-element padded row of values and uint16 columns
+      const uint32_t cpad16 = ((uint32_t)c.capC + 15u) & ~15u;
+      o += align16(cpad16 * cf_size(h->cfmt));
+      c.off_cc = o;
+      o += align16(cpad16 * 2);
+    }
+    c.off_cp = o;  // padded C products (one gap per 8; CSR format only)
+    if (h->cfmt == CF_CSR) o += align16((uint32_t)(c.capC + c.capC / 8 + 8) * 8);
     c.stage_bytes = align16(o);
     c.bar_bytes = 128;
     h->fused_smem = c.bar_bytes + (size_t)warps * c.nstage * c.stage_bytes;
@@ -320,8 +434,8 @@ abft_status plan_fused(abft_ctx *h, cudaStream_t s) {
   }
   c.warps = warps;
   int per_sm = 0;
-  CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_lean<true, false>, warps * 32,
-                                                   h->fused_smem));
+  CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_lean<true, false, CF_CSR>,
+                                                   warps * 32, h->fused_smem));
   per_sm = std::max(per_sm, 1);
   if (const char *e = getenv("ABFT_CTAS_PER_SM")) per_sm = std::max(1, std::min(per_sm, atoi(e)));
   const int64_t need = (h->ngroups + warps - 1) / warps;  // >= 1 group per warp
@@ -375,7 +489,7 @@ abft_status abft_destroy(abft_handle_t h) {
 
 abft_status abft_encode(const abft_csr_t *A, int32_t block_size, int32_t max_rounds,
                         uint32_t flags, void *stream, abft_handle_t *out) {
-  if (!A || !out || flags != 0) return ABFT_EINVAL;
+  if (!A || !out || (flags & ~(uint32_t)ABFT_ENCODE_C_CSR)) return ABFT_EINVAL;
   *out = nullptr;
   if (A->n <= 0 || A->n >= ((int64_t)1 << 31) - 64 || A->nnz < 0 || A->nnz >= ((int64_t)1 << 31))
     return ABFT_EINVAL;
@@ -458,6 +572,7 @@ abft_status abft_encode(const abft_csr_t *A, int32_t block_size, int32_t max_rou
   if ((e = cudaMemsetAsync(h->c_col + h->nnz_c, 0, 8 * sizeof(int32_t), s)) ||
       (e = cudaMemsetAsync(h->c_val + h->nnz_c, 0, 8 * sizeof(double), s)))
     return fail(cuda_fail(e, "pad"));
+  if (!(flags & ABFT_ENCODE_C_CSR) && (st = build_compact_c(h, s)) != ABFT_OK) return fail(st);
 
   // per-call scratch
   if ((st = dalloc(h, &h->gsum, (size_t)h->ngroups)) || (st = dalloc(h, &h->done, 1)) ||
@@ -559,6 +674,26 @@ abft_status abft_spmv_host(abft_handle_t h, const double *x_host, double *y_host
   if (n_flagged_host)
     CK(cudaMemcpyAsync(n_flagged_host, h->n_flags, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
   CK(cudaStreamSynchronize(s));
+  return ABFT_OK;
+}
+
+abft_status abft_info(abft_handle_t h, abft_info_t *info) {
+  if (!h || !info) return ABFT_EINVAL;
+  memset(info, 0, sizeof *info);
+  info->n = h->n;
+  info->nnz = h->nnz;
+  info->nb = h->nb;
+  info->nnz_c = h->nnz_c;
+  info->block_size = h->bs;
+  info->c_format = h->cfmt;
+  if (h->cfmt == CF_CSR)
+    info->c_bytes = 12 * h->nnz_c + 4 * (h->nb + 1);
+  else
+    info->c_bytes = (int64_t)(cf_size(h->cfmt) + 2) * h->nnz_cpad + 8 * (h->nb + 1) + 4 * h->nb;
+  info->groups = h->ngroups;
+  info->general_groups = h->lean ? h->n_glist : h->ngroups;
+  info->lean = h->lean ? 1 : 0;
+  info->max_rounds = h->max_rounds;
   return ABFT_OK;
 }
 

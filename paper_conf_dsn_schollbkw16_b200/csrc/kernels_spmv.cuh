@@ -32,8 +32,15 @@
 #pragma once
 #include "abft_device.cuh"
 #include "bulk.cuh"
+#include "kernels_encode.cuh"
 
 namespace abft {
+
+// Element type of the compact checksum matrix for each format (CF_*).
+template <int CF> struct CType { using T = double; };
+template <> struct CType<CF_I8> { using T = int8_t; };
+template <> struct CType<CF_I16> { using T = int16_t; };
+template <> struct CType<CF_F32> { using T = float; };
 
 constexpr int kLeanWarps = 4;  // warps per CTA of k_lean (<= 4)
 
@@ -59,6 +66,10 @@ struct SpmvArgs {
   const int32_t *__restrict__ crp;
   const int32_t *__restrict__ ccol;
   const double *__restrict__ cval;
+  const void *__restrict__ cval_n;       // compact C values (CF != CF_CSR)
+  const uint16_t *__restrict__ ccol16;  // compact C columns: offset from cbase
+  const int32_t *__restrict__ cbase;    // first column of each C row
+  const int32_t *__restrict__ crp_c;    // compact row starts (16-element aligned)
   const double *__restrict__ K;
   const double *__restrict__ x;
   double *__restrict__ y;
@@ -416,13 +427,45 @@ __device__ __forceinline__ bool lean_eligible(const SpmvArgs &a, int64_t g, int3
   return (g * 32 + 32) <= a.n && (ea - sa) <= a.sc.capA && (ec - sc) <= a.sc.capC;
 }
 
+// Eight consecutive elements of a 16-B aligned staged compact-C row.
+__device__ __forceinline__ void load8(int8_t (&v)[8], const unsigned char *p) {
+  const uint2 w = *reinterpret_cast<const uint2 *>(p);
+#pragma unroll
+  for (int u = 0; u < 4; ++u) {
+    v[u] = (int8_t)((w.x >> (8 * u)) & 0xff);
+    v[u + 4] = (int8_t)((w.y >> (8 * u)) & 0xff);
+  }
+}
+__device__ __forceinline__ void load8(int16_t (&v)[8], const unsigned char *p) {
+  const uint4 w = *reinterpret_cast<const uint4 *>(p);
+  const uint32_t ww[4] = {w.x, w.y, w.z, w.w};
+#pragma unroll
+  for (int u = 0; u < 8; ++u) v[u] = (int16_t)((ww[u >> 1] >> (16 * (u & 1))) & 0xffff);
+}
+__device__ __forceinline__ void load8(float (&v)[8], const unsigned char *p) {
+  const float4 a = *reinterpret_cast<const float4 *>(p);
+  const float4 b = *reinterpret_cast<const float4 *>(p + 16);
+  v[0] = a.x; v[1] = a.y; v[2] = a.z; v[3] = a.w;
+  v[4] = b.x; v[5] = b.y; v[6] = b.z; v[7] = b.w;
+}
+__device__ __forceinline__ void load8(double (&v)[8], const unsigned char *p) {
+#pragma unroll
+  for (int u = 0; u < 4; ++u) {
+    const double2 d = *reinterpret_cast<const double2 *>(p + 16 * u);
+    v[2 * u] = d.x;
+    v[2 * u + 1] = d.y;
+  }
+}
+
 // Padded slot of C product e: one gap every 8 doubles, so lane l can read its
 // 8 consecutive products e = 8l..8l+7 without bank conflicts.
 __device__ __forceinline__ int cpad(int e) { return e + (e >> 3); }
 
-template <bool CHECK, bool INJECT>
+template <bool CHECK, bool INJECT, int CF>
 __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa, int32_t ea,
-                                        int32_t sc, int32_t ec, unsigned char *st, int lane) {
+                                        int32_t sc, int32_t ec, int32_t cb, unsigned char *st,
+                                        int lane) {
+  using CT = typename CType<CF>::T;
   const StageCfg &c = a.sc;
   const int64_t i = g * 32 + lane;
   // A: values and columns staged on the same 4-element grid from sa & ~3, so
@@ -471,7 +514,7 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
     }
   }
   // phase 1b: C products into the padded layout (lane-strided, 8 gathers)
-  if (CHECK) {
+  if (CHECK && CF == CF_CSR) {
 #pragma unroll 1
     for (int base = 0; base < nC; base += 256) {
       const double *cvl = cv + base + lane;
@@ -526,21 +569,52 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
   if (!CHECK) return;
 
   double t2 = bfly32(yv);  // step 2: t2_k = w_k^T y_k
-  // step 1: t1_k = c_k . x.  Lane l owns products 8l..8l+7 of
+  // step 1: t1_k = c_k . x.  Lane l owns elements 8l..8l+7 of
   // each aligned 256-chunk: an 8-leaf tree in registers, then the butterfly
   // over lanes -- exactly the PW tree of the chunk; chunks by a 4-leaf tree.
   double q[4];
+  if (CF != CF_CSR) {
+    // compact C: the row is staged 16-B aligned; values and uint16 column
+    // offsets come in with vector loads, products never touch shared memory
+    const unsigned char *cvb = st + c.off_cv;
+    const uint16_t *c16 = reinterpret_cast<const uint16_t *>(st + c.off_cc);
 #pragma unroll
-  for (int t = 0; t < 4; ++t) {
-    if (t * 256 < nC) {
-      const double *cpl = cp + t * 288 + lane * 9;  // cpad(t*256 + 8 lane + u)
-      const int rc = nC - t * 256 - lane * 8;
+    for (int t = 0; t < 4; ++t) {
       double v[8];
+      const int j0 = t * 256 + lane * 8;
+      if (t * 256 < nC) {
+        if (j0 < nC) {
+          CT cvv[8];
+          load8(cvv, cvb + (size_t)j0 * sizeof(CT));
+          const uint4 o4 = *reinterpret_cast<const uint4 *>(c16 + j0);
+          const uint32_t ow[4] = {o4.x, o4.y, o4.z, o4.w};
 #pragma unroll
-      for (int u = 0; u < 8; ++u) v[u] = u < rc ? cpl[u] : kAbsent;
-      q[t] = bfly32(tree<8>(v));
-    } else {
-      q[t] = kAbsent;
+          for (int u = 0; u < 8; ++u) {
+            const int32_t col = cb + (int32_t)((ow[u >> 1] >> (16 * (u & 1))) & 0xffffu);
+            v[u] = j0 + u < nC ? dmul((double)cvv[u], ld_x(a.x + col)) : kAbsent;
+          }
+        } else {
+#pragma unroll
+          for (int u = 0; u < 8; ++u) v[u] = kAbsent;
+        }
+        q[t] = bfly32(tree<8>(v));
+      } else {
+        q[t] = kAbsent;
+      }
+    }
+  } else {
+#pragma unroll
+    for (int t = 0; t < 4; ++t) {
+      if (t * 256 < nC) {
+        const double *cpl = cp + t * 288 + lane * 9;  // cpad(t*256 + 8 lane + u)
+        const int rc = nC - t * 256 - lane * 8;
+        double v[8];
+#pragma unroll
+        for (int u = 0; u < 8; ++u) v[u] = u < rc ? cpl[u] : kAbsent;
+        q[t] = bfly32(tree<8>(v));
+      } else {
+        q[t] = kAbsent;
+      }
     }
   }
   double t1 = nC > 0 ? tree<4>(q) : 0.0;
@@ -560,30 +634,61 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
   }
 }
 
-// Group bounds from the per-warp window: lane l holds rp[32 (wb+l)] and
-// crp[wb+l] (b_s = 32; clamped to n / nb).
+// Group bounds from the per-warp window: lane l holds rp[32 (wb+l)],
+// crp[wb+l] and (compact C) cbase[wb+l] (b_s = 32; clamped to n / nb).
+template <int CF>
 struct Window {
   int64_t wb;
-  int32_t rpw, crpw;
+  int32_t rpw, crpw, cbw, ccw;
   __device__ __forceinline__ void load(const SpmvArgs &a, int64_t base, int lane) {
     wb = base;
     rpw = ld_stream(a.rp + min64((base + lane) * 32, a.n));
     crpw = ld_stream(a.crp + min64(base + lane, a.nb));
+    if (CF != CF_CSR) {
+      cbw = ld_stream(a.cbase + min64(base + lane, a.nb - 1));
+      ccw = ld_stream(a.crp_c + min64(base + lane, a.nb));
+    }
   }
+  // sc/ec: C row bounds (CSR); cb: first column; cc: compact row start
   __device__ __forceinline__ void get(int64_t g, int32_t &sa, int32_t &ea, int32_t &sc,
-                                      int32_t &ec) const {
+                                      int32_t &ec, int32_t &cb, int32_t &cc) const {
     const int j = (int)(g - wb);
     sa = __shfl_sync(kFull, rpw, j);
     ea = __shfl_sync(kFull, rpw, j + 1);
     sc = __shfl_sync(kFull, crpw, j);
     ec = __shfl_sync(kFull, crpw, j + 1);
+    cb = CF != CF_CSR ? __shfl_sync(kFull, cbw, j) : 0;
+    cc = CF != CF_CSR ? __shfl_sync(kFull, ccw, j) : 0;
   }
 };
 
-// Issue the bulk copies of group g into stage `st` (lane 0 only).
+// Issue the bulk copies of group g into stage `st` (lane 0 only).  The
+// unprotected baseline (CHECK = false) does not touch C.
+template <bool CHECK, int CF>
 __device__ __forceinline__ void issue_stage(const SpmvArgs &a, int64_t g, int32_t sa, int32_t ea,
-                                            int32_t sc, int32_t ec, unsigned char *st,
+                                            int32_t sc, int32_t ec, int32_t cc, unsigned char *st,
                                             uint64_t *bar, uint64_t pol) {
+  if (CF != CF_CSR) {
+    using CT = typename CType<CF>::T;
+    const StageCfg &c = a.sc;
+    const int64_t r0 = g * 32;
+    const int64_t nnz4 = a.nnz & ~3ll;
+    const int64_t sa4 = sa & ~3, ea4 = min64((ea + 3) & ~3, nnz4);
+    const uint32_t bav = ea4 > sa4 ? (uint32_t)(ea4 - sa4) * 8 : 0;
+    const uint32_t bac = ea4 > sa4 ? (uint32_t)(ea4 - sa4) * 4 : 0;
+    const int32_t plen = (ec - sc + 15) & ~15;  // compact row: 16-element aligned
+    const int64_t v0 = (int64_t)cc * (int64_t)sizeof(CT), k0 = (int64_t)cc * 2;
+    const uint32_t bcv = CHECK ? (uint32_t)plen * (uint32_t)sizeof(CT) : 0;
+    const uint32_t bcc = CHECK ? (uint32_t)plen * 2 : 0;
+    mbar_arrive_expect_tx(bar, 128 + 256 + bav + bac + bcv + bcc);
+    bulk_g2s(st + c.off_rp, a.rp + r0, 128, bar, pol);
+    bulk_g2s(st + c.off_x, a.x + r0, 256, bar, pol);
+    if (bav) bulk_g2s(st + c.off_av, a.va + sa4, bav, bar, pol);
+    if (bac) bulk_g2s(st + c.off_ac, a.ci + sa4, bac, bar, pol);
+    if (bcv) bulk_g2s(st + c.off_cv, reinterpret_cast<const char *>(a.cval_n) + v0, bcv, bar, pol);
+    if (bcc) bulk_g2s(st + c.off_cc, reinterpret_cast<const char *>(a.ccol16) + k0, bcc, bar, pol);
+    return;
+  }
   const StageCfg &c = a.sc;
   const int64_t r0 = g * 32;
   const int64_t nnz4 = a.nnz & ~3ll;
@@ -592,8 +697,8 @@ __device__ __forceinline__ void issue_stage(const SpmvArgs &a, int64_t g, int32_
   const int64_t sc4 = sc & ~3, ec4 = (ec + 3) & ~3;
   const uint32_t bav = ea4 > sa4 ? (uint32_t)(ea4 - sa4) * 8 : 0;
   const uint32_t bac = ea4 > sa4 ? (uint32_t)(ea4 - sa4) * 4 : 0;
-  const uint32_t bcv = ec8 > sc8 ? (uint32_t)(ec8 - sc8) * 8 : 0;
-  const uint32_t bcc = ec4 > sc4 ? (uint32_t)(ec4 - sc4) * 4 : 0;
+  const uint32_t bcv = CHECK && ec8 > sc8 ? (uint32_t)(ec8 - sc8) * 8 : 0;
+  const uint32_t bcc = CHECK && ec4 > sc4 ? (uint32_t)(ec4 - sc4) * 4 : 0;
   mbar_arrive_expect_tx(bar, 128 + 256 + bav + bac + bcv + bcc);
   bulk_g2s(st + c.off_rp, a.rp + r0, 128, bar, pol);  // rp[r0 .. r0+31]; rp[r0+32] = ea
   bulk_g2s(st + c.off_x, a.x + r0, 256, bar, pol);
@@ -603,7 +708,7 @@ __device__ __forceinline__ void issue_stage(const SpmvArgs &a, int64_t g, int32_
   if (bcc) bulk_g2s(st + c.off_cc, a.ccol + sc4, bcc, bar, pol);
 }
 
-template <bool CHECK, bool INJECT>
+template <bool CHECK, bool INJECT, int CF>
 __global__ void __launch_bounds__(kLeanWarps * 32, 4) k_lean(const SpmvArgs a) {
   extern __shared__ __align__(128) unsigned char smem[];
   __shared__ double s_red[kLeanWarps * 32];
@@ -627,24 +732,24 @@ __global__ void __launch_bounds__(kLeanWarps * 32, 4) k_lean(const SpmvArgs a) {
     if (CHECK) finalize_ticket(a, s_red, s_flag);
     return;
   }
-  Window win;
+  Window<CF> win;
   win.load(a, g0, lane);
-  int32_t sa, ea, sc, ec;  // bounds of the current group, carried from its prefetch
-  win.get(g0, sa, ea, sc, ec);
+  int32_t sa, ea, sc, ec, cb, cc;  // bounds of the current group, carried from its prefetch
+  win.get(g0, sa, ea, sc, ec, cb, cc);
   bool elig = lean_eligible(a, g0, sa, ea, sc, ec);
-  if (lane == 0 && elig) issue_stage(a, g0, sa, ea, sc, ec, wst, bars, pol);
+  if (lane == 0 && elig) issue_stage<CHECK, CF>(a, g0, sa, ea, sc, ec, cc, wst, bars, pol);
   uint32_t phase = 0;  // bit s = parity of stage s's next completion
   for (int64_t g = g0; g < g1; ++g) {
     const int s = (int)(g - g0) & 1;
-    int32_t nsa = 0, nea = 0, nsc = 0, nec = 0;
+    int32_t nsa = 0, nea = 0, nsc = 0, nec = 0, ncb = 0, ncc = 0;
     bool nelig = false;
     if (g + 1 < g1) {  // prefetch g + 1 into the other stage
       if (g + 2 > win.wb + 31) win.load(a, g, lane);
-      win.get(g + 1, nsa, nea, nsc, nec);
+      win.get(g + 1, nsa, nea, nsc, nec, ncb, ncc);
       nelig = lean_eligible(a, g + 1, nsa, nea, nsc, nec);
       if (lane == 0 && nelig)
-        issue_stage(a, g + 1, nsa, nea, nsc, nec, wst + (size_t)(s ^ 1) * c.stage_bytes,
-                    bars + (s ^ 1), pol);
+        issue_stage<CHECK, CF>(a, g + 1, nsa, nea, nsc, nec, ncc,
+                               wst + (size_t)(s ^ 1) * c.stage_bytes, bars + (s ^ 1), pol);
     }
     if (elig) {
       unsigned char *st = wst + (size_t)s * c.stage_bytes;
@@ -660,7 +765,7 @@ __global__ void __launch_bounds__(kLeanWarps * 32, 4) k_lean(const SpmvArgs a) {
         }
         __syncwarp();
       }
-      group32<CHECK, INJECT>(a, g, sa, ea, sc, ec, st, lane);
+      group32<CHECK, INJECT, CF>(a, g, sa, ea, sc, ec, cb, st, lane);
       __syncwarp();
       fence_proxy_async_smem();  // generic accesses of this stage precede its next bulk write
     }
@@ -668,6 +773,8 @@ __global__ void __launch_bounds__(kLeanWarps * 32, 4) k_lean(const SpmvArgs a) {
     ea = nea;
     sc = nsc;
     ec = nec;
+    cb = ncb;
+    cc = ncc;
     elig = nelig;
   }
   if (CHECK) finalize_ticket(a, s_red, s_flag);

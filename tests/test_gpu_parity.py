@@ -57,11 +57,11 @@ def gpu_inject(plan=None, rate=None):
 class Case:
     """Encode A on both sides once; run protected SpMVs on both."""
 
-    def __init__(self, O, torch, A, bs=32, max_rounds=4):
+    def __init__(self, O, torch, A, bs=32, max_rounds=4, c_csr=False):
         from paper_conf_dsn_schollbkw16_b200 import encode
         self.O, self.torch, self.A, self.bs = O, torch, A, bs
         self.enc = O.encode(A, bs)
-        self.h = encode(A, bs, max_rounds)
+        self.h = encode(A, bs, max_rounds, c_csr=c_csr)
         self.max_rounds = max_rounds
 
     def check_encoding(self):
@@ -114,10 +114,11 @@ MATRICES = {
 }
 
 
+@pytest.mark.parametrize("c_csr", [False, True])
 @pytest.mark.parametrize("name", sorted(MATRICES))
-def test_encode_and_spmv_error_free(O, torch_cuda, name):
+def test_encode_and_spmv_error_free(O, torch_cuda, name, c_csr):
     A = MATRICES[name]()
-    c = Case(O, torch_cuda, A)
+    c = Case(O, torch_cuda, A, c_csr=c_csr)
     c.check_encoding()
     for seed in (42, 43):
         ref = c.run(G.uniform_vector(A.n, seed))
@@ -149,10 +150,11 @@ def test_single_bit_flips_config0(O, torch_cuda):
     assert detected > 30
 
 
+@pytest.mark.parametrize("c_csr", [False, True])
 @pytest.mark.parametrize("target", [0, 1, 2])
-def test_checksum_and_result_targets(O, torch_cuda, target):
+def test_checksum_and_result_targets(O, torch_cuda, target, c_csr):
     A = MATRICES["st27_11"]()
-    c = Case(O, torch_cuda, A)
+    c = Case(O, torch_cuda, A, c_csr=c_csr)
     n_el = A.n if target == 0 else c.enc.nb
     rng = np.random.default_rng(target)
     idx = rng.choice(n_el, 12, replace=False)
@@ -189,6 +191,28 @@ def test_rate_mode_rmat_bs8(O, torch_cuda):
     A = MATRICES["rmat11"]()
     c = Case(O, torch_cuda, A, bs=8)
     c.run(G.uniform_vector(A.n, 1), rate=dict(seed=5, lam=1e-3, targets=0b111, call=7))
+
+
+def test_compact_formats_chosen(O, torch_cuda):
+    # the encoder picks the narrowest exact type
+    from paper_conf_dsn_schollbkw16_b200 import encode
+    cases = [(G.laplacian_3d_7pt(16), "int8+u16"), (G.random_csr(500, 0.02, 1), "f64+u16"),
+             (G.random_csr(300, 0.05, 2, integer=True, max_int=100), "int16+u16")]
+    for A, fmt in cases:
+        info = encode(A).info()
+        assert info["c_format_name"] == fmt, (A.name, info)
+    info = encode(G.laplacian_3d_7pt(16), c_csr=True).info()
+    assert info["c_format_name"] == "csr-f64"
+    A = G.laplacian_3d_7pt(16)
+    info = encode(A).info()
+    assert info["general_groups"] == 0 and info["lean"] == 1
+
+
+@pytest.mark.parametrize("lam", [1e-4])
+def test_rate_mode_csr_c(O, torch_cuda, lam):
+    A = MATRICES["lap3d_16"]()
+    c = Case(O, torch_cuda, A, c_csr=True)
+    c.run(G.uniform_vector(A.n, 11), rate=dict(seed=99, lam=lam, targets=0b111, call=5))
 
 
 def test_x_norm_given(O, torch_cuda):
