@@ -43,6 +43,9 @@ template <> struct CType<CF_I16> { using T = int16_t; };
 template <> struct CType<CF_F32> { using T = float; };
 
 constexpr int kLeanWarps = 4;  // warps per CTA of k_lean (<= 4)
+#ifndef ABFT_LEAN_MINB
+#define ABFT_LEAN_MINB 5  // min resident CTAs per SM the register budget targets (measured best)
+#endif
 
 struct StageCfg {
   int32_t capA, capC;     // staged capacity (elements) of a group's A / C segment
@@ -709,7 +712,7 @@ __device__ __forceinline__ void issue_stage(const SpmvArgs &a, int64_t g, int32_
 }
 
 template <bool CHECK, bool INJECT, int CF>
-__global__ void __launch_bounds__(kLeanWarps * 32, 4) k_lean(const SpmvArgs a) {
+__global__ void __launch_bounds__(kLeanWarps * 32, ABFT_LEAN_MINB) k_lean(const SpmvArgs a) {
   extern __shared__ __align__(128) unsigned char smem[];
   __shared__ double s_red[kLeanWarps * 32];
   __shared__ int s_flag[2];
