@@ -171,6 +171,52 @@ def oracle_baseline(A, x, seconds=12.0, check=True):
     return enc, dt, reps
 
 
+def run_pcg(args):
+    """configs[4]: Jacobi-PCG on the 3-D 7-pt Laplacian with the protected
+    SpMV: time-to-solution, iterations and overhead vs the same
+    solver with unprotected SpMVs, at a low and a 10^4x higher error rate."""
+    import torch
+
+    from paper_conf_dsn_schollbkw16_b200 import Inject, encode
+    from paper_conf_dsn_schollbkw16_b200 import inputs as G
+    world, rank, local = dist_init()
+    n3 = args.pcg_n
+    A = G.laplacian_3d_7pt(n3)
+    h = encode(A, 32, args.max_rounds)
+    # b = A x* with x* seeded (R15/Q20); computed through the library's own
+    # plain SpMV (inputs, not a parity check)
+    xs = torch.from_numpy(G.uniform_vector(A.n, 43)).cuda()
+    b = h.spmv(xs, mode=0)
+    x0 = torch.from_numpy(G.uniform_vector(A.n, 44)).cuda()
+    torch.cuda.synchronize()
+    res = {}
+    for label, check, lam in [("unprotected", False, 0.0), ("protected", True, 0.0),
+                              ("protected_lam1e-8", True, 1e-8), ("protected_lam1e-4", True, 1e-4),
+                              ("unprotected_lam1e-4", False, 1e-4)]:
+        inj = Inject.rate(seed=7, lam=lam) if lam > 0 else None
+        times, st = [], None
+        for rep in range(max(1, args.pcg_reps)):
+            x = x0.clone()
+            torch.cuda.synchronize()
+            t0 = time.perf_counter()
+            status, st = h.pcg(b, x, tol=1e-6, inject=inj, check=check)
+            times.append(time.perf_counter() - t0)
+        # solution check: fault-free true residual (Q17)
+        r = b - h.spmv(x, mode=0)
+        rel = float(torch.linalg.norm(r) / torch.linalg.norm(b))
+        res[label] = {"status": status, "ms": round(1e3 * statistics.median(times), 3),
+                      "iters": st["iters"], "flagged_blocks": st["flagged_blocks"],
+                      "recomputed_blocks": st["recomputed_blocks"],
+                      "true_rel_residual": rel, "correct": bool(status == 0 and rel <= 1e-5)}
+    base = res["unprotected"]["ms"]
+    for k, v in res.items():
+        v["overhead_pct"] = round((v["ms"] / base - 1) * 100, 2)
+    if rank == 0:
+        print(json.dumps({"metric": "PCG time-to-solution (ms), Jacobi, tol 1e-6",
+                          "workload": f"3-D 7-point Laplacian {n3}^3 (BASELINE configs[4])",
+                          "n": A.n, "nnz": A.nnz, "n_gpus": world, "results": res}), flush=True)
+
+
 def run_reference(args):
     """--impl reference: the CPU oracle (oracle/liboracle.so), rank 0 only."""
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -364,11 +410,16 @@ def main():
     ap.add_argument("--max-rounds", type=int, default=4)
     ap.add_argument("--lam", type=float, default=0.0, help="rate-mode fault rate per op")
     ap.add_argument("--c-csr", action="store_true", help="paper-literal CSR checksum matrix")
+    ap.add_argument("--pcg", action="store_true", help="configs[4]: PCG time-to-solution")
+    ap.add_argument("--pcg-n", type=int, default=192)
+    ap.add_argument("--pcg-reps", type=int, default=3)
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     args = ap.parse_args()
     if args.impl == "reference":
         run_reference(args)
+    elif args.pcg:
+        run_pcg(args)
     else:
         run_ours(args)
 

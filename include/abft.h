@@ -193,6 +193,8 @@ typedef struct {
  * unprotected baseline with the same kernels.  inj: nullable; its `call`
  * is the index of the first SpMV (call + j for the j-th).  res_hist:
  * nullable device [max_iter + 1] of ||r_j||_2.  stats: nullable (host).
+ * b, x, diag and res_hist must be 16-byte aligned (128-bit vector accesses;
+ * ABFT_EINVAL otherwise).
  * Synchronises the stream.  Returns ABFT_OK, ABFT_ENOCONV or ABFT_EBREAKDOWN. */
 abft_status abft_pcg(abft_handle_t h, const double *b, double *x, const double *diag,
                      double tol, int64_t max_iter, const abft_inject_t *inj, int32_t check,

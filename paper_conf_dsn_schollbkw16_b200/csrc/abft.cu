@@ -67,8 +67,8 @@ struct abft_ctx {
   int cfmt = CF_CSR;         // format of C streamed by k_lean
   void *cval_n = nullptr;    // compact C values
   uint16_t *ccol16 = nullptr;
-  int32_t *cbase = nullptr;
-  int32_t *crp_c = nullptr;  // compact row starts (16-element aligned)
+  int32_t *cb8 = nullptr;    // compact C: column base per 8-entry chunk
+  int32_t *crp_c = nullptr;  // compact row starts (32-entry aligned)
   int64_t nnz_cpad = 0;      // compact slots incl. row padding
   StageCfg stage{};
   bool lean = false;        // k_lean usable (b_s = 32, 16-B aligned A)
@@ -96,7 +96,7 @@ struct abft_ctx {
   double *pcg_sc = nullptr;
   int32_t *pcg_state = nullptr;
   int64_t pcg_n = 0;
-  int64_t ncta256 = 0;  // ceil(n / 256): PCG vector-kernel grid
+  int64_t ncta256 = 0;  // ceil(n / kPcgRows): PCG vector-kernel grid
   std::vector<void *> owned;
   int device = 0;
   int num_sms = 148;
@@ -137,7 +137,7 @@ SpmvArgs make_args(const abft_ctx *h, const double *x, double *y, const double *
   a.cval = h->c_val;
   a.cval_n = h->cval_n;
   a.ccol16 = h->ccol16;
-  a.cbase = h->cbase;
+  a.cb8 = h->cb8;
   a.crp_c = h->crp_c;
   a.K = h->K;
   a.x = x;
@@ -321,20 +321,18 @@ abft_status init_device_once(int device) {
 abft_status build_compact_c(abft_ctx *h, cudaStream_t s) {
   if (h->nnz_c == 0) return ABFT_OK;
   int32_t *dev = nullptr;
-  TRY(dalloc(h, &dev, 2));
-  TRY(dalloc(h, &h->cbase, (size_t)h->nb));
-  CK(cudaMemsetAsync(dev, 0, 2 * sizeof(int32_t), s));
+  TRY(dalloc(h, &dev, 1));
+  CK(cudaMemsetAsync(dev, 0, sizeof(int32_t), s));
   const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((h->nb + 7) / 8, 65535));
-  k_cformat_scan<<<grid, 256, 0, s>>>(h->nb, h->c_rp, h->c_col, h->c_val, dev, dev + 1, h->cbase);
+  k_cformat_scan<<<grid, 256, 0, s>>>(h->nb, h->c_rp, h->c_col, h->c_val, dev);
   CK(cudaGetLastError());
-  int32_t hv[2];
-  CK(cudaMemcpyAsync(hv, dev, sizeof hv, cudaMemcpyDeviceToHost, s));
+  int32_t props = 0;
+  CK(cudaMemcpyAsync(&props, dev, sizeof props, cudaMemcpyDeviceToHost, s));
   CK(cudaStreamSynchronize(s));
-  const int32_t props = hv[0], span = hv[1];
-  if (span >= 65536) return ABFT_OK;  // columns do not fit uint16 offsets: keep CSR
+  if (props & 8) return ABFT_OK;  // a chunk spans >= 65536 columns: keep CSR
   const int cf = !(props & 1) ? CF_I8 : !(props & 2) ? CF_I16 : !(props & 4) ? CF_F32 : CF_F64;
   const size_t sz = (size_t)cf_size(cf);
-  // compact row starts: exclusive scan of the 16-element padded row lengths
+  // compact row starts: exclusive scan of the 32-entry padded row lengths
   int32_t *plen = nullptr, *totals = nullptr;
   const int64_t nscan = (h->nb + 1023) / 1024;
   TRY(dalloc(h, &plen, (size_t)h->nb));
@@ -352,28 +350,29 @@ abft_status build_compact_c(abft_ctx *h, cudaStream_t s) {
   char *cv = nullptr;
   TRY(dalloc(h, &cv, (size_t)npad * sz + 64));
   TRY(dalloc(h, &h->ccol16, (size_t)npad + 32));
+  TRY(dalloc(h, &h->cb8, (size_t)npad / 8 + 8));
   CK(cudaMemsetAsync(cv, 0, (size_t)npad * sz + 64, s));
   CK(cudaMemsetAsync(h->ccol16, 0, ((size_t)npad + 32) * 2, s));
+  CK(cudaMemsetAsync(h->cb8, 0, ((size_t)npad / 8 + 8) * 4, s));
   switch (cf) {
     case CF_I8:
       k_cformat_fill<int8_t><<<grid, 256, 0, s>>>(h->nb, h->c_rp, h->crp_c, h->c_col, h->c_val,
-                                                  h->cbase, reinterpret_cast<int8_t *>(cv),
-                                                  h->ccol16);
+                                                  reinterpret_cast<int8_t *>(cv), h->ccol16,
+                                                  h->cb8);
       break;
     case CF_I16:
       k_cformat_fill<int16_t><<<grid, 256, 0, s>>>(h->nb, h->c_rp, h->crp_c, h->c_col, h->c_val,
-                                                   h->cbase, reinterpret_cast<int16_t *>(cv),
-                                                   h->ccol16);
+                                                   reinterpret_cast<int16_t *>(cv), h->ccol16,
+                                                   h->cb8);
       break;
     case CF_F32:
       k_cformat_fill<float><<<grid, 256, 0, s>>>(h->nb, h->c_rp, h->crp_c, h->c_col, h->c_val,
-                                                 h->cbase, reinterpret_cast<float *>(cv),
-                                                 h->ccol16);
+                                                 reinterpret_cast<float *>(cv), h->ccol16, h->cb8);
       break;
     default:
       k_cformat_fill<double><<<grid, 256, 0, s>>>(h->nb, h->c_rp, h->crp_c, h->c_col, h->c_val,
-                                                  h->cbase, reinterpret_cast<double *>(cv),
-                                                  h->ccol16);
+                                                  reinterpret_cast<double *>(cv), h->ccol16,
+                                                  h->cb8);
       break;
   }
   CK(cudaGetLastError());
@@ -412,11 +411,13 @@ abft_status plan_fused(abft_ctx *h, cudaStream_t s) {
       o += align16((uint32_t)(c.capC + 2) * 8);
       c.off_cc = o;
       o += align16((uint32_t)(c.capC + 6) * 4);
-    } else {  // compact: a 16-element padded row of values and uint16 columns
-      const uint32_t cpad16 = ((uint32_t)c.capC + 15u) & ~15u;
-      o += align16(cpad16 * cf_size(h->cfmt));
+    } else {  // compact: a padded row of values, uint16 offsets, chunk bases
+      const uint32_t cpad = ((uint32_t)c.capC + kCRowAlign - 1) & ~(uint32_t)(kCRowAlign - 1);
+      o += align16(cpad * cf_size(h->cfmt));
       c.off_cc = o;
-      o += align16(cpad16 * 2);
+      o += align16(cpad * 2);
+      c.off_cb = o;
+      o += align16(cpad / 2);
     }
     c.off_cp = o;  // padded C products (one gap per 8; CSR format only)
     if (h->cfmt == CF_CSR) o += align16((uint32_t)(c.capC + c.capC / 8 + 8) * 8);
@@ -522,7 +523,7 @@ abft_status abft_encode(const abft_csr_t *A, int32_t block_size, int32_t max_rou
   h->rp = A->row_ptr;
   h->ci = A->col_idx;
   h->va = A->val;
-  h->ncta256 = (h->n + 255) / 256;
+  h->ncta256 = (h->n + kPcgRows - 1) / kPcgRows;
 
   abft_status st;
   int32_t *counts = nullptr, *totals = nullptr, *stats = nullptr;
@@ -689,7 +690,8 @@ abft_status abft_info(abft_handle_t h, abft_info_t *info) {
   if (h->cfmt == CF_CSR)
     info->c_bytes = 12 * h->nnz_c + 4 * (h->nb + 1);
   else
-    info->c_bytes = (int64_t)(cf_size(h->cfmt) + 2) * h->nnz_cpad + 8 * (h->nb + 1) + 4 * h->nb;
+    info->c_bytes = (int64_t)(cf_size(h->cfmt) + 2) * h->nnz_cpad + h->nnz_cpad / 2 +
+                    8 * (h->nb + 1);
   info->groups = h->ngroups;
   info->general_groups = h->lean ? h->n_glist : h->ngroups;
   info->lean = h->lean ? 1 : 0;

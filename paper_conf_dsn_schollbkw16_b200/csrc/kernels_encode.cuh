@@ -112,20 +112,22 @@ __global__ void __launch_bounds__(256) k_encode(const EncodeArgs a) {
 
 // Compact checksum matrix: the values of C in the
 // narrowest type that holds every one of them exactly, and the columns as
-// uint16 offsets from each row's first column.  Lossless: the kernels
-// recover bit-identical c_kj and column indices.
+// uint16 offsets from a per-chunk base (one int32 per 8 entries).  Rows start
+// on 32-entry boundaries so every staged piece is 16-B aligned.  Lossless:
+// the kernels recover bit-identical c_kj and column indices.
 enum { CF_CSR = 0, CF_I8 = 1, CF_I16 = 2, CF_F32 = 3, CF_F64 = 4 };
+constexpr int kCRowAlign = 32;  // compact row alignment (entries)
 
 // props bits: 1 = some value is not an integer in [-128,127], 2 = not in
-// [-32768,32767], 4 = not exactly representable in float; span = max over
-// rows of (last column - first column).
+// [-32768,32767], 4 = not exactly representable in float, 8 = some 8-entry
+// chunk spans >= 65536 columns (no uint16 offsets).
 __global__ void k_cformat_scan(int64_t nb, const int32_t *__restrict__ crp,
                                const int32_t *__restrict__ ccol, const double *__restrict__ cval,
-                               int32_t *props, int32_t *span, int32_t *cbase) {
+                               int32_t *props) {
   const int lane = threadIdx.x & 31;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
-  int32_t pr = 0, sp = 0;
+  int32_t pr = 0;
   for (int64_t k = gw; k < nb; k += nw) {
     const int32_t b = crp[k], e = crp[k + 1];
     for (int32_t q = b + lane; q < e; q += 32) {
@@ -134,42 +136,37 @@ __global__ void k_cformat_scan(int64_t nb, const int32_t *__restrict__ crp,
       if (!(v == rint(v)) || v < -32768.0 || v > 32767.0) pr |= 2;
       if (!((double)(float)v == v) && v == v) pr |= 4;
       if (v != v) pr |= 7;  // NaN: keep f64
-    }
-    if (lane == 0) {
-      cbase[k] = e > b ? ccol[b] : 0;
-      if (e > b) sp = max(sp, ccol[e - 1] - ccol[b]);
+      if (((q - b) & 7) == 0) {
+        const int32_t last = min(q + 7, e - 1);
+        if (ccol[last] - ccol[q] >= 65536) pr |= 8;
+      }
     }
   }
   pr = __reduce_or_sync(kFull, pr);
-  sp = warp_max_i(sp);
-  if (lane == 0) {
-    atomicOr(props, pr);
-    atomicMax(span, sp);
-  }
+  if (lane == 0) atomicOr(props, pr);
 }
 
-// Compact rows start on 16-element boundaries (crp_c = exclusive scan of the
-// padded lengths), so a row lands 16-B aligned in the kernels' staging buffers
-// and lane l can load elements 8l .. 8l+7 with vector loads.  Pad slots are 0.
 __global__ void k_cformat_padlen(int64_t nb, const int32_t *__restrict__ crp, int32_t *plen) {
   for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < nb;
        k += (int64_t)gridDim.x * blockDim.x)
-    plen[k] = (crp[k + 1] - crp[k] + 15) & ~15;
+    plen[k] = (crp[k + 1] - crp[k] + kCRowAlign - 1) & ~(kCRowAlign - 1);
 }
 
 template <typename T>
 __global__ void k_cformat_fill(int64_t nb, const int32_t *__restrict__ crp,
                                const int32_t *__restrict__ crp_c, const int32_t *__restrict__ ccol,
-                               const double *__restrict__ cval, const int32_t *__restrict__ cbase,
-                               T *cv, uint16_t *cc16) {
+                               const double *__restrict__ cval, T *cv, uint16_t *cc16,
+                               int32_t *cb8) {
   const int lane = threadIdx.x & 31;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
   for (int64_t k = gw; k < nb; k += nw) {
-    const int32_t b = crp[k], e = crp[k + 1], base = cbase[k], d = crp_c[k] - b;
+    const int32_t b = crp[k], e = crp[k + 1], d = crp_c[k] - b;
     for (int32_t q = b + lane; q < e; q += 32) {
+      const int32_t base = ccol[b + ((q - b) & ~7)];  // first column of the chunk
       cv[q + d] = (T)cval[q];
       cc16[q + d] = (uint16_t)(ccol[q] - base);
+      if (((q - b) & 7) == 0) cb8[(q + d) >> 3] = base;
     }
   }
 }

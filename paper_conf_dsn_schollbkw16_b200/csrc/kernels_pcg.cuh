@@ -1,16 +1,23 @@
 // kernels_pcg.cuh -- Jacobi-PCG vector kernels (SVI-A; Saad
-// Alg. 9.1).  The SpMV q = A p is the protected k_fused/k_correct pair; these
-// kernels fuse the vector updates with their dot products.  Every dot is PW
-// over the global index (R2): each CTA reduces its aligned 256-row subtree,
-// the last CTA (atomic ticket) completes the tree and updates the scalars, so
-// the iteration runs without host round trips.  A device `state` word makes
-// every kernel of a converged / broken-down solve a no-op.
+// Alg. 9.1).  The SpMV q = A p is the protected k_lean/k_general/k_correct
+// set; these kernels fuse the vector updates with their dot products.
+//
+// Every dot is PW over the global index (R2): a CTA owns an aligned chunk of
+// kPcgRows = 2048 rows; thread t holds rows 8t..8t+7 of it (vector loads),
+// reduces them with an 8-leaf register tree, the warp's 32 sums by the xor
+// butterfly (an aligned 256-row node) and the 8 warp sums by a tree -- the
+// chunk's PW node.  The last CTA (atomic ticket) completes the tree over the
+// chunk sums and updates the scalars, so an iteration needs no host round
+// trip.  A device `state` word turns every kernel of a finished solve into a
+// no-op.
 #pragma once
 #include "abft_device.cuh"
 
 namespace abft {
 
 constexpr int kPcgThreads = 256;
+constexpr int kPcgPer = 8;                         // rows per thread
+constexpr int kPcgRows = kPcgThreads * kPcgPer;    // rows per CTA (aligned)
 
 enum { PCG_RUN = 0, PCG_CONVERGED = 1, PCG_BREAKDOWN = 2, PCG_MAXITER = 3 };
 
@@ -27,7 +34,7 @@ struct PcgArgs {
   const double *__restrict__ b;
   double *x, *r, *z, *p, *q;
   const double *__restrict__ d;
-  double *part0, *part1, *part2;  // per-CTA partial sums
+  double *part0, *part1, *part2;  // per-CTA chunk sums
   unsigned *ticket;
   PcgScalars *sc;
   double *hist;                   // nullable
@@ -37,13 +44,42 @@ struct PcgArgs {
   int32_t check;
 };
 
-// CTA-level PW of one value per thread (thread t <-> row base + t): butterfly
-// in each warp, tree over the 8 warp sums.  All threads get the result.
-__device__ __forceinline__ double cta_pw256(double v, double *s_w) {
+// Eight consecutive doubles v[0..8) at p + 8t (or absent past n).
+__device__ __forceinline__ void ld8(double (&v)[8], const double *p, int64_t i0, int64_t n) {
+  if (i0 + 8 <= n) {
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const double2 w = *reinterpret_cast<const double2 *>(p + i0 + 2 * u);
+      v[2 * u] = w.x;
+      v[2 * u + 1] = w.y;
+    }
+  } else {
+#pragma unroll
+    for (int u = 0; u < 8; ++u) v[u] = i0 + u < n ? p[i0 + u] : 0.0;
+  }
+}
+__device__ __forceinline__ void st8(double *p, const double (&v)[8], int64_t i0, int64_t n) {
+  if (i0 + 8 <= n) {
+#pragma unroll
+    for (int u = 0; u < 4; ++u)
+      *reinterpret_cast<double2 *>(p + i0 + 2 * u) = make_double2(v[2 * u], v[2 * u + 1]);
+  } else {
+#pragma unroll
+    for (int u = 0; u < 8; ++u)
+      if (i0 + u < n) p[i0 + u] = v[u];
+  }
+}
+
+// CTA chunk sum: per-thread 8-leaf tree (absent past n), warp butterfly,
+// tree over the 8 warps.  All threads get the result.
+__device__ __forceinline__ double cta_pw(double (&v)[8], int64_t i0, int64_t n, double *s_w) {
+#pragma unroll
+  for (int u = 0; u < 8; ++u)
+    if (i0 + u >= n) v[u] = kAbsent;
+  double t = bfly32(tree<8>(v));
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  v = bfly32(v);
   __syncthreads();
-  if (lane == 0) s_w[warp] = v;
+  if (lane == 0) s_w[warp] = t;
   __syncthreads();
   double w[8];
 #pragma unroll
@@ -51,16 +87,26 @@ __device__ __forceinline__ double cta_pw256(double v, double *s_w) {
   return tree<8>(w);
 }
 
-// Last-CTA completion of PW over partials[0..ncta) (aligned 256-row
-// subtrees).  Called by all threads of the last CTA.
+// Last-CTA completion of PW over partials[0..ncta) (aligned chunk nodes):
+// thread t reduces an aligned run of m <= 32 partials in registers (PwSeq
+// beyond), then a shared-memory tree over the threads.
 __device__ __forceinline__ double grid_pw(const double *partials, int ncta, double *s_red) {
   int m = 1;
   while (m * kPcgThreads < ncta) m <<= 1;
-  PwSeq acc;
   const int b = threadIdx.x * m;
-  for (int q = b; q < min(b + m, ncta); ++q) acc.push(__ldcg(partials + q));
+  double t;
+  if (m <= 32) {
+    double v[32];
+#pragma unroll
+    for (int q = 0; q < 32; ++q) v[q] = (q < m && b + q < ncta) ? __ldcg(partials + b + q) : kAbsent;
+    t = tree<32>(v);
+  } else {
+    PwSeq acc;
+    for (int q = b; q < min(b + m, ncta); ++q) acc.push(__ldcg(partials + q));
+    t = acc.finish();
+  }
   __syncthreads();
-  s_red[threadIdx.x] = acc.finish();
+  s_red[threadIdx.x] = t;
   __syncthreads();
   for (int s = 1; s < kPcgThreads; s <<= 1) {
     if ((threadIdx.x & (2 * s - 1)) == 0)
@@ -70,8 +116,7 @@ __device__ __forceinline__ double grid_pw(const double *partials, int ncta, doub
   return s_red[0];
 }
 
-// Ticket: returns true in the last CTA to finish (after its partials are
-// written).  The last CTA resets the ticket for the next kernel.
+// Ticket: true in the last CTA to finish (after its partials are written).
 __device__ __forceinline__ bool last_cta(unsigned *ticket, int *s_flag) {
   __syncthreads();
   if (threadIdx.x == 0) {
@@ -86,6 +131,16 @@ __device__ __forceinline__ bool last_cta(unsigned *ticket, int *s_flag) {
 
 __device__ __forceinline__ bool pcg_skip(const PcgScalars *sc) {
   return *(volatile const int32_t *)&sc->state != PCG_RUN;
+}
+
+__device__ __forceinline__ void pcg_stats(const PcgArgs &a, PcgScalars *sc) {
+  sc->calls += 1;
+  if (a.check) {
+    const int32_t *nf = a.n_flags;
+    sc->flagged += nf[0];
+    for (int r = 0; r < a.max_rounds; ++r) sc->recomputed += nf[r];
+    if (nf[a.max_rounds] > 0) sc->uncorrected += 1;
+  }
 }
 
 // diag(A) (R21; missing diagonal -> 0, as the oracle)
@@ -105,26 +160,29 @@ __global__ void __launch_bounds__(kPcgThreads) k_pcg_init(const PcgArgs a) {
   __shared__ double s_w[8];
   __shared__ double s_red[kPcgThreads];
   __shared__ int s_flag;
-  const int64_t i = (int64_t)blockIdx.x * kPcgThreads + threadIdx.x;
-  double rz = kAbsent, rr = kAbsent, bb = kAbsent;
-  if (i < a.n) {
-    const double bi = a.b[i];
-    const double ri = dsub(bi, a.q[i]);
-    const double zi = __ddiv_rn(ri, a.d[i]);
-    a.r[i] = ri;
-    a.z[i] = zi;
-    a.p[i] = zi;
-    rz = dmul(ri, zi);
-    rr = dmul(ri, ri);
-    bb = dmul(bi, bi);
+  const int64_t i0 = (int64_t)blockIdx.x * kPcgRows + threadIdx.x * kPcgPer;
+  double bv[8], qv[8], dv[8], r[8], z[8], rz[8], rr[8], bb[8];
+  ld8(bv, a.b, i0, a.n);
+  ld8(qv, a.q, i0, a.n);
+  ld8(dv, a.d, i0, a.n);
+#pragma unroll
+  for (int u = 0; u < 8; ++u) {
+    r[u] = dsub(bv[u], qv[u]);
+    z[u] = __ddiv_rn(r[u], dv[u]);
+    rz[u] = dmul(r[u], z[u]);
+    rr[u] = dmul(r[u], r[u]);
+    bb[u] = dmul(bv[u], bv[u]);
   }
-  rz = cta_pw256(rz, s_w);
-  rr = cta_pw256(rr, s_w);
-  bb = cta_pw256(bb, s_w);
+  st8(a.r, r, i0, a.n);
+  st8(a.z, z, i0, a.n);
+  st8(a.p, z, i0, a.n);
+  const double RZc = cta_pw(rz, i0, a.n, s_w);
+  const double RRc = cta_pw(rr, i0, a.n, s_w);
+  const double BBc = cta_pw(bb, i0, a.n, s_w);
   if (threadIdx.x == 0) {
-    a.part0[blockIdx.x] = rz;
-    a.part1[blockIdx.x] = rr;
-    a.part2[blockIdx.x] = bb;
+    a.part0[blockIdx.x] = RZc;
+    a.part1[blockIdx.x] = RRc;
+    a.part2[blockIdx.x] = BBc;
   }
   if (!last_cta(a.ticket, &s_flag)) return;
   const double RZ = grid_pw(a.part0, gridDim.x, s_red);
@@ -132,13 +190,7 @@ __global__ void __launch_bounds__(kPcgThreads) k_pcg_init(const PcgArgs a) {
   const double BB = grid_pw(a.part2, gridDim.x, s_red);
   if (threadIdx.x == 0) {
     PcgScalars *sc = a.sc;
-    sc->calls += 1;  // the SpMV q = A x0
-    if (a.check) {
-      const int32_t *nf = a.n_flags;
-      sc->flagged += nf[0];
-      for (int r = 0; r < a.max_rounds; ++r) sc->recomputed += nf[r];
-      if (nf[a.max_rounds] > 0) sc->uncorrected += 1;
-    }
+    pcg_stats(a, sc);  // the SpMV q = A x0
     sc->rho = RZ;
     sc->res = __dsqrt_rn(RR);
     sc->thr = dmul(a.tol, __dsqrt_rn(BB));
@@ -156,28 +208,24 @@ __global__ void __launch_bounds__(kPcgThreads) k_pcg_dot(const PcgArgs a) {
   __shared__ double s_red[kPcgThreads];
   __shared__ int s_flag;
   if (pcg_skip(a.sc)) return;
-  const int64_t i = (int64_t)blockIdx.x * kPcgThreads + threadIdx.x;
-  double pq = kAbsent;
-  if (i < a.n) pq = dmul(a.p[i], a.q[i]);
-  pq = cta_pw256(pq, s_w);
-  if (threadIdx.x == 0) a.part0[blockIdx.x] = pq;
+  const int64_t i0 = (int64_t)blockIdx.x * kPcgRows + threadIdx.x * kPcgPer;
+  double pv[8], qv[8];
+  ld8(pv, a.p, i0, a.n);
+  ld8(qv, a.q, i0, a.n);
+#pragma unroll
+  for (int u = 0; u < 8; ++u) pv[u] = dmul(pv[u], qv[u]);
+  const double PQc = cta_pw(pv, i0, a.n, s_w);
+  if (threadIdx.x == 0) a.part0[blockIdx.x] = PQc;
   if (!last_cta(a.ticket, &s_flag)) return;
   const double PQ = grid_pw(a.part0, gridDim.x, s_red);
   if (threadIdx.x == 0) {
     PcgScalars *sc = a.sc;
-    sc->calls += 1;
-    if (a.check) {
-      const int32_t *nf = a.n_flags;
-      sc->flagged += nf[0];
-      for (int r = 0; r < a.max_rounds; ++r) sc->recomputed += nf[r];
-      if (nf[a.max_rounds] > 0) sc->uncorrected += 1;
-    }
+    pcg_stats(a, sc);
     sc->pq = PQ;
-    if (!(PQ > 0.0)) {
+    if (!(PQ > 0.0))
       sc->state = PCG_BREAKDOWN;
-    } else {
+    else
       sc->alpha = __ddiv_rn(sc->rho, PQ);
-    }
     *a.ticket = 0u;
   }
 }
@@ -190,23 +238,29 @@ __global__ void __launch_bounds__(kPcgThreads) k_pcg_update(const PcgArgs a) {
   __shared__ int s_flag;
   if (pcg_skip(a.sc)) return;
   const double alpha = a.sc->alpha;
-  const int64_t i = (int64_t)blockIdx.x * kPcgThreads + threadIdx.x;
-  double rz = kAbsent, rr = kAbsent;
-  if (i < a.n) {
-    const double pi = a.p[i];
-    a.x[i] = dadd(a.x[i], dmul(alpha, pi));
-    const double ri = dsub(a.r[i], dmul(alpha, a.q[i]));
-    const double zi = __ddiv_rn(ri, a.d[i]);
-    a.r[i] = ri;
-    a.z[i] = zi;
-    rz = dmul(ri, zi);
-    rr = dmul(ri, ri);
+  const int64_t i0 = (int64_t)blockIdx.x * kPcgRows + threadIdx.x * kPcgPer;
+  double xv[8], pv[8], rv[8], qv[8], dv[8], rz[8], rr[8];
+  ld8(xv, a.x, i0, a.n);
+  ld8(pv, a.p, i0, a.n);
+  ld8(rv, a.r, i0, a.n);
+  ld8(qv, a.q, i0, a.n);
+  ld8(dv, a.d, i0, a.n);
+#pragma unroll
+  for (int u = 0; u < 8; ++u) {
+    xv[u] = dadd(xv[u], dmul(alpha, pv[u]));
+    rv[u] = dsub(rv[u], dmul(alpha, qv[u]));
+    dv[u] = __ddiv_rn(rv[u], dv[u]);  // z
+    rz[u] = dmul(rv[u], dv[u]);
+    rr[u] = dmul(rv[u], rv[u]);
   }
-  rz = cta_pw256(rz, s_w);
-  rr = cta_pw256(rr, s_w);
+  st8(a.x, xv, i0, a.n);
+  st8(a.r, rv, i0, a.n);
+  st8(a.z, dv, i0, a.n);
+  const double RZc = cta_pw(rz, i0, a.n, s_w);
+  const double RRc = cta_pw(rr, i0, a.n, s_w);
   if (threadIdx.x == 0) {
-    a.part0[blockIdx.x] = rz;
-    a.part1[blockIdx.x] = rr;
+    a.part0[blockIdx.x] = RZc;
+    a.part1[blockIdx.x] = RRc;
   }
   if (!last_cta(a.ticket, &s_flag)) return;
   const double RZ = grid_pw(a.part0, gridDim.x, s_red);
@@ -231,8 +285,14 @@ __global__ void __launch_bounds__(kPcgThreads) k_pcg_update(const PcgArgs a) {
 __global__ void __launch_bounds__(kPcgThreads) k_pcg_p(const PcgArgs a, int64_t iter) {
   const int64_t it = *(volatile const int64_t *)&a.sc->it;
   if (it != iter) return;  // this iteration did not execute
-  const int64_t i = (int64_t)blockIdx.x * kPcgThreads + threadIdx.x;
-  if (i < a.n) a.p[i] = dadd(a.z[i], dmul(a.sc->beta, a.p[i]));
+  const double beta = a.sc->beta;
+  const int64_t i0 = (int64_t)blockIdx.x * kPcgRows + threadIdx.x * kPcgPer;
+  double zv[8], pv[8];
+  ld8(zv, a.z, i0, a.n);
+  ld8(pv, a.p, i0, a.n);
+#pragma unroll
+  for (int u = 0; u < 8; ++u) pv[u] = dadd(zv[u], dmul(beta, pv[u]));
+  st8(a.p, pv, i0, a.n);
 }
 
 }  // namespace abft

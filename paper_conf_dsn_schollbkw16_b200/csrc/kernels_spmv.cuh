@@ -53,7 +53,7 @@ struct StageCfg {
   int32_t warps;          // warps per CTA
   uint32_t stage_bytes;   // bytes per stage
   uint32_t bar_bytes;     // mbarrier region at the start of dynamic smem
-  uint32_t off_rp, off_x, off_av, off_ac, off_cv, off_cc, off_cp;
+  uint32_t off_rp, off_x, off_av, off_ac, off_cv, off_cc, off_cp, off_cb;
 };
 
 struct SpmvArgs {
@@ -70,9 +70,9 @@ struct SpmvArgs {
   const int32_t *__restrict__ ccol;
   const double *__restrict__ cval;
   const void *__restrict__ cval_n;       // compact C values (CF != CF_CSR)
-  const uint16_t *__restrict__ ccol16;  // compact C columns: offset from cbase
-  const int32_t *__restrict__ cbase;    // first column of each C row
-  const int32_t *__restrict__ crp_c;    // compact row starts (16-element aligned)
+  const uint16_t *__restrict__ ccol16;  // compact C columns: offset from the chunk base
+  const int32_t *__restrict__ cb8;      // compact C: column base of each 8-entry chunk
+  const int32_t *__restrict__ crp_c;    // compact row starts (32-entry aligned)
   const double *__restrict__ K;
   const double *__restrict__ x;
   double *__restrict__ y;
@@ -466,8 +466,7 @@ __device__ __forceinline__ int cpad(int e) { return e + (e >> 3); }
 
 template <bool CHECK, bool INJECT, int CF>
 __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa, int32_t ea,
-                                        int32_t sc, int32_t ec, int32_t cb, unsigned char *st,
-                                        int lane) {
+                                        int32_t sc, int32_t ec, unsigned char *st, int lane) {
   using CT = typename CType<CF>::T;
   const StageCfg &c = a.sc;
   const int64_t i = g * 32 + lane;
@@ -581,6 +580,7 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
     // offsets come in with vector loads, products never touch shared memory
     const unsigned char *cvb = st + c.off_cv;
     const uint16_t *c16 = reinterpret_cast<const uint16_t *>(st + c.off_cc);
+    const int32_t *cbs = reinterpret_cast<const int32_t *>(st + c.off_cb);
 #pragma unroll
     for (int t = 0; t < 4; ++t) {
       double v[8];
@@ -591,6 +591,7 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
           load8(cvv, cvb + (size_t)j0 * sizeof(CT));
           const uint4 o4 = *reinterpret_cast<const uint4 *>(c16 + j0);
           const uint32_t ow[4] = {o4.x, o4.y, o4.z, o4.w};
+          const int32_t cb = cbs[j0 >> 3];
 #pragma unroll
           for (int u = 0; u < 8; ++u) {
             const int32_t col = cb + (int32_t)((ow[u >> 1] >> (16 * (u & 1))) & 0xffffu);
@@ -638,29 +639,25 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
 }
 
 // Group bounds from the per-warp window: lane l holds rp[32 (wb+l)],
-// crp[wb+l] and (compact C) cbase[wb+l] (b_s = 32; clamped to n / nb).
+// crp[wb+l] and (compact C) crp_c[wb+l] (b_s = 32; clamped to n / nb).
 template <int CF>
 struct Window {
   int64_t wb;
-  int32_t rpw, crpw, cbw, ccw;
+  int32_t rpw, crpw, ccw;
   __device__ __forceinline__ void load(const SpmvArgs &a, int64_t base, int lane) {
     wb = base;
     rpw = ld_stream(a.rp + min64((base + lane) * 32, a.n));
     crpw = ld_stream(a.crp + min64(base + lane, a.nb));
-    if (CF != CF_CSR) {
-      cbw = ld_stream(a.cbase + min64(base + lane, a.nb - 1));
-      ccw = ld_stream(a.crp_c + min64(base + lane, a.nb));
-    }
+    if (CF != CF_CSR) ccw = ld_stream(a.crp_c + min64(base + lane, a.nb));
   }
-  // sc/ec: C row bounds (CSR); cb: first column; cc: compact row start
+  // sc/ec: C row bounds (CSR); cc: compact row start
   __device__ __forceinline__ void get(int64_t g, int32_t &sa, int32_t &ea, int32_t &sc,
-                                      int32_t &ec, int32_t &cb, int32_t &cc) const {
+                                      int32_t &ec, int32_t &cc) const {
     const int j = (int)(g - wb);
     sa = __shfl_sync(kFull, rpw, j);
     ea = __shfl_sync(kFull, rpw, j + 1);
     sc = __shfl_sync(kFull, crpw, j);
     ec = __shfl_sync(kFull, crpw, j + 1);
-    cb = CF != CF_CSR ? __shfl_sync(kFull, cbw, j) : 0;
     cc = CF != CF_CSR ? __shfl_sync(kFull, ccw, j) : 0;
   }
 };
@@ -679,17 +676,19 @@ __device__ __forceinline__ void issue_stage(const SpmvArgs &a, int64_t g, int32_
     const int64_t sa4 = sa & ~3, ea4 = min64((ea + 3) & ~3, nnz4);
     const uint32_t bav = ea4 > sa4 ? (uint32_t)(ea4 - sa4) * 8 : 0;
     const uint32_t bac = ea4 > sa4 ? (uint32_t)(ea4 - sa4) * 4 : 0;
-    const int32_t plen = (ec - sc + 15) & ~15;  // compact row: 16-element aligned
+    const int32_t plen = (ec - sc + kCRowAlign - 1) & ~(kCRowAlign - 1);  // padded row
     const int64_t v0 = (int64_t)cc * (int64_t)sizeof(CT), k0 = (int64_t)cc * 2;
     const uint32_t bcv = CHECK ? (uint32_t)plen * (uint32_t)sizeof(CT) : 0;
     const uint32_t bcc = CHECK ? (uint32_t)plen * 2 : 0;
-    mbar_arrive_expect_tx(bar, 128 + 256 + bav + bac + bcv + bcc);
+    const uint32_t bcb = CHECK ? (uint32_t)plen / 2 : 0;  // one int32 per 8 entries
+    mbar_arrive_expect_tx(bar, 128 + 256 + bav + bac + bcv + bcc + bcb);
     bulk_g2s(st + c.off_rp, a.rp + r0, 128, bar, pol);
     bulk_g2s(st + c.off_x, a.x + r0, 256, bar, pol);
     if (bav) bulk_g2s(st + c.off_av, a.va + sa4, bav, bar, pol);
     if (bac) bulk_g2s(st + c.off_ac, a.ci + sa4, bac, bar, pol);
     if (bcv) bulk_g2s(st + c.off_cv, reinterpret_cast<const char *>(a.cval_n) + v0, bcv, bar, pol);
     if (bcc) bulk_g2s(st + c.off_cc, reinterpret_cast<const char *>(a.ccol16) + k0, bcc, bar, pol);
+    if (bcb) bulk_g2s(st + c.off_cb, a.cb8 + (cc >> 3), bcb, bar, pol);
     return;
   }
   const StageCfg &c = a.sc;
@@ -737,18 +736,18 @@ __global__ void __launch_bounds__(kLeanWarps * 32, ABFT_LEAN_MINB) k_lean(const 
   }
   Window<CF> win;
   win.load(a, g0, lane);
-  int32_t sa, ea, sc, ec, cb, cc;  // bounds of the current group, carried from its prefetch
-  win.get(g0, sa, ea, sc, ec, cb, cc);
+  int32_t sa, ea, sc, ec, cc;  // bounds of the current group, carried from its prefetch
+  win.get(g0, sa, ea, sc, ec, cc);
   bool elig = lean_eligible(a, g0, sa, ea, sc, ec);
   if (lane == 0 && elig) issue_stage<CHECK, CF>(a, g0, sa, ea, sc, ec, cc, wst, bars, pol);
   uint32_t phase = 0;  // bit s = parity of stage s's next completion
   for (int64_t g = g0; g < g1; ++g) {
     const int s = (int)(g - g0) & 1;
-    int32_t nsa = 0, nea = 0, nsc = 0, nec = 0, ncb = 0, ncc = 0;
+    int32_t nsa = 0, nea = 0, nsc = 0, nec = 0, ncc = 0;
     bool nelig = false;
     if (g + 1 < g1) {  // prefetch g + 1 into the other stage
       if (g + 2 > win.wb + 31) win.load(a, g, lane);
-      win.get(g + 1, nsa, nea, nsc, nec, ncb, ncc);
+      win.get(g + 1, nsa, nea, nsc, nec, ncc);
       nelig = lean_eligible(a, g + 1, nsa, nea, nsc, nec);
       if (lane == 0 && nelig)
         issue_stage<CHECK, CF>(a, g + 1, nsa, nea, nsc, nec, ncc,
@@ -768,7 +767,7 @@ __global__ void __launch_bounds__(kLeanWarps * 32, ABFT_LEAN_MINB) k_lean(const 
         }
         __syncwarp();
       }
-      group32<CHECK, INJECT, CF>(a, g, sa, ea, sc, ec, cb, st, lane);
+      group32<CHECK, INJECT, CF>(a, g, sa, ea, sc, ec, st, lane);
       __syncwarp();
       fence_proxy_async_smem();  // generic accesses of this stage precede its next bulk write
     }
@@ -776,7 +775,6 @@ __global__ void __launch_bounds__(kLeanWarps * 32, ABFT_LEAN_MINB) k_lean(const 
     ea = nea;
     sc = nsc;
     ec = nec;
-    cb = ncb;
     cc = ncc;
     elig = nelig;
   }
