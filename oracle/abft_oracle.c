@@ -257,33 +257,167 @@ static uint64_t burst_from_words(uint32_t w_start, uint32_t w_len) {
   return m;
 }
 
-/* The XOR mask for the value produced for (round, target, index).
- * List mode: XOR of all plan entries that match.  Rate mode (R13):
- * each produced value is faulty with probability p = min(1, lambda * ops),
- * decided by Philox(ctr = {index lo, index hi, call, round<<8 | target},
- * key = {seed lo, seed hi}): faulty iff out[0] < floor(p * 2^32); then
- * burst start = out[1] & 63 and length from out[2] via T (R12). */
+/* The XOR mask for the value produced for (round, target, index) under an
+ * explicit fault list: XOR of all entries that match (R13, list mode). */
 uint64_t or_fault_mask(const or_inject *inj, int32_t round, int32_t target, int64_t index,
                        int64_t ops) {
-  if (!inj || inj->mode == OR_INJ_NONE) return 0;
-  if (inj->mode == OR_INJ_LIST) {
-    uint64_t m = 0;
-    for (int64_t e = 0; e < inj->n_list; ++e)
-      if (inj->list_round[e] == round && inj->list_target[e] == target &&
-          inj->list_index[e] == index)
-        m ^= inj->list_mask[e];
-    return m;
+  (void)ops;
+  if (!inj || inj->mode != OR_INJ_LIST) return 0;
+  uint64_t m = 0;
+  for (int64_t e = 0; e < inj->n_list; ++e)
+    if (inj->list_round[e] == round && inj->list_target[e] == target &&
+        inj->list_index[e] == index)
+      m ^= inj->list_mask[e];
+  return m;
+}
+
+/* ------------------------------------------------------------------------ */
+/* Rate mode (R13): "we determine the error events from an           */
+/* exponential distribution with an error rate lambda ... 1/lambda [is] the  */
+/* expected number of arithmetic operations between two consecutive error   */
+/* events" -- a Poisson process over the call's arithmetic operations.       */
+/* Op space of one call (per round): y_i owns 2 len_i ops, then t1_k owns    */
+/* 2 n_k ops, then t2_k owns rows-in-block ops (y only when unprotected).    */
+/* It is cut into chunks of CH ops (CH = 2^24 halved while lambda*CH > 4);   */
+/* chunk c holds K ~ Poisson(lambda * len_c) events, K drawn by inversion of */
+/* the CDF table T[k] = floor(2^32 P(K <= k)) with Philox word 0 of counter  */
+/* {c, 0, call, r<<8 | 0x80}; event e in 1..K takes counter {c, e, call,     */
+/* r<<8 | 0x40}: position = c*CH + floor(w0 * len_c / 2^32), burst start =   */
+/* w1 & 63, burst length from w2 (R12).  Events of disabled targets are      */
+/* dropped (thinning).  Output: list entries ordered by (round, op position).*/
+/* ------------------------------------------------------------------------ */
+int64_t or_rate_chunk(double lambda) {
+  int64_t ch = (int64_t)1 << 24;
+  while (ch > 1 && lambda * (double)ch > 4.0) ch /= 2;
+  return ch;
+}
+
+/* Poisson(mu) CDF table; returns its length (last entry = 2^32). */
+int or_poisson_table(double mu, uint64_t *T, int cap) {
+  double p = exp(-mu), cdf = p;
+  int k = 0;
+  for (;;) {
+    double c = cdf < 1.0 ? cdf : 1.0;
+    T[k] = (uint64_t)floor(ldexp(c, 32));
+    if (T[k] >= ((uint64_t)1 << 32) - 1 || k == cap - 1) {
+      T[k] = (uint64_t)1 << 32;
+      return k + 1;
+    }
+    ++k;
+    p = p * mu / (double)k;
+    cdf = cdf + p;
   }
-  if (!(inj->targets & (1u << target))) return 0;
-  double p = inj->lambda * (double)ops;
-  uint64_t thr = p >= 1.0 ? ((uint64_t)1 << 32) : (uint64_t)(p * 4294967296.0);
-  uint32_t ctr[4] = {(uint32_t)(uint64_t)index, (uint32_t)((uint64_t)index >> 32),
-                     (uint32_t)inj->call, ((uint32_t)round << 8) | (uint32_t)target};
+}
+
+/* Fill (round, target, index, mask) lists for rounds 0..max_rounds; returns
+ * the number of events (call with NULL outputs to count). */
+int64_t or_rate_plan(const or_csr *A, int32_t bs, const int32_t *c_row_ptr, int32_t check,
+                     const or_inject *inj, int32_t max_rounds, int32_t *o_round,
+                     int32_t *o_target, int64_t *o_index, uint64_t *o_mask) {
+  int64_t n = A->n, nb = (n + bs - 1) / bs, nnz = A->row_ptr[n];
+  int64_t nnzc = check ? c_row_ptr[nb] : 0;
+  int64_t y_ops = 2 * nnz, t1_ops = check ? 2 * nnzc : 0, t2_ops = check ? n : 0;
+  int64_t ops = y_ops + t1_ops + t2_ops;
+  int64_t ch = or_rate_chunk(inj->lambda);
+  int64_t nch = (ops + ch - 1) / ch;
   uint32_t key[2] = {(uint32_t)inj->seed, (uint32_t)(inj->seed >> 32)};
-  uint32_t w[4];
-  or_philox4x32_10(ctr, key, w);
-  if ((uint64_t)w[0] >= thr) return 0;
-  return burst_from_words(w[1], w[2]);
+  uint64_t Tf[32], Tl[32];  /* mean <= 4 events per chunk: K <= 31 */
+  int nf = or_poisson_table(inj->lambda * (double)ch, Tf, 32);
+  int64_t last = ops - (nch - 1) * ch;
+  int nl = or_poisson_table(inj->lambda * (double)last, Tl, 32);
+  int64_t cnt = 0;
+  int rounds = check ? max_rounds : 0;
+  uint64_t *pos = (uint64_t *)malloc(sizeof(uint64_t) * 32 * 2);
+  for (int32_t r = 0; r <= rounds; ++r)
+    for (int64_t c = 0; c < nch; ++c) {
+      int64_t len = c == nch - 1 ? last : ch;
+      const uint64_t *T = c == nch - 1 ? Tl : Tf;
+      int tn = c == nch - 1 ? nl : nf;
+      uint32_t ctr[4] = {(uint32_t)c, 0u, (uint32_t)inj->call, ((uint32_t)r << 8) | 0x80u};
+      uint32_t w[4];
+      or_philox4x32_10(ctr, key, w);
+      int K = 0;
+      while (K < tn - 1 && (uint64_t)w[0] >= T[K]) ++K;
+      /* events: (position << 16 | e) so equal positions keep event order */
+      for (int e = 1; e <= K; ++e) {
+        uint32_t c2[4] = {(uint32_t)c, (uint32_t)e, (uint32_t)inj->call, ((uint32_t)r << 8) | 0x40u};
+        or_philox4x32_10(c2, key, w);
+        uint64_t off = ((uint64_t)w[0] * (uint64_t)len) >> 32;
+        pos[2 * (e - 1)] = (off << 16) | (uint64_t)e;
+        pos[2 * (e - 1) + 1] = ((uint64_t)w[1] << 32) | w[2];
+      }
+      /* sort by (offset, e): pairs -- simple insertion sort on the keys */
+      for (int i = 1; i < K; ++i) {
+        uint64_t k0 = pos[2 * i], k1 = pos[2 * i + 1];
+        int j = i - 1;
+        while (j >= 0 && pos[2 * j] > k0) {
+          pos[2 * (j + 1)] = pos[2 * j];
+          pos[2 * (j + 1) + 1] = pos[2 * j + 1];
+          --j;
+        }
+        pos[2 * (j + 1)] = k0;
+        pos[2 * (j + 1) + 1] = k1;
+      }
+      for (int i = 0; i < K; ++i) {
+        int64_t p = c * ch + (int64_t)(pos[2 * i] >> 16);
+        int32_t tgt;
+        int64_t idx;
+        if (p < y_ops) { /* row i with 2 rp[i] <= p < 2 rp[i+1] */
+          int64_t lo = 0, hi = n; /* largest i with 2 rp[i] <= p */
+          while (lo < hi) {
+            int64_t mid = lo + (hi - lo + 1) / 2;
+            if (2 * (int64_t)A->row_ptr[mid] <= p) lo = mid; else hi = mid - 1;
+          }
+          tgt = OR_T_Y;
+          idx = lo;
+        } else if (p < y_ops + t1_ops) {
+          int64_t q = p - y_ops, lo = 0, hi = nb;
+          while (lo < hi) {
+            int64_t mid = lo + (hi - lo + 1) / 2;
+            if (2 * (int64_t)c_row_ptr[mid] <= q) lo = mid; else hi = mid - 1;
+          }
+          tgt = OR_T_T1;
+          idx = lo;
+        } else {
+          tgt = OR_T_T2;
+          idx = (p - y_ops - t1_ops) / bs;
+        }
+        if (!(inj->targets & (1u << tgt))) continue;
+        if (o_round) {
+          uint32_t ws = (uint32_t)(pos[2 * i + 1] >> 32), wl = (uint32_t)pos[2 * i + 1];
+          o_round[cnt] = r;
+          o_target[cnt] = tgt;
+          o_index[cnt] = idx;
+          o_mask[cnt] = burst_from_words(ws, wl);
+        }
+        ++cnt;
+      }
+    }
+  free(pos);
+  return cnt;
+}
+
+/* Expand a rate-mode spec into an explicit list (malloc'd; caller frees). */
+static or_inject rate_to_list(const or_csr *A, int32_t bs, const int32_t *c_row_ptr,
+                              int32_t check, const or_inject *inj, int32_t max_rounds,
+                              void **keep) {
+  or_inject L;
+  memset(&L, 0, sizeof L);
+  L.mode = OR_INJ_LIST;
+  int64_t cnt = or_rate_plan(A, bs, c_row_ptr, check, inj, max_rounds, NULL, NULL, NULL, NULL);
+  size_t m = (size_t)(cnt > 0 ? cnt : 1);
+  char *buf = (char *)malloc(m * (4 + 4 + 8 + 8));
+  int32_t *r = (int32_t *)buf, *t = (int32_t *)(buf + 4 * m);
+  int64_t *ix = (int64_t *)(buf + 8 * m);
+  uint64_t *mk = (uint64_t *)(buf + 16 * m);
+  or_rate_plan(A, bs, c_row_ptr, check, inj, max_rounds, r, t, ix, mk);
+  L.n_list = cnt;
+  L.list_round = r;
+  L.list_target = t;
+  L.list_index = ix;
+  L.list_mask = mk;
+  *keep = buf;
+  return L;
 }
 
 static double xor_double(double v, uint64_t m) {
@@ -354,10 +488,17 @@ static int check_block(const or_csr *A, int32_t bs, const int32_t *c_row_ptr,
 }
 
 int or_abft_spmv(const or_csr *A, int32_t bs, const int32_t *c_row_ptr, const int32_t *c_col,
-                 const double *c_val, const double *K, const double *x, const or_inject *inj,
+                 const double *c_val, const double *K, const double *x, const or_inject *inj_in,
                  int32_t max_rounds, double *y, double *y_pre, double *t1, double *t2,
                  double *s, double *beta_out, int32_t *flag_counts, int32_t *flags) {
   int64_t n = A->n, nb = (n + bs - 1) / bs;
+  void *keep = NULL;
+  or_inject lst;
+  const or_inject *inj = inj_in;
+  if (inj_in && inj_in->mode == OR_INJ_RATE) {
+    lst = rate_to_list(A, bs, c_row_ptr, 1, inj_in, max_rounds, &keep);
+    inj = &lst;
+  }
   /* step 2: beta = ||x||_2 = sqrt(PW(x_i^2)) (R10) */
   double *sq = (double *)malloc(sizeof(double) * (size_t)(n > 0 ? n : 1));
   for (int64_t i = 0; i < n; ++i) sq[i] = x[i] * x[i];
@@ -391,6 +532,7 @@ int or_abft_spmv(const or_csr *A, int32_t bs, const int32_t *c_row_ptr, const in
   if (max_rounds > 0 && flag_counts[max_rounds] > 0) rc = -6;
   free(slot);
   free(pres);
+  free(keep);
   return rc;
 }
 
@@ -443,12 +585,15 @@ int or_pcg(const or_csr *A, int32_t bs, const int32_t *c_row_ptr, const int32_t 
       for (int32_t rr = 0; rr < max_rounds; ++rr) stats[3] += fc[rr];                      \
       if (st) stats[4] += 1;                                                               \
     } else {                                                                               \
+      void *keep_ = NULL;                                                                  \
+      or_inject l_ = inj;                                                                  \
+      if (inj.mode == OR_INJ_RATE)                                                         \
+        l_ = rate_to_list(A, bs, c_row_ptr, 0, &inj, 0, &keep_);                            \
       for (int64_t i_ = 0; i_ < n; ++i_) {                                                 \
         double v_ = or_row_dot(A, i_, vin);                                                \
-        yout[i_] = xor_double(v_, or_fault_mask(&inj, 0, OR_T_Y, i_,                       \
-                                                2 * (int64_t)(A->row_ptr[i_ + 1] -          \
-                                                              A->row_ptr[i_])));            \
+        yout[i_] = xor_double(v_, or_fault_mask(&l_, 0, OR_T_Y, i_, 0));                   \
       }                                                                                    \
+      free(keep_);                                                                         \
     }                                                                                      \
     calls++;                                                                               \
   } while (0)

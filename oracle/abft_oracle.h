@@ -70,6 +70,11 @@ void or_philox4x32_10(const uint32_t ctr[4], const uint32_t key[2], uint32_t out
 void or_burst_table(uint64_t T[65]);
 uint64_t or_fault_mask(const or_inject *inj, int32_t round, int32_t target, int64_t index,
                        int64_t ops);
+int64_t or_rate_chunk(double lambda);
+int or_poisson_table(double mu, uint64_t *T, int cap);
+int64_t or_rate_plan(const or_csr *A, int32_t bs, const int32_t *c_row_ptr, int32_t check,
+                     const or_inject *inj, int32_t max_rounds, int32_t *o_round,
+                     int32_t *o_target, int64_t *o_index, uint64_t *o_mask);
 
 /* --- protected SpMV: steps 1-5 of Fig. 1 ---
  * flags: [(max_rounds+1) * nb], round r's sorted flagged blocks at flags + r*nb,

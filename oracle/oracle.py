@@ -63,6 +63,12 @@ def lib():
         L.or_burst_table.argtypes = [P]
         L.or_fault_mask.restype = C.c_uint64
         L.or_fault_mask.argtypes = [P, i32, i32, i64, i64]
+        L.or_rate_chunk.restype = i64
+        L.or_rate_chunk.argtypes = [d]
+        L.or_poisson_table.restype = C.c_int
+        L.or_poisson_table.argtypes = [d, P, C.c_int]
+        L.or_rate_plan.restype = i64
+        L.or_rate_plan.argtypes = [P, i32, P, i32, P, i32, P, P, P, P]
         L.or_abft_spmv.restype = C.c_int
         L.or_abft_spmv.argtypes = [P, i32, P, P, P, P, P, P, i32, P, P, P, P, P, P, P, P]
         L.or_pcg.restype = C.c_int
@@ -188,6 +194,32 @@ def burst_table() -> np.ndarray:
     t = np.empty(65, dtype=np.uint64)
     lib().or_burst_table(_p(t))
     return t
+
+
+def rate_chunk(lam: float) -> int:
+    return int(lib().or_rate_chunk(lam))
+
+
+def poisson_table(mu: float, cap: int = 1024) -> np.ndarray:
+    t = np.zeros(cap, dtype=np.uint64)
+    k = lib().or_poisson_table(mu, _p(t), cap)
+    return t[:k].copy()
+
+
+def rate_plan(A, enc: "Encoded", inj: Inject, max_rounds: int = 4, check: bool = True):
+    """The explicit fault list a rate-mode spec expands to (R13): arrays
+    (round, target, index, mask) ordered by (round, op position)."""
+    r = _CsrRef(A)
+    s = inj._struct()
+    L = lib()
+    cnt = L.or_rate_plan(r.ref(), enc.bs, _p(enc.row_ptr), 1 if check else 0, C.byref(s),
+                         max_rounds, None, None, None, None)
+    m = max(cnt, 1)
+    ro, ta = np.zeros(m, np.int32), np.zeros(m, np.int32)
+    ix, mk = np.zeros(m, np.int64), np.zeros(m, np.uint64)
+    L.or_rate_plan(r.ref(), enc.bs, _p(enc.row_ptr), 1 if check else 0, C.byref(s), max_rounds,
+                   _p(ro), _p(ta), _p(ix), _p(mk))
+    return ro[:cnt], ta[:cnt], ix[:cnt], mk[:cnt]
 
 
 def fault_mask(inj: Inject, round_: int, target: int, index: int, ops: int) -> int:

@@ -12,7 +12,7 @@ ROOT = os.path.dirname(PKG)
 
 NVCC_FLAGS = [
     "-gencode", "arch=compute_100a,code=sm_100a",
-    "-O3", "-lineinfo", "-std=c++17",
+    "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-ffp-contract=off",
     "-fmad=false",            # no FMA contraction anywhere (R1)
     "-Xcompiler", "-fPIC", "-shared",
     "-cudart", "static",

@@ -79,7 +79,7 @@ struct abft_ctx {
   int correct_grid = 1;
   // scratch
   double *gsum = nullptr;
-  unsigned *done = nullptr;
+  double *bpart = nullptr;   // beta partials (k_finish)
   int32_t *n_cand = nullptr, *cand = nullptr;
   double *cand_s = nullptr;
   int32_t *flags = nullptr, *n_flags = nullptr;
@@ -89,6 +89,12 @@ struct abft_ctx {
   double *dbg_t1 = nullptr, *dbg_t2 = nullptr;
   uint64_t *inj_keys = nullptr, *inj_masks = nullptr;
   int64_t inj_cap = 0;
+  // rate-mode plan scratch
+  int32_t *plan_counts = nullptr, *plan_offs = nullptr, *plan_tot = nullptr, *plan_len = nullptr;
+  uint64_t *plan_tab = nullptr;
+  int64_t plan_slots = 0;
+  double plan_lambda = -1.0;  // the tables on the device belong to (lambda, ops)
+  int64_t plan_ops = -1;
   double *hx = nullptr, *hy = nullptr;  // device staging for abft_spmv_host
   // PCG scratch
   double *pcg = nullptr;  // r, z, p, q, d : 5 n
@@ -144,7 +150,7 @@ SpmvArgs make_args(const abft_ctx *h, const double *x, double *y, const double *
   a.y = y;
   a.x_norm = x_norm;
   a.gsum = h->gsum;
-  a.done = h->done;
+  a.bpart = h->bpart;
   a.n_cand = h->n_cand;
   a.cand = h->cand;
   a.cand_s = h->cand_s;
@@ -158,19 +164,120 @@ SpmvArgs make_args(const abft_ctx *h, const double *x, double *y, const double *
   return a;
 }
 
-// Upload a list-mode fault plan (sorted keys) and fill the device descriptor.
-abft_status prepare_inject(abft_ctx *h, const abft_inject_t *inj, cudaStream_t s, InjDev *d) {
+abft_status ensure_list(abft_ctx *h, int64_t need) {
+  if (need <= h->inj_cap) return ABFT_OK;
+  const int64_t cap = std::max<int64_t>(need, 1024);
+  TRY(dalloc(h, &h->inj_keys, (size_t)cap));
+  TRY(dalloc(h, &h->inj_masks, (size_t)cap));
+  h->inj_cap = cap;
+  return ABFT_OK;
+}
+
+// Rate mode (R13): expand a Poisson process over the call's
+// arithmetic operations into a sorted fault list on the device (no host
+// sync).  The chunking and the CDF tables are computed here exactly as the
+// oracle computes them.
+int64_t rate_chunk(double lambda) {
+  int64_t ch = (int64_t)1 << 24;
+  while (ch > 1 && lambda * (double)ch > 4.0) ch /= 2;
+  return ch;
+}
+
+int poisson_table(double mu, uint64_t *T, int cap) {
+  double p = std::exp(-mu), cdf = p;
+  int k = 0;
+  for (;;) {
+    const double c = cdf < 1.0 ? cdf : 1.0;
+    T[k] = (uint64_t)std::floor(std::ldexp(c, 32));
+    if (T[k] >= ((uint64_t)1 << 32) - 1 || k == cap - 1) {
+      T[k] = (uint64_t)1 << 32;
+      return k + 1;
+    }
+    ++k;
+    p = p * mu / (double)k;
+    cdf = cdf + p;
+  }
+}
+
+abft_status gen_rate_plan(abft_ctx *h, const abft_inject_t *inj, uint64_t call, bool check,
+                          cudaStream_t s, InjDev *d) {
+  RatePlanArgs r;
+  memset(&r, 0, sizeof r);
+  r.n = h->n;
+  r.nb = h->nb;
+  r.bs = h->bs;
+  r.y_ops = 2 * h->nnz;
+  r.t1_ops = check ? 2 * h->nnz_c : 0;
+  r.ops = r.y_ops + r.t1_ops + (check ? h->n : 0);
+  r.rounds = check ? h->max_rounds : 0;
+  r.ch = rate_chunk(inj->lambda);
+  r.nch = std::max<int64_t>(1, (r.ops + r.ch - 1) / r.ch);
+  r.key0 = (uint32_t)inj->seed;
+  r.key1 = (uint32_t)(inj->seed >> 32);
+  r.call = (uint32_t)call;
+  r.targets = inj->targets;
+  r.rp = h->rp;
+  r.crp = h->c_rp;
+  uint64_t tab[2 * kRateTab];
+  r.nf = poisson_table(inj->lambda * (double)r.ch, tab, kRateTab);
+  r.nl = poisson_table(inj->lambda * (double)(r.ops - (r.nch - 1) * r.ch), tab + kRateTab, kRateTab);
+  const int64_t slots = (int64_t)(r.rounds + 1) * r.nch;
+  if (slots > (1ll << 30)) return ABFT_EINVAL;
+  if (slots > h->plan_slots) {
+    const int64_t m = std::max<int64_t>(slots, 4096);
+    TRY(dalloc(h, &h->plan_counts, (size_t)m));
+    TRY(dalloc(h, &h->plan_offs, (size_t)m + 1));
+    TRY(dalloc(h, &h->plan_tot, (size_t)(m + 1023) / 1024 + 1));
+    h->plan_slots = m;
+  }
+  if (!h->plan_tab) {
+    TRY(dalloc(h, &h->plan_tab, 2 * kRateTab));
+    TRY(dalloc(h, &h->plan_len, 1));
+  }
+  // expected events + a wide margin; a longer list is truncated (never seen)
+  const double mean = inj->lambda * (double)r.ops * (double)(r.rounds + 1);
+  const int64_t cap = std::min<int64_t>(slots * (kRateTab - 1),
+                                        (int64_t)(mean + 16.0 * std::sqrt(mean)) + 4096);
+  TRY(ensure_list(h, cap));
+  if (h->plan_lambda != inj->lambda || h->plan_ops != r.ops) {
+    // pageable upload synchronises the stream: only when the tables change
+    CK(cudaMemcpyAsync(h->plan_tab, tab, sizeof tab, cudaMemcpyHostToDevice, s));
+    h->plan_lambda = inj->lambda;
+    h->plan_ops = r.ops;
+  }
+  r.tab = h->plan_tab;
+  r.counts = h->plan_counts;
+  r.offs = h->plan_offs;
+  r.keys = h->inj_keys;
+  r.masks = h->inj_masks;
+  r.cap = cap;
+  const unsigned grid = (unsigned)((slots + 127) / 128);
+  k_rate_plan<false><<<grid, 128, 0, s>>>(r);
+  const int64_t nscan = (slots + 1023) / 1024;
+  k_scan_local<<<(unsigned)nscan, 1024, 0, s>>>(h->plan_counts, h->plan_offs, slots, h->plan_tot);
+  k_scan_totals<<<1, 1024, 0, s>>>(h->plan_tot, nscan, h->plan_len);
+  k_scan_add<<<(unsigned)nscan, 1024, 0, s>>>(h->plan_offs, slots, h->plan_tot);
+  k_rate_plan<true><<<grid, 128, 0, s>>>(r);
+  CK(cudaGetLastError());
+  d->mode = 1;
+  d->n_list = 0;
+  d->n_list_dev = h->plan_len;
+  d->cap = (int32_t)std::min<int64_t>(cap, INT32_MAX);
+  d->keys = h->inj_keys;
+  d->masks = h->inj_masks;
+  return ABFT_OK;
+}
+
+// Fill the device descriptor: upload a list-mode plan (sorted keys), or
+// generate the rate-mode plan of call inj->call.
+abft_status prepare_inject(abft_ctx *h, const abft_inject_t *inj, bool check, cudaStream_t s,
+                           InjDev *d) {
   memset(d, 0, sizeof *d);
   if (!inj || inj->mode == ABFT_INJ_NONE) return ABFT_OK;
   if (inj->mode == ABFT_INJ_RATE) {
-    if (!(inj->lambda >= 0.0)) return ABFT_EINVAL;
-    d->mode = 2;
-    d->key0 = (uint32_t)inj->seed;
-    d->key1 = (uint32_t)(inj->seed >> 32);
-    d->call = (uint32_t)inj->call;
-    d->lambda = inj->lambda;
-    d->targets = inj->targets;
-    return ABFT_OK;
+    if (!(inj->lambda >= 0.0) || !(inj->lambda <= 1.0)) return ABFT_EINVAL;
+    if (inj->lambda == 0.0) return ABFT_OK;  // no events: the fault-free kernels
+    return gen_rate_plan(h, inj, inj->call, check, s, d);
   }
   if (inj->mode != ABFT_INJ_LIST) return ABFT_EINVAL;
   if (inj->n_list < 0 || inj->n_list > (1 << 30)) return ABFT_EINVAL;
@@ -189,12 +296,7 @@ abft_status prepare_inject(abft_ctx *h, const abft_inject_t *inj, cudaStream_t s
   }
   std::sort(kv.begin(), kv.end(),
             [](const auto &p, const auto &q) { return p.first < q.first; });
-  if (inj->n_list > h->inj_cap) {
-    int64_t cap = std::max<int64_t>(inj->n_list, 1024);
-    TRY(dalloc(h, &h->inj_keys, (size_t)cap));
-    TRY(dalloc(h, &h->inj_masks, (size_t)cap));
-    h->inj_cap = cap;
-  }
+  TRY(ensure_list(h, inj->n_list));
   std::vector<uint64_t> keys(kv.size()), masks(kv.size());
   for (size_t e = 0; e < kv.size(); ++e) {
     keys[e] = kv[e].first;
@@ -232,7 +334,6 @@ abft_status launch_fused_t(const abft_ctx *h, SpmvArgs a, cudaStream_t s) {
   a.glist = lean ? h->glist : nullptr;
   a.n_glist = ngen;
   const int ggrid = ngen > 0 ? general_grid(h, ngen) : 0;
-  a.ticket_total = (unsigned)((lean ? h->fused_grid : 0) + ggrid);
   if (lean) launch_lean<CHECK, INJECT>(h, a, s);
   if (ggrid) k_general<CHECK, INJECT><<<ggrid, 256, 0, s>>>(a);
   CK(cudaGetLastError());
@@ -245,9 +346,11 @@ abft_status launch_fused(const abft_ctx *h, const SpmvArgs &a, bool check, cudaS
   return inj ? launch_fused_t<false, true>(h, a, s) : launch_fused_t<false, false>(h, a, s);
 }
 
-// One launch for all correction rounds, as a programmatic dependent launch so
-// its launch latency overlaps the fused kernel (it waits on griddepcontrol).
-abft_status launch_correct(const abft_ctx *h, const SpmvArgs &a, int rounds, cudaStream_t s) {
+// Steps 4-5 in one launch (k_finish), as a programmatic dependent launch so
+// its launch latency overlaps the fused kernels (it waits on griddepcontrol).
+// confirm: turn the fused pass's candidates into round 0's flags first.
+abft_status launch_finish(const abft_ctx *h, const SpmvArgs &a, int rounds, bool confirm,
+                          cudaStream_t s) {
   cudaLaunchConfig_t cfg;
   memset(&cfg, 0, sizeof cfg);
   cfg.gridDim = dim3((unsigned)h->correct_grid);
@@ -259,10 +362,18 @@ abft_status launch_correct(const abft_ctx *h, const SpmvArgs &a, int rounds, cud
   attr[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
-  if (a.inj.mode != 0)
-    CK(cudaLaunchKernelEx(&cfg, k_correct<true>, a, rounds));
-  else
-    CK(cudaLaunchKernelEx(&cfg, k_correct<false>, a, rounds));
+  const bool inj = a.inj.mode != 0;
+  if (confirm) {
+    if (inj)
+      CK(cudaLaunchKernelEx(&cfg, k_finish<true, true>, a, rounds));
+    else
+      CK(cudaLaunchKernelEx(&cfg, k_finish<false, true>, a, rounds));
+  } else {
+    if (inj)
+      CK(cudaLaunchKernelEx(&cfg, k_finish<true, false>, a, rounds));
+    else
+      CK(cudaLaunchKernelEx(&cfg, k_finish<false, false>, a, rounds));
+  }
   return ABFT_OK;
 }
 
@@ -576,7 +687,8 @@ abft_status abft_encode(const abft_csr_t *A, int32_t block_size, int32_t max_rou
   if (!(flags & ABFT_ENCODE_C_CSR) && (st = build_compact_c(h, s)) != ABFT_OK) return fail(st);
 
   // per-call scratch
-  if ((st = dalloc(h, &h->gsum, (size_t)h->ngroups)) || (st = dalloc(h, &h->done, 1)) ||
+  if ((st = dalloc(h, &h->gsum, (size_t)h->ngroups)) ||
+      (st = dalloc(h, &h->bpart, (size_t)(h->ngroups + kBetaChunk - 1) / kBetaChunk)) ||
       (st = dalloc(h, &h->n_cand, 1)) || (st = dalloc(h, &h->cand, (size_t)h->nb)) ||
       (st = dalloc(h, &h->cand_s, (size_t)h->nb)) ||
       (st = dalloc(h, &h->flags, (size_t)(h->max_rounds + 1) * h->nb)) ||
@@ -584,8 +696,7 @@ abft_status abft_encode(const abft_csr_t *A, int32_t block_size, int32_t max_rou
       (st = dalloc(h, &h->beta_valid, 1)) || (st = dalloc(h, &h->gbar, 2)) ||
       (st = dalloc(h, &h->dbg_t1, (size_t)h->nb)) || (st = dalloc(h, &h->dbg_t2, (size_t)h->nb)))
     return fail(st);
-  if ((e = cudaMemsetAsync(h->done, 0, sizeof(unsigned), s)) ||
-      (e = cudaMemsetAsync(h->n_cand, 0, sizeof(int32_t), s)) ||
+  if ((e = cudaMemsetAsync(h->n_cand, 0, sizeof(int32_t), s)) ||
       (e = cudaMemsetAsync(h->n_flags, 0, sizeof(int32_t) * (h->max_rounds + 1), s)) ||
       (e = cudaMemsetAsync(h->beta, 0, sizeof(double), s)) ||
       (e = cudaMemsetAsync(h->beta_valid, 0, sizeof(int32_t), s)) ||
@@ -602,14 +713,14 @@ abft_status abft_spmv(abft_handle_t h, const double *x, double *y, const double 
   if (mode & ~7u) return ABFT_EINVAL;
   cudaStream_t s = (cudaStream_t)stream;
   SpmvArgs a = make_args(h, x, y, x_norm);
-  TRY(prepare_inject(h, inj, s, &a.inj));
   const bool check = (mode & ABFT_CHECK) || (mode & ABFT_AUTOCORRECT);
+  TRY(prepare_inject(h, inj, check, s, &a.inj));
   if (check && (mode & ABFT_DEBUG_CHECKSUMS)) {
     a.dbg_t1 = h->dbg_t1;
     a.dbg_t2 = h->dbg_t2;
   }
   TRY(launch_fused(h, a, check, s));
-  if (mode & ABFT_AUTOCORRECT) TRY(launch_correct(h, a, h->max_rounds, s));
+  if (check) TRY(launch_finish(h, a, (mode & ABFT_AUTOCORRECT) ? h->max_rounds : 0, true, s));
   return ABFT_OK;
 }
 
@@ -620,8 +731,10 @@ abft_status abft_correct(abft_handle_t h, const double *x, double *y, int32_t ma
   if (max_rounds > h->max_rounds) return ABFT_EINVAL;
   cudaStream_t s = (cudaStream_t)stream;
   SpmvArgs a = make_args(h, x, y, nullptr);
-  TRY(prepare_inject(h, inj, s, &a.inj));
-  return launch_correct(h, a, max_rounds, s);
+  // rate mode: the plan of the preceding abft_spmv (same call) is still on
+  // the device; regenerating it is deterministic, so do that for clarity
+  TRY(prepare_inject(h, inj, true, s, &a.inj));
+  return launch_finish(h, a, max_rounds, false, s);
 }
 
 abft_status abft_flags(abft_handle_t h, int32_t round, const int32_t **flagged,
@@ -635,7 +748,7 @@ abft_status abft_flags(abft_handle_t h, int32_t round, const int32_t **flagged,
 abft_status abft_beta(abft_handle_t h, void *stream, const double **beta) {
   if (!h || !beta) return ABFT_EINVAL;
   SpmvArgs a = make_args(h, h->beta, h->beta + 1, nullptr);
-  k_beta<<<1, 1024, 0, (cudaStream_t)stream>>>(a);  // no-op when already valid
+  k_beta<<<1, 256, 0, (cudaStream_t)stream>>>(a);  // no-op when already valid
   CK(cudaGetLastError());
   *beta = h->beta;
   return ABFT_OK;

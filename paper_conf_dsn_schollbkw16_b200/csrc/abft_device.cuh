@@ -111,11 +111,10 @@ __device__ __forceinline__ double ld_x(const double *p) { return __ldg(p); }
 // implemented independently of the oracle.
 // ---------------------------------------------------------------------------
 struct InjDev {
-  int mode;          // 0 none, 1 list, 2 rate
-  uint32_t key0, key1, call;
-  double lambda;
-  uint32_t targets;
-  int32_t n_list;
+  int mode;          // 0 none, 1 list
+  int32_t n_list;    // list length (host-known), or
+  const int32_t *n_list_dev;  // device-resident list length (rate-mode plans)
+  int32_t cap;       // capacity of a device-generated list
   const uint64_t *keys;   // sorted (round << 58) | (target << 56) | index
   const uint64_t *masks;
 };
@@ -142,32 +141,157 @@ __device__ __forceinline__ uint64_t list_key(int round, int target, int64_t inde
   return ((uint64_t)round << 58) | ((uint64_t)target << 56) | (uint64_t)index;
 }
 
+__device__ __forceinline__ int list_len(const InjDev &inj) {
+  return inj.n_list_dev ? min(*inj.n_list_dev, inj.cap) : inj.n_list;
+}
+
+// First list position with key >= k.
+__device__ __forceinline__ int list_lower(const InjDev &inj, int len, uint64_t k) {
+  int lo = 0, hi = len;
+  while (lo < hi) {
+    const int mid = (lo + hi) >> 1;
+    if (__ldg(inj.keys + mid) < k) lo = mid + 1; else hi = mid;
+  }
+  return lo;
+}
+
+// XOR of the masks of entries [lo, hi) whose key equals k.
+__device__ __forceinline__ uint64_t list_mask_in(const InjDev &inj, int lo, int hi, uint64_t k) {
+  uint64_t m = 0;
+  for (int e = lo; e < hi; ++e)
+    if (__ldg(inj.keys + e) == k) m ^= __ldg(inj.masks + e);
+  return m;
+}
+
+// The XOR mask for one produced value (R13): the explicit fault list, or the
+// list a rate-mode spec was expanded to before the launch.
 __device__ __noinline__ uint64_t fault_mask(const InjDev &inj, int round, int target,
                                             int64_t index, int64_t ops) {
-  if (inj.mode == 1) {
-    uint64_t key = list_key(round, target, index);
-    int lo = 0, hi = inj.n_list;
-    while (lo < hi) {
-      int mid = (lo + hi) >> 1;
-      if (inj.keys[mid] < key) lo = mid + 1; else hi = mid;
+  (void)ops;
+  if (inj.mode != 1) return 0;
+  const int len = list_len(inj);
+  if (len == 0) return 0;
+  const uint64_t key = list_key(round, target, index);
+  const int lo = list_lower(inj, len, key);
+  uint64_t m = 0;
+  for (int e = lo; e < len && __ldg(inj.keys + e) == key; ++e) m ^= __ldg(inj.masks + e);
+  return m;
+}
+
+// Per-warp y-fault masks for rows r0 .. r0+31: one pair of binary searches
+// for the group (lane 0), then each lane scans the (usually empty) range.
+__device__ __forceinline__ uint64_t group_y_mask(const InjDev &inj, int round, int64_t r0,
+                                                 int64_t i, int lane) {
+  int lo = 0, hi = 0;
+  if (lane == 0) {
+    const int len = list_len(inj);
+    if (len > 0) {
+      lo = list_lower(inj, len, list_key(round, 0, r0));
+      hi = list_lower(inj, len, list_key(round, 0, r0 + 32));
     }
-    uint64_t m = 0;
-    for (int e = lo; e < inj.n_list && inj.keys[e] == key; ++e) m ^= inj.masks[e];
-    return m;
   }
-  if (inj.mode != 2 || !(inj.targets & (1u << target))) return 0;
-  double p = dmul(inj.lambda, (double)ops);
-  uint64_t thr = p >= 1.0 ? (1ull << 32) : __double2ull_rz(dmul(p, 4294967296.0));
-  uint32_t c[4] = {(uint32_t)(uint64_t)index, (uint32_t)((uint64_t)index >> 32), inj.call,
-                   ((uint32_t)round << 8) | (uint32_t)target};
-  philox10(c, inj.key0, inj.key1);
-  if ((uint64_t)c[0] >= thr) return 0;
-  int start = (int)(c[1] & 63u);
-  int len = 1;
-  while (len < 64 && (uint64_t)c[2] >= c_burst_T[len]) ++len;
-  int hi = min(start + len - 1, 63);
-  uint64_t span = (hi - start + 1) == 64 ? ~0ull : ((1ull << (hi - start + 1)) - 1ull);
-  return span << start;
+  lo = __shfl_sync(0xffffffffu, lo, 0);
+  hi = __shfl_sync(0xffffffffu, hi, 0);
+  return lo < hi ? list_mask_in(inj, lo, hi, list_key(round, 0, i)) : 0ull;
+}
+
+// ---------------------------------------------------------------------------
+// Rate mode (R13): a Poisson process over the call's
+// arithmetic operations, generated as an explicit sorted fault list.
+// Op space per round: y_i owns 2 len_i ops, then t1_k 2 n_k, then t2_k
+// rows-in-block (y only when unprotected).  Chunks of ch ops; chunk c holds
+// K ~ Poisson(lambda len_c) events (inversion of a host-computed CDF table,
+// Philox word 0 of {c, 0, call, r<<8 | 0x80}); event e (1..K) takes Philox
+// {c, e, call, r<<8 | 0x40}: offset floor(w0 len_c / 2^32), burst from w1, w2.
+// One thread per (round, chunk); pass 1 counts the kept events, pass 2
+// writes them (ordered by offset) at the scanned positions.
+// ---------------------------------------------------------------------------
+constexpr int kRateTab = 32;  // table length cap: at most 31 events per chunk
+
+struct RatePlanArgs {
+  int64_t n, nb, ch, nch, y_ops, t1_ops, ops;
+  int32_t bs, rounds;
+  uint32_t key0, key1, call, targets;
+  const int32_t *rp;
+  const int32_t *crp;
+  const uint64_t *tab;  // [2][kRateTab]: full chunks, last chunk
+  int32_t nf, nl;
+  int32_t *counts;      // [(rounds+1) * nch]
+  const int32_t *offs;  // exclusive scan of counts
+  uint64_t *keys, *masks;
+  int64_t cap;          // capacity of keys/masks
+};
+
+template <bool WRITE>
+__global__ void k_rate_plan(const RatePlanArgs a) {
+  const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (tid >= (int64_t)(a.rounds + 1) * a.nch) return;
+  const int r = (int)(tid / a.nch);
+  const int64_t c = tid - (int64_t)r * a.nch;
+  const bool lastc = c == a.nch - 1;
+  const int64_t len = lastc ? a.ops - c * a.ch : a.ch;
+  const uint64_t *T = a.tab + (lastc ? kRateTab : 0);
+  const int tn = lastc ? a.nl : a.nf;
+  uint32_t w[4] = {(uint32_t)c, 0u, a.call, ((uint32_t)r << 8) | 0x80u};
+  philox10(w, a.key0, a.key1);
+  int K = 0;
+  while (K < tn - 1 && (uint64_t)w[0] >= T[K]) ++K;
+  uint64_t ev[kRateTab], pay[kRateTab];
+  for (int e = 1; e <= K; ++e) {
+    uint32_t q[4] = {(uint32_t)c, (uint32_t)e, a.call, ((uint32_t)r << 8) | 0x40u};
+    philox10(q, a.key0, a.key1);
+    const uint64_t off = ((uint64_t)q[0] * (uint64_t)len) >> 32;
+    uint64_t k0 = (off << 16) | (uint64_t)e, k1 = ((uint64_t)q[1] << 32) | q[2];
+    int j = e - 2;  // insertion sort by (offset, e)
+    while (j >= 0 && ev[j] > k0) {
+      ev[j + 1] = ev[j];
+      pay[j + 1] = pay[j];
+      --j;
+    }
+    ev[j + 1] = k0;
+    pay[j + 1] = k1;
+  }
+  int kept = 0;
+  const int64_t base = WRITE ? a.offs[tid] : 0;
+  for (int e = 0; e < K; ++e) {
+    const int64_t p = c * a.ch + (int64_t)(ev[e] >> 16);
+    int tgt;
+    int64_t idx;
+    if (p < a.y_ops) {  // largest row i with 2 rp[i] <= p
+      int64_t lo = 0, hi = a.n;
+      while (lo < hi) {
+        const int64_t mid = lo + (hi - lo + 1) / 2;
+        if (2 * (int64_t)a.rp[mid] <= p) lo = mid; else hi = mid - 1;
+      }
+      tgt = 0;
+      idx = lo;
+    } else if (p < a.y_ops + a.t1_ops) {
+      const int64_t qq = p - a.y_ops;
+      int64_t lo = 0, hi = a.nb;
+      while (lo < hi) {
+        const int64_t mid = lo + (hi - lo + 1) / 2;
+        if (2 * (int64_t)a.crp[mid] <= qq) lo = mid; else hi = mid - 1;
+      }
+      tgt = 1;
+      idx = lo;
+    } else {
+      tgt = 2;
+      idx = (p - a.y_ops - a.t1_ops) / a.bs;
+    }
+    if (!(a.targets & (1u << tgt))) continue;
+    if (WRITE && base + kept < a.cap) {
+      const uint32_t ws = (uint32_t)(pay[e] >> 32), wl = (uint32_t)pay[e];
+      const int start = (int)(ws & 63u);
+      int blen = 1;
+      while (blen < 64 && (uint64_t)wl >= c_burst_T[blen]) ++blen;
+      const int hib = min(start + blen - 1, 63);
+      const uint64_t span = (hib - start + 1) == 64 ? ~0ull : ((1ull << (hib - start + 1)) - 1ull);
+      a.keys[base + kept] = list_key(r, tgt, idx);
+      a.masks[base + kept] = span << start;
+    }
+    ++kept;
+  }
+  if (!WRITE) a.counts[tid] = kept;
 }
 
 __device__ __forceinline__ double apply_mask(double v, uint64_t m) {

@@ -1,5 +1,5 @@
 // kernels_pcg.cuh -- Jacobi-PCG vector kernels (SVI-A; Saad
-// Alg. 9.1).  The SpMV q = A p is the protected k_lean/k_general/k_correct
+// Alg. 9.1).  The SpMV q = A p is the protected k_lean/k_general/k_finish
 // set; these kernels fuse the vector updates with their dot products.
 //
 // Every dot is PW over the global index (R2): a CTA owns an aligned chunk of

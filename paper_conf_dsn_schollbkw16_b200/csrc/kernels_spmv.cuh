@@ -25,10 +25,10 @@
 // k_general: every group k_lean cannot take (b_s < 32, the ragged last group,
 // segments beyond the staging capacity, unaligned operands) -- one warp per
 // group, operands read directly from global memory.
-// Both kernels share one completion ticket: the last CTA to finish confirms
-// the candidates against tau_k = K_k beta with beta = sqrt(PW(gsum)) --
-// computed only when a candidate exists (or taken from x_norm) -- and writes
-// the flagged-block list.
+// k_finish (one PDL launch after them) confirms the candidates against
+// tau_k = K_k beta, beta = sqrt(PW(gsum)) computed by all SMs only when a
+// candidate exists (or taken from x_norm), writes the flagged-block list and
+// runs the correction rounds.
 #pragma once
 #include "abft_device.cuh"
 #include "bulk.cuh"
@@ -78,9 +78,8 @@ struct SpmvArgs {
   double *__restrict__ y;
   const double *x_norm;   // nullable device scalar
   double *gsum;           // [ngroups] x^2 subtree of each group
-  unsigned *done;         // completion ticket (reset by the last CTA)
-  unsigned ticket_total;  // CTAs of all kernels of this call
-  int32_t *n_cand;        // candidate count (reset by the last CTA)
+  double *bpart;          // [ceil(ngroups / 1024)] beta partials (k_finish)
+  int32_t *n_cand;        // candidate count (reset by k_finish)
   int32_t *cand;          // [nb]
   double *cand_s;         // [nb]
   int32_t *flags;         // [(max_rounds+1) * nb]; round r at flags + r*nb
@@ -275,57 +274,6 @@ __device__ __forceinline__ void test_block_lo(const SpmvArgs &a, int64_t k, doub
   }
 }
 
-// Last CTA of the call (ticket over a.ticket_total CTAs): beta, confirm the
-// candidates against tau_k = K_k beta, write round 0's flag list.
-__device__ __forceinline__ void finalize_ticket(const SpmvArgs &a, double *s_red, int *s_flag) {
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    __threadfence();
-    const unsigned t = atomicAdd(a.done, 1u);
-    s_flag[0] = (t == a.ticket_total - 1);
-    s_flag[1] = 0;
-  }
-  __syncthreads();
-  if (!s_flag[0]) return;
-  __threadfence();
-  const int nthr = blockDim.x;
-  const int nc = __ldcg(a.n_cand);
-  double beta = 0.0;
-  if (a.x_norm) {
-    beta = __ldcg(a.x_norm);
-  } else if (nc > 0) {
-    // beta = sqrt(PW over the group subtrees) (R10)
-    int64_t m = 1;
-    while (m * nthr < a.ngroups) m <<= 1;
-    PwSeq acc;
-    const int64_t b = (int64_t)threadIdx.x * m;
-    for (int64_t q = b; q < min64(b + m, a.ngroups); ++q) acc.push(__ldcg(a.gsum + q));
-    s_red[threadIdx.x] = acc.finish();
-    __syncthreads();
-    for (int st = 1; st < nthr; st <<= 1) {
-      if ((threadIdx.x & (2 * st - 1)) == 0 && threadIdx.x + st < nthr)
-        s_red[threadIdx.x] = dadd(s_red[threadIdx.x], s_red[threadIdx.x + st]);
-      __syncthreads();
-    }
-    beta = __dsqrt_rn(s_red[0]);
-  }
-  for (int q = threadIdx.x; q < nc; q += nthr) {
-    const int32_t kk = __ldcg(a.cand + q);
-    const double s = __ldcg(a.cand_s + q);
-    const double tau = dmul(__ldg(a.K + kk), beta);  // tau_k = K_k * beta
-    if (!(fabs(s) <= tau)) a.flags[atomicAdd(&s_flag[1], 1)] = kk;
-  }
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    *a.beta = beta;
-    *a.beta_valid = (a.x_norm || nc > 0) ? 1 : 0;
-    a.n_flags[0] = s_flag[1];
-    for (int r = 1; r <= a.max_rounds; ++r) a.n_flags[r] = 0;
-    *a.n_cand = 0;
-    *a.done = 0u;
-  }
-}
-
 // ---------------------------------------------------------------------------
 // General path: one group, operands from global memory (any b_s <= 32).
 // ---------------------------------------------------------------------------
@@ -358,7 +306,10 @@ __device__ __forceinline__ void group_general(const SpmvArgs &a, int64_t g, int 
     }
   }
   if (len == 0) yv = 0.0;  // PW of an empty row is +0.0 (R2)
-  if (INJECT && valid) yv = apply_mask(yv, fault_mask(a.inj, 0, 0, i, 2 * (int64_t)len));
+  if (INJECT) {
+    const uint64_t m = group_y_mask(a.inj, 0, r0, i, lane);
+    if (valid) yv = apply_mask(yv, m);
+  }
   if (valid) a.y[i] = yv;
   if (!CHECK) return;
 
@@ -407,8 +358,6 @@ __device__ __forceinline__ void group_general(const SpmvArgs &a, int64_t g, int 
 
 template <bool CHECK, bool INJECT>
 __global__ void __launch_bounds__(256) k_general(const SpmvArgs a) {
-  __shared__ double s_red[256];
-  __shared__ int s_flag[2];
   if (skip_call(a)) return;
   const int lane = threadIdx.x & 31;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -417,7 +366,6 @@ __global__ void __launch_bounds__(256) k_general(const SpmvArgs a) {
     const int64_t g = a.glist ? (int64_t)__ldg(a.glist + q) : q;
     group_general<CHECK, INJECT>(a, g, lane);
   }
-  if (CHECK) finalize_ticket(a, s_red, s_flag);
 }
 
 // ---------------------------------------------------------------------------
@@ -464,9 +412,40 @@ __device__ __forceinline__ void load8(double (&v)[8], const unsigned char *p) {
 // 8 consecutive products e = 8l..8l+7 without bank conflicts.
 __device__ __forceinline__ int cpad(int e) { return e + (e >> 3); }
 
+// Fault-list ranges of a warp's contiguous group range (INJECT only): list
+// positions [y0, y1) hold the y faults of its rows, [k0, k1) / [q0, q1) the
+// t1 / t2 faults of its blocks (round 0).
+struct InjRange {
+  int y0, y1, k0, k1, q0, q1;
+};
+
+__device__ __forceinline__ InjRange inj_range(const InjDev &inj, int64_t g0, int64_t g1,
+                                              int lane) {
+  InjRange R{0, 0, 0, 0, 0, 0};
+  if (lane == 0 && inj.mode == 1) {
+    const int len = list_len(inj);
+    if (len > 0) {
+      R.y0 = list_lower(inj, len, list_key(0, 0, g0 * 32));
+      R.y1 = list_lower(inj, len, list_key(0, 0, g1 * 32));
+      R.k0 = list_lower(inj, len, list_key(0, 1, g0));
+      R.k1 = list_lower(inj, len, list_key(0, 1, g1));
+      R.q0 = list_lower(inj, len, list_key(0, 2, g0));
+      R.q1 = list_lower(inj, len, list_key(0, 2, g1));
+    }
+  }
+  R.y0 = __shfl_sync(kFull, R.y0, 0);
+  R.y1 = __shfl_sync(kFull, R.y1, 0);
+  R.k0 = __shfl_sync(kFull, R.k0, 0);
+  R.k1 = __shfl_sync(kFull, R.k1, 0);
+  R.q0 = __shfl_sync(kFull, R.q0, 0);
+  R.q1 = __shfl_sync(kFull, R.q1, 0);
+  return R;
+}
+
 template <bool CHECK, bool INJECT, int CF>
 __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa, int32_t ea,
-                                        int32_t sc, int32_t ec, unsigned char *st, int lane) {
+                                        int32_t sc, int32_t ec, unsigned char *st, int lane,
+                                        const InjRange &R) {
   using CT = typename CType<CF>::T;
   const StageCfg &c = a.sc;
   const int64_t i = g * 32 + lane;
@@ -566,7 +545,7 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
     }
   }
   if (len == 0) yv = 0.0;  // PW of an empty row is +0.0 (R2)
-  if (INJECT) yv = apply_mask(yv, fault_mask(a.inj, 0, 0, i, 2 * (int64_t)len));
+  if (INJECT && R.y0 < R.y1) yv = apply_mask(yv, list_mask_in(a.inj, R.y0, R.y1, list_key(0, 0, i)));
   a.y[i] = yv;
   if (!CHECK) return;
 
@@ -623,8 +602,8 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
   }
   double t1 = nC > 0 ? tree<4>(q) : 0.0;
   if (INJECT && lane == 0) {
-    t1 = apply_mask(t1, fault_mask(a.inj, 0, 1, g, 2 * (int64_t)nC));
-    t2 = apply_mask(t2, fault_mask(a.inj, 0, 2, g, 32));
+    if (R.k0 < R.k1) t1 = apply_mask(t1, list_mask_in(a.inj, R.k0, R.k1, list_key(0, 1, g)));
+    if (R.q0 < R.q1) t2 = apply_mask(t2, list_mask_in(a.inj, R.q0, R.q1, list_key(0, 2, g)));
   }
   if (lane == 0 && a.dbg_t1) {
     a.dbg_t1[g] = t1;
@@ -713,8 +692,6 @@ __device__ __forceinline__ void issue_stage(const SpmvArgs &a, int64_t g, int32_
 template <bool CHECK, bool INJECT, int CF>
 __global__ void __launch_bounds__(kLeanWarps * 32, ABFT_LEAN_MINB) k_lean(const SpmvArgs a) {
   extern __shared__ __align__(128) unsigned char smem[];
-  __shared__ double s_red[kLeanWarps * 32];
-  __shared__ int s_flag[2];
   if (skip_call(a)) return;
   const StageCfg &c = a.sc;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -730,10 +707,9 @@ __global__ void __launch_bounds__(kLeanWarps * 32, ABFT_LEAN_MINB) k_lean(const 
   const int64_t tw = (int64_t)gridDim.x * c.warps;
   const int64_t gw = (int64_t)blockIdx.x * c.warps + warp;
   const int64_t g0 = gw * a.ngroups / tw, g1 = (gw + 1) * a.ngroups / tw;
-  if (g0 >= g1) {
-    if (CHECK) finalize_ticket(a, s_red, s_flag);
-    return;
-  }
+  if (g0 >= g1) return;
+  InjRange R{0, 0, 0, 0, 0, 0};
+  if (INJECT) R = inj_range(a.inj, g0, g1, lane);
   Window<CF> win;
   win.load(a, g0, lane);
   int32_t sa, ea, sc, ec, cc;  // bounds of the current group, carried from its prefetch
@@ -767,7 +743,7 @@ __global__ void __launch_bounds__(kLeanWarps * 32, ABFT_LEAN_MINB) k_lean(const 
         }
         __syncwarp();
       }
-      group32<CHECK, INJECT, CF>(a, g, sa, ea, sc, ec, st, lane);
+      group32<CHECK, INJECT, CF>(a, g, sa, ea, sc, ec, st, lane, R);
       __syncwarp();
       fence_proxy_async_smem();  // generic accesses of this stage precede its next bulk write
     }
@@ -778,7 +754,6 @@ __global__ void __launch_bounds__(kLeanWarps * 32, ABFT_LEAN_MINB) k_lean(const 
     cc = ncc;
     elig = nelig;
   }
-  if (CHECK) finalize_ticket(a, s_red, s_flag);
 }
 
 // Encode-time helper: the groups k_lean does not take (appended, unordered).
@@ -791,24 +766,50 @@ __global__ void k_glist(const SpmvArgs a, int32_t *glist, int32_t *count) {
   }
 }
 
-// beta on demand (abft_beta): PW over the group subtrees, one CTA.
-__global__ void __launch_bounds__(1024) k_beta(const SpmvArgs a) {
-  __shared__ double s_red[1024];
-  if (*(volatile int32_t *)a.beta_valid) return;
+// PW over n doubles at p by one CTA of 256 threads: thread t owns an aligned
+// run of m = 2^k values, reduced 32 at a time in registers (32 loads in
+// flight), runs by a shared-memory tree.  Called by all threads.
+__device__ __forceinline__ double cta_pw_array(const double *p, int64_t n, double *s_red) {
+  constexpr int T = 256;
   int64_t m = 1;
-  while (m * 1024 < a.ngroups) m <<= 1;
-  PwSeq acc;
+  while (m * T < n) m <<= 1;
   const int64_t b = (int64_t)threadIdx.x * m;
-  for (int64_t q = b; q < min64(b + m, a.ngroups); ++q) acc.push(__ldcg(a.gsum + q));
-  s_red[threadIdx.x] = acc.finish();
+  double acc = kAbsent;
+  if (m <= 32) {
+    double v[32];
+#pragma unroll
+    for (int q = 0; q < 32; ++q) v[q] = (q < m && b + q < n) ? __ldcg(p + b + q) : kAbsent;
+    acc = tree<32>(v);
+  } else {
+    PwSeq sub;  // runs of 32 (aligned nodes), combined by the binary counter
+    for (int64_t o = 0; o < m && b + o < n; o += 32) {
+      double v[32];
+#pragma unroll
+      for (int q = 0; q < 32; ++q) v[q] = (b + o + q < n) ? __ldcg(p + b + o + q) : kAbsent;
+      sub.push(tree<32>(v));
+    }
+    acc = sub.finish();
+  }
   __syncthreads();
-  for (int st = 1; st < 1024; st <<= 1) {
+  s_red[threadIdx.x] = acc;
+  __syncthreads();
+  for (int st = 1; st < T; st <<= 1) {
     if ((threadIdx.x & (2 * st - 1)) == 0)
       s_red[threadIdx.x] = dadd(s_red[threadIdx.x], s_red[threadIdx.x + st]);
     __syncthreads();
   }
+  const double r = s_red[0];
+  __syncthreads();
+  return r;
+}
+
+// beta on demand (abft_beta): PW over the group subtrees, one CTA.
+__global__ void __launch_bounds__(256) k_beta(const SpmvArgs a) {
+  __shared__ double s_red[256];
+  if (*(volatile int32_t *)a.beta_valid) return;
+  const double b2 = cta_pw_array(a.gsum, a.ngroups, s_red);
   if (threadIdx.x == 0) {
-    *a.beta = __dsqrt_rn(s_red[0]);
+    *a.beta = __dsqrt_rn(b2);
     *a.beta_valid = 1;
   }
 }
@@ -832,17 +833,68 @@ __device__ __forceinline__ void grid_sync(unsigned *bar) {
   __syncthreads();
 }
 
-// Step 5, all rounds in one launch: round r recomputes the rows
-// of every block in round (r-1)'s list, recomputes t1/t2 and re-checks;
-// survivors form round r's list.  One warp per flagged block, grid-stride;
-// rounds separated by a grid barrier.  Launched as a programmatic dependent
-// launch: its launch latency overlaps the fused kernels.
-template <bool INJECT>
-__global__ void __launch_bounds__(256) k_correct(const SpmvArgs a, int rounds) {
+constexpr int kBetaChunk = 1024;  // groups per aligned beta partial (k_finish)
+
+// Steps 4-5 after the fused pass, one launch (programmatic dependent launch:
+// its launch latency overlaps the fused kernels; griddepcontrol.wait orders
+// it after them).  One CTA per SM, software grid barrier.
+//  * CONFIRM: if the fused pass left candidates, beta = sqrt(PW(gsum))
+//    (aligned 1024-group partials reduced by all CTAs, then the partials by
+//    every CTA redundantly -- the same bits everywhere), and each candidate
+//    is flagged iff NOT(|s_k| <= K_k beta).  No candidates: flags
+//    are empty and the kernel returns at once.
+//  * rounds r = 1..R (step 5): recompute the rows of the blocks
+//    flagged in round r-1, recompute t1/t2, re-check; survivors form round
+//    r's list.  One warp per flagged block, grid-stride.
+template <bool INJECT, bool CONFIRM>
+__global__ void __launch_bounds__(256) k_finish(const SpmvArgs a, int rounds) {
+  __shared__ double s_red[256];
+  __shared__ double s_beta;
   asm volatile("griddepcontrol.wait;" ::: "memory");
   if (skip_call(a)) return;
-  if (__ldcg(a.n_flags) == 0) return;
   const int lane = threadIdx.x & 31;
+  if (CONFIRM) {
+    const int nc = __ldcg(a.n_cand);
+    if (nc == 0) {
+      if (blockIdx.x == 0 && threadIdx.x == 0) {
+        for (int r = 0; r <= a.max_rounds; ++r) a.n_flags[r] = 0;
+        if (a.x_norm) *a.beta = __ldcg(a.x_norm);
+        *a.beta_valid = a.x_norm ? 1 : 0;
+      }
+      return;
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0)
+      for (int r = 0; r <= a.max_rounds; ++r) a.n_flags[r] = 0;
+    double beta;
+    if (a.x_norm) {
+      beta = __ldcg(a.x_norm);
+    } else {
+      const int64_t nch = (a.ngroups + kBetaChunk - 1) / kBetaChunk;
+      for (int64_t c = blockIdx.x; c < nch; c += gridDim.x) {
+        const double v = cta_pw_array(a.gsum + c * kBetaChunk,
+                                      min64(kBetaChunk, a.ngroups - c * kBetaChunk), s_red);
+        if (threadIdx.x == 0) a.bpart[c] = v;
+      }
+      grid_sync(a.gbar);
+      beta = __dsqrt_rn(cta_pw_array(a.bpart, nch, s_red));  // R10
+    }
+    if (threadIdx.x == 0) s_beta = beta;
+    grid_sync(a.gbar);  // n_flags zeroed, partials consumed
+    beta = s_beta;
+    for (int q = blockIdx.x * blockDim.x + threadIdx.x; q < nc; q += gridDim.x * blockDim.x) {
+      const int32_t kk = __ldcg(a.cand + q);
+      const double sv = __ldcg(a.cand_s + q);
+      const double tau = dmul(__ldg(a.K + kk), beta);  // tau_k = K_k * beta
+      if (!(fabs(sv) <= tau)) a.flags[atomicAdd(a.n_flags, 1)] = kk;
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+      *a.beta = beta;
+      *a.beta_valid = 1;
+    }
+    grid_sync(a.gbar);  // round 0's list complete; every CTA has read n_cand
+    if (blockIdx.x == 0 && threadIdx.x == 0) *a.n_cand = 0;
+  }
+  if (rounds == 0 || __ldcg(a.n_flags) == 0) return;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
   const double beta = __ldcg(a.beta);
@@ -876,7 +928,10 @@ __global__ void __launch_bounds__(256) k_correct(const SpmvArgs a, int rounds) {
         }
       }
       if (len == 0) yv = 0.0;
-      if (INJECT && valid) yv = apply_mask(yv, fault_mask(a.inj, round, 0, i, 2 * (int64_t)len));
+      if (INJECT) {
+        const uint64_t m = group_y_mask(a.inj, round, k << a.log2bs, i, lane);
+        if (valid) yv = apply_mask(yv, m);
+      }
       if (valid) a.y[i] = yv;
       double t2 = bfly32(valid ? yv : kAbsent);
       const int32_t cb = __ldg(a.crp + k), ce = __ldg(a.crp + k + 1);
@@ -886,8 +941,8 @@ __global__ void __launch_bounds__(256) k_correct(const SpmvArgs a, int rounds) {
           t1 = apply_mask(t1, fault_mask(a.inj, round, 1, k, 2 * (int64_t)(ce - cb)));
           t2 = apply_mask(t2, fault_mask(a.inj, round, 2, k, min64(a.bs, n - (k << a.log2bs))));
         }
-        const double s = dsub(t1, t2);
-        if (!(fabs(s) <= dmul(__ldg(a.K + k), beta)))
+        const double sv = dsub(t1, t2);
+        if (!(fabs(sv) <= dmul(__ldg(a.K + k), beta)))
           next[atomicAdd(a.n_flags + round, 1)] = (int32_t)k;
       }
     }

@@ -394,31 +394,77 @@ class TestFaultModel:
         mean = float((np.arange(1, 65) * pmf).sum())
         assert abs(mean - L.mean()) < 5e-3
 
-    def test_rate_mode_frequency(self, O):
-        # lambda = probability that an arithmetic op returns an
-        # erroneous result -> a value produced by `ops` ops is faulty with
-        # probability ~ lambda * ops.  Binomial check.
-        inj = O.Inject.rate(seed=123, lam=1e-3, targets=0b111)
-        hits = sum(O.fault_mask(inj, 0, 0, i, 14) != 0 for i in range(40000))
-        p = 14e-3
-        assert abs(hits - 40000 * p) < 5 * math.sqrt(40000 * p * (1 - p))
-        inj0 = O.Inject.rate(seed=123, lam=0.0)
-        assert all(O.fault_mask(inj0, 0, 0, i, 14) == 0 for i in range(1000))
-        inj1 = O.Inject.rate(seed=123, lam=1.0)
-        assert all(O.fault_mask(inj1, 0, 0, i, 14) != 0 for i in range(1000))
+    def test_poisson_table_vs_scipy(self, O):
+        # R13: K ~ Poisson(mu) by inversion of T[k] = floor(2^32 P(K <= k))
+        from scipy.stats import poisson
+        assert O.poisson_table(0.0).tolist() == [2 ** 32]
+        for mu in [1e-6, 0.5, 3.0, 31.9]:
+            T = O.poisson_table(mu).astype(np.float64)
+            assert T[-1] == 2 ** 32 and np.all(np.diff(T) >= 0)
+            ks = np.arange(len(T) - 1)
+            assert np.max(np.abs(T[:-1] / 2 ** 32 - poisson.cdf(ks, mu))) < 1e-9
 
-    def test_rate_mode_masks_are_bursts(self, O):
-        inj = O.Inject.rate(seed=5, lam=1.0)
-        for i in range(2000):
-            m = O.fault_mask(inj, 1, 2, i, 1)
-            assert m != 0
+    def test_rate_chunk(self, O):
+        assert O.rate_chunk(0.0) == 2 ** 24 and O.rate_chunk(1e-8) == 2 ** 24
+        for lam in [1e-6, 1e-4, 1e-2, 0.5]:
+            ch = O.rate_chunk(lam)
+            assert lam * ch <= 4 and (ch == 1 or lam * ch * 2 > 4)
+
+    def _lap(self, O):
+        A = G.laplacian_3d_7pt(12)
+        return A, O.encode(A, 32)
+
+    def test_rate_plan_is_poisson_process(self, O):
+        # error events form a Poisson process over the arithmetic ops
+        # (exponential gaps, mean 1/lambda): the count per call is
+        # Poisson(lambda * ops), positions are uniform over the ops.
+        A, enc = self._lap(O)
+        ops_y, ops_t1, ops_t2 = 2 * A.nnz, 2 * int(enc.col.size), A.n
+        ops = ops_y + ops_t1 + ops_t2
+        lam = 20.0 / ops
+        counts, tg = [], []
+        for call in range(400):
+            ro, ta, ix, mk = O.rate_plan(A, enc, O.Inject.rate(seed=3, lam=lam, call=call), 0)
+            counts.append(len(ro))
+            tg.extend(ta.tolist())
+        counts = np.array(counts)
+        assert abs(counts.mean() - 20.0) < 5 * math.sqrt(20.0 / 400)
+        assert 0.7 < counts.var() / counts.mean() < 1.3  # Poisson dispersion
+        tg = np.array(tg)
+        for t, o in [(0, ops_y), (1, ops_t1), (2, ops_t2)]:
+            p = o / ops
+            assert abs((tg == t).mean() - p) < 5 * math.sqrt(p * (1 - p) / tg.size)
+
+    def test_rate_plan_elements_weighted_by_ops(self, O):
+        # a row with more entries (more ops) receives proportionally more events
+        A, enc = self._lap(O)
+        lam = 200.0 / (2 * A.nnz)
+        idx = []
+        for call in range(100):
+            ro, ta, ix, mk = O.rate_plan(A, enc, O.Inject.rate(seed=5, lam=lam, call=call, targets=1), 0)
+            assert np.all(ta == 0)
+            idx.extend(ix.tolist())
+        lens = A.row_lengths()
+        hits = np.bincount(np.array(idx), minlength=A.n)
+        for L in (4, 7):  # corner rows (4 entries) vs interior rows (7)
+            sel = lens == L
+            rate = hits[sel].sum() / sel.sum()
+            expect = len(idx) * 2 * L / (2 * A.nnz)
+            assert abs(rate - expect) < 0.15 * expect
+
+    def test_rate_plan_masks_and_rounds(self, O):
+        A, enc = self._lap(O)
+        ro, ta, ix, mk = O.rate_plan(A, enc, O.Inject.rate(seed=1, lam=1e-3, call=2), 3)
+        assert set(np.unique(ro).tolist()) <= {0, 1, 2, 3} and len(ro) > 100
+        key = ro.astype(np.int64) * 4 + ta
+        assert np.all(np.diff(key) >= 0)  # ordered by round, then op position
+        for m in mk.tolist():
             lo = (m & -m).bit_length() - 1
             run = m >> lo
-            assert run & (run + 1) == 0  # contiguous ones
-
-    def test_rate_targets_mask(self, O):
-        inj = O.Inject.rate(seed=5, lam=1.0, targets=0b010)
-        assert O.fault_mask(inj, 0, 0, 3, 1) == 0 and O.fault_mask(inj, 0, 1, 3, 1) != 0
+            assert m != 0 and run & (run + 1) == 0
+        ro0, *_ = O.rate_plan(A, enc, O.Inject.rate(seed=1, lam=1e-3, call=2), 3, check=False)
+        assert np.all(ro0 == 0)
+        assert len(O.rate_plan(A, enc, O.Inject.rate(seed=1, lam=0.0), 3)[0]) == 0
 
 
 # --------------------------------------------------------------------------
