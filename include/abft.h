@@ -48,15 +48,22 @@ typedef enum {
   ABFT_EBREAKDOWN = -7     /* PCG: p.q <= 0 or NaN residual */
 } abft_status;
 
-/* Square CSR matrix, DEVICE arrays. row_ptr[n+1], col_idx[nnz], val[nnz].
+/* CSR matrix, DEVICE arrays. row_ptr[n+1], col_idx[nnz], val[nnz].
  * The caller owns the arrays; they must outlive the handle (correction and
- * PCG re-read A; it is never copied). */
+ * PCG re-read A; it is never copied).
+ * Square (n_cols == 0 or n_cols == n, x_offset == 0), or -- for a row-block
+ * shard of a distributed matrix -- n rows over n_cols >= x_offset + n local
+ * columns: the operand x then has n_cols entries and the shard's own rows'
+ * entries are x[x_offset .. x_offset + n) (halo columns before and after,
+ * numbered in global order so every sum keeps the single-GPU order). */
 typedef struct {
   int64_t n;
   int64_t nnz;
   const int32_t *row_ptr;
   const int32_t *col_idx;
   const double *val;
+  int64_t n_cols;    /* 0 -> n */
+  int64_t x_offset;  /* 0 for a square matrix */
 } abft_csr_t;
 
 typedef struct abft_ctx *abft_handle_t;
@@ -95,7 +102,9 @@ enum {
   ABFT_NOCHECK = 0,          /* plain y = A x (the unprotected baseline) */
   ABFT_CHECK = 1,            /* steps 1-4: y, t1, t2, s, beta, tau, flags */
   ABFT_AUTOCORRECT = 2,      /* + step 5: up to max_rounds correction rounds */
-  ABFT_DEBUG_CHECKSUMS = 4   /* also store t1, t2 per block (abft_debug_checksums) */
+  ABFT_DEBUG_CHECKSUMS = 4,  /* also store t1, t2 per block (abft_debug_checksums) */
+  ABFT_DEFER_FINISH = 8      /* distributed: run steps 1-3 only; beta comes from all
+                                ranks (abft_beta_partial + abft_finish) */
 };
 
 /* Build C (CSR: nb rows, ascending columns = the non-empty columns of A_k,
@@ -139,6 +148,18 @@ abft_status abft_info(abft_handle_t h, abft_info_t *info);
  * (abft_flags); nothing is copied to the host. */
 abft_status abft_spmv(abft_handle_t h, const double *x, double *y, const double *x_norm,
                       const abft_inject_t *inj, uint32_t mode, void *stream);
+
+/* Distributed protected SpMV (row-block shards).  After
+ * abft_spmv(..., mode | ABFT_DEFER_FINISH), abft_beta_partial enqueues the
+ * PW of this shard's sum of x_i^2 over its own rows into the caller's device
+ * scalar *partial.  Gather the partials of all ranks in rank order (e.g. an NCCL
+ * all-gather) into a device array and call abft_finish: beta =
+ * sqrt(PW(parts)) -- bit-identical to the single-GPU beta when every shard
+ * owns an aligned power-of-two row range -- then step 4 (flags) and up to
+ * `rounds` correction rounds (step 5). */
+abft_status abft_beta_partial(abft_handle_t h, double *partial, void *stream);
+abft_status abft_finish(abft_handle_t h, const double *x, double *y, const double *parts,
+                        int32_t nparts, int32_t rounds, const abft_inject_t *inj, void *stream);
 
 /* Step 5 alone: rounds r = 1..max_rounds recompute the rows of
  * the blocks flagged in round r-1, recompute t1/t2 and re-check; blocks that

@@ -18,14 +18,14 @@ from . import _build
 _LIB = None
 
 OK, EINVAL, ECUDA, ENOMEM, ENOTSUP, ENOCONV, EUNCORRECTED, EBREAKDOWN = 0, -1, -2, -3, -4, -5, -6, -7
-NOCHECK, CHECK, AUTOCORRECT, DEBUG_CHECKSUMS = 0, 1, 2, 4
+NOCHECK, CHECK, AUTOCORRECT, DEBUG_CHECKSUMS, DEFER_FINISH = 0, 1, 2, 4, 8
 INJ_NONE, INJ_LIST, INJ_RATE = 0, 1, 2
 
 SYMBOLS = [
     "abft_encode", "abft_spmv", "abft_correct", "abft_flags", "abft_beta",
     "abft_checksum_matrix", "abft_debug_checksums", "abft_spmv_host", "abft_pcg",
     "abft_destroy", "abft_memcpy", "abft_status_string", "abft_last_cuda_error",
-    "abft_burst_table", "abft_version", "abft_info",
+    "abft_burst_table", "abft_version", "abft_info", "abft_beta_partial", "abft_finish",
 ]
 ENCODE_C_CSR = 1
 CFMT_NAMES = {0: "csr-f64", 1: "int8+u16", 2: "int16+u16", 3: "f32+u16", 4: "f64+u16"}
@@ -42,7 +42,8 @@ class AbftError(RuntimeError):
 
 class _Csr(C.Structure):
     _fields_ = [("n", C.c_int64), ("nnz", C.c_int64), ("row_ptr", C.c_void_p),
-                ("col_idx", C.c_void_p), ("val", C.c_void_p)]
+                ("col_idx", C.c_void_p), ("val", C.c_void_p), ("n_cols", C.c_int64),
+                ("x_offset", C.c_int64)]
 
 
 class _Inj(C.Structure):
@@ -118,6 +119,10 @@ def lib():
         L.abft_version.restype = C.c_char_p
         L.abft_info.restype = st
         L.abft_info.argtypes = [P, C.POINTER(Info)]
+        L.abft_beta_partial.restype = st
+        L.abft_beta_partial.argtypes = [P, P, P]
+        L.abft_finish.restype = st
+        L.abft_finish.argtypes = [P, P, P, P, i32, i32, P, P]
         _LIB = L
     return _LIB
 
@@ -177,11 +182,15 @@ class Inject:
 
 @dataclass
 class CsrDevice:
-    """CSR matrix resident on the device (torch tensors)."""
+    """CSR matrix resident on the device (torch tensors).  A row-block shard
+    has n rows over n_cols local columns, its own rows' x entries starting at
+    x_offset (include/abft.h abft_csr_t)."""
     n: int
     row_ptr: object
     col: object
     val: object
+    n_cols: int = 0
+    x_offset: int = 0
 
     @property
     def nnz(self):
@@ -207,7 +216,7 @@ class Handle:
         self.nb = (A.n + block_size - 1) // block_size
         self.max_rounds = max_rounds if max_rounds > 0 else 4
         csr = _Csr(A.n, A.nnz, A.row_ptr.data_ptr(), A.col.data_ptr() if A.nnz else 0,
-                   A.val.data_ptr() if A.nnz else 0)
+                   A.val.data_ptr() if A.nnz else 0, A.n_cols, A.x_offset)
         h = C.c_void_p()
         _check(lib().abft_encode(C.byref(csr), block_size, max_rounds,
                                  ENCODE_C_CSR if c_csr else 0, _stream(stream), C.byref(h)),
@@ -239,6 +248,22 @@ class Handle:
         _check(lib().abft_spmv(self._h, _ptr(x), _ptr(y), _ptr(x_norm),
                                C.byref(inj) if inj is not None else None, mode, _stream(stream)),
                "abft_spmv")
+        return y
+
+    def beta_partial(self, out, stream=None):
+        """Enqueue this shard's PW sum of x_i^2 (after a DEFER_FINISH spmv)
+        into the device f64 tensor `out` (one element)."""
+        _check(lib().abft_beta_partial(self._h, _ptr(out), _stream(stream)), "abft_beta_partial")
+        return out
+
+    def finish(self, x, y, parts, rounds=None, inject: Inject | None = None, stream=None):
+        """Steps 4-5 with beta = sqrt(PW(parts)) (parts: device f64 tensor of
+        the per-rank partials in rank order)."""
+        inj = inject.struct() if inject is not None else None
+        r = self.max_rounds if rounds is None else rounds
+        _check(lib().abft_finish(self._h, _ptr(x), _ptr(y), _ptr(parts), int(parts.numel()), r,
+                                 C.byref(inj) if inj is not None else None, _stream(stream)),
+               "abft_finish")
         return y
 
     def correct(self, x, y, max_rounds=0, inject: Inject | None = None, stream=None):

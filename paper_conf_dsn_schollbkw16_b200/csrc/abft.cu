@@ -57,6 +57,8 @@ uint32_t align16(uint32_t v) { return (v + 15u) & ~15u; }
 
 struct abft_ctx {
   int64_t n = 0, nnz = 0, nb = 0, ngroups = 0;
+  int64_t n_cols = 0, x_offset = 0;  // shard layout (square: n, 0)
+  double *bnorm = nullptr;           // [2]: local partial, external beta
   int32_t bs = 32, log2bs = 5, max_rounds = 4;
   const int32_t *rp = nullptr, *ci = nullptr;
   const double *va = nullptr;
@@ -147,6 +149,7 @@ SpmvArgs make_args(const abft_ctx *h, const double *x, double *y, const double *
   a.crp_c = h->crp_c;
   a.K = h->K;
   a.x = x;
+  a.xr = x ? x + h->x_offset : nullptr;
   a.y = y;
   a.x_norm = x_norm;
   a.gsum = h->gsum;
@@ -329,7 +332,7 @@ void launch_lean(const abft_ctx *h, const SpmvArgs &a, cudaStream_t s) {
 template <bool CHECK, bool INJECT>
 abft_status launch_fused_t(const abft_ctx *h, SpmvArgs a, cudaStream_t s) {
   // k_lean needs 16-B aligned operands for its bulk copies (x per call)
-  const bool lean = h->lean && aligned16(a.x);
+  const bool lean = h->lean && aligned16(a.xr);
   const int64_t ngen = lean ? h->n_glist : h->ngroups;
   a.glist = lean ? h->glist : nullptr;
   a.n_glist = ngen;
@@ -605,6 +608,9 @@ abft_status abft_encode(const abft_csr_t *A, int32_t block_size, int32_t max_rou
   *out = nullptr;
   if (A->n <= 0 || A->n >= ((int64_t)1 << 31) - 64 || A->nnz < 0 || A->nnz >= ((int64_t)1 << 31))
     return ABFT_EINVAL;
+  const int64_t ncols = A->n_cols > 0 ? A->n_cols : A->n;
+  if (A->x_offset < 0 || A->x_offset + A->n > ncols || ncols >= ((int64_t)1 << 31))
+    return ABFT_EINVAL;
   if (!A->row_ptr || (A->nnz > 0 && (!A->col_idx || !A->val))) return ABFT_EINVAL;
   if (block_size <= 0 || (block_size & (block_size - 1)) != 0) return ABFT_EINVAL;
   if (block_size > 32) return ABFT_ENOTSUP;
@@ -625,6 +631,8 @@ abft_status abft_encode(const abft_csr_t *A, int32_t block_size, int32_t max_rou
   h->num_sms = num_sms;
   h->n = A->n;
   h->nnz = A->nnz;
+  h->n_cols = ncols;
+  h->x_offset = A->x_offset;
   h->bs = block_size;
   h->log2bs = 0;
   while ((1 << h->log2bs) < block_size) ++h->log2bs;
@@ -694,6 +702,7 @@ abft_status abft_encode(const abft_csr_t *A, int32_t block_size, int32_t max_rou
       (st = dalloc(h, &h->flags, (size_t)(h->max_rounds + 1) * h->nb)) ||
       (st = dalloc(h, &h->n_flags, (size_t)h->max_rounds + 1)) || (st = dalloc(h, &h->beta, 1)) ||
       (st = dalloc(h, &h->beta_valid, 1)) || (st = dalloc(h, &h->gbar, 2)) ||
+      (st = dalloc(h, &h->bnorm, 2)) ||
       (st = dalloc(h, &h->dbg_t1, (size_t)h->nb)) || (st = dalloc(h, &h->dbg_t2, (size_t)h->nb)))
     return fail(st);
   if ((e = cudaMemsetAsync(h->n_cand, 0, sizeof(int32_t), s)) ||
@@ -710,7 +719,7 @@ abft_status abft_encode(const abft_csr_t *A, int32_t block_size, int32_t max_rou
 abft_status abft_spmv(abft_handle_t h, const double *x, double *y, const double *x_norm,
                       const abft_inject_t *inj, uint32_t mode, void *stream) {
   if (!h || !x || !y || x == y) return ABFT_EINVAL;
-  if (mode & ~7u) return ABFT_EINVAL;
+  if (mode & ~15u) return ABFT_EINVAL;
   cudaStream_t s = (cudaStream_t)stream;
   SpmvArgs a = make_args(h, x, y, x_norm);
   const bool check = (mode & ABFT_CHECK) || (mode & ABFT_AUTOCORRECT);
@@ -720,8 +729,33 @@ abft_status abft_spmv(abft_handle_t h, const double *x, double *y, const double 
     a.dbg_t2 = h->dbg_t2;
   }
   TRY(launch_fused(h, a, check, s));
-  if (check) TRY(launch_finish(h, a, (mode & ABFT_AUTOCORRECT) ? h->max_rounds : 0, true, s));
+  if (check && !(mode & ABFT_DEFER_FINISH))
+    TRY(launch_finish(h, a, (mode & ABFT_AUTOCORRECT) ? h->max_rounds : 0, true, s));
   return ABFT_OK;
+}
+
+abft_status abft_beta_partial(abft_handle_t h, double *partial, void *stream) {
+  if (!h || !partial) return ABFT_EINVAL;
+  cudaStream_t s = (cudaStream_t)stream;
+  SpmvArgs a = make_args(h, nullptr, nullptr, nullptr);
+  const int64_t nch = (h->ngroups + kBetaChunk - 1) / kBetaChunk;
+  k_bpart<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>(nch, (int64_t)h->num_sms * 4)), 256,
+            0, s>>>(a);
+  k_bpart_top<<<1, 256, 0, s>>>(a, partial);
+  CK(cudaGetLastError());
+  return ABFT_OK;
+}
+
+abft_status abft_finish(abft_handle_t h, const double *x, double *y, const double *parts,
+                        int32_t nparts, int32_t rounds, const abft_inject_t *inj, void *stream) {
+  if (!h || !x || !y || !parts || nparts <= 0) return ABFT_EINVAL;
+  if (rounds < 0 || rounds > h->max_rounds) return ABFT_EINVAL;
+  cudaStream_t s = (cudaStream_t)stream;
+  k_norm_parts<<<1, 256, 0, s>>>(parts, nparts, h->bnorm + 1);
+  CK(cudaGetLastError());
+  SpmvArgs a = make_args(h, x, y, h->bnorm + 1);
+  TRY(prepare_inject(h, inj, true, s, &a.inj));
+  return launch_finish(h, a, rounds, true, s);
 }
 
 abft_status abft_correct(abft_handle_t h, const double *x, double *y, int32_t max_rounds,
@@ -779,10 +813,10 @@ abft_status abft_spmv_host(abft_handle_t h, const double *x_host, double *y_host
   if (!h || !x_host || !y_host) return ABFT_EINVAL;
   cudaStream_t s = (cudaStream_t)stream;
   if (!h->hx) {
-    TRY(dalloc(h, &h->hx, (size_t)h->n));
+    TRY(dalloc(h, &h->hx, (size_t)h->n_cols));
     TRY(dalloc(h, &h->hy, (size_t)h->n));
   }
-  CK(cudaMemcpyAsync(h->hx, x_host, sizeof(double) * h->n, cudaMemcpyHostToDevice, s));
+  CK(cudaMemcpyAsync(h->hx, x_host, sizeof(double) * h->n_cols, cudaMemcpyHostToDevice, s));
   TRY(abft_spmv(h, h->hx, h->hy, nullptr, nullptr, mode, stream));
   CK(cudaMemcpyAsync(y_host, h->hy, sizeof(double) * h->n, cudaMemcpyDeviceToHost, s));
   if (n_flagged_host)

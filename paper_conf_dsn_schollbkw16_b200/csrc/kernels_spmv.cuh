@@ -74,7 +74,8 @@ struct SpmvArgs {
   const int32_t *__restrict__ cb8;      // compact C: column base of each 8-entry chunk
   const int32_t *__restrict__ crp_c;    // compact row starts (32-entry aligned)
   const double *__restrict__ K;
-  const double *__restrict__ x;
+  const double *__restrict__ x;   // gather base: column j reads x[j]
+  const double *__restrict__ xr;  // row-aligned view: row i's own entry is xr[i]
   double *__restrict__ y;
   const double *x_norm;   // nullable device scalar
   double *gsum;           // [ngroups] x^2 subtree of each group
@@ -288,7 +289,7 @@ __device__ __forceinline__ void group_general(const SpmvArgs &a, int64_t g, int 
   if (valid) {
     rs = __ldg(a.rp + i);
     re = __ldg(a.rp + i + 1);
-    xv = __ldg(a.x + i);
+    xv = __ldg(a.xr + i);
   }
   const GlobalSrc As{a.va, a.ci}, Cs{a.cval, a.ccol};
   const int len = re - rs;
@@ -662,7 +663,7 @@ __device__ __forceinline__ void issue_stage(const SpmvArgs &a, int64_t g, int32_
     const uint32_t bcb = CHECK ? (uint32_t)plen / 2 : 0;  // one int32 per 8 entries
     mbar_arrive_expect_tx(bar, 128 + 256 + bav + bac + bcv + bcc + bcb);
     bulk_g2s(st + c.off_rp, a.rp + r0, 128, bar, pol);
-    bulk_g2s(st + c.off_x, a.x + r0, 256, bar, pol);
+    bulk_g2s(st + c.off_x, a.xr + r0, 256, bar, pol);
     if (bav) bulk_g2s(st + c.off_av, a.va + sa4, bav, bar, pol);
     if (bac) bulk_g2s(st + c.off_ac, a.ci + sa4, bac, bar, pol);
     if (bcv) bulk_g2s(st + c.off_cv, reinterpret_cast<const char *>(a.cval_n) + v0, bcv, bar, pol);
@@ -682,7 +683,7 @@ __device__ __forceinline__ void issue_stage(const SpmvArgs &a, int64_t g, int32_
   const uint32_t bcc = CHECK && ec4 > sc4 ? (uint32_t)(ec4 - sc4) * 4 : 0;
   mbar_arrive_expect_tx(bar, 128 + 256 + bav + bac + bcv + bcc);
   bulk_g2s(st + c.off_rp, a.rp + r0, 128, bar, pol);  // rp[r0 .. r0+31]; rp[r0+32] = ea
-  bulk_g2s(st + c.off_x, a.x + r0, 256, bar, pol);
+  bulk_g2s(st + c.off_x, a.xr + r0, 256, bar, pol);
   if (bav) bulk_g2s(st + c.off_av, a.va + sa4, bav, bar, pol);
   if (bac) bulk_g2s(st + c.off_ac, a.ci + sa4, bac, bar, pol);
   if (bcv) bulk_g2s(st + c.off_cv, a.cval + sc8, bcv, bar, pol);
@@ -766,6 +767,8 @@ __global__ void k_glist(const SpmvArgs a, int32_t *glist, int32_t *count) {
   }
 }
 
+constexpr int kBetaChunk = 1024;  // groups per aligned beta partial (k_finish, k_bpart)
+
 // PW over n doubles at p by one CTA of 256 threads: thread t owns an aligned
 // run of m = 2^k values, reduced 32 at a time in registers (32 loads in
 // flight), runs by a shared-memory tree.  Called by all threads.
@@ -803,6 +806,31 @@ __device__ __forceinline__ double cta_pw_array(const double *p, int64_t n, doubl
   return r;
 }
 
+// Local ||x||^2 partial of this handle's rows (distributed use): aligned
+// 1024-group chunks by many CTAs, then the chunk sums by one CTA.
+__global__ void __launch_bounds__(256) k_bpart(const SpmvArgs a) {
+  __shared__ double s_red[256];
+  const int64_t nch = (a.ngroups + kBetaChunk - 1) / kBetaChunk;
+  for (int64_t c = blockIdx.x; c < nch; c += gridDim.x) {
+    const double v = cta_pw_array(a.gsum + c * kBetaChunk,
+                                  min64(kBetaChunk, a.ngroups - c * kBetaChunk), s_red);
+    if (threadIdx.x == 0) a.bpart[c] = v;
+  }
+}
+__global__ void __launch_bounds__(256) k_bpart_top(const SpmvArgs a, double *out) {
+  __shared__ double s_red[256];
+  const int64_t nch = (a.ngroups + kBetaChunk - 1) / kBetaChunk;
+  const double v = cta_pw_array(a.bpart, nch, s_red);
+  if (threadIdx.x == 0) *out = v;
+}
+// beta = sqrt(PW over per-rank partials, in rank order) -> *out (x_norm).
+__global__ void __launch_bounds__(256) k_norm_parts(const double *parts, int64_t nparts,
+                                                    double *out) {
+  __shared__ double s_red[256];
+  const double v = cta_pw_array(parts, nparts, s_red);
+  if (threadIdx.x == 0) *out = __dsqrt_rn(v);
+}
+
 // beta on demand (abft_beta): PW over the group subtrees, one CTA.
 __global__ void __launch_bounds__(256) k_beta(const SpmvArgs a) {
   __shared__ double s_red[256];
@@ -833,7 +861,6 @@ __device__ __forceinline__ void grid_sync(unsigned *bar) {
   __syncthreads();
 }
 
-constexpr int kBetaChunk = 1024;  // groups per aligned beta partial (k_finish)
 
 // Steps 4-5 after the fused pass, one launch (programmatic dependent launch:
 // its launch latency overlaps the fused kernels; griddepcontrol.wait orders

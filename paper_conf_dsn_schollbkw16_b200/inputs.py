@@ -30,6 +30,7 @@ __all__ = [
     "laplacian_3d_7pt",
     "stencil_3d_27pt",
     "stencil_for_config",
+    "stencil_rows",
     "rmat",
     "random_csr",
     "splitmix64",
@@ -79,14 +80,17 @@ class CSR:
         return f"CSR({self.name!r}, n={self.n}, nnz={self.nnz})"
 
 
-def _stencil(shape, offsets, diag, off, name):
+def _stencil(shape, offsets, diag, off, name, z_range=None):
     """Generic constant-coefficient stencil on a (nz, ny, nx) grid, natural
-    ordering, Dirichlet boundary (neighbours outside the grid are dropped)."""
+    ordering, Dirichlet boundary (neighbours outside the grid are dropped).
+    z_range = (z0, z1) generates only the rows of planes z0..z1-1 (a row-block
+    shard), with GLOBAL column indices."""
     nz, ny, nx = shape
-    n = nz * ny * nx
-    if n >= 2**31:
+    if nz * ny * nx >= 2**31:
         raise ValueError("grid too large for int32 indices")
-    idx = np.arange(n, dtype=np.int64)
+    z0, z1 = z_range if z_range is not None else (0, nz)
+    n = (z1 - z0) * ny * nx
+    idx = np.arange(z0 * ny * nx, z1 * ny * nx, dtype=np.int64)
     x = idx % nx
     y = (idx // nx) % ny
     z = idx // (nx * ny)
@@ -114,12 +118,13 @@ def _stencil(shape, offsets, diag, off, name):
     col = np.empty(nnz, dtype=np.int32)
     val = np.empty(nnz, dtype=np.float64)
     pos = row_ptr[:-1].copy()
+    base = z0 * ny * nx
     for (dz, dy, dx), l, v in zip(offsets, lin, valids):
         rows = idx[v]
-        p = pos[rows]
+        p = pos[rows - base]
         col[p] = (rows + l).astype(np.int32)
         val[p] = diag if (dz, dy, dx) == (0, 0, 0) else off
-        pos[rows] += 1
+        pos[rows - base] += 1
         del rows, p
     return CSR(row_ptr.astype(np.int32), col, val, name)
 
@@ -149,6 +154,21 @@ def stencil_3d_27pt(n: int, ny: int | None = None, nz: int | None = None) -> CSR
     return _stencil((nz, ny, n), offs, 26.0, -1.0, f"st3d27_{n}x{ny}x{nz}")
 
 
+_OFFS = {
+    "5pt": [(0, 0, 0), (0, 0, -1), (0, 0, 1), (0, -1, 0), (0, 1, 0)],
+    "7pt": [(0, 0, 0), (0, 0, -1), (0, 0, 1), (0, -1, 0), (0, 1, 0), (-1, 0, 0), (1, 0, 0)],
+    "27pt": [(dz, dy, dx) for dz in (-1, 0, 1) for dy in (-1, 0, 1) for dx in (-1, 0, 1)],
+}
+_DIAG = {"5pt": 4.0, "7pt": 6.0, "27pt": 26.0}
+
+
+def stencil_rows(kind: str, nx: int, ny: int, nz: int, z0: int, z1: int) -> CSR:
+    """Rows of planes z0..z1-1 of the (nz, ny, nx) `kind` stencil, global
+    column indices (the row-block shard a rank owns)."""
+    return _stencil((nz, ny, nx), list(_OFFS[kind]), _DIAG[kind], -1.0,
+                    f"{kind}_{nx}x{ny}x{nz}[z{z0}:{z1}]", z_range=(z0, z1))
+
+
 def stencil_for_config(kind: str, n: int) -> CSR:
     return {"5pt": lambda: laplacian_2d_5pt(n), "7pt": lambda: laplacian_3d_7pt(n),
             "27pt": lambda: stencil_3d_27pt(n)}[kind]()
@@ -166,9 +186,10 @@ def splitmix64(seed: int, count: int, start: int = 0) -> np.ndarray:
     return z
 
 
-def uniform_vector(n: int, seed: int) -> np.ndarray:
-    """x_i ~ U[-1, 1): ((u >> 11) * 2^-53) * 2 - 1, exact in binary64."""
-    u = splitmix64(seed, n)
+def uniform_vector(n: int, seed: int, start: int = 0) -> np.ndarray:
+    """x_i ~ U[-1, 1): ((u >> 11) * 2^-53) * 2 - 1, exact in binary64.
+    `start` gives entries start .. start+n-1 of the same sequence (a shard)."""
+    u = splitmix64(seed, n, start)
     return (u >> np.uint64(11)).astype(np.float64) * (2.0 ** -53) * 2.0 - 1.0
 
 

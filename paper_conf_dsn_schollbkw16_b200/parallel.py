@@ -1,0 +1,218 @@
+"""Row-block sharding of the protected SpMV across ranks (one process per GPU).
+
+SURVEY.md §8(e): the rows of A are split into contiguous, 32-row-aligned
+ranges; row blocks never straddle ranks, so C's rows, the detection and the
+correction stay rank-local.  Each call needs one exchange step (the x halo)
+and one scalar reduction (beta = ||x||_2):
+
+* Local column numbering keeps GLOBAL order: the columns a rank references
+  are sorted, so its x vector is laid out [halo below | own rows | halo above]
+  and every pairwise sum (R2) sees the same operands in the same
+  order as on one GPU -- y, t1, t2, s and the flags are bit-identical.
+* The halo comes from the owning ranks over NCCL point-to-point (NVLink /
+  NVSwitch on the B200 box; gloo in the CPU tests).  Owned ranges are
+  contiguous, so each neighbour's halo is one contiguous slice of the local x.
+* beta: each rank's PW sum of its own x_i^2 is an aligned node of the global
+  PW tree when the ranges are equal powers of two; the partials are
+  all-gathered (8 bytes per rank) and finished in rank order on the device
+  (abft_finish) -- the single-GPU beta bit for bit.
+
+The host logic here is plain data movement (partitioning, renumbering, index
+lists); every step of the method itself runs in libabft.so.
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass, field
+
+import numpy as np
+
+from . import inputs as G
+
+
+def block_partition(n: int, world: int, align: int = 32) -> list[tuple[int, int]]:
+    """Contiguous row ranges, boundaries multiples of `align` (the last range
+    takes the remainder).  Equal power-of-two ranges keep beta bit-exact."""
+    groups = (n + align - 1) // align
+    out, g0 = [], 0
+    for r in range(world):
+        g1 = groups * (r + 1) // world
+        out.append((min(g0 * align, n), min(g1 * align, n)))
+        g0 = g1
+    return out
+
+
+@dataclass
+class Shard:
+    """The local view of one rank: rows [row0, row1) of the global matrix."""
+    rank: int
+    world: int
+    row0: int
+    row1: int
+    csr: G.CSR                # local rows, local (global-order) column indices
+    n_cols: int               # local columns = len(cols)
+    x_offset: int             # local index of global row0
+    cols: np.ndarray          # global index of each local column (sorted)
+    recv: dict = field(default_factory=dict)   # q -> (local start, count): halo from rank q
+    send: dict = field(default_factory=dict)   # q -> local own indices rank q needs
+
+    @property
+    def n(self) -> int:
+        return self.row1 - self.row0
+
+
+def make_shard(rows: G.CSR, row0: int, row1: int, rank: int, world: int,
+               ranges: list[tuple[int, int]]) -> Shard:
+    """Renumber a rank's rows (global column indices) to the local layout
+    [halo below | own | halo above] in global order and record, per owning
+    rank, the contiguous local slice its halo lands in."""
+    own = np.arange(row0, row1, dtype=np.int64)
+    ref = np.unique(rows.col.astype(np.int64))
+    cols = np.union1d(ref, own)
+    local = np.searchsorted(cols, rows.col.astype(np.int64)).astype(np.int32)
+    x_offset = int(np.searchsorted(cols, row0))
+    sh = Shard(rank, world, row0, row1, G.CSR(rows.row_ptr, local, rows.val, rows.name),
+               int(cols.shape[0]), x_offset, cols)
+    for q, (a, b) in enumerate(ranges):
+        if q == rank or a == b:
+            continue
+        lo, hi = np.searchsorted(cols, a), np.searchsorted(cols, b)
+        if hi > lo:
+            sh.recv[q] = (int(lo), int(hi - lo))
+    return sh
+
+
+def exchange_plans(shards_or_needs, ranks) -> None:
+    """Given every rank's shard (or, distributed, the gathered halo needs),
+    fill each shard's send lists: rank r sends to q the own entries q needs,
+    in q's (global) order."""
+    by_rank = {sh.rank: sh for sh in shards_or_needs}
+    for q in ranks:
+        shq = by_rank[q]
+        for r, (start, count) in shq.recv.items():
+            need = shq.cols[start:start + count]          # global indices owned by r
+            shr = by_rank[r]
+            shr.send[q] = (need - shr.row0 + shr.x_offset).astype(np.int64)
+
+
+def plan_from_needs(sh: Shard, needs: dict) -> None:
+    """Distributed variant: `needs[q]` = the global indices rank q needs from
+    this rank (gathered from all ranks)."""
+    for q, need in needs.items():
+        sh.send[q] = (np.asarray(need, dtype=np.int64) - sh.row0 + sh.x_offset)
+
+
+def halo_needs(sh: Shard) -> dict:
+    """Global indices this rank needs from each owning rank."""
+    return {q: sh.cols[s:s + c].tolist() for q, (s, c) in sh.recv.items()}
+
+
+# ---------------------------------------------------------------------------
+# Exchange backends (x_ext: the local extended vector, a torch tensor)
+# ---------------------------------------------------------------------------
+class TorchDistComm:
+    """Halo exchange with torch.distributed point-to-point (NCCL on GPUs,
+    gloo on CPU) and the beta partials with all_gather_into_tensor."""
+
+    def __init__(self, group=None):
+        import torch.distributed as dist
+        self.dist = dist
+        self.group = group
+        self.rank = dist.get_rank(group)
+        self.world = dist.get_world_size(group)
+        self._idx = {}
+
+    def halo(self, sh: Shard, x_ext) -> None:
+        import torch
+        ops = []
+        bufs = []
+        for q, idx in sorted(sh.send.items()):
+            key = (id(sh), q, x_ext.device)
+            if key not in self._idx:
+                self._idx[key] = torch.as_tensor(idx, device=x_ext.device)
+            buf = x_ext.index_select(0, self._idx[key])
+            bufs.append(buf)
+            ops.append(self.dist.P2POp(self.dist.isend, buf, q, self.group))
+        for q, (start, count) in sorted(sh.recv.items()):
+            ops.append(self.dist.P2POp(self.dist.irecv, x_ext[start:start + count], q, self.group))
+        if ops:
+            for w in self.dist.batch_isend_irecv(ops):
+                w.wait()
+
+    def gather_partials(self, partial, out) -> None:
+        self.dist.all_gather_into_tensor(out, partial, group=self.group)
+
+    def gather_needs(self, sh: Shard) -> dict:
+        """All-to-all of halo needs (once, at setup)."""
+        mine = halo_needs(sh)
+        allneeds = [None] * self.world
+        self.dist.all_gather_object(allneeds, mine, group=self.group)
+        return {q: allneeds[q][sh.rank] for q in range(self.world)
+                if q != sh.rank and sh.rank in allneeds[q]}
+
+
+class LocalComm:
+    """All shards in one process (logical shards on one GPU, tests): the halo
+    is copied from the owners' extended vectors."""
+
+    def __init__(self, shards, xs):
+        self.shards = {s.rank: s for s in shards}
+        self.xs = xs  # rank -> x_ext tensor
+
+    def halo(self, sh: Shard, x_ext) -> None:
+        for q, (start, count) in sh.recv.items():
+            owner = self.shards[q]
+            idx = owner.send[sh.rank]
+            src = self.xs[q]
+            import torch
+            x_ext[start:start + count] = src.index_select(
+                0, torch.as_tensor(idx, device=src.device))
+
+
+# ---------------------------------------------------------------------------
+# Distributed protected SpMV on top of the C ABI
+# ---------------------------------------------------------------------------
+class DistSpmv:
+    """One rank's protected SpMV: halo exchange, fused multiply+detect on the
+    local shard (ABFT_DEFER_FINISH), beta partial, all-gather, finish."""
+
+    def __init__(self, shard: Shard, block_size: int = 32, max_rounds: int = 4,
+                 device="cuda"):
+        import torch
+
+        from .abft import CsrDevice, Handle
+        self.sh = shard
+        A = CsrDevice(shard.n, torch.from_numpy(shard.csr.row_ptr).to(device),
+                      torch.from_numpy(shard.csr.col).to(device),
+                      torch.from_numpy(shard.csr.val).to(device),
+                      n_cols=shard.n_cols, x_offset=shard.x_offset)
+        self.h = Handle(A, block_size, max_rounds)
+        self.max_rounds = max_rounds
+        self.x_ext = torch.zeros(shard.n_cols, dtype=torch.float64, device=device)
+        self.y = torch.empty(shard.n, dtype=torch.float64, device=device)
+        self.parts = torch.empty(shard.world, dtype=torch.float64, device=device)
+
+    def own(self):
+        s = self.sh
+        return self.x_ext[s.x_offset:s.x_offset + s.n]
+
+    def step1(self, comm, inject=None):
+        """Halo + fused pass (steps 1-3) + this rank's beta partial."""
+        import torch
+
+        from .abft import CHECK, DEFER_FINISH
+        comm.halo(self.sh, self.x_ext)
+        self.h.spmv(self.x_ext, self.y, inject=inject, mode=CHECK | DEFER_FINISH)
+        if not hasattr(self, "_part"):
+            self._part = torch.empty(1, dtype=torch.float64, device=self.x_ext.device)
+        return self.h.beta_partial(self._part)
+
+    def spmv(self, comm, inject=None, rounds=None):
+        """One distributed protected SpMV (all ranks call it)."""
+        part = self.step1(comm, inject)
+        comm.gather_partials(part, self.parts)
+        return self.step2(rounds, inject)
+
+    def step2(self, rounds=None, inject=None):
+        """Steps 4-5 with beta from all ranks' partials (self.parts)."""
+        self.h.finish(self.x_ext, self.y, self.parts, rounds, inject)
+        return self.y
