@@ -115,8 +115,13 @@ def dist_init():
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if world > 1:
         import torch.distributed as dist
-        torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        dev = local % max(1, torch.cuda.device_count())
+        torch.cuda.set_device(dev)
+        backend = os.environ.get("ABFT_DIST_BACKEND", "nccl")  # gloo: 1-GPU rehearsal
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", dev))
+        else:
+            dist.init_process_group(backend)
     elif torch.cuda.is_available():
         torch.cuda.set_device(local)
     return world, rank, local
@@ -133,7 +138,8 @@ def max_over_ranks(v, world):
         return v
     import torch
     import torch.distributed as dist
-    t = torch.tensor([v], dtype=torch.float64, device="cuda")
+    dev = "cuda" if dist.get_backend() == "nccl" else "cpu"
+    t = torch.tensor([v], dtype=torch.float64, device=dev)
     dist.all_reduce(t, op=dist.ReduceOp.MAX)
     return float(t.item())
 
@@ -249,6 +255,91 @@ def run_reference(args):
                 "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
+
+
+def run_ours_dist(args):
+    """N > 1: weak scaling.  Rank r owns planes [r*nz, (r+1)*nz) of a
+    (nz*N) x ny x nx grid of the workload's stencil (the configs[1] 128^3 slab
+    per rank); one step = halo exchange (NCCL P2P) + fused multiply+detect +
+    beta partial + all-gather (NCCL) + finish/correct."""
+    import torch
+
+    from paper_conf_dsn_schollbkw16_b200 import inputs as G
+    from paper_conf_dsn_schollbkw16_b200 import parallel as PL
+    world, rank, local = dist_init()
+    kind, nx = {"7pt128": ("7pt", 128), "27pt128": ("27pt", 128), "27pt256": ("27pt", 256),
+                "5pt64": ("5pt", 64)}[args.workload]
+    ny, nzl = (nx, nx) if kind != "5pt" else (nx, 1)
+    nz = nzl * world
+    plane = nx * ny
+    ranges = [(r * nzl * plane, (r + 1) * nzl * plane) for r in range(world)]
+    a, b = ranges[rank]
+    rows = G.stencil_rows(kind, nx, ny, nz, rank * nzl, (rank + 1) * nzl)
+    sh = PL.make_shard(rows, a, b, rank, world, ranges)
+    comm = PL.TorchDistComm()
+    PL.plan_from_needs(sh, comm.gather_needs(sh))
+    d = PL.DistSpmv(sh, args.block_size, args.max_rounds)
+    d.own().copy_(torch.from_numpy(G.uniform_vector(sh.n, 42, start=a)))
+    info = d.h.info()
+    torch.cuda.synchronize()
+
+    def step():
+        d.spmv(comm)
+
+    for _ in range(max(args.warmup, 3)):
+        step()
+    torch.cuda.synchronize()
+    clocks = ClockSampler(torch.cuda.current_device())
+    clocks.start()
+    t_end = time.perf_counter() + 1.0
+    while time.perf_counter() < t_end:
+        for _ in range(20):
+            step()
+        torch.cuda.synchronize()
+    ms = timed(step, args.steps, world)
+    clk = clocks.stop()
+    # local bytes: A rows + own x + halo x + y + C + K
+    nbytes = (12 * sh.csr.nnz + 4 * (sh.n + 1) + 8 * sh.n_cols + 8 * sh.n + info["c_bytes"]
+              + 8 * info["nb"])
+    value = world * nbytes / (ms * 1e-3) / 1e9
+    # end to end: host x slice in, host y slice out, per rank
+    xh = torch.from_numpy(G.uniform_vector(sh.n, 42, start=a)).pin_memory()
+    yh = torch.empty(sh.n, dtype=torch.float64).pin_memory()
+    k_e2e = max(3, min(args.steps, 100))
+    barrier(world)
+    t0 = time.perf_counter()
+    for _ in range(k_e2e):
+        d.own().copy_(xh, non_blocking=True)
+        step()
+        yh.copy_(d.y, non_blocking=True)
+        torch.cuda.synchronize()
+    dt_e2e = max_over_ranks((time.perf_counter() - t0) / k_e2e, world)
+    peak, peak_src = load_peaks()
+    if rank == 0:
+        print(json.dumps({
+            "metric": METRIC, "value": round(value, 2), "unit": "GB/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms, 5),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic",
+            "config": {"workload": f"{kind} stencil {nx}x{ny}x{nzl} rows per GPU, "
+                                   f"global {nx}x{ny}x{nz}, row-block sharded",
+                       "rows_per_gpu": sh.n, "nnz_per_gpu": sh.csr.nnz,
+                       "parallelism": f"rowblock{world}", "c_format": info["c_format_name"],
+                       "l2": "no flush: per-GPU working set > L2",
+                       "step": "halo (NCCL P2P) + k_lean (DEFER) + beta partial + all-gather "
+                               "(NCCL) + k_finish",
+                       "bytes_per_step_per_gpu": nbytes},
+            "roofline": {"bound": "hbm", "kernel": "whole step", "achieved": round(value / world, 2),
+                         "peak": peak, "unit": "GB/s", "frac": round(value / world / peak, 4),
+                         "traffic": None, "peak_source": peak_src},
+            "cpu_baseline": None,
+            "e2e": {"value": round(world * nbytes / dt_e2e / 1e9, 3), "unit": "GB/s",
+                    "h2d_bytes_per_step": 8 * sh.n * world, "d2h_bytes_per_step": 8 * sh.n * world,
+                    "ms_per_step": round(dt_e2e * 1e3, 4)},
+            "gpu_launches": args.steps * 5,
+            "clocks": clk}), flush=True)
+    import torch.distributed as dist
+    dist.destroy_process_group()
 
 
 def run_ours(args):
@@ -420,6 +511,8 @@ def main():
         run_reference(args)
     elif args.pcg:
         run_pcg(args)
+    elif int(os.environ.get("WORLD_SIZE", "1")) > 1:
+        run_ours_dist(args)
     else:
         run_ours(args)
 

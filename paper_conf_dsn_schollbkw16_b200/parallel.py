@@ -120,26 +120,42 @@ class TorchDistComm:
         self.rank = dist.get_rank(group)
         self.world = dist.get_world_size(group)
         self._idx = {}
+        # gloo carries CPU tensors only: stage device buffers through the host
+        self.stage = dist.get_backend(group) != "nccl"
 
     def halo(self, sh: Shard, x_ext) -> None:
         import torch
-        ops = []
-        bufs = []
+        stage = self.stage and x_ext.is_cuda
+        ops, bufs, recvs = [], [], []
         for q, idx in sorted(sh.send.items()):
             key = (id(sh), q, x_ext.device)
             if key not in self._idx:
                 self._idx[key] = torch.as_tensor(idx, device=x_ext.device)
             buf = x_ext.index_select(0, self._idx[key])
+            if stage:
+                buf = buf.cpu()
             bufs.append(buf)
             ops.append(self.dist.P2POp(self.dist.isend, buf, q, self.group))
         for q, (start, count) in sorted(sh.recv.items()):
-            ops.append(self.dist.P2POp(self.dist.irecv, x_ext[start:start + count], q, self.group))
+            dst = x_ext[start:start + count]
+            if stage:
+                tmp = torch.empty(count, dtype=x_ext.dtype)
+                recvs.append((dst, tmp))
+                dst = tmp
+            ops.append(self.dist.P2POp(self.dist.irecv, dst, q, self.group))
         if ops:
             for w in self.dist.batch_isend_irecv(ops):
                 w.wait()
+        for dst, tmp in recvs:
+            dst.copy_(tmp)
 
     def gather_partials(self, partial, out) -> None:
-        self.dist.all_gather_into_tensor(out, partial, group=self.group)
+        if self.stage and partial.is_cuda:
+            o = out.cpu()
+            self.dist.all_gather_into_tensor(o, partial.cpu(), group=self.group)
+            out.copy_(o)
+        else:
+            self.dist.all_gather_into_tensor(out, partial, group=self.group)
 
     def gather_needs(self, sh: Shard) -> dict:
         """All-to-all of halo needs (once, at setup)."""
