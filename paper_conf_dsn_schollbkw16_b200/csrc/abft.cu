@@ -68,8 +68,7 @@ struct abft_ctx {
   int32_t max_seg_a = 0, max_seg_c = 0;
   int cfmt = CF_CSR;         // format of C streamed by k_lean
   void *cval_n = nullptr;    // compact C values
-  uint16_t *ccol16 = nullptr;
-  int32_t *cb8 = nullptr;    // compact C: column base per 8-entry chunk
+  uint16_t *cmap = nullptr;  // compact C: A-slot index of each entry
   int32_t *crp_c = nullptr;  // compact row starts (32-entry aligned)
   int64_t nnz_cpad = 0;      // compact slots incl. row padding
   StageCfg stage{};
@@ -144,8 +143,7 @@ SpmvArgs make_args(const abft_ctx *h, const double *x, double *y, const double *
   a.ccol = h->c_col;
   a.cval = h->c_val;
   a.cval_n = h->cval_n;
-  a.ccol16 = h->ccol16;
-  a.cb8 = h->cb8;
+  a.cmap = h->cmap;
   a.crp_c = h->crp_c;
   a.K = h->K;
   a.x = x;
@@ -433,7 +431,7 @@ abft_status init_device_once(int device) {
 // Lossless compact C: pick the narrowest exact value
 // type and uint16 column offsets when every row spans < 65536 columns.
 abft_status build_compact_c(abft_ctx *h, cudaStream_t s) {
-  if (h->nnz_c == 0) return ABFT_OK;
+  if (h->nnz_c == 0 || h->bs != 32) return ABFT_OK;  // compact C serves the b_s = 32 fast path
   int32_t *dev = nullptr;
   TRY(dalloc(h, &dev, 1));
   CK(cudaMemsetAsync(dev, 0, sizeof(int32_t), s));
@@ -443,7 +441,6 @@ abft_status build_compact_c(abft_ctx *h, cudaStream_t s) {
   int32_t props = 0;
   CK(cudaMemcpyAsync(&props, dev, sizeof props, cudaMemcpyDeviceToHost, s));
   CK(cudaStreamSynchronize(s));
-  if (props & 8) return ABFT_OK;  // a chunk spans >= 65536 columns: keep CSR
   const int cf = !(props & 1) ? CF_I8 : !(props & 2) ? CF_I16 : !(props & 4) ? CF_F32 : CF_F64;
   const size_t sz = (size_t)cf_size(cf);
   // compact row starts: exclusive scan of the 32-entry padded row lengths
@@ -462,33 +459,28 @@ abft_status build_compact_c(abft_ctx *h, cudaStream_t s) {
   CK(cudaStreamSynchronize(s));
   h->nnz_cpad = npad;
   char *cv = nullptr;
+  int32_t *bad = nullptr;
   TRY(dalloc(h, &cv, (size_t)npad * sz + 64));
-  TRY(dalloc(h, &h->ccol16, (size_t)npad + 32));
-  TRY(dalloc(h, &h->cb8, (size_t)npad / 8 + 8));
+  TRY(dalloc(h, &h->cmap, (size_t)npad + 32));
+  TRY(dalloc(h, &bad, 1));
   CK(cudaMemsetAsync(cv, 0, (size_t)npad * sz + 64, s));
-  CK(cudaMemsetAsync(h->ccol16, 0, ((size_t)npad + 32) * 2, s));
-  CK(cudaMemsetAsync(h->cb8, 0, ((size_t)npad / 8 + 8) * 4, s));
+  CK(cudaMemsetAsync(h->cmap, 0, ((size_t)npad + 32) * 2, s));
+  CK(cudaMemsetAsync(bad, 0, sizeof(int32_t), s));
+#define FILL(T)                                                                              \
+  k_cformat_fill<T><<<grid, 256, 0, s>>>(h->nb, h->n, h->rp, h->ci, h->c_rp, h->crp_c,        \
+                                         h->c_col, h->c_val, reinterpret_cast<T *>(cv),       \
+                                         h->cmap, bad)
   switch (cf) {
-    case CF_I8:
-      k_cformat_fill<int8_t><<<grid, 256, 0, s>>>(h->nb, h->c_rp, h->crp_c, h->c_col, h->c_val,
-                                                  reinterpret_cast<int8_t *>(cv), h->ccol16,
-                                                  h->cb8);
-      break;
-    case CF_I16:
-      k_cformat_fill<int16_t><<<grid, 256, 0, s>>>(h->nb, h->c_rp, h->crp_c, h->c_col, h->c_val,
-                                                   reinterpret_cast<int16_t *>(cv), h->ccol16,
-                                                   h->cb8);
-      break;
-    case CF_F32:
-      k_cformat_fill<float><<<grid, 256, 0, s>>>(h->nb, h->c_rp, h->crp_c, h->c_col, h->c_val,
-                                                 reinterpret_cast<float *>(cv), h->ccol16, h->cb8);
-      break;
-    default:
-      k_cformat_fill<double><<<grid, 256, 0, s>>>(h->nb, h->c_rp, h->crp_c, h->c_col, h->c_val,
-                                                  reinterpret_cast<double *>(cv), h->ccol16,
-                                                  h->cb8);
-      break;
+    case CF_I8: FILL(int8_t); break;
+    case CF_I16: FILL(int16_t); break;
+    case CF_F32: FILL(float); break;
+    default: FILL(double); break;
   }
+#undef FILL
+  int32_t hbad = 0;
+  CK(cudaMemcpyAsync(&hbad, bad, sizeof hbad, cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  if (hbad) return ABFT_OK;  // some block's A segment exceeds uint16 slots: keep CSR
   CK(cudaGetLastError());
   h->cval_n = cv;
   h->cfmt = cf;
@@ -530,11 +522,11 @@ abft_status plan_fused(abft_ctx *h, cudaStream_t s) {
       o += align16(cpad * cf_size(h->cfmt));
       c.off_cc = o;
       o += align16(cpad * 2);
-      c.off_cb = o;
-      o += align16(cpad / 2);
     }
     c.off_cp = o;  // padded C products (one gap per 8; CSR format only)
     if (h->cfmt == CF_CSR) o += align16((uint32_t)(c.capC + c.capC / 8 + 8) * 8);
+    c.off_xg = o;  // gathered x per A slot (compact format only)
+    if (h->cfmt != CF_CSR) o += align16((uint32_t)(c.capA + 6) * 8);
     c.stage_bytes = align16(o);
     c.bar_bytes = 128;
     h->fused_smem = c.bar_bytes + (size_t)warps * c.nstage * c.stage_bytes;
@@ -837,8 +829,7 @@ abft_status abft_info(abft_handle_t h, abft_info_t *info) {
   if (h->cfmt == CF_CSR)
     info->c_bytes = 12 * h->nnz_c + 4 * (h->nb + 1);
   else
-    info->c_bytes = (int64_t)(cf_size(h->cfmt) + 2) * h->nnz_cpad + h->nnz_cpad / 2 +
-                    8 * (h->nb + 1);
+    info->c_bytes = (int64_t)(cf_size(h->cfmt) + 2) * h->nnz_cpad + 8 * (h->nb + 1);
   info->groups = h->ngroups;
   info->general_groups = h->lean ? h->n_glist : h->ngroups;
   info->lean = h->lean ? 1 : 0;

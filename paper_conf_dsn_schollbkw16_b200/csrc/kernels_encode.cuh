@@ -111,16 +111,16 @@ __global__ void __launch_bounds__(256) k_encode(const EncodeArgs a) {
 }
 
 // Compact checksum matrix: the values of C in the
-// narrowest type that holds every one of them exactly, and the columns as
-// uint16 offsets from a per-chunk base (one int32 per 8 entries).  Rows start
-// on 32-entry boundaries so every staged piece is 16-B aligned.  Lossless:
-// the kernels recover bit-identical c_kj and column indices.
+// narrowest type that holds every one of them exactly, and per entry a uint16
+// index of an A entry of the same block with the same column (so the kernel
+// reuses that entry's gathered x_j).  Rows start on 16-entry boundaries so
+// every staged piece is 16-B aligned.  Lossless: the kernels recover
+// bit-identical c_kj and x_j.
 enum { CF_CSR = 0, CF_I8 = 1, CF_I16 = 2, CF_F32 = 3, CF_F64 = 4 };
-constexpr int kCRowAlign = 32;  // compact row alignment (entries)
+constexpr int kCRowAlign = 16;  // compact row alignment (entries)
 
 // props bits: 1 = some value is not an integer in [-128,127], 2 = not in
-// [-32768,32767], 4 = not exactly representable in float, 8 = some 8-entry
-// chunk spans >= 65536 columns (no uint16 offsets).
+// [-32768,32767], 4 = not exactly representable in float.
 __global__ void k_cformat_scan(int64_t nb, const int32_t *__restrict__ crp,
                                const int32_t *__restrict__ ccol, const double *__restrict__ cval,
                                int32_t *props) {
@@ -136,10 +136,6 @@ __global__ void k_cformat_scan(int64_t nb, const int32_t *__restrict__ crp,
       if (!(v == rint(v)) || v < -32768.0 || v > 32767.0) pr |= 2;
       if (!((double)(float)v == v) && v == v) pr |= 4;
       if (v != v) pr |= 7;  // NaN: keep f64
-      if (((q - b) & 7) == 0) {
-        const int32_t last = min(q + 7, e - 1);
-        if (ccol[last] - ccol[q] >= 65536) pr |= 8;
-      }
     }
   }
   pr = __reduce_or_sync(kFull, pr);
@@ -152,21 +148,37 @@ __global__ void k_cformat_padlen(int64_t nb, const int32_t *__restrict__ crp, in
     plen[k] = (crp[k + 1] - crp[k] + kCRowAlign - 1) & ~(kCRowAlign - 1);
 }
 
+// Compact C for the staged fast path (b_s = 32): value c_kj in the narrow type
+// and, instead of its column, the staging slot of an A entry of the same
+// block with that column (slot = position in A's arrays - (rp[32k] & ~3)):
+// the fused kernel multiplies c_kj with the x_j it already gathered for A.
 template <typename T>
-__global__ void k_cformat_fill(int64_t nb, const int32_t *__restrict__ crp,
+__global__ void k_cformat_fill(int64_t nb, int64_t n, const int32_t *__restrict__ rp,
+                               const int32_t *__restrict__ ci, const int32_t *__restrict__ crp,
                                const int32_t *__restrict__ crp_c, const int32_t *__restrict__ ccol,
-                               const double *__restrict__ cval, T *cv, uint16_t *cc16,
-                               int32_t *cb8) {
+                               const double *__restrict__ cval, T *cv, uint16_t *cmap,
+                               int32_t *bad) {
   const int lane = threadIdx.x & 31;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
   for (int64_t k = gw; k < nb; k += nw) {
     const int32_t b = crp[k], e = crp[k + 1], d = crp_c[k] - b;
+    const int64_t r0 = k * 32, r1 = min64(r0 + 32, n);
+    const int32_t s0 = rp[r0] & ~3;
     for (int32_t q = b + lane; q < e; q += 32) {
-      const int32_t base = ccol[b + ((q - b) & ~7)];  // first column of the chunk
+      const int32_t j = ccol[q];
+      int64_t slot = -1;
+      for (int64_t r = r0; r < r1 && slot < 0; ++r) {  // first row of the block holding j
+        int32_t lo = rp[r], hi = rp[r + 1];
+        while (lo < hi) {
+          const int32_t mid = (lo + hi) >> 1;
+          if (ci[mid] < j) lo = mid + 1; else hi = mid;
+        }
+        if (lo < rp[r + 1] && ci[lo] == j) slot = lo - s0;
+      }
+      if (slot < 0 || slot > 65535) atomicOr(bad, 1);
       cv[q + d] = (T)cval[q];
-      cc16[q + d] = (uint16_t)(ccol[q] - base);
-      if (((q - b) & 7) == 0) cb8[(q + d) >> 3] = base;
+      cmap[q + d] = (uint16_t)(slot < 0 ? 0 : slot);
     }
   }
 }

@@ -53,7 +53,7 @@ struct StageCfg {
   int32_t warps;          // warps per CTA
   uint32_t stage_bytes;   // bytes per stage
   uint32_t bar_bytes;     // mbarrier region at the start of dynamic smem
-  uint32_t off_rp, off_x, off_av, off_ac, off_cv, off_cc, off_cp, off_cb;
+  uint32_t off_rp, off_x, off_av, off_ac, off_cv, off_cc, off_cp, off_xg;
 };
 
 struct SpmvArgs {
@@ -70,8 +70,7 @@ struct SpmvArgs {
   const int32_t *__restrict__ ccol;
   const double *__restrict__ cval;
   const void *__restrict__ cval_n;       // compact C values (CF != CF_CSR)
-  const uint16_t *__restrict__ ccol16;  // compact C columns: offset from the chunk base
-  const int32_t *__restrict__ cb8;      // compact C: column base of each 8-entry chunk
+  const uint16_t *__restrict__ cmap;   // compact C: staging slot of an A entry, same column
   const int32_t *__restrict__ crp_c;    // compact row starts (32-entry aligned)
   const double *__restrict__ K;
   const double *__restrict__ x;   // gather base: column j reads x[j]
@@ -459,8 +458,15 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
   const double *cv = reinterpret_cast<const double *>(st + c.off_cv) + (sc & 1);  // sc + e
   const int32_t *cc = reinterpret_cast<const int32_t *>(st + c.off_cc) + (sc & 3);
   double *cp = reinterpret_cast<double *>(st + c.off_cp);  // C products, padded
+  double *xg = reinterpret_cast<double *>(st + c.off_xg);   // gathered x per A slot
   const int nS = ((ea + 3) & ~3) - (sa & ~3);
   const int nC = CHECK ? ec - sc : 0;
+  // row bounds first: the max-reduction's latency overlaps the gathers below
+  const int32_t rs = reinterpret_cast<const int32_t *>(st + c.off_rp)[lane];
+  int32_t re = __shfl_down_sync(kFull, rs, 1);
+  if (lane == 31) re = ea;
+  const int len = re - rs;
+  const int maxlen = warp_max_i(len);
   // phase 1a: A products in place; lane l owns slots 4l + 128u .. +3
   // (128-bit shared loads/stores), 8 gathers in flight per lane.
 #pragma unroll 1
@@ -480,10 +486,16 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
     for (int u = 0; u < 2; ++u) {
       const int s0 = base + u * 128 + lane * 4;
       if (s0 < nS) {
-        v[2 * u].x = dmul(v[2 * u].x, ld_x(a.x + ci[u].x));
-        v[2 * u].y = dmul(v[2 * u].y, ld_x(a.x + ci[u].y));
-        v[2 * u + 1].x = dmul(v[2 * u + 1].x, ld_x(a.x + ci[u].z));
-        v[2 * u + 1].y = dmul(v[2 * u + 1].y, ld_x(a.x + ci[u].w));
+        const double x0 = ld_x(a.x + ci[u].x), x1 = ld_x(a.x + ci[u].y);
+        const double x2 = ld_x(a.x + ci[u].z), x3 = ld_x(a.x + ci[u].w);
+        if (CHECK && CF != CF_CSR) {  // keep x_j for C's entries (compact map)
+          *reinterpret_cast<double2 *>(xg + s0) = make_double2(x0, x1);
+          *reinterpret_cast<double2 *>(xg + s0 + 2) = make_double2(x2, x3);
+        }
+        v[2 * u].x = dmul(v[2 * u].x, x0);
+        v[2 * u].y = dmul(v[2 * u].y, x1);
+        v[2 * u + 1].x = dmul(v[2 * u + 1].x, x2);
+        v[2 * u + 1].y = dmul(v[2 * u + 1].y, x3);
       }
     }
 #pragma unroll
@@ -522,11 +534,6 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
   __syncwarp();
   // y_i = PW over the row's products (lane-private tree; PW is padding
   // independent, so P = 8 serves every row of length <= 8)
-  const int32_t rs = reinterpret_cast<const int32_t *>(st + c.off_rp)[lane];
-  int32_t re = __shfl_down_sync(kFull, rs, 1);
-  if (lane == 31) re = ea;
-  const int len = re - rs;
-  const int maxlen = warp_max_i(len);
   const double *row = pv + (rs - sa);
   double yv;
   if (maxlen <= 8) {
@@ -550,17 +557,20 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
   a.y[i] = yv;
   if (!CHECK) return;
 
-  double t2 = bfly32(yv);  // step 2: t2_k = w_k^T y_k
+  // the three warp butterflies (t2, chunk sums of t1, x^2) are independent:
+  // they run interleaved in one loop below, so their latencies overlap
+  double t2 = yv;  // step 2: t2_k = w_k^T y_k -- butterflied below
+  const double xv = reinterpret_cast<const double *>(st + c.off_x)[lane];
+  double gs = dmul(xv, xv);  // the group's x^2 subtree -- butterflied below
   // step 1: t1_k = c_k . x.  Lane l owns elements 8l..8l+7 of
   // each aligned 256-chunk: an 8-leaf tree in registers, then the butterfly
   // over lanes -- exactly the PW tree of the chunk; chunks by a 4-leaf tree.
   double q[4];
   if (CF != CF_CSR) {
-    // compact C: the row is staged 16-B aligned; values and uint16 column
-    // offsets come in with vector loads, products never touch shared memory
+    // compact C: the row is staged 16-B aligned; values and A-slot indices
+    // come in with vector loads, x_j from the A pass (shared memory only)
     const unsigned char *cvb = st + c.off_cv;
-    const uint16_t *c16 = reinterpret_cast<const uint16_t *>(st + c.off_cc);
-    const int32_t *cbs = reinterpret_cast<const int32_t *>(st + c.off_cb);
+    const uint16_t *cm = reinterpret_cast<const uint16_t *>(st + c.off_cc);
 #pragma unroll
     for (int t = 0; t < 4; ++t) {
       double v[8];
@@ -569,19 +579,18 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
         if (j0 < nC) {
           CT cvv[8];
           load8(cvv, cvb + (size_t)j0 * sizeof(CT));
-          const uint4 o4 = *reinterpret_cast<const uint4 *>(c16 + j0);
+          const uint4 o4 = *reinterpret_cast<const uint4 *>(cm + j0);
           const uint32_t ow[4] = {o4.x, o4.y, o4.z, o4.w};
-          const int32_t cb = cbs[j0 >> 3];
 #pragma unroll
           for (int u = 0; u < 8; ++u) {
-            const int32_t col = cb + (int32_t)((ow[u >> 1] >> (16 * (u & 1))) & 0xffffu);
-            v[u] = j0 + u < nC ? dmul((double)cvv[u], ld_x(a.x + col)) : kAbsent;
+            const int slot = (int)((ow[u >> 1] >> (16 * (u & 1))) & 0xffffu);
+            v[u] = j0 + u < nC ? dmul((double)cvv[u], xg[slot]) : kAbsent;
           }
         } else {
 #pragma unroll
           for (int u = 0; u < 8; ++u) v[u] = kAbsent;
         }
-        q[t] = bfly32(tree<8>(v));
+        q[t] = tree<8>(v);
       } else {
         q[t] = kAbsent;
       }
@@ -595,11 +604,27 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
         double v[8];
 #pragma unroll
         for (int u = 0; u < 8; ++u) v[u] = u < rc ? cpl[u] : kAbsent;
-        q[t] = bfly32(tree<8>(v));
+        q[t] = tree<8>(v);
       } else {
         q[t] = kAbsent;
       }
     }
+  }
+  if (nC <= 256) {  // the common case: one chunk
+#pragma unroll
+    for (int m = 1; m < 32; m <<= 1) {
+      const double a0 = __shfl_xor_sync(kFull, t2, m), a1 = __shfl_xor_sync(kFull, gs, m),
+                   a2 = __shfl_xor_sync(kFull, q[0], m);
+      t2 = dadd(t2, a0);
+      gs = dadd(gs, a1);
+      q[0] = dadd(q[0], a2);
+    }
+  } else {
+    t2 = bfly32(t2);
+    gs = bfly32(gs);
+#pragma unroll
+    for (int t = 0; t < 4; ++t)
+      if (t * 256 < nC) q[t] = bfly32(q[t]);
   }
   double t1 = nC > 0 ? tree<4>(q) : 0.0;
   if (INJECT && lane == 0) {
@@ -610,8 +635,6 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
     a.dbg_t1[g] = t1;
     a.dbg_t2[g] = t2;
   }
-  const double xv = reinterpret_cast<const double *>(st + c.off_x)[lane];
-  const double gs = bfly32(dmul(xv, xv));  // the group's x^2 subtree
   if (lane == 0) {
     a.gsum[g] = gs;
     test_block_lo(a, g, dsub(t1, t2), gs);  // steps 3-4
@@ -660,15 +683,13 @@ __device__ __forceinline__ void issue_stage(const SpmvArgs &a, int64_t g, int32_
     const int64_t v0 = (int64_t)cc * (int64_t)sizeof(CT), k0 = (int64_t)cc * 2;
     const uint32_t bcv = CHECK ? (uint32_t)plen * (uint32_t)sizeof(CT) : 0;
     const uint32_t bcc = CHECK ? (uint32_t)plen * 2 : 0;
-    const uint32_t bcb = CHECK ? (uint32_t)plen / 2 : 0;  // one int32 per 8 entries
-    mbar_arrive_expect_tx(bar, 128 + 256 + bav + bac + bcv + bcc + bcb);
+    mbar_arrive_expect_tx(bar, 128 + 256 + bav + bac + bcv + bcc);
     bulk_g2s(st + c.off_rp, a.rp + r0, 128, bar, pol);
     bulk_g2s(st + c.off_x, a.xr + r0, 256, bar, pol);
     if (bav) bulk_g2s(st + c.off_av, a.va + sa4, bav, bar, pol);
     if (bac) bulk_g2s(st + c.off_ac, a.ci + sa4, bac, bar, pol);
     if (bcv) bulk_g2s(st + c.off_cv, reinterpret_cast<const char *>(a.cval_n) + v0, bcv, bar, pol);
-    if (bcc) bulk_g2s(st + c.off_cc, reinterpret_cast<const char *>(a.ccol16) + k0, bcc, bar, pol);
-    if (bcb) bulk_g2s(st + c.off_cb, a.cb8 + (cc >> 3), bcb, bar, pol);
+    if (bcc) bulk_g2s(st + c.off_cc, reinterpret_cast<const char *>(a.cmap) + k0, bcc, bar, pol);
     return;
   }
   const StageCfg &c = a.sc;
