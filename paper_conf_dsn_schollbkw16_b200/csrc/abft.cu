@@ -508,6 +508,8 @@ abft_status plan_fused(abft_ctx *h, cudaStream_t s) {
     o += 144;
     c.off_x = o;
     o += 256;
+    c.off_k = o;  // K[g & ~1], K[g | 1]
+    o += 16;
     c.off_av = o;
     o += align16((uint32_t)(c.capA + 6) * 8);
     c.off_ac = o;
@@ -525,8 +527,10 @@ abft_status plan_fused(abft_ctx *h, cudaStream_t s) {
     }
     c.off_cp = o;  // padded C products (one gap per 8; CSR format only)
     if (h->cfmt == CF_CSR) o += align16((uint32_t)(c.capC + c.capC / 8 + 8) * 8);
-    c.off_xg = o;  // gathered x per A slot (compact format only)
-    if (h->cfmt != CF_CSR) o += align16((uint32_t)(c.capA + 6) * 8);
+    // gathered x per A slot (compact format only), after a 16-B slot whose
+    // upper half is the -0.0 sentinel the padding entries of C select
+    c.off_xg = o + 16;
+    if (h->cfmt != CF_CSR) o += 16 + align16((uint32_t)(c.capA + 6) * 8);
     c.stage_bytes = align16(o);
     c.bar_bytes = 128;
     h->fused_smem = c.bar_bytes + (size_t)warps * c.nstage * c.stage_bytes;
@@ -641,7 +645,7 @@ abft_status abft_encode(const abft_csr_t *A, int32_t block_size, int32_t max_rou
   const int64_t nscan = (h->nb + 1023) / 1024;
   if ((st = dalloc(h, &h->c_rp, (size_t)h->nb + 1)) || (st = dalloc(h, &counts, (size_t)h->nb)) ||
       (st = dalloc(h, &totals, (size_t)nscan)) || (st = dalloc(h, &stats, 2)) ||
-      (st = dalloc(h, &h->K, (size_t)h->nb)))
+      (st = dalloc(h, &h->K, (size_t)h->nb + 2)))  // + pad: k_lean stages K in 16-B pairs
     return fail(st);
   cudaError_t e;
   if ((e = cudaMemsetAsync(stats, 0, 2 * sizeof(int32_t), s)) != cudaSuccess)

@@ -152,6 +152,8 @@ __global__ void k_cformat_padlen(int64_t nb, const int32_t *__restrict__ crp, in
 // and, instead of its column, the staging slot of an A entry of the same
 // block with that column (slot = position in A's arrays - (rp[32k] & ~3)):
 // the fused kernel multiplies c_kj with the x_j it already gathered for A.
+// Stored as slot + 1: index 0 (the row padding, value 0) selects a -0.0
+// sentinel, so padded products are -0.0, the exact identity of the sum.
 template <typename T>
 __global__ void k_cformat_fill(int64_t nb, int64_t n, const int32_t *__restrict__ rp,
                                const int32_t *__restrict__ ci, const int32_t *__restrict__ crp,
@@ -176,9 +178,9 @@ __global__ void k_cformat_fill(int64_t nb, int64_t n, const int32_t *__restrict_
         }
         if (lo < rp[r + 1] && ci[lo] == j) slot = lo - s0;
       }
-      if (slot < 0 || slot > 65535) atomicOr(bad, 1);
+      if (slot < 0 || slot > 65534) atomicOr(bad, 1);
       cv[q + d] = (T)cval[q];
-      cmap[q + d] = (uint16_t)(slot < 0 ? 0 : slot);
+      cmap[q + d] = (uint16_t)(slot < 0 ? 0 : slot + 1);  // 0 = row padding (value 0)
     }
   }
 }

@@ -43,6 +43,12 @@ template <> struct CType<CF_I16> { using T = int16_t; };
 template <> struct CType<CF_F32> { using T = float; };
 
 constexpr int kLeanWarps = 4;  // warps per CTA of k_lean (<= 4)
+// Timing experiments only (scripts/exp_libs.sh; results are NOT the method):
+// 1 = no C products, 2 = C neither staged nor multiplied, 3 = no butterflies,
+// 4 = no test, 5 = 1 + 3 + 4.  0 (the default) = the method.
+#ifndef ABFT_EXP
+#define ABFT_EXP 0
+#endif
 #ifndef ABFT_LEAN_MINB
 #define ABFT_LEAN_MINB 5  // min resident CTAs per SM the register budget targets (measured best)
 #endif
@@ -53,7 +59,7 @@ struct StageCfg {
   int32_t warps;          // warps per CTA
   uint32_t stage_bytes;   // bytes per stage
   uint32_t bar_bytes;     // mbarrier region at the start of dynamic smem
-  uint32_t off_rp, off_x, off_av, off_ac, off_cv, off_cc, off_cp, off_xg;
+  uint32_t off_rp, off_x, off_k, off_av, off_ac, off_cv, off_cc, off_cp, off_xg;
 };
 
 struct SpmvArgs {
@@ -263,10 +269,11 @@ __device__ __forceinline__ void test_block(const SpmvArgs &a, int64_t k, double 
 // Same test with a cheaper exact lower bound of beta_g: gs rounded down to
 // float, square root rounded down -- beta_lo <= sqrt(gs) <= beta, so the
 // pre-filter stays exact (a passing block provably passes against tau_k).
-__device__ __forceinline__ void test_block_lo(const SpmvArgs &a, int64_t k, double s, double gs) {
+__device__ __forceinline__ void test_block_lo(const SpmvArgs &a, int64_t k, double s, double gs,
+                                              double Kk) {
   const double beta_lo = a.x_norm ? __ldg(a.x_norm)
                                   : (double)__fsqrt_rd(__double2float_rd(gs));
-  if (!(fabs(s) <= dmul(__ldg(a.K + k), beta_lo))) {
+  if (!(fabs(s) <= dmul(Kk, beta_lo))) {
     const int pos = atomicAdd(a.n_cand, 1);
     a.cand[pos] = (int32_t)k;
     a.cand_s[pos] = s;
@@ -566,11 +573,14 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
   // each aligned 256-chunk: an 8-leaf tree in registers, then the butterfly
   // over lanes -- exactly the PW tree of the chunk; chunks by a 4-leaf tree.
   double q[4];
-  if (CF != CF_CSR) {
+  if (ABFT_EXP == 1 || ABFT_EXP == 2 || ABFT_EXP == 5) {
+    q[0] = q[1] = q[2] = q[3] = kAbsent;
+  } else if (CF != CF_CSR) {
     // compact C: the row is staged 16-B aligned; values and A-slot indices
     // come in with vector loads, x_j from the A pass (shared memory only)
     const unsigned char *cvb = st + c.off_cv;
     const uint16_t *cm = reinterpret_cast<const uint16_t *>(st + c.off_cc);
+    const double *xgm1 = xg - 1;  // slot + 1 indexing; xg[-1] = -0.0 (padding)
 #pragma unroll
     for (int t = 0; t < 4; ++t) {
       double v[8];
@@ -582,9 +592,9 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
           const uint4 o4 = *reinterpret_cast<const uint4 *>(cm + j0);
           const uint32_t ow[4] = {o4.x, o4.y, o4.z, o4.w};
 #pragma unroll
-          for (int u = 0; u < 8; ++u) {
+          for (int u = 0; u < 8; ++u) {  // slot + 1; 0 = padding -> -0.0 sentinel
             const int slot = (int)((ow[u >> 1] >> (16 * (u & 1))) & 0xffffu);
-            v[u] = j0 + u < nC ? dmul((double)cvv[u], xg[slot]) : kAbsent;
+            v[u] = dmul((double)cvv[u], xgm1[slot]);
           }
         } else {
 #pragma unroll
@@ -610,7 +620,8 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
       }
     }
   }
-  if (nC <= 256) {  // the common case: one chunk
+  if (ABFT_EXP == 3 || ABFT_EXP == 5) {
+  } else if (nC <= 256) {  // the common case: one chunk
 #pragma unroll
     for (int m = 1; m < 32; m <<= 1) {
       const double a0 = __shfl_xor_sync(kFull, t2, m), a1 = __shfl_xor_sync(kFull, gs, m),
@@ -637,7 +648,8 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
   }
   if (lane == 0) {
     a.gsum[g] = gs;
-    test_block_lo(a, g, dsub(t1, t2), gs);  // steps 3-4
+    if (ABFT_EXP != 4 && ABFT_EXP != 5) test_block_lo(a, g, dsub(t1, t2), gs,  // steps 3-4
+                    reinterpret_cast<const double *>(st + c.off_k)[g & 1]);
   }
 }
 
@@ -681,11 +693,12 @@ __device__ __forceinline__ void issue_stage(const SpmvArgs &a, int64_t g, int32_
     const uint32_t bac = ea4 > sa4 ? (uint32_t)(ea4 - sa4) * 4 : 0;
     const int32_t plen = (ec - sc + kCRowAlign - 1) & ~(kCRowAlign - 1);  // padded row
     const int64_t v0 = (int64_t)cc * (int64_t)sizeof(CT), k0 = (int64_t)cc * 2;
-    const uint32_t bcv = CHECK ? (uint32_t)plen * (uint32_t)sizeof(CT) : 0;
-    const uint32_t bcc = CHECK ? (uint32_t)plen * 2 : 0;
-    mbar_arrive_expect_tx(bar, 128 + 256 + bav + bac + bcv + bcc);
+    const uint32_t bcv = CHECK && ABFT_EXP != 2 ? (uint32_t)plen * (uint32_t)sizeof(CT) : 0;
+    const uint32_t bcc = CHECK && ABFT_EXP != 2 ? (uint32_t)plen * 2 : 0;
+    mbar_arrive_expect_tx(bar, 128 + 256 + (CHECK ? 16 : 0) + bav + bac + bcv + bcc);
     bulk_g2s(st + c.off_rp, a.rp + r0, 128, bar, pol);
     bulk_g2s(st + c.off_x, a.xr + r0, 256, bar, pol);
+    if (CHECK) bulk_g2s(st + c.off_k, a.K + (g & ~1ll), 16, bar, pol);
     if (bav) bulk_g2s(st + c.off_av, a.va + sa4, bav, bar, pol);
     if (bac) bulk_g2s(st + c.off_ac, a.ci + sa4, bac, bar, pol);
     if (bcv) bulk_g2s(st + c.off_cv, reinterpret_cast<const char *>(a.cval_n) + v0, bcv, bar, pol);
@@ -702,9 +715,10 @@ __device__ __forceinline__ void issue_stage(const SpmvArgs &a, int64_t g, int32_
   const uint32_t bac = ea4 > sa4 ? (uint32_t)(ea4 - sa4) * 4 : 0;
   const uint32_t bcv = CHECK && ec8 > sc8 ? (uint32_t)(ec8 - sc8) * 8 : 0;
   const uint32_t bcc = CHECK && ec4 > sc4 ? (uint32_t)(ec4 - sc4) * 4 : 0;
-  mbar_arrive_expect_tx(bar, 128 + 256 + bav + bac + bcv + bcc);
+  mbar_arrive_expect_tx(bar, 128 + 256 + (CHECK ? 16 : 0) + bav + bac + bcv + bcc);
   bulk_g2s(st + c.off_rp, a.rp + r0, 128, bar, pol);  // rp[r0 .. r0+31]; rp[r0+32] = ea
   bulk_g2s(st + c.off_x, a.xr + r0, 256, bar, pol);
+  if (CHECK) bulk_g2s(st + c.off_k, a.K + (g & ~1ll), 16, bar, pol);
   if (bav) bulk_g2s(st + c.off_av, a.va + sa4, bav, bar, pol);
   if (bac) bulk_g2s(st + c.off_ac, a.ci + sa4, bac, bar, pol);
   if (bcv) bulk_g2s(st + c.off_cv, a.cval + sc8, bcv, bar, pol);
@@ -724,6 +738,8 @@ __global__ void __launch_bounds__(kLeanWarps * 32, ABFT_LEAN_MINB) k_lean(const 
     mbar_init(bars + 1, 1);
     fence_mbar_init();
   }
+  if (CHECK && CF != CF_CSR && lane < 2)  // -0.0 sentinel below each stage's xg (padding of C)
+    reinterpret_cast<double *>(wst + (size_t)lane * c.stage_bytes + c.off_xg)[-1] = -0.0;
   __syncwarp();
   const uint64_t pol = policy_evict_first();
   const int64_t tw = (int64_t)gridDim.x * c.warps;
