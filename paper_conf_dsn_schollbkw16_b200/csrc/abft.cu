@@ -67,8 +67,7 @@ struct abft_ctx {
   int64_t nnz_c = 0;
   int32_t max_seg_a = 0, max_seg_c = 0;
   int cfmt = CF_CSR;         // format of C streamed by k_lean
-  void *cval_n = nullptr;    // compact C values
-  uint16_t *cmap = nullptr;  // compact C: A-slot index of each entry
+  unsigned char *grec = nullptr;  // compact C: one record per group (kernels_encode.cuh)
   int32_t *crp_c = nullptr;  // compact row starts (32-entry aligned)
   int64_t nnz_cpad = 0;      // compact slots incl. row padding
   StageCfg stage{};
@@ -142,8 +141,7 @@ SpmvArgs make_args(const abft_ctx *h, const double *x, double *y, const double *
   a.crp = h->c_rp;
   a.ccol = h->c_col;
   a.cval = h->c_val;
-  a.cval_n = h->cval_n;
-  a.cmap = h->cmap;
+  a.grec = h->grec;
   a.crp_c = h->crp_c;
   a.K = h->K;
   a.x = x;
@@ -429,7 +427,7 @@ abft_status init_device_once(int device) {
 }
 
 // Lossless compact C: pick the narrowest exact value
-// type and uint16 column offsets when every row spans < 65536 columns.
+// type and build the per-group records (values + A-slot map + header).
 abft_status build_compact_c(abft_ctx *h, cudaStream_t s) {
   if (h->nnz_c == 0 || h->bs != 32) return ABFT_OK;  // compact C serves the b_s = 32 fast path
   int32_t *dev = nullptr;
@@ -458,18 +456,16 @@ abft_status build_compact_c(abft_ctx *h, cudaStream_t s) {
   CK(cudaMemcpyAsync(&npad, h->crp_c + h->nb, sizeof npad, cudaMemcpyDeviceToHost, s));
   CK(cudaStreamSynchronize(s));
   h->nnz_cpad = npad;
-  char *cv = nullptr;
+  const size_t rec_bytes = (size_t)kRecHead * (size_t)h->nb + (size_t)npad * (sz + 2) + 64;
+  unsigned char *rec = nullptr;
   int32_t *bad = nullptr;
-  TRY(dalloc(h, &cv, (size_t)npad * sz + 64));
-  TRY(dalloc(h, &h->cmap, (size_t)npad + 32));
+  TRY(dalloc(h, &rec, rec_bytes));
   TRY(dalloc(h, &bad, 1));
-  CK(cudaMemsetAsync(cv, 0, (size_t)npad * sz + 64, s));
-  CK(cudaMemsetAsync(h->cmap, 0, ((size_t)npad + 32) * 2, s));
+  CK(cudaMemsetAsync(rec, 0, rec_bytes, s));
   CK(cudaMemsetAsync(bad, 0, sizeof(int32_t), s));
 #define FILL(T)                                                                              \
   k_cformat_fill<T><<<grid, 256, 0, s>>>(h->nb, h->n, h->rp, h->ci, h->c_rp, h->crp_c,        \
-                                         h->c_col, h->c_val, reinterpret_cast<T *>(cv),       \
-                                         h->cmap, bad)
+                                         h->c_col, h->c_val, rec, bad)
   switch (cf) {
     case CF_I8: FILL(int8_t); break;
     case CF_I16: FILL(int16_t); break;
@@ -477,12 +473,13 @@ abft_status build_compact_c(abft_ctx *h, cudaStream_t s) {
     default: FILL(double); break;
   }
 #undef FILL
+  k_cformat_head<<<grid, 256, 0, s>>>(h->nb, h->n, h->rp, h->K, h->crp_c, (int)sz, rec);
   int32_t hbad = 0;
   CK(cudaMemcpyAsync(&hbad, bad, sizeof hbad, cudaMemcpyDeviceToHost, s));
   CK(cudaStreamSynchronize(s));
   if (hbad) return ABFT_OK;  // some block's A segment exceeds uint16 slots: keep CSR
   CK(cudaGetLastError());
-  h->cval_n = cv;
+  h->grec = rec;
   h->cfmt = cf;
   return ABFT_OK;
 }
@@ -498,39 +495,45 @@ abft_status plan_fused(abft_ctx *h, cudaStream_t s) {
   if (!h->lean) return ABFT_OK;
   c.capA = std::min(h->max_seg_a, kCapALimit);
   c.capC = std::min(h->max_seg_c, kCapCLimit);
+  if (h->cfmt != CF_CSR) c.capC = (c.capC + kCRowAlign - 1) & ~(kCRowAlign - 1);  // padded rows
   c.nstage = 2;  // double buffering (measured best)
   int warps = kStageWarps;
   // tuning overrides (benchmark sweeps only)
   if (const char *e = getenv("ABFT_WARPS")) warps = std::max(1, std::min(kLeanWarps, atoi(e)));
   for (;;) {
     uint32_t o = 0;
-    c.off_rp = o;
-    o += 144;
-    c.off_x = o;
-    o += 256;
-    c.off_k = o;  // K[g & ~1], K[g | 1]
-    o += 16;
-    c.off_av = o;
-    o += align16((uint32_t)(c.capA + 6) * 8);
-    c.off_ac = o;
-    o += align16((uint32_t)(c.capA + 6) * 4);
-    c.off_cv = o;
     if (h->cfmt == CF_CSR) {
+      c.off_rp = o;
+      o += 144;
+      c.off_x = o;
+      o += 256;
+      c.off_k = o;  // K[g & ~1], K[g | 1]
+      o += 16;
+      c.off_av = o;
+      o += align16((uint32_t)(c.capA + 6) * 8);
+      c.off_ac = o;
+      o += align16((uint32_t)(c.capA + 6) * 4);
+      c.off_cv = o;
       o += align16((uint32_t)(c.capC + 2) * 8);
       c.off_cc = o;
       o += align16((uint32_t)(c.capC + 6) * 4);
-    } else {  // compact: a padded row of values, uint16 offsets, chunk bases
-      const uint32_t cpad = ((uint32_t)c.capC + kCRowAlign - 1) & ~(uint32_t)(kCRowAlign - 1);
-      o += align16(cpad * cf_size(h->cfmt));
-      c.off_cc = o;
-      o += align16(cpad * 2);
+      c.off_cp = o;  // padded C products (one gap per 8)
+      o += align16((uint32_t)(c.capC + c.capC / 8 + 8) * 8);
+    } else {
+      // compact: the group's record (header, values, A-slot map), the x
+      // slice, A, and the gathered x per A slot after a 16-B slot whose
+      // upper half is the -0.0 sentinel the padding entries of C select
+      c.off_rp = o;  // record
+      o += kRecHead + (uint32_t)c.capC * (uint32_t)(cf_size(h->cfmt) + 2);
+      c.off_x = o;
+      o += 256;
+      c.off_av = o;
+      o += align16((uint32_t)(c.capA + 6) * 8);
+      c.off_ac = o;
+      o += align16((uint32_t)(c.capA + 6) * 4);
+      c.off_xg = o + 16;
+      o += 16 + align16((uint32_t)(c.capA + 6) * 8);
     }
-    c.off_cp = o;  // padded C products (one gap per 8; CSR format only)
-    if (h->cfmt == CF_CSR) o += align16((uint32_t)(c.capC + c.capC / 8 + 8) * 8);
-    // gathered x per A slot (compact format only), after a 16-B slot whose
-    // upper half is the -0.0 sentinel the padding entries of C select
-    c.off_xg = o + 16;
-    if (h->cfmt != CF_CSR) o += 16 + align16((uint32_t)(c.capA + 6) * 8);
     c.stage_bytes = align16(o);
     c.bar_bytes = 128;
     h->fused_smem = c.bar_bytes + (size_t)warps * c.nstage * c.stage_bytes;
@@ -541,6 +544,7 @@ abft_status plan_fused(abft_ctx *h, cudaStream_t s) {
     } else {
       c.capA /= 2;
       c.capC /= 2;
+      if (h->cfmt != CF_CSR) c.capC &= ~(kCRowAlign - 1);
     }
   }
   c.warps = warps;
@@ -833,7 +837,9 @@ abft_status abft_info(abft_handle_t h, abft_info_t *info) {
   if (h->cfmt == CF_CSR)
     info->c_bytes = 12 * h->nnz_c + 4 * (h->nb + 1);
   else
-    info->c_bytes = (int64_t)(cf_size(h->cfmt) + 2) * h->nnz_cpad + 8 * (h->nb + 1);
+    // values + A-slot map + compact row starts (the record headers re-encode
+    // K and row_ptr, which the byte model counts once as K and A)
+    info->c_bytes = (int64_t)(cf_size(h->cfmt) + 2) * h->nnz_cpad + 4 * (h->nb + 1);
   info->groups = h->ngroups;
   info->general_groups = h->lean ? h->n_glist : h->ngroups;
   info->lean = h->lean ? 1 : 0;

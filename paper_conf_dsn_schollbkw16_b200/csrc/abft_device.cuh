@@ -40,16 +40,9 @@ __device__ __forceinline__ double bfly32(double v) {
   return v;
 }
 
-__device__ __forceinline__ int warp_max_i(int v) {
-#pragma unroll
-  for (int m = 16; m > 0; m >>= 1) v = max(v, __shfl_xor_sync(kFull, v, m));
-  return v;
-}
-__device__ __forceinline__ int warp_min_i(int v) {
-#pragma unroll
-  for (int m = 16; m > 0; m >>= 1) v = min(v, __shfl_xor_sync(kFull, v, m));
-  return v;
-}
+// one REDUX instruction each (sm_80+), not a 5-step shuffle chain
+__device__ __forceinline__ int warp_max_i(int v) { return __reduce_max_sync(kFull, v); }
+__device__ __forceinline__ int warp_min_i(int v) { return __reduce_min_sync(kFull, v); }
 
 // In-register PW tree over P leaves (P a power of two).
 template <int P>

@@ -148,23 +148,45 @@ __global__ void k_cformat_padlen(int64_t nb, const int32_t *__restrict__ crp, in
     plen[k] = (crp[k + 1] - crp[k] + kCRowAlign - 1) & ~(kCRowAlign - 1);
 }
 
-// Compact C for the staged fast path (b_s = 32): value c_kj in the narrow type
-// and, instead of its column, the staging slot of an A entry of the same
-// block with that column (slot = position in A's arrays - (rp[32k] & ~3)):
-// the fused kernel multiplies c_kj with the x_j it already gathered for A.
-// Stored as slot + 1: index 0 (the row padding, value 0) selects a -0.0
-// sentinel, so padded products are -0.0, the exact identity of the sum.
+// Compact C for the staged fast path (b_s = 32), stored as one record per
+// 32-row group so the fused kernel stages all of a group's handle-owned data
+// with ONE bulk copy:
+//
+//   [0, 8)    K_g (double)
+//   [8, 74)   ro[0..32]: row starts relative to rp[32g] (uint16)
+//   [74, 76)  max row length of the group (uint16)
+//   [76, 80)  zero
+//   [80, ..)  plen values c_kj in the narrow type T (plen = row length of C
+//             padded to 16 entries; padding values 0)
+//   [.., ..)  plen uint16 A-slot indices + 1 (0 = padding)
+//
+// Record g starts at byte 80 g + crp_c[g] (sizeof(T) + 2); every part is
+// 16-B aligned.  Instead of its column, an entry stores the staging slot of
+// an A entry of the same block with that column (slot = position in A's
+// arrays - (rp[32k] & ~3)), so the kernel multiplies c_kj with the x_j it
+// already gathered for A; slot index 0 selects a -0.0 sentinel, so padded
+// products are -0.0, the exact identity of the sum (R2).
+constexpr int kRecHead = 80;  // record header bytes
+
+__device__ __forceinline__ int64_t rec_offset(int64_t k, const int32_t *crp_c, int tsize) {
+  return (int64_t)kRecHead * k + (int64_t)crp_c[k] * (tsize + 2);
+}
+
 template <typename T>
 __global__ void k_cformat_fill(int64_t nb, int64_t n, const int32_t *__restrict__ rp,
                                const int32_t *__restrict__ ci, const int32_t *__restrict__ crp,
                                const int32_t *__restrict__ crp_c, const int32_t *__restrict__ ccol,
-                               const double *__restrict__ cval, T *cv, uint16_t *cmap,
+                               const double *__restrict__ cval, unsigned char *rec,
                                int32_t *bad) {
   const int lane = threadIdx.x & 31;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
   for (int64_t k = gw; k < nb; k += nw) {
-    const int32_t b = crp[k], e = crp[k + 1], d = crp_c[k] - b;
+    const int32_t b = crp[k], e = crp[k + 1];
+    const int32_t plen = crp_c[k + 1] - crp_c[k];
+    unsigned char *rk = rec + rec_offset(k, crp_c, (int)sizeof(T));
+    T *cv = reinterpret_cast<T *>(rk + kRecHead);
+    uint16_t *cmap = reinterpret_cast<uint16_t *>(rk + kRecHead + (int64_t)plen * sizeof(T));
     const int64_t r0 = k * 32, r1 = min64(r0 + 32, n);
     const int32_t s0 = rp[r0] & ~3;
     for (int32_t q = b + lane; q < e; q += 32) {
@@ -179,8 +201,35 @@ __global__ void k_cformat_fill(int64_t nb, int64_t n, const int32_t *__restrict_
         if (lo < rp[r + 1] && ci[lo] == j) slot = lo - s0;
       }
       if (slot < 0 || slot > 65534) atomicOr(bad, 1);
-      cv[q + d] = (T)cval[q];
-      cmap[q + d] = (uint16_t)(slot < 0 ? 0 : slot + 1);  // 0 = row padding (value 0)
+      cv[q - b] = (T)cval[q];
+      cmap[q - b] = (uint16_t)(slot < 0 ? 0 : slot + 1);  // 0 = row padding (value 0)
+    }
+  }
+}
+
+// Record headers: K_g, the group's relative row starts and its longest row
+// (one warp per group; values past 65535 only occur in groups the fused
+// kernel does not take).
+__global__ void k_cformat_head(int64_t nb, int64_t n, const int32_t *__restrict__ rp,
+                               const double *__restrict__ K, const int32_t *__restrict__ crp_c,
+                               int tsize, unsigned char *rec) {
+  const int lane = threadIdx.x & 31;
+  const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t k = gw; k < nb; k += nw) {
+    unsigned char *rk = rec + rec_offset(k, crp_c, tsize);
+    uint16_t *ro = reinterpret_cast<uint16_t *>(rk + 8);
+    const int64_t r0 = k * 32;
+    const int32_t base = rp[r0];
+    const int32_t s = rp[min64(r0 + lane, n)] - base, e = rp[min64(r0 + lane + 1, n)] - base;
+    ro[lane] = (uint16_t)min(s, 65535);
+    const int ml = warp_max_i(e - s);
+    if (lane == 0) {
+      *reinterpret_cast<double *>(rk) = K[k];
+      ro[32] = (uint16_t)min(rp[min64(r0 + 32, n)] - base, 65535);
+      ro[33] = (uint16_t)min(ml, 65535);
+      ro[34] = 0;
+      ro[35] = 0;
     }
   }
 }

@@ -75,9 +75,8 @@ struct SpmvArgs {
   const int32_t *__restrict__ crp;
   const int32_t *__restrict__ ccol;
   const double *__restrict__ cval;
-  const void *__restrict__ cval_n;       // compact C values (CF != CF_CSR)
-  const uint16_t *__restrict__ cmap;   // compact C: staging slot of an A entry, same column
-  const int32_t *__restrict__ crp_c;    // compact row starts (32-entry aligned)
+  const unsigned char *__restrict__ grec;  // compact C: per-group records (kernels_encode.cuh)
+  const int32_t *__restrict__ crp_c;    // compact row starts (16-entry aligned)
   const double *__restrict__ K;
   const double *__restrict__ x;   // gather base: column j reads x[j]
   const double *__restrict__ xr;  // row-aligned view: row i's own entry is xr[i]
@@ -469,11 +468,21 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
   const int nS = ((ea + 3) & ~3) - (sa & ~3);
   const int nC = CHECK ? ec - sc : 0;
   // row bounds first: the max-reduction's latency overlaps the gathers below
-  const int32_t rs = reinterpret_cast<const int32_t *>(st + c.off_rp)[lane];
-  int32_t re = __shfl_down_sync(kFull, rs, 1);
-  if (lane == 31) re = ea;
+  // (compact C: relative row starts and the longest row come with the record)
+  int32_t rs, re;
+  int maxlen;
+  if (CF != CF_CSR) {
+    const uint16_t *ro = reinterpret_cast<const uint16_t *>(st + c.off_rp + 8);
+    rs = sa + ro[lane];
+    re = sa + ro[lane + 1];
+    maxlen = ro[33];
+  } else {
+    rs = reinterpret_cast<const int32_t *>(st + c.off_rp)[lane];
+    re = __shfl_down_sync(kFull, rs, 1);
+    if (lane == 31) re = ea;
+    maxlen = warp_max_i(re - rs);
+  }
   const int len = re - rs;
-  const int maxlen = warp_max_i(len);
   // phase 1a: A products in place; lane l owns slots 4l + 128u .. +3
   // (128-bit shared loads/stores), 8 gathers in flight per lane.
 #pragma unroll 1
@@ -578,8 +587,8 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
   } else if (CF != CF_CSR) {
     // compact C: the row is staged 16-B aligned; values and A-slot indices
     // come in with vector loads, x_j from the A pass (shared memory only)
-    const unsigned char *cvb = st + c.off_cv;
-    const uint16_t *cm = reinterpret_cast<const uint16_t *>(st + c.off_cc);
+    const unsigned char *cvb = st + c.off_rp + kRecHead;
+    const uint16_t *cm = reinterpret_cast<const uint16_t *>(cvb + (size_t)nC * sizeof(CT));
     const double *xgm1 = xg - 1;  // slot + 1 indexing; xg[-1] = -0.0 (padding)
 #pragma unroll
     for (int t = 0; t < 4; ++t) {
@@ -637,7 +646,8 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
     for (int t = 0; t < 4; ++t)
       if (t * 256 < nC) q[t] = bfly32(q[t]);
   }
-  double t1 = nC > 0 ? tree<4>(q) : 0.0;
+  // PW over the chunk sums (one chunk: q[0] itself; an empty row: +0.0)
+  double t1 = nC > 256 ? tree<4>(q) : nC > 0 ? q[0] : 0.0;
   if (INJECT && lane == 0) {
     if (R.k0 < R.k1) t1 = apply_mask(t1, list_mask_in(a.inj, R.k0, R.k1, list_key(0, 1, g)));
     if (R.q0 < R.q1) t2 = apply_mask(t2, list_mask_in(a.inj, R.q0, R.q1, list_key(0, 2, g)));
@@ -649,7 +659,8 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
   if (lane == 0) {
     a.gsum[g] = gs;
     if (ABFT_EXP != 4 && ABFT_EXP != 5) test_block_lo(a, g, dsub(t1, t2), gs,  // steps 3-4
-                    reinterpret_cast<const double *>(st + c.off_k)[g & 1]);
+                    CF != CF_CSR ? *reinterpret_cast<const double *>(st + c.off_rp)
+                                 : reinterpret_cast<const double *>(st + c.off_k)[g & 1]);
   }
 }
 
@@ -658,22 +669,31 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
 template <int CF>
 struct Window {
   int64_t wb;
-  int32_t rpw, crpw, ccw;
+  int32_t rpw, crpw, ccw;  // CSR C uses crpw, compact C ccw
   __device__ __forceinline__ void load(const SpmvArgs &a, int64_t base, int lane) {
     wb = base;
     rpw = ld_stream(a.rp + min64((base + lane) * 32, a.n));
-    crpw = ld_stream(a.crp + min64(base + lane, a.nb));
-    if (CF != CF_CSR) ccw = ld_stream(a.crp_c + min64(base + lane, a.nb));
+    if (CF == CF_CSR)
+      crpw = ld_stream(a.crp + min64(base + lane, a.nb));
+    else
+      ccw = ld_stream(a.crp_c + min64(base + lane, a.nb));
   }
-  // sc/ec: C row bounds (CSR); cc: compact row start
+  // CSR C: sc/ec = C row bounds.  Compact C: sc = 0, ec = padded row length
+  // (so ec - sc bounds the staged entries either way), cc = compact row start
   __device__ __forceinline__ void get(int64_t g, int32_t &sa, int32_t &ea, int32_t &sc,
                                       int32_t &ec, int32_t &cc) const {
     const int j = (int)(g - wb);
     sa = __shfl_sync(kFull, rpw, j);
     ea = __shfl_sync(kFull, rpw, j + 1);
-    sc = __shfl_sync(kFull, crpw, j);
-    ec = __shfl_sync(kFull, crpw, j + 1);
-    cc = CF != CF_CSR ? __shfl_sync(kFull, ccw, j) : 0;
+    if (CF == CF_CSR) {
+      sc = __shfl_sync(kFull, crpw, j);
+      ec = __shfl_sync(kFull, crpw, j + 1);
+      cc = 0;
+    } else {
+      cc = __shfl_sync(kFull, ccw, j);
+      sc = 0;
+      ec = __shfl_sync(kFull, ccw, j + 1) - cc;
+    }
   }
 };
 
@@ -683,7 +703,7 @@ template <bool CHECK, int CF>
 __device__ __forceinline__ void issue_stage(const SpmvArgs &a, int64_t g, int32_t sa, int32_t ea,
                                             int32_t sc, int32_t ec, int32_t cc, unsigned char *st,
                                             uint64_t *bar, uint64_t pol) {
-  if (CF != CF_CSR) {
+  if (CF != CF_CSR) {  // compact C: record, x slice, A values, A columns
     using CT = typename CType<CF>::T;
     const StageCfg &c = a.sc;
     const int64_t r0 = g * 32;
@@ -691,18 +711,14 @@ __device__ __forceinline__ void issue_stage(const SpmvArgs &a, int64_t g, int32_
     const int64_t sa4 = sa & ~3, ea4 = min64((ea + 3) & ~3, nnz4);
     const uint32_t bav = ea4 > sa4 ? (uint32_t)(ea4 - sa4) * 8 : 0;
     const uint32_t bac = ea4 > sa4 ? (uint32_t)(ea4 - sa4) * 4 : 0;
-    const int32_t plen = (ec - sc + kCRowAlign - 1) & ~(kCRowAlign - 1);  // padded row
-    const int64_t v0 = (int64_t)cc * (int64_t)sizeof(CT), k0 = (int64_t)cc * 2;
-    const uint32_t bcv = CHECK && ABFT_EXP != 2 ? (uint32_t)plen * (uint32_t)sizeof(CT) : 0;
-    const uint32_t bcc = CHECK && ABFT_EXP != 2 ? (uint32_t)plen * 2 : 0;
-    mbar_arrive_expect_tx(bar, 128 + 256 + (CHECK ? 16 : 0) + bav + bac + bcv + bcc);
-    bulk_g2s(st + c.off_rp, a.rp + r0, 128, bar, pol);
+    const uint32_t brec = kRecHead + (CHECK && ABFT_EXP != 2
+                                          ? (uint32_t)ec * (uint32_t)(sizeof(CT) + 2) : 0u);
+    const unsigned char *rec = a.grec + (int64_t)kRecHead * g + (int64_t)cc * (sizeof(CT) + 2);
+    mbar_arrive_expect_tx(bar, brec + 256 + bav + bac);
+    bulk_g2s(st + c.off_rp, rec, brec, bar, pol);
     bulk_g2s(st + c.off_x, a.xr + r0, 256, bar, pol);
-    if (CHECK) bulk_g2s(st + c.off_k, a.K + (g & ~1ll), 16, bar, pol);
     if (bav) bulk_g2s(st + c.off_av, a.va + sa4, bav, bar, pol);
     if (bac) bulk_g2s(st + c.off_ac, a.ci + sa4, bac, bar, pol);
-    if (bcv) bulk_g2s(st + c.off_cv, reinterpret_cast<const char *>(a.cval_n) + v0, bcv, bar, pol);
-    if (bcc) bulk_g2s(st + c.off_cc, reinterpret_cast<const char *>(a.cmap) + k0, bcc, bar, pol);
     return;
   }
   const StageCfg &c = a.sc;
