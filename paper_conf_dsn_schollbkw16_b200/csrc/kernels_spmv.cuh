@@ -50,7 +50,7 @@ constexpr int kLeanWarps = 4;  // warps per CTA of k_lean (<= 4)
 #define ABFT_EXP 0
 #endif
 #ifndef ABFT_LEAN_MINB
-#define ABFT_LEAN_MINB 5  // min resident CTAs per SM the register budget targets (measured best)
+#define ABFT_LEAN_MINB 4  // min resident CTAs per SM the register budget targets (measured best; 5 spills)
 #endif
 
 struct StageCfg {
@@ -448,6 +448,27 @@ __device__ __forceinline__ InjRange inj_range(const InjDev &inj, int64_t g0, int
   return R;
 }
 
+// One aligned 8-leaf subtree of a lane-owned row: entries o .. o+min(len,8)-1
+// of the staged arrays; PW with absent (-0.0) leaves past the row's end.
+template <bool KEEPX>
+__device__ __forceinline__ double tpr_chunk8(const double *av, const int32_t *ac, double *xg,
+                                             int o, int len, const double *__restrict__ x) {
+  double v[8], xj[8];
+#pragma unroll
+  for (int j = 0; j < 8; ++j)
+    if (j < len) xj[j] = ld_x(x + ac[o + j]);
+#pragma unroll
+  for (int j = 0; j < 8; ++j) {
+    if (j < len) {
+      if (KEEPX) xg[o + j] = xj[j];
+      v[j] = dmul(av[o + j], xj[j]);
+    } else {
+      v[j] = kAbsent;
+    }
+  }
+  return tree<8>(v);
+}
+
 template <bool CHECK, bool INJECT, int CF>
 __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa, int32_t ea,
                                         int32_t sc, int32_t ec, unsigned char *st, int lane,
@@ -483,47 +504,83 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
     maxlen = warp_max_i(re - rs);
   }
   const int len = re - rs;
-  // phase 1a: A products in place; lane l owns slots 4l + 128u .. +3
-  // (128-bit shared loads/stores), 8 gathers in flight per lane.
+  double yv;
+  if (maxlen <= 32) {
+    // rows of <= 32 entries: lane l computes row 32g + l on its own (staged
+    // values and columns read at the row's slots -- conflict-free for the
+    // near-constant row strides of stencils; x gathers of one instruction
+    // hit 32 consecutive rows' j-th neighbours, i.e. a few lines), products
+    // stay in registers, and (compact C) the gathered x_j goes to xg[slot].
+    const int o = rs - (sa & ~3);  // staging slot of the row's first entry
+    constexpr bool KEEPX = CHECK && CF != CF_CSR;
+    if (maxlen <= 8) {
+      yv = tpr_chunk8<KEEPX>(av, ac, xg, o, len, a.x);
+    } else {
+      // 16 / 32 leaves: aligned 8-leaf subtrees one at a time (bounded
+      // register use), tree<4>((q0 + q1) + (q2 + q3)) with absent = -0.0
+      double s01 = kAbsent, s23 = kAbsent;
 #pragma unroll 1
-  for (int base = 0; base < nS; base += 256) {
-    double2 v[4];
-    int4 ci[2];
-#pragma unroll
-    for (int u = 0; u < 2; ++u) {
-      const int s0 = base + u * 128 + lane * 4;
-      if (s0 < nS) {
-        v[2 * u] = *reinterpret_cast<const double2 *>(av + s0);
-        v[2 * u + 1] = *reinterpret_cast<const double2 *>(av + s0 + 2);
-        ci[u] = *reinterpret_cast<const int4 *>(ac + s0);
+      for (int t = 0; t < 4 && len > 8 * t; ++t) {
+        const double qt = tpr_chunk8<KEEPX>(av, ac, xg, o + 8 * t, len - 8 * t, a.x);
+        if (t < 2)
+          s01 = t == 0 ? qt : dadd(s01, qt);
+        else
+          s23 = t == 2 ? qt : dadd(s23, qt);
       }
+      yv = dadd(s01, s23);
     }
+  } else {
+    // long rows: phase 1a computes every product in place (lane l owns slots
+    // 4l + 128u .. +3, 8 gathers in flight per lane), then the warp reduces
+    // each row from shared memory
+#pragma unroll 1
+    for (int base = 0; base < nS; base += 256) {
+      double2 v[4];
+      int4 ci[2];
 #pragma unroll
-    for (int u = 0; u < 2; ++u) {
-      const int s0 = base + u * 128 + lane * 4;
-      if (s0 < nS) {
-        const double x0 = ld_x(a.x + ci[u].x), x1 = ld_x(a.x + ci[u].y);
-        const double x2 = ld_x(a.x + ci[u].z), x3 = ld_x(a.x + ci[u].w);
-        if (CHECK && CF != CF_CSR) {  // keep x_j for C's entries (compact map)
-          *reinterpret_cast<double2 *>(xg + s0) = make_double2(x0, x1);
-          *reinterpret_cast<double2 *>(xg + s0 + 2) = make_double2(x2, x3);
+      for (int u = 0; u < 2; ++u) {
+        const int s0 = base + u * 128 + lane * 4;
+        if (s0 < nS) {
+          v[2 * u] = *reinterpret_cast<const double2 *>(av + s0);
+          v[2 * u + 1] = *reinterpret_cast<const double2 *>(av + s0 + 2);
+          ci[u] = *reinterpret_cast<const int4 *>(ac + s0);
         }
-        v[2 * u].x = dmul(v[2 * u].x, x0);
-        v[2 * u].y = dmul(v[2 * u].y, x1);
-        v[2 * u + 1].x = dmul(v[2 * u + 1].x, x2);
-        v[2 * u + 1].y = dmul(v[2 * u + 1].y, x3);
+      }
+#pragma unroll
+      for (int u = 0; u < 2; ++u) {
+        const int s0 = base + u * 128 + lane * 4;
+        if (s0 < nS) {
+          const double x0 = ld_x(a.x + ci[u].x), x1 = ld_x(a.x + ci[u].y);
+          const double x2 = ld_x(a.x + ci[u].z), x3 = ld_x(a.x + ci[u].w);
+          if (CHECK && CF != CF_CSR) {  // keep x_j for C's entries (compact map)
+            *reinterpret_cast<double2 *>(xg + s0) = make_double2(x0, x1);
+            *reinterpret_cast<double2 *>(xg + s0 + 2) = make_double2(x2, x3);
+          }
+          v[2 * u].x = dmul(v[2 * u].x, x0);
+          v[2 * u].y = dmul(v[2 * u].y, x1);
+          v[2 * u + 1].x = dmul(v[2 * u + 1].x, x2);
+          v[2 * u + 1].y = dmul(v[2 * u + 1].y, x3);
+        }
+      }
+#pragma unroll
+      for (int u = 0; u < 2; ++u) {
+        const int s0 = base + u * 128 + lane * 4;
+        if (s0 < nS) {
+          *reinterpret_cast<double2 *>(av + s0) = v[2 * u];
+          *reinterpret_cast<double2 *>(av + s0 + 2) = v[2 * u + 1];
+        }
       }
     }
-#pragma unroll
-    for (int u = 0; u < 2; ++u) {
-      const int s0 = base + u * 128 + lane * 4;
-      if (s0 < nS) {
-        *reinterpret_cast<double2 *>(av + s0) = v[2 * u];
-        *reinterpret_cast<double2 *>(av + s0 + 2) = v[2 * u + 1];
-      }
+    __syncwarp();
+    yv = 0.0;
+    for (int j = 0; j < 32; ++j) {
+      const int32_t rb = __shfl_sync(kFull, rs, j);
+      const int rl = __shfl_sync(kFull, len, j);
+      const double t = warp_sum_smem(smem_u32(pv + (rb - sa)), rl, lane);
+      if (lane == j) yv = t;
     }
   }
-  // phase 1b: C products into the padded layout (lane-strided, 8 gathers)
+  // phase 1b (CSR C): C products into the padded layout (lane-strided, 8 gathers)
   if (CHECK && CF == CF_CSR) {
 #pragma unroll 1
     for (int base = 0; base < nC; base += 256) {
@@ -547,27 +604,7 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
         if (u * 32 < rc) cpl[u * 36] = vc[u];
     }
   }
-  __syncwarp();
-  // y_i = PW over the row's products (lane-private tree; PW is padding
-  // independent, so P = 8 serves every row of length <= 8)
-  const double *row = pv + (rs - sa);
-  double yv;
-  if (maxlen <= 8) {
-    double v[8];
-#pragma unroll
-    for (int j = 0; j < 8; ++j) v[j] = j < len ? row[j] : kAbsent;
-    yv = tree<8>(v);
-  } else if (maxlen <= 32) {
-    yv = lane_sum_smem_any(smem_u32(row), len, maxlen);
-  } else {
-    yv = 0.0;
-    for (int j = 0; j < 32; ++j) {
-      const int32_t rb = __shfl_sync(kFull, rs, j);
-      const int rl = __shfl_sync(kFull, len, j);
-      const double t = warp_sum_smem(smem_u32(pv + (rb - sa)), rl, lane);
-      if (lane == j) yv = t;
-    }
-  }
+  if (CHECK) __syncwarp();  // xg / cp complete before the C pass reads them
   if (len == 0) yv = 0.0;  // PW of an empty row is +0.0 (R2)
   if (INJECT && R.y0 < R.y1) yv = apply_mask(yv, list_mask_in(a.inj, R.y0, R.y1, list_key(0, 0, i)));
   a.y[i] = yv;
