@@ -521,18 +521,18 @@ abft_status plan_fused(abft_ctx *h, cudaStream_t s) {
       o += align16((uint32_t)(c.capC + c.capC / 8 + 8) * 8);
     } else {
       // compact: the group's record (header, values, A-slot map), the x
-      // slice, A, and the gathered x per A slot after a 16-B slot whose
-      // upper half is the -0.0 sentinel the padding entries of C select
+      // slice, and A after a 16-B slot whose upper half is the -0.0
+      // sentinel the padding entries of C select (the kernel overwrites the
+      // staged a_ij with the gathered x_j, which C's entries index by slot)
       c.off_rp = o;  // record
       o += kRecHead + (uint32_t)c.capC * (uint32_t)(cf_size(h->cfmt) + 2);
       c.off_x = o;
-      o += 256;
+      o += 256 + 16;
       c.off_av = o;
       o += align16((uint32_t)(c.capA + 6) * 8);
       c.off_ac = o;
       o += align16((uint32_t)(c.capA + 6) * 4);
-      c.off_xg = o + 16;
-      o += 16 + align16((uint32_t)(c.capA + 6) * 8);
+      c.off_xg = c.off_av;
     }
     c.stage_bytes = align16(o);
     c.bar_bytes = 128;

@@ -450,6 +450,8 @@ __device__ __forceinline__ InjRange inj_range(const InjDev &inj, int64_t g0, int
 
 // One aligned 8-leaf subtree of a lane-owned row: entries o .. o+min(len,8)-1
 // of the staged arrays; PW with absent (-0.0) leaves past the row's end.
+// KEEPX: the gathered x_j replaces a_ij in the staged values (xg == av; each
+// slot belongs to one row, so only its owner lane touches it here).
 template <bool KEEPX>
 __device__ __forceinline__ double tpr_chunk8(const double *av, const int32_t *ac, double *xg,
                                              int o, int len, const double *__restrict__ x) {
@@ -460,8 +462,8 @@ __device__ __forceinline__ double tpr_chunk8(const double *av, const int32_t *ac
 #pragma unroll
   for (int j = 0; j < 8; ++j) {
     if (j < len) {
+      v[j] = dmul(av[o + j], xj[j]);  // a_ij read before x_j takes its slot (xg == av)
       if (KEEPX) xg[o + j] = xj[j];
-      v[j] = dmul(av[o + j], xj[j]);
     } else {
       v[j] = kAbsent;
     }
@@ -485,7 +487,7 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
   const double *cv = reinterpret_cast<const double *>(st + c.off_cv) + (sc & 1);  // sc + e
   const int32_t *cc = reinterpret_cast<const int32_t *>(st + c.off_cc) + (sc & 3);
   double *cp = reinterpret_cast<double *>(st + c.off_cp);  // C products, padded
-  double *xg = reinterpret_cast<double *>(st + c.off_xg);   // gathered x per A slot
+  double *xg = av;  // compact C, rows <= 32: gathered x_j per A slot, in place of a_ij
   const int nS = ((ea + 3) & ~3) - (sa & ~3);
   const int nC = CHECK ? ec - sc : 0;
   // row bounds first: the max-reduction's latency overlaps the gathers below
@@ -510,7 +512,8 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
     // values and columns read at the row's slots -- conflict-free for the
     // near-constant row strides of stencils; x gathers of one instruction
     // hit 32 consecutive rows' j-th neighbours, i.e. a few lines), products
-    // stay in registers, and (compact C) the gathered x_j goes to xg[slot].
+    // stay in registers, and (compact C) the gathered x_j replaces a_ij in
+    // the staged values (xg[slot], read by the C pass).
     const int o = rs - (sa & ~3);  // staging slot of the row's first entry
     constexpr bool KEEPX = CHECK && CF != CF_CSR;
     if (maxlen <= 8) {
@@ -532,7 +535,7 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
   } else {
     // long rows: phase 1a computes every product in place (lane l owns slots
     // 4l + 128u .. +3, 8 gathers in flight per lane), then the warp reduces
-    // each row from shared memory
+    // each row from shared memory; the C pass re-gathers x by column (ac)
 #pragma unroll 1
     for (int base = 0; base < nS; base += 256) {
       double2 v[4];
@@ -552,10 +555,6 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
         if (s0 < nS) {
           const double x0 = ld_x(a.x + ci[u].x), x1 = ld_x(a.x + ci[u].y);
           const double x2 = ld_x(a.x + ci[u].z), x3 = ld_x(a.x + ci[u].w);
-          if (CHECK && CF != CF_CSR) {  // keep x_j for C's entries (compact map)
-            *reinterpret_cast<double2 *>(xg + s0) = make_double2(x0, x1);
-            *reinterpret_cast<double2 *>(xg + s0 + 2) = make_double2(x2, x3);
-          }
           v[2 * u].x = dmul(v[2 * u].x, x0);
           v[2 * u].y = dmul(v[2 * u].y, x1);
           v[2 * u + 1].x = dmul(v[2 * u + 1].x, x2);
@@ -623,7 +622,8 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
     q[0] = q[1] = q[2] = q[3] = kAbsent;
   } else if (CF != CF_CSR) {
     // compact C: the row is staged 16-B aligned; values and A-slot indices
-    // come in with vector loads, x_j from the A pass (shared memory only)
+    // come in with vector loads, x_j from the A pass (in place of a_ij;
+    // groups with rows > 32 entries re-gather it by the slot's column)
     const unsigned char *cvb = st + c.off_rp + kRecHead;
     const uint16_t *cm = reinterpret_cast<const uint16_t *>(cvb + (size_t)nC * sizeof(CT));
     const double *xgm1 = xg - 1;  // slot + 1 indexing; xg[-1] = -0.0 (padding)
@@ -640,7 +640,12 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
 #pragma unroll
           for (int u = 0; u < 8; ++u) {  // slot + 1; 0 = padding -> -0.0 sentinel
             const int slot = (int)((ow[u >> 1] >> (16 * (u & 1))) & 0xffffu);
-            v[u] = dmul((double)cvv[u], xgm1[slot]);
+            double xj;
+            if (maxlen <= 32)
+              xj = xgm1[slot];
+            else
+              xj = slot ? ld_x(a.x + ac[slot - 1]) : kAbsent;
+            v[u] = dmul((double)cvv[u], xj);
           }
         } else {
 #pragma unroll
@@ -791,8 +796,8 @@ __global__ void __launch_bounds__(kLeanWarps * 32, ABFT_LEAN_MINB) k_lean(const 
     mbar_init(bars + 1, 1);
     fence_mbar_init();
   }
-  if (CHECK && CF != CF_CSR && lane < 2)  // -0.0 sentinel below each stage's xg (padding of C)
-    reinterpret_cast<double *>(wst + (size_t)lane * c.stage_bytes + c.off_xg)[-1] = -0.0;
+  if (CHECK && CF != CF_CSR && lane < 2)  // -0.0 sentinel below each stage's A values (padding of C)
+    reinterpret_cast<double *>(wst + (size_t)lane * c.stage_bytes + c.off_av)[-1] = -0.0;
   __syncwarp();
   const uint64_t pol = policy_evict_first();
   const int64_t tw = (int64_t)gridDim.x * c.warps;
