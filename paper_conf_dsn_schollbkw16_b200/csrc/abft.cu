@@ -74,6 +74,12 @@ struct abft_ctx {
   bool lean = false;        // k_lean usable (b_s = 32, 16-B aligned A)
   size_t fused_smem = 0;
   int fused_grid = 1;       // k_lean grid (persistent, one wave)
+  uint8_t *lean_ok = nullptr;  // [ngroups] groups k_lean takes
+  int64_t *hub_beg = nullptr;  // hub chunk items
+  uint32_t *hub_len = nullptr;
+  double *hub_part = nullptr;
+  int32_t *own_key = nullptr, *own_first = nullptr, *own_n = nullptr;
+  int32_t n_hub = 0, n_own = 0;
   int32_t *glist = nullptr; // groups k_lean does not take
   int64_t n_glist = 0;
   int correct_grid = 1;
@@ -160,6 +166,15 @@ SpmvArgs make_args(const abft_ctx *h, const double *x, double *y, const double *
   a.beta_valid = h->beta_valid;
   a.gbar = h->gbar;
   a.sc = h->stage;
+  a.lean_ok = h->lean_ok;
+  a.hub_beg = h->hub_beg;
+  a.hub_len = h->hub_len;
+  a.hub_part = h->hub_part;
+  a.n_hub = h->n_hub;
+  a.own_key = h->own_key;
+  a.own_first = h->own_first;
+  a.own_n = h->own_n;
+  a.n_own = h->n_own;
   return a;
 }
 
@@ -309,8 +324,9 @@ abft_status prepare_inject(abft_ctx *h, const abft_inject_t *inj, bool check, cu
   return ABFT_OK;
 }
 
-int general_grid(const abft_ctx *h, int64_t groups) {
-  return (int)std::max<int64_t>(1, std::min<int64_t>((int64_t)h->num_sms * 8, (groups + 7) / 8));
+int general_grid(const abft_ctx *h, int64_t groups) {  // kGenWarps warps per CTA
+  return (int)std::max<int64_t>(
+      1, std::min<int64_t>((int64_t)h->num_sms * 16, (groups + kGenWarps - 1) / kGenWarps));
 }
 
 template <bool CHECK, bool INJECT>
@@ -333,8 +349,10 @@ abft_status launch_fused_t(const abft_ctx *h, SpmvArgs a, cudaStream_t s) {
   a.glist = lean ? h->glist : nullptr;
   a.n_glist = ngen;
   const int ggrid = ngen > 0 ? general_grid(h, ngen) : 0;
+  if (h->n_hub > 0)  // chunk sums of hub rows, read by the group kernels
+    k_hub<<<general_grid(h, h->n_hub), kGenWarps * 32, 0, s>>>(a);
   if (lean) launch_lean<CHECK, INJECT>(h, a, s);
-  if (ggrid) k_general<CHECK, INJECT><<<ggrid, 256, 0, s>>>(a);
+  if (ggrid) k_general<CHECK, INJECT><<<ggrid, kGenWarps * 32, 0, s>>>(a);
   CK(cudaGetLastError());
   return ABFT_OK;
 }
@@ -484,90 +502,191 @@ abft_status build_compact_c(abft_ctx *h, cudaStream_t s) {
   return ABFT_OK;
 }
 
-// Stage layout and grid of k_lean, and the list of groups it does not take
-// (DESIGN.md "Kernels").  Synchronises the stream once (list length).
+// Stage layout for capacities (capA, capC).
+uint32_t stage_layout(const abft_ctx *h, StageCfg &c) {
+  uint32_t o = 0;
+  if (h->cfmt == CF_CSR) {
+    c.off_rp = o;
+    o += 144;
+    c.off_x = o;
+    o += 256;
+    c.off_k = o;  // K[g & ~1], K[g | 1]
+    o += 16;
+    c.off_av = o;
+    o += align16((uint32_t)(c.capA + 6) * 8);
+    c.off_ac = o;
+    o += align16((uint32_t)(c.capA + 6) * 4);
+    c.off_cv = o;
+    o += align16((uint32_t)(c.capC + 2) * 8);
+    c.off_cc = o;
+    o += align16((uint32_t)(c.capC + 6) * 4);
+    c.off_cp = o;  // padded C products (one gap per 8)
+    o += align16((uint32_t)(c.capC + c.capC / 8 + 8) * 8);
+  } else {
+    // compact: the group's record (header, values, A-slot map), the x
+    // slice, and A after a 16-B slot whose upper half is the -0.0
+    // sentinel the padding entries of C select (the kernel overwrites the
+    // staged a_ij with the gathered x_j, which C's entries index by slot)
+    c.off_rp = o;  // record
+    o += kRecHead + (uint32_t)c.capC * (uint32_t)(cf_size(h->cfmt) + 2);
+    c.off_x = o;
+    o += 256 + 16;
+    c.off_av = o;
+    o += align16((uint32_t)(c.capA + 6) * 8);
+    c.off_ac = o;
+    o += align16((uint32_t)(c.capA + 6) * 4);
+    c.off_xg = c.off_av;
+  }
+  return align16(o);
+}
+
+template <typename T>
+abft_status upload(abft_ctx *h, T **dst, const std::vector<T> &v, cudaStream_t s) {
+  TRY(dalloc(h, dst, v.size()));
+  if (!v.empty())
+    CK(cudaMemcpyAsync(*dst, v.data(), v.size() * sizeof(T), cudaMemcpyHostToDevice, s));
+  return ABFT_OK;
+}
+
+// Encode-time plan of the fused pass ("Long rows"):
+//  * hub rows: A rows and C rows longer than kHubLen entries, split into
+//    aligned kHubLen-entry chunks for k_hub;
+//  * the groups k_lean takes (b_s = 32, full group, every row <= 32 entries,
+//    segments within the staging capacity) -- lean_ok[g] -- and the list of
+//    the others for k_general;
+//  * k_lean's staging capacity: the largest segment, unless a capacity that
+//    still covers >= 90% of the candidate groups lets 3+ CTAs share an SM.
+// Synchronises the stream (host copies of the row pointers).
 abft_status plan_fused(abft_ctx *h, cudaStream_t s) {
   StageCfg &c = h->stage;
   memset(&c, 0, sizeof c);
   h->correct_grid = h->num_sms;  // one CTA per SM: co-resident for the grid barrier
   h->lean = h->bs == 32 && aligned16(h->rp) && aligned16(h->ci) && aligned16(h->va);
-  h->n_glist = h->ngroups;
-  if (!h->lean) return ABFT_OK;
-  c.capA = std::min(h->max_seg_a, kCapALimit);
-  c.capC = std::min(h->max_seg_c, kCapCLimit);
-  if (h->cfmt != CF_CSR) c.capC = (c.capC + kCRowAlign - 1) & ~(kCRowAlign - 1);  // padded rows
-  c.nstage = 2;  // double buffering (measured best)
-  int warps = kStageWarps;
-  // tuning overrides (benchmark sweeps only)
-  if (const char *e = getenv("ABFT_WARPS")) warps = std::max(1, std::min(kLeanWarps, atoi(e)));
-  for (;;) {
-    uint32_t o = 0;
-    if (h->cfmt == CF_CSR) {
-      c.off_rp = o;
-      o += 144;
-      c.off_x = o;
-      o += 256;
-      c.off_k = o;  // K[g & ~1], K[g | 1]
-      o += 16;
-      c.off_av = o;
-      o += align16((uint32_t)(c.capA + 6) * 8);
-      c.off_ac = o;
-      o += align16((uint32_t)(c.capA + 6) * 4);
-      c.off_cv = o;
-      o += align16((uint32_t)(c.capC + 2) * 8);
-      c.off_cc = o;
-      o += align16((uint32_t)(c.capC + 6) * 4);
-      c.off_cp = o;  // padded C products (one gap per 8)
-      o += align16((uint32_t)(c.capC + c.capC / 8 + 8) * 8);
-    } else {
-      // compact: the group's record (header, values, A-slot map), the x
-      // slice, and A after a 16-B slot whose upper half is the -0.0
-      // sentinel the padding entries of C select (the kernel overwrites the
-      // staged a_ij with the gathered x_j, which C's entries index by slot)
-      c.off_rp = o;  // record
-      o += kRecHead + (uint32_t)c.capC * (uint32_t)(cf_size(h->cfmt) + 2);
-      c.off_x = o;
-      o += 256 + 16;
-      c.off_av = o;
-      o += align16((uint32_t)(c.capA + 6) * 8);
-      c.off_ac = o;
-      o += align16((uint32_t)(c.capA + 6) * 4);
-      c.off_xg = c.off_av;
+  std::vector<int32_t> rp((size_t)h->n + 1), crp((size_t)h->nb + 1), crpc;
+  CK(cudaMemcpyAsync(rp.data(), h->rp, rp.size() * 4, cudaMemcpyDeviceToHost, s));
+  CK(cudaMemcpyAsync(crp.data(), h->c_rp, crp.size() * 4, cudaMemcpyDeviceToHost, s));
+  if (h->cfmt != CF_CSR) {
+    crpc.resize((size_t)h->nb + 1);
+    CK(cudaMemcpyAsync(crpc.data(), h->crp_c, crpc.size() * 4, cudaMemcpyDeviceToHost, s));
+  }
+  CK(cudaStreamSynchronize(s));
+  // hub rows and hub C rows, owner table sorted by (group, kind, index)
+  std::vector<int64_t> hbeg;
+  std::vector<uint32_t> hlen;
+  std::vector<std::pair<int32_t, std::pair<int32_t, int32_t>>> own;
+  auto add_hub = [&](int64_t b, int64_t len, bool crow, int32_t key) {
+    const int32_t first = (int32_t)hbeg.size();
+    for (int64_t o = 0; o < len; o += kHubLen) {
+      hbeg.push_back(b + o);
+      hlen.push_back((uint32_t)std::min<int64_t>(kHubLen, len - o) | (crow ? 1u << 31 : 0u));
     }
-    c.stage_bytes = align16(o);
-    c.bar_bytes = 128;
-    h->fused_smem = c.bar_bytes + (size_t)warps * c.nstage * c.stage_bytes;
-    if (h->fused_smem <= g_dyn_smem_limit / 2 || (warps == 1 && h->fused_smem <= g_dyn_smem_limit))
-      break;
-    if (warps > 1) {
-      warps /= 2;
+    own.push_back({key, {first, (int32_t)hbeg.size() - first}});
+  };
+  for (int64_t i = 0; i < h->n; ++i)
+    if (rp[i + 1] - rp[i] > kHubLen) add_hub(rp[i], rp[i + 1] - rp[i], false, (int32_t)((i / 32) * 64 + (i % 32)));
+  for (int64_t k = 0; k < h->nb; ++k)
+    if (crp[k + 1] - crp[k] > kHubLen) {
+      const int64_t r = k * h->bs;
+      add_hub(crp[k], crp[k + 1] - crp[k], true, (int32_t)((r / 32) * 64 + 32 + (r % 32) / h->bs));
+    }
+  std::sort(own.begin(), own.end());
+  {
+    std::vector<int32_t> ok(own.size()), of(own.size()), on(own.size());
+    for (size_t e = 0; e < own.size(); ++e) {
+      ok[e] = own[e].first;
+      of[e] = own[e].second.first;
+      on[e] = own[e].second.second;
+    }
+    TRY(upload(h, &h->hub_beg, hbeg, s));
+    TRY(upload(h, &h->hub_len, hlen, s));
+    TRY(dalloc(h, &h->hub_part, hbeg.size()));
+    TRY(upload(h, &h->own_key, ok, s));
+    TRY(upload(h, &h->own_first, of, s));
+    TRY(upload(h, &h->own_n, on, s));
+    h->n_hub = (int32_t)hbeg.size();
+    h->n_own = (int32_t)own.size();
+  }
+  // k_lean candidates: (segment, C length) per group
+  std::vector<uint8_t> lean_ok((size_t)h->ngroups, 0);
+  std::vector<int32_t> glist;
+  if (h->lean) {
+    std::vector<int32_t> segs, cls;
+    std::vector<int32_t> segA((size_t)h->ngroups, -1), segC((size_t)h->ngroups, 0);
+    for (int64_t g = 0; g < h->ngroups; ++g) {
+      if (g * 32 + 32 > h->n) continue;  // ragged last group
+      int32_t ml = 0;
+      for (int64_t i = g * 32; i < g * 32 + 32; ++i) ml = std::max(ml, rp[i + 1] - rp[i]);
+      if (ml > 32) continue;
+      segA[g] = rp[g * 32 + 32] - rp[g * 32];
+      segC[g] = h->cfmt != CF_CSR ? crpc[g + 1] - crpc[g] : crp[g + 1] - crp[g];
+      if (segA[g] > kCapALimit || segC[g] > kCapCLimit) {
+        segA[g] = -1;
+        continue;
+      }
+      segs.push_back(segA[g]);
+    }
+    if (!segs.empty()) {
+      std::vector<int32_t> sorted = segs;
+      std::sort(sorted.begin(), sorted.end());
+      auto capc_for = [&](int32_t capA) {
+        int32_t m = 0;
+        for (int64_t g = 0; g < h->ngroups; ++g)
+          if (segA[g] >= 0 && segA[g] <= capA) m = std::max(m, segC[g]);
+        if (h->cfmt != CF_CSR) m = (m + kCRowAlign - 1) & ~(kCRowAlign - 1);
+        return m;
+      };
+      const size_t per_sm = 228 * 1024;
+      int32_t capA = sorted.back();
+      int32_t capC = capc_for(capA);
+      for (double q : {1.0, 0.99, 0.95, 0.9}) {
+        StageCfg t{};
+        t.capA = sorted[(size_t)std::min<double>((double)sorted.size() - 1, q * (double)sorted.size())];
+        if (q == 1.0) t.capA = sorted.back();
+        t.capC = capc_for(t.capA);
+        const size_t smem = 128 + (size_t)kStageWarps * 2 * stage_layout(h, t);
+        if (3 * (smem + 1024) <= per_sm) {
+          capA = t.capA;
+          capC = t.capC;
+          break;
+        }
+      }
+      c.capA = capA;
+      c.capC = capC;
+      c.nstage = 2;  // double buffering (measured best)
+      int warps = kStageWarps;
+      if (const char *e = getenv("ABFT_WARPS")) warps = std::max(1, std::min(kLeanWarps, atoi(e)));
+      c.stage_bytes = stage_layout(h, c);
+      c.bar_bytes = 128;
+      h->fused_smem = c.bar_bytes + (size_t)warps * c.nstage * c.stage_bytes;
+      while (h->fused_smem > g_dyn_smem_limit && warps > 1) {
+        warps /= 2;
+        h->fused_smem = c.bar_bytes + (size_t)warps * c.nstage * c.stage_bytes;
+      }
+      if (h->fused_smem > g_dyn_smem_limit) h->lean = false;
+      c.warps = warps;
+      for (int64_t g = 0; g < h->ngroups && h->lean; ++g)
+        lean_ok[g] = segA[g] >= 0 && segA[g] <= c.capA && segC[g] <= c.capC;
     } else {
-      c.capA /= 2;
-      c.capC /= 2;
-      if (h->cfmt != CF_CSR) c.capC &= ~(kCRowAlign - 1);
+      h->lean = false;
     }
   }
-  c.warps = warps;
-  int per_sm = 0;
-  CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_lean<true, false, CF_CSR>,
-                                                   warps * 32, h->fused_smem));
-  per_sm = std::max(per_sm, 1);
-  if (const char *e = getenv("ABFT_CTAS_PER_SM")) per_sm = std::max(1, std::min(per_sm, atoi(e)));
-  const int64_t need = (h->ngroups + warps - 1) / warps;  // >= 1 group per warp
-  h->fused_grid = (int)std::max<int64_t>(1, std::min<int64_t>((int64_t)h->num_sms * per_sm, need));
-  // groups k_lean does not take
-  int32_t *count = nullptr;
-  TRY(dalloc(h, &h->glist, (size_t)h->ngroups));
-  TRY(dalloc(h, &count, 1));
-  CK(cudaMemsetAsync(count, 0, sizeof(int32_t), s));
-  SpmvArgs a = make_args(h, nullptr, nullptr, nullptr);
-  k_glist<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>((h->ngroups + 255) / 256, 4096)), 256,
-            0, s>>>(a, h->glist, count);
-  CK(cudaGetLastError());
-  int32_t cnt = 0;
-  CK(cudaMemcpyAsync(&cnt, count, sizeof cnt, cudaMemcpyDeviceToHost, s));
-  CK(cudaStreamSynchronize(s));
-  h->n_glist = cnt;
+  if (h->lean) {
+    for (int64_t g = 0; g < h->ngroups; ++g)
+      if (!lean_ok[g]) glist.push_back((int32_t)g);
+    int per_sm = 0;
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_lean<true, false, CF_CSR>,
+                                                     c.warps * 32, h->fused_smem));
+    per_sm = std::max(per_sm, 1);
+    if (const char *e = getenv("ABFT_CTAS_PER_SM")) per_sm = std::max(1, std::min(per_sm, atoi(e)));
+    const int64_t need = (h->ngroups + c.warps - 1) / c.warps;  // >= 1 group per warp
+    h->fused_grid = (int)std::max<int64_t>(1, std::min<int64_t>((int64_t)h->num_sms * per_sm, need));
+    TRY(upload(h, &h->lean_ok, lean_ok, s));
+    TRY(upload(h, &h->glist, glist, s));
+    h->n_glist = (int64_t)glist.size();
+  } else {
+    h->n_glist = h->ngroups;
+  }
+  CK(cudaStreamSynchronize(s));  // host vectors die at return
   return ABFT_OK;
 }
 

@@ -97,6 +97,18 @@ struct SpmvArgs {
   int64_t n_glist;
   double *dbg_t1, *dbg_t2;  // nullable
   const int32_t *skip;      // nullable device flag: != 0 -> kernels are no-ops (PCG)
+  const uint8_t *lean_ok;   // [ngroups] 1 = k_lean takes the group (encode-time plan)
+  // hub rows: A rows / C rows longer than kHubLen are
+  // split into aligned kHubLen-entry chunks, summed by k_hub before the fused
+  // pass; the group kernels combine the chunk sums (PW: aligned subtrees).
+  const int64_t *hub_beg;   // [n_hub] first entry of the chunk (A or C arrays)
+  const uint32_t *hub_len;  // [n_hub] entries | (1u << 31 for a C row)
+  double *hub_part;         // [n_hub] PW of the chunk's products
+  int32_t n_hub;
+  const int32_t *own_key;   // [n_own] sorted: g * 64 + (C ? 32 : 0) + row / block index in group
+  const int32_t *own_first; // [n_own] first chunk item
+  const int32_t *own_n;     // [n_own] chunk items
+  int32_t n_own;
   StageCfg sc;
   InjDev inj;
 };
@@ -253,6 +265,112 @@ __device__ __forceinline__ double warp_sum_smem(uint32_t addr, int n, int lane) 
 }
 
 // ---------------------------------------------------------------------------
+// Long rows.  kHubLen = the longest row a warp reduces
+// through its scratch in one pass; longer rows are hub rows (k_hub chunks).
+// ---------------------------------------------------------------------------
+constexpr int kHubLen = 1024;
+constexpr int kScr = kHubLen + kHubLen / 32;  // padded scratch (doubles per warp)
+constexpr int kGenWarps = 4;                  // warps per CTA of k_general / k_hub
+
+// PW over the products of entries [b, b+n), n <= kHubLen, whole warp: 256-entry
+// windows of coalesced lane-strided loads and gathers, products into the
+// warp's scratch at e + e/32 (conflict-free both ways); lane l then reduces
+// the aligned 32-entry subtree 32l..32l+31 (four 8-leaf trees and a 4-leaf
+// tree) and the butterfly joins the 32 subtrees: the PW tree of the row.
+// +0.0 when n == 0 (R2).
+template <class Src>
+__device__ __forceinline__ double warp_row_pw(const Src &s, int64_t b, int n,
+                                              const double *__restrict__ x, double *scr,
+                                              int lane) {
+  if (n <= 0) return 0.0;
+#pragma unroll 1
+  for (int w = 0; w < n; w += 256) {
+    double v[8];
+    int c[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      const int e = w + u * 32 + lane;
+      if (e < n) {
+        v[u] = s.val(b + e);
+        c[u] = s.col(b + e);
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      const int e = w + u * 32 + lane;
+      if (e < n) scr[e + (e >> 5)] = dmul(v[u], ld_x(x + c[u]));
+    }
+  }
+  __syncwarp();
+  const int e0 = lane * 32;
+  const double *p = scr + lane * 33;
+  double q[4];
+#pragma unroll
+  for (int t = 0; t < 4; ++t) {
+    double v[8];
+#pragma unroll
+    for (int j = 0; j < 8; ++j) v[j] = e0 + 8 * t + j < n ? p[8 * t + j] : kAbsent;
+    q[t] = tree<8>(v);
+  }
+  const double r = bfly32(tree<4>(q));
+  __syncwarp();  // scratch reusable
+  return r;
+}
+
+// Chunk sums of hub items (one warp per item; items are independent).
+__global__ void __launch_bounds__(kGenWarps * 32) k_hub(const SpmvArgs a) {
+  __shared__ double scr_all[kGenWarps][kScr];
+  if (a.skip && *(volatile const int32_t *)a.skip != 0) return;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t q = gw; q < a.n_hub; q += nw) {
+    const uint32_t L = __ldg(a.hub_len + q);
+    const int64_t b = __ldg(a.hub_beg + q);
+    const int n = (int)(L & 0x7fffffffu);
+    double r;
+    if (L >> 31) {
+      struct { const double *v; const int32_t *c;
+        __device__ double val(int64_t e) const { return ld_stream(v + e); }
+        __device__ int32_t col(int64_t e) const { return ld_stream(c + e); } } Cs{a.cval, a.ccol};
+      r = warp_row_pw(Cs, b, n, a.x, scr_all[warp], lane);
+    } else {
+      struct { const double *v; const int32_t *c;
+        __device__ double val(int64_t e) const { return ld_stream(v + e); }
+        __device__ int32_t col(int64_t e) const { return ld_stream(c + e); } } As{a.va, a.ci};
+      r = warp_row_pw(As, b, n, a.x, scr_all[warp], lane);
+    }
+    if (lane == 0) a.hub_part[q] = r;
+  }
+}
+
+// PW over a hub row's chunk sums (aligned kHubLen-subtrees, in order).
+__device__ __forceinline__ double hub_sum(const SpmvArgs &a, int32_t first, int32_t cnt) {
+  PwSeq acc;
+  for (int32_t t = 0; t < cnt; ++t) acc.push(__ldcg(a.hub_part + first + t));
+  return acc.finish();
+}
+
+// Range [lo, hi) of the group's entries in the sorted owner table.
+__device__ __forceinline__ void own_range(const SpmvArgs &a, int64_t g, int &lo, int &hi) {
+  lo = hi = 0;
+  if (a.n_own == 0) return;
+  const int32_t k0 = (int32_t)(g * 64), k1 = (int32_t)(g * 64 + 64);
+  int l = 0, r = a.n_own;
+  while (l < r) {
+    const int m = (l + r) >> 1;
+    if (__ldg(a.own_key + m) < k0) l = m + 1; else r = m;
+  }
+  lo = l;
+  r = a.n_own;
+  while (l < r) {
+    const int m = (l + r) >> 1;
+    if (__ldg(a.own_key + m) < k1) l = m + 1; else r = m;
+  }
+  hi = l;
+}
+
+// ---------------------------------------------------------------------------
 // Candidate test (step 4 pre-filter) shared by both kernels.
 // ---------------------------------------------------------------------------
 __device__ __forceinline__ void test_block(const SpmvArgs &a, int64_t k, double s, double gs) {
@@ -284,7 +402,7 @@ __device__ __forceinline__ void test_block_lo(const SpmvArgs &a, int64_t k, doub
 // General path: one group, operands from global memory (any b_s <= 32).
 // ---------------------------------------------------------------------------
 template <bool CHECK, bool INJECT>
-__device__ __forceinline__ void group_general(const SpmvArgs &a, int64_t g, int lane) {
+__device__ __forceinline__ void group_general(const SpmvArgs &a, int64_t g, int lane, double *scr) {
   const int64_t n = a.n;
   const int64_t r0 = g * 32;
   const int64_t i = r0 + lane;
@@ -298,18 +416,30 @@ __device__ __forceinline__ void group_general(const SpmvArgs &a, int64_t g, int 
   }
   const GlobalSrc As{a.va, a.ci}, Cs{a.cval, a.ccol};
   const int len = re - rs;
-  const int maxlen = warp_max_i(len);
+  // hub rows / hub C rows of this group (rare: an empty range almost always)
+  int olo, ohi;
+  own_range(a, g, olo, ohi);
+  bool hub = false;
   double yv = 0.0;
-  if (maxlen <= 32) {
-    if (valid) yv = lane_dot_any(As, rs, len, maxlen, a.x);
-  } else {
-    for (int j = 0; j < 32; ++j) {
-      const int32_t rb = __shfl_sync(kFull, rs, j);
-      const int rl = __shfl_sync(kFull, len, j);
-      if (r0 + j >= n) break;
-      const double t = warp_dot(As, rb, rl, a.x, lane);
-      if (lane == j) yv = t;
+  for (int e = olo; e < ohi; ++e) {
+    const int32_t key = __ldg(a.own_key + e);
+    if ((key & 63) == lane) {  // A row 32g + lane (key & 32 == 0)
+      hub = true;
+      yv = hub_sum(a, __ldg(a.own_first + e), __ldg(a.own_n + e));
     }
+  }
+  // row-length-adaptive y: rows <= 32 entries lane-private (an aligned tree of
+  // P = 2^ceil(log2 maxlen) leaves), longer ones by the warp (warp_row_pw)
+  const bool small = !hub && len <= 32;
+  const int maxs = warp_max_i(small ? len : 0);
+  if (small && valid) yv = lane_dot_any(As, rs, len, maxs, a.x);
+  unsigned longm = __ballot_sync(kFull, valid && !hub && len > 32);
+  while (longm) {
+    const int j = __ffs(longm) - 1;
+    longm &= longm - 1;
+    const double t = warp_row_pw(As, __shfl_sync(kFull, rs, j), __shfl_sync(kFull, len, j), a.x,
+                                 scr, lane);
+    if (lane == j) yv = t;
   }
   if (len == 0) yv = 0.0;  // PW of an empty row is +0.0 (R2)
   if (INJECT) {
@@ -322,7 +452,7 @@ __device__ __forceinline__ void group_general(const SpmvArgs &a, int64_t g, int 
   // step 2: t2_k = w_k^T y_k over the b_s slots; absent past n.
   double t2 = bfly(valid ? yv : kAbsent, a.bs);
   // step 1: t1_k = c_k . x: the 32/b_s C rows of the group,
-  // lane-per-C-row when short, warp-cooperative otherwise.
+  // lane-per-C-row when short, warp-cooperative otherwise, hub rows by chunks.
   const int bl = lane >> a.log2bs;
   const int64_t k = (r0 >> a.log2bs) + bl;
   const bool leader = ((lane & (a.bs - 1)) == 0) && valid;
@@ -334,19 +464,28 @@ __device__ __forceinline__ void group_general(const SpmvArgs &a, int64_t g, int 
     ce = __ldg(a.crp + kl + 1);
   }
   const int nkl = ce - cb;
-  const int maxnk = warp_max_i(nkl);
+  bool chub = false;
   double t1l = 0.0;
-  if (nblk > 1 && maxnk <= 32) {
-    if (lane < nblk) t1l = lane_dot_any(Cs, cb, nkl, maxnk, a.x);
-    if (nkl == 0) t1l = 0.0;
-  } else {
-    for (int l = 0; l < nblk; ++l) {
-      const int32_t b = __shfl_sync(kFull, cb, l);
-      const int m = __shfl_sync(kFull, nkl, l);
-      const double t = warp_dot(Cs, b, m, a.x, lane);
-      if (lane == l) t1l = t;
+  for (int e = olo; e < ohi; ++e) {
+    const int32_t key = __ldg(a.own_key + e);
+    if ((key & 32) && (key & 31) == lane) {
+      chub = true;
+      t1l = hub_sum(a, __ldg(a.own_first + e), __ldg(a.own_n + e));
     }
   }
+  const bool csmall = nblk > 1 && !chub && nkl <= 32;
+  const int maxnk = warp_max_i(csmall ? nkl : 0);
+  if (csmall && lane < nblk) t1l = lane_dot_any(Cs, cb, nkl, maxnk, a.x);
+  unsigned cl = __ballot_sync(kFull, lane < nblk && !chub && !csmall);
+  while (cl) {
+    const int l = __ffs(cl) - 1;
+    cl &= cl - 1;
+    const int32_t b = __shfl_sync(kFull, cb, l);
+    const int m = __shfl_sync(kFull, nkl, l);
+    const double t = warp_row_pw(Cs, b, m, a.x, scr, lane);
+    if (lane == l) t1l = t;
+  }
+  if (nkl == 0) t1l = 0.0;
   double t1 = __shfl_sync(kFull, t1l, bl);
   const int nk = __shfl_sync(kFull, nkl, bl);
   if (INJECT && leader) {
@@ -363,14 +502,15 @@ __device__ __forceinline__ void group_general(const SpmvArgs &a, int64_t g, int 
 }
 
 template <bool CHECK, bool INJECT>
-__global__ void __launch_bounds__(256) k_general(const SpmvArgs a) {
+__global__ void __launch_bounds__(kGenWarps * 32) k_general(const SpmvArgs a) {
+  __shared__ double scr_all[kGenWarps][kScr];
   if (skip_call(a)) return;
   const int lane = threadIdx.x & 31;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
   for (int64_t q = gw; q < a.n_glist; q += nw) {
     const int64_t g = a.glist ? (int64_t)__ldg(a.glist + q) : q;
-    group_general<CHECK, INJECT>(a, g, lane);
+    group_general<CHECK, INJECT>(a, g, lane, scr_all[threadIdx.x >> 5]);
   }
 }
 
@@ -379,10 +519,6 @@ __global__ void __launch_bounds__(256) k_general(const SpmvArgs a) {
 // is addressed through pointers derived from the kernel's shared array (so
 // guarded accesses compile to predicated LDS/STS, not branches).
 // ---------------------------------------------------------------------------
-__device__ __forceinline__ bool lean_eligible(const SpmvArgs &a, int64_t g, int32_t sa,
-                                              int32_t ea, int32_t sc, int32_t ec) {
-  return (g * 32 + 32) <= a.n && (ea - sa) <= a.sc.capA && (ec - sc) <= a.sc.capC;
-}
 
 // Eight consecutive elements of a 16-B aligned staged compact-C row.
 __device__ __forceinline__ void load8(int8_t (&v)[8], const unsigned char *p) {
@@ -479,16 +615,13 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
   const StageCfg &c = a.sc;
   const int64_t i = g * 32 + lane;
   // A: values and columns staged on the same 4-element grid from sa & ~3, so
-  // slot s holds element (sa & ~3) + s in both arrays; slots [0, nS) were
-  // copied (gap slots hold real neighbouring entries -- valid columns).
+  // slot s holds element (sa & ~3) + s in both arrays.
   double *av = reinterpret_cast<double *>(st + c.off_av);
   const int32_t *ac = reinterpret_cast<const int32_t *>(st + c.off_ac);
-  double *pv = av + (sa & 3);  // product of element sa + e at pv[e]
   const double *cv = reinterpret_cast<const double *>(st + c.off_cv) + (sc & 1);  // sc + e
   const int32_t *cc = reinterpret_cast<const int32_t *>(st + c.off_cc) + (sc & 3);
   double *cp = reinterpret_cast<double *>(st + c.off_cp);  // C products, padded
   double *xg = av;  // compact C, rows <= 32: gathered x_j per A slot, in place of a_ij
-  const int nS = ((ea + 3) & ~3) - (sa & ~3);
   const int nC = CHECK ? ec - sc : 0;
   // row bounds first: the max-reduction's latency overlaps the gathers below
   // (compact C: relative row starts and the longest row come with the record)
@@ -507,8 +640,9 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
   }
   const int len = re - rs;
   double yv;
-  if (maxlen <= 32) {
-    // rows of <= 32 entries: lane l computes row 32g + l on its own (staged
+  {
+    // rows of <= 32 entries (the encode-time plan gives k_lean no group with
+    // a longer row): lane l computes row 32g + l on its own (staged
     // values and columns read at the row's slots -- conflict-free for the
     // near-constant row strides of stencils; x gathers of one instruction
     // hit 32 consecutive rows' j-th neighbours, i.e. a few lines), products
@@ -531,52 +665,6 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
           s23 = t == 2 ? qt : dadd(s23, qt);
       }
       yv = dadd(s01, s23);
-    }
-  } else {
-    // long rows: phase 1a computes every product in place (lane l owns slots
-    // 4l + 128u .. +3, 8 gathers in flight per lane), then the warp reduces
-    // each row from shared memory; the C pass re-gathers x by column (ac)
-#pragma unroll 1
-    for (int base = 0; base < nS; base += 256) {
-      double2 v[4];
-      int4 ci[2];
-#pragma unroll
-      for (int u = 0; u < 2; ++u) {
-        const int s0 = base + u * 128 + lane * 4;
-        if (s0 < nS) {
-          v[2 * u] = *reinterpret_cast<const double2 *>(av + s0);
-          v[2 * u + 1] = *reinterpret_cast<const double2 *>(av + s0 + 2);
-          ci[u] = *reinterpret_cast<const int4 *>(ac + s0);
-        }
-      }
-#pragma unroll
-      for (int u = 0; u < 2; ++u) {
-        const int s0 = base + u * 128 + lane * 4;
-        if (s0 < nS) {
-          const double x0 = ld_x(a.x + ci[u].x), x1 = ld_x(a.x + ci[u].y);
-          const double x2 = ld_x(a.x + ci[u].z), x3 = ld_x(a.x + ci[u].w);
-          v[2 * u].x = dmul(v[2 * u].x, x0);
-          v[2 * u].y = dmul(v[2 * u].y, x1);
-          v[2 * u + 1].x = dmul(v[2 * u + 1].x, x2);
-          v[2 * u + 1].y = dmul(v[2 * u + 1].y, x3);
-        }
-      }
-#pragma unroll
-      for (int u = 0; u < 2; ++u) {
-        const int s0 = base + u * 128 + lane * 4;
-        if (s0 < nS) {
-          *reinterpret_cast<double2 *>(av + s0) = v[2 * u];
-          *reinterpret_cast<double2 *>(av + s0 + 2) = v[2 * u + 1];
-        }
-      }
-    }
-    __syncwarp();
-    yv = 0.0;
-    for (int j = 0; j < 32; ++j) {
-      const int32_t rb = __shfl_sync(kFull, rs, j);
-      const int rl = __shfl_sync(kFull, len, j);
-      const double t = warp_sum_smem(smem_u32(pv + (rb - sa)), rl, lane);
-      if (lane == j) yv = t;
     }
   }
   // phase 1b (CSR C): C products into the padded layout (lane-strided, 8 gathers)
@@ -622,8 +710,7 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
     q[0] = q[1] = q[2] = q[3] = kAbsent;
   } else if (CF != CF_CSR) {
     // compact C: the row is staged 16-B aligned; values and A-slot indices
-    // come in with vector loads, x_j from the A pass (in place of a_ij;
-    // groups with rows > 32 entries re-gather it by the slot's column)
+    // come in with vector loads, x_j from the A pass (in place of a_ij)
     const unsigned char *cvb = st + c.off_rp + kRecHead;
     const uint16_t *cm = reinterpret_cast<const uint16_t *>(cvb + (size_t)nC * sizeof(CT));
     const double *xgm1 = xg - 1;  // slot + 1 indexing; xg[-1] = -0.0 (padding)
@@ -640,12 +727,7 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
 #pragma unroll
           for (int u = 0; u < 8; ++u) {  // slot + 1; 0 = padding -> -0.0 sentinel
             const int slot = (int)((ow[u >> 1] >> (16 * (u & 1))) & 0xffffu);
-            double xj;
-            if (maxlen <= 32)
-              xj = xgm1[slot];
-            else
-              xj = slot ? ld_x(a.x + ac[slot - 1]) : kAbsent;
-            v[u] = dmul((double)cvv[u], xj);
+            v[u] = dmul((double)cvv[u], xgm1[slot]);
           }
         } else {
 #pragma unroll
@@ -712,13 +794,18 @@ template <int CF>
 struct Window {
   int64_t wb;
   int32_t rpw, crpw, ccw;  // CSR C uses crpw, compact C ccw
+  int32_t okw;             // lean_ok of group wb + lane
   __device__ __forceinline__ void load(const SpmvArgs &a, int64_t base, int lane) {
     wb = base;
+    okw = a.lean_ok[min64(base + lane, a.ngroups - 1)];
     rpw = ld_stream(a.rp + min64((base + lane) * 32, a.n));
     if (CF == CF_CSR)
       crpw = ld_stream(a.crp + min64(base + lane, a.nb));
     else
       ccw = ld_stream(a.crp_c + min64(base + lane, a.nb));
+  }
+  __device__ __forceinline__ bool ok(int64_t g) const {
+    return __shfl_sync(kFull, okw, (int)(g - wb)) != 0;
   }
   // CSR C: sc/ec = C row bounds.  Compact C: sc = 0, ec = padded row length
   // (so ec - sc bounds the staged entries either way), cc = compact row start
@@ -810,7 +897,7 @@ __global__ void __launch_bounds__(kLeanWarps * 32, ABFT_LEAN_MINB) k_lean(const 
   win.load(a, g0, lane);
   int32_t sa, ea, sc, ec, cc;  // bounds of the current group, carried from its prefetch
   win.get(g0, sa, ea, sc, ec, cc);
-  bool elig = lean_eligible(a, g0, sa, ea, sc, ec);
+  bool elig = win.ok(g0);
   if (lane == 0 && elig) issue_stage<CHECK, CF>(a, g0, sa, ea, sc, ec, cc, wst, bars, pol);
   uint32_t phase = 0;  // bit s = parity of stage s's next completion
   for (int64_t g = g0; g < g1; ++g) {
@@ -820,7 +907,7 @@ __global__ void __launch_bounds__(kLeanWarps * 32, ABFT_LEAN_MINB) k_lean(const 
     if (g + 1 < g1) {  // prefetch g + 1 into the other stage
       if (g + 2 > win.wb + 31) win.load(a, g, lane);
       win.get(g + 1, nsa, nea, nsc, nec, ncc);
-      nelig = lean_eligible(a, g + 1, nsa, nea, nsc, nec);
+      nelig = win.ok(g + 1);
       if (lane == 0 && nelig)
         issue_stage<CHECK, CF>(a, g + 1, nsa, nea, nsc, nec, ncc,
                                wst + (size_t)(s ^ 1) * c.stage_bytes, bars + (s ^ 1), pol);
@@ -849,16 +936,6 @@ __global__ void __launch_bounds__(kLeanWarps * 32, ABFT_LEAN_MINB) k_lean(const 
     ec = nec;
     cc = ncc;
     elig = nelig;
-  }
-}
-
-// Encode-time helper: the groups k_lean does not take (appended, unordered).
-__global__ void k_glist(const SpmvArgs a, int32_t *glist, int32_t *count) {
-  for (int64_t g = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; g < a.ngroups;
-       g += (int64_t)gridDim.x * blockDim.x) {
-    const int32_t sa = a.rp[min64(g * 32, a.n)], ea = a.rp[min64(g * 32 + 32, a.n)];
-    const int32_t sc = a.crp[min64(g, a.nb)], ec = a.crp[min64(g + 1, a.nb)];
-    if (!lean_eligible(a, g, sa, ea, sc, ec)) glist[atomicAdd(count, 1)] = (int32_t)g;
   }
 }
 

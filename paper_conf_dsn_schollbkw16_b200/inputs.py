@@ -248,6 +248,25 @@ def random_csr(n: int, density: float, seed: int, integer: bool = False,
     return CSR(row_ptr.astype(np.int32), cols.astype(np.int32), vals, f"rand{n}_{density}")
 
 
+def hub_csr(n: int, seed: int, hub_lens=(1500, 4100), mid_frac: float = 0.08,
+            mid_len=(33, 400), short_len=(0, 12)) -> CSR:
+    """Random square CSR with every row-length class of the fused kernels:
+    short rows (<= 32 entries), medium rows (33..1024) and hub rows (> 1024
+    entries, split into chunks), placed at fixed rows; values ~ U[-1,1)."""
+    rng = np.random.Generator(np.random.PCG64(seed))
+    lens = rng.integers(short_len[0], short_len[1] + 1, size=n)
+    mid = rng.random(n) < mid_frac
+    lens[mid] = rng.integers(mid_len[0], mid_len[1] + 1, size=int(mid.sum()))
+    for t, L in enumerate(hub_lens):
+        lens[(37 + t * (n // 2 + 5)) % n] = min(L, n)
+    cols = [np.sort(rng.choice(n, size=int(L), replace=False)) for L in lens]
+    row_ptr = np.zeros(n + 1, dtype=np.int64)
+    np.cumsum(lens, out=row_ptr[1:])
+    col = np.concatenate(cols).astype(np.int32) if n else np.zeros(0, np.int32)
+    val = rng.uniform(-1.0, 1.0, size=col.shape[0])
+    return CSR(row_ptr.astype(np.int32), col, val, f"hub{n}")
+
+
 def burst_mask(start_bit: int, length: int) -> int:
     """XOR mask of a burst of `length` flipped bits starting at `start_bit`,
     truncated at bit 63 (no wrap) -- SURVEY.md §8(c) Q12 reading of P:196."""

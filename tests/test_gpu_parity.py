@@ -108,6 +108,7 @@ MATRICES = {
     "rand_dense": lambda: G.random_csr(300, 0.3, 4),        # rows > 32: warp fallback
     "rmat11": lambda: G.rmat(11, 16, 5),                    # power law, long rows
     "rmat11_natural": lambda: G.rmat(11, 8, 6, permute=False),  # empty blocks
+    "hubs": lambda: G.hub_csr(5000, 11),                    # rows / C rows > 1024: hub chunks
     "tiny1": lambda: G.CSR([0, 1], [0], [2.5]),
     "tiny33": lambda: G.random_csr(33, 0.2, 9),
     "all_empty": lambda: G.CSR(np.zeros(101, np.int32), np.zeros(0, np.int32), np.zeros(0)),
@@ -126,7 +127,7 @@ def test_encode_and_spmv_error_free(O, torch_cuda, name, c_csr):
 
 
 @pytest.mark.parametrize("bs", [1, 2, 4, 8, 16])
-@pytest.mark.parametrize("name", ["lap3d_ragged", "rmat11", "rand_dense"])
+@pytest.mark.parametrize("name", ["lap3d_ragged", "rmat11", "rand_dense", "hubs"])
 def test_block_sizes(O, torch_cuda, name, bs):
     A = MATRICES[name]()
     c = Case(O, torch_cuda, A, bs=bs)
@@ -135,6 +136,21 @@ def test_block_sizes(O, torch_cuda, name, bs):
     plan = G.FaultPlan([0, 0, 0], [0, 1, 2], [A.n // 2, 1, c.enc.nb - 1], [1 << 62, 1 << 61, 1 << 60])
     ref = c.run(G.uniform_vector(A.n, 8), plan=plan)
     assert ref.flagged.size >= 1
+
+
+@pytest.mark.parametrize("c_csr", [False, True])
+def test_hub_rows_faults(O, torch_cuda, c_csr):
+    """Faults in hub rows (> 1024 entries, chunked by k_hub) and in the
+    checksums of blocks whose C row is a hub: flagged, localized, corrected."""
+    A = MATRICES["hubs"]()
+    c = Case(O, torch_cuda, A, c_csr=c_csr)
+    hub_rows = np.nonzero(np.diff(A.row_ptr) > 1024)[0]
+    assert hub_rows.size >= 2
+    kb = int(hub_rows[1]) // 32
+    plan = G.FaultPlan([0, 0, 0, 1], [0, 0, 1, 0], [int(hub_rows[0]), int(hub_rows[1]) , kb, 5],
+                       [1 << 62, 1 << 55, 1 << 60, 1 << 61])
+    ref = c.run(G.uniform_vector(A.n, 21), plan=plan)
+    assert set(ref.flags[0].tolist()) >= {int(hub_rows[0]) // 32, kb}
 
 
 def test_single_bit_flips_config0(O, torch_cuda):
