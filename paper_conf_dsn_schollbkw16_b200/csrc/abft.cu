@@ -670,9 +670,11 @@ abft_status plan_fused(abft_ctx *h, cudaStream_t s) {
       h->lean = false;
     }
   }
+  for (const auto &o : own) lean_ok[(size_t)(o.first >> 6)] |= 2;  // groups owning hub rows
+  TRY(upload(h, &h->lean_ok, lean_ok, s));
   if (h->lean) {
     for (int64_t g = 0; g < h->ngroups; ++g)
-      if (!lean_ok[g]) glist.push_back((int32_t)g);
+      if (!(lean_ok[g] & 1)) glist.push_back((int32_t)g);
     int per_sm = 0;
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_lean<true, false, CF_CSR>,
                                                      c.warps * 32, h->fused_smem));
@@ -680,7 +682,6 @@ abft_status plan_fused(abft_ctx *h, cudaStream_t s) {
     if (const char *e = getenv("ABFT_CTAS_PER_SM")) per_sm = std::max(1, std::min(per_sm, atoi(e)));
     const int64_t need = (h->ngroups + c.warps - 1) / c.warps;  // >= 1 group per warp
     h->fused_grid = (int)std::max<int64_t>(1, std::min<int64_t>((int64_t)h->num_sms * per_sm, need));
-    TRY(upload(h, &h->lean_ok, lean_ok, s));
     TRY(upload(h, &h->glist, glist, s));
     h->n_glist = (int64_t)glist.size();
   } else {

@@ -97,7 +97,7 @@ struct SpmvArgs {
   int64_t n_glist;
   double *dbg_t1, *dbg_t2;  // nullable
   const int32_t *skip;      // nullable device flag: != 0 -> kernels are no-ops (PCG)
-  const uint8_t *lean_ok;   // [ngroups] 1 = k_lean takes the group (encode-time plan)
+  const uint8_t *lean_ok;   // [ngroups] bit 0: k_lean takes the group; bit 1: it owns hub rows
   // hub rows: A rows / C rows longer than kHubLen are
   // split into aligned kHubLen-entry chunks, summed by k_hub before the fused
   // pass; the group kernels combine the chunk sums (PW: aligned subtrees).
@@ -195,16 +195,23 @@ __device__ __forceinline__ double lane_dot(const Src &s, int64_t b, int len,
   if constexpr (P <= 8) {
     return lane_dot8<P>(s, b, len, x);
   } else {
-    double q[P / 8];
-#pragma unroll
-    for (int t = 0; t < P / 8; ++t)
-      q[t] = (t * 8 < len) ? lane_dot8<8>(s, b + t * 8, len - t * 8, x) : kAbsent;
-    return tree<P / 8>(q);
+    // aligned 8-leaf subtrees one at a time (bounded register use):
+    // tree<4>((q0 + q1) + (q2 + q3)), absent subtrees = -0.0 (P = 16: q2 = q3 absent)
+    double s01 = kAbsent, s23 = kAbsent;
+#pragma unroll 1
+    for (int t = 0; t < P / 8 && t * 8 < len; ++t) {
+      const double qt = lane_dot8<8>(s, b + t * 8, len - t * 8, x);
+      if (t < 2)
+        s01 = t == 0 ? qt : dadd(s01, qt);
+      else
+        s23 = t == 2 ? qt : dadd(s23, qt);
+    }
+    return dadd(s01, s23);
   }
 }
 
 template <class Src>
-__device__ __forceinline__ double lane_dot_any(const Src &s, int64_t b, int len, int maxlen,
+__device__ __noinline__ double lane_dot_any(const Src &s, int64_t b, int len, int maxlen,
                                                const double *__restrict__ x) {
   if (maxlen <= 1) return lane_dot<1>(s, b, len, x);
   if (maxlen <= 2) return lane_dot<2>(s, b, len, x);
@@ -272,23 +279,23 @@ constexpr int kHubLen = 1024;
 constexpr int kScr = kHubLen + kHubLen / 32;  // padded scratch (doubles per warp)
 constexpr int kGenWarps = 4;                  // warps per CTA of k_general / k_hub
 
-// PW over the products of entries [b, b+n), n <= kHubLen, whole warp: 256-entry
+// PW over the products of entries [b, b+n), n <= kHubLen, whole warp: 32U-entry
 // windows of coalesced lane-strided loads and gathers, products into the
 // warp's scratch at e + e/32 (conflict-free both ways); lane l then reduces
 // the aligned 32-entry subtree 32l..32l+31 (four 8-leaf trees and a 4-leaf
 // tree) and the butterfly joins the 32 subtrees: the PW tree of the row.
 // +0.0 when n == 0 (R2).
-template <class Src>
-__device__ __forceinline__ double warp_row_pw(const Src &s, int64_t b, int n,
+template <int U, class Src>
+__device__ __noinline__ double warp_row_pw(const Src &s, int64_t b, int n,
                                               const double *__restrict__ x, double *scr,
                                               int lane) {
   if (n <= 0) return 0.0;
 #pragma unroll 1
-  for (int w = 0; w < n; w += 256) {
-    double v[8];
-    int c[8];
+  for (int w = 0; w < n; w += 32 * U) {  // U loads, then U gathers in flight per lane
+    double v[U];
+    int c[U];
 #pragma unroll
-    for (int u = 0; u < 8; ++u) {
+    for (int u = 0; u < U; ++u) {
       const int e = w + u * 32 + lane;
       if (e < n) {
         v[u] = s.val(b + e);
@@ -296,7 +303,7 @@ __device__ __forceinline__ double warp_row_pw(const Src &s, int64_t b, int n,
       }
     }
 #pragma unroll
-    for (int u = 0; u < 8; ++u) {
+    for (int u = 0; u < U; ++u) {
       const int e = w + u * 32 + lane;
       if (e < n) scr[e + (e >> 5)] = dmul(v[u], ld_x(x + c[u]));
     }
@@ -333,19 +340,19 @@ __global__ void __launch_bounds__(kGenWarps * 32) k_hub(const SpmvArgs a) {
       struct { const double *v; const int32_t *c;
         __device__ double val(int64_t e) const { return ld_stream(v + e); }
         __device__ int32_t col(int64_t e) const { return ld_stream(c + e); } } Cs{a.cval, a.ccol};
-      r = warp_row_pw(Cs, b, n, a.x, scr_all[warp], lane);
+      r = warp_row_pw<16>(Cs, b, n, a.x, scr_all[warp], lane);
     } else {
       struct { const double *v; const int32_t *c;
         __device__ double val(int64_t e) const { return ld_stream(v + e); }
         __device__ int32_t col(int64_t e) const { return ld_stream(c + e); } } As{a.va, a.ci};
-      r = warp_row_pw(As, b, n, a.x, scr_all[warp], lane);
+      r = warp_row_pw<16>(As, b, n, a.x, scr_all[warp], lane);
     }
     if (lane == 0) a.hub_part[q] = r;
   }
 }
 
 // PW over a hub row's chunk sums (aligned kHubLen-subtrees, in order).
-__device__ __forceinline__ double hub_sum(const SpmvArgs &a, int32_t first, int32_t cnt) {
+__device__ __noinline__ double hub_sum(const SpmvArgs &a, int32_t first, int32_t cnt) {
   PwSeq acc;
   for (int32_t t = 0; t < cnt; ++t) acc.push(__ldcg(a.hub_part + first + t));
   return acc.finish();
@@ -417,8 +424,8 @@ __device__ __forceinline__ void group_general(const SpmvArgs &a, int64_t g, int 
   const GlobalSrc As{a.va, a.ci}, Cs{a.cval, a.ccol};
   const int len = re - rs;
   // hub rows / hub C rows of this group (rare: an empty range almost always)
-  int olo, ohi;
-  own_range(a, g, olo, ohi);
+  int olo = 0, ohi = 0;
+  if (a.lean_ok[g] & 2) own_range(a, g, olo, ohi);  // bit 1: the group owns hub rows
   bool hub = false;
   double yv = 0.0;
   for (int e = olo; e < ohi; ++e) {
@@ -437,7 +444,7 @@ __device__ __forceinline__ void group_general(const SpmvArgs &a, int64_t g, int 
   while (longm) {
     const int j = __ffs(longm) - 1;
     longm &= longm - 1;
-    const double t = warp_row_pw(As, __shfl_sync(kFull, rs, j), __shfl_sync(kFull, len, j), a.x,
+    const double t = warp_row_pw<8>(As, __shfl_sync(kFull, rs, j), __shfl_sync(kFull, len, j), a.x,
                                  scr, lane);
     if (lane == j) yv = t;
   }
@@ -482,7 +489,7 @@ __device__ __forceinline__ void group_general(const SpmvArgs &a, int64_t g, int 
     cl &= cl - 1;
     const int32_t b = __shfl_sync(kFull, cb, l);
     const int m = __shfl_sync(kFull, nkl, l);
-    const double t = warp_row_pw(Cs, b, m, a.x, scr, lane);
+    const double t = warp_row_pw<8>(Cs, b, m, a.x, scr, lane);
     if (lane == l) t1l = t;
   }
   if (nkl == 0) t1l = 0.0;
@@ -502,7 +509,7 @@ __device__ __forceinline__ void group_general(const SpmvArgs &a, int64_t g, int 
 }
 
 template <bool CHECK, bool INJECT>
-__global__ void __launch_bounds__(kGenWarps * 32) k_general(const SpmvArgs a) {
+__global__ void __launch_bounds__(kGenWarps * 32, 4) k_general(const SpmvArgs a) {
   __shared__ double scr_all[kGenWarps][kScr];
   if (skip_call(a)) return;
   const int lane = threadIdx.x & 31;
@@ -805,7 +812,7 @@ struct Window {
       ccw = ld_stream(a.crp_c + min64(base + lane, a.nb));
   }
   __device__ __forceinline__ bool ok(int64_t g) const {
-    return __shfl_sync(kFull, okw, (int)(g - wb)) != 0;
+    return (__shfl_sync(kFull, okw, (int)(g - wb)) & 1) != 0;
   }
   // CSR C: sc/ec = C row bounds.  Compact C: sc = 0, ec = padded row length
   // (so ec - sc bounds the staged entries either way), cc = compact row start
