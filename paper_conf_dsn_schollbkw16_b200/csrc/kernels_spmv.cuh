@@ -50,7 +50,7 @@ constexpr int kLeanWarps = 4;  // warps per CTA of k_lean (<= 4)
 #define ABFT_EXP 0
 #endif
 #ifndef ABFT_LEAN_MINB
-#define ABFT_LEAN_MINB 4  // min resident CTAs per SM the register budget targets (measured best; 5 spills)
+#define ABFT_LEAN_MINB 5  // min resident CTAs per SM the register budget targets (measured best)
 #endif
 
 struct StageCfg {
