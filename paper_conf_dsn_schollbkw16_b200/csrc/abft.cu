@@ -332,13 +332,17 @@ int general_grid(const abft_ctx *h, int64_t groups) {  // kGenWarps warps per CT
 template <bool CHECK, bool INJECT>
 void launch_lean(const abft_ctx *h, const SpmvArgs &a, cudaStream_t s) {
   const dim3 grid(h->fused_grid), block(h->stage.warps * 32);
+#define LEAN(CF)                                                                      \
+  (h->stage.nstage == 3 ? k_lean<CHECK, INJECT, CF, 3><<<grid, block, h->fused_smem, s>>>(a) \
+                        : k_lean<CHECK, INJECT, CF, 2><<<grid, block, h->fused_smem, s>>>(a))
   switch (h->cfmt) {
-    case CF_I8: k_lean<CHECK, INJECT, CF_I8><<<grid, block, h->fused_smem, s>>>(a); break;
-    case CF_I16: k_lean<CHECK, INJECT, CF_I16><<<grid, block, h->fused_smem, s>>>(a); break;
-    case CF_F32: k_lean<CHECK, INJECT, CF_F32><<<grid, block, h->fused_smem, s>>>(a); break;
-    case CF_F64: k_lean<CHECK, INJECT, CF_F64><<<grid, block, h->fused_smem, s>>>(a); break;
-    default: k_lean<CHECK, INJECT, CF_CSR><<<grid, block, h->fused_smem, s>>>(a); break;
+    case CF_I8: LEAN(CF_I8); break;
+    case CF_I16: LEAN(CF_I16); break;
+    case CF_F32: LEAN(CF_F32); break;
+    case CF_F64: LEAN(CF_F64); break;
+    default: LEAN(CF_CSR); break;
   }
+#undef LEAN
 }
 
 template <bool CHECK, bool INJECT>
@@ -411,10 +415,14 @@ abft_status set_smem_attrs(Kern kern, int optin) {
 
 template <int CF>
 abft_status set_lean_attrs(int optin) {
-  TRY(set_smem_attrs(k_lean<true, true, CF>, optin));
-  TRY(set_smem_attrs(k_lean<true, false, CF>, optin));
-  TRY(set_smem_attrs(k_lean<false, true, CF>, optin));
-  TRY(set_smem_attrs(k_lean<false, false, CF>, optin));
+  TRY(set_smem_attrs(k_lean<true, true, CF, 2>, optin));
+  TRY(set_smem_attrs(k_lean<true, false, CF, 2>, optin));
+  TRY(set_smem_attrs(k_lean<false, true, CF, 2>, optin));
+  TRY(set_smem_attrs(k_lean<false, false, CF, 2>, optin));
+  TRY(set_smem_attrs(k_lean<true, true, CF, 3>, optin));
+  TRY(set_smem_attrs(k_lean<true, false, CF, 3>, optin));
+  TRY(set_smem_attrs(k_lean<false, true, CF, 3>, optin));
+  TRY(set_smem_attrs(k_lean<false, false, CF, 3>, optin));
   return ABFT_OK;
 }
 
@@ -515,7 +523,7 @@ uint32_t stage_layout(const abft_ctx *h, StageCfg &c) {
     c.off_av = o;
     o += align16((uint32_t)(c.capA + 6) * 8);
     c.off_ac = o;
-    o += align16((uint32_t)(c.capA + 6) * 4);
+    o += align16((uint32_t)(c.capA + 6 + 8) * 4);  // + 8: unpredicated column reads past a row
     c.off_cv = o;
     o += align16((uint32_t)(c.capC + 2) * 8);
     c.off_cc = o;
@@ -534,7 +542,7 @@ uint32_t stage_layout(const abft_ctx *h, StageCfg &c) {
     c.off_av = o;
     o += align16((uint32_t)(c.capA + 6) * 8);
     c.off_ac = o;
-    o += align16((uint32_t)(c.capA + 6) * 4);
+    o += align16((uint32_t)(c.capA + 6 + 8) * 4);  // + 8: unpredicated column reads past a row
     c.off_xg = c.off_av;
   }
   return align16(o);
@@ -652,11 +660,14 @@ abft_status plan_fused(abft_ctx *h, cudaStream_t s) {
       }
       c.capA = capA;
       c.capC = capC;
-      c.nstage = 2;  // double buffering (measured best)
       int warps = kStageWarps;
       if (const char *e = getenv("ABFT_WARPS")) warps = std::max(1, std::min(kLeanWarps, atoi(e)));
       c.stage_bytes = stage_layout(h, c);
       c.bar_bytes = 128;
+      // three stages (gathers one group ahead) when 5 CTAs still fit an SM,
+      // else double buffering
+      c.nstage = (c.bar_bytes + (size_t)warps * 3 * c.stage_bytes + 1024) * 5 <= per_sm ? 3 : 2;
+      if (const char *e = getenv("ABFT_STAGES")) c.nstage = atoi(e) == 3 ? 3 : 2;
       h->fused_smem = c.bar_bytes + (size_t)warps * c.nstage * c.stage_bytes;
       while (h->fused_smem > g_dyn_smem_limit && warps > 1) {
         warps /= 2;
@@ -676,7 +687,7 @@ abft_status plan_fused(abft_ctx *h, cudaStream_t s) {
     for (int64_t g = 0; g < h->ngroups; ++g)
       if (!(lean_ok[g] & 1)) glist.push_back((int32_t)g);
     int per_sm = 0;
-    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_lean<true, false, CF_CSR>,
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_lean<true, false, CF_CSR, 2>,
                                                      c.warps * 32, h->fused_smem));
     per_sm = std::max(per_sm, 1);
     if (const char *e = getenv("ABFT_CTAS_PER_SM")) per_sm = std::max(1, std::min(per_sm, atoi(e)));

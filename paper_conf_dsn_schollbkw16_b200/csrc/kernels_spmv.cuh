@@ -595,29 +595,101 @@ __device__ __forceinline__ InjRange inj_range(const InjDev &inj, int64_t g0, int
 // of the staged arrays; PW with absent (-0.0) leaves past the row's end.
 // KEEPX: the gathered x_j replaces a_ij in the staged values (xg == av; each
 // slot belongs to one row, so only its owner lane touches it here).
-template <bool KEEPX>
-__device__ __forceinline__ double tpr_chunk8(const double *av, const int32_t *ac, double *xg,
-                                             int o, int len, const double *__restrict__ x) {
-  double v[8], xj[8];
+__device__ __forceinline__ void tpr_gather8(const int32_t *ac, int o, int len,
+                                            const double *__restrict__ x, double (&xj)[8]) {
+  const int32_t *acp = ac + o;
 #pragma unroll
   for (int j = 0; j < 8; ++j)
-    if (j < len) xj[j] = ld_x(x + ac[o + j]);
+    if (j < len) xj[j] = ld_x(x + acp[j]);
+}
+
+// PW over the leaves v[0 .. len) of an 8-leaf tree: a node whose right
+// subtree is absent passes its left one through (== -0.0 padding, R2), so
+// absent leaves are never read and need no value.
+__device__ __forceinline__ double tree8_len(double (&v)[8], int len) {
+  if (len > 1) v[0] = dadd(v[0], v[1]);
+  if (len > 3) v[2] = dadd(v[2], v[3]);
+  if (len > 5) v[4] = dadd(v[4], v[5]);
+  if (len > 7) v[6] = dadd(v[6], v[7]);
+  if (len > 2) v[0] = dadd(v[0], v[2]);
+  if (len > 6) v[4] = dadd(v[4], v[6]);
+  if (len > 4) v[0] = dadd(v[0], v[4]);
+  return v[0];  // meaningful when len > 0
+}
+
+template <bool KEEPX>
+__device__ __forceinline__ double tpr_finish8(const double *av, double *xg, int o, int len,
+                                              const double (&xj)[8]) {
+  double v[8];
+  const double *avp = av + o;
+  double *xgp = xg + o;
 #pragma unroll
   for (int j = 0; j < 8; ++j) {
     if (j < len) {
-      v[j] = dmul(av[o + j], xj[j]);  // a_ij read before x_j takes its slot (xg == av)
-      if (KEEPX) xg[o + j] = xj[j];
-    } else {
-      v[j] = kAbsent;
+      v[j] = dmul(avp[j], xj[j]);  // a_ij read before x_j takes its slot (xg == av)
+      if (KEEPX) xgp[j] = xj[j];
     }
   }
+#pragma unroll
+  for (int j = 0; j < 8; ++j)
+    if (j >= len) v[j] = kAbsent;
   return tree<8>(v);
+}
+template <bool KEEPX>
+__device__ __forceinline__ double tpr_chunk8(const double *av, const int32_t *ac, double *xg,
+                                             int o, int len, const double *__restrict__ x) {
+  double xj[8];
+  tpr_gather8(ac, o, len, x, xj);
+  return tpr_finish8<KEEPX>(av, xg, o, len, xj);
+}
+
+// A group's row bounds and, for rows of <= 8 entries, its x gathers already
+// in flight (k_lean issues them one group ahead: their L2 latency overlaps
+// the previous group's C pass and butterflies).
+struct Pre {
+  int32_t rs, re;
+  int maxlen;
+  double xj[8];
+};
+
+// Row bounds of staged group g (+ the gathers when every row has <= 8
+// entries).  Also stages the A slots past the arrays' last 4-element
+// boundary, which the bulk copy cannot cover.
+template <int CF>
+__device__ __forceinline__ void pregather(const SpmvArgs &a, int32_t sa, int32_t ea,
+                                          unsigned char *st, int lane, Pre &p) {
+  const StageCfg &c = a.sc;
+  if (ea > (a.nnz & ~3ll)) {  // A slots past the arrays' last 4-element boundary
+    const int64_t nnz4 = a.nnz & ~3ll;
+    const int64_t e = nnz4 + lane;  // slots of elements nnz4 .. nnz4+3
+    if (lane < 4 && e >= (sa & ~3)) {
+      const bool real = e < a.nnz;
+      reinterpret_cast<int32_t *>(st + c.off_ac)[e - (sa & ~3)] = real ? __ldg(a.ci + e) : 0;
+      reinterpret_cast<double *>(st + c.off_av)[e - (sa & ~3)] = real ? __ldg(a.va + e) : 0.0;
+    }
+    __syncwarp();
+  }
+  // compact C: relative row starts and the longest row come with the record
+  if (CF != CF_CSR) {
+    const uint16_t *ro = reinterpret_cast<const uint16_t *>(st + c.off_rp + 8);
+    p.rs = sa + ro[lane];
+    p.re = sa + ro[lane + 1];
+    p.maxlen = ro[33];
+  } else {
+    p.rs = reinterpret_cast<const int32_t *>(st + c.off_rp)[lane];
+    p.re = __shfl_down_sync(kFull, p.rs, 1);
+    if (lane == 31) p.re = ea;
+    p.maxlen = warp_max_i(p.re - p.rs);
+  }
+  if (p.maxlen <= 8)
+    tpr_gather8(reinterpret_cast<const int32_t *>(st + c.off_ac), p.rs - (sa & ~3), p.re - p.rs,
+                a.x, p.xj);
 }
 
 template <bool CHECK, bool INJECT, int CF>
 __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa, int32_t ea,
                                         int32_t sc, int32_t ec, unsigned char *st, int lane,
-                                        const InjRange &R) {
+                                        const InjRange &R, const Pre &p) {
   using CT = typename CType<CF>::T;
   const StageCfg &c = a.sc;
   const int64_t i = g * 32 + lane;
@@ -630,22 +702,9 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
   double *cp = reinterpret_cast<double *>(st + c.off_cp);  // C products, padded
   double *xg = av;  // compact C, rows <= 32: gathered x_j per A slot, in place of a_ij
   const int nC = CHECK ? ec - sc : 0;
-  // row bounds first: the max-reduction's latency overlaps the gathers below
-  // (compact C: relative row starts and the longest row come with the record)
-  int32_t rs, re;
-  int maxlen;
-  if (CF != CF_CSR) {
-    const uint16_t *ro = reinterpret_cast<const uint16_t *>(st + c.off_rp + 8);
-    rs = sa + ro[lane];
-    re = sa + ro[lane + 1];
-    maxlen = ro[33];
-  } else {
-    rs = reinterpret_cast<const int32_t *>(st + c.off_rp)[lane];
-    re = __shfl_down_sync(kFull, rs, 1);
-    if (lane == 31) re = ea;
-    maxlen = warp_max_i(re - rs);
-  }
-  const int len = re - rs;
+  const int32_t rs = p.rs;
+  const int maxlen = p.maxlen;
+  const int len = p.re - p.rs;
   double yv;
   {
     // rows of <= 32 entries (the encode-time plan gives k_lean no group with
@@ -658,7 +717,7 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
     const int o = rs - (sa & ~3);  // staging slot of the row's first entry
     constexpr bool KEEPX = CHECK && CF != CF_CSR;
     if (maxlen <= 8) {
-      yv = tpr_chunk8<KEEPX>(av, ac, xg, o, len, a.x);
+      yv = tpr_finish8<KEEPX>(av, xg, o, len, p.xj);  // gathers issued by pregather
     } else {
       // 16 / 32 leaves: aligned 8-leaf subtrees one at a time (bounded
       // register use), tree<4>((q0 + q1) + (q2 + q3)) with absent = -0.0
@@ -723,27 +782,22 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
     const double *xgm1 = xg - 1;  // slot + 1 indexing; xg[-1] = -0.0 (padding)
 #pragma unroll
     for (int t = 0; t < 4; ++t) {
-      double v[8];
       const int j0 = t * 256 + lane * 8;
-      if (t * 256 < nC) {
-        if (j0 < nC) {
-          CT cvv[8];
-          load8(cvv, cvb + (size_t)j0 * sizeof(CT));
-          const uint4 o4 = *reinterpret_cast<const uint4 *>(cm + j0);
-          const uint32_t ow[4] = {o4.x, o4.y, o4.z, o4.w};
+      double qt = kAbsent;  // rows are padded to 16 entries: a lane's 8 are all in or all out
+      if (j0 < nC) {
+        double v[8];
+        CT cvv[8];
+        load8(cvv, cvb + (size_t)j0 * sizeof(CT));
+        const uint4 o4 = *reinterpret_cast<const uint4 *>(cm + j0);
+        const uint32_t ow[4] = {o4.x, o4.y, o4.z, o4.w};
 #pragma unroll
-          for (int u = 0; u < 8; ++u) {  // slot + 1; 0 = padding -> -0.0 sentinel
-            const int slot = (int)((ow[u >> 1] >> (16 * (u & 1))) & 0xffffu);
-            v[u] = dmul((double)cvv[u], xgm1[slot]);
-          }
-        } else {
-#pragma unroll
-          for (int u = 0; u < 8; ++u) v[u] = kAbsent;
+        for (int u = 0; u < 8; ++u) {  // slot + 1; 0 = padding -> -0.0 sentinel
+          const int slot = (int)((ow[u >> 1] >> (16 * (u & 1))) & 0xffffu);
+          v[u] = dmul((double)cvv[u], xgm1[slot]);
         }
-        q[t] = tree<8>(v);
-      } else {
-        q[t] = kAbsent;
+        qt = tree<8>(v);
       }
+      q[t] = qt;
     }
   } else {
 #pragma unroll
@@ -877,20 +931,23 @@ __device__ __forceinline__ void issue_stage(const SpmvArgs &a, int64_t g, int32_
   if (bcc) bulk_g2s(st + c.off_cc, a.ccol + sc4, bcc, bar, pol);
 }
 
-template <bool CHECK, bool INJECT, int CF>
+// NST = 2: double buffering, each group's gathers issued right before its
+// products.  NST = 3 (small stages): prefetch distance 2, and group g+1's x
+// gathers are issued before group g's products, C pass and butterflies.
+template <bool CHECK, bool INJECT, int CF, int NST>
 __global__ void __launch_bounds__(kLeanWarps * 32, ABFT_LEAN_MINB) k_lean(const SpmvArgs a) {
   extern __shared__ __align__(128) unsigned char smem[];
   if (skip_call(a)) return;
   const StageCfg &c = a.sc;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  uint64_t *bars = reinterpret_cast<uint64_t *>(smem) + warp * 2;
-  unsigned char *wst = smem + c.bar_bytes + (size_t)warp * 2 * c.stage_bytes;
+  uint64_t *bars = reinterpret_cast<uint64_t *>(smem) + warp * NST;
+  unsigned char *wst = smem + c.bar_bytes + (size_t)warp * NST * c.stage_bytes;
   if (lane == 0) {
-    mbar_init(bars, 1);
-    mbar_init(bars + 1, 1);
+#pragma unroll
+    for (int t = 0; t < NST; ++t) mbar_init(bars + t, 1);
     fence_mbar_init();
   }
-  if (CHECK && CF != CF_CSR && lane < 2)  // -0.0 sentinel below each stage's A values (padding of C)
+  if (CHECK && CF != CF_CSR && lane < NST)  // -0.0 sentinel below each stage's A values (padding of C)
     reinterpret_cast<double *>(wst + (size_t)lane * c.stage_bytes + c.off_av)[-1] = -0.0;
   __syncwarp();
   const uint64_t pol = policy_evict_first();
@@ -902,47 +959,83 @@ __global__ void __launch_bounds__(kLeanWarps * 32, ABFT_LEAN_MINB) k_lean(const 
   if (INJECT) R = inj_range(a.inj, g0, g1, lane);
   Window<CF> win;
   win.load(a, g0, lane);
-  int32_t sa, ea, sc, ec, cc;  // bounds of the current group, carried from its prefetch
+  // bounds of groups g (and g + 1 for NST = 3), carried from their prefetch
+  int32_t sa, ea, sc, ec, cc, sa1 = 0, ea1 = 0, sc1 = 0, ec1 = 0, cc1 = 0;
   win.get(g0, sa, ea, sc, ec, cc);
-  bool elig = win.ok(g0);
+  bool elig = win.ok(g0), elig1 = false;
   if (lane == 0 && elig) issue_stage<CHECK, CF>(a, g0, sa, ea, sc, ec, cc, wst, bars, pol);
   uint32_t phase = 0;  // bit s = parity of stage s's next completion
-  for (int64_t g = g0; g < g1; ++g) {
-    const int s = (int)(g - g0) & 1;
-    int32_t nsa = 0, nea = 0, nsc = 0, nec = 0, ncc = 0;
-    bool nelig = false;
-    if (g + 1 < g1) {  // prefetch g + 1 into the other stage
-      if (g + 2 > win.wb + 31) win.load(a, g, lane);
-      win.get(g + 1, nsa, nea, nsc, nec, ncc);
-      nelig = win.ok(g + 1);
-      if (lane == 0 && nelig)
-        issue_stage<CHECK, CF>(a, g + 1, nsa, nea, nsc, nec, ncc,
-                               wst + (size_t)(s ^ 1) * c.stage_bytes, bars + (s ^ 1), pol);
+  Pre pc;
+  if (NST == 3) {
+    if (g0 + 1 < g1) {
+      win.get(g0 + 1, sa1, ea1, sc1, ec1, cc1);
+      elig1 = win.ok(g0 + 1);
+      if (lane == 0 && elig1)
+        issue_stage<CHECK, CF>(a, g0 + 1, sa1, ea1, sc1, ec1, cc1, wst + c.stage_bytes, bars + 1, pol);
     }
     if (elig) {
-      unsigned char *st = wst + (size_t)s * c.stage_bytes;
-      mbar_wait(bars + s, (phase >> s) & 1u);
-      phase ^= 1u << s;
-      if (ea > (a.nnz & ~3ll)) {  // A slots past the arrays' last 4-element boundary
-        const int64_t nnz4 = a.nnz & ~3ll;
-        const int64_t e = nnz4 + lane;  // slots of elements nnz4 .. nnz4+3
-        if (lane < 4 && e >= (sa & ~3)) {
-          const bool real = e < a.nnz;
-          reinterpret_cast<int32_t *>(st + c.off_ac)[e - (sa & ~3)] = real ? __ldg(a.ci + e) : 0;
-          reinterpret_cast<double *>(st + c.off_av)[e - (sa & ~3)] = real ? __ldg(a.va + e) : 0.0;
-        }
-        __syncwarp();
-      }
-      group32<CHECK, INJECT, CF>(a, g, sa, ea, sc, ec, st, lane, R);
-      __syncwarp();
-      fence_proxy_async_smem();  // generic accesses of this stage precede its next bulk write
+      mbar_wait(bars, 0);
+      phase ^= 1u;
+      pregather<CF>(a, sa, ea, wst, lane, pc);
     }
-    sa = nsa;
-    ea = nea;
-    sc = nsc;
-    ec = nec;
-    cc = ncc;
-    elig = nelig;
+  }
+  int s = 0;  // stage of group g
+  for (int64_t g = g0; g < g1; ++g) {
+    const int s1 = s + 1 == NST ? 0 : s + 1;
+    if (NST == 2) {
+      int32_t nsa = 0, nea = 0, nsc = 0, nec = 0, ncc = 0;
+      bool nelig = false;
+      if (g + 1 < g1) {  // prefetch g + 1 into the other stage
+        if (g + 2 > win.wb + 31) win.load(a, g, lane);
+        win.get(g + 1, nsa, nea, nsc, nec, ncc);
+        nelig = win.ok(g + 1);
+        if (lane == 0 && nelig)
+          issue_stage<CHECK, CF>(a, g + 1, nsa, nea, nsc, nec, ncc, wst + (size_t)s1 * c.stage_bytes,
+                                 bars + s1, pol);
+      }
+      if (elig) {
+        unsigned char *st = wst + (size_t)s * c.stage_bytes;
+        mbar_wait(bars + s, (phase >> s) & 1u);
+        phase ^= 1u << s;
+        pregather<CF>(a, sa, ea, st, lane, pc);
+        group32<CHECK, INJECT, CF>(a, g, sa, ea, sc, ec, st, lane, R, pc);
+        __syncwarp();
+        fence_proxy_async_smem();  // generic accesses of this stage precede its next bulk write
+      }
+      sa = nsa; ea = nea; sc = nsc; ec = nec; cc = ncc;
+      elig = nelig;
+    } else {
+      const int s2 = s1 + 1 == NST ? 0 : s1 + 1;
+      int32_t nsa = 0, nea = 0, nsc = 0, nec = 0, ncc = 0;
+      bool nelig = false;
+      if (g + 2 < g1) {  // prefetch g + 2 into the stage group g - 1 used
+        if (g + 3 > win.wb + 31) win.load(a, g + 2, lane);
+        win.get(g + 2, nsa, nea, nsc, nec, ncc);
+        nelig = win.ok(g + 2);
+        if (lane == 0 && nelig)
+          issue_stage<CHECK, CF>(a, g + 2, nsa, nea, nsc, nec, ncc, wst + (size_t)s2 * c.stage_bytes,
+                                 bars + s2, pol);
+      }
+      Pre pn;
+      if (elig1) {  // group g + 1: row bounds and x gathers in flight
+        unsigned char *st1 = wst + (size_t)s1 * c.stage_bytes;
+        mbar_wait(bars + s1, (phase >> s1) & 1u);
+        phase ^= 1u << s1;
+        pregather<CF>(a, sa1, ea1, st1, lane, pn);
+      }
+      if (elig) {
+        unsigned char *st = wst + (size_t)s * c.stage_bytes;
+        group32<CHECK, INJECT, CF>(a, g, sa, ea, sc, ec, st, lane, R, pc);
+        __syncwarp();
+        fence_proxy_async_smem();  // generic accesses of this stage precede its next bulk write
+      }
+      pc = pn;
+      sa = sa1; ea = ea1; sc = sc1; ec = ec1; cc = cc1;
+      elig = elig1;
+      sa1 = nsa; ea1 = nea; sc1 = nsc; ec1 = nec; cc1 = ncc;
+      elig1 = nelig;
+    }
+    s = s1;
   }
 }
 
