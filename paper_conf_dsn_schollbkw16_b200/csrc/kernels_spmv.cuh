@@ -390,13 +390,19 @@ __device__ __forceinline__ void test_block(const SpmvArgs &a, int64_t k, double 
   }
 }
 
-// Same test with a cheaper exact lower bound of beta_g: gs rounded down to
-// float, square root rounded down -- beta_lo <= sqrt(gs) <= beta, so the
-// pre-filter stays exact (a passing block provably passes against tau_k).
+// Same test with a cheaper exact lower bound of beta_g: for gs in [2^e,
+// 2^(e+1)), beta_lo = 2^floor(e/2) <= sqrt(gs) <= beta (0 for zero,
+// subnormal, Inf or NaN gs), so the pre-filter stays exact (a passing block
+// provably passes against tau_k; the rest are confirmed by k_finish).
+__device__ __forceinline__ double beta_lower(double gs) {
+  const int hi = __double2hiint(gs);
+  const int ef = (hi >> 20) & 0x7ff;
+  const int h = (ef - 1023) >> 1;  // floor(e / 2)
+  return (ef == 0 || ef == 0x7ff) ? 0.0 : __hiloint2double((h + 1023) << 20, 0);
+}
 __device__ __forceinline__ void test_block_lo(const SpmvArgs &a, int64_t k, double s, double gs,
                                               double Kk) {
-  const double beta_lo = a.x_norm ? __ldg(a.x_norm)
-                                  : (double)__fsqrt_rd(__double2float_rd(gs));
+  const double beta_lo = a.x_norm ? __ldg(a.x_norm) : beta_lower(gs);
   if (!(fabs(s) <= dmul(Kk, beta_lo))) {
     const int pos = atomicAdd(a.n_cand, 1);
     a.cand[pos] = (int32_t)k;
@@ -780,8 +786,13 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
     const unsigned char *cvb = st + c.off_rp + kRecHead;
     const uint16_t *cm = reinterpret_cast<const uint16_t *>(cvb + (size_t)nC * sizeof(CT));
     const double *xgm1 = xg - 1;  // slot + 1 indexing; xg[-1] = -0.0 (padding)
+    const int nt = nC <= 256 ? 1 : 4;  // uniform: one 256-chunk in the common case
 #pragma unroll
     for (int t = 0; t < 4; ++t) {
+      if (t >= nt) {
+        q[t] = kAbsent;
+        continue;
+      }
       const int j0 = t * 256 + lane * 8;
       double qt = kAbsent;  // rows are padded to 16 entries: a lane's 8 are all in or all out
       if (j0 < nC) {
@@ -815,15 +826,22 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
     }
   }
   if (ABFT_EXP == 3 || ABFT_EXP == 5) {
-  } else if (nC <= 256) {  // the common case: one chunk
+  } else if (nC <= 256) {
+    // the common case, one chunk: the three butterflies as one reduce-scatter
+    // (levels 1 and 2 split the values over lane pairs, levels 3-5 are plain
+    // butterflies) -- each value still sees the ascending-offset pairing of
+    // PW; afterwards lane 4m holds t2, 4m+1 t1's chunk and 4m+2 the x^2 sum
+    const bool b0 = lane & 1, b1 = lane & 2;
+    const double s0 = b0 ? t2 : q[0], s1 = b0 ? gs : kAbsent;  // sent at level 1
+    const double k0 = b0 ? q[0] : t2, k1 = b0 ? kAbsent : gs;  // kept
+    const double r0 = dadd(k0, __shfl_xor_sync(kFull, s0, 1));
+    const double r1 = dadd(k1, __shfl_xor_sync(kFull, s1, 1));
+    double v = dadd(b1 ? r1 : r0, __shfl_xor_sync(kFull, b1 ? r0 : r1, 2));
 #pragma unroll
-    for (int m = 1; m < 32; m <<= 1) {
-      const double a0 = __shfl_xor_sync(kFull, t2, m), a1 = __shfl_xor_sync(kFull, gs, m),
-                   a2 = __shfl_xor_sync(kFull, q[0], m);
-      t2 = dadd(t2, a0);
-      gs = dadd(gs, a1);
-      q[0] = dadd(q[0], a2);
-    }
+    for (int m = 4; m < 32; m <<= 1) v = dadd(v, __shfl_xor_sync(kFull, v, m));
+    t2 = v;
+    q[0] = __shfl_sync(kFull, v, 1);
+    gs = __shfl_sync(kFull, v, 2);
   } else {
     t2 = bfly32(t2);
     gs = bfly32(gs);
