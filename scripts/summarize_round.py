@@ -4,7 +4,8 @@ R = sys.argv[1] if len(sys.argv) > 1 else "r01"
 src = "gpurun_out/prof_round"
 dst = "profiles"
 os.makedirs(dst, exist_ok=True)
-for f in ["bench.jsonl", "bench_reference.jsonl", "pcg.jsonl", "coverage.jsonl", "gpu.csv"]:
+for f in ["bench.jsonl", "bench_reference.jsonl", "pcg.jsonl", "coverage.jsonl", "gpu.csv",
+          "bench_27pt128.jsonl", "bench_27pt256.jsonl", "bench_rmat20.jsonl", "bench_5pt64.jsonl"]:
     p = os.path.join(src, f)
     if os.path.exists(p):
         lines = [l for l in open(p) if l.strip().startswith("{") or f.endswith(".csv")]
