@@ -38,6 +38,10 @@ WORKLOADS = {
     "27pt128": ("3-D 27-point stencil 128^3 FP64 ABFT-SpMV", lambda G: G.stencil_3d_27pt(128)),
     "rmat20": ("R-MAT scale 20, edge factor 16, permuted, FP64 ABFT-SpMV",
                lambda G: G.rmat(20, 16, 1)),
+    "rmat22": ("R-MAT scale 22, edge factor 16, permuted, FP64 ABFT-SpMV",
+               lambda G: G.rmat(22, 16, 1)),
+    "rmat24": ("R-MAT scale 24, edge factor 16, permuted, FP64 ABFT-SpMV (BASELINE configs[2])",
+               lambda G: G.rmat(24, 16, 1)),
 }
 
 

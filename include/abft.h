@@ -137,6 +137,7 @@ typedef struct {
   int64_t groups, general_groups;  /* 32-row groups; those on the general path */
   int32_t lean;             /* staged (TMA) path available */
   int32_t max_rounds;
+  int64_t irr_groups;       /* 32-row groups on the irregular-row path (k_irr) */
 } abft_info_t;
 abft_status abft_info(abft_handle_t h, abft_info_t *info);
 

@@ -12,6 +12,7 @@
 #include "kernels_encode.cuh"
 #include "kernels_pcg.cuh"
 #include "kernels_spmv.cuh"
+#include "kernels_irr.cuh"
 
 using namespace abft;
 
@@ -80,8 +81,12 @@ struct abft_ctx {
   double *hub_part = nullptr;
   int32_t *own_key = nullptr, *own_first = nullptr, *own_n = nullptr;
   int32_t n_hub = 0, n_own = 0;
-  int32_t *glist = nullptr; // groups k_lean does not take
+  int32_t *glist = nullptr; // k_general's groups while k_lean runs
   int64_t n_glist = 0;
+  int32_t *glist_nl = nullptr;  // k_general's groups when k_lean cannot run (x unaligned)
+  int64_t n_glist_nl = 0;
+  int32_t *ilist = nullptr; // k_irr's groups (irregular rows)
+  int64_t n_ilist = 0;
   int correct_grid = 1;
   // scratch
   double *gsum = nullptr;
@@ -167,6 +172,8 @@ SpmvArgs make_args(const abft_ctx *h, const double *x, double *y, const double *
   a.gbar = h->gbar;
   a.sc = h->stage;
   a.lean_ok = h->lean_ok;
+  a.ilist = h->ilist;
+  a.n_ilist = h->n_ilist;
   a.hub_beg = h->hub_beg;
   a.hub_len = h->hub_len;
   a.hub_part = h->hub_part;
@@ -346,16 +353,34 @@ void launch_lean(const abft_ctx *h, const SpmvArgs &a, cudaStream_t s) {
 }
 
 template <bool CHECK, bool INJECT>
+void launch_irr(const abft_ctx *h, const SpmvArgs &a, cudaStream_t s) {
+  const size_t smem = kIrrWarps * kIrrSmemPerWarp;
+  const int64_t need = (h->n_ilist + kIrrWarps - 1) / kIrrWarps;
+  const dim3 grid((unsigned)std::max<int64_t>(1, std::min<int64_t>((int64_t)h->num_sms * kIrrMinB, need)));
+  const dim3 block(kIrrWarps * 32);
+  switch (h->cfmt) {
+    case CF_I8: k_irr<CHECK, INJECT, CF_I8><<<grid, block, smem, s>>>(a); break;
+    case CF_I16: k_irr<CHECK, INJECT, CF_I16><<<grid, block, smem, s>>>(a); break;
+    case CF_F32: k_irr<CHECK, INJECT, CF_F32><<<grid, block, smem, s>>>(a); break;
+    case CF_F64: k_irr<CHECK, INJECT, CF_F64><<<grid, block, smem, s>>>(a); break;
+    default: k_irr<CHECK, INJECT, CF_CSR><<<grid, block, smem, s>>>(a); break;
+  }
+}
+
+template <bool CHECK, bool INJECT>
 abft_status launch_fused_t(const abft_ctx *h, SpmvArgs a, cudaStream_t s) {
   // k_lean needs 16-B aligned operands for its bulk copies (x per call)
   const bool lean = h->lean && aligned16(a.xr);
-  const int64_t ngen = lean ? h->n_glist : h->ngroups;
-  a.glist = lean ? h->glist : nullptr;
+  const int64_t ngen = lean ? h->n_glist : h->n_glist_nl;
+  a.glist = lean ? h->glist : h->glist_nl;
   a.n_glist = ngen;
+  a.ilist = h->ilist;
+  a.n_ilist = h->n_ilist;
   const int ggrid = ngen > 0 ? general_grid(h, ngen) : 0;
   if (h->n_hub > 0)  // chunk sums of hub rows, read by the group kernels
     k_hub<<<general_grid(h, h->n_hub), kGenWarps * 32, 0, s>>>(a);
   if (lean) launch_lean<CHECK, INJECT>(h, a, s);
+  if (h->n_ilist > 0) launch_irr<CHECK, INJECT>(h, a, s);
   if (ggrid) k_general<CHECK, INJECT><<<ggrid, kGenWarps * 32, 0, s>>>(a);
   CK(cudaGetLastError());
   return ABFT_OK;
@@ -423,6 +448,10 @@ abft_status set_lean_attrs(int optin) {
   TRY(set_smem_attrs(k_lean<true, false, CF, 3>, optin));
   TRY(set_smem_attrs(k_lean<false, true, CF, 3>, optin));
   TRY(set_smem_attrs(k_lean<false, false, CF, 3>, optin));
+  for (auto kern : {k_irr<true, true, CF>, k_irr<true, false, CF>, k_irr<false, true, CF>,
+                    k_irr<false, false, CF>})
+    CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                            (int)(kIrrWarps * kIrrSmemPerWarp)));
   return ABFT_OK;
 }
 
@@ -686,10 +715,38 @@ abft_status plan_fused(abft_ctx *h, cudaStream_t s) {
     }
   }
   for (const auto &o : own) lean_ok[(size_t)(o.first >> 6)] |= 2;  // groups owning hub rows
+  // k_irr (b_s = 32): full groups without hub rows / hub C rows whose A
+  // segment fits the warp scratch on the staging grid.  When k_lean would
+  // take only a minority of the groups (power-law matrices), k_irr takes
+  // those too: k_lean's per-warp ranges would be mostly idle.
+  int64_t n_lean = 0;
+  for (int64_t g = 0; g < h->ngroups && h->lean; ++g) n_lean += lean_ok[g] & 1;
+  auto irr_ok = [&](int64_t g) {
+    if (h->bs != 32 || g * 32 + 32 > h->n || (lean_ok[g] & 2)) return false;
+    if ((int64_t)rp[g * 32 + 32] - rp[g * 32] + 3 > kIrrCap) return false;
+    const int32_t lc = h->cfmt != CF_CSR ? crpc[g + 1] - crpc[g] : crp[g + 1] - crp[g];
+    return lc <= 1024;
+  };
+  if (h->lean && 2 * n_lean < h->ngroups && !getenv("ABFT_NO_IRR")) {
+    h->lean = false;
+    for (auto &o : lean_ok) o &= (uint8_t)~1u;
+  }
+  std::vector<int32_t> ilist, glist_nl;
+  for (int64_t g = 0; g < h->ngroups; ++g) {
+    const bool in_lean = h->lean && (lean_ok[g] & 1);
+    const bool irr = !in_lean && !getenv("ABFT_NO_IRR") && irr_ok(g);
+    if (irr) ilist.push_back((int32_t)g);
+    if (!in_lean && !irr) glist.push_back((int32_t)g);
+    if (!irr) glist_nl.push_back((int32_t)g);
+  }
   TRY(upload(h, &h->lean_ok, lean_ok, s));
+  TRY(upload(h, &h->ilist, ilist, s));
+  TRY(upload(h, &h->glist, glist, s));
+  TRY(upload(h, &h->glist_nl, glist_nl, s));
+  h->n_ilist = (int64_t)ilist.size();
+  h->n_glist = (int64_t)glist.size();
+  h->n_glist_nl = (int64_t)glist_nl.size();
   if (h->lean) {
-    for (int64_t g = 0; g < h->ngroups; ++g)
-      if (!(lean_ok[g] & 1)) glist.push_back((int32_t)g);
     int per_sm = 0;
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_lean<true, false, CF_CSR, 2>,
                                                      c.warps * 32, h->fused_smem));
@@ -697,10 +754,6 @@ abft_status plan_fused(abft_ctx *h, cudaStream_t s) {
     if (const char *e = getenv("ABFT_CTAS_PER_SM")) per_sm = std::max(1, std::min(per_sm, atoi(e)));
     const int64_t need = (h->ngroups + c.warps - 1) / c.warps;  // >= 1 group per warp
     h->fused_grid = (int)std::max<int64_t>(1, std::min<int64_t>((int64_t)h->num_sms * per_sm, need));
-    TRY(upload(h, &h->glist, glist, s));
-    h->n_glist = (int64_t)glist.size();
-  } else {
-    h->n_glist = h->ngroups;
   }
   CK(cudaStreamSynchronize(s));  // host vectors die at return
   return ABFT_OK;
@@ -976,7 +1029,8 @@ abft_status abft_info(abft_handle_t h, abft_info_t *info) {
     // K and row_ptr, which the byte model counts once as K and A)
     info->c_bytes = (int64_t)(cf_size(h->cfmt) + 2) * h->nnz_cpad + 4 * (h->nb + 1);
   info->groups = h->ngroups;
-  info->general_groups = h->lean ? h->n_glist : h->ngroups;
+  info->general_groups = h->lean ? h->n_glist : h->n_glist_nl;
+  info->irr_groups = h->n_ilist;
   info->lean = h->lean ? 1 : 0;
   info->max_rounds = h->max_rounds;
   return ABFT_OK;

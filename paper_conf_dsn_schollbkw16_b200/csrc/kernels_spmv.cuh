@@ -95,6 +95,8 @@ struct SpmvArgs {
   unsigned *gbar;         // [2] grid barrier of the correction pass
   const int32_t *glist;   // k_general: groups to process (nullptr: all groups)
   int64_t n_glist;
+  const int32_t *ilist;   // k_irr: irregular groups (kernels_irr.cuh)
+  int64_t n_ilist;
   double *dbg_t1, *dbg_t2;  // nullable
   const int32_t *skip;      // nullable device flag: != 0 -> kernels are no-ops (PCG)
   const uint8_t *lean_ok;   // [ngroups] bit 0: k_lean takes the group; bit 1: it owns hub rows

@@ -99,6 +99,25 @@ class Case:
         return ref
 
 
+def _mixed_lean_irr():
+    """Mostly short rows (k_lean majority) with a few groups holding rows of
+    33..600 entries (k_irr) and one hub row > 1024 entries (k_general)."""
+    rng = np.random.Generator(np.random.PCG64(17))
+    n = 4096
+    lens = rng.integers(0, 9, n)
+    lens[[70, 1000, 1001, 2050, 3333]] = [40, 300, 600, 33, 129]
+    lens[3900] = 1500
+    rows, cols = [], []
+    for i, L in enumerate(lens):
+        c = np.sort(rng.choice(n, size=int(L), replace=False))
+        rows.append(np.full(c.size, i))
+        cols.append(c)
+    cols = np.concatenate(cols).astype(np.int32)
+    rp = np.zeros(n + 1, np.int64)
+    np.cumsum(lens, out=rp[1:])
+    return G.CSR(rp.astype(np.int32), cols, rng.uniform(-1, 1, cols.size), "mixed_lean_irr")
+
+
 MATRICES = {
     "lap2d_64": lambda: G.laplacian_2d_5pt(64),           # BASELINE configs[0]
     "lap3d_16": lambda: G.laplacian_3d_7pt(16),
@@ -109,6 +128,7 @@ MATRICES = {
     "rmat11": lambda: G.rmat(11, 16, 5),                    # power law, long rows
     "rmat11_natural": lambda: G.rmat(11, 8, 6, permute=False),  # empty blocks
     "hubs": lambda: G.hub_csr(5000, 11),                    # rows / C rows > 1024: hub chunks
+    "mixed_lean_irr": lambda: _mixed_lean_irr(),            # k_lean + k_irr + k_general
     "tiny1": lambda: G.CSR([0, 1], [0], [2.5]),
     "tiny33": lambda: G.random_csr(33, 0.2, 9),
     "all_empty": lambda: G.CSR(np.zeros(101, np.int32), np.zeros(0, np.int32), np.zeros(0)),
@@ -345,3 +365,35 @@ def test_pcg_unprotected_and_maxiter(O, torch_cuda):
     assert status == ref.status == -5 and st["iters"] == ref.iters == 7
     assert_bits_equal(hist, ref.res_hist, "truncated history")
     assert_bits_equal(x, ref.x, "truncated solution")
+
+
+def test_irregular_path_routing(O, torch_cuda):
+    # power-law rows take k_irr; a lean majority
+    # keeps k_lean and sends only the long-row groups to k_irr; hub rows stay
+    # with k_general
+    from paper_conf_dsn_schollbkw16_b200 import encode
+    info = encode(MATRICES["rmat11"]()).info()
+    assert info["irr_groups"] > 0 and info["lean"] == 0, info
+    info = encode(MATRICES["mixed_lean_irr"]()).info()
+    assert info["lean"] == 1 and info["irr_groups"] >= 3 and info["general_groups"] >= 2, info
+    info = encode(MATRICES["hubs"]()).info()
+    assert info["irr_groups"] > 0 and info["general_groups"] > 0, info
+
+
+@pytest.mark.parametrize("c_csr", [False, True])
+@pytest.mark.parametrize("name", ["rmat11", "mixed_lean_irr", "hubs"])
+def test_irregular_faults(O, torch_cuda, name, c_csr):
+    # list faults into y rows, t1 and t2 of irregular groups (k_irr's INJECT
+    # instantiation), then a rate-mode call at b_s = 32
+    A = MATRICES[name]()
+    c = Case(O, torch_cuda, A, c_csr=c_csr)
+    rl = np.diff(A.row_ptr)
+    long_rows = np.nonzero(rl > 32)[0][:3]
+    blocks = sorted({int(r) // 32 for r in long_rows})
+    plan = G.FaultPlan([0] * (len(long_rows) + 2 * len(blocks)),
+                       [0] * len(long_rows) + [1] * len(blocks) + [2] * len(blocks),
+                       [int(r) for r in long_rows] + blocks + blocks,
+                       [1 << 62] * len(long_rows) + [1 << 61] * len(blocks) + [1 << 60] * len(blocks))
+    ref = c.run(G.uniform_vector(A.n, 21), plan=plan)
+    assert set(blocks) <= set(ref.flagged.tolist())
+    c.run(G.uniform_vector(A.n, 22), rate=dict(seed=9, lam=1e-4, targets=0b111, call=3))
