@@ -537,6 +537,93 @@ int or_abft_spmv(const or_csr *A, int32_t bs, const int32_t *c_row_ptr, const in
 }
 
 /* ------------------------------------------------------------------------ */
+/* Related-work baseline: the DENSE CHECK of [30, 31] (P:44-48,       */
+/* P:250-252) with COMPLETE RECOMPUTATION [31].  One   */
+/* checksum over all N rows: c = w^T A with w = 1 (eq. 1), so       */
+/* c_j = sum of column j; t1 = c . x, t2 = w^T y.  Readings (DESIGN.md */
+/* R23-R25): c_j = PW over column j's entries in ascending row order; t1 =   */
+/* PW over the n columns of fl(c_j x_j) (c_j = +0.0 for an empty column);    */
+/* t2 = PW over the N entries of y; the bound is either the norm-based       */
+/* tau = ||x||_2 of [30] or the analytical bound of [35] */
+/* with m = N rows and n columns: tau = K35 * ||x||_2,                        */
+/* K35 = fl(fl(fl((n + 2N - 2) * PW_i ||a_i||_2) + fl(n * ||c||_2)) * 2^-53). */
+/* Flag iff NOT(|t1 - t2| <= tau); a flag triggers a complete recomputation  */
+/* of y (round r + 1), re-checked, at most max_rounds times.                  */
+/* ------------------------------------------------------------------------ */
+void or_dense_encode(const or_csr *A, double *c, double *k35) {
+  int64_t n = A->n;
+  int64_t nnz = A->row_ptr[n];
+  /* column lists in ascending row order (a counting sort by column) */
+  int64_t *cnt = (int64_t *)calloc((size_t)n + 1, sizeof(int64_t));
+  for (int64_t e = 0; e < nnz; ++e) cnt[A->col[e] + 1]++;
+  for (int64_t j = 0; j < n; ++j) cnt[j + 1] += cnt[j];
+  double *cv = (double *)malloc(sizeof(double) * (size_t)(nnz > 0 ? nnz : 1));
+  int64_t *pos = (int64_t *)malloc(sizeof(int64_t) * (size_t)(n > 0 ? n : 1));
+  for (int64_t j = 0; j < n; ++j) pos[j] = cnt[j];
+  for (int64_t i = 0; i < n; ++i)
+    for (int64_t q = A->row_ptr[i]; q < A->row_ptr[i + 1]; ++q) cv[pos[A->col[q]]++] = A->val[q];
+  for (int64_t j = 0; j < n; ++j) c[j] = or_pw(cv + cnt[j], cnt[j + 1] - cnt[j]);
+  if (k35) {
+    double *tmp = (double *)malloc(sizeof(double) * (size_t)(n > 0 ? n : 1));
+    for (int64_t i = 0; i < n; ++i) {
+      int64_t b = A->row_ptr[i], e = A->row_ptr[i + 1];
+      double *sq = (double *)malloc(sizeof(double) * (size_t)(e > b ? e - b : 1));
+      for (int64_t q = b; q < e; ++q) sq[q - b] = A->val[q] * A->val[q];
+      tmp[i] = sqrt(or_pw(sq, e - b));
+      free(sq);
+    }
+    double S = or_pw(tmp, n);
+    for (int64_t j = 0; j < n; ++j) tmp[j] = c[j] * c[j];
+    double cn = sqrt(or_pw(tmp, n));
+    double m = (double)(n + 2 * n - 2); /* n columns + 2m - 2 with m = N = n rows */
+    *k35 = ((m * S) + ((double)n * cn)) * 0x1p-53;
+    free(tmp);
+  }
+  free(cnt);
+  free(cv);
+  free(pos);
+}
+
+int or_dense_spmv(const or_csr *A, const double *c, double k35, int32_t bound35,
+                  const double *x, const or_inject *inj, int32_t max_rounds, double *y,
+                  double *y_pre, double *out, int32_t *flag_rounds) {
+  int64_t n = A->n;
+  if (inj && inj->mode == OR_INJ_RATE) return -1; /* list mode only */
+  double *tmp = (double *)malloc(sizeof(double) * (size_t)(n > 0 ? n : 1));
+  for (int64_t i = 0; i < n; ++i) tmp[i] = x[i] * x[i];
+  double beta = sqrt(or_pw(tmp, n)); /* ||x||_2, R10 */
+  double tau = bound35 ? k35 * beta : beta;
+  int rc = 0;
+  for (int32_t r = 0; r <= max_rounds; ++r) {
+    /* round 0: the SpMV; round r >= 1: the r-th complete recomputation */
+    for (int64_t i = 0; i < n; ++i) {
+      double v = or_row_dot(A, i, x);
+      int64_t ops = 2 * (int64_t)(A->row_ptr[i + 1] - A->row_ptr[i]);
+      y[i] = xor_double(v, or_fault_mask(inj, r, OR_T_Y, i, ops));
+    }
+    if (r == 0 && y_pre) memcpy(y_pre, y, sizeof(double) * (size_t)n);
+    for (int64_t j = 0; j < n; ++j) tmp[j] = c[j] * x[j];
+    double t1 = xor_double(or_pw(tmp, n), or_fault_mask(inj, r, OR_T_T1, 0, 2 * n));
+    double t2 = xor_double(or_pw(y, n), or_fault_mask(inj, r, OR_T_T2, 0, n));
+    int flagged = !(fabs(t1 - t2) <= tau);
+    flag_rounds[r] = flagged;
+    if (r == 0 && out) {
+      out[0] = t1;
+      out[1] = t2;
+      out[2] = beta;
+      out[3] = tau;
+    }
+    if (!flagged) {
+      for (int32_t q = r + 1; q <= max_rounds; ++q) flag_rounds[q] = 0;
+      break;
+    }
+    if (r == max_rounds) rc = -6;
+  }
+  free(tmp);
+  return rc;
+}
+
+/* ------------------------------------------------------------------------ */
 /* Jacobi-preconditioned CG (Saad, Alg. 9.1) using the protected */
 /* SpMV for every product with A.  Stop when ||r||_2 <= tol * ||b||_2 (R16)  */
 /* or after max_iter iterations (10 N by default).  M = diag(A) and  */

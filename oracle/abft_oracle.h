@@ -87,6 +87,19 @@ int or_abft_spmv(const or_csr *A, int32_t bs, const int32_t *c_row_ptr, const in
                  int32_t max_rounds, double *y, double *y_pre, double *t1, double *t2,
                  double *s, double *beta_out, int32_t *flag_counts, int32_t *flags);
 
+/* --- related-work baseline: dense check [30, 31] + complete recomputation ---
+ * (R23-R25)
+ * c [n]: c_j = PW over column j in row order; *k35: the [35] constant (m = N).
+ * or_dense_spmv: bound35 = 0 -> tau = ||x||_2 (norm-based), 1 -> tau =
+ * k35 ||x||_2.  flag_rounds [max_rounds+1]: 1 where round r's check failed
+ * (round r >= 1 = r-th complete recomputation).  out [4] (nullable): round 0's
+ * t1, t2, beta, tau.  List injection only (index 0 for t1 / t2).  Returns 0,
+ * -6 if still flagged after max_rounds recomputations, -1 for rate mode. */
+void or_dense_encode(const or_csr *A, double *c, double *k35);
+int or_dense_spmv(const or_csr *A, const double *c, double k35, int32_t bound35,
+                  const double *x, const or_inject *inj, int32_t max_rounds, double *y,
+                  double *y_pre, double *out, int32_t *flag_rounds);
+
 /* --- Jacobi-PCG with the protected SpMV (Saad Alg. 9.1) ---
  * res_hist [max_iter+1].  stats: [0] iters, [1] spmv calls, [2] flagged blocks
  * (round 0, summed), [3] recomputed blocks (summed over rounds), [4] uncorrected

@@ -71,6 +71,9 @@ def lib():
         L.or_rate_plan.argtypes = [P, i32, P, i32, P, i32, P, P, P, P]
         L.or_abft_spmv.restype = C.c_int
         L.or_abft_spmv.argtypes = [P, i32, P, P, P, P, P, P, i32, P, P, P, P, P, P, P, P]
+        L.or_dense_encode.argtypes = [P, P, P]
+        L.or_dense_spmv.restype = C.c_int
+        L.or_dense_spmv.argtypes = [P, P, d, i32, P, P, i32, P, P, P, P]
         L.or_pcg.restype = C.c_int
         L.or_pcg.argtypes = [P, i32, P, P, P, P, P, P, P, d, i64, P, i32, i32, P, P]
     return _lib
@@ -266,6 +269,49 @@ def abft_spmv(A, enc: Encoded, x, inj: Inject | None = None, max_rounds: int = 4
                             C.byref(beta), _p(fc), _p(fl))
     flags = [fl[q * nb: q * nb + fc[q]].copy() for q in range(max_rounds + 1)]
     return SpmvResult(st, y, y_pre, t1, t2, s, beta.value, flags)
+
+
+@dataclass
+class DenseEncoded:
+    """Dense-check checksum (related work [30, 31]; oracle/abft_oracle.h)."""
+    c: np.ndarray   # [n] column sums, PW over each column in row order (R23)
+    k35: float      # [35]'s bound constant with m = N rows (R24)
+
+
+def dense_encode(A) -> DenseEncoded:
+    r = _CsrRef(A)
+    c = np.empty(A.n)
+    k = C.c_double(0.0)
+    lib().or_dense_encode(r.ref(), _p(c), C.byref(k))
+    return DenseEncoded(c, k.value)
+
+
+@dataclass
+class DenseResult:
+    status: int
+    y: np.ndarray          # after the last round
+    y_pre: np.ndarray      # after round 0 (faults included)
+    t1: float
+    t2: float
+    beta: float
+    tau: float
+    flag_rounds: np.ndarray  # [max_rounds+1] 1 where round r's check failed
+
+
+def dense_spmv(A, enc: DenseEncoded, x, bound35: bool = False, inj: "Inject | None" = None,
+               max_rounds: int = 4) -> DenseResult:
+    """Dense check + complete recomputation."""
+    r = _CsrRef(A)
+    x = np.ascontiguousarray(x, dtype=np.float64)
+    y = np.empty(A.n)
+    y_pre = np.empty(A.n)
+    out = np.zeros(4)
+    fr = np.zeros(max_rounds + 1, dtype=np.int32)
+    ist = inj._struct() if inj is not None else None
+    st = lib().or_dense_spmv(r.ref(), _p(enc.c), enc.k35, int(bound35), _p(x),
+                             C.byref(ist) if ist is not None else None, max_rounds, _p(y),
+                             _p(y_pre), _p(out), _p(fr))
+    return DenseResult(st, y, y_pre, out[0], out[1], out[2], out[3], fr)
 
 
 @dataclass

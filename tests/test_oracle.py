@@ -535,3 +535,111 @@ class TestPcg:
         r = O.pcg(A, enc, b, x0, tol=1e-6, inj=O.Inject.rate(seed=9, lam=1e-4), check=False)
         assert not np.array_equal(r.res_hist[: min(len(r.res_hist), len(clean.res_hist))],
                                   clean.res_hist[: min(len(r.res_hist), len(clean.res_hist))])
+
+
+# --------------------------------------------------------------------------
+# Related-work baseline: dense check [30, 31] with complete
+# recomputation [31] (DESIGN.md
+# R23-R25).  Pinned against column sums, eq. (1)'s invariant, the closed
+# form of [35], the method's own encode at b_s = N, and fault behaviour.
+# --------------------------------------------------------------------------
+class TestDenseCheck:
+    def test_c_is_column_sums_integer(self, O):
+        A = G.random_csr(200, 0.05, 31, integer=True, empty_rows=0.1)
+        D = np.zeros((A.n, A.n))
+        for i in range(A.n):
+            for q in range(A.row_ptr[i], A.row_ptr[i + 1]):
+                D[i, A.col[q]] = A.val[q]
+        e = O.dense_encode(A)
+        assert np.array_equal(e.c, D.sum(axis=0))  # w = 1: c = 1^T A
+
+    def test_c_laplacian_values(self, O):
+        # 7-pt Dirichlet Laplacian (6 / -1): column sums are 6 - #neighbours
+        e = O.dense_encode(G.laplacian_3d_7pt(6))
+        assert set(np.unique(e.c).tolist()) == {0.0, 1.0, 2.0, 3.0}
+
+    def test_c_pairwise_in_row_order(self, O):
+        # column 0 holds (1, 1e16, -1e16, 1) in rows 0..3: PW gives
+        # (1 + 1e16) + (-1e16 + 1) = 0; a left fold would give 1 (R23)
+        D = np.array([[1.0, 1], [1e16, 0], [-1e16, 0], [1.0, 0]])
+        D = np.pad(D, ((0, 0), (0, 2)))
+        D[0, 1] = 1.0
+        A = csr_from_dense(D)
+        assert O.dense_encode(A).c[0] == 0.0
+
+    def test_k35_closed_form(self, O):
+        # A = diag(3, 4): sum ||a_i|| = 7, c = (3, 4), ||c|| = 5, n = m = 2:
+        # ((2 + 2*2 - 2) * 7 + 2 * 5) * 2^-53 = 38 * 2^-53
+        e = O.dense_encode(csr_from_dense(np.diag([3.0, 4.0])))
+        assert e.k35 == 38.0 * EPS
+
+    def test_k35_equals_method_bound_at_bs_n(self, O):
+        # b_s = N: the method's bound reduces to [35];
+        # integer stencil with every column present, N a power of two
+        A = G.laplacian_2d_5pt(16)
+        enc = O.encode(A, A.n)
+        assert enc.nb == 1
+        assert O.dense_encode(A).k35 == enc.K[0]
+
+    def test_invariant_integer(self, O):
+        # eq. (1)-(2): c^T x == w^T (A x) exactly for integer A and x
+        A = G.random_csr(300, 0.04, 32, integer=True)
+        x = np.random.default_rng(3).integers(-5, 6, A.n).astype(np.float64)
+        r = O.dense_spmv(A, O.dense_encode(A), x)
+        assert r.t1 == r.t2 and r.flag_rounds.sum() == 0
+
+    @pytest.mark.parametrize("bound35", [False, True])
+    def test_no_false_positive(self, O, bound35):
+        for A in (G.laplacian_3d_7pt(10), G.random_csr(500, 0.02, 33), G.rmat(9, 8, 2)):
+            e = O.dense_encode(A)
+            for seed in range(3):
+                x = G.uniform_vector(A.n, seed)
+                r = O.dense_spmv(A, e, x, bound35=bound35)
+                assert r.status == 0 and r.flag_rounds.sum() == 0
+                assert np.array_equal(r.y, O.spmv(A, x))
+                assert r.tau == (e.k35 * r.beta if bound35 else r.beta)  # P:262 / [35]
+
+    @staticmethod
+    def scale_mask(v, f=2.0 ** 20):
+        """XOR mask that turns v into v * f (an exponent-field burst)."""
+        return int(np.float64(v * f).view(np.uint64) ^ np.float64(v).view(np.uint64))
+
+    def test_fault_flagged_and_recomputed(self, O):
+        A = G.laplacian_3d_7pt(8)
+        e = O.dense_encode(A)
+        x = G.uniform_vector(A.n, 5)
+        y = O.spmv(A, x)
+        inj = O.Inject.from_plan(G.FaultPlan([0], [0], [77], [self.scale_mask(y[77])]))
+        r = O.dense_spmv(A, e, x, inj=inj)
+        assert r.status == 0 and r.flag_rounds.tolist() == [1, 0, 0, 0, 0]
+        assert r.y_pre[77] == y[77] * 2.0 ** 20
+        assert np.array_equal(r.y, y)  # complete recomputation (P:240)
+
+    def test_faults_every_round_exhaust(self, O):
+        A = G.laplacian_2d_5pt(8)
+        e = O.dense_encode(A)
+        x = G.uniform_vector(A.n, 6)
+        y = O.spmv(A, x)
+        m = self.scale_mask(y[3])
+        r0 = O.dense_spmv(A, e, x)
+        mt1 = self.scale_mask(r0.t1)
+        inj = O.Inject.from_plan(G.FaultPlan([0, 1, 2], [0, 1, 0], [3, 0, 3], [m, mt1, m]))
+        r = O.dense_spmv(A, e, x, inj=inj, max_rounds=2)
+        assert r.status == -6 and r.flag_rounds.tolist() == [1, 1, 1]
+
+    def test_small_fault_below_norm_bound_missed(self, O):
+        # the norm-based bound tau = ||x|| (P:262) misses a fault the sparse
+        # bound catches: the coverage gap of Fig. 7 (P:264-270)
+        A = G.laplacian_3d_7pt(8)
+        x = G.uniform_vector(A.n, 7)
+        e = O.dense_encode(A)
+        beta = math.sqrt(float(np.sum(x * x)))
+        y = O.spmv(A, x)
+        i = 100
+        delta_target = 1e-3 * beta
+        mask = np.float64(y[i] + delta_target).view(np.uint64) ^ np.float64(y[i]).view(np.uint64)
+        inj = O.Inject.from_plan(G.FaultPlan([0], [0], [i], [int(mask)]))
+        assert O.dense_spmv(A, e, x, inj=inj).flag_rounds[0] == 0
+        enc = O.encode(A, 32)
+        ref = O.abft_spmv(A, enc, x, inj)
+        assert ref.flags[0].tolist() == [i // 32]
