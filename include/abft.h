@@ -222,6 +222,33 @@ abft_status abft_pcg(abft_handle_t h, const double *b, double *x, const double *
                      double tol, int64_t max_iter, const abft_inject_t *inj, int32_t check,
                      double *res_hist, abft_pcg_stats_t *stats, void *stream);
 
+/* --- Related-work baseline: DENSE CHECK [30, 31] + COMPLETE RECOMPUTATION ---
+ * (eq. (1), P:148-152 [35]'s bound, P:240, P:250-252,
+ * P:258, R23-R25.)  One checksum
+ * over all N rows: c = 1^T A (c_j = PW over column j in row order), t1 = PW_j
+ * c_j x_j, t2 = PW_i y_i, flag iff NOT(|t1 - t2| <= tau) with tau = ||x||_2
+ * (the norm-based bound of [30]) or, with ABFT_DENSE_BOUND35,
+ * tau = K35 ||x||_2, K35 = ((n + 2N - 2) PW_i ||a_i||_2 + n ||c||_2) 2^-53.
+ * A flag under ABFT_AUTOCORRECT recomputes ALL of y and re-checks, at most
+ * max_rounds times (complete recomputation).  Square handles only
+ * (ABFT_ENOTSUP for shards); list injection only (target 1 / 2 index 0 = t1 /
+ * t2; rate mode: ABFT_ENOTSUP).
+ * abft_dense_encode: builds c and K35 on the device (owned by the handle;
+ *   temporaries of ~17 B per nonzero during the call); synchronises.
+ * abft_spmv_dense: the method's SpMV kernels with the check off, then one
+ *   persistent check/recompute kernel; asynchronous, results stay on device.
+ * abft_dense_result: host copies of round 0's (t1, t2, beta, tau) [4], the
+ *   per-round flags [max_rounds+1] (1 = round r's check failed) and K35;
+ *   each pointer nullable; synchronises. */
+#define ABFT_DENSE_BOUND35 16u
+abft_status abft_dense_encode(abft_handle_t h, void *stream);
+abft_status abft_spmv_dense(abft_handle_t h, const double *x, double *y,
+                            const abft_inject_t *inj, uint32_t mode, void *stream);
+abft_status abft_dense_result(abft_handle_t h, double *out, int32_t *flag_rounds, double *k35,
+                              void *stream);
+/* Device pointer to c [n] (valid until abft_destroy). */
+abft_status abft_dense_checksum(abft_handle_t h, const double **c);
+
 abft_status abft_destroy(abft_handle_t h);
 
 /* Plumbing for bindings: cudaMemcpyAsync(dst, src, bytes, cudaMemcpyDefault)

@@ -19,6 +19,7 @@ _LIB = None
 
 OK, EINVAL, ECUDA, ENOMEM, ENOTSUP, ENOCONV, EUNCORRECTED, EBREAKDOWN = 0, -1, -2, -3, -4, -5, -6, -7
 NOCHECK, CHECK, AUTOCORRECT, DEBUG_CHECKSUMS, DEFER_FINISH = 0, 1, 2, 4, 8
+DENSE_BOUND35 = 16  # abft_spmv_dense: tau = K35 ||x|| ([35]) instead of ||x|| ([30])
 INJ_NONE, INJ_LIST, INJ_RATE = 0, 1, 2
 
 SYMBOLS = [
@@ -26,6 +27,7 @@ SYMBOLS = [
     "abft_checksum_matrix", "abft_debug_checksums", "abft_spmv_host", "abft_pcg",
     "abft_destroy", "abft_memcpy", "abft_status_string", "abft_last_cuda_error",
     "abft_burst_table", "abft_version", "abft_info", "abft_beta_partial", "abft_finish",
+    "abft_dense_encode", "abft_spmv_dense", "abft_dense_result", "abft_dense_checksum",
 ]
 ENCODE_C_CSR = 1
 CFMT_NAMES = {0: "csr-f64", 1: "int8+u16", 2: "int16+u16", 3: "f32+u16", 4: "f64+u16"}
@@ -121,6 +123,14 @@ def lib():
         L.abft_info.argtypes = [P, C.POINTER(Info)]
         L.abft_beta_partial.restype = st
         L.abft_beta_partial.argtypes = [P, P, P]
+        L.abft_dense_encode.restype = st
+        L.abft_dense_encode.argtypes = [P, P]
+        L.abft_spmv_dense.restype = st
+        L.abft_spmv_dense.argtypes = [P, P, P, P, u32, P]
+        L.abft_dense_result.restype = st
+        L.abft_dense_result.argtypes = [P, P, P, P, P]
+        L.abft_dense_checksum.restype = st
+        L.abft_dense_checksum.argtypes = [P, C.POINTER(P)]
         L.abft_finish.restype = st
         L.abft_finish.argtypes = [P, P, P, P, i32, i32, P, P]
         _LIB = L
@@ -326,6 +336,39 @@ class Handle:
                "abft_debug_checksums")
         return (self._d2h(t1, self.nb, np.float64, stream),
                 self._d2h(t2, self.nb, np.float64, stream))
+
+    # -- related-work baseline: dense check + complete recomputation -------
+    def dense_encode(self, stream=None):
+        """Build c = 1^T A and K35 for the dense check (include/abft.h)."""
+        _check(lib().abft_dense_encode(self._h, _stream(stream)), "abft_dense_encode")
+        return self
+
+    def spmv_dense(self, x, y=None, inject: Inject | None = None, correct=True, bound35=False,
+                   stream=None):
+        import torch
+        if y is None:
+            y = torch.empty_like(x)
+        inj = inject.struct() if inject is not None else None
+        mode = (AUTOCORRECT if correct else 0) | (DENSE_BOUND35 if bound35 else 0)
+        _check(lib().abft_spmv_dense(self._h, _ptr(x), _ptr(y),
+                                     C.byref(inj) if inj is not None else None, mode,
+                                     _stream(stream)), "abft_spmv_dense")
+        return y
+
+    def dense_result(self, stream=None) -> dict:
+        out = np.zeros(4)
+        fr = np.zeros(self.max_rounds + 1, dtype=np.int32)
+        k = C.c_double(0.0)
+        _check(lib().abft_dense_result(self._h, out.ctypes.data_as(C.c_void_p),
+                                       fr.ctypes.data_as(C.c_void_p), C.byref(k),
+                                       _stream(stream)), "abft_dense_result")
+        return {"t1": out[0], "t2": out[1], "beta": out[2], "tau": out[3], "flag_rounds": fr,
+                "k35": k.value}
+
+    def dense_checksum(self, stream=None) -> np.ndarray:
+        c = C.c_void_p()
+        _check(lib().abft_dense_checksum(self._h, C.byref(c)), "abft_dense_checksum")
+        return self._d2h(c, self.n, np.float64, stream)
 
     # -- PCG ----------------------------------------------------------------
     def pcg(self, b, x, diag=None, tol=1e-6, max_iter=0, inject: Inject | None = None,

@@ -13,6 +13,9 @@
 #include "kernels_pcg.cuh"
 #include "kernels_spmv.cuh"
 #include "kernels_irr.cuh"
+#include "kernels_dense.cuh"
+
+#include <cub/device/device_radix_sort.cuh>
 
 using namespace abft;
 
@@ -85,6 +88,9 @@ struct abft_ctx {
   int64_t n_glist = 0;
   int32_t *glist_nl = nullptr;  // k_general's groups when k_lean cannot run (x unaligned)
   int64_t n_glist_nl = 0;
+  // dense-check baseline (kernels_dense.cuh): c = 1^T A, K35, per-call results
+  double *dn_c = nullptr, *dn_k35 = nullptr, *dn_part = nullptr, *dn_res = nullptr;
+  int32_t *dn_flags = nullptr;
   int32_t *ilist = nullptr; // k_irr's groups (irregular rows)
   int64_t n_ilist = 0;
   int correct_grid = 1;
@@ -1048,3 +1054,4 @@ abft_status abft_memcpy(void *dst, const void *src, int64_t bytes, void *stream)
 }  // extern "C"
 
 #include "abft_pcg_api.inc"
+#include "abft_dense_api.inc"
