@@ -11,7 +11,7 @@
 // column lists in row order; short columns are reduced lane-private, long
 // ones by the warp.  K35 = ((n + 2N - 2) PW_i ||a_i|| + n ||c||) 2^-53.
 // Per call: the SpMV, then ONE persistent kernel (PDL launch, one CTA per SM,
-// software grid barrier): aligned 8192-row chunk partials of y, c o x and x^2,
+// software grid barrier): aligned 2048-row chunk partials of y, c o x and x^2,
 // every CTA finishes the three PW totals from the partials (so all CTAs agree
 // on the flag without another barrier), flag iff NOT(|t1 - t2| <= tau); on a
 // flag it recomputes all of y (round r + 1) and checks again, <= R rounds.
@@ -20,7 +20,8 @@
 
 namespace abft {
 
-constexpr int kDenseChunk = 8192;  // rows per aligned partial (power of two)
+constexpr int kDenseChunk = 8192;  // rows per aligned partial of the encode-time sums
+constexpr int kDenseRows = 2048;   // rows per aligned partial of the per-call sums (one CTA)
 
 // Column id of every entry (rows expanded), the sort key.
 __global__ void k_dense_keys(int64_t n, const int32_t *__restrict__ rp,
@@ -222,14 +223,51 @@ __device__ __forceinline__ void dense_recompute(const SpmvArgs &a, int round) {
   }
 }
 
+// Aligned 2048-row partial of the three dense-check sums (rows b .. b+2047,
+// absent past n) by a CTA of 256 threads: lane l of warp w owns the aligned
+// 8-run b + 256 w + 8 l, an 8-leaf tree in registers, the butterfly joins the
+// warp's 256, a tree over the 8 warps (shared memory) the CTA's 2048 -- the
+// PW tree of the chunk (R2).  Called by all threads; valid in thread 0.
+__device__ __forceinline__ void dense_chunk(const DenseArgs &d, int64_t b, double (*s_w)[8],
+                                            double out[3]) {
+  const SpmvArgs &a = d.a;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int64_t r0 = b + 256 * warp + 8 * lane;
+  double vy[8], vc[8], vx[8];
+#pragma unroll
+  for (int u = 0; u < 8; ++u) {
+    const bool in = r0 + u < a.n;
+    vy[u] = in ? __ldcg(a.y + r0 + u) : kAbsent;
+    vx[u] = in ? __ldg(a.x + r0 + u) : 0.0;
+    vc[u] = in ? __ldg(d.c + r0 + u) : 0.0;
+  }
+#pragma unroll
+  for (int u = 0; u < 8; ++u) {
+    const bool in = r0 + u < a.n;
+    vc[u] = in ? dmul(vc[u], vx[u]) : kAbsent;
+    vx[u] = in ? dmul(vx[u], vx[u]) : kAbsent;
+  }
+  double w[3] = {bfly32(tree<8>(vy)), bfly32(tree<8>(vc)), bfly32(tree<8>(vx))};
+  if (lane == 0)
+    for (int k = 0; k < 3; ++k) s_w[k][warp] = w[k];
+  __syncthreads();
+  if (threadIdx.x == 0)
+    for (int k = 0; k < 3; ++k) {
+      double v[8];
+      for (int q = 0; q < 8; ++q) v[q] = s_w[k][q];
+      out[k] = tree<8>(v);
+    }
+  __syncthreads();
+}
+
 template <bool INJECT>
 __global__ void __launch_bounds__(256) k_dense(const DenseArgs d) {
   __shared__ double s_red[256];
-  __shared__ double s_tmp[3][1024];  // staging of one aligned 1024-row slice
+  __shared__ double s_w[3][8];
   asm volatile("griddepcontrol.wait;" ::: "memory");
   const SpmvArgs &a = d.a;
   const int64_t n = a.n;
-  const int64_t nch = (n + kDenseChunk - 1) / kDenseChunk;
+  const int64_t nch = (n + kDenseRows - 1) / kDenseRows;
   double beta = 0.0, tau = 0.0;
   if (blockIdx.x == 0 && threadIdx.x == 0)
     for (int q = 0; q <= a.max_rounds; ++q) d.flag_rounds[q] = 0;
@@ -238,26 +276,11 @@ __global__ void __launch_bounds__(256) k_dense(const DenseArgs d) {
       dense_recompute<INJECT>(a, r);
       grid_sync(a.gbar);
     }
-    // chunk partials: PW over aligned kDenseChunk rows of y, c o x and x^2
-    // (8 slices of 1024 rows, each an aligned subtree, then a tree over 8)
     for (int64_t ch = blockIdx.x; ch < nch; ch += gridDim.x) {
-      double q[3][8];
-      for (int sl = 0; sl < 8; ++sl) {
-        const int64_t b = ch * kDenseChunk + sl * 1024;
-        const int64_t m = b < n ? min64(1024, n - b) : 0;
-        for (int64_t t = threadIdx.x; t < 1024; t += blockDim.x) {
-          const bool in = t < m;
-          const double yv = in ? __ldcg(a.y + b + t) : kAbsent;
-          const double xv = in ? __ldg(a.x + b + t) : kAbsent;
-          s_tmp[0][t] = yv;
-          s_tmp[1][t] = in ? dmul(__ldg(d.c + b + t), xv) : kAbsent;
-          s_tmp[2][t] = in ? dmul(xv, xv) : kAbsent;
-        }
-        __syncthreads();
-        for (int k = 0; k < 3; ++k) q[k][sl] = cta_pw_smem1024(s_tmp[k], s_red);
-      }
+      double o[3];
+      dense_chunk(d, ch * kDenseRows, s_w, o);
       if (threadIdx.x == 0)
-        for (int k = 0; k < 3; ++k) d.part[k * nch + ch] = tree<8>(q[k]);
+        for (int k = 0; k < 3; ++k) d.part[k * nch + ch] = o[k];
     }
     grid_sync(a.gbar);
     // every CTA finishes the totals itself (same bits everywhere)
