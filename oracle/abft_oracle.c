@@ -732,3 +732,124 @@ int or_pcg(const or_csr *A, int32_t bs, const int32_t *c_row_ptr, const int32_t 
   free(fl);
   return rc;
 }
+
+/* ------------------------------------------------------------------------ */
+/* Related-work baseline for the PCG case study: the         */
+/* CHECKPOINTING approach of P:286-292 -- every SpMV protected by the dense  */
+/* check with the norm-based bound, the solver state sampled every   */
+/* `ckpt_every` (20) iterations, and on a detection a rollback to the */
+/* last sample and re-execution from there.  DESIGN.md R26-R27:              */
+/*  * state = (x, r, z, p, rho, it); the first sample is taken after the     */
+/*    initial residual; a flagged initial SpMV is simply redone;             */
+/*  * SpMV call j (the j-th executed product, initial one = 0) draws its      */
+/*    faults from the rate plan of call inj->call + j over y only (the       */
+/*    dense check's own 3N detection ops are not injected);                  */
+/*  * max_iter bounds EXECUTED iterations (re-executions count).      */
+/* The updates are those of or_pcg (R15).  stats: [0] iterations of the     */
+/* returned solution, [1] SpMV calls, [2] rollbacks, [3] executed            */
+/* iterations, [4] 0.  Returns 0 converged, -5 not converged, -7 breakdown. */
+/* ------------------------------------------------------------------------ */
+int or_pcg_cr(const or_csr *A, const double *c, const double *b, double *x, const double *diag,
+              double tol, int64_t max_iter, const or_inject *inj_in, int32_t ckpt_every,
+              double *res_hist, int64_t *stats) {
+  int64_t n = A->n;
+  if (max_iter <= 0) max_iter = 10 * n;
+  size_t vb = sizeof(double) * (size_t)(n > 0 ? n : 1);
+  double *r = (double *)malloc(vb), *z = (double *)malloc(vb), *p = (double *)malloc(vb);
+  double *q = (double *)malloc(vb), *tmp = (double *)malloc(vb), *d = (double *)malloc(vb);
+  double *cx = (double *)malloc(vb), *cr = (double *)malloc(vb), *cz = (double *)malloc(vb);
+  double *cp = (double *)malloc(vb);
+  or_inject inj;
+  memset(&inj, 0, sizeof inj);
+  if (inj_in) inj = *inj_in;
+  uint64_t call0 = inj.call;
+  int64_t calls = 0, rollbacks = 0, executed = 0;
+  for (int i = 0; i < 5; ++i) stats[i] = 0;
+  for (int64_t i = 0; i < n; ++i) {
+    double v = 0.0;
+    if (diag) v = diag[i];
+    else if (!find_entry(A, i, (int32_t)i, &v)) v = 0.0;
+    d[i] = v;
+  }
+  /* y = A v with this call's y faults, then the dense check (t1 = c.v,
+     t2 = sum y, tau = ||v||): returns 1 when flagged */
+#define CHECKED_SPMV(vin, yout, flagged)                                         \
+  do {                                                                           \
+    inj.call = call0 + (uint64_t)calls;                                          \
+    void *keep_ = NULL;                                                          \
+    or_inject l_ = inj;                                                          \
+    if (inj.mode == OR_INJ_RATE) l_ = rate_to_list(A, 32, NULL, 0, &inj, 0, &keep_); \
+    for (int64_t i_ = 0; i_ < n; ++i_)                                           \
+      yout[i_] = xor_double(or_row_dot(A, i_, vin), or_fault_mask(&l_, 0, OR_T_Y, i_, 0)); \
+    free(keep_);                                                                 \
+    for (int64_t i_ = 0; i_ < n; ++i_) tmp[i_] = c[i_] * vin[i_];               \
+    double t1_ = or_pw(tmp, n);                                                  \
+    double t2_ = or_pw(yout, n);                                                 \
+    double bt_ = sqrt(dot_pw(vin, vin, n, tmp));                                 \
+    flagged = !(fabs(t1_ - t2_) <= bt_);                                         \
+    calls++;                                                                     \
+  } while (0)
+
+  int fl = 1, rc = 0;
+  while (fl && calls < max_iter + 1) CHECKED_SPMV(x, q, fl); /* q = A x0 */
+  for (int64_t i = 0; i < n; ++i) r[i] = b[i] - q[i];
+  for (int64_t i = 0; i < n; ++i) z[i] = r[i] / d[i];
+  for (int64_t i = 0; i < n; ++i) p[i] = z[i];
+  double rho = dot_pw(r, z, n, tmp);
+  double bnorm = sqrt(dot_pw(b, b, n, tmp));
+  double thr = tol * bnorm;
+  double res = sqrt(dot_pw(r, r, n, tmp));
+  res_hist[0] = res;
+  int64_t it = 0;
+  /* sample 0 */
+  memcpy(cx, x, vb); memcpy(cr, r, vb); memcpy(cz, z, vb); memcpy(cp, p, vb);
+  double c_rho = rho, c_res = res;
+  int64_t c_it = 0;
+  while (!(res <= thr) && executed < max_iter) {
+    if (res != res) {
+      rc = -7;
+      break;
+    }
+    ++executed;
+    CHECKED_SPMV(p, q, fl);
+    if (fl) { /* rollback to the last sample */
+      memcpy(x, cx, vb); memcpy(r, cr, vb); memcpy(z, cz, vb); memcpy(p, cp, vb);
+      rho = c_rho;
+      res = c_res;
+      it = c_it;
+      ++rollbacks;
+      continue;
+    }
+    double pq = dot_pw(p, q, n, tmp);
+    if (!(pq > 0.0)) {
+      rc = -7;
+      break;
+    }
+    double alpha = rho / pq;
+    for (int64_t i = 0; i < n; ++i) x[i] = x[i] + alpha * p[i];
+    for (int64_t i = 0; i < n; ++i) r[i] = r[i] - alpha * q[i];
+    for (int64_t i = 0; i < n; ++i) z[i] = r[i] / d[i];
+    double rho_new = dot_pw(r, z, n, tmp);
+    res = sqrt(dot_pw(r, r, n, tmp));
+    ++it;
+    res_hist[it] = res;
+    double beta = rho_new / rho;
+    rho = rho_new;
+    for (int64_t i = 0; i < n; ++i) p[i] = z[i] + beta * p[i];
+    if (ckpt_every > 0 && it % ckpt_every == 0) { /* sample the state */
+      memcpy(cx, x, vb); memcpy(cr, r, vb); memcpy(cz, z, vb); memcpy(cp, p, vb);
+      c_rho = rho;
+      c_res = res;
+      c_it = it;
+    }
+  }
+#undef CHECKED_SPMV
+  if (rc == 0 && !(res <= thr)) rc = -5;
+  stats[0] = it;
+  stats[1] = calls;
+  stats[2] = rollbacks;
+  stats[3] = executed;
+  free(r); free(z); free(p); free(q); free(tmp); free(d);
+  free(cx); free(cr); free(cz); free(cp);
+  return rc;
+}

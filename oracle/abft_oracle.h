@@ -109,6 +109,18 @@ int or_pcg(const or_csr *A, int32_t bs, const int32_t *c_row_ptr, const int32_t 
            const double *diag, double tol, int64_t max_iter, const or_inject *inj,
            int32_t max_rounds, int32_t check, double *res_hist, int64_t *stats);
 
+/* --- related-work baseline for the PCG case study: checkpoint-rollback ---
+ * (R26-R27) Jacobi-PCG whose every SpMV
+ * is checked by the dense check with tau = ||v||_2; the state
+ * (x, r, z, p, rho, it) is sampled every ckpt_every iterations (20)
+ * and restored on a detection.  c: or_dense_encode's checksum.  Rate faults
+ * hit y only (call j = inj->call + j-th executed SpMV).  max_iter bounds
+ * executed iterations (<= 0 -> 10 N).  stats [5]: iterations of the result,
+ * SpMV calls, rollbacks, executed iterations, 0.  Returns 0 / -5 / -7. */
+int or_pcg_cr(const or_csr *A, const double *c, const double *b, double *x, const double *diag,
+              double tol, int64_t max_iter, const or_inject *inj, int32_t ckpt_every,
+              double *res_hist, int64_t *stats);
+
 #ifdef __cplusplus
 }
 #endif

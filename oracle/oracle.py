@@ -74,6 +74,8 @@ def lib():
         L.or_dense_encode.argtypes = [P, P, P]
         L.or_dense_spmv.restype = C.c_int
         L.or_dense_spmv.argtypes = [P, P, d, i32, P, P, i32, P, P, P, P]
+        L.or_pcg_cr.restype = C.c_int
+        L.or_pcg_cr.argtypes = [P, P, P, P, P, d, i64, P, i32, P, P]
         L.or_pcg.restype = C.c_int
         L.or_pcg.argtypes = [P, i32, P, P, P, P, P, P, P, d, i64, P, i32, i32, P, P]
     return _lib
@@ -342,3 +344,33 @@ def pcg(A, enc: Encoded, b, x0, diag=None, tol=1e-6, max_iter=0, inj: Inject | N
     it = int(stats[0])
     return PcgResult(st, x, hist[: it + 1].copy(), it, int(stats[1]), int(stats[2]),
                      int(stats[3]), int(stats[4]))
+
+
+def pcg_cr(A, denc: DenseEncoded, b, x0, diag=None, tol=1e-6, max_iter=0,
+           inj: "Inject | None" = None, ckpt_every: int = 20) -> "CrResult":
+    """Checkpoint-rollback PCG baseline (abft_oracle.h or_pcg_cr).
+    stats: iters, spmv_calls, rollbacks, executed, 0."""
+    r = _CsrRef(A)
+    n = A.n
+    x = np.array(x0, dtype=np.float64, copy=True)
+    b = np.ascontiguousarray(b, dtype=np.float64)
+    mi = max_iter if max_iter > 0 else 10 * n
+    hist = np.zeros(mi + 1)
+    st = np.zeros(5, dtype=np.int64)
+    dg = None if diag is None else np.ascontiguousarray(diag, dtype=np.float64)
+    ist = inj._struct() if inj is not None else None
+    status = lib().or_pcg_cr(r.ref(), _p(denc.c), _p(b), _p(x), _p(dg), tol, mi,
+                             C.byref(ist) if ist is not None else None, ckpt_every, _p(hist),
+                             _p(st))
+    return CrResult(status, x, hist[: st[0] + 1], int(st[0]), int(st[1]), int(st[2]), int(st[3]))
+
+
+@dataclass
+class CrResult:
+    status: int
+    x: np.ndarray
+    res_hist: np.ndarray
+    iters: int        # iterations of the returned solution
+    spmv_calls: int
+    rollbacks: int
+    executed: int     # executed iterations (re-executions count)

@@ -643,3 +643,51 @@ class TestDenseCheck:
         enc = O.encode(A, 32)
         ref = O.abft_spmv(A, enc, x, inj)
         assert ref.flags[0].tolist() == [i // 32]
+
+
+# --------------------------------------------------------------------------
+# Related-work baseline: checkpoint-rollback PCG with dense
+# checks (R26-R27).  Pinned: without faults it IS the
+# plain Jacobi-PCG (itself pinned to SciPy above), bit for bit; under faults
+# its bookkeeping obeys the rollback identities.  The rollback trajectory
+# under random faults has no external reference (parity partially pinned).
+# --------------------------------------------------------------------------
+class TestPcgCheckpoint:
+    def test_fault_free_equals_plain_pcg(self, O):
+        A = G.laplacian_3d_7pt(10)
+        enc = O.encode(A, 32)
+        den = O.dense_encode(A)
+        b = O.spmv(A, G.uniform_vector(A.n, 43))
+        x0 = G.uniform_vector(A.n, 44)
+        ref = O.pcg(A, enc, b, x0, tol=1e-6, check=False)
+        r = O.pcg_cr(A, den, b, x0, tol=1e-6)
+        assert r.status == 0 and r.rollbacks == 0
+        assert r.iters == ref.iters == r.executed and r.spmv_calls == ref.iters + 1
+        assert np.array_equal(r.res_hist, ref.res_hist) and np.array_equal(r.x, ref.x)
+
+    def test_rollback_bookkeeping(self, O):
+        A = G.laplacian_3d_7pt(8)
+        den = O.dense_encode(A)
+        xs = G.uniform_vector(A.n, 43)
+        b = O.spmv(A, xs)
+        x0 = G.uniform_vector(A.n, 44)
+        r = O.pcg_cr(A, den, b, x0, tol=1e-6, inj=O.Inject.rate(seed=9, lam=1e-4, targets=1))
+        assert r.rollbacks > 0
+        # every executed iteration either advanced or was rolled back; each
+        # rollback discards at most ckpt_every - 1 advanced iterations
+        assert r.executed >= r.iters + r.rollbacks
+        assert r.executed <= r.iters + r.rollbacks * 20
+        assert r.spmv_calls >= r.executed + 1
+        if r.status == 0:  # converged: the recursive residual met the test
+            assert r.res_hist[-1] <= 1e-6 * np.linalg.norm(b)
+
+    def test_sample_every_iteration_loses_nothing(self, O):
+        # ckpt_every = 1: a rollback restores the state of the iteration it
+        # interrupted, so executed = iters + rollbacks exactly
+        A = G.laplacian_3d_7pt(8)
+        den = O.dense_encode(A)
+        b = O.spmv(A, G.uniform_vector(A.n, 43))
+        x0 = G.uniform_vector(A.n, 44)
+        r = O.pcg_cr(A, den, b, x0, tol=1e-6, ckpt_every=1,
+                     inj=O.Inject.rate(seed=9, lam=1e-4, targets=1))
+        assert r.rollbacks > 0 and r.executed == r.iters + r.rollbacks
