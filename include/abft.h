@@ -211,8 +211,14 @@ typedef struct {
  * initial guess in x (overwritten with the solution).  diag: nullable device
  * [n] (NULL -> the diagonal of A).  Stops when ||r||_2 <= tol * ||b||_2
  * (R16) or after max_iter iterations (<= 0 -> 10 N).
- * check != 0 protects every SpMV (detect + correct); check == 0 runs the
- * unprotected baseline with the same kernels.  inj: nullable; its `call`
+ * check == 1 protects every SpMV (detect + correct); check == 0 runs the
+ * unprotected baseline with the same kernels; check == 2 runs the related-work
+ * CHECKPOINTING baseline: every SpMV checked by
+ * the dense check with tau = ||v||_2 (needs abft_dense_encode), the
+ * state (x, r, z, p, rho) sampled every 20 iterations and restored
+ * on a detection; rate faults hit y only; max_iter bounds executed
+ * iterations; stats: flagged_blocks = rollbacks, recomputed_blocks =
+ * discarded iterations (R26-R27).  inj: nullable; its `call`
  * is the index of the first SpMV (call + j for the j-th).  res_hist:
  * nullable device [max_iter + 1] of ||r_j||_2.  stats: nullable (host).
  * b, x, diag and res_hist must be 16-byte aligned (128-bit vector accesses;

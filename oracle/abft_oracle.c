@@ -588,7 +588,12 @@ int or_dense_spmv(const or_csr *A, const double *c, double k35, int32_t bound35,
                   const double *x, const or_inject *inj, int32_t max_rounds, double *y,
                   double *y_pre, double *out, int32_t *flag_rounds) {
   int64_t n = A->n;
-  if (inj && inj->mode == OR_INJ_RATE) return -1; /* list mode only */
+  void *keep = NULL;
+  or_inject lst;
+  if (inj && inj->mode == OR_INJ_RATE) { /* rate mode: y ops of round 0 only (R25) */
+    lst = rate_to_list(A, 32, NULL, 0, inj, 0, &keep);
+    inj = &lst;
+  }
   double *tmp = (double *)malloc(sizeof(double) * (size_t)(n > 0 ? n : 1));
   for (int64_t i = 0; i < n; ++i) tmp[i] = x[i] * x[i];
   double beta = sqrt(or_pw(tmp, n)); /* ||x||_2, R10 */
@@ -620,6 +625,7 @@ int or_dense_spmv(const or_csr *A, const double *c, double k35, int32_t bound35,
     if (r == max_rounds) rc = -6;
   }
   free(tmp);
+  free(keep);
   return rc;
 }
 

@@ -93,8 +93,9 @@ int or_abft_spmv(const or_csr *A, int32_t bs, const int32_t *c_row_ptr, const in
  * or_dense_spmv: bound35 = 0 -> tau = ||x||_2 (norm-based), 1 -> tau =
  * k35 ||x||_2.  flag_rounds [max_rounds+1]: 1 where round r's check failed
  * (round r >= 1 = r-th complete recomputation).  out [4] (nullable): round 0's
- * t1, t2, beta, tau.  List injection only (index 0 for t1 / t2).  Returns 0,
- * -6 if still flagged after max_rounds recomputations, -1 for rate mode. */
+ * t1, t2, beta, tau.  List faults: index 0 for t1 / t2; rate mode: the plan
+ * over the SpMV's y ops of round 0 (R25).  Returns 0, -6 if still flagged
+ * after max_rounds recomputations. */
 void or_dense_encode(const or_csr *A, double *c, double *k35);
 int or_dense_spmv(const or_csr *A, const double *c, double k35, int32_t bound35,
                   const double *x, const or_inject *inj, int32_t max_rounds, double *y,

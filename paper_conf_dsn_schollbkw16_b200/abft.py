@@ -373,10 +373,15 @@ class Handle:
     # -- PCG ----------------------------------------------------------------
     def pcg(self, b, x, diag=None, tol=1e-6, max_iter=0, inject: Inject | None = None,
             check=True, res_hist=None, stream=None):
+        # check: True = the method's protected SpMV, False = unprotected,
+        # "checkpoint" = dense-check checkpoint-rollback baseline (
+        # needs dense_encode(); stats: flagged_blocks = rollbacks,
+        # recomputed_blocks = discarded iterations)
         st = PcgStats()
         inj = inject.struct() if inject is not None else None
+        mode = 2 if check == "checkpoint" else (1 if check else 0)
         status = lib().abft_pcg(self._h, _ptr(b), _ptr(x), _ptr(diag), tol, max_iter,
-                                C.byref(inj) if inj is not None else None, 1 if check else 0,
+                                C.byref(inj) if inj is not None else None, mode,
                                 _ptr(res_hist), C.byref(st), _stream(stream))
         if status not in (OK, ENOCONV, EBREAKDOWN):
             _check(status, "abft_pcg")

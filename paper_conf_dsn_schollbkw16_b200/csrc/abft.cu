@@ -440,6 +440,36 @@ abft_status launch_finish(const abft_ctx *h, const SpmvArgs &a, int rounds, bool
   return ABFT_OK;
 }
 
+// Dense-check baseline after a plain SpMV (kernels_dense.cuh): one PDL-
+// launched persistent kernel; rounds > 0 = complete recomputations.
+abft_status launch_dense(const abft_ctx *h, const SpmvArgs &a, int rounds, bool bound35,
+                         cudaStream_t s) {
+  DenseArgs d;
+  d.a = a;
+  d.c = h->dn_c;
+  d.k35 = h->dn_k35;
+  d.bound35 = bound35 ? 1 : 0;
+  d.rounds = rounds;
+  d.part = h->dn_part;
+  d.res = h->dn_res;
+  d.flag_rounds = h->dn_flags;
+  cudaLaunchConfig_t cfg;
+  memset(&cfg, 0, sizeof cfg);
+  cfg.gridDim = dim3((unsigned)h->correct_grid);
+  cfg.blockDim = dim3(256);
+  cfg.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  if (a.inj.mode != 0)
+    CK(cudaLaunchKernelEx(&cfg, k_dense<true>, d));
+  else
+    CK(cudaLaunchKernelEx(&cfg, k_dense<false>, d));
+  return ABFT_OK;
+}
+
 size_t g_dyn_smem_limit = 0;  // opt-in shared memory per block minus static smem
 
 template <typename Kern>

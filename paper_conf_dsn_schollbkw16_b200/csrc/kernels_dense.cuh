@@ -266,6 +266,7 @@ __global__ void __launch_bounds__(256) k_dense(const DenseArgs d) {
   __shared__ double s_w[3][8];
   asm volatile("griddepcontrol.wait;" ::: "memory");
   const SpmvArgs &a = d.a;
+  if (skip_call(a)) return;  // PCG: solver no longer running
   const int64_t n = a.n;
   const int64_t nch = (n + kDenseRows - 1) / kDenseRows;
   double beta = 0.0, tau = 0.0;

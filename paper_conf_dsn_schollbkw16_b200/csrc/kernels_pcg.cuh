@@ -26,7 +26,10 @@ struct PcgScalars {
   int64_t it, max_iter;
   int64_t flagged, recomputed, uncorrected, calls;
   int32_t state;
-  int32_t pad;
+  int32_t skip_it;           // checkpoint mode: this iteration was rolled back
+  int64_t upd;               // host iteration index of the last executed update
+  double ck_rho, ck_res;     // checkpoint mode: sampled scalars
+  int64_t ck_it;
 };
 
 struct PcgArgs {
@@ -42,6 +45,12 @@ struct PcgArgs {
   const int32_t *n_flags;         // protected-SpMV flag counts (stats)
   int32_t max_rounds;
   int32_t check;
+  // checkpoint-rollback baseline: dense-check flag of the
+  // iteration's SpMV, sampled x | r | z | p (4 n), sampling interval
+  int32_t cr;
+  int32_t ckpt_every;
+  const int32_t *dflag;
+  double *ck;
 };
 
 // Eight consecutive doubles v[0..8) at p + 8t (or absent past n).
@@ -130,10 +139,12 @@ __device__ __forceinline__ bool last_cta(unsigned *ticket, int *s_flag) {
 }
 
 __device__ __forceinline__ bool pcg_skip(const PcgScalars *sc) {
-  return *(volatile const int32_t *)&sc->state != PCG_RUN;
+  return *(volatile const int32_t *)&sc->state != PCG_RUN ||
+         *(volatile const int32_t *)&sc->skip_it != 0;
 }
 
 __device__ __forceinline__ void pcg_stats(const PcgArgs &a, PcgScalars *sc) {
+  if (a.cr) return;  // checkpoint mode counts in k_pcg_cr
   sc->calls += 1;
   if (a.check) {
     const int32_t *nf = a.n_flags;
@@ -176,6 +187,14 @@ __global__ void __launch_bounds__(kPcgThreads) k_pcg_init(const PcgArgs a) {
   st8(a.r, r, i0, a.n);
   st8(a.z, z, i0, a.n);
   st8(a.p, z, i0, a.n);
+  if (a.cr) {  // sample 0: x0, r0, z0, p0
+    double xv[8];
+    ld8(xv, a.x, i0, a.n);
+    st8(a.ck, xv, i0, a.n);
+    st8(a.ck + a.n, r, i0, a.n);
+    st8(a.ck + 2 * a.n, z, i0, a.n);
+    st8(a.ck + 3 * a.n, z, i0, a.n);
+  }
   const double RZc = cta_pw(rz, i0, a.n, s_w);
   const double RRc = cta_pw(rr, i0, a.n, s_w);
   const double BBc = cta_pw(bb, i0, a.n, s_w);
@@ -198,6 +217,13 @@ __global__ void __launch_bounds__(kPcgThreads) k_pcg_init(const PcgArgs a) {
     if (a.hist) a.hist[0] = sc->res;
     sc->state = (sc->res <= sc->thr) ? PCG_CONVERGED : (sc->max_iter <= 0 ? PCG_MAXITER : PCG_RUN);
     if (!(sc->res == sc->res)) sc->state = PCG_BREAKDOWN;
+    if (a.cr) {
+      sc->calls += 1;
+      sc->skip_it = 0;
+      sc->ck_rho = sc->rho;
+      sc->ck_res = sc->res;
+      sc->ck_it = 0;
+    }
     *a.ticket = 0u;
   }
 }
@@ -232,7 +258,7 @@ __global__ void __launch_bounds__(kPcgThreads) k_pcg_dot(const PcgArgs a) {
 
 // x += alpha p; r -= alpha q; z = r / d; rho' = PW(r.z); res = ||r||;
 // beta = rho'/rho; convergence test (R15, R16).
-__global__ void __launch_bounds__(kPcgThreads) k_pcg_update(const PcgArgs a) {
+__global__ void __launch_bounds__(kPcgThreads) k_pcg_update(const PcgArgs a, int64_t iter) {
   __shared__ double s_w[8];
   __shared__ double s_red[kPcgThreads];
   __shared__ int s_flag;
@@ -273,6 +299,7 @@ __global__ void __launch_bounds__(kPcgThreads) k_pcg_update(const PcgArgs a) {
     if (a.hist) a.hist[sc->it] = res;
     sc->beta = __ddiv_rn(RZ, sc->rho);
     sc->rho = RZ;
+    sc->upd = iter;
     if (res <= sc->thr) sc->state = PCG_CONVERGED;
     else if (!(res == res)) sc->state = PCG_BREAKDOWN;
     else if (sc->it >= sc->max_iter) sc->state = PCG_MAXITER;
@@ -283,8 +310,7 @@ __global__ void __launch_bounds__(kPcgThreads) k_pcg_update(const PcgArgs a) {
 // p = z + beta p.  Runs in the iteration that converged too (as the oracle);
 // skipped only when this iteration's update was skipped.
 __global__ void __launch_bounds__(kPcgThreads) k_pcg_p(const PcgArgs a, int64_t iter) {
-  const int64_t it = *(volatile const int64_t *)&a.sc->it;
-  if (it != iter) return;  // this iteration did not execute
+  if (*(volatile const int64_t *)&a.sc->upd != iter) return;  // this iteration did not execute
   const double beta = a.sc->beta;
   const int64_t i0 = (int64_t)blockIdx.x * kPcgRows + threadIdx.x * kPcgPer;
   double zv[8], pv[8];
@@ -293,6 +319,54 @@ __global__ void __launch_bounds__(kPcgThreads) k_pcg_p(const PcgArgs a, int64_t 
 #pragma unroll
   for (int u = 0; u < 8; ++u) pv[u] = dadd(zv[u], dmul(beta, pv[u]));
   st8(a.p, pv, i0, a.n);
+  // checkpoint mode: sample (x, r, z, p, rho, it) every ckpt_every iterations
+  const int64_t it = a.sc->it;
+  if (a.cr && a.ckpt_every > 0 && it % a.ckpt_every == 0) {
+    double xv[8], rv[8];
+    ld8(xv, a.x, i0, a.n);
+    ld8(rv, a.r, i0, a.n);
+    st8(a.ck, xv, i0, a.n);
+    st8(a.ck + a.n, rv, i0, a.n);
+    st8(a.ck + 2 * a.n, zv, i0, a.n);
+    st8(a.ck + 3 * a.n, pv, i0, a.n);
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+      a.sc->ck_rho = a.sc->rho;
+      a.sc->ck_res = a.sc->res;
+      a.sc->ck_it = it;
+    }
+  }
+}
+
+// Checkpoint mode: after the dense check of this iteration's
+// SpMV, either continue (skip_it = 0) or restore the last sample and mark
+// the iteration rolled back (its dot / update / p kernels then return).
+__global__ void __launch_bounds__(kPcgThreads) k_pcg_cr(const PcgArgs a) {
+  if (*(volatile const int32_t *)&a.sc->state != PCG_RUN) return;
+  const bool flagged = *(volatile const int32_t *)a.dflag != 0;
+  if (flagged) {
+    const int64_t i0 = (int64_t)blockIdx.x * kPcgRows + threadIdx.x * kPcgPer;
+    double v[8];
+    ld8(v, a.ck, i0, a.n);
+    st8(a.x, v, i0, a.n);
+    ld8(v, a.ck + a.n, i0, a.n);
+    st8(a.r, v, i0, a.n);
+    ld8(v, a.ck + 2 * a.n, i0, a.n);
+    st8(a.z, v, i0, a.n);
+    ld8(v, a.ck + 3 * a.n, i0, a.n);
+    st8(a.p, v, i0, a.n);
+  }
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    PcgScalars *sc = a.sc;
+    sc->calls += 1;
+    sc->skip_it = flagged ? 1 : 0;
+    if (flagged) {
+      sc->rho = sc->ck_rho;
+      sc->res = sc->ck_res;
+      sc->recomputed += sc->it - sc->ck_it;  // advanced iterations discarded
+      sc->it = sc->ck_it;
+      sc->flagged += 1;                      // detections = rollbacks
+    }
+  }
 }
 
 }  // namespace abft

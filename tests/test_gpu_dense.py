@@ -83,3 +83,55 @@ def test_dense_detect_only(torch_cuda, O):
     plan = G.FaultPlan([0], [0], [7], [scale_mask(y[7])])
     ref, _ = run_pair(O, torch_cuda, A, x, plan=plan, correct=False)
     assert ref.flag_rounds.tolist() == [1]
+
+
+# --------------------------------------------------------------------------
+# Checkpoint-rollback PCG baseline vs or_pcg_cr
+# --------------------------------------------------------------------------
+def _cr_case(O, torch, A, inj_kw=None, max_iter=0):
+    from paper_conf_dsn_schollbkw16_b200 import encode
+    den = O.dense_encode(A)
+    b = O.spmv(A, G.uniform_vector(A.n, 43))
+    x0 = G.uniform_vector(A.n, 44)
+    oinj = O.Inject.rate(**inj_kw) if inj_kw else None
+    ref = O.pcg_cr(A, den, b, x0, tol=1e-6, inj=oinj, max_iter=max_iter)
+    h = encode(A, 32).dense_encode()
+    bd = torch.from_numpy(b).cuda()
+    xd = torch.from_numpy(x0.copy()).cuda()
+    mi = max_iter if max_iter > 0 else 10 * A.n
+    hist = torch.zeros(mi + 1, dtype=torch.float64, device="cuda")
+    status, st = h.pcg(bd, xd, tol=1e-6, inject=gpu_inject(rate=inj_kw) if inj_kw else None,
+                       check="checkpoint", res_hist=hist, max_iter=max_iter)
+    torch.cuda.synchronize()
+    return ref, status, st, xd.cpu().numpy(), hist.cpu().numpy()[: st["iters"] + 1]
+
+
+@pytest.mark.parametrize("inj", [None, dict(seed=9, lam=1e-4, targets=1),
+                                 dict(seed=5, lam=3e-4, targets=1, call=11)])
+def test_pcg_checkpoint_parity(O, torch_cuda, inj):
+    A = G.laplacian_3d_7pt(8) if inj else G.laplacian_3d_7pt(16)
+    ref, status, st, x, hist = _cr_case(O, torch_cuda, A, inj)
+    assert status == ref.status
+    assert st["iters"] == ref.iters and st["spmv_calls"] == ref.spmv_calls
+    assert st["flagged_blocks"] == ref.rollbacks
+    assert st["recomputed_blocks"] == ref.executed - ref.iters - ref.rollbacks
+    assert_bits_equal(hist, ref.res_hist, "residual history")
+    assert_bits_equal(x, ref.x, "solution")
+    if inj and inj["seed"] == 9:
+        assert ref.rollbacks > 0
+
+
+def test_dense_rate_mode(O, torch_cuda):
+    # rate faults on the dense-check SpMV: the y-only plan (R25), both sides
+    A = MATRICES["lap3d_16"]()
+    x = G.uniform_vector(A.n, 15)
+    from paper_conf_dsn_schollbkw16_b200 import encode
+    h = encode(A, 32).dense_encode()
+    e = O.dense_encode(A)
+    rate = dict(seed=4, lam=1e-4, targets=1, call=2)
+    ref = O.dense_spmv(A, e, x, inj=O.Inject.rate(**rate))
+    y = h.spmv_dense(torch_cuda.from_numpy(x).cuda(), inject=gpu_inject(rate=rate))
+    r = h.dense_result()
+    assert r["flag_rounds"].tolist() == ref.flag_rounds.tolist()
+    assert_bits_equal([r["t1"], r["t2"]], [ref.t1, ref.t2], "t1 t2")
+    assert_bits_equal(y.cpu().numpy(), ref.y, "y")
