@@ -182,9 +182,16 @@ def oracle_baseline(A, x, seconds=12.0, check=True):
 
 
 def run_pcg(args):
-    """configs[4]: Jacobi-PCG on the 3-D 7-pt Laplacian with the protected
-    SpMV: time-to-solution, iterations and overhead vs the same
-    solver with unprotected SpMVs, at a low and a 10^4x higher error rate."""
+    """configs[4]: Jacobi-PCG on the 3-D 7-pt Laplacian:
+    time-to-solution, iterations, success (Q17: converged and fault-free true
+    residual <= 10 tol) and overhead vs the same solver with unprotected SpMVs
+    (successful runs only), for the method (protected SpMV), the
+    related-work checkpointing baseline (dense checks, rollback to a sample
+    taken every 20 iterations) and no protection,
+    at lambda = 0, 1e-8, 1e-6, 1e-4.  --pcg-seeds fault seeds per
+    (scheme, lambda) give the success rates of Fig. 9.  Runs of
+    the checkpointing baseline are capped at 10x the fault-free iteration
+    count (10 N executed iterations at N = 7.1M is not runnable)."""
     import torch
 
     from paper_conf_dsn_schollbkw16_b200 import Inject, encode
@@ -192,39 +199,68 @@ def run_pcg(args):
     world, rank, local = dist_init()
     n3 = args.pcg_n
     A = G.laplacian_3d_7pt(n3)
-    h = encode(A, 32, args.max_rounds)
+    h = encode(A, 32, args.max_rounds).dense_encode()
     # b = A x* with x* seeded (R15/Q20); computed through the library's own
     # plain SpMV (inputs, not a parity check)
     xs = torch.from_numpy(G.uniform_vector(A.n, 43)).cuda()
     b = h.spmv(xs, mode=0)
     x0 = torch.from_numpy(G.uniform_vector(A.n, 44)).cuda()
+    bn = float(torch.linalg.norm(b))
     torch.cuda.synchronize()
+
+    def solve(check, lam, seed, max_iter=0):
+        inj = Inject.rate(seed=seed, lam=lam, targets=0b001 if check == "checkpoint" else 0b111) \
+            if lam > 0 else None
+        x = x0.clone()
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        status, st = h.pcg(b, x, tol=1e-6, inject=inj, check=check, max_iter=max_iter)
+        dt = time.perf_counter() - t0
+        rel = float(torch.linalg.norm(b - h.spmv(x, mode=0))) / bn
+        return dt, status, st, rel, bool(status == 0 and rel <= 1e-5)
+
+    solve(True, 0.0, 0)  # warm-up
+    clean_iters = None
     res = {}
-    for label, check, lam in [("unprotected", False, 0.0), ("protected", True, 0.0),
-                              ("protected_lam1e-8", True, 1e-8), ("protected_lam1e-4", True, 1e-4),
-                              ("unprotected_lam1e-4", False, 1e-4)]:
-        inj = Inject.rate(seed=7, lam=lam) if lam > 0 else None
-        times, st = [], None
-        for rep in range(max(1, args.pcg_reps)):
-            x = x0.clone()
-            torch.cuda.synchronize()
-            t0 = time.perf_counter()
-            status, st = h.pcg(b, x, tol=1e-6, inject=inj, check=check)
-            times.append(time.perf_counter() - t0)
-        # solution check: fault-free true residual (Q17)
-        r = b - h.spmv(x, mode=0)
-        rel = float(torch.linalg.norm(r) / torch.linalg.norm(b))
-        res[label] = {"status": status, "ms": round(1e3 * statistics.median(times), 3),
-                      "iters": st["iters"], "flagged_blocks": st["flagged_blocks"],
-                      "recomputed_blocks": st["recomputed_blocks"],
-                      "true_rel_residual": rel, "correct": bool(status == 0 and rel <= 1e-5)}
-    base = res["unprotected"]["ms"]
-    for k, v in res.items():
-        v["overhead_pct"] = round((v["ms"] / base - 1) * 100, 2)
+    schemes = [("unprotected", False), ("protected", True), ("checkpoint", "checkpoint")]
+    for lam in (0.0, 1e-8, 1e-6, 1e-4):
+        for name, check in schemes:
+            if name == "unprotected" and lam not in (0.0, 1e-4):
+                continue
+            cap = 0 if (check != "checkpoint" or lam == 0 or clean_iters is None) else 10 * clean_iters
+            reps = max(1, args.pcg_reps) if lam == 0 else max(1, args.pcg_seeds)
+            times, ok, stt = [], 0, None
+            for rep in range(reps):
+                dt, status, st, rel, good = solve(check, lam, 7 + rep, cap)
+                ok += int(good)
+                if good:
+                    times.append(dt)
+                stt = (status, st, rel)
+            if name == "unprotected" and lam == 0:
+                clean_iters = stt[1]["iters"]
+            status, st, rel = stt
+            res[f"{name}_lam{lam:g}"] = {
+                "scheme": name, "lambda": lam, "runs": reps, "success_rate": round(ok / reps, 3),
+                "ms": round(1e3 * statistics.median(times), 3) if times else None,
+                "iters": st["iters"], "spmv_calls": st["spmv_calls"],
+                "detections": st["flagged_blocks"], "recomputed": st["recomputed_blocks"],
+                "last_status": status, "last_true_rel_residual": rel,
+                "max_iter_cap": cap or "10N"}
+    base = res["unprotected_lam0"]["ms"]
+    for v in res.values():
+        v["overhead_pct"] = round((v["ms"] / base - 1) * 100, 2) if v["ms"] else None
     if rank == 0:
         print(json.dumps({"metric": "PCG time-to-solution (ms), Jacobi, tol 1e-6",
                           "workload": f"3-D 7-point Laplacian {n3}^3 (BASELINE configs[4])",
-                          "n": A.n, "nnz": A.nnz, "n_gpus": world, "results": res}), flush=True)
+                          "n": A.n, "nnz": A.nnz, "n_gpus": world,
+                          "schemes": "protected = this method (b_s 32, detect + partial "
+                                     "recomputation); checkpoint = dense check + rollback to a "
+                                     "sample every 20 iterations (P:286-292); faults: rate mode "
+                                     "per arithmetic op (P:284), checkpoint baseline on y only",
+                          "paper_context": "K80, SuiteSparse: overhead 39.8% (ours) / 62.9% "
+                                           "(checkpointing) at 1e-8, 52.3% / 162.9% at 1e-4 "
+                                           "(P:310-316)",
+                          "results": res}), flush=True)
 
 
 def run_reference(args):
@@ -572,6 +608,7 @@ def main():
                     help="SURVEY §8(f)1: the method vs the dense check + complete recomputation")
     ap.add_argument("--pcg-n", type=int, default=192)
     ap.add_argument("--pcg-reps", type=int, default=3)
+    ap.add_argument("--pcg-seeds", type=int, default=3, help="fault seeds per (scheme, lambda)")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     args = ap.parse_args()
