@@ -42,7 +42,7 @@ typedef enum {
   ABFT_EINVAL = -1,        /* bad argument (host-detected) */
   ABFT_ECUDA = -2,         /* CUDA runtime error (see abft_last_cuda_error) */
   ABFT_ENOMEM = -3,        /* device allocation failed */
-  ABFT_ENOTSUP = -4,       /* unsupported configuration (e.g. block_size > 32) */
+  ABFT_ENOTSUP = -4,       /* unsupported configuration (e.g. block_size > 1024) */
   ABFT_ENOCONV = -5,       /* PCG: not converged within max_iter */
   ABFT_EUNCORRECTED = -6,  /* blocks still flagged after max_rounds recomputations */
   ABFT_EBREAKDOWN = -7     /* PCG: p.q <= 0 or NaN residual */
@@ -110,8 +110,10 @@ enum {
 /* Build C (CSR: nb rows, ascending columns = the non-empty columns of A_k,
  * values = column sums of A_k) and K_k = ((n_k + 2 b_s - 2)
  * * sum_{i in k} ||a_i||_2 + n_k ||c_k||_2) * 2^-53 (eps_M of P:154),
- * so that tau_k = K_k * ||x||_2.  block_size: power of two in [1, 32]
- * (default 32 = the paper's choice); otherwise ABFT_ENOTSUP.
+ * so that tau_k = K_k * ||x||_2.  block_size: power of two in [1, 1024]
+ * (default 32 = the paper's choice; 64 .. 1024 run the
+ * block-size sweep kernels of kernels_bigblock.cuh, one warp per block, for
+ * Fig. 4 / Fig. 7 of P:248-270, not a tuned path); larger: ABFT_ENOTSUP.
  * max_rounds: correction rounds for ABFT_AUTOCORRECT / abft_pcg (>= 1, <= 16;
  * 0 -> 4).  flags: 0, or ABFT_ENCODE_C_CSR to stream C in the paper's plain
  * CSR form (FP64 values, int32 columns) instead of the lossless compact form

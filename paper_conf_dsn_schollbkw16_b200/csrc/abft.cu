@@ -14,6 +14,7 @@
 #include "kernels_spmv.cuh"
 #include "kernels_irr.cuh"
 #include "kernels_dense.cuh"
+#include "kernels_bigblock.cuh"
 
 #include <cub/device/device_radix_sort.cuh>
 
@@ -387,6 +388,13 @@ void launch_irr(const abft_ctx *h, const SpmvArgs &a, cudaStream_t s) {
 template <bool CHECK, bool INJECT>
 abft_status launch_fused_t(const abft_ctx *h, SpmvArgs a, cudaStream_t s) {
   // k_lean needs 16-B aligned operands for its bulk copies (x per call)
+  if (h->bs > 32) {  // SURVEY §8(f)2 sweep: one warp per big block
+    const int64_t need = (h->nb + 3) / 4;
+    k_bigblock<CHECK, INJECT><<<(unsigned)std::max<int64_t>(1, std::min<int64_t>((int64_t)h->num_sms * 16, need)),
+                                128, 0, s>>>(a);
+    CK(cudaGetLastError());
+    return ABFT_OK;
+  }
   const bool lean = h->lean && aligned16(a.xr);
   const int64_t ngen = lean ? h->n_glist : h->n_glist_nl;
   a.glist = lean ? h->glist : h->glist_nl;
@@ -666,9 +674,9 @@ abft_status plan_fused(abft_ctx *h, cudaStream_t s) {
     }
     own.push_back({key, {first, (int32_t)hbeg.size() - first}});
   };
-  for (int64_t i = 0; i < h->n; ++i)
+  for (int64_t i = 0; i < h->n && h->bs <= 32; ++i)  // b_s > 32: k_bigblock reduces any length
     if (rp[i + 1] - rp[i] > kHubLen) add_hub(rp[i], rp[i + 1] - rp[i], false, (int32_t)((i / 32) * 64 + (i % 32)));
-  for (int64_t k = 0; k < h->nb; ++k)
+  for (int64_t k = 0; k < h->nb && h->bs <= 32; ++k)
     if (crp[k + 1] - crp[k] > kHubLen) {
       const int64_t r = k * h->bs;
       add_hub(crp[k], crp[k + 1] - crp[k], true, (int32_t)((r / 32) * 64 + 32 + (r % 32) / h->bs));
@@ -848,7 +856,7 @@ abft_status abft_encode(const abft_csr_t *A, int32_t block_size, int32_t max_rou
     return ABFT_EINVAL;
   if (!A->row_ptr || (A->nnz > 0 && (!A->col_idx || !A->val))) return ABFT_EINVAL;
   if (block_size <= 0 || (block_size & (block_size - 1)) != 0) return ABFT_EINVAL;
-  if (block_size > 32) return ABFT_ENOTSUP;
+  if (block_size > 1024) return ABFT_ENOTSUP;
   if (max_rounds == 0) max_rounds = 4;
   if (max_rounds < 1 || max_rounds > 16) return ABFT_EINVAL;
   cudaStream_t s = (cudaStream_t)stream;
@@ -901,7 +909,11 @@ abft_status abft_encode(const abft_csr_t *A, int32_t block_size, int32_t max_rou
   ea.crp = h->c_rp;
   ea.K = h->K;
   const unsigned egrid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((h->nb + 7) / 8, 65535));
-  k_encode<false><<<egrid, 256, 0, s>>>(ea);
+  const unsigned bgrid = (unsigned)std::max<int64_t>(1, std::min<int64_t>(h->nb, (int64_t)num_sms * 8));
+  if (h->bs > 32)
+    k_encode_big<false><<<bgrid, h->bs, 0, s>>>(ea);
+  else
+    k_encode<false><<<egrid, 256, 0, s>>>(ea);
   k_scan_local<<<(unsigned)nscan, 1024, 0, s>>>(counts, h->c_rp, h->nb, totals);
   k_scan_totals<<<1, 1024, 0, s>>>(totals, nscan, h->c_rp + h->nb);
   k_scan_add<<<(unsigned)nscan, 1024, 0, s>>>(h->c_rp, h->nb, totals);
@@ -922,7 +934,10 @@ abft_status abft_encode(const abft_csr_t *A, int32_t block_size, int32_t max_rou
     return fail(st);
   ea.ccol = h->c_col;
   ea.cval = h->c_val;
-  k_encode<true><<<egrid, 256, 0, s>>>(ea);
+  if (h->bs > 32)
+    k_encode_big<true><<<bgrid, h->bs, 0, s>>>(ea);
+  else
+    k_encode<true><<<egrid, 256, 0, s>>>(ea);
   if ((e = cudaGetLastError()) != cudaSuccess) return fail(cuda_fail(e, "encode fill"));
   if ((e = cudaMemsetAsync(h->c_col + h->nnz_c, 0, 8 * sizeof(int32_t), s)) ||
       (e = cudaMemsetAsync(h->c_val + h->nnz_c, 0, 8 * sizeof(double), s)))

@@ -65,7 +65,7 @@ struct StageCfg {
 struct SpmvArgs {
   int64_t n;
   int64_t nnz;
-  int32_t bs;        // block size, power of two <= 32
+  int32_t bs;        // block size, power of two <= 1024 (> 32: kernels_bigblock.cuh)
   int32_t log2bs;
   int64_t nb;
   int64_t ngroups;
@@ -1134,6 +1134,82 @@ __global__ void __launch_bounds__(256) k_beta(const SpmvArgs a) {
   }
 }
 
+// ---------------------------------------------------------------------------
+// Row blocks larger than a warp (b_s = 64 .. 1024; kernels_bigblock.cuh).
+// ---------------------------------------------------------------------------
+// y rows of group g (round `round` of the fault model), lane per row; rows
+// longer than 32 entries by the warp.  Returns this lane's y (absent past n).
+template <bool INJECT>
+__device__ __forceinline__ double group_rows(const SpmvArgs &a, int64_t g, int round, int lane) {
+  const int64_t r0 = g * 32, i = r0 + lane;
+  const bool valid = i < a.n;
+  const GlobalSrc As{a.va, a.ci};
+  int32_t rs = 0, len = 0;
+  if (valid) {
+    rs = __ldg(a.rp + i);
+    len = __ldg(a.rp + i + 1) - rs;
+  }
+  const int small = len <= 32 ? len : 0;
+  const int maxs = warp_max_i(small);
+  double yv = 0.0;
+  if (valid && len <= 32 && maxs > 0) yv = lane_dot_any(As, rs, small, maxs, a.x);
+  unsigned longm = __ballot_sync(kFull, valid && len > 32);
+  while (longm) {
+    const int j = __ffs(longm) - 1;
+    longm &= longm - 1;
+    const double t = warp_dot(As, __shfl_sync(kFull, rs, j), __shfl_sync(kFull, len, j), a.x, lane);
+    if (lane == j) yv = t;
+  }
+  if (len == 0) yv = 0.0;
+  if (INJECT) {
+    const uint64_t m = group_y_mask(a.inj, round, r0, i, lane);
+    if (valid) yv = apply_mask(yv, m);
+  }
+  if (valid) a.y[i] = yv;
+  return valid ? yv : kAbsent;
+}
+
+// Block k (b_s > 32) of round `round`: y rows, t1, t2, and (round 0) the
+// groups' x^2 subtrees; returns s_k = t1 - t2 on every lane, *gs_out the
+// block's x^2 node (an aligned node of beta^2's tree).
+template <bool CHECK, bool INJECT>
+__device__ __forceinline__ double big_block(const SpmvArgs &a, int64_t k, int round, int lane,
+                                           double *gs_out) {
+  const int ngr = a.bs >> 5;
+  const int64_t g0 = k * ngr;
+  PwSeq t2s, gss;
+  for (int sub = 0; sub < ngr; ++sub) {
+    const int64_t g = g0 + sub;
+    if (g * 32 >= a.n) break;  // trailing absent subtrees
+    const double yv = group_rows<INJECT>(a, g, round, lane);
+    if (CHECK) {
+      t2s.push(bfly32(yv));
+      if (round == 0) {
+        const int64_t i = g * 32 + lane;
+        const double xv = i < a.n ? __ldg(a.xr + i) : 0.0;
+        const double gs = bfly32(i < a.n ? dmul(xv, xv) : kAbsent);
+        if (lane == 0) a.gsum[g] = gs;
+        gss.push(gs);
+      }
+    }
+  }
+  if (!CHECK) return 0.0;
+  double t2 = t2s.finish();
+  const int32_t cb = __ldg(a.crp + k), ce = __ldg(a.crp + k + 1);
+  const GlobalSrc Cs{a.cval, a.ccol};
+  double t1 = warp_dot(Cs, cb, ce - cb, a.x, lane);
+  if (INJECT && lane == 0) {
+    t1 = apply_mask(t1, fault_mask(a.inj, round, 1, k, 2 * (int64_t)(ce - cb)));
+    t2 = apply_mask(t2, fault_mask(a.inj, round, 2, k, min64(a.bs, a.n - k * a.bs)));
+  }
+  if (round == 0 && lane == 0 && a.dbg_t1) {
+    a.dbg_t1[k] = t1;
+    a.dbg_t2[k] = t2;
+  }
+  if (gs_out) *gs_out = gss.finish();
+  return dsub(t1, t2);
+}
+
 // Software grid barrier (all CTAs co-resident: grid <= SM count).
 // bar[0] = arrivals, bar[1] = generation.
 __device__ __forceinline__ void grid_sync(unsigned *bar) {
@@ -1226,6 +1302,12 @@ __global__ void __launch_bounds__(256) k_finish(const SpmvArgs a, int rounds) {
     int32_t *next = a.flags + (int64_t)round * a.nb;
     for (int64_t q = gw; q < nprev; q += nw) {
       const int64_t k = __ldcg(prev + q);
+      if (a.bs > 32) {  // big blocks: recompute the block's groups, re-verify
+        const double sv = big_block<true, INJECT>(a, k, round, lane, nullptr);
+        if (lane == 0 && !(fabs(sv) <= dmul(__ldg(a.K + k), beta)))
+          next[atomicAdd(a.n_flags + round, 1)] = (int32_t)k;
+        continue;
+      }
       const int64_t i = (k << a.log2bs) + lane;
       const bool valid = lane < a.bs && i < n;
       int32_t rs = 0, len = 0;

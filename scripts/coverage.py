@@ -177,7 +177,7 @@ def main():
         # SURVEY §8(f)2 / Fig. 7 vs block size: F1 per b_s
         runs = args.runs
         args.runs = args.bs_runs
-        for bs in (1, 2, 4, 8, 16, 32):
+        for bs in (1, 2, 4, 8, 16, 32, 64, 128, 256, 512):
             single_fault(args, bs=bs, dense=False)
         args.runs = runs
     print(json.dumps({"elapsed_s": round(time.time() - t0, 1)}))

@@ -77,5 +77,5 @@ def test_encode_rejects_bad_args_without_gpu(L):
     assert L.abft_encode(C.byref(csr), 32, 4, 0, None, C.byref(h)) == abft.EINVAL
     csr = abft._Csr(10, 0, 8, 0, 0)
     assert L.abft_encode(C.byref(csr), 3, 4, 0, None, C.byref(h)) == abft.EINVAL
-    assert L.abft_encode(C.byref(csr), 64, 4, 0, None, C.byref(h)) == abft.ENOTSUP
+    assert L.abft_encode(C.byref(csr), 2048, 4, 0, None, C.byref(h)) == abft.ENOTSUP
     assert L.abft_spmv(None, None, None, None, None, 1, None) == abft.EINVAL

@@ -397,3 +397,21 @@ def test_irregular_faults(O, torch_cuda, name, c_csr):
     ref = c.run(G.uniform_vector(A.n, 21), plan=plan)
     assert set(blocks) <= set(ref.flagged.tolist())
     c.run(G.uniform_vector(A.n, 22), rate=dict(seed=9, lam=1e-4, targets=0b111, call=3))
+
+
+@pytest.mark.parametrize("bs", [64, 128, 512])
+@pytest.mark.parametrize("name", ["lap3d_ragged", "rmat11", "hubs", "lap2d_64"])
+def test_big_block_sizes(O, torch_cuda, name, bs):
+    # b_s beyond a warp (kernels_bigblock.cuh) -- C, K, y, t1,
+    # t2, flags and corrections bit-exact against the oracle
+    A = MATRICES[name]()
+    c = Case(O, torch_cuda, A, bs=bs)
+    c.check_encoding()
+    ref = c.run(G.uniform_vector(A.n, 7))
+    assert ref.flagged.size == 0
+    nb = c.enc.nb
+    plan = G.FaultPlan([0, 0, 0, 1], [0, 1, 2, 0], [A.n // 2, 0, nb - 1, A.n // 2],
+                       [1 << 62, 1 << 61, 1 << 60, 1 << 59])
+    ref = c.run(G.uniform_vector(A.n, 8), plan=plan)
+    assert ref.flagged.size >= 1
+    c.run(G.uniform_vector(A.n, 9), rate=dict(seed=2, lam=1e-4, targets=0b111, call=1))
