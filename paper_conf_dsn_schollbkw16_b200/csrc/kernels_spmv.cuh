@@ -1060,6 +1060,7 @@ __global__ void __launch_bounds__(kLeanWarps * 32, ABFT_LEAN_MINB) k_lean(const 
 }
 
 constexpr int kBetaChunk = 1024;  // groups per aligned beta partial (k_finish, k_bpart)
+constexpr int kFewCand = 32;     // k_finish: up to this many candidates, CTA 0 alone confirms + corrects
 
 // PW over n doubles at p by one CTA of 256 threads: thread t owns an aligned
 // run of m = 2^k values, reduced 32 at a time in registers (32 loads in
@@ -1248,6 +1249,7 @@ __global__ void __launch_bounds__(256) k_finish(const SpmvArgs a, int rounds) {
   asm volatile("griddepcontrol.wait;" ::: "memory");
   if (skip_call(a)) return;
   const int lane = threadIdx.x & 31;
+  bool solo = false;  // CTA 0 alone runs confirmation and rounds
   if (CONFIRM) {
     const int nc = __ldcg(a.n_cand);
     if (nc == 0) {
@@ -1260,6 +1262,9 @@ __global__ void __launch_bounds__(256) k_finish(const SpmvArgs a, int rounds) {
     }
     if (blockIdx.x == 0 && threadIdx.x == 0)
       for (int r = 0; r <= a.max_rounds; ++r) a.n_flags[r] = 0;
+    // few candidates (the usual faulty call): after the beta partials CTA 0
+    // alone confirms and corrects, with block barriers instead of grid ones
+    solo = nc <= kFewCand;
     double beta;
     if (a.x_norm) {
       beta = __ldcg(a.x_norm);
@@ -1271,10 +1276,15 @@ __global__ void __launch_bounds__(256) k_finish(const SpmvArgs a, int rounds) {
         if (threadIdx.x == 0) a.bpart[c] = v;
       }
       grid_sync(a.gbar);
+      if (solo && blockIdx.x != 0) return;
       beta = __dsqrt_rn(cta_pw_array(a.bpart, nch, s_red));  // R10
     }
+    if (solo && blockIdx.x != 0) return;
     if (threadIdx.x == 0) s_beta = beta;
-    grid_sync(a.gbar);  // n_flags zeroed, partials consumed
+    if (solo)
+      __syncthreads();
+    else
+      grid_sync(a.gbar);  // n_flags zeroed, partials consumed
     beta = s_beta;
     for (int q = blockIdx.x * blockDim.x + threadIdx.x; q < nc; q += gridDim.x * blockDim.x) {
       const int32_t kk = __ldcg(a.cand + q);
@@ -1286,12 +1296,16 @@ __global__ void __launch_bounds__(256) k_finish(const SpmvArgs a, int rounds) {
       *a.beta = beta;
       *a.beta_valid = 1;
     }
-    grid_sync(a.gbar);  // round 0's list complete; every CTA has read n_cand
+    if (solo)
+      __syncthreads();
+    else
+      grid_sync(a.gbar);  // round 0's list complete; every CTA has read n_cand
     if (blockIdx.x == 0 && threadIdx.x == 0) *a.n_cand = 0;
   }
   if (rounds == 0 || __ldcg(a.n_flags) == 0) return;
-  const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  const int64_t gw = solo ? (int64_t)(threadIdx.x >> 5)
+                          : ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = solo ? (int64_t)(blockDim.x >> 5) : ((int64_t)gridDim.x * blockDim.x) >> 5;
   const double beta = __ldcg(a.beta);
   const int64_t n = a.n;
   const LdgSrc As{a.va, a.ci}, Cs{a.cval, a.ccol};
@@ -1347,7 +1361,12 @@ __global__ void __launch_bounds__(256) k_finish(const SpmvArgs a, int rounds) {
           next[atomicAdd(a.n_flags + round, 1)] = (int32_t)k;
       }
     }
-    if (round < rounds) grid_sync(a.gbar);
+    if (round < rounds) {
+      if (solo)
+        __syncthreads();
+      else
+        grid_sync(a.gbar);
+    }
   }
 }
 
