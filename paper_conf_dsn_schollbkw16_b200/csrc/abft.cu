@@ -77,6 +77,7 @@ struct abft_ctx {
   int64_t nnz_cpad = 0;      // compact slots incl. row padding
   StageCfg stage{};
   bool lean = false;        // k_lean usable (b_s = 32, 16-B aligned A)
+  bool lean_short = false;  // every k_lean group's rows <= 8 entries (SHORT instantiation)
   size_t fused_smem = 0;
   int fused_grid = 1;       // k_lean grid (persistent, one wave)
   uint8_t *lean_ok = nullptr;  // [ngroups] groups k_lean takes
@@ -358,7 +359,8 @@ template <bool CHECK, bool INJECT>
 void launch_lean(const abft_ctx *h, const SpmvArgs &a, cudaStream_t s) {
   const dim3 grid(h->fused_grid), block(h->stage.warps * 32);
 #define LEAN(CF)                                                                      \
-  (h->stage.nstage == 3 ? k_lean<CHECK, INJECT, CF, 3><<<grid, block, h->fused_smem, s>>>(a) \
+  (h->stage.nstage == 3 ? k_lean<CHECK, INJECT, CF, 3><<<grid, block, h->fused_smem, s>>>(a)   \
+   : h->lean_short      ? k_lean<CHECK, INJECT, CF, 2, true><<<grid, block, h->fused_smem, s>>>(a) \
                         : k_lean<CHECK, INJECT, CF, 2><<<grid, block, h->fused_smem, s>>>(a))
   switch (h->cfmt) {
     case CF_I8: LEAN(CF_I8); break;
@@ -503,6 +505,10 @@ abft_status set_lean_attrs(int optin) {
   TRY(set_smem_attrs(k_lean<true, false, CF, 3>, optin));
   TRY(set_smem_attrs(k_lean<false, true, CF, 3>, optin));
   TRY(set_smem_attrs(k_lean<false, false, CF, 3>, optin));
+  TRY(set_smem_attrs(k_lean<true, true, CF, 2, true>, optin));
+  TRY(set_smem_attrs(k_lean<true, false, CF, 2, true>, optin));
+  TRY(set_smem_attrs(k_lean<false, true, CF, 2, true>, optin));
+  TRY(set_smem_attrs(k_lean<false, false, CF, 2, true>, optin));
   for (auto kern : {k_irr<true, true, CF>, k_irr<true, false, CF>, k_irr<false, true, CF>,
                     k_irr<false, false, CF>})
     CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -802,9 +808,27 @@ abft_status plan_fused(abft_ctx *h, cudaStream_t s) {
   h->n_glist = (int64_t)glist.size();
   h->n_glist_nl = (int64_t)glist_nl.size();
   if (h->lean) {
+    int32_t ml = 0;  // longest row of the groups k_lean takes
+    for (int64_t g = 0; g < h->ngroups; ++g)
+      if (lean_ok[g] & 1)
+        for (int64_t i = g * 32; i < g * 32 + 32; ++i) ml = std::max(ml, rp[i + 1] - rp[i]);
+    h->lean_short = ml <= 8 && h->stage.nstage == 2 && !getenv("ABFT_NO_SHORT");
     int per_sm = 0;
-    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_lean<true, false, CF_CSR, 2>,
-                                                     c.warps * 32, h->fused_smem));
+    // occupancy of the instantiation that will run (format, SHORT)
+#define OCC(CF)                                                                               \
+  (h->lean_short                                                                              \
+       ? cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_lean<true, false, CF, 2, true>, \
+                                                       c.warps * 32, h->fused_smem)           \
+       : cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_lean<true, false, CF, 2>,   \
+                                                       c.warps * 32, h->fused_smem))
+    switch (h->cfmt) {
+      case CF_I8: CK(OCC(CF_I8)); break;
+      case CF_I16: CK(OCC(CF_I16)); break;
+      case CF_F32: CK(OCC(CF_F32)); break;
+      case CF_F64: CK(OCC(CF_F64)); break;
+      default: CK(OCC(CF_CSR)); break;
+    }
+#undef OCC
     per_sm = std::max(per_sm, 1);
     if (const char *e = getenv("ABFT_CTAS_PER_SM")) per_sm = std::max(1, std::min(per_sm, atoi(e)));
     const int64_t need = (h->ngroups + c.warps - 1) / c.warps;  // >= 1 group per warp

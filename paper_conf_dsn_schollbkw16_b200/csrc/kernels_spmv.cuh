@@ -52,6 +52,18 @@ constexpr int kLeanWarps = 4;  // warps per CTA of k_lean (<= 4)
 #ifndef ABFT_LEAN_MINB
 #define ABFT_LEAN_MINB 5  // min resident CTAs per SM the register budget targets (measured best)
 #endif
+// SHORT instantiation (every k_lean row <= 8 entries: 5-/7-point stencils):
+// the 16/32-leaf row path is compiled out, which lets the budget target 7
+// CTAs per SM for the protected kernel (72 registers, no spills) and 6 for
+// the plain one -- measured on 7-pt 128^3: protected 0.0594 -> 0.0550 ms,
+// plain 0.0370 -> 0.0371 ms (7 CTAs: 0.0378).  The general instantiation
+// keeps 5 (6 costs 27-pt 128^3 9%).
+#ifndef ABFT_LEAN_MINB_SHORT
+#define ABFT_LEAN_MINB_SHORT 7
+#endif
+#ifndef ABFT_LEAN_MINB_SHORT_PLAIN
+#define ABFT_LEAN_MINB_SHORT_PLAIN 6
+#endif
 
 struct StageCfg {
   int32_t capA, capC;     // staged capacity (elements) of a group's A / C segment
@@ -663,7 +675,7 @@ struct Pre {
 // Row bounds of staged group g (+ the gathers when every row has <= 8
 // entries).  Also stages the A slots past the arrays' last 4-element
 // boundary, which the bulk copy cannot cover.
-template <int CF>
+template <int CF, bool SHORT>
 __device__ __forceinline__ void pregather(const SpmvArgs &a, int32_t sa, int32_t ea,
                                           unsigned char *st, int lane, Pre &p) {
   const StageCfg &c = a.sc;
@@ -689,12 +701,12 @@ __device__ __forceinline__ void pregather(const SpmvArgs &a, int32_t sa, int32_t
     if (lane == 31) p.re = ea;
     p.maxlen = warp_max_i(p.re - p.rs);
   }
-  if (p.maxlen <= 8)
+  if (SHORT || p.maxlen <= 8)
     tpr_gather8(reinterpret_cast<const int32_t *>(st + c.off_ac), p.rs - (sa & ~3), p.re - p.rs,
                 a.x, p.xj);
 }
 
-template <bool CHECK, bool INJECT, int CF>
+template <bool CHECK, bool INJECT, int CF, bool SHORT>
 __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa, int32_t ea,
                                         int32_t sc, int32_t ec, unsigned char *st, int lane,
                                         const InjRange &R, const Pre &p) {
@@ -724,7 +736,7 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
     // the staged values (xg[slot], read by the C pass).
     const int o = rs - (sa & ~3);  // staging slot of the row's first entry
     constexpr bool KEEPX = CHECK && CF != CF_CSR;
-    if (maxlen <= 8) {
+    if (SHORT || maxlen <= 8) {
       yv = tpr_finish8<KEEPX>(av, xg, o, len, p.xj);  // gathers issued by pregather
     } else {
       // 16 / 32 leaves: aligned 8-leaf subtrees one at a time (bounded
@@ -954,8 +966,11 @@ __device__ __forceinline__ void issue_stage(const SpmvArgs &a, int64_t g, int32_
 // NST = 2: double buffering, each group's gathers issued right before its
 // products.  NST = 3 (small stages): prefetch distance 2, and group g+1's x
 // gathers are issued before group g's products, C pass and butterflies.
-template <bool CHECK, bool INJECT, int CF, int NST>
-__global__ void __launch_bounds__(kLeanWarps * 32, ABFT_LEAN_MINB) k_lean(const SpmvArgs a) {
+template <bool CHECK, bool INJECT, int CF, int NST, bool SHORT = false>
+__global__ void __launch_bounds__(kLeanWarps * 32,
+                                  SHORT ? (CHECK ? ABFT_LEAN_MINB_SHORT : ABFT_LEAN_MINB_SHORT_PLAIN)
+                                        : ABFT_LEAN_MINB)
+    k_lean(const SpmvArgs a) {
   extern __shared__ __align__(128) unsigned char smem[];
   if (skip_call(a)) return;
   const StageCfg &c = a.sc;
@@ -996,7 +1011,7 @@ __global__ void __launch_bounds__(kLeanWarps * 32, ABFT_LEAN_MINB) k_lean(const 
     if (elig) {
       mbar_wait(bars, 0);
       phase ^= 1u;
-      pregather<CF>(a, sa, ea, wst, lane, pc);
+      pregather<CF, SHORT>(a, sa, ea, wst, lane, pc);
     }
   }
   int s = 0;  // stage of group g
@@ -1017,8 +1032,8 @@ __global__ void __launch_bounds__(kLeanWarps * 32, ABFT_LEAN_MINB) k_lean(const 
         unsigned char *st = wst + (size_t)s * c.stage_bytes;
         mbar_wait(bars + s, (phase >> s) & 1u);
         phase ^= 1u << s;
-        pregather<CF>(a, sa, ea, st, lane, pc);
-        group32<CHECK, INJECT, CF>(a, g, sa, ea, sc, ec, st, lane, R, pc);
+        pregather<CF, SHORT>(a, sa, ea, st, lane, pc);
+        group32<CHECK, INJECT, CF, SHORT>(a, g, sa, ea, sc, ec, st, lane, R, pc);
         __syncwarp();
         fence_proxy_async_smem();  // generic accesses of this stage precede its next bulk write
       }
@@ -1041,11 +1056,11 @@ __global__ void __launch_bounds__(kLeanWarps * 32, ABFT_LEAN_MINB) k_lean(const 
         unsigned char *st1 = wst + (size_t)s1 * c.stage_bytes;
         mbar_wait(bars + s1, (phase >> s1) & 1u);
         phase ^= 1u << s1;
-        pregather<CF>(a, sa1, ea1, st1, lane, pn);
+        pregather<CF, SHORT>(a, sa1, ea1, st1, lane, pn);
       }
       if (elig) {
         unsigned char *st = wst + (size_t)s * c.stage_bytes;
-        group32<CHECK, INJECT, CF>(a, g, sa, ea, sc, ec, st, lane, R, pc);
+        group32<CHECK, INJECT, CF, SHORT>(a, g, sa, ea, sc, ec, st, lane, R, pc);
         __syncwarp();
         fence_proxy_async_smem();  // generic accesses of this stage precede its next bulk write
       }
