@@ -5,7 +5,9 @@ src = "gpurun_out/prof_round"
 dst = "profiles"
 os.makedirs(dst, exist_ok=True)
 for f in ["bench.jsonl", "bench_reference.jsonl", "pcg.jsonl", "coverage.jsonl", "gpu.csv",
-          "bench_27pt128.jsonl", "bench_27pt256.jsonl", "bench_rmat20.jsonl", "bench_5pt64.jsonl"]:
+          "bench_27pt128.jsonl", "bench_27pt256.jsonl", "bench_rmat20.jsonl", "bench_5pt64.jsonl",
+          "bench_rmat24.jsonl", "compare_7pt128.jsonl", "compare_27pt128.jsonl",
+          "compare_rmat20.jsonl", "compare_5pt64.jsonl"]:
     p = os.path.join(src, f)
     if os.path.exists(p):
         lines = [l for l in open(p) if l.strip().startswith("{") or f.endswith(".csv")]
@@ -31,7 +33,7 @@ out = subprocess.run([sys.executable, "scripts/ncu_summary.py", rep, "65536", "3
 lines = subprocess.run([sys.executable, "scripts/ncu_lines.py", rep, "65536", "30"],
                        capture_output=True, text=True).stdout
 open(os.path.join(dst, f"{R}_k_lean_ncu_summary.txt"), "w").write(
-    "ncu --set full --clock-control none -k regex:k_lean (bench workload 7pt128, k_lean<CHECK>)\n"
+    "ncu --set full --clock-control none -k regex:k_lean (bench workload 7pt128, k_lean<CHECK, SHORT>)\n"
     "per-unit counts are per 32-row group (65536 groups)\n\n" + out + "\nper source line:\n" + lines)
 raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True,
                      text=True).stdout.splitlines()
