@@ -26,10 +26,19 @@
 
 namespace abft {
 
-constexpr int kIrrWarps = 4;      // warps per CTA
-constexpr int kIrrCap = 1024;     // staging-grid slots per group (segment + (rp & 3))
-constexpr int kIrrU = 16;         // A entries in flight per lane
-constexpr int kIrrMinB = 3;       // resident CTAs per SM the budget targets
+#ifndef ABFT_IRR_CAP
+#define ABFT_IRR_CAP 1024
+#endif
+#ifndef ABFT_IRR_U
+#define ABFT_IRR_U 16
+#endif
+#ifndef ABFT_IRR_MINB
+#define ABFT_IRR_MINB 3
+#endif
+constexpr int kIrrWarps = 4;             // warps per CTA
+constexpr int kIrrCap = ABFT_IRR_CAP;    // staging-grid slots per group (segment + (rp & 3))
+constexpr int kIrrU = ABFT_IRR_U;        // A entries in flight per lane
+constexpr int kIrrMinB = ABFT_IRR_MINB;  // resident CTAs per SM the budget targets
 constexpr size_t kIrrSmemPerWarp = 2 * (size_t)kIrrCap * sizeof(double);  // products + x_j
 
 // PW of 8 aligned 32-subtrees held lane-strided (v[u] = element 32u + lane of

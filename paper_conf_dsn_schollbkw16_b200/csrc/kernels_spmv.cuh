@@ -58,9 +58,6 @@ constexpr int kLeanWarps = 4;  // warps per CTA of k_lean (<= 4)
 // the plain one -- measured on 7-pt 128^3: protected 0.0594 -> 0.0550 ms,
 // plain 0.0370 -> 0.0371 ms (7 CTAs: 0.0378).  The general instantiation
 // keeps 5 (6 costs 27-pt 128^3 9%).
-#ifndef ABFT_LEAN_PAIR
-#define ABFT_LEAN_PAIR 0  // rows of 9..32 entries: two 8-leaf subtrees per gather step
-#endif
 #ifndef ABFT_LEAN_MINB_SHORT
 #define ABFT_LEAN_MINB_SHORT 7
 #endif
@@ -745,23 +742,6 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
       // 16 / 32 leaves: aligned 8-leaf subtrees one at a time (bounded
       // register use), tree<4>((q0 + q1) + (q2 + q3)) with absent = -0.0
       double s01 = kAbsent, s23 = kAbsent;
-#if ABFT_LEAN_PAIR
-      // two 8-leaf subtrees per step: 16 gathers in flight per lane (half the
-      // dependent L2 round trips); q + (-0.0) == q keeps the bits when the
-      // second subtree is absent
-#pragma unroll 1
-      for (int t = 0; t < 4 && len > 8 * t; t += 2) {
-        double xa[8], xb[8];
-        tpr_gather8(ac, o + 8 * t, len - 8 * t, a.x, xa);
-        tpr_gather8(ac, o + 8 * t + 8, len - 8 * t - 8, a.x, xb);
-        const double qa = tpr_finish8<KEEPX>(av, xg, o + 8 * t, len - 8 * t, xa);
-        const double qb = tpr_finish8<KEEPX>(av, xg, o + 8 * t + 8, len - 8 * t - 8, xb);
-        if (t == 0)
-          s01 = dadd(qa, qb);
-        else
-          s23 = dadd(qa, qb);
-      }
-#else
 #pragma unroll 1
       for (int t = 0; t < 4 && len > 8 * t; ++t) {
         const double qt = tpr_chunk8<KEEPX>(av, ac, xg, o + 8 * t, len - 8 * t, a.x);
@@ -770,7 +750,6 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
         else
           s23 = t == 2 ? qt : dadd(s23, qt);
       }
-#endif
       yv = dadd(s01, s23);
     }
   }
