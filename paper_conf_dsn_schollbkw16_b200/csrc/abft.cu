@@ -788,7 +788,7 @@ abft_status plan_fused(abft_ctx *h, cudaStream_t s) {
     const int32_t lc = h->cfmt != CF_CSR ? crpc[g + 1] - crpc[g] : crp[g + 1] - crp[g];
     return lc <= 1024;
   };
-  if (h->lean && 2 * n_lean < h->ngroups && !getenv("ABFT_NO_IRR")) {
+  if (h->lean && (2 * n_lean < h->ngroups || getenv("ABFT_FORCE_IRR")) && !getenv("ABFT_NO_IRR")) {
     h->lean = false;
     for (auto &o : lean_ok) o &= (uint8_t)~1u;
   }
