@@ -812,7 +812,8 @@ abft_status plan_fused(abft_ctx *h, cudaStream_t s) {
     for (int64_t g = 0; g < h->ngroups; ++g)
       if (lean_ok[g] & 1)
         for (int64_t i = g * 32; i < g * 32 + 32; ++i) ml = std::max(ml, rp[i + 1] - rp[i]);
-    h->lean_short = ml <= 8 && h->stage.nstage == 2 && !getenv("ABFT_NO_SHORT");
+    h->lean_short = ml <= 8 && h->stage.capC <= 256 && h->stage.nstage == 2 &&
+                    !getenv("ABFT_NO_SHORT");
     int per_sm = 0;
     // occupancy of the instantiation that will run (format, SHORT)
 #define OCC(CF)                                                                               \

@@ -791,7 +791,7 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
   // step 1: t1_k = c_k . x.  Lane l owns elements 8l..8l+7 of
   // each aligned 256-chunk: an 8-leaf tree in registers, then the butterfly
   // over lanes -- exactly the PW tree of the chunk; chunks by a 4-leaf tree.
-  double q[4];
+  double q[4] = {kAbsent, kAbsent, kAbsent, kAbsent};
   if (ABFT_EXP == 1 || ABFT_EXP == 2 || ABFT_EXP == 5) {
     q[0] = q[1] = q[2] = q[3] = kAbsent;
   } else if (CF != CF_CSR) {
@@ -800,9 +800,11 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
     const unsigned char *cvb = st + c.off_rp + kRecHead;
     const uint16_t *cm = reinterpret_cast<const uint16_t *>(cvb + (size_t)nC * sizeof(CT));
     const double *xgm1 = xg - 1;  // slot + 1 indexing; xg[-1] = -0.0 (padding)
-    const int nt = nC <= 256 ? 1 : 4;  // uniform: one 256-chunk in the common case
+    // uniform: one 256-chunk in the common case (SHORT: always -- the plan
+    // takes SHORT only when every staged C row has <= 256 entries)
+    const int nt = (SHORT || nC <= 256) ? 1 : 4;
 #pragma unroll
-    for (int t = 0; t < 4; ++t) {
+    for (int t = 0; t < (SHORT ? 1 : 4); ++t) {
       if (t >= nt) {
         q[t] = kAbsent;
         continue;
@@ -840,7 +842,7 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
     }
   }
   if (ABFT_EXP == 3 || ABFT_EXP == 5) {
-  } else if (nC <= 256) {
+  } else if (SHORT || nC <= 256) {
     // the common case, one chunk: the three butterflies as one reduce-scatter
     // (levels 1 and 2 split the values over lane pairs, levels 3-5 are plain
     // butterflies) -- each value still sees the ascending-offset pairing of
@@ -864,7 +866,7 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
       if (t * 256 < nC) q[t] = bfly32(q[t]);
   }
   // PW over the chunk sums (one chunk: q[0] itself; an empty row: +0.0)
-  double t1 = nC > 256 ? tree<4>(q) : nC > 0 ? q[0] : 0.0;
+  double t1 = (!SHORT && nC > 256) ? tree<4>(q) : nC > 0 ? q[0] : 0.0;
   if (INJECT && lane == 0) {
     if (R.k0 < R.k1) t1 = apply_mask(t1, list_mask_in(a.inj, R.k0, R.k1, list_key(0, 1, g)));
     if (R.q0 < R.q1) t2 = apply_mask(t2, list_mask_in(a.inj, R.q0, R.q1, list_key(0, 2, g)));
