@@ -391,6 +391,14 @@ __device__ __forceinline__ void own_range(const SpmvArgs &a, int64_t g, int &lo,
   hi = l;
 }
 
+// Owner-table entry with low key bits `low` (row index, or 32 + block index
+// for a C row) among [lo, hi) of one group; -1 when absent.
+__device__ __forceinline__ int own_find(const SpmvArgs &a, int lo, int hi, int low) {
+  for (int e = lo; e < hi; ++e)
+    if ((__ldg(a.own_key + e) & 63) == low) return e;
+  return -1;
+}
+
 // ---------------------------------------------------------------------------
 // Candidate test (step 4 pre-filter) shared by both kernels.
 // ---------------------------------------------------------------------------
@@ -1331,8 +1339,43 @@ __global__ void __launch_bounds__(256) k_finish(const SpmvArgs a, int rounds) {
     if (nprev == 0) break;  // uniform: every CTA reads it after the barrier
     const int32_t *prev = a.flags + (int64_t)(round - 1) * a.nb;
     int32_t *next = a.flags + (int64_t)round * a.nb;
+    // solo rounds on a matrix with hub rows (> kHubLen entries): first the
+    // flagged blocks' hub chunk sums, spread over the CTA's warps (a hub row
+    // of 40k entries is 40 chunks, not one warp's serial chain), then the
+    // blocks below combine them (hub_sum: aligned subtrees == PW)
+    const bool hubs = solo && a.n_own > 0 && a.bs <= 32;
+    if (hubs) {
+      int item = 0;  // running chunk index over the flagged blocks (uniform)
+      const int per_g = 32 >> a.log2bs;
+      for (int q = 0; q < nprev; ++q) {
+        const int64_t k = __ldcg(prev + q);
+        const int64_t g = (k << a.log2bs) >> 5;
+        if (!(__ldg(a.lean_ok + g) & 2)) continue;
+        const int kb = (int)(k & (per_g - 1));
+        int lo, hi;
+        own_range(a, g, lo, hi);
+        for (int e = lo; e < hi; ++e) {
+          const int32_t key = __ldg(a.own_key + e);
+          const bool crow = (key & 32) != 0;
+          if ((crow ? (key & 31) : ((key & 31) >> a.log2bs)) != kb) continue;  // another block
+          const int32_t f = __ldg(a.own_first + e), cnt = __ldg(a.own_n + e);
+          for (int t = 0; t < cnt; ++t, ++item) {
+            if (item % nw != gw) continue;
+            const uint32_t L = __ldg(a.hub_len + f + t);
+            const int64_t b = __ldg(a.hub_beg + f + t);
+            const double r = (L >> 31) ? warp_dot(Cs, b, (int)(L & 0x7fffffffu), a.x, lane)
+                                       : warp_dot(As, b, (int)(L & 0x7fffffffu), a.x, lane);
+            if (lane == 0) a.hub_part[f + t] = r;
+          }
+        }
+      }
+      __syncthreads();
+    }
     for (int64_t q = gw; q < nprev; q += nw) {
       const int64_t k = __ldcg(prev + q);
+      int olo = 0, ohi = 0;  // hub rows of the block's group (solo rounds)
+      if (hubs && (__ldg(a.lean_ok + ((k << a.log2bs) >> 5)) & 2))
+        own_range(a, (k << a.log2bs) >> 5, olo, ohi);
       if (a.bs > 32) {  // big blocks: recompute the block's groups, re-verify
         const double sv = big_block<true, INJECT>(a, k, round, lane, nullptr);
         if (lane == 0 && !(fabs(sv) <= dmul(__ldg(a.K + k), beta)))
@@ -1355,7 +1398,12 @@ __global__ void __launch_bounds__(256) k_finish(const SpmvArgs a, int rounds) {
           const int32_t rb = __shfl_sync(kFull, rs, j);
           const int rl = __shfl_sync(kFull, len, j);
           if ((k << a.log2bs) + j >= n) break;
-          const double t = warp_dot(As, rb, rl, a.x, lane);
+          double t;
+          const int e = rl > kHubLen ? own_find(a, olo, ohi, (int)(((k << a.log2bs) + j) & 31)) : -1;
+          if (e >= 0)
+            t = hub_sum(a, __ldg(a.own_first + e), __ldg(a.own_n + e));
+          else
+            t = warp_dot(As, rb, rl, a.x, lane);
           if (lane == j) yv = t;
         }
       }
@@ -1367,7 +1415,10 @@ __global__ void __launch_bounds__(256) k_finish(const SpmvArgs a, int rounds) {
       if (valid) a.y[i] = yv;
       double t2 = bfly32(valid ? yv : kAbsent);
       const int32_t cb = __ldg(a.crp + k), ce = __ldg(a.crp + k + 1);
-      double t1 = warp_dot(Cs, cb, ce - cb, a.x, lane);
+      const int ec = ce - cb > kHubLen
+                         ? own_find(a, olo, ohi, 32 + (int)(k & ((32 >> a.log2bs) - 1))) : -1;
+      double t1 = ec >= 0 ? hub_sum(a, __ldg(a.own_first + ec), __ldg(a.own_n + ec))
+                          : warp_dot(Cs, cb, ce - cb, a.x, lane);
       if (lane == 0) {
         if (INJECT) {
           t1 = apply_mask(t1, fault_mask(a.inj, round, 1, k, 2 * (int64_t)(ce - cb)));
