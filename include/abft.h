@@ -198,6 +198,25 @@ abft_status abft_debug_checksums(abft_handle_t h, const double **t1, const doubl
 abft_status abft_spmv_host(abft_handle_t h, const double *x_host, double *y_host,
                            int32_t *n_flagged_host, uint32_t mode, void *stream);
 
+/* The same for a stream of nsteps products with HOST buffers: step k copies
+ * x_hosts[k] (n_cols doubles, pinned recommended) in, runs abft_spmv(mode)
+ * and copies y_hosts[k] (n doubles) and n_flagged_hosts[k] (nullable array,
+ * round-0 flag count) out.  Two device buffer slots and separate copy-in /
+ * copy-out streams overlap step k's copies with steps k-1 / k+1 (x_k's
+ * upload, y_{k-1}'s download and the products run concurrently).  No
+ * injection.  Synchronises before returning. */
+/* Page-locked host memory from the library's own CUDA runtime (the host
+ * buffers of the two calls above: the library's runtime then sees them as
+ * pinned, so its copies are asynchronous and overlap; memory pinned by
+ * another runtime instance may be staged synchronously).  abft_host_free
+ * releases it. */
+abft_status abft_host_alloc(int64_t bytes, void **p);
+abft_status abft_host_free(void *p);
+
+abft_status abft_spmv_host_pipelined(abft_handle_t h, const double *const *x_hosts,
+                                     double *const *y_hosts, int32_t nsteps,
+                                     int32_t *n_flagged_hosts, uint32_t mode, void *stream);
+
 /* PCG statistics (host struct). */
 typedef struct {
   int64_t iters;

@@ -28,6 +28,7 @@ SYMBOLS = [
     "abft_destroy", "abft_memcpy", "abft_status_string", "abft_last_cuda_error",
     "abft_burst_table", "abft_version", "abft_info", "abft_beta_partial", "abft_finish",
     "abft_dense_encode", "abft_spmv_dense", "abft_dense_result", "abft_dense_checksum",
+    "abft_spmv_host_pipelined", "abft_host_alloc", "abft_host_free",
 ]
 ENCODE_C_CSR = 1
 CFMT_NAMES = {0: "csr-f64", 1: "int8+u16", 2: "int16+u16", 3: "f32+u16", 4: "f64+u16"}
@@ -123,6 +124,12 @@ def lib():
         L.abft_info.argtypes = [P, C.POINTER(Info)]
         L.abft_beta_partial.restype = st
         L.abft_beta_partial.argtypes = [P, P, P]
+        L.abft_host_alloc.restype = st
+        L.abft_host_alloc.argtypes = [i64, C.POINTER(P)]
+        L.abft_host_free.restype = st
+        L.abft_host_free.argtypes = [P]
+        L.abft_spmv_host_pipelined.restype = st
+        L.abft_spmv_host_pipelined.argtypes = [P, P, P, i32, P, u32, P]
         L.abft_dense_encode.restype = st
         L.abft_dense_encode.argtypes = [P, P]
         L.abft_spmv_dense.restype = st
@@ -291,6 +298,18 @@ class Handle:
                                     _stream(stream)), "abft_spmv_host")
         return nf.value
 
+    def spmv_host_pipelined(self, x_hosts, y_hosts, mode=CHECK | AUTOCORRECT,
+                            stream=None) -> np.ndarray:
+        """len(x_hosts) products with host numpy buffers, copies overlapped
+        across steps (include/abft.h); returns the round-0 flag counts."""
+        k = len(x_hosts)
+        xs = (C.c_void_p * k)(*[a.ctypes.data for a in x_hosts])
+        ys = (C.c_void_p * k)(*[a.ctypes.data for a in y_hosts])
+        nf = np.zeros(k, dtype=np.int32)
+        _check(lib().abft_spmv_host_pipelined(self._h, xs, ys, k, nf.ctypes.data_as(C.c_void_p),
+                                              mode, _stream(stream)), "abft_spmv_host_pipelined")
+        return nf
+
     # -- results (device-resident; copied out on request) ----------------
     def _d2h(self, ptr, count, dtype, stream=None):
         out = np.empty(count, dtype=dtype)
@@ -386,6 +405,26 @@ class Handle:
         if status not in (OK, ENOCONV, EBREAKDOWN):
             _check(status, "abft_pcg")
         return status, st.as_dict()
+
+
+class PinnedArray:
+    """Page-locked host float64 array from the library's runtime
+    (abft_host_alloc), for the host-buffer calls; .a is the numpy view."""
+
+    def __init__(self, n: int):
+        p = C.c_void_p()
+        _check(lib().abft_host_alloc(8 * max(int(n), 1), C.byref(p)), "abft_host_alloc")
+        self._p = p
+        buf = (C.c_double * max(int(n), 1)).from_address(p.value)
+        self.a = np.ctypeslib.as_array(buf)[: int(n)]
+
+    def __del__(self):
+        try:
+            if self._p:
+                lib().abft_host_free(self._p)
+                self._p = None
+        except Exception:
+            pass
 
 
 def encode(A, block_size: int = 32, max_rounds: int = 4, stream=None,

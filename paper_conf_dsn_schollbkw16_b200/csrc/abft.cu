@@ -117,6 +117,13 @@ struct abft_ctx {
   double plan_lambda = -1.0;  // the tables on the device belong to (lambda, ops)
   int64_t plan_ops = -1;
   double *hx = nullptr, *hy = nullptr;  // device staging for abft_spmv_host
+  // abft_spmv_host_pipelined: double-buffered x / y, copy-in / copy-out
+  // streams and their events (created on first use)
+  double *px[2] = {nullptr, nullptr}, *py[2] = {nullptr, nullptr};
+  int32_t *pnf = nullptr;  // [pnf_cap] per-step round-0 flag counts
+  int32_t pnf_cap = 0;
+  cudaStream_t s_in = nullptr, s_out = nullptr;
+  cudaEvent_t ev_x[2] = {nullptr, nullptr}, ev_c[2] = {nullptr, nullptr}, ev_o[2] = {nullptr, nullptr};
   // PCG scratch
   double *pcg = nullptr;  // r, z, p, q, d : 5 n
   double *pcg_part = nullptr;
@@ -865,6 +872,17 @@ void abft_burst_table(uint64_t T[65]) { host_burst_table(T); }
 
 abft_status abft_destroy(abft_handle_t h) {
   if (!h) return ABFT_EINVAL;
+  if (h->s_in) {
+    cudaStreamSynchronize(h->s_in);
+    cudaStreamSynchronize(h->s_out);
+    cudaStreamDestroy(h->s_in);
+    cudaStreamDestroy(h->s_out);
+    for (int q = 0; q < 2; ++q) {
+      cudaEventDestroy(h->ev_x[q]);
+      cudaEventDestroy(h->ev_c[q]);
+      cudaEventDestroy(h->ev_o[q]);
+    }
+  }
   for (void *p : h->owned) cudaFree(p);
   delete h;
   return ABFT_OK;
@@ -1097,6 +1115,85 @@ abft_status abft_spmv_host(abft_handle_t h, const double *x_host, double *y_host
   if (n_flagged_host)
     CK(cudaMemcpyAsync(n_flagged_host, h->n_flags, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
   CK(cudaStreamSynchronize(s));
+  return ABFT_OK;
+}
+
+abft_status abft_host_alloc(int64_t bytes, void **p) {
+  if (!p || bytes < 0) return ABFT_EINVAL;
+  *p = nullptr;
+  cudaError_t e = cudaHostAlloc(p, (size_t)std::max<int64_t>(bytes, 16), cudaHostAllocPortable);
+  if (e == cudaErrorMemoryAllocation) {
+    cudaGetLastError();
+    return ABFT_ENOMEM;
+  }
+  if (e != cudaSuccess) return cuda_fail(e, "cudaHostAlloc");
+  return ABFT_OK;
+}
+
+abft_status abft_host_free(void *p) {
+  if (p) CK(cudaFreeHost(p));
+  return ABFT_OK;
+}
+
+__global__ void k_copy_i32(int32_t *dst, const int32_t *src) {
+  if (threadIdx.x == 0) *dst = *(volatile const int32_t *)src;
+}
+
+abft_status abft_spmv_host_pipelined(abft_handle_t h, const double *const *x_hosts,
+                                     double *const *y_hosts, int32_t nsteps,
+                                     int32_t *n_flagged_hosts, uint32_t mode, void *stream) {
+  if (!h || !x_hosts || !y_hosts || nsteps < 0) return ABFT_EINVAL;
+  if (nsteps == 0) return ABFT_OK;
+  cudaStream_t s = (cudaStream_t)stream;
+  if (!h->s_in) {
+    for (int q = 0; q < 2; ++q) {
+      TRY(dalloc(h, &h->px[q], (size_t)h->n_cols));
+      TRY(dalloc(h, &h->py[q], (size_t)h->n));
+    }
+    CK(cudaStreamCreateWithFlags(&h->s_in, cudaStreamNonBlocking));
+    CK(cudaStreamCreateWithFlags(&h->s_out, cudaStreamNonBlocking));
+    for (int q = 0; q < 2; ++q) {
+      CK(cudaEventCreateWithFlags(&h->ev_x[q], cudaEventDisableTiming));
+      CK(cudaEventCreateWithFlags(&h->ev_c[q], cudaEventDisableTiming));
+      CK(cudaEventCreateWithFlags(&h->ev_o[q], cudaEventDisableTiming));
+    }
+  }
+  // per-step flag counts stay on the device until the end (a D2H copy into
+  // a pageable host array would block the host every step)
+  if (n_flagged_hosts && nsteps > h->pnf_cap) {
+    TRY(dalloc(h, &h->pnf, (size_t)nsteps));
+    h->pnf_cap = nsteps;
+  }
+  // the copy streams start after everything already queued on `stream`
+  cudaEvent_t start = h->ev_c[0];
+  CK(cudaEventRecord(start, s));
+  CK(cudaStreamWaitEvent(h->s_in, start, 0));
+  CK(cudaStreamWaitEvent(h->s_out, start, 0));
+  for (int32_t k = 0; k < nsteps; ++k) {
+    const int sl = k & 1;
+    if (!x_hosts[k] || !y_hosts[k]) return ABFT_EINVAL;
+    // x_k -> slot (after step k-2's compute read it)
+    if (k >= 2) CK(cudaStreamWaitEvent(h->s_in, h->ev_c[sl], 0));
+    CK(cudaMemcpyAsync(h->px[sl], x_hosts[k], sizeof(double) * h->n_cols, cudaMemcpyHostToDevice,
+                       h->s_in));
+    CK(cudaEventRecord(h->ev_x[sl], h->s_in));
+    // compute (after x_k arrived and step k-2's y left the slot)
+    CK(cudaStreamWaitEvent(s, h->ev_x[sl], 0));
+    if (k >= 2) CK(cudaStreamWaitEvent(s, h->ev_o[sl], 0));
+    TRY(abft_spmv(h, h->px[sl], h->py[sl], nullptr, nullptr, mode, stream));
+    if (n_flagged_hosts) k_copy_i32<<<1, 32, 0, s>>>(h->pnf + k, h->n_flags);
+    CK(cudaEventRecord(h->ev_c[sl], s));
+    // y_k -> host
+    CK(cudaStreamWaitEvent(h->s_out, h->ev_c[sl], 0));
+    CK(cudaMemcpyAsync(y_hosts[k], h->py[sl], sizeof(double) * h->n, cudaMemcpyDeviceToHost,
+                       h->s_out));
+    CK(cudaEventRecord(h->ev_o[sl], h->s_out));
+  }
+  CK(cudaStreamSynchronize(h->s_out));
+  CK(cudaStreamSynchronize(s));
+  CK(cudaStreamSynchronize(h->s_in));
+  if (n_flagged_hosts)
+    CK(cudaMemcpy(n_flagged_hosts, h->pnf, sizeof(int32_t) * nsteps, cudaMemcpyDeviceToHost));
   return ABFT_OK;
 }
 

@@ -415,3 +415,20 @@ def test_big_block_sizes(O, torch_cuda, name, bs):
     ref = c.run(G.uniform_vector(A.n, 8), plan=plan)
     assert ref.flagged.size >= 1
     c.run(G.uniform_vector(A.n, 9), rate=dict(seed=2, lam=1e-4, targets=0b111, call=1))
+
+
+def test_host_pipelined_matches_device(O, torch_cuda):
+    # abft_spmv_host_pipelined (include/abft.h): per-step host x in, y out,
+    # copies overlapped across steps -- same bits as the device call and the
+    # oracle, per step
+    from paper_conf_dsn_schollbkw16_b200 import AUTOCORRECT, CHECK, encode
+    A = MATRICES["lap3d_ragged"]()
+    h = encode(A, 32)
+    torch = torch_cuda
+    xs = [torch.from_numpy(G.uniform_vector(A.n, 60 + k)).pin_memory() for k in range(5)]
+    ys = [torch.empty(A.n, dtype=torch.float64).pin_memory() for _ in range(5)]
+    nf = h.spmv_host_pipelined([x.numpy() for x in xs], [y.numpy() for y in ys],
+                               CHECK | AUTOCORRECT)
+    assert nf.tolist() == [0] * 5
+    for k in range(5):
+        assert_bits_equal(ys[k].numpy(), O.spmv(A, xs[k].numpy()), f"y step {k}")
