@@ -368,6 +368,7 @@ void launch_lean(const abft_ctx *h, const SpmvArgs &a, cudaStream_t s) {
 #define LEAN(CF)                                                                      \
   (h->stage.nstage == 3 ? k_lean<CHECK, INJECT, CF, 3><<<grid, block, h->fused_smem, s>>>(a)   \
    : h->lean_short      ? k_lean<CHECK, INJECT, CF, 2, true><<<grid, block, h->fused_smem, s>>>(a) \
+   : h->stage.colg      ? k_lean<CHECK, INJECT, CF, 2, false, true><<<grid, block, h->fused_smem, s>>>(a) \
                         : k_lean<CHECK, INJECT, CF, 2><<<grid, block, h->fused_smem, s>>>(a))
   switch (h->cfmt) {
     case CF_I8: LEAN(CF_I8); break;
@@ -516,6 +517,10 @@ abft_status set_lean_attrs(int optin) {
   TRY(set_smem_attrs(k_lean<true, false, CF, 2, true>, optin));
   TRY(set_smem_attrs(k_lean<false, true, CF, 2, true>, optin));
   TRY(set_smem_attrs(k_lean<false, false, CF, 2, true>, optin));
+  TRY(set_smem_attrs(k_lean<true, true, CF, 2, false, true>, optin));
+  TRY(set_smem_attrs(k_lean<true, false, CF, 2, false, true>, optin));
+  TRY(set_smem_attrs(k_lean<false, true, CF, 2, false, true>, optin));
+  TRY(set_smem_attrs(k_lean<false, false, CF, 2, false, true>, optin));
   for (auto kern : {k_irr<true, true, CF>, k_irr<true, false, CF>, k_irr<false, true, CF>,
                     k_irr<false, false, CF>})
     CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -639,7 +644,8 @@ uint32_t stage_layout(const abft_ctx *h, StageCfg &c) {
     c.off_av = o;
     o += align16((uint32_t)(c.capA + 6) * 8);
     c.off_ac = o;
-    o += align16((uint32_t)(c.capA + 6 + 8) * 4);  // + 8: unpredicated column reads past a row
+    if (!c.colg)  // COLG: columns come from global memory
+      o += align16((uint32_t)(c.capA + 6 + 8) * 4);  // + 8: unpredicated column reads past a row
     c.off_xg = c.off_av;
   }
   return align16(o);
@@ -821,12 +827,33 @@ abft_status plan_fused(abft_ctx *h, cudaStream_t s) {
         for (int64_t i = g * 32; i < g * 32 + 32; ++i) ml = std::max(ml, rp[i + 1] - rp[i]);
     h->lean_short = ml <= 8 && h->stage.capC <= 256 && h->stage.nstage == 2 &&
                     !getenv("ABFT_NO_SHORT");
+    // COLG (compact C, general instantiation; opt-in experiment, ABFT_COLG=1):
+    // drop the staged A columns when that lets more CTAs share an SM.  Measured
+    // on 27-pt 128^3 (2 -> 3 CTAs per SM): protected 0.201 -> 0.268 ms, plain
+    // 0.146 -> 0.247 ms -- the per-lane column loads cost more than the
+    // occupancy gains, so the default keeps the columns staged.
+    if (!h->lean_short && h->cfmt != CF_CSR && c.nstage == 2 && getenv("ABFT_COLG")) {
+      const size_t per_sm_b = 228 * 1024;
+      StageCfg t = c;
+      t.colg = 1;
+      const uint32_t sb = stage_layout(h, t);
+      const size_t smem_g = c.bar_bytes + (size_t)c.warps * 2 * sb;
+      const size_t k_now = per_sm_b / (h->fused_smem + 1024), k_g = per_sm_b / (smem_g + 1024);
+      if ((k_g > k_now && k_now < (size_t)ABFT_LEAN_MINB) || getenv("ABFT_FORCE_COLG")) {
+        t.stage_bytes = sb;
+        c = t;
+        h->fused_smem = smem_g;
+      }
+    }
     int per_sm = 0;
     // occupancy of the instantiation that will run (format, SHORT)
 #define OCC(CF)                                                                               \
   (h->lean_short                                                                              \
        ? cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_lean<true, false, CF, 2, true>, \
                                                        c.warps * 32, h->fused_smem)           \
+   : c.colg                                                                                   \
+       ? cudaOccupancyMaxActiveBlocksPerMultiprocessor(                                       \
+             &per_sm, k_lean<true, false, CF, 2, false, true>, c.warps * 32, h->fused_smem)   \
        : cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_lean<true, false, CF, 2>,   \
                                                        c.warps * 32, h->fused_smem))
     switch (h->cfmt) {

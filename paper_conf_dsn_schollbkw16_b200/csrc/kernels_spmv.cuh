@@ -72,6 +72,7 @@ struct StageCfg {
   uint32_t stage_bytes;   // bytes per stage
   uint32_t bar_bytes;     // mbarrier region at the start of dynamic smem
   uint32_t off_rp, off_x, off_k, off_av, off_ac, off_cv, off_cc, off_cp, off_xg;
+  int32_t colg;           // A columns read from global memory, not staged (COLG)
 };
 
 struct SpmvArgs {
@@ -683,7 +684,16 @@ struct Pre {
 // Row bounds of staged group g (+ the gathers when every row has <= 8
 // entries).  Also stages the A slots past the arrays' last 4-element
 // boundary, which the bulk copy cannot cover.
-template <int CF, bool SHORT>
+// A columns of the group on the staging grid: staged, or (COLG) straight from
+// global memory (L1-cached loads), which frees a third of each stage.
+template <bool COLG>
+__device__ __forceinline__ const int32_t *cols_base(const SpmvArgs &a, int32_t sa,
+                                                    const unsigned char *st) {
+  if (COLG) return a.ci + (sa & ~3);
+  return reinterpret_cast<const int32_t *>(st + a.sc.off_ac);
+}
+
+template <int CF, bool SHORT, bool COLG>
 __device__ __forceinline__ void pregather(const SpmvArgs &a, int32_t sa, int32_t ea,
                                           unsigned char *st, int lane, Pre &p) {
   const StageCfg &c = a.sc;
@@ -692,7 +702,8 @@ __device__ __forceinline__ void pregather(const SpmvArgs &a, int32_t sa, int32_t
     const int64_t e = nnz4 + lane;  // slots of elements nnz4 .. nnz4+3
     if (lane < 4 && e >= (sa & ~3)) {
       const bool real = e < a.nnz;
-      reinterpret_cast<int32_t *>(st + c.off_ac)[e - (sa & ~3)] = real ? __ldg(a.ci + e) : 0;
+      if (!COLG)
+        reinterpret_cast<int32_t *>(st + c.off_ac)[e - (sa & ~3)] = real ? __ldg(a.ci + e) : 0;
       reinterpret_cast<double *>(st + c.off_av)[e - (sa & ~3)] = real ? __ldg(a.va + e) : 0.0;
     }
     __syncwarp();
@@ -710,11 +721,11 @@ __device__ __forceinline__ void pregather(const SpmvArgs &a, int32_t sa, int32_t
     p.maxlen = warp_max_i(p.re - p.rs);
   }
   if (SHORT || p.maxlen <= 8)
-    tpr_gather8(reinterpret_cast<const int32_t *>(st + c.off_ac), p.rs - (sa & ~3), p.re - p.rs,
+    tpr_gather8(cols_base<COLG>(a, sa, st), p.rs - (sa & ~3), p.re - p.rs,
                 a.x, p.xj);
 }
 
-template <bool CHECK, bool INJECT, int CF, bool SHORT>
+template <bool CHECK, bool INJECT, int CF, bool SHORT, bool COLG>
 __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa, int32_t ea,
                                         int32_t sc, int32_t ec, unsigned char *st, int lane,
                                         const InjRange &R, const Pre &p) {
@@ -724,7 +735,7 @@ __device__ __forceinline__ void group32(const SpmvArgs &a, int64_t g, int32_t sa
   // A: values and columns staged on the same 4-element grid from sa & ~3, so
   // slot s holds element (sa & ~3) + s in both arrays.
   double *av = reinterpret_cast<double *>(st + c.off_av);
-  const int32_t *ac = reinterpret_cast<const int32_t *>(st + c.off_ac);
+  const int32_t *ac = cols_base<COLG>(a, sa, st);
   const double *cv = reinterpret_cast<const double *>(st + c.off_cv) + (sc & 1);  // sc + e
   const int32_t *cc = reinterpret_cast<const int32_t *>(st + c.off_cc) + (sc & 3);
   double *cp = reinterpret_cast<double *>(st + c.off_cp);  // C products, padded
@@ -931,7 +942,7 @@ struct Window {
 
 // Issue the bulk copies of group g into stage `st` (lane 0 only).  The
 // unprotected baseline (CHECK = false) does not touch C.
-template <bool CHECK, int CF>
+template <bool CHECK, int CF, bool COLG>
 __device__ __forceinline__ void issue_stage(const SpmvArgs &a, int64_t g, int32_t sa, int32_t ea,
                                             int32_t sc, int32_t ec, int32_t cc, unsigned char *st,
                                             uint64_t *bar, uint64_t pol) {
@@ -942,7 +953,7 @@ __device__ __forceinline__ void issue_stage(const SpmvArgs &a, int64_t g, int32_
     const int64_t nnz4 = a.nnz & ~3ll;
     const int64_t sa4 = sa & ~3, ea4 = min64((ea + 3) & ~3, nnz4);
     const uint32_t bav = ea4 > sa4 ? (uint32_t)(ea4 - sa4) * 8 : 0;
-    const uint32_t bac = ea4 > sa4 ? (uint32_t)(ea4 - sa4) * 4 : 0;
+    const uint32_t bac = (!COLG && ea4 > sa4) ? (uint32_t)(ea4 - sa4) * 4 : 0;
     const uint32_t brec = kRecHead + (CHECK && ABFT_EXP != 2
                                           ? (uint32_t)ec * (uint32_t)(sizeof(CT) + 2) : 0u);
     const unsigned char *rec = a.grec + (int64_t)kRecHead * g + (int64_t)cc * (sizeof(CT) + 2);
@@ -976,7 +987,7 @@ __device__ __forceinline__ void issue_stage(const SpmvArgs &a, int64_t g, int32_
 // NST = 2: double buffering, each group's gathers issued right before its
 // products.  NST = 3 (small stages): prefetch distance 2, and group g+1's x
 // gathers are issued before group g's products, C pass and butterflies.
-template <bool CHECK, bool INJECT, int CF, int NST, bool SHORT = false>
+template <bool CHECK, bool INJECT, int CF, int NST, bool SHORT = false, bool COLG = false>
 __global__ void __launch_bounds__(kLeanWarps * 32,
                                   SHORT ? (CHECK ? ABFT_LEAN_MINB_SHORT : ABFT_LEAN_MINB_SHORT_PLAIN)
                                         : ABFT_LEAN_MINB)
@@ -1008,7 +1019,7 @@ __global__ void __launch_bounds__(kLeanWarps * 32,
   int32_t sa, ea, sc, ec, cc, sa1 = 0, ea1 = 0, sc1 = 0, ec1 = 0, cc1 = 0;
   win.get(g0, sa, ea, sc, ec, cc);
   bool elig = win.ok(g0), elig1 = false;
-  if (lane == 0 && elig) issue_stage<CHECK, CF>(a, g0, sa, ea, sc, ec, cc, wst, bars, pol);
+  if (lane == 0 && elig) issue_stage<CHECK, CF, COLG>(a, g0, sa, ea, sc, ec, cc, wst, bars, pol);
   uint32_t phase = 0;  // bit s = parity of stage s's next completion
   Pre pc;
   if (NST == 3) {
@@ -1016,12 +1027,12 @@ __global__ void __launch_bounds__(kLeanWarps * 32,
       win.get(g0 + 1, sa1, ea1, sc1, ec1, cc1);
       elig1 = win.ok(g0 + 1);
       if (lane == 0 && elig1)
-        issue_stage<CHECK, CF>(a, g0 + 1, sa1, ea1, sc1, ec1, cc1, wst + c.stage_bytes, bars + 1, pol);
+        issue_stage<CHECK, CF, COLG>(a, g0 + 1, sa1, ea1, sc1, ec1, cc1, wst + c.stage_bytes, bars + 1, pol);
     }
     if (elig) {
       mbar_wait(bars, 0);
       phase ^= 1u;
-      pregather<CF, SHORT>(a, sa, ea, wst, lane, pc);
+      pregather<CF, SHORT, COLG>(a, sa, ea, wst, lane, pc);
     }
   }
   int s = 0;  // stage of group g
@@ -1035,15 +1046,15 @@ __global__ void __launch_bounds__(kLeanWarps * 32,
         win.get(g + 1, nsa, nea, nsc, nec, ncc);
         nelig = win.ok(g + 1);
         if (lane == 0 && nelig)
-          issue_stage<CHECK, CF>(a, g + 1, nsa, nea, nsc, nec, ncc, wst + (size_t)s1 * c.stage_bytes,
+          issue_stage<CHECK, CF, COLG>(a, g + 1, nsa, nea, nsc, nec, ncc, wst + (size_t)s1 * c.stage_bytes,
                                  bars + s1, pol);
       }
       if (elig) {
         unsigned char *st = wst + (size_t)s * c.stage_bytes;
         mbar_wait(bars + s, (phase >> s) & 1u);
         phase ^= 1u << s;
-        pregather<CF, SHORT>(a, sa, ea, st, lane, pc);
-        group32<CHECK, INJECT, CF, SHORT>(a, g, sa, ea, sc, ec, st, lane, R, pc);
+        pregather<CF, SHORT, COLG>(a, sa, ea, st, lane, pc);
+        group32<CHECK, INJECT, CF, SHORT, COLG>(a, g, sa, ea, sc, ec, st, lane, R, pc);
         __syncwarp();
         fence_proxy_async_smem();  // generic accesses of this stage precede its next bulk write
       }
@@ -1058,7 +1069,7 @@ __global__ void __launch_bounds__(kLeanWarps * 32,
         win.get(g + 2, nsa, nea, nsc, nec, ncc);
         nelig = win.ok(g + 2);
         if (lane == 0 && nelig)
-          issue_stage<CHECK, CF>(a, g + 2, nsa, nea, nsc, nec, ncc, wst + (size_t)s2 * c.stage_bytes,
+          issue_stage<CHECK, CF, COLG>(a, g + 2, nsa, nea, nsc, nec, ncc, wst + (size_t)s2 * c.stage_bytes,
                                  bars + s2, pol);
       }
       Pre pn;
@@ -1066,11 +1077,11 @@ __global__ void __launch_bounds__(kLeanWarps * 32,
         unsigned char *st1 = wst + (size_t)s1 * c.stage_bytes;
         mbar_wait(bars + s1, (phase >> s1) & 1u);
         phase ^= 1u << s1;
-        pregather<CF, SHORT>(a, sa1, ea1, st1, lane, pn);
+        pregather<CF, SHORT, COLG>(a, sa1, ea1, st1, lane, pn);
       }
       if (elig) {
         unsigned char *st = wst + (size_t)s * c.stage_bytes;
-        group32<CHECK, INJECT, CF, SHORT>(a, g, sa, ea, sc, ec, st, lane, R, pc);
+        group32<CHECK, INJECT, CF, SHORT, COLG>(a, g, sa, ea, sc, ec, st, lane, R, pc);
         __syncwarp();
         fence_proxy_async_smem();  // generic accesses of this stage precede its next bulk write
       }

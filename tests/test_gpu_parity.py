@@ -432,3 +432,20 @@ def test_host_pipelined_matches_device(O, torch_cuda):
     assert nf.tolist() == [0] * 5
     for k in range(5):
         assert_bits_equal(ys[k].numpy(), O.spmv(A, xs[k].numpy()), f"y step {k}")
+
+
+@pytest.mark.parametrize("name", ["st27_11", "lap3d_ragged", "mixed_lean_irr", "rand_empty"])
+def test_lean_columns_from_global(O, torch_cuda, name, monkeypatch):
+    # COLG: k_lean reading A's columns from global memory
+    # instead of staging them -- same bits, error-free and with faults
+    monkeypatch.setenv("ABFT_COLG", "1")
+    monkeypatch.setenv("ABFT_FORCE_COLG", "1")
+    A = MATRICES[name]()
+    c = Case(O, torch_cuda, A)
+    monkeypatch.delenv("ABFT_FORCE_COLG")
+    monkeypatch.delenv("ABFT_COLG")
+    c.check_encoding()
+    ref = c.run(G.uniform_vector(A.n, 31))
+    assert ref.flagged.size == 0
+    plan = G.FaultPlan([0, 0], [0, 1], [A.n // 3, 0], [1 << 62, 1 << 61])
+    c.run(G.uniform_vector(A.n, 32), plan=plan)
