@@ -519,7 +519,8 @@ def run_ours(args):
             "plain_spmv_gbs": round(plain_gbs, 2),
             "plain_ms": round(ms_plain, 5),
             "paper_literal_csr_c": csr_c,
-            "roofline": {"bound": "hbm", "kernel": "k_lean<CHECK>" + (", SHORT" if info["c_format"] != 0 and args.workload in ("7pt128", "5pt64") else ""),
+            "roofline": {"bound": "hbm", "kernel": "k_lean<CHECK" + (", SHORT" if info.get("lean_short") else "")
+                                   + (", RUNS" if info.get("lean_runs") else "") + ">",
                          "achieved": round(fused_gbs, 2), "peak": peak, "unit": "GB/s",
                          "frac": round(fused_gbs / peak, 4), "traffic": traffic,
                          "peak_source": peak_src, "launch_ms": round(ms_fused, 5),

@@ -140,6 +140,8 @@ typedef struct {
   int32_t lean;             /* staged (TMA) path available */
   int32_t max_rounds;
   int64_t irr_groups;       /* 32-row groups on the irregular-row path (k_irr) */
+  int32_t lean_short;       /* k_lean SHORT instantiation (all its rows <= 8 entries) */
+  int32_t lean_runs;        /* k_lean walks interleaved runs of groups (large matrices) */
 } abft_info_t;
 abft_status abft_info(abft_handle_t h, abft_info_t *info);
 

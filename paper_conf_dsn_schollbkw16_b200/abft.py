@@ -60,7 +60,8 @@ class Info(C.Structure):
     _fields_ = [("n", C.c_int64), ("nnz", C.c_int64), ("nb", C.c_int64), ("nnz_c", C.c_int64),
                 ("block_size", C.c_int32), ("c_format", C.c_int32), ("c_bytes", C.c_int64),
                 ("groups", C.c_int64), ("general_groups", C.c_int64), ("lean", C.c_int32),
-                ("max_rounds", C.c_int32), ("irr_groups", C.c_int64)]
+                ("max_rounds", C.c_int32), ("irr_groups", C.c_int64), ("lean_short", C.c_int32),
+                ("lean_runs", C.c_int32)]
 
     def as_dict(self):
         d = {f: getattr(self, f) for f, _ in self._fields_}

@@ -78,6 +78,7 @@ struct abft_ctx {
   StageCfg stage{};
   bool lean = false;        // k_lean usable (b_s = 32, 16-B aligned A)
   bool lean_short = false;  // every k_lean group's rows <= 8 entries (SHORT instantiation)
+  bool lean_runs = false;   // k_lean walks interleaved runs (RUNS instantiation)
   size_t fused_smem = 0;
   int fused_grid = 1;       // k_lean grid (persistent, one wave)
   uint8_t *lean_ok = nullptr;  // [ngroups] groups k_lean takes
@@ -367,6 +368,9 @@ void launch_lean(const abft_ctx *h, const SpmvArgs &a, cudaStream_t s) {
   const dim3 grid(h->fused_grid), block(h->stage.warps * 32);
 #define LEAN(CF)                                                                      \
   (h->stage.nstage == 3 ? k_lean<CHECK, INJECT, CF, 3><<<grid, block, h->fused_smem, s>>>(a)   \
+   : h->lean_runs && h->lean_short                                                            \
+       ? k_lean<CHECK, INJECT, CF, 2, true, false, true><<<grid, block, h->fused_smem, s>>>(a) \
+   : h->lean_runs ? k_lean<CHECK, INJECT, CF, 2, false, false, true><<<grid, block, h->fused_smem, s>>>(a) \
    : h->lean_short      ? k_lean<CHECK, INJECT, CF, 2, true><<<grid, block, h->fused_smem, s>>>(a) \
    : h->stage.colg      ? k_lean<CHECK, INJECT, CF, 2, false, true><<<grid, block, h->fused_smem, s>>>(a) \
                         : k_lean<CHECK, INJECT, CF, 2><<<grid, block, h->fused_smem, s>>>(a))
@@ -517,6 +521,14 @@ abft_status set_lean_attrs(int optin) {
   TRY(set_smem_attrs(k_lean<true, false, CF, 2, true>, optin));
   TRY(set_smem_attrs(k_lean<false, true, CF, 2, true>, optin));
   TRY(set_smem_attrs(k_lean<false, false, CF, 2, true>, optin));
+  TRY(set_smem_attrs(k_lean<true, true, CF, 2, true, false, true>, optin));
+  TRY(set_smem_attrs(k_lean<true, false, CF, 2, true, false, true>, optin));
+  TRY(set_smem_attrs(k_lean<false, true, CF, 2, true, false, true>, optin));
+  TRY(set_smem_attrs(k_lean<false, false, CF, 2, true, false, true>, optin));
+  TRY(set_smem_attrs(k_lean<true, true, CF, 2, false, false, true>, optin));
+  TRY(set_smem_attrs(k_lean<true, false, CF, 2, false, false, true>, optin));
+  TRY(set_smem_attrs(k_lean<false, true, CF, 2, false, false, true>, optin));
+  TRY(set_smem_attrs(k_lean<false, false, CF, 2, false, false, true>, optin));
   TRY(set_smem_attrs(k_lean<true, true, CF, 2, false, true>, optin));
   TRY(set_smem_attrs(k_lean<true, false, CF, 2, false, true>, optin));
   TRY(set_smem_attrs(k_lean<false, true, CF, 2, false, true>, optin));
@@ -868,6 +880,11 @@ abft_status plan_fused(abft_ctx *h, cudaStream_t s) {
     if (const char *e = getenv("ABFT_CTAS_PER_SM")) per_sm = std::max(1, std::min(per_sm, atoi(e)));
     const int64_t need = (h->ngroups + c.warps - 1) / c.warps;  // >= 1 group per warp
     h->fused_grid = (int)std::max<int64_t>(1, std::min<int64_t>((int64_t)h->num_sms * per_sm, need));
+    // more groups than one run per warp: interleaved runs keep the gathered x
+    // in L2 (kernels_spmv.cuh LeanRuns); the occupancy of the RUNS variants
+    // equals their siblings' (same register budget)
+    h->lean_runs = c.nstage == 2 && !c.colg && !getenv("ABFT_NO_RUNS") &&
+                   h->ngroups > (int64_t)h->fused_grid * c.warps * kLeanRun;
   }
   CK(cudaStreamSynchronize(s));  // host vectors die at return
   return ABFT_OK;
@@ -1242,6 +1259,8 @@ abft_status abft_info(abft_handle_t h, abft_info_t *info) {
   info->groups = h->ngroups;
   info->general_groups = h->lean ? h->n_glist : h->n_glist_nl;
   info->irr_groups = h->n_ilist;
+  info->lean_short = h->lean_short ? 1 : 0;
+  info->lean_runs = h->lean_runs ? 1 : 0;
   info->lean = h->lean ? 1 : 0;
   info->max_rounds = h->max_rounds;
   return ABFT_OK;

@@ -984,10 +984,44 @@ __device__ __forceinline__ void issue_stage(const SpmvArgs &a, int64_t g, int32_
   if (bcc) bulk_g2s(st + c.off_cc, a.ccol + sc4, bcc, bar, pol);
 }
 
+// Work runs of k_lean (RUNS instantiation, NST = 2, chosen when ngroups >
+// tw * kLeanRun): the groups are cut into super-chunks of tw * kLeanRun
+// groups and warp gw takes the kLeanRun-group run at gw * kLeanRun of each;
+// the last, partial super-chunk is split evenly.  Groups in flight at the same
+// time then lie within ~tw * kLeanRun groups of each other, so the x entries
+// they gather stay in L2 even when x does not fit (27-pt 256^3: 134 MB of x;
+// the contiguous split spreads the warps over all of it).
+#ifndef ABFT_LEAN_RUN
+#define ABFT_LEAN_RUN 16
+#endif
+constexpr int64_t kLeanRun = ABFT_LEAN_RUN;
+struct LeanRuns {
+  int64_t full, rem, tw, gw;
+  // run r of this warp: [b, e); false when there is none
+  __device__ __forceinline__ bool get(int64_t r, int64_t &b, int64_t &e) const {
+    if (r < full) {
+      b = (r * tw + gw) * kLeanRun;
+      e = b + kLeanRun;
+      return true;
+    }
+    if (r == full && rem > 0) {
+      b = full * tw * kLeanRun + gw * rem / tw;
+      e = full * tw * kLeanRun + (gw + 1) * rem / tw;
+      return b < e;
+    }
+    return false;
+  }
+  __device__ __forceinline__ int64_t last() const {
+    int64_t b, e;
+    return (rem > 0 && get(full, b, e)) ? full : full - 1;
+  }
+};
+
 // NST = 2: double buffering, each group's gathers issued right before its
 // products.  NST = 3 (small stages): prefetch distance 2, and group g+1's x
 // gathers are issued before group g's products, C pass and butterflies.
-template <bool CHECK, bool INJECT, int CF, int NST, bool SHORT = false, bool COLG = false>
+template <bool CHECK, bool INJECT, int CF, int NST, bool SHORT = false, bool COLG = false,
+          bool RUNS = false>
 __global__ void __launch_bounds__(kLeanWarps * 32,
                                   SHORT ? (CHECK ? ABFT_LEAN_MINB_SHORT : ABFT_LEAN_MINB_SHORT_PLAIN)
                                         : ABFT_LEAN_MINB)
@@ -1009,7 +1043,16 @@ __global__ void __launch_bounds__(kLeanWarps * 32,
   const uint64_t pol = policy_evict_first();
   const int64_t tw = (int64_t)gridDim.x * c.warps;
   const int64_t gw = (int64_t)blockIdx.x * c.warps + warp;
-  const int64_t g0 = gw * a.ngroups / tw, g1 = (gw + 1) * a.ngroups / tw;
+  int64_t g0, g1;
+  const LeanRuns runs{a.ngroups / (tw * kLeanRun), a.ngroups % (tw * kLeanRun), tw, gw};
+  if constexpr (RUNS) {
+    int64_t e0, bl;
+    if (!runs.get(0, g0, e0)) return;
+    runs.get(runs.last(), bl, g1);
+  } else {
+    g0 = gw * a.ngroups / tw;
+    g1 = (gw + 1) * a.ngroups / tw;
+  }
   if (g0 >= g1) return;
   InjRange R{0, 0, 0, 0, 0, 0};
   if (INJECT) R = inj_range(a.inj, g0, g1, lane);
@@ -1036,6 +1079,48 @@ __global__ void __launch_bounds__(kLeanWarps * 32,
     }
   }
   int s = 0;  // stage of group g
+  if constexpr (RUNS && NST == 2) {
+    int64_t r = 0, g = g0, re = 0;
+    {
+      int64_t b0;
+      runs.get(0, b0, re);
+    }
+    while (true) {
+      const int s1 = s + 1 == NST ? 0 : s + 1;
+      // the next group: g + 1 in this run, else the first of the next run
+      int64_t gn = g + 1, rn = r, ren = re;
+      if (gn >= re) {
+        ++rn;
+        if (!runs.get(rn, gn, ren)) gn = -1;
+      }
+      int32_t nsa = 0, nea = 0, nsc = 0, nec = 0, ncc = 0;
+      bool nelig = false;
+      if (gn >= 0) {  // prefetch it into the other stage
+        if (gn < win.wb || gn + 1 > win.wb + 31) win.load(a, gn, lane);
+        win.get(gn, nsa, nea, nsc, nec, ncc);
+        nelig = win.ok(gn);
+        if (lane == 0 && nelig)
+          issue_stage<CHECK, CF, COLG>(a, gn, nsa, nea, nsc, nec, ncc,
+                                       wst + (size_t)s1 * c.stage_bytes, bars + s1, pol);
+      }
+      if (elig) {
+        unsigned char *st = wst + (size_t)s * c.stage_bytes;
+        mbar_wait(bars + s, (phase >> s) & 1u);
+        phase ^= 1u << s;
+        pregather<CF, SHORT, COLG>(a, sa, ea, st, lane, pc);
+        group32<CHECK, INJECT, CF, SHORT, COLG>(a, g, sa, ea, sc, ec, st, lane, R, pc);
+        __syncwarp();
+        fence_proxy_async_smem();  // generic accesses of this stage precede its next bulk write
+      }
+      if (gn < 0) break;
+      sa = nsa; ea = nea; sc = nsc; ec = nec; cc = ncc;
+      elig = nelig;
+      g = gn;
+      r = rn;
+      re = ren;
+      s = s1;
+    }
+  } else {
   for (int64_t g = g0; g < g1; ++g) {
     const int s1 = s + 1 == NST ? 0 : s + 1;
     if (NST == 2) {
@@ -1092,6 +1177,7 @@ __global__ void __launch_bounds__(kLeanWarps * 32,
       elig1 = nelig;
     }
     s = s1;
+  }
   }
 }
 

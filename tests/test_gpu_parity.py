@@ -449,3 +449,16 @@ def test_lean_columns_from_global(O, torch_cuda, name, monkeypatch):
     assert ref.flagged.size == 0
     plan = G.FaultPlan([0, 0], [0, 1], [A.n // 3, 0], [1 << 62, 1 << 61])
     c.run(G.uniform_vector(A.n, 32), plan=plan)
+
+
+def test_lean_runs_large(O, torch_cuda):
+    # LeanRuns (kernels_spmv.cuh): more groups than one 16-group run per warp
+    # -> interleaved runs; bit-exact y / t1 / t2 / flags / corrections on a
+    # 7-pt 160^3 Laplacian (4.1M rows) with faults
+    A = G.laplacian_3d_7pt(160)
+    c = Case(O, torch_cuda, A)
+    info = c.h.info()
+    assert info["lean_runs"] == 1 and info["lean_short"] == 1, info
+    plan = G.FaultPlan([0, 0, 0], [0, 1, 2], [A.n - 5, 4000, 12345], [1 << 62, 1 << 61, 1 << 60])
+    ref = c.run(G.uniform_vector(A.n, 33), plan=plan)
+    assert ref.flagged.size == 3
