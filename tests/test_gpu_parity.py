@@ -462,3 +462,30 @@ def test_lean_runs_large(O, torch_cuda):
     plan = G.FaultPlan([0, 0, 0], [0, 1, 2], [A.n - 5, 4000, 12345], [1 << 62, 1 << 61, 1 << 60])
     ref = c.run(G.uniform_vector(A.n, 33), plan=plan)
     assert ref.flagged.size == 3
+
+
+def test_config0_single_fault_sweep(O, torch_cuda):
+    # BASELINE configs[0] / SURVEY §8(d) config 1: one seeded burst per run on
+    # a uniformly chosen y element, 1000 runs: round-0 flags,
+    # pre-correction y and corrected y bit-exact against the oracle, run by run
+    from paper_conf_dsn_schollbkw16_b200 import AUTOCORRECT, CHECK, Inject, encode
+    torch = torch_cuda
+    A = G.laplacian_2d_5pt(64)
+    enc = O.encode(A, 32)
+    h = encode(A, 32)
+    xh = G.uniform_vector(A.n, 42)
+    x = torch.from_numpy(xh).cuda()
+    y0 = O.spmv(A, xh)
+    flagged_runs = 0
+    for seed in range(1000):
+        plan = G.single_fault_plan(A.n, seed)
+        ref = O.abft_spmv(A, enc, xh, O.Inject.from_plan(plan), 4)
+        y = h.spmv(x, inject=Inject.from_plan(plan), mode=CHECK | AUTOCORRECT)
+        fl = h.flags(0)
+        assert np.array_equal(fl, ref.flags[0]), (seed, fl, ref.flags[0])
+        yc = y.cpu().numpy()
+        assert_bits_equal(yc, ref.y, f"corrected y, seed {seed}")
+        if fl.size:
+            flagged_runs += 1
+            assert_bits_equal(yc, y0, f"corrected y == fault-free y, seed {seed}")
+    assert flagged_runs > 500
