@@ -13,7 +13,7 @@ timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --c
   --log-file $O/launches.csv python bench.py --steps 5 --warmup 3 --no-cpu-baseline > $O/ncu_launch.log 2>&1
 # full capture of the fused kernel (protected)
 timeout 900 ncu --set full --clock-control none --import-source on --kernel-name-base demangled \
-  -k 'regex:k_lean<.bool.1, .bool.0, .int.1, .int.2, .bool.1>' -s 4 -c 1 \
+  -k 'regex:k_lean<.bool.1, .bool.0, .int.1, .int.2, .bool.1, .bool.0, .bool.0>' -s 4 -c 1 \
   -o $O/k_lean -f python bench.py --steps 3 --warmup 3 --no-cpu-baseline > $O/ncu_full.log 2>&1
 timeout 900 python bench.py --pcg > $O/pcg.jsonl 2>&1
 timeout 900 python scripts/coverage.py > $O/coverage.jsonl 2>&1
