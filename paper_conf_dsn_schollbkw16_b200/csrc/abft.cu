@@ -368,9 +368,10 @@ void launch_lean(const abft_ctx *h, const SpmvArgs &a, cudaStream_t s) {
   const dim3 grid(h->fused_grid), block(h->stage.warps * 32);
 #define LEAN(CF)                                                                      \
   (h->stage.nstage == 3 ? k_lean<CHECK, INJECT, CF, 3><<<grid, block, h->fused_smem, s>>>(a)   \
-   : h->lean_runs && h->lean_short                                                            \
+   : h->lean_runs && !INJECT && h->lean_short                                                 \
        ? k_lean<CHECK, INJECT, CF, 2, true, false, true><<<grid, block, h->fused_smem, s>>>(a) \
-   : h->lean_runs ? k_lean<CHECK, INJECT, CF, 2, false, false, true><<<grid, block, h->fused_smem, s>>>(a) \
+   : h->lean_runs && !INJECT                                                                   \
+       ? k_lean<CHECK, INJECT, CF, 2, false, false, true><<<grid, block, h->fused_smem, s>>>(a) \
    : h->lean_short      ? k_lean<CHECK, INJECT, CF, 2, true><<<grid, block, h->fused_smem, s>>>(a) \
    : h->stage.colg      ? k_lean<CHECK, INJECT, CF, 2, false, true><<<grid, block, h->fused_smem, s>>>(a) \
                         : k_lean<CHECK, INJECT, CF, 2><<<grid, block, h->fused_smem, s>>>(a))
@@ -883,8 +884,12 @@ abft_status plan_fused(abft_ctx *h, cudaStream_t s) {
     // more groups than one run per warp: interleaved runs keep the gathered x
     // in L2 (kernels_spmv.cuh LeanRuns); the occupancy of the RUNS variants
     // equals their siblings' (same register budget)
+    // only when x is large against L2 (half of the 126 MB): with x resident
+    // the runs only cost (27-pt 128^3: 0.202 -> 0.237 ms, 7-pt 192^3 plain
+    // PCG +15%), with x = 134 MB they gain (27-pt 256^3: 1.950 -> 1.816 ms)
     h->lean_runs = c.nstage == 2 && !c.colg && !getenv("ABFT_NO_RUNS") &&
-                   h->ngroups > (int64_t)h->fused_grid * c.warps * kLeanRun;
+                   h->ngroups > (int64_t)h->fused_grid * c.warps * kLeanRun &&
+                   (h->n_cols * 8 > ((int64_t)64 << 20) || getenv("ABFT_FORCE_RUNS"));
   }
   CK(cudaStreamSynchronize(s));  // host vectors die at return
   return ABFT_OK;

@@ -451,14 +451,19 @@ def test_lean_columns_from_global(O, torch_cuda, name, monkeypatch):
     c.run(G.uniform_vector(A.n, 32), plan=plan)
 
 
-def test_lean_runs_large(O, torch_cuda):
+def test_lean_runs_large(O, torch_cuda, monkeypatch):
     # LeanRuns (kernels_spmv.cuh): more groups than one 16-group run per warp
-    # -> interleaved runs; bit-exact y / t1 / t2 / flags / corrections on a
-    # 7-pt 160^3 Laplacian (4.1M rows) with faults
+    # -> interleaved runs (forced: x of 160^3 fits L2); bit-exact y / t1 /
+    # t2 / flags error-free, and with faults (the INJECT kernels walk
+    # contiguous ranges) corrections
+    monkeypatch.setenv("ABFT_FORCE_RUNS", "1")
     A = G.laplacian_3d_7pt(160)
     c = Case(O, torch_cuda, A)
+    monkeypatch.delenv("ABFT_FORCE_RUNS")
     info = c.h.info()
     assert info["lean_runs"] == 1 and info["lean_short"] == 1, info
+    ref = c.run(G.uniform_vector(A.n, 34))
+    assert ref.flagged.size == 0
     plan = G.FaultPlan([0, 0, 0], [0, 1, 2], [A.n - 5, 4000, 12345], [1 << 62, 1 << 61, 1 << 60])
     ref = c.run(G.uniform_vector(A.n, 33), plan=plan)
     assert ref.flagged.size == 3
