@@ -494,3 +494,21 @@ def test_config0_single_fault_sweep(O, torch_cuda):
             flagged_runs += 1
             assert_bits_equal(yc, y0, f"corrected y == fault-free y, seed {seed}")
     assert flagged_runs > 500
+
+
+@pytest.mark.parametrize("name", ["7pt128", "27pt128", "rmat20"])
+def test_bench_workloads_full_size(O, torch_cuda, name):
+    # the bench's own workloads at full size, in the launch configuration
+    # bench.py times (7-pt 128^3 = configs[1]: k_lean SHORT; 27-pt 128^3: the
+    # general k_lean; R-MAT scale 20: k_irr + k_hub + k_general), every output
+    # against the oracle with faults in y, t1 and t2
+    A = {"7pt128": lambda: G.laplacian_3d_7pt(128), "27pt128": lambda: G.stencil_3d_27pt(128),
+         "rmat20": lambda: G.rmat(20, 16, 1)}[name]()
+    c = Case(O, torch_cuda, A)
+    ref = c.run(G.uniform_vector(A.n, 42))
+    assert ref.flagged.size == 0
+    nb = c.enc.nb
+    plan = G.FaultPlan([0, 0, 0, 0], [0, 0, 1, 2], [7, A.n - 1, nb // 2, nb - 3],
+                       [1 << 62, 1 << 55, 1 << 61, 1 << 60])
+    ref = c.run(G.uniform_vector(A.n, 43), plan=plan)
+    assert ref.flagged.size >= 3
