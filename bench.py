@@ -540,8 +540,11 @@ def run_ours(args):
             "plain_ms": round(ms_plain, 5),
             "paper_literal_csr_c": csr_c,
             "cusparse_plain": cusparse,
-            "roofline": {"bound": "hbm", "kernel": "k_lean<CHECK" + (", SHORT" if info.get("lean_short") else "")
-                                   + (", RUNS" if info.get("lean_runs") else "") + ">",
+            "roofline": {"bound": "hbm", "kernel": (("k_lean<CHECK" + (", SHORT" if info.get("lean_short") else "")
+                                     + (", RUNS" if info.get("lean_runs") else "") + ">")
+                                    if info.get("lean") else
+                                    ("fused pass: k_hub + k_irr<CHECK> + k_general<CHECK>"
+                                     if info.get("irr_groups") else "k_general<CHECK>")),
                          "achieved": round(fused_gbs, 2), "peak": peak, "unit": "GB/s",
                          "frac": round(fused_gbs / peak, 4), "traffic": traffic,
                          "peak_source": peak_src, "launch_ms": round(ms_fused, 5),
