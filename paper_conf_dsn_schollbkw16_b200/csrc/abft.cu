@@ -618,7 +618,7 @@ abft_status build_compact_c(abft_ctx *h, cudaStream_t s) {
   int32_t hbad = 0;
   CK(cudaMemcpyAsync(&hbad, bad, sizeof hbad, cudaMemcpyDeviceToHost, s));
   CK(cudaStreamSynchronize(s));
-  if (hbad) return ABFT_OK;  // some block's A segment exceeds uint16 slots: keep CSR
+  if (hbad) return ABFT_OK;  // a mappable block lacks a slot (cannot happen): keep CSR
   CK(cudaGetLastError());
   h->grec = rec;
   h->cfmt = cf;

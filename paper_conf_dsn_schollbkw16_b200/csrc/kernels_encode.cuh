@@ -189,8 +189,17 @@ __global__ void k_cformat_fill(int64_t nb, int64_t n, const int32_t *__restrict_
     uint16_t *cmap = reinterpret_cast<uint16_t *>(rk + kRecHead + (int64_t)plen * sizeof(T));
     const int64_t r0 = k * 32, r1 = min64(r0 + 32, n);
     const int32_t s0 = rp[r0] & ~3;
+    // blocks whose A segment exceeds the uint16 slot range (hub blocks) are
+    // never taken by the compact-C kernels (k_lean / k_irr stage at most 1024
+    // entries; k_general streams CSR C): their record is left unmapped
+    const bool mapped = (int64_t)rp[r1] - s0 <= 65534;
     for (int32_t q = b + lane; q < e; q += 32) {
       const int32_t j = ccol[q];
+      cv[q - b] = (T)cval[q];
+      if (!mapped) {
+        cmap[q - b] = 0;
+        continue;
+      }
       int64_t slot = -1;
       for (int64_t r = r0; r < r1 && slot < 0; ++r) {  // first row of the block holding j
         int32_t lo = rp[r], hi = rp[r + 1];
@@ -201,7 +210,6 @@ __global__ void k_cformat_fill(int64_t nb, int64_t n, const int32_t *__restrict_
         if (lo < rp[r + 1] && ci[lo] == j) slot = lo - s0;
       }
       if (slot < 0 || slot > 65534) atomicOr(bad, 1);
-      cv[q - b] = (T)cval[q];
       cmap[q - b] = (uint16_t)(slot < 0 ? 0 : slot + 1);  // 0 = row padding (value 0)
     }
   }

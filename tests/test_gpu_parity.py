@@ -512,3 +512,26 @@ def test_bench_workloads_full_size(O, torch_cuda, name):
                        [1 << 62, 1 << 55, 1 << 61, 1 << 60])
     ref = c.run(G.uniform_vector(A.n, 43), plan=plan)
     assert ref.flagged.size >= 3
+
+
+def test_compact_c_with_huge_hub_row(O, torch_cuda):
+    # a block whose A segment exceeds the uint16 slot range keeps an unmapped
+    # compact record (k_general streams CSR C for it); every other block is
+    # compact -- parity with faults, including in the huge block
+    from paper_conf_dsn_schollbkw16_b200 import encode
+    rng = np.random.Generator(np.random.PCG64(23))
+    n = 80000
+    lens = rng.integers(1, 9, n)
+    lens[40001] = 70000
+    cols = [np.sort(rng.choice(n, size=int(L), replace=False)) for L in lens]
+    rp = np.zeros(n + 1, np.int64)
+    np.cumsum(lens, out=rp[1:])
+    col = np.concatenate(cols).astype(np.int32)
+    A = G.CSR(rp.astype(np.int32), col, rng.uniform(-1, 1, col.size), "huge_hub")
+    info = encode(A).info()
+    assert info["c_format_name"] != "csr-f64", info
+    c = Case(O, torch_cuda, A)
+    assert c.run(G.uniform_vector(n, 3)).flagged.size == 0
+    plan = G.FaultPlan([0, 0, 0], [0, 0, 1], [40001, 17, 40001 // 32], [1 << 62, 1 << 61, 1 << 60])
+    ref = c.run(G.uniform_vector(n, 4), plan=plan)
+    assert set([40001 // 32, 0]) <= set(ref.flagged.tolist())
