@@ -374,3 +374,65 @@ class CrResult:
     spmv_calls: int
     rollbacks: int
     executed: int     # executed iterations (re-executions count)
+
+
+def dot_ranks(a, b, ranges) -> float:
+    """Global dot product of the distributed PCG (R28): PW over the
+    ranks (in rank order, padded with absent slots) of each rank's PW over
+    its own rows.  One range [(0, n)] is the single-GPU PW dot (R2)."""
+    prod = np.asarray(a, dtype=np.float64) * np.asarray(b, dtype=np.float64)
+    return pw(np.array([pw(prod[r0:r1]) for r0, r1 in ranges], dtype=np.float64))
+
+
+def pcg_ranks(A, b, x0, ranges, diag=None, tol=1e-6, max_iter=0) -> PcgResult:
+    """Fault-free Jacobi-PCG (Saad Alg. 9.1, the paper's [19]) with
+    every global reduction computed as `dot_ranks` over the row partition
+    `ranges` -- the oracle of the distributed PCG.  Steps and
+    rounding follow or_pcg line by line; without faults the protected SpMV's
+    y is the plain SpMV (corrections recompute identical bits), so q = A p is
+    `spmv`.  Status 0 / -5 (ENOCONV) / -7 (EBREAKDOWN) as or_pcg."""
+    n = A.n
+    b = np.ascontiguousarray(b, dtype=np.float64)
+    x = np.array(x0, dtype=np.float64, copy=True)
+    mi = max_iter if max_iter > 0 else 10 * n
+    if diag is None:
+        d = np.zeros(n)  # diag(A), a missing diagonal -> 0 (R21)
+        rows = np.repeat(np.arange(n), np.diff(np.asarray(A.row_ptr, dtype=np.int64)))
+        on = np.asarray(A.col) == rows
+        d[rows[on]] = np.asarray(A.val)[on]
+    else:
+        d = np.asarray(diag, dtype=np.float64)
+    calls = 1
+    q = spmv(A, x)
+    r = b - q
+    z = r / d
+    p = z.copy()
+    rho = dot_ranks(r, z, ranges)
+    thr = tol * np.sqrt(dot_ranks(b, b, ranges))
+    res = np.sqrt(dot_ranks(r, r, ranges))
+    hist = [res]
+    it, status = 0, 0
+    while not (res <= thr) and it < mi:
+        if res != res:
+            status = -7
+            break
+        q = spmv(A, p)
+        calls += 1
+        pq = dot_ranks(p, q, ranges)
+        if not (pq > 0.0):
+            status = -7
+            break
+        alpha = rho / pq
+        x = x + alpha * p
+        r = r - alpha * q
+        z = r / d
+        rho_new = dot_ranks(r, z, ranges)
+        res = np.sqrt(dot_ranks(r, r, ranges))
+        it += 1
+        hist.append(res)
+        beta = rho_new / rho
+        rho = rho_new
+        p = z + beta * p
+    if status == 0 and not (res <= thr):
+        status = -5
+    return PcgResult(status, x, np.array(hist), it, calls, 0, 0, 0)

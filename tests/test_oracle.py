@@ -691,3 +691,64 @@ class TestPcgCheckpoint:
         r = O.pcg_cr(A, den, b, x0, tol=1e-6, ckpt_every=1,
                      inj=O.Inject.rate(seed=9, lam=1e-4, targets=1))
         assert r.rollbacks > 0 and r.executed == r.iters + r.rollbacks
+
+
+# --------------------------------------------------------------------------
+# Distributed PCG oracle (R28): dots partitioned by
+# rank.  Pinned to the C oracle's PCG (independent code) and to SciPy's CG.
+# --------------------------------------------------------------------------
+class TestPcgRanks:
+    def _problem(self, O, A):
+        b = O.spmv(A, G.uniform_vector(A.n, 43))
+        return b, G.uniform_vector(A.n, 44)
+
+    def test_one_rank_is_single_gpu_pcg(self, O):
+        A = G.laplacian_3d_7pt(10)
+        b, x0 = self._problem(O, A)
+        ref = O.pcg(A, O.encode(A, 32), b, x0, tol=1e-6, check=False)
+        r = O.pcg_ranks(A, b, x0, [(0, A.n)], tol=1e-6)
+        assert r.status == ref.status == 0 and r.iters == ref.iters
+        assert np.array_equal(r.res_hist.view(np.uint64), ref.res_hist.view(np.uint64))
+        assert np.array_equal(r.x.view(np.uint64), ref.x.view(np.uint64))
+
+    @pytest.mark.parametrize("world", [2, 4])
+    def test_power_of_two_ranks_are_bit_identical(self, O, world):
+        # PW is padding independent (R2): equal power-of-two row ranges are
+        # aligned subtrees, so rank partials + a tree over ranks = global PW.
+        A = G.laplacian_3d_7pt(16)  # 4096 rows
+        b, x0 = self._problem(O, A)
+        ref = O.pcg(A, O.encode(A, 32), b, x0, tol=1e-6, check=False)
+        ranges = [(r * A.n // world, (r + 1) * A.n // world) for r in range(world)]
+        r = O.pcg_ranks(A, b, x0, ranges, tol=1e-6)
+        assert r.iters == ref.iters
+        assert np.array_equal(r.res_hist.view(np.uint64), ref.res_hist.view(np.uint64))
+        assert np.array_equal(r.x.view(np.uint64), ref.x.view(np.uint64))
+
+    def test_uneven_ranks_match_scipy(self, O):
+        # 3 ranks of 12^3 / 3-plane-aligned rows: the summation order differs
+        # from one GPU, the iterates still follow CG (SciPy) to rounding.
+        import scipy.sparse as sp
+        import scipy.sparse.linalg as spla
+        A = G.laplacian_3d_7pt(12)
+        b, x0 = self._problem(O, A)
+        ranges = [(0, 576), (576, 1152), (1152, A.n)]
+        r = O.pcg_ranks(A, b, x0, ranges, tol=1e-6)
+        assert r.status == 0
+        S = sp.csr_matrix((A.val, A.col, A.row_ptr), shape=(A.n, A.n))
+        d = S.diagonal()
+        M = spla.LinearOperator(S.shape, matvec=lambda v: v / d)
+        hist = []
+        xsc, info = spla.cg(S, b, x0=x0.copy(), rtol=1e-6, atol=0.0, M=M,
+                            callback=lambda xk: hist.append(np.linalg.norm(b - S @ xk)))
+        assert info == 0 and r.iters == len(hist)
+        assert np.max(np.abs(np.array(hist) - r.res_hist[1:])) < 1e-10 * np.linalg.norm(b)
+        assert np.linalg.norm(r.x - xsc) <= 1e-9 * np.linalg.norm(xsc)
+
+    def test_dot_ranks_special_cases(self, O):
+        v = G.uniform_vector(1000, 5)
+        w = G.uniform_vector(1000, 6)
+        assert O.dot_ranks(v, w, [(0, 1000)]) == O.pw(v * w)
+        # exact small-integer sums: any order gives the exact result
+        a = np.arange(1, 101, dtype=np.float64)
+        assert O.dot_ranks(a, np.ones(100), [(0, 7), (7, 50), (50, 100)]) == 5050.0
+        assert O.dot_ranks(a, a, [(0, 0), (0, 100)]) == float(np.sum(a * a))
