@@ -251,6 +251,48 @@ abft_status abft_pcg(abft_handle_t h, const double *b, double *x, const double *
                      double tol, int64_t max_iter, const abft_inject_t *inj, int32_t check,
                      double *res_hist, abft_pcg_stats_t *stats, void *stream);
 
+/* --- Distributed Jacobi-PCG (Saad Alg. 9.1) ---
+ * The rows are sharded across ranks (one process per GPU); the handle is the
+ * rank's shard (abft_encode of the local rows, n_cols / x_offset set).  The
+ * iteration is abft_pcg's, split at its global reductions so the caller can
+ * all-gather the per-rank partials between the kernels (NCCL; 24 bytes per
+ * rank per phase) and then finish them on the device in rank order:
+ *   begin; SpMV q = A x0 (the caller's distributed protected SpMV over the
+ *   halo-extended operand); local(INIT) -> gather -> combine(INIT);
+ *   per iteration j = 1, 2, ...: SpMV q = A p; local(DOT) -> gather ->
+ *   combine(DOT); local(UPDATE, j) -> gather -> combine(UPDATE, j);
+ *   local(P, j); poll abft_pcg_dist_status every few iterations.
+ * A global sum is PW over the ranks (padded with absent slots) of each rank's
+ * PW over its own rows (R2, R28): for equal power-of-two row ranges
+ * aligned to 2048 rows, the single-GPU sums bit for bit.
+ * abft_pcg_dist_begin: b, x (in x0, out x), q (the SpMV result, [n]) and diag
+ *   (nullable: the diagonal of A at local column row + x_offset) are the
+ *   rank's own rows, 16-byte aligned; pext is the own slice of the SpMV's
+ *   halo-extended operand (any alignment; p is written there too); max_iter
+ *   > 0 (the caller passes 10 N of the global matrix); check 0 | 1 as
+ *   abft_pcg; res_hist nullable device [max_iter + 1].  Stream-ordered.
+ * abft_pcg_dist_local: phase 0 INIT (r = b - q, z = r/d, p = z; partials
+ *   r.z, r.r, b.b), 1 DOT (p.q), 2 UPDATE (x, r, z; partials r.z, r.r),
+ *   3 P (p = z + beta p; no partial).  send: device double[3] (unused for P).
+ *   Kernels of a finished solve are no-ops.
+ * abft_pcg_dist_combine: recv = device double[3 * world] (rank r at 3r);
+ *   1 <= world <= 64; phases 0-2; updates the device scalars.
+ * abft_pcg_dist_status: host copies of the state (0 running, 1 converged, 2
+ *   breakdown, 3 max_iter) and rank-local stats; synchronises the stream. */
+#define ABFT_PCG_PHASE_INIT 0
+#define ABFT_PCG_PHASE_DOT 1
+#define ABFT_PCG_PHASE_UPDATE 2
+#define ABFT_PCG_PHASE_P 3
+abft_status abft_pcg_dist_begin(abft_handle_t h, const double *b, double *x, double *pext,
+                                double *q, const double *diag, double tol, int64_t max_iter,
+                                int32_t check, double *res_hist, void *stream);
+abft_status abft_pcg_dist_local(abft_handle_t h, int32_t phase, int64_t iter, double *send,
+                                void *stream);
+abft_status abft_pcg_dist_combine(abft_handle_t h, int32_t phase, int64_t iter,
+                                  const double *recv, int32_t world, void *stream);
+abft_status abft_pcg_dist_status(abft_handle_t h, int32_t *state, abft_pcg_stats_t *stats,
+                                 void *stream);
+
 /* --- Related-work baseline: DENSE CHECK [30, 31] + COMPLETE RECOMPUTATION ---
  * (eq. (1), P:148-152 [35]'s bound, P:240, P:250-252,
  * P:258, R23-R25.)  One checksum

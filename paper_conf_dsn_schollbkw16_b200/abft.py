@@ -29,7 +29,10 @@ SYMBOLS = [
     "abft_burst_table", "abft_version", "abft_info", "abft_beta_partial", "abft_finish",
     "abft_dense_encode", "abft_spmv_dense", "abft_dense_result", "abft_dense_checksum",
     "abft_spmv_host_pipelined", "abft_host_alloc", "abft_host_free",
+    "abft_pcg_dist_begin", "abft_pcg_dist_local", "abft_pcg_dist_combine",
+    "abft_pcg_dist_status",
 ]
+PCG_PHASE_INIT, PCG_PHASE_DOT, PCG_PHASE_UPDATE, PCG_PHASE_P = 0, 1, 2, 3
 ENCODE_C_CSR = 1
 CFMT_NAMES = {0: "csr-f64", 1: "int8+u16", 2: "int16+u16", 3: "f32+u16", 4: "f64+u16"}
 
@@ -112,6 +115,14 @@ def lib():
         L.abft_spmv_host.argtypes = [P, P, P, P, u32, P]
         L.abft_pcg.restype = st
         L.abft_pcg.argtypes = [P, P, P, P, d, i64, P, i32, P, C.POINTER(PcgStats), P]
+        L.abft_pcg_dist_begin.restype = st
+        L.abft_pcg_dist_begin.argtypes = [P, P, P, P, P, P, d, i64, i32, P, P]
+        L.abft_pcg_dist_local.restype = st
+        L.abft_pcg_dist_local.argtypes = [P, i32, i64, P, P]
+        L.abft_pcg_dist_combine.restype = st
+        L.abft_pcg_dist_combine.argtypes = [P, i32, i64, P, i32, P]
+        L.abft_pcg_dist_status.restype = st
+        L.abft_pcg_dist_status.argtypes = [P, C.POINTER(i32), C.POINTER(PcgStats), P]
         L.abft_destroy.restype = st
         L.abft_destroy.argtypes = [P]
         L.abft_memcpy.restype = st
@@ -406,6 +417,27 @@ class Handle:
         if status not in (OK, ENOCONV, EBREAKDOWN):
             _check(status, "abft_pcg")
         return status, st.as_dict()
+
+    # -- distributed PCG steps (abft_pcg_dist_*; parallel.DistPcg drives them)
+    def pcg_dist_begin(self, b, x, pext, q, diag=None, tol=1e-6, max_iter=1, check=True,
+                       res_hist=None, stream=None):
+        _check(lib().abft_pcg_dist_begin(self._h, _ptr(b), _ptr(x), _ptr(pext), _ptr(q),
+                                         _ptr(diag), tol, max_iter, 1 if check else 0,
+                                         _ptr(res_hist), _stream(stream)), "abft_pcg_dist_begin")
+
+    def pcg_dist_local(self, phase, it, send=None, stream=None):
+        _check(lib().abft_pcg_dist_local(self._h, phase, it, _ptr(send), _stream(stream)),
+               "abft_pcg_dist_local")
+
+    def pcg_dist_combine(self, phase, it, recv, world, stream=None):
+        _check(lib().abft_pcg_dist_combine(self._h, phase, it, _ptr(recv), world,
+                                           _stream(stream)), "abft_pcg_dist_combine")
+
+    def pcg_dist_status(self, stream=None):
+        st, state = PcgStats(), C.c_int32(0)
+        _check(lib().abft_pcg_dist_status(self._h, C.byref(state), C.byref(st),
+                                          _stream(stream)), "abft_pcg_dist_status")
+        return state.value, st.as_dict()
 
 
 class PinnedArray:

@@ -132,6 +132,8 @@ struct abft_ctx {
   int32_t *pcg_state = nullptr;
   int64_t pcg_n = 0;
   int64_t ncta256 = 0;  // ceil(n / kPcgRows): PCG vector-kernel grid
+  abft::PcgArgs pcg_dist{};  // distributed PCG (abft_pcg_dist_*): set by _begin
+  bool pcg_dist_on = false;
   std::vector<void *> owned;
   int device = 0;
   int num_sms = 148;

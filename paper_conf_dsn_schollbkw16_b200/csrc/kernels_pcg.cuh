@@ -34,6 +34,7 @@ struct PcgScalars {
 
 struct PcgArgs {
   int64_t n;
+  int64_t ns;  // stride of the scratch vectors (n rounded up to even: 16-B aligned)
   const double *__restrict__ b;
   double *x, *r, *z, *p, *q;
   const double *__restrict__ d;
@@ -51,6 +52,12 @@ struct PcgArgs {
   int32_t ckpt_every;
   const int32_t *dflag;
   double *ck;
+  // distributed PCG (abft_pcg_dist_*): nullable.  dsend: the last CTA writes
+  // this rank's chunk-tree sums here instead of updating the scalars (the
+  // combine kernel finishes them over all ranks); pext: p is also written to
+  // the own slice of the halo-extended SpMV operand (any alignment).
+  double *dsend;
+  double *pext;
 };
 
 // Eight consecutive doubles v[0..8) at p + 8t (or absent past n).
@@ -155,15 +162,70 @@ __device__ __forceinline__ void pcg_stats(const PcgArgs &a, PcgScalars *sc) {
 }
 
 // diag(A) (R21; missing diagonal -> 0, as the oracle)
-__global__ void k_pcg_diag(int64_t n, const int32_t *__restrict__ rp,
+__global__ void k_pcg_diag(int64_t n, int64_t off, const int32_t *__restrict__ rp,
                            const int32_t *__restrict__ ci, const double *__restrict__ va,
                            double *d) {
   const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
   double v = 0.0;
   for (int32_t q = rp[i]; q < rp[i + 1]; ++q)
-    if (ci[q] == i) v = va[q];
+    if (ci[q] == i + off) v = va[q];
   d[i] = v;
+}
+
+// Scalar steps of each kernel's last CTA, shared with the distributed
+// combine (k_pcg_comb), which calls them with the all-rank sums.
+__device__ __forceinline__ void init_scalars(const PcgArgs &a, double RZ, double RR, double BB) {
+  PcgScalars *sc = a.sc;
+  pcg_stats(a, sc);  // the SpMV q = A x0
+  sc->rho = RZ;
+  sc->res = __dsqrt_rn(RR);
+  sc->thr = dmul(a.tol, __dsqrt_rn(BB));
+  sc->it = 0;
+  if (a.hist) a.hist[0] = sc->res;
+  sc->state = (sc->res <= sc->thr) ? PCG_CONVERGED : (sc->max_iter <= 0 ? PCG_MAXITER : PCG_RUN);
+  if (!(sc->res == sc->res)) sc->state = PCG_BREAKDOWN;
+  if (a.cr) {
+    sc->calls += 1;
+    sc->skip_it = 0;
+    sc->ck_rho = sc->rho;
+    sc->ck_res = sc->res;
+    sc->ck_it = 0;
+  }
+}
+
+__device__ __forceinline__ void dot_scalars(const PcgArgs &a, double PQ) {
+  PcgScalars *sc = a.sc;
+  pcg_stats(a, sc);
+  sc->pq = PQ;
+  if (!(PQ > 0.0))
+    sc->state = PCG_BREAKDOWN;
+  else
+    sc->alpha = __ddiv_rn(sc->rho, PQ);
+}
+
+__device__ __forceinline__ void update_scalars(const PcgArgs &a, int64_t iter, double RZ,
+                                               double RR) {
+  PcgScalars *sc = a.sc;
+  const double res = __dsqrt_rn(RR);
+  sc->it += 1;
+  sc->res = res;
+  if (a.hist) a.hist[sc->it] = res;
+  sc->beta = __ddiv_rn(RZ, sc->rho);
+  sc->rho = RZ;
+  sc->upd = iter;
+  if (res <= sc->thr) sc->state = PCG_CONVERGED;
+  else if (!(res == res)) sc->state = PCG_BREAKDOWN;
+  else if (sc->it >= sc->max_iter) sc->state = PCG_MAXITER;
+}
+
+// p's copy in the halo-extended operand (distributed PCG): scalar stores,
+// the own slice need not be 16-byte aligned.
+__device__ __forceinline__ void st8_ext(double *p, const double (&v)[8], int64_t i0, int64_t n) {
+  if (!p) return;
+#pragma unroll
+  for (int u = 0; u < 8; ++u)
+    if (i0 + u < n) p[i0 + u] = v[u];
 }
 
 // r = b - q; z = r / d; p = z; rho = PW(r.z); res = ||r||; thr = tol ||b||
@@ -187,13 +249,14 @@ __global__ void __launch_bounds__(kPcgThreads) k_pcg_init(const PcgArgs a) {
   st8(a.r, r, i0, a.n);
   st8(a.z, z, i0, a.n);
   st8(a.p, z, i0, a.n);
+  st8_ext(a.pext, z, i0, a.n);
   if (a.cr) {  // sample 0: x0, r0, z0, p0
     double xv[8];
     ld8(xv, a.x, i0, a.n);
     st8(a.ck, xv, i0, a.n);
-    st8(a.ck + a.n, r, i0, a.n);
-    st8(a.ck + 2 * a.n, z, i0, a.n);
-    st8(a.ck + 3 * a.n, z, i0, a.n);
+    st8(a.ck + a.ns, r, i0, a.n);
+    st8(a.ck + 2 * a.ns, z, i0, a.n);
+    st8(a.ck + 3 * a.ns, z, i0, a.n);
   }
   const double RZc = cta_pw(rz, i0, a.n, s_w);
   const double RRc = cta_pw(rr, i0, a.n, s_w);
@@ -208,21 +271,12 @@ __global__ void __launch_bounds__(kPcgThreads) k_pcg_init(const PcgArgs a) {
   const double RR = grid_pw(a.part1, gridDim.x, s_red);
   const double BB = grid_pw(a.part2, gridDim.x, s_red);
   if (threadIdx.x == 0) {
-    PcgScalars *sc = a.sc;
-    pcg_stats(a, sc);  // the SpMV q = A x0
-    sc->rho = RZ;
-    sc->res = __dsqrt_rn(RR);
-    sc->thr = dmul(a.tol, __dsqrt_rn(BB));
-    sc->it = 0;
-    if (a.hist) a.hist[0] = sc->res;
-    sc->state = (sc->res <= sc->thr) ? PCG_CONVERGED : (sc->max_iter <= 0 ? PCG_MAXITER : PCG_RUN);
-    if (!(sc->res == sc->res)) sc->state = PCG_BREAKDOWN;
-    if (a.cr) {
-      sc->calls += 1;
-      sc->skip_it = 0;
-      sc->ck_rho = sc->rho;
-      sc->ck_res = sc->res;
-      sc->ck_it = 0;
+    if (a.dsend) {
+      a.dsend[0] = RZ;
+      a.dsend[1] = RR;
+      a.dsend[2] = BB;
+    } else {
+      init_scalars(a, RZ, RR, BB);
     }
     *a.ticket = 0u;
   }
@@ -245,13 +299,10 @@ __global__ void __launch_bounds__(kPcgThreads) k_pcg_dot(const PcgArgs a) {
   if (!last_cta(a.ticket, &s_flag)) return;
   const double PQ = grid_pw(a.part0, gridDim.x, s_red);
   if (threadIdx.x == 0) {
-    PcgScalars *sc = a.sc;
-    pcg_stats(a, sc);
-    sc->pq = PQ;
-    if (!(PQ > 0.0))
-      sc->state = PCG_BREAKDOWN;
+    if (a.dsend)
+      a.dsend[0] = PQ;
     else
-      sc->alpha = __ddiv_rn(sc->rho, PQ);
+      dot_scalars(a, PQ);
     *a.ticket = 0u;
   }
 }
@@ -292,17 +343,12 @@ __global__ void __launch_bounds__(kPcgThreads) k_pcg_update(const PcgArgs a, int
   const double RZ = grid_pw(a.part0, gridDim.x, s_red);
   const double RR = grid_pw(a.part1, gridDim.x, s_red);
   if (threadIdx.x == 0) {
-    PcgScalars *sc = a.sc;
-    const double res = __dsqrt_rn(RR);
-    sc->it += 1;
-    sc->res = res;
-    if (a.hist) a.hist[sc->it] = res;
-    sc->beta = __ddiv_rn(RZ, sc->rho);
-    sc->rho = RZ;
-    sc->upd = iter;
-    if (res <= sc->thr) sc->state = PCG_CONVERGED;
-    else if (!(res == res)) sc->state = PCG_BREAKDOWN;
-    else if (sc->it >= sc->max_iter) sc->state = PCG_MAXITER;
+    if (a.dsend) {
+      a.dsend[0] = RZ;
+      a.dsend[1] = RR;
+    } else {
+      update_scalars(a, iter, RZ, RR);
+    }
     *a.ticket = 0u;
   }
 }
@@ -319,6 +365,7 @@ __global__ void __launch_bounds__(kPcgThreads) k_pcg_p(const PcgArgs a, int64_t 
 #pragma unroll
   for (int u = 0; u < 8; ++u) pv[u] = dadd(zv[u], dmul(beta, pv[u]));
   st8(a.p, pv, i0, a.n);
+  st8_ext(a.pext, pv, i0, a.n);
   // checkpoint mode: sample (x, r, z, p, rho, it) every ckpt_every iterations
   const int64_t it = a.sc->it;
   if (a.cr && a.ckpt_every > 0 && it % a.ckpt_every == 0) {
@@ -326,9 +373,9 @@ __global__ void __launch_bounds__(kPcgThreads) k_pcg_p(const PcgArgs a, int64_t 
     ld8(xv, a.x, i0, a.n);
     ld8(rv, a.r, i0, a.n);
     st8(a.ck, xv, i0, a.n);
-    st8(a.ck + a.n, rv, i0, a.n);
-    st8(a.ck + 2 * a.n, zv, i0, a.n);
-    st8(a.ck + 3 * a.n, pv, i0, a.n);
+    st8(a.ck + a.ns, rv, i0, a.n);
+    st8(a.ck + 2 * a.ns, zv, i0, a.n);
+    st8(a.ck + 3 * a.ns, pv, i0, a.n);
     if (blockIdx.x == 0 && threadIdx.x == 0) {
       a.sc->ck_rho = a.sc->rho;
       a.sc->ck_res = a.sc->res;
@@ -348,11 +395,11 @@ __global__ void __launch_bounds__(kPcgThreads) k_pcg_cr(const PcgArgs a) {
     double v[8];
     ld8(v, a.ck, i0, a.n);
     st8(a.x, v, i0, a.n);
-    ld8(v, a.ck + a.n, i0, a.n);
+    ld8(v, a.ck + a.ns, i0, a.n);
     st8(a.r, v, i0, a.n);
-    ld8(v, a.ck + 2 * a.n, i0, a.n);
+    ld8(v, a.ck + 2 * a.ns, i0, a.n);
     st8(a.z, v, i0, a.n);
-    ld8(v, a.ck + 3 * a.n, i0, a.n);
+    ld8(v, a.ck + 3 * a.ns, i0, a.n);
     st8(a.p, v, i0, a.n);
   }
   if (blockIdx.x == 0 && threadIdx.x == 0) {
@@ -367,6 +414,35 @@ __global__ void __launch_bounds__(kPcgThreads) k_pcg_cr(const PcgArgs a) {
       sc->flagged += 1;                      // detections = rollbacks
     }
   }
+}
+
+// Distributed PCG: finish a phase's dot products over all ranks.  recv holds
+// world x 3 partials (rank r at [3r, 3r+3), gathered in rank order); each
+// component is PW over the ranks (R2: pad with absent slots to a power of
+// two).  One thread; the scalar steps are the single-GPU ones.
+__device__ __forceinline__ double pw_ranks(const double *recv, int world, int c) {
+  double v[64];
+  int m = 1;
+  while (m < world) m <<= 1;
+  for (int q = 0; q < m; ++q) v[q] = q < world ? recv[3 * q + c] : kAbsent;
+  for (int s = 1; s < m; s <<= 1)
+    for (int q = 0; q + s < m; q += 2 * s) v[q] = dadd(v[q], v[q + s]);
+  return v[0];
+}
+
+enum { PCG_PHASE_INIT = 0, PCG_PHASE_DOT = 1, PCG_PHASE_UPDATE = 2, PCG_PHASE_P = 3 };
+
+__global__ void k_pcg_comb(const PcgArgs a, int phase, int64_t iter, const double *recv,
+                           int world) {
+  if (threadIdx.x != 0 || blockIdx.x != 0) return;
+  if (phase != PCG_PHASE_INIT && pcg_skip(a.sc)) return;
+  const double s0 = pw_ranks(recv, world, 0);
+  if (phase == PCG_PHASE_INIT)
+    init_scalars(a, s0, pw_ranks(recv, world, 1), pw_ranks(recv, world, 2));
+  else if (phase == PCG_PHASE_DOT)
+    dot_scalars(a, s0);
+  else
+    update_scalars(a, iter, s0, pw_ranks(recv, world, 1));
 }
 
 }  // namespace abft

@@ -232,3 +232,136 @@ class DistSpmv:
         """Steps 4-5 with beta from all ranks' partials (self.parts)."""
         self.h.finish(self.x_ext, self.y, self.parts, rounds, inject)
         return self.y
+
+    def plain(self, comm):
+        """Unprotected SpMV (same kernels, check off) over the extended x."""
+        from .abft import NOCHECK
+        comm.halo(self.sh, self.x_ext)
+        self.h.spmv(self.x_ext, self.y, mode=NOCHECK)
+        return self.y
+
+
+# ---------------------------------------------------------------------------
+# Distributed Jacobi-PCG (SURVEY §8(e), P:294-300) on top of the C ABI
+# ---------------------------------------------------------------------------
+class DistPcg:
+    """One rank's share of the distributed PCG.  Vector kernels and scalar
+    updates run in libabft.so (abft_pcg_dist_*); this class only sequences
+    them around the two exchanges: the x halo of every SpMV (DistSpmv) and the
+    all-gather of the per-phase dot partials (3 doubles per rank), finished in
+    rank order on the device (R28).  Iterates like abft_pcg: the
+    device state word is read every `poll` iterations; every rank computes
+    identical scalars from identical partials, so all stop together."""
+
+    def __init__(self, ds: DistSpmv, check: bool = True):
+        import torch
+        self.ds, self.check = ds, check
+        dev = ds.x_ext.device
+        world = ds.sh.world
+        self.send = torch.zeros(3, dtype=torch.float64, device=dev)
+        self.recv = torch.zeros(3 * world, dtype=torch.float64, device=dev)
+
+    def begin(self, b, x, n_global, tol=1e-6, max_iter=0, res_hist=None, diag=None):
+        mi = max_iter if max_iter > 0 else 10 * n_global
+        self.x, self.mi = x, mi
+        self.ds.h.pcg_dist_begin(b, x, self.ds.own(), self.ds.y, diag, tol, mi, self.check,
+                                 res_hist)
+        self.ds.own().copy_(x)  # the first SpMV operand is x0
+        return mi
+
+    # -- the phases, each rank's half of one exchange --------------------------
+    def spmv_local(self, comm):
+        """Steps 1-3 of the SpMV (halo + fused pass); returns the beta partial
+        to gather (None for the unprotected baseline)."""
+        if not self.check:
+            self.ds.plain(comm)
+            return None
+        return self.ds.step1(comm)
+
+    def spmv_finish(self):
+        if self.check:
+            self.ds.step2()
+
+    def local(self, phase, it=0):
+        from .abft import PCG_PHASE_P
+        self.ds.h.pcg_dist_local(phase, it, None if phase == PCG_PHASE_P else self.send)
+        return self.send
+
+    def combine(self, phase, it=0):
+        self.ds.h.pcg_dist_combine(phase, it, self.recv, self.ds.sh.world)
+
+    def status(self):
+        return self.ds.h.pcg_dist_status()
+
+    # -- driver over torch.distributed (one process per GPU) -----------------
+    def solve(self, comm: TorchDistComm, b, x, n_global, tol=1e-6, max_iter=0, res_hist=None,
+              diag=None, poll=16):
+        from .abft import PCG_PHASE_DOT, PCG_PHASE_INIT, PCG_PHASE_P, PCG_PHASE_UPDATE
+
+        def spmv():
+            part = self.spmv_local(comm)
+            if part is not None:
+                comm.gather_partials(part, self.ds.parts)
+                self.spmv_finish()
+
+        def reduce(phase, it):
+            comm.gather_partials(self.local(phase, it), self.recv)
+            self.combine(phase, it)
+
+        mi = self.begin(b, x, n_global, tol, max_iter, res_hist, diag)
+        spmv()
+        reduce(PCG_PHASE_INIT, 0)
+        j = 0
+        while True:
+            state, stats = self.status()
+            if state != 0 or j >= mi:
+                return state, stats
+            for _ in range(min(poll, mi - j)):
+                j += 1
+                spmv()  # q = A p (p sits in the operand's own slice)
+                reduce(PCG_PHASE_DOT, j)
+                reduce(PCG_PHASE_UPDATE, j)
+                self.local(PCG_PHASE_P, j)
+
+
+def pcg_lockstep(pcgs, comm: LocalComm, bs, xs, n_global, tol=1e-6, max_iter=0, hists=None,
+                 poll=16):
+    """Logical ranks in one process (tests): every phase runs on all ranks,
+    then the partials are concatenated in rank order -- the exchange pattern
+    of DistPcg.solve without a process group."""
+    import torch
+
+    from .abft import PCG_PHASE_DOT, PCG_PHASE_INIT, PCG_PHASE_P, PCG_PHASE_UPDATE
+    hists = hists or [None] * len(pcgs)
+
+    def spmv():
+        parts = [p.spmv_local(comm) for p in pcgs]
+        if parts[0] is not None:
+            allp = torch.cat(parts)
+            for p in pcgs:
+                p.ds.parts.copy_(allp)
+                p.spmv_finish()
+
+    def reduce(phase, it):
+        sends = torch.cat([p.local(phase, it).clone() for p in pcgs])
+        for p in pcgs:
+            p.recv.copy_(sends)
+            p.combine(phase, it)
+
+    mi = 0
+    for p, b, x, h in zip(pcgs, bs, xs, hists):
+        mi = p.begin(b, x, n_global, tol, max_iter, h)
+    spmv()
+    reduce(PCG_PHASE_INIT, 0)
+    j = 0
+    while True:
+        sts = [p.status() for p in pcgs]
+        if sts[0][0] != 0 or j >= mi:
+            return sts
+        for _ in range(min(poll, mi - j)):
+            j += 1
+            spmv()
+            reduce(PCG_PHASE_DOT, j)
+            reduce(PCG_PHASE_UPDATE, j)
+            for p in pcgs:
+                p.local(PCG_PHASE_P, j)

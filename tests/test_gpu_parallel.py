@@ -86,3 +86,89 @@ def test_shards_match_oracle(O, torch_cuda, name, world):
     for r in range(5):
         assert np.array_equal(flags[r], ref.flags[r]), (r, flags[r], ref.flags[r])
     assert np.array_equal(y.view(np.uint64), ref.y.view(np.uint64))
+
+
+# ---------------------------------------------------------------------------
+# Distributed PCG (abft_pcg_dist_*): logical ranks in lockstep on one GPU,
+# against the rank-partitioned oracle (R28) bit for bit.
+# ---------------------------------------------------------------------------
+def make_shards(A, ranges):
+    world = len(ranges)
+    shards = []
+    for r, (a, b) in enumerate(ranges):
+        rows = G.CSR(A.row_ptr[a:b + 1] - A.row_ptr[a], A.col[A.row_ptr[a]:A.row_ptr[b]],
+                     A.val[A.row_ptr[a]:A.row_ptr[b]])
+        shards.append(PL.make_shard(rows, a, b, r, world, ranges))
+    PL.exchange_plans(shards, range(world))
+    return shards
+
+
+def run_dist_pcg(torch, A, ranges, b, x0, check=True, tol=1e-6, max_iter=0):
+    shards = make_shards(A, ranges)
+    ds = [PL.DistSpmv(sh) for sh in shards]
+    comm = PL.LocalComm(shards, {d.sh.rank: d.x_ext for d in ds})
+    pcgs = [PL.DistPcg(d, check) for d in ds]
+    mi = max_iter if max_iter > 0 else 10 * A.n
+    dev = lambda v: torch.from_numpy(np.ascontiguousarray(v)).cuda()
+    bs = [dev(b[sh.row0:sh.row1]) for sh in shards]
+    xs = [dev(x0[sh.row0:sh.row1]) for sh in shards]
+    hists = [torch.zeros(mi + 1, dtype=torch.float64, device="cuda") for _ in shards]
+    sts = PL.pcg_lockstep(pcgs, comm, bs, xs, A.n, tol, max_iter, hists)
+    torch.cuda.synchronize()
+    x = np.concatenate([v.cpu().numpy() for v in xs])
+    it = sts[0][1]["iters"]
+    for s in sts:  # every rank holds the same scalars
+        assert s[0] == sts[0][0] and s[1]["iters"] == it
+        assert s[1]["final_residual"] == sts[0][1]["final_residual"]
+    return sts[0][0], x, hists[0][: it + 1].cpu().numpy(), sts
+
+
+@pytest.mark.parametrize("check", [True, False])
+@pytest.mark.parametrize("case", ["pow2-2", "pow2-4", "planes-3", "st27-3", "ragged-2"])
+def test_dist_pcg_matches_oracle(O, torch_cuda, case, check):
+    if case.startswith("pow2"):
+        A = G.laplacian_3d_7pt(32)  # 32768 rows: ranks of 16384 / 8192 (aligned)
+        w = int(case[-1])
+        ranges = [(r * A.n // w, (r + 1) * A.n // w) for r in range(w)]
+    elif case == "planes-3":
+        A = G.laplacian_3d_7pt(24)  # 8 planes per rank, not powers of two
+        ranges = [(0, 4608), (4608, 9216), (9216, A.n)]
+    elif case == "st27-3":
+        A = G.stencil_3d_27pt(20, 20, 24)  # odd halo widths: unaligned own slices
+        ranges = PL.block_partition(A.n, 3)
+    else:
+        A = G.laplacian_3d_7pt(21)  # 9261 rows, ragged last block
+        ranges = PL.block_partition(A.n, 2)
+    b = O.spmv(A, G.uniform_vector(A.n, 43))
+    x0 = G.uniform_vector(A.n, 44)
+    ref = O.pcg_ranks(A, b, x0, ranges, tol=1e-6)
+    assert ref.status == 0
+    st, x, hist, sts = run_dist_pcg(torch_cuda, A, ranges, b, x0, check)
+    assert st == 1  # converged
+    assert sts[0][1]["iters"] == ref.iters
+    assert np.array_equal(hist.view(np.uint64), ref.res_hist.view(np.uint64))
+    assert np.array_equal(x.view(np.uint64), ref.x.view(np.uint64))
+    calls = sum(s[1]["spmv_calls"] for s in sts) // len(sts)
+    assert calls == ref.spmv_calls
+    if check:
+        assert all(s[1]["uncorrected_calls"] == 0 for s in sts)
+
+
+def test_dist_pcg_pow2_equals_single_gpu(O, torch_cuda):
+    """Equal power-of-two ranges: the distributed solve is the single-GPU
+    abft_pcg bit for bit (R2 padding independence)."""
+    from paper_conf_dsn_schollbkw16_b200 import abft
+    torch = torch_cuda
+    A = G.laplacian_3d_7pt(32)
+    b = O.spmv(A, G.uniform_vector(A.n, 43))
+    x0 = G.uniform_vector(A.n, 44)
+    h = abft.encode(A)
+    xd = torch.from_numpy(x0.copy()).cuda()
+    hist1 = torch.zeros(10 * A.n + 1, dtype=torch.float64, device="cuda")
+    status, st1 = h.pcg(torch.from_numpy(b).cuda(), xd, tol=1e-6, res_hist=hist1)
+    ranges = [(r * A.n // 4, (r + 1) * A.n // 4) for r in range(4)]
+    st, x, hist, sts = run_dist_pcg(torch, A, ranges, b, x0)
+    assert st1["iters"] == sts[0][1]["iters"]
+    assert np.array_equal(x.view(np.uint64), xd.cpu().numpy().view(np.uint64))
+    assert np.array_equal(hist.view(np.uint64),
+                          hist1[: st1["iters"] + 1].cpu().numpy().view(np.uint64))

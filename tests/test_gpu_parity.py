@@ -356,6 +356,16 @@ def test_pcg_parity(O, torch_cuda, inj):
         assert st["flagged_blocks"] > 0
 
 
+def test_pcg_odd_n(O, torch_cuda):
+    # odd N: the scratch vectors keep a 16-byte aligned stride (n rounded up)
+    A = G.laplacian_3d_7pt(21)  # 9261 rows
+    for inj in (None, dict(seed=5, lam=1e-4, targets=0b111)):
+        ref, status, st, x, hist = _pcg_case(O, torch_cuda, A, inj)
+        assert status == ref.status == 0 and st["iters"] == ref.iters
+        assert_bits_equal(hist, ref.res_hist, "odd-n residual history")
+        assert_bits_equal(x, ref.x, "odd-n solution")
+
+
 def test_pcg_unprotected_and_maxiter(O, torch_cuda):
     A = G.laplacian_3d_7pt(12)
     ref, status, st, x, hist = _pcg_case(O, torch_cuda, A, dict(seed=3, lam=1e-5), check=False)
