@@ -297,6 +297,74 @@ def run_reference(args):
     print(json.dumps(line), flush=True)
 
 
+def run_pcg_dist(args):
+    """configs[4] sharded: the 192^3 PCG split into 192/N-plane
+    slabs, one per rank (strong scaling: the total problem is fixed).  Every
+    SpMV is the distributed protected one (x halo over NCCL P2P + beta
+    partials all-gathered); every PCG reduction is an all-gather of 3 doubles
+    per rank finished in rank order on the device (abft_pcg_dist_*).  Fault
+    free; time-to-solution on the device (CUDA events, max over ranks) for the
+    method and for unprotected SpMVs on the same path."""
+    import torch
+
+    from paper_conf_dsn_schollbkw16_b200 import inputs as G
+    from paper_conf_dsn_schollbkw16_b200 import parallel as PL
+    world, rank, local = dist_init()
+    n3 = args.pcg_n
+    ranges_z = [(n3 * r // world, n3 * (r + 1) // world) for r in range(world)]
+    plane = n3 * n3
+    ranges = [(z0 * plane, z1 * plane) for z0, z1 in ranges_z]
+    a, b_ = ranges[rank]
+    rows = G.stencil_rows("7pt", n3, n3, n3, *ranges_z[rank])
+    sh = PL.make_shard(rows, a, b_, rank, world, ranges)
+    if world > 1:
+        comm = PL.TorchDistComm()
+        PL.plan_from_needs(sh, comm.gather_needs(sh))
+    d = PL.DistSpmv(sh, args.block_size, args.max_rounds)
+    n_glob = n3 ** 3
+    # b = A x* (x* seeded, R15/Q20) through the library's plain SpMV
+    d.own().copy_(torch.from_numpy(G.uniform_vector(sh.n, 43, start=a)))
+    class _Solo:  # world 1: no halo, partials need no exchange
+        def gather_partials(self, part, out):
+            out.copy_(part)
+
+        def halo(self, sh_, x_ext):
+            pass
+
+    c = comm if world > 1 else _Solo()
+    b = d.plain(c).clone()
+    x0 = torch.from_numpy(G.uniform_vector(sh.n, 44, start=a)).cuda()
+    torch.cuda.synchronize()
+    res = {}
+    for name, check in (("unprotected", False), ("protected", True)):
+        p = PL.DistPcg(d, check)
+        times = []
+        for rep in range(max(1, args.pcg_reps) + 1):  # first: warm-up
+            x = x0.clone()
+            barrier(world)
+            torch.cuda.synchronize()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            state, st = p.solve(c, b, x, n_glob, tol=1e-6)
+            e1.record()
+            torch.cuda.synchronize()
+            barrier(world)
+            if rep:
+                times.append(max_over_ranks(e0.elapsed_time(e1), world))
+        res[name] = {"ms": round(statistics.median(times), 3), "iters": st["iters"],
+                     "converged": bool(state == 1), "final_residual": st["final_residual"],
+                     "spmv_calls": st["spmv_calls"], "runs": len(times)}
+    res["protected"]["overhead_pct"] = round(
+        (res["protected"]["ms"] / res["unprotected"]["ms"] - 1) * 100, 2)
+    if rank == 0:
+        print(json.dumps({"metric": "PCG time-to-solution (ms), Jacobi, tol 1e-6, sharded",
+                          "workload": f"3-D 7-point Laplacian {n3}^3 (BASELINE configs[4])",
+                          "n": n_glob, "n_gpus": world, "scaling": "strong",
+                          "parallelism": f"rowblock{world}",
+                          "backend": os.environ.get("ABFT_DIST_BACKEND", "nccl") if world > 1
+                          else "none", "results": res}), flush=True)
+
+
 def run_ours_dist(args):
     """N > 1: weak scaling.  Rank r owns planes [r*nz, (r+1)*nz) of a
     (nz*N) x ny x nx grid of the workload's stencil (the configs[1] 128^3 slab
@@ -639,6 +707,8 @@ def main():
     ap.add_argument("--lam", type=float, default=0.0, help="rate-mode fault rate per op")
     ap.add_argument("--c-csr", action="store_true", help="paper-literal CSR checksum matrix")
     ap.add_argument("--pcg", action="store_true", help="configs[4]: PCG time-to-solution")
+    ap.add_argument("--pcg-dist", action="store_true",
+                    help="configs[4] through the sharded PCG (implied by --pcg at N > 1)")
     ap.add_argument("--compare", action="store_true",
                     help="SURVEY §8(f)1: the method vs the dense check + complete recomputation")
     ap.add_argument("--pcg-n", type=int, default=192)
@@ -649,6 +719,8 @@ def main():
     args = ap.parse_args()
     if args.impl == "reference":
         run_reference(args)
+    elif args.pcg_dist or (args.pcg and int(os.environ.get("WORLD_SIZE", "1")) > 1):
+        run_pcg_dist(args)
     elif args.pcg:
         run_pcg(args)
     elif args.compare:

@@ -172,3 +172,64 @@ def test_dist_pcg_pow2_equals_single_gpu(O, torch_cuda):
     assert np.array_equal(x.view(np.uint64), xd.cpu().numpy().view(np.uint64))
     assert np.array_equal(hist.view(np.uint64),
                           hist1[: st1["iters"] + 1].cpu().numpy().view(np.uint64))
+
+
+def _dist_pcg_worker(rank, world, port, outdir):
+    """One process per rank on the same GPU (gloo process group: the NCCL
+    path needs one GPU per rank): DistPcg.solve with TorchDistComm."""
+    import os
+
+    import torch
+    import torch.distributed as dist
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    torch.cuda.set_device(0)
+    n3 = 24
+    A = G.laplacian_3d_7pt(n3)
+    ranges = PL.block_partition(A.n, world, align=n3 * n3)
+    a, b_ = ranges[rank]
+    rows = G.stencil_rows("7pt", n3, n3, n3, a // (n3 * n3), b_ // (n3 * n3))
+    sh = PL.make_shard(rows, a, b_, rank, world, ranges)
+    comm = PL.TorchDistComm()
+    PL.plan_from_needs(sh, comm.gather_needs(sh))
+    d = PL.DistSpmv(sh)
+    bfull = np.load(os.path.join(outdir, "b.npy"))
+    x0 = np.load(os.path.join(outdir, "x0.npy"))
+    b = torch.from_numpy(bfull[a:b_].copy()).cuda()
+    x = torch.from_numpy(x0[a:b_].copy()).cuda()
+    hist = torch.zeros(10 * A.n + 1, dtype=torch.float64, device="cuda")
+    state, st = PL.DistPcg(d, True).solve(comm, b, x, A.n, tol=1e-6, res_hist=hist)
+    torch.cuda.synchronize()
+    np.save(os.path.join(outdir, f"x{rank}.npy"), x.cpu().numpy())
+    np.save(os.path.join(outdir, f"h{rank}.npy"), hist[: st["iters"] + 1].cpu().numpy())
+    np.save(os.path.join(outdir, f"s{rank}.npy"), np.array([state, st["iters"]]))
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_dist_pcg_processes(O, torch_cuda, tmp_path, world):
+    """DistPcg.solve across real processes (torch.distributed, gloo staging
+    through the host) == the rank-partitioned oracle bit for bit."""
+    import socket
+
+    import torch.multiprocessing as mp
+    n3 = 24
+    A = G.laplacian_3d_7pt(n3)
+    b = O.spmv(A, G.uniform_vector(A.n, 43))
+    x0 = G.uniform_vector(A.n, 44)
+    np.save(tmp_path / "b.npy", b)
+    np.save(tmp_path / "x0.npy", x0)
+    ranges = PL.block_partition(A.n, world, align=n3 * n3)
+    ref = O.pcg_ranks(A, b, x0, ranges, tol=1e-6)
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        port = s.getsockname()[1]
+    mp.start_processes(_dist_pcg_worker, args=(world, port, str(tmp_path)), nprocs=world,
+                       join=True, start_method="spawn")
+    x = np.concatenate([np.load(tmp_path / f"x{r}.npy") for r in range(world)])
+    for r in range(world):
+        state, it = np.load(tmp_path / f"s{r}.npy")
+        assert state == 1 and it == ref.iters
+        assert np.array_equal(np.load(tmp_path / f"h{r}.npy").view(np.uint64),
+                              ref.res_hist.view(np.uint64))
+    assert np.array_equal(x.view(np.uint64), ref.x.view(np.uint64))
