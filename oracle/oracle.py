@@ -436,3 +436,77 @@ def pcg_ranks(A, b, x0, ranges, diag=None, tol=1e-6, max_iter=0) -> PcgResult:
     if status == 0 and not (res <= thr):
         status = -5
     return PcgResult(status, x, np.array(hist), it, calls, 0, 0, 0)
+
+
+def pcg_cg1_ranks(A, b, x0, ranges, diag=None, tol=1e-6, max_iter=0) -> PcgResult:
+    """Single-reduction Jacobi-PCG (Chronopoulos & Gear 1989, preconditioned
+    form, R29 -- beyond the paper, which uses the
+    textbook PCG of P:294-300).  The recurrence s = A p replaces the second
+    reduction: per iteration the three dots (r, u), (r, r), (w, u) with
+    u = M^-1 r, w = A u are one reduction.  Fault free; dots by `dot_ranks`.
+        r0 = b - A x0, u0 = r0 / d, gamma0 = (r0, u0), res0 = ||r0||
+        w0 = A u0, delta0 = (w0, u0), alpha0 = gamma0 / delta0, beta0 = 0,
+        p = u0, s = w0
+        j = 1, 2, ...: p = u + beta p; s = w + beta s; x = x + alpha p;
+          r = r - alpha s; u = r / d; gamma' = (r, u); res = ||r||;
+          w = A u; delta = (w, u); stop if res <= tol ||b||;
+          beta = gamma' / gamma; alpha = gamma' / (delta - beta gamma' / alpha)
+    In exact arithmetic the iterates are those of `pcg_ranks`; one SpMV more
+    (w0).  Status 0 / -5 / -7 as or_pcg."""
+    n = A.n
+    b = np.ascontiguousarray(b, dtype=np.float64)
+    x = np.array(x0, dtype=np.float64, copy=True)
+    mi = max_iter if max_iter > 0 else 10 * n
+    if diag is None:
+        d = np.zeros(n)  # diag(A), a missing diagonal -> 0 (R21)
+        rows = np.repeat(np.arange(n), np.diff(np.asarray(A.row_ptr, dtype=np.int64)))
+        on = np.asarray(A.col) == rows
+        d[rows[on]] = np.asarray(A.val)[on]
+    else:
+        d = np.asarray(diag, dtype=np.float64)
+    r = b - spmv(A, x)
+    u = r / d
+    gamma = dot_ranks(r, u, ranges)
+    thr = tol * np.sqrt(dot_ranks(b, b, ranges))
+    res = np.sqrt(dot_ranks(r, r, ranges))
+    hist, it, calls = [res], 0, 1
+    if res <= thr:
+        return PcgResult(0, x, np.array(hist), 0, calls, 0, 0, 0)
+    w = spmv(A, u)
+    calls += 1
+    delta = dot_ranks(w, u, ranges)
+    if not (delta > 0.0):
+        return PcgResult(-7, x, np.array(hist), 0, calls, 0, 0, 0)
+    alpha, beta = gamma / delta, 0.0
+    p, s = u.copy(), w.copy()
+    status = -5
+    while it < mi:
+        p = u + beta * p
+        s = w + beta * s
+        x = x + alpha * p
+        r = r - alpha * s
+        u = r / d
+        g_new = dot_ranks(r, u, ranges)
+        rr = dot_ranks(r, r, ranges)
+        w = spmv(A, u)
+        calls += 1
+        delta = dot_ranks(w, u, ranges)
+        it += 1
+        res = np.sqrt(rr)
+        hist.append(res)
+        if res <= thr:
+            status = 0
+            break
+        if res != res:
+            status = -7
+            break
+        if it >= mi:
+            break
+        beta = g_new / gamma
+        den = delta - beta * g_new / alpha
+        if not (den > 0.0):
+            status = -7
+            break
+        alpha = g_new / den
+        gamma = g_new
+    return PcgResult(status, x, np.array(hist), it, calls, 0, 0, 0)

@@ -752,3 +752,51 @@ class TestPcgRanks:
         a = np.arange(1, 101, dtype=np.float64)
         assert O.dot_ranks(a, np.ones(100), [(0, 7), (7, 50), (50, 100)]) == 5050.0
         assert O.dot_ranks(a, a, [(0, 0), (0, 100)]) == float(np.sum(a * a))
+
+
+class TestPcgSingleReduction:
+    """Chronopoulos-Gear PCG (R29): same Krylov iterates as PCG in exact
+    arithmetic.  Pins: SciPy's CG (independent), finite termination on a
+    diagonal matrix, and agreement with the textbook oracle to rounding."""
+
+    def test_matches_scipy_cg(self, O):
+        import scipy.sparse as sp
+        import scipy.sparse.linalg as spla
+        A = G.laplacian_3d_7pt(12)
+        b = O.spmv(A, G.uniform_vector(A.n, 43))
+        x0 = G.uniform_vector(A.n, 44)
+        r = O.pcg_cg1_ranks(A, b, x0, [(0, A.n)], tol=1e-6)
+        assert r.status == 0
+        S = sp.csr_matrix((A.val, A.col, A.row_ptr), shape=(A.n, A.n))
+        d = S.diagonal()
+        M = spla.LinearOperator(S.shape, matvec=lambda v: v / d)
+        hist = []
+        xsc, info = spla.cg(S, b, x0=x0.copy(), rtol=1e-6, atol=0.0, M=M,
+                            callback=lambda xk: hist.append(np.linalg.norm(b - S @ xk)))
+        assert info == 0 and r.iters == len(hist)
+        assert r.spmv_calls == r.iters + 2
+        assert np.max(np.abs(np.array(hist) - r.res_hist[1:])) < 1e-9 * np.linalg.norm(b)
+        assert np.linalg.norm(r.x - xsc) <= 1e-8 * np.linalg.norm(xsc)
+
+    def test_diagonal_matrix_one_iteration(self, O):
+        # M^-1 A = I: the first step solves exactly (alpha = 1, x = x0 + u0)
+        n = 64
+        vals = 2.0 ** np.arange(-3, 3, dtype=np.float64).repeat(11)[:n]
+        A = G.CSR(np.arange(n + 1, dtype=np.int32), np.arange(n, dtype=np.int32), vals)
+        xs = G.uniform_vector(n, 3)
+        b = vals * xs
+        r = O.pcg_cg1_ranks(A, b, np.zeros(n), [(0, 32), (32, 64)], tol=1e-12)
+        assert r.status == 0 and r.iters == 1
+        assert np.array_equal(r.x, xs)
+
+    def test_close_to_textbook_pcg(self, O):
+        A = G.stencil_3d_27pt(10, 10, 12)
+        b = O.spmv(A, G.uniform_vector(A.n, 43))
+        x0 = G.uniform_vector(A.n, 44)
+        ranges = [(0, 400), (400, A.n)]
+        ref = O.pcg_ranks(A, b, x0, ranges, tol=1e-8)
+        r = O.pcg_cg1_ranks(A, b, x0, ranges, tol=1e-8)
+        assert r.status == ref.status == 0 and abs(r.iters - ref.iters) <= 1
+        k = min(r.iters, ref.iters)
+        assert np.max(np.abs(r.res_hist[:k] - ref.res_hist[:k])) < 1e-10 * np.linalg.norm(b)
+        assert np.linalg.norm(r.x - ref.x) <= 1e-8 * np.linalg.norm(ref.x)
