@@ -336,8 +336,10 @@ def run_pcg_dist(args):
     x0 = torch.from_numpy(G.uniform_vector(sh.n, 44, start=a)).cuda()
     torch.cuda.synchronize()
     res = {}
-    for name, check in (("unprotected", False), ("protected", True)):
-        p = PL.DistPcg(d, check)
+    for name, check, variant in (("unprotected", False, "pcg"), ("protected", True, "pcg"),
+                                  ("unprotected_cg1", False, "cg1"),
+                                  ("protected_cg1", True, "cg1")):
+        p = PL.DistPcg(d, check, variant)
         times = []
         for rep in range(max(1, args.pcg_reps) + 1):  # first: warm-up
             x = x0.clone()
@@ -354,13 +356,17 @@ def run_pcg_dist(args):
         res[name] = {"ms": round(statistics.median(times), 3), "iters": st["iters"],
                      "converged": bool(state == 1), "final_residual": st["final_residual"],
                      "spmv_calls": st["spmv_calls"], "runs": len(times)}
-    res["protected"]["overhead_pct"] = round(
-        (res["protected"]["ms"] / res["unprotected"]["ms"] - 1) * 100, 2)
+    for v in ("", "_cg1"):
+        res["protected" + v]["overhead_pct"] = round(
+            (res["protected" + v]["ms"] / res["unprotected" + v]["ms"] - 1) * 100, 2)
     if rank == 0:
         print(json.dumps({"metric": "PCG time-to-solution (ms), Jacobi, tol 1e-6, sharded",
                           "workload": f"3-D 7-point Laplacian {n3}^3 (BASELINE configs[4])",
                           "n": n_glob, "n_gpus": world, "scaling": "strong",
                           "parallelism": f"rowblock{world}",
+                          "variants": "pcg = textbook (2 reductions + SpMV beta gather per "
+                                      "iteration); cg1 = single reduction (Chronopoulos-Gear, "
+                                      "1 reduction + SpMV beta gather, one extra SpMV)",
                           "backend": os.environ.get("ABFT_DIST_BACKEND", "nccl") if world > 1
                           else "none", "results": res}), flush=True)
 

@@ -283,6 +283,16 @@ abft_status abft_pcg(abft_handle_t h, const double *b, double *x, const double *
 #define ABFT_PCG_PHASE_DOT 1
 #define ABFT_PCG_PHASE_UPDATE 2
 #define ABFT_PCG_PHASE_P 3
+/* Single-reduction (Chronopoulos-Gear) variant (DESIGN.md
+ * R29; beyond the paper): s = A p is carried by recurrence, so each
+ * iteration needs ONE gather of (r.u, r.r, w.u) instead of two.  Sequence
+ * after begin: SpMV q = A x0; local(INIT) -> gather -> combine(INIT); SpMV
+ * w = A u0 (the operand's own slice holds u0); local(CG1_DOT, 0) -> gather ->
+ * combine(CG1_DOT, 0); per iteration j >= 1: local(CG1_UPDATE, j) (p, s, x,
+ * r, u; partials r.u, r.r in send[0..2)); SpMV w = A u; local(CG1_DOT, j)
+ * (partial w.u in send[2]); gather -> combine(CG1_DOT, j).  q is w. */
+#define ABFT_PCG_PHASE_CG1_UPDATE 4
+#define ABFT_PCG_PHASE_CG1_DOT 5
 abft_status abft_pcg_dist_begin(abft_handle_t h, const double *b, double *x, double *pext,
                                 double *q, const double *diag, double tol, int64_t max_iter,
                                 int32_t check, double *res_hist, void *stream);

@@ -33,6 +33,7 @@ SYMBOLS = [
     "abft_pcg_dist_status",
 ]
 PCG_PHASE_INIT, PCG_PHASE_DOT, PCG_PHASE_UPDATE, PCG_PHASE_P = 0, 1, 2, 3
+PCG_PHASE_CG1_UPDATE, PCG_PHASE_CG1_DOT = 4, 5  # single-reduction variant
 ENCODE_C_CSR = 1
 CFMT_NAMES = {0: "csr-f64", 1: "int8+u16", 2: "int16+u16", 3: "f32+u16", 4: "f64+u16"}
 

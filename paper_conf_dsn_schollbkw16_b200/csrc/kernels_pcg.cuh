@@ -58,6 +58,7 @@ struct PcgArgs {
   // the own slice of the halo-extended SpMV operand (any alignment).
   double *dsend;
   double *pext;
+  double *s;  // single-reduction variant (cg1): s = A p, updated by recurrence
 };
 
 // Eight consecutive doubles v[0..8) at p + 8t (or absent past n).
@@ -416,6 +417,136 @@ __global__ void __launch_bounds__(kPcgThreads) k_pcg_cr(const PcgArgs a) {
   }
 }
 
+
+// ---------------------------------------------------------------------------
+// Single-reduction PCG (Chronopoulos-Gear, R29):
+// the iteration recurs s = A p so that (r.u), (r.r) and (w.u) with w = A u
+// are ONE all-gather per iteration instead of two.  Vectors: x, r, u (the z
+// slot), w (the SpMV output q), p, s; scalars: gamma (rho), delta (pq),
+// alpha, beta.  Distributed API only (phases 4 and 5).
+// ---------------------------------------------------------------------------
+enum { PCG_PHASE_CG1_UPDATE = 4, PCG_PHASE_CG1_DOT = 5 };
+
+// p = u + beta p; s = w + beta s; x += alpha p; r -= alpha s; u = r / d;
+// partials (r.u, r.r) -> dsend[0..2)
+__global__ void __launch_bounds__(kPcgThreads) k_cg1_update(const PcgArgs a) {
+  __shared__ double s_w[8];
+  __shared__ double s_red[kPcgThreads];
+  __shared__ int s_flag;
+  if (pcg_skip(a.sc)) return;
+  const double alpha = a.sc->alpha, beta = a.sc->beta;
+  const int64_t i0 = (int64_t)blockIdx.x * kPcgRows + threadIdx.x * kPcgPer;
+  double uv[8], wv[8], pv[8], sv[8], xv[8], rv[8], dv[8], ru[8], rr[8];
+  ld8(uv, a.z, i0, a.n);
+  ld8(wv, a.q, i0, a.n);
+  ld8(pv, a.p, i0, a.n);
+  ld8(sv, a.s, i0, a.n);
+  ld8(xv, a.x, i0, a.n);
+  ld8(rv, a.r, i0, a.n);
+  ld8(dv, a.d, i0, a.n);
+#pragma unroll
+  for (int u = 0; u < 8; ++u) {
+    pv[u] = dadd(uv[u], dmul(beta, pv[u]));
+    sv[u] = dadd(wv[u], dmul(beta, sv[u]));
+    xv[u] = dadd(xv[u], dmul(alpha, pv[u]));
+    rv[u] = dsub(rv[u], dmul(alpha, sv[u]));
+    uv[u] = __ddiv_rn(rv[u], dv[u]);
+    ru[u] = dmul(rv[u], uv[u]);
+    rr[u] = dmul(rv[u], rv[u]);
+  }
+  st8(a.p, pv, i0, a.n);
+  st8(a.s, sv, i0, a.n);
+  st8(a.x, xv, i0, a.n);
+  st8(a.r, rv, i0, a.n);
+  st8(a.z, uv, i0, a.n);
+  st8_ext(a.pext, uv, i0, a.n);  // the next SpMV's operand is u
+  const double RUc = cta_pw(ru, i0, a.n, s_w);
+  const double RRc = cta_pw(rr, i0, a.n, s_w);
+  if (threadIdx.x == 0) {
+    a.part0[blockIdx.x] = RUc;
+    a.part1[blockIdx.x] = RRc;
+  }
+  if (!last_cta(a.ticket, &s_flag)) return;
+  const double RU = grid_pw(a.part0, gridDim.x, s_red);
+  const double RR = grid_pw(a.part1, gridDim.x, s_red);
+  if (threadIdx.x == 0) {
+    a.dsend[0] = RU;
+    a.dsend[1] = RR;
+    *a.ticket = 0u;
+  }
+}
+
+// partial (w.u) -> dsend[2]; first call (iter 0): also s = w (s_0 = A p_0
+// with p_0 = u_0)
+__global__ void __launch_bounds__(kPcgThreads) k_cg1_dot(const PcgArgs a, int64_t iter) {
+  __shared__ double s_w[8];
+  __shared__ double s_red[kPcgThreads];
+  __shared__ int s_flag;
+  if (pcg_skip(a.sc)) return;
+  const int64_t i0 = (int64_t)blockIdx.x * kPcgRows + threadIdx.x * kPcgPer;
+  double wv[8], uv[8];
+  ld8(wv, a.q, i0, a.n);
+  ld8(uv, a.z, i0, a.n);
+  if (iter == 0) st8(a.s, wv, i0, a.n);
+#pragma unroll
+  for (int u = 0; u < 8; ++u) uv[u] = dmul(wv[u], uv[u]);
+  const double WUc = cta_pw(uv, i0, a.n, s_w);
+  if (threadIdx.x == 0) a.part2[blockIdx.x] = WUc;
+  if (!last_cta(a.ticket, &s_flag)) return;
+  const double WU = grid_pw(a.part2, gridDim.x, s_red);
+  if (threadIdx.x == 0) {
+    a.dsend[2] = WU;
+    *a.ticket = 0u;
+  }
+}
+
+// Scalars after the iteration's single reduction.  iter 0: delta_0 = (w.u),
+// alpha_0 = gamma_0 / delta_0, beta_0 = 0.  iter j > 0: gamma' = (r.u),
+// res = sqrt(r.r) (convergence), beta = gamma'/gamma,
+// alpha = gamma' / (delta - beta gamma' / alpha).
+__device__ __forceinline__ void cg1_scalars(const PcgArgs &a, int64_t iter, double RU, double RR,
+                                            double WU) {
+  PcgScalars *sc = a.sc;
+  pcg_stats(a, sc);  // the SpMV w = A u of this step
+  if (iter == 0) {
+    sc->pq = WU;
+    if (!(WU > 0.0)) {
+      sc->state = PCG_BREAKDOWN;
+      return;
+    }
+    sc->alpha = __ddiv_rn(sc->rho, WU);
+    sc->beta = 0.0;
+    return;
+  }
+  const double res = __dsqrt_rn(RR);
+  sc->it += 1;
+  sc->res = res;
+  if (a.hist) a.hist[sc->it] = res;
+  sc->upd = iter;
+  if (res <= sc->thr) {
+    sc->state = PCG_CONVERGED;
+    return;
+  }
+  if (!(res == res)) {
+    sc->state = PCG_BREAKDOWN;
+    return;
+  }
+  if (sc->it >= sc->max_iter) {
+    sc->state = PCG_MAXITER;
+    return;
+  }
+  const double beta = __ddiv_rn(RU, sc->rho);
+  const double den = dsub(WU, __ddiv_rn(dmul(beta, RU), sc->alpha));
+  sc->pq = WU;
+  if (!(den > 0.0)) {
+    sc->state = PCG_BREAKDOWN;
+    return;
+  }
+  sc->beta = beta;
+  sc->alpha = __ddiv_rn(RU, den);
+  sc->rho = RU;
+}
+
 // Distributed PCG: finish a phase's dot products over all ranks.  recv holds
 // world x 3 partials (rank r at [3r, 3r+3), gathered in rank order); each
 // component is PW over the ranks (R2: pad with absent slots to a power of
@@ -441,8 +572,11 @@ __global__ void k_pcg_comb(const PcgArgs a, int phase, int64_t iter, const doubl
     init_scalars(a, s0, pw_ranks(recv, world, 1), pw_ranks(recv, world, 2));
   else if (phase == PCG_PHASE_DOT)
     dot_scalars(a, s0);
-  else
+  else if (phase == PCG_PHASE_UPDATE)
     update_scalars(a, iter, s0, pw_ranks(recv, world, 1));
+  else  // PCG_PHASE_CG1_DOT
+    cg1_scalars(a, iter, iter ? s0 : 0.0, iter ? pw_ranks(recv, world, 1) : 0.0,
+                pw_ranks(recv, world, 2));
 }
 
 }  // namespace abft

@@ -253,9 +253,11 @@ class DistPcg:
     device state word is read every `poll` iterations; every rank computes
     identical scalars from identical partials, so all stop together."""
 
-    def __init__(self, ds: DistSpmv, check: bool = True):
+    def __init__(self, ds: DistSpmv, check: bool = True, variant: str = "pcg"):
         import torch
-        self.ds, self.check = ds, check
+        if variant not in ("pcg", "cg1"):
+            raise ValueError(variant)
+        self.ds, self.check, self.variant = ds, check, variant
         dev = ds.x_ext.device
         world = ds.sh.world
         self.send = torch.zeros(3, dtype=torch.float64, device=dev)
@@ -293,45 +295,64 @@ class DistPcg:
     def status(self):
         return self.ds.h.pcg_dist_status()
 
+    # -- the iteration, over any exchange ------------------------------------
+    def run(self, spmv, reduce, local, status, mi, poll=16):
+        """Sequence one solve (after begin).  spmv(): the distributed SpMV of
+        the operand's own slice into ds.y; reduce(phases): run each
+        (phase, it) local kernel, gather the send slots, combine the last
+        phase; local(phase, it): a kernel without a reduction; status():
+        (state, stats).  variant "pcg": standard (two reductions per
+        iteration); "cg1": single reduction (Chronopoulos-Gear, R29)."""
+        from .abft import (PCG_PHASE_CG1_DOT, PCG_PHASE_CG1_UPDATE, PCG_PHASE_DOT,
+                           PCG_PHASE_INIT, PCG_PHASE_P, PCG_PHASE_UPDATE)
+        spmv()
+        reduce([(PCG_PHASE_INIT, 0)])
+        if self.variant == "cg1":
+            spmv()  # w_0 = A u_0
+            reduce([(PCG_PHASE_CG1_DOT, 0)])
+        j = 0
+        while True:
+            state = status()
+            if state[0] != 0 or j >= mi:
+                return state
+            for _ in range(min(poll, mi - j)):
+                j += 1
+                if self.variant == "cg1":
+                    local(PCG_PHASE_CG1_UPDATE, j)
+                    spmv()  # w = A u
+                    reduce([(PCG_PHASE_CG1_DOT, j)])
+                else:
+                    spmv()  # q = A p (p sits in the operand's own slice)
+                    reduce([(PCG_PHASE_DOT, j)])
+                    reduce([(PCG_PHASE_UPDATE, j)])
+                    local(PCG_PHASE_P, j)
+
     # -- driver over torch.distributed (one process per GPU) -----------------
     def solve(self, comm: TorchDistComm, b, x, n_global, tol=1e-6, max_iter=0, res_hist=None,
               diag=None, poll=16):
-        from .abft import PCG_PHASE_DOT, PCG_PHASE_INIT, PCG_PHASE_P, PCG_PHASE_UPDATE
-
         def spmv():
             part = self.spmv_local(comm)
             if part is not None:
                 comm.gather_partials(part, self.ds.parts)
                 self.spmv_finish()
 
-        def reduce(phase, it):
-            comm.gather_partials(self.local(phase, it), self.recv)
-            self.combine(phase, it)
+        def reduce(phases):
+            for ph, it in phases:
+                self.local(ph, it)
+            comm.gather_partials(self.send, self.recv)
+            self.combine(*phases[-1])
 
         mi = self.begin(b, x, n_global, tol, max_iter, res_hist, diag)
-        spmv()
-        reduce(PCG_PHASE_INIT, 0)
-        j = 0
-        while True:
-            state, stats = self.status()
-            if state != 0 or j >= mi:
-                return state, stats
-            for _ in range(min(poll, mi - j)):
-                j += 1
-                spmv()  # q = A p (p sits in the operand's own slice)
-                reduce(PCG_PHASE_DOT, j)
-                reduce(PCG_PHASE_UPDATE, j)
-                self.local(PCG_PHASE_P, j)
+        return self.run(spmv, reduce, self.local, self.status, mi, poll)
 
 
 def pcg_lockstep(pcgs, comm: LocalComm, bs, xs, n_global, tol=1e-6, max_iter=0, hists=None,
                  poll=16):
     """Logical ranks in one process (tests): every phase runs on all ranks,
     then the partials are concatenated in rank order -- the exchange pattern
-    of DistPcg.solve without a process group."""
+    of DistPcg.solve without a process group.  Rank 0's DistPcg.run sequences
+    the solve; its callbacks act on every rank."""
     import torch
-
-    from .abft import PCG_PHASE_DOT, PCG_PHASE_INIT, PCG_PHASE_P, PCG_PHASE_UPDATE
     hists = hists or [None] * len(pcgs)
 
     def spmv():
@@ -342,26 +363,21 @@ def pcg_lockstep(pcgs, comm: LocalComm, bs, xs, n_global, tol=1e-6, max_iter=0, 
                 p.ds.parts.copy_(allp)
                 p.spmv_finish()
 
-    def reduce(phase, it):
-        sends = torch.cat([p.local(phase, it).clone() for p in pcgs])
+    def reduce(phases):
+        for p in pcgs:
+            for ph, it in phases:
+                p.local(ph, it)
+        sends = torch.cat([p.send for p in pcgs])
         for p in pcgs:
             p.recv.copy_(sends)
-            p.combine(phase, it)
+            p.combine(*phases[-1])
+
+    def local(phase, it=0):
+        for p in pcgs:
+            p.local(phase, it)
 
     mi = 0
     for p, b, x, h in zip(pcgs, bs, xs, hists):
         mi = p.begin(b, x, n_global, tol, max_iter, h)
-    spmv()
-    reduce(PCG_PHASE_INIT, 0)
-    j = 0
-    while True:
-        sts = [p.status() for p in pcgs]
-        if sts[0][0] != 0 or j >= mi:
-            return sts
-        for _ in range(min(poll, mi - j)):
-            j += 1
-            spmv()
-            reduce(PCG_PHASE_DOT, j)
-            reduce(PCG_PHASE_UPDATE, j)
-            for p in pcgs:
-                p.local(PCG_PHASE_P, j)
+    pcgs[0].run(spmv, reduce, local, pcgs[0].status, mi, poll)
+    return [p.status() for p in pcgs]

@@ -103,11 +103,11 @@ def make_shards(A, ranges):
     return shards
 
 
-def run_dist_pcg(torch, A, ranges, b, x0, check=True, tol=1e-6, max_iter=0):
+def run_dist_pcg(torch, A, ranges, b, x0, check=True, tol=1e-6, max_iter=0, variant="pcg"):
     shards = make_shards(A, ranges)
     ds = [PL.DistSpmv(sh) for sh in shards]
     comm = PL.LocalComm(shards, {d.sh.rank: d.x_ext for d in ds})
-    pcgs = [PL.DistPcg(d, check) for d in ds]
+    pcgs = [PL.DistPcg(d, check, variant) for d in ds]
     mi = max_iter if max_iter > 0 else 10 * A.n
     dev = lambda v: torch.from_numpy(np.ascontiguousarray(v)).cuda()
     bs = [dev(b[sh.row0:sh.row1]) for sh in shards]
@@ -174,7 +174,7 @@ def test_dist_pcg_pow2_equals_single_gpu(O, torch_cuda):
                           hist1[: st1["iters"] + 1].cpu().numpy().view(np.uint64))
 
 
-def _dist_pcg_worker(rank, world, port, outdir):
+def _dist_pcg_worker(rank, world, port, outdir, variant="pcg"):
     """One process per rank on the same GPU (gloo process group: the NCCL
     path needs one GPU per rank): DistPcg.solve with TorchDistComm."""
     import os
@@ -198,7 +198,7 @@ def _dist_pcg_worker(rank, world, port, outdir):
     b = torch.from_numpy(bfull[a:b_].copy()).cuda()
     x = torch.from_numpy(x0[a:b_].copy()).cuda()
     hist = torch.zeros(10 * A.n + 1, dtype=torch.float64, device="cuda")
-    state, st = PL.DistPcg(d, True).solve(comm, b, x, A.n, tol=1e-6, res_hist=hist)
+    state, st = PL.DistPcg(d, True, variant).solve(comm, b, x, A.n, tol=1e-6, res_hist=hist)
     torch.cuda.synchronize()
     np.save(os.path.join(outdir, f"x{rank}.npy"), x.cpu().numpy())
     np.save(os.path.join(outdir, f"h{rank}.npy"), hist[: st["iters"] + 1].cpu().numpy())
@@ -206,8 +206,8 @@ def _dist_pcg_worker(rank, world, port, outdir):
     dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("world", [2, 3])
-def test_dist_pcg_processes(O, torch_cuda, tmp_path, world):
+@pytest.mark.parametrize("world,variant", [(2, "pcg"), (3, "pcg"), (2, "cg1")])
+def test_dist_pcg_processes(O, torch_cuda, tmp_path, world, variant):
     """DistPcg.solve across real processes (torch.distributed, gloo staging
     through the host) == the rank-partitioned oracle bit for bit."""
     import socket
@@ -220,11 +220,11 @@ def test_dist_pcg_processes(O, torch_cuda, tmp_path, world):
     np.save(tmp_path / "b.npy", b)
     np.save(tmp_path / "x0.npy", x0)
     ranges = PL.block_partition(A.n, world, align=n3 * n3)
-    ref = O.pcg_ranks(A, b, x0, ranges, tol=1e-6)
+    ref = (O.pcg_cg1_ranks if variant == "cg1" else O.pcg_ranks)(A, b, x0, ranges, tol=1e-6)
     with socket.socket() as s:
         s.bind(("127.0.0.1", 0))
         port = s.getsockname()[1]
-    mp.start_processes(_dist_pcg_worker, args=(world, port, str(tmp_path)), nprocs=world,
+    mp.start_processes(_dist_pcg_worker, args=(world, port, str(tmp_path), variant), nprocs=world,
                        join=True, start_method="spawn")
     x = np.concatenate([np.load(tmp_path / f"x{r}.npy") for r in range(world)])
     for r in range(world):
@@ -232,4 +232,48 @@ def test_dist_pcg_processes(O, torch_cuda, tmp_path, world):
         assert state == 1 and it == ref.iters
         assert np.array_equal(np.load(tmp_path / f"h{r}.npy").view(np.uint64),
                               ref.res_hist.view(np.uint64))
+    assert np.array_equal(x.view(np.uint64), ref.x.view(np.uint64))
+
+
+@pytest.mark.parametrize("check", [True, False])
+@pytest.mark.parametrize("case", ["1", "pow2-4", "planes-3", "st27-3", "ragged-2"])
+def test_dist_cg1_matches_oracle(O, torch_cuda, case, check):
+    """Single-reduction PCG (R29) == oracle pcg_cg1_ranks bit for bit."""
+    if case == "1":
+        A = G.laplacian_3d_7pt(20)
+        ranges = [(0, A.n)]
+    elif case == "pow2-4":
+        A = G.laplacian_3d_7pt(32)
+        ranges = [(r * A.n // 4, (r + 1) * A.n // 4) for r in range(4)]
+    elif case == "planes-3":
+        A = G.laplacian_3d_7pt(24)
+        ranges = [(0, 4608), (4608, 9216), (9216, A.n)]
+    elif case == "st27-3":
+        A = G.stencil_3d_27pt(20, 20, 24)
+        ranges = PL.block_partition(A.n, 3)
+    else:
+        A = G.laplacian_3d_7pt(21)
+        ranges = PL.block_partition(A.n, 2)
+    b = O.spmv(A, G.uniform_vector(A.n, 43))
+    x0 = G.uniform_vector(A.n, 44)
+    ref = O.pcg_cg1_ranks(A, b, x0, ranges, tol=1e-6)
+    assert ref.status == 0
+    st, x, hist, sts = run_dist_pcg(torch_cuda, A, ranges, b, x0, check, variant="cg1")
+    assert st == 1
+    assert sts[0][1]["iters"] == ref.iters
+    assert sts[0][1]["spmv_calls"] == ref.spmv_calls
+    assert np.array_equal(hist.view(np.uint64), ref.res_hist.view(np.uint64))
+    assert np.array_equal(x.view(np.uint64), ref.x.view(np.uint64))
+
+
+def test_dist_cg1_maxiter(O, torch_cuda):
+    A = G.laplacian_3d_7pt(16)
+    b = O.spmv(A, G.uniform_vector(A.n, 43))
+    x0 = G.uniform_vector(A.n, 44)
+    ranges = PL.block_partition(A.n, 2)
+    ref = O.pcg_cg1_ranks(A, b, x0, ranges, tol=1e-6, max_iter=5)
+    st, x, hist, sts = run_dist_pcg(torch_cuda, A, ranges, b, x0, True, max_iter=5,
+                                    variant="cg1")
+    assert ref.status == -5 and st == 3 and sts[0][1]["iters"] == ref.iters == 5
+    assert np.array_equal(hist.view(np.uint64), ref.res_hist.view(np.uint64))
     assert np.array_equal(x.view(np.uint64), ref.x.view(np.uint64))
