@@ -429,7 +429,7 @@ enum { PCG_PHASE_CG1_UPDATE = 4, PCG_PHASE_CG1_DOT = 5 };
 
 // p = u + beta p; s = w + beta s; x += alpha p; r -= alpha s; u = r / d;
 // partials (r.u, r.r) -> dsend[0..2)
-__global__ void __launch_bounds__(kPcgThreads) k_cg1_update(const PcgArgs a) {
+__global__ void __launch_bounds__(kPcgThreads, 2) k_cg1_update(const PcgArgs a) {
   __shared__ double s_w[8];
   __shared__ double s_red[kPcgThreads];
   __shared__ int s_flag;
