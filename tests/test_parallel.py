@@ -135,3 +135,182 @@ def test_gloo_halo_exchange():
     for p in procs:
         p.join(timeout=60)
     assert res == {0: True, 1: True}
+
+
+# ---------------------------------------------------------------------------
+# Distributed PCG host protocol (parallel.DistPcg) on CPU: the device phases
+# are replaced by a numpy test double with the semantics include/abft.h
+# documents for abft_pcg_dist_*, so the sequencing, the halo of p / u and the
+# rank-ordered partial gathers are exercised over real gloo processes and
+# compared with the rank-partitioned oracle.
+# ---------------------------------------------------------------------------
+class _FakeHandle:
+    def __init__(self, O):
+        self.O = O
+
+    def pcg_dist_begin(self, b, x, pext, q, diag, tol, mi, check, hist):
+        self.b, self.x, self.pext, self.q = b.numpy(), x.numpy(), pext.numpy(), q.numpy()
+        self.d = self.diag
+        n = self.b.shape[0]
+        self.r, self.z, self.p, self.s = (np.zeros(n) for _ in range(4))
+        self.tol, self.mi, self.hist = tol, mi, hist
+        self.sc = dict(state=0, it=0, rho=0.0, alpha=0.0, beta=0.0, calls=0, upd=-1)
+
+    def pcg_dist_local(self, phase, it, send):
+        O, sc = self.O, self.sc
+        if phase not in (0, 3) and sc["state"] != 0:
+            return
+        sd = None if send is None else send.numpy()
+        if phase == 0:
+            self.r = self.b - self.q
+            self.z = self.r / self.d
+            self.p = self.z.copy()
+            self.pext[:] = self.z
+            sd[:3] = [O.pw(self.r * self.z), O.pw(self.r * self.r), O.pw(self.b * self.b)]
+        elif phase == 1:
+            sd[0] = O.pw(self.p * self.q)
+        elif phase == 2:
+            self.x[:] = self.x + sc["alpha"] * self.p
+            self.r = self.r - sc["alpha"] * self.q
+            self.z = self.r / self.d
+            sd[:2] = [O.pw(self.r * self.z), O.pw(self.r * self.r)]
+        elif phase == 3:
+            if sc["upd"] == it:
+                self.p = self.z + sc["beta"] * self.p
+                self.pext[:] = self.p
+        elif phase == 4:
+            self.p = self.z + sc["beta"] * self.p
+            self.s = self.q + sc["beta"] * self.s
+            self.x[:] = self.x + sc["alpha"] * self.p
+            self.r = self.r - sc["alpha"] * self.s
+            self.z = self.r / self.d
+            self.pext[:] = self.z
+            sd[:2] = [O.pw(self.r * self.z), O.pw(self.r * self.r)]
+        elif phase == 5:
+            if it == 0:
+                self.s = self.q.copy()
+            sd[2] = O.pw(self.q * self.z)
+
+    def pcg_dist_combine(self, phase, it, recv, world):
+        O, sc = self.O, self.sc
+        if phase != 0 and sc["state"] != 0:
+            return
+        rv = recv.numpy().reshape(world, 3)
+        t = [O.pw(rv[:, c].copy()) for c in range(3)]
+        sc["calls"] += 1 if phase in (0, 1, 5) else 0
+        if phase == 0:
+            sc["rho"], sc["res"] = t[0], np.sqrt(t[1])
+            sc["thr"] = self.tol * np.sqrt(t[2])
+            self.hist.append(sc["res"])
+            sc["state"] = 1 if sc["res"] <= sc["thr"] else 0
+        elif phase == 1:
+            sc["alpha"] = sc["rho"] / t[0]
+        elif phase == 2 or (phase == 5 and it > 0):
+            ru, rr = t[0], t[1]
+            sc["it"] += 1
+            sc["res"] = np.sqrt(rr)
+            self.hist.append(sc["res"])
+            sc["upd"] = it
+            if sc["res"] <= sc["thr"]:
+                sc["state"] = 1
+            elif sc["it"] >= self.mi:
+                sc["state"] = 3
+            elif phase == 2:
+                sc["beta"], sc["rho"] = ru / sc["rho"], ru
+            else:
+                beta = ru / sc["rho"]
+                den = t[2] - beta * ru / sc["alpha"]
+                sc["beta"], sc["alpha"], sc["rho"] = beta, ru / den, ru
+        else:  # cg1, iteration 0
+            sc["alpha"], sc["beta"] = sc["rho"] / t[2], 0.0
+
+    def pcg_dist_status(self):
+        return self.sc["state"], {"iters": self.sc["it"], "spmv_calls": self.sc["calls"]}
+
+
+class _FakeDs:
+    """DistSpmv stand-in: the halo exchange is the real TorchDistComm; the
+    local product is the oracle's row sums over the extended x."""
+
+    def __init__(self, O, sh):
+        import torch
+        self.O, self.sh = O, sh
+        self.x_ext = torch.zeros(sh.n_cols, dtype=torch.float64)
+        self.y = torch.zeros(sh.n, dtype=torch.float64)
+        self.h = _FakeHandle(O)
+        c = sh.csr
+        rows = np.repeat(np.arange(sh.n), np.diff(c.row_ptr))
+        self.h.diag = np.zeros(sh.n)
+        on = c.col == rows + sh.x_offset
+        self.h.diag[rows[on]] = c.val[on]
+
+    def own(self):
+        return self.x_ext[self.sh.x_offset:self.sh.x_offset + self.sh.n]
+
+    def plain(self, comm):
+        comm.halo(self.sh, self.x_ext)
+        c, xe = self.sh.csr, self.x_ext.numpy()
+        self.y.numpy()[:] = [self.O.pw(c.val[c.row_ptr[i]:c.row_ptr[i + 1]] *
+                                       xe[c.col[c.row_ptr[i]:c.row_ptr[i + 1]]])
+                             for i in range(self.sh.n)]
+        return self.y
+
+
+def _gloo_pcg_worker(rank, world, port, variant, q):
+    import torch
+    import torch.distributed as dist
+
+    from oracle import oracle as O
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        A = G.laplacian_3d_7pt(8)
+        ranges = PL.block_partition(A.n, world, align=64)
+        a, b_ = ranges[rank]
+        rows = G.stencil_rows("7pt", 8, 8, 8, a // 64, b_ // 64)
+        sh = PL.make_shard(rows, a, b_, rank, world, ranges)
+        comm = PL.TorchDistComm()
+        PL.plan_from_needs(sh, comm.gather_needs(sh))
+        ds = _FakeDs(O, sh)
+        p = PL.DistPcg.__new__(PL.DistPcg)
+        p.ds, p.check, p.variant = ds, False, variant
+        p.send = torch.zeros(3, dtype=torch.float64)
+        p.recv = torch.zeros(3 * world, dtype=torch.float64)
+        bfull = O.spmv(A, G.uniform_vector(A.n, 43))
+        b = torch.from_numpy(bfull[a:b_].copy())
+        x = torch.from_numpy(G.uniform_vector(A.n, 44)[a:b_].copy())
+        hist = []
+        state, st = p.solve(comm, b, x, A.n, tol=1e-6, res_hist=hist, poll=4)
+        q.put((rank, state, st["iters"], st["spmv_calls"], x.numpy().tolist(), hist))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("variant,world", [("pcg", 2), ("cg1", 2), ("pcg", 3)])
+def test_gloo_dist_pcg_protocol(O, variant, world):
+    import socket
+
+    import torch.multiprocessing as mp
+    A = G.laplacian_3d_7pt(8)
+    ranges = PL.block_partition(A.n, world, align=64)
+    b = O.spmv(A, G.uniform_vector(A.n, 43))
+    x0 = G.uniform_vector(A.n, 44)
+    ref = (O.pcg_cg1_ranks if variant == "cg1" else O.pcg_ranks)(A, b, x0, ranges, tol=1e-6)
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        port = s.getsockname()[1]
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_gloo_pcg_worker, args=(r, world, port, variant, q))
+             for r in range(world)]
+    for p in procs:
+        p.start()
+    res = sorted(q.get(timeout=180) for _ in procs)
+    for p in procs:
+        p.join(timeout=60)
+    x = np.concatenate([np.array(r[4]) for r in res])
+    for r in res:
+        assert r[1] == 1 and r[2] == ref.iters and r[3] == ref.spmv_calls
+        assert np.array_equal(np.array(r[5]), ref.res_hist)
+    assert np.array_equal(x.view(np.uint64), ref.x.view(np.uint64))
