@@ -336,10 +336,17 @@ def run_pcg_dist(args):
     x0 = torch.from_numpy(G.uniform_vector(sh.n, 44, start=a)).cuda()
     torch.cuda.synchronize()
     res = {}
-    for name, check, variant in (("unprotected", False, "pcg"), ("protected", True, "pcg"),
-                                  ("unprotected_cg1", False, "cg1"),
-                                  ("protected_cg1", True, "cg1")):
-        p = PL.DistPcg(d, check, variant)
+    from paper_conf_dsn_schollbkw16_b200 import Inject
+    schemes = [("unprotected", False, "pcg", 0.0), ("protected", True, "pcg", 0.0),
+               ("unprotected_cg1", False, "cg1", 0.0), ("protected_cg1", True, "cg1", 0.0)]
+    for lam in ((1e-8, 1e-6) if args.lam <= 0 else (args.lam,)):
+        schemes += [(f"protected_lam{lam:g}", True, "pcg", lam),
+                    (f"protected_cg1_lam{lam:g}", True, "cg1", lam)]
+    for name, check, variant, lam in schemes:
+        # rate-mode faults per arithmetic op in every rank's SpMVs
+        inj = (lambda call, lam=lam: Inject.rate(seed=1000 * rank + 7, lam=lam, call=call)) \
+            if lam > 0 else None
+        p = PL.DistPcg(d, check, variant, inj)
         times = []
         for rep in range(max(1, args.pcg_reps) + 1):  # first: warm-up
             x = x0.clone()
@@ -355,10 +362,13 @@ def run_pcg_dist(args):
                 times.append(max_over_ranks(e0.elapsed_time(e1), world))
         res[name] = {"ms": round(statistics.median(times), 3), "iters": st["iters"],
                      "converged": bool(state == 1), "final_residual": st["final_residual"],
-                     "spmv_calls": st["spmv_calls"], "runs": len(times)}
-    for v in ("", "_cg1"):
-        res["protected" + v]["overhead_pct"] = round(
-            (res["protected" + v]["ms"] / res["unprotected" + v]["ms"] - 1) * 100, 2)
+                     "spmv_calls": st["spmv_calls"], "runs": len(times), "lambda": lam,
+                     "flagged_blocks_rank0": st["flagged_blocks"],
+                     "uncorrected_calls_rank0": st["uncorrected_calls"]}
+    for k, v in res.items():
+        if k.startswith("protected"):
+            base = res["unprotected_cg1" if "cg1" in k else "unprotected"]["ms"]
+            v["overhead_pct"] = round((v["ms"] / base - 1) * 100, 2)
     if rank == 0:
         print(json.dumps({"metric": "PCG time-to-solution (ms), Jacobi, tol 1e-6, sharded",
                           "workload": f"3-D 7-point Laplacian {n3}^3 (BASELINE configs[4])",

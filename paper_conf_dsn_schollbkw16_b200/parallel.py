@@ -253,11 +253,14 @@ class DistPcg:
     device state word is read every `poll` iterations; every rank computes
     identical scalars from identical partials, so all stop together."""
 
-    def __init__(self, ds: DistSpmv, check: bool = True, variant: str = "pcg"):
+    def __init__(self, ds: DistSpmv, check: bool = True, variant: str = "pcg", inject=None):
         import torch
         if variant not in ("pcg", "cg1"):
             raise ValueError(variant)
-        self.ds, self.check, self.variant = ds, check, variant
+        if inject is not None and not check:
+            raise ValueError("fault injection needs the protected SpMV")
+        self.ds, self.check, self.variant, self.inject = ds, check, variant, inject
+        self.calls, self._inj = 0, None
         dev = ds.x_ext.device
         world = ds.sh.world
         self.send = torch.zeros(3, dtype=torch.float64, device=dev)
@@ -265,7 +268,7 @@ class DistPcg:
 
     def begin(self, b, x, n_global, tol=1e-6, max_iter=0, res_hist=None, diag=None):
         mi = max_iter if max_iter > 0 else 10 * n_global
-        self.x, self.mi = x, mi
+        self.x, self.mi, self.calls = x, mi, 0
         self.ds.h.pcg_dist_begin(b, x, self.ds.own(), self.ds.y, diag, tol, mi, self.check,
                                  res_hist)
         self.ds.own().copy_(x)  # the first SpMV operand is x0
@@ -274,15 +277,19 @@ class DistPcg:
     # -- the phases, each rank's half of one exchange --------------------------
     def spmv_local(self, comm):
         """Steps 1-3 of the SpMV (halo + fused pass); returns the beta partial
-        to gather (None for the unprotected baseline)."""
+        to gather (None for the unprotected baseline).  With `inject` set
+        (a function of the solve's SpMV call index -> Inject or None), the
+        call's faults go into the protected pass and its correction rounds."""
+        self._inj = self.inject(self.calls) if self.inject is not None else None
+        self.calls += 1
         if not self.check:
             self.ds.plain(comm)
             return None
-        return self.ds.step1(comm)
+        return self.ds.step1(comm, self._inj)
 
     def spmv_finish(self):
         if self.check:
-            self.ds.step2()
+            self.ds.step2(None, self._inj)
 
     def local(self, phase, it=0):
         from .abft import PCG_PHASE_P

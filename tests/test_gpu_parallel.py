@@ -103,11 +103,15 @@ def make_shards(A, ranges):
     return shards
 
 
-def run_dist_pcg(torch, A, ranges, b, x0, check=True, tol=1e-6, max_iter=0, variant="pcg"):
+def run_dist_pcg(torch, A, ranges, b, x0, check=True, tol=1e-6, max_iter=0, variant="pcg",
+                 lam=0.0):
     shards = make_shards(A, ranges)
     ds = [PL.DistSpmv(sh) for sh in shards]
     comm = PL.LocalComm(shards, {d.sh.rank: d.x_ext for d in ds})
-    pcgs = [PL.DistPcg(d, check, variant) for d in ds]
+    from paper_conf_dsn_schollbkw16_b200 import Inject
+    inj = (lambda r: (lambda call: Inject.rate(seed=100 + r, lam=lam, call=call))) if lam else \
+        (lambda r: None)
+    pcgs = [PL.DistPcg(d, check, variant, inj(d.sh.rank)) for d in ds]
     mi = max_iter if max_iter > 0 else 10 * A.n
     dev = lambda v: torch.from_numpy(np.ascontiguousarray(v)).cuda()
     bs = [dev(b[sh.row0:sh.row1]) for sh in shards]
@@ -277,3 +281,23 @@ def test_dist_cg1_maxiter(O, torch_cuda):
     assert ref.status == -5 and st == 3 and sts[0][1]["iters"] == ref.iters == 5
     assert np.array_equal(hist.view(np.uint64), ref.res_hist.view(np.uint64))
     assert np.array_equal(x.view(np.uint64), ref.x.view(np.uint64))
+
+
+@pytest.mark.parametrize("variant", ["pcg", "cg1"])
+def test_dist_pcg_under_faults(O, torch_cuda, variant):
+    """Rate-mode faults (lambda per arithmetic op) in every rank's
+    protected SpMVs: the solve still converges, faults are flagged and
+    corrected (none left uncorrected), and the solution solves A x = b."""
+    A = G.laplacian_3d_7pt(24)
+    ranges = [(0, 4608), (4608, 9216), (9216, A.n)]
+    b = O.spmv(A, G.uniform_vector(A.n, 43))
+    x0 = G.uniform_vector(A.n, 44)
+    st, x, hist, sts = run_dist_pcg(torch_cuda, A, ranges, b, x0, True, variant=variant,
+                                    lam=1e-5)
+    assert st == 1
+    assert sum(s[1]["flagged_blocks"] for s in sts) > 0
+    assert all(s[1]["uncorrected_calls"] == 0 for s in sts)
+    ref = (O.pcg_cg1_ranks if variant == "cg1" else O.pcg_ranks)(A, b, x0, ranges, tol=1e-6)
+    assert abs(sts[0][1]["iters"] - ref.iters) <= 2
+    rel = np.linalg.norm(b - O.spmv(A, x)) / np.linalg.norm(b)
+    assert rel <= 1e-5

@@ -273,10 +273,7 @@ def _gloo_pcg_worker(rank, world, port, variant, q):
         comm = PL.TorchDistComm()
         PL.plan_from_needs(sh, comm.gather_needs(sh))
         ds = _FakeDs(O, sh)
-        p = PL.DistPcg.__new__(PL.DistPcg)
-        p.ds, p.check, p.variant = ds, False, variant
-        p.send = torch.zeros(3, dtype=torch.float64)
-        p.recv = torch.zeros(3 * world, dtype=torch.float64)
+        p = PL.DistPcg(ds, False, variant)
         bfull = O.spmv(A, G.uniform_vector(A.n, 43))
         b = torch.from_numpy(bfull[a:b_].copy())
         x = torch.from_numpy(G.uniform_vector(A.n, 44)[a:b_].copy())
