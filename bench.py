@@ -342,7 +342,15 @@ def run_pcg_dist(args):
     for lam in ((1e-8, 1e-6) if args.lam <= 0 else (args.lam,)):
         schemes += [(f"protected_lam{lam:g}", True, "pcg", lam),
                     (f"protected_cg1_lam{lam:g}", True, "cg1", lam)]
+    # CUDA-graph replay of 16-iteration batches, on request (ABFT_PCG_GRAPH=1;
+    # NCCL capture untested on this pool).  Measured at N = 1 it did not beat
+    # host sequencing (capture + instantiate per solve).
+    graph = os.environ.get("ABFT_PCG_GRAPH") == "1"
+    if graph:
+        schemes += [("unprotected_eager", False, "pcg", -1.0), ("protected_eager", True, "pcg", -1.0)]
     for name, check, variant, lam in schemes:
+        eager = lam < 0
+        lam = max(lam, 0.0)
         # rate-mode faults per arithmetic op in every rank's SpMVs
         inj = (lambda call, lam=lam: Inject.rate(seed=1000 * rank + 7, lam=lam, call=call)) \
             if lam > 0 else None
@@ -354,7 +362,8 @@ def run_pcg_dist(args):
             torch.cuda.synchronize()
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record()
-            state, st = p.solve(c, b, x, n_glob, tol=1e-6)
+            state, st = p.solve(c, b, x, n_glob, tol=1e-6,
+                                graph=graph and lam == 0 and not eager)
             e1.record()
             torch.cuda.synchronize()
             barrier(world)
@@ -367,7 +376,8 @@ def run_pcg_dist(args):
                      "uncorrected_calls_rank0": st["uncorrected_calls"]}
     for k, v in res.items():
         if k.startswith("protected"):
-            base = res["unprotected_cg1" if "cg1" in k else "unprotected"]["ms"]
+            base = res["unprotected_cg1" if "cg1" in k else
+                       ("unprotected_eager" if "eager" in k else "unprotected")]["ms"]
             v["overhead_pct"] = round((v["ms"] / base - 1) * 100, 2)
     if rank == 0:
         print(json.dumps({"metric": "PCG time-to-solution (ms), Jacobi, tol 1e-6, sharded",
@@ -377,6 +387,8 @@ def run_pcg_dist(args):
                           "variants": "pcg = textbook (2 reductions + SpMV beta gather per "
                                       "iteration); cg1 = single reduction (Chronopoulos-Gear, "
                                       "1 reduction + SpMV beta gather, one extra SpMV)",
+                          "graph": "fault-free schemes replay a CUDA graph of 16 iterations "
+                                   "(*_eager: host-sequenced)" if graph else "none",
                           "backend": os.environ.get("ABFT_DIST_BACKEND", "nccl") if world > 1
                           else "none", "results": res}), flush=True)
 

@@ -173,15 +173,16 @@ class LocalComm:
     def __init__(self, shards, xs):
         self.shards = {s.rank: s for s in shards}
         self.xs = xs  # rank -> x_ext tensor
+        self._idx = {}  # device index lists, uploaded once (graph capture safe)
 
     def halo(self, sh: Shard, x_ext) -> None:
+        import torch
         for q, (start, count) in sh.recv.items():
-            owner = self.shards[q]
-            idx = owner.send[sh.rank]
             src = self.xs[q]
-            import torch
-            x_ext[start:start + count] = src.index_select(
-                0, torch.as_tensor(idx, device=src.device))
+            key = (q, sh.rank, src.device)
+            if key not in self._idx:
+                self._idx[key] = torch.as_tensor(self.shards[q].send[sh.rank], device=src.device)
+            x_ext[start:start + count] = src.index_select(0, self._idx[key])
 
 
 # ---------------------------------------------------------------------------
@@ -303,13 +304,15 @@ class DistPcg:
         return self.ds.h.pcg_dist_status()
 
     # -- the iteration, over any exchange ------------------------------------
-    def run(self, spmv, reduce, local, status, mi, poll=16):
+    def run(self, spmv, reduce, local, status, mi, poll=16, graph=False):
         """Sequence one solve (after begin).  spmv(): the distributed SpMV of
         the operand's own slice into ds.y; reduce(phases): run each
         (phase, it) local kernel, gather the send slots, combine the last
         phase; local(phase, it): a kernel without a reduction; status():
         (state, stats).  variant "pcg": standard (two reductions per
-        iteration); "cg1": single reduction (Chronopoulos-Gear, R29)."""
+        iteration); "cg1": single reduction (Chronopoulos-Gear, R29).
+        graph: capture `poll` iterations once and replay them (fault-free
+        solves; every call in an iteration must be capturable)."""
         from .abft import (PCG_PHASE_CG1_DOT, PCG_PHASE_CG1_UPDATE, PCG_PHASE_DOT,
                            PCG_PHASE_INIT, PCG_PHASE_P, PCG_PHASE_UPDATE)
         spmv()
@@ -317,13 +320,8 @@ class DistPcg:
         if self.variant == "cg1":
             spmv()  # w_0 = A u_0
             reduce([(PCG_PHASE_CG1_DOT, 0)])
-        j = 0
-        while True:
-            state = status()
-            if state[0] != 0 or j >= mi:
-                return state
-            for _ in range(min(poll, mi - j)):
-                j += 1
+        def batch(j0, count):
+            for j in range(j0 + 1, j0 + count + 1):
                 if self.variant == "cg1":
                     local(PCG_PHASE_CG1_UPDATE, j)
                     spmv()  # w = A u
@@ -334,9 +332,32 @@ class DistPcg:
                     reduce([(PCG_PHASE_UPDATE, j)])
                     local(PCG_PHASE_P, j)
 
+        j, g = 0, None
+        while True:
+            state = status()
+            if state[0] != 0 or j >= mi:
+                return state
+            if graph and mi - j >= poll:
+                # One CUDA graph of `poll` iterations, replayed until the
+                # device state leaves RUN.  The baked iteration indices
+                # 1..poll only pair each update with its p step (upd ==
+                # iter); kernels of a finished solve are no-ops and the host
+                # never replays after one, so reuse is exact.
+                if g is None:
+                    import torch
+                    g = torch.cuda.CUDAGraph()
+                    with torch.cuda.graph(g):
+                        batch(0, poll)
+                g.replay()
+                j += poll
+            else:
+                n = min(poll, mi - j)
+                batch(j, n)
+                j += n
+
     # -- driver over torch.distributed (one process per GPU) -----------------
     def solve(self, comm: TorchDistComm, b, x, n_global, tol=1e-6, max_iter=0, res_hist=None,
-              diag=None, poll=16):
+              diag=None, poll=16, graph=False):
         def spmv():
             part = self.spmv_local(comm)
             if part is not None:
@@ -349,12 +370,14 @@ class DistPcg:
             comm.gather_partials(self.send, self.recv)
             self.combine(*phases[-1])
 
+        if graph and self.inject is not None:
+            raise ValueError("graph replay needs a fault-free solve (per-call fault plans)")
         mi = self.begin(b, x, n_global, tol, max_iter, res_hist, diag)
-        return self.run(spmv, reduce, self.local, self.status, mi, poll)
+        return self.run(spmv, reduce, self.local, self.status, mi, poll, graph)
 
 
 def pcg_lockstep(pcgs, comm: LocalComm, bs, xs, n_global, tol=1e-6, max_iter=0, hists=None,
-                 poll=16):
+                 poll=16, graph=False):
     """Logical ranks in one process (tests): every phase runs on all ranks,
     then the partials are concatenated in rank order -- the exchange pattern
     of DistPcg.solve without a process group.  Rank 0's DistPcg.run sequences
@@ -386,5 +409,5 @@ def pcg_lockstep(pcgs, comm: LocalComm, bs, xs, n_global, tol=1e-6, max_iter=0, 
     mi = 0
     for p, b, x, h in zip(pcgs, bs, xs, hists):
         mi = p.begin(b, x, n_global, tol, max_iter, h)
-    pcgs[0].run(spmv, reduce, local, pcgs[0].status, mi, poll)
+    pcgs[0].run(spmv, reduce, local, pcgs[0].status, mi, poll, graph)
     return [p.status() for p in pcgs]

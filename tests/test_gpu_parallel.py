@@ -104,7 +104,7 @@ def make_shards(A, ranges):
 
 
 def run_dist_pcg(torch, A, ranges, b, x0, check=True, tol=1e-6, max_iter=0, variant="pcg",
-                 lam=0.0):
+                 lam=0.0, graph=False):
     shards = make_shards(A, ranges)
     ds = [PL.DistSpmv(sh) for sh in shards]
     comm = PL.LocalComm(shards, {d.sh.rank: d.x_ext for d in ds})
@@ -117,7 +117,7 @@ def run_dist_pcg(torch, A, ranges, b, x0, check=True, tol=1e-6, max_iter=0, vari
     bs = [dev(b[sh.row0:sh.row1]) for sh in shards]
     xs = [dev(x0[sh.row0:sh.row1]) for sh in shards]
     hists = [torch.zeros(mi + 1, dtype=torch.float64, device="cuda") for _ in shards]
-    sts = PL.pcg_lockstep(pcgs, comm, bs, xs, A.n, tol, max_iter, hists)
+    sts = PL.pcg_lockstep(pcgs, comm, bs, xs, A.n, tol, max_iter, hists, graph=graph)
     torch.cuda.synchronize()
     x = np.concatenate([v.cpu().numpy() for v in xs])
     it = sts[0][1]["iters"]
@@ -301,3 +301,23 @@ def test_dist_pcg_under_faults(O, torch_cuda, variant):
     assert abs(sts[0][1]["iters"] - ref.iters) <= 2
     rel = np.linalg.norm(b - O.spmv(A, x)) / np.linalg.norm(b)
     assert rel <= 1e-5
+
+
+@pytest.mark.parametrize("variant", ["pcg", "cg1"])
+@pytest.mark.parametrize("check", [True, False])
+def test_dist_pcg_graph_replay(O, torch_cuda, variant, check):
+    """CUDA-graph replay of 16-iteration batches == the oracle bit for bit
+    (2 logical ranks; max_iter not a multiple of the batch: the tail runs
+    eagerly)."""
+    A = G.laplacian_3d_7pt(24)
+    ranges = PL.block_partition(A.n, 2)
+    b = O.spmv(A, G.uniform_vector(A.n, 43))
+    x0 = G.uniform_vector(A.n, 44)
+    f = O.pcg_cg1_ranks if variant == "cg1" else O.pcg_ranks
+    for mi in (0, 37):
+        ref = f(A, b, x0, ranges, tol=1e-6, max_iter=mi)
+        st, x, hist, sts = run_dist_pcg(torch_cuda, A, ranges, b, x0, check, max_iter=mi,
+                                        variant=variant, graph=True)
+        assert sts[0][1]["iters"] == ref.iters
+        assert np.array_equal(hist.view(np.uint64), ref.res_hist.view(np.uint64))
+        assert np.array_equal(x.view(np.uint64), ref.x.view(np.uint64))
