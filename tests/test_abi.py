@@ -79,3 +79,16 @@ def test_encode_rejects_bad_args_without_gpu(L):
     assert L.abft_encode(C.byref(csr), 3, 4, 0, None, C.byref(h)) == abft.EINVAL
     assert L.abft_encode(C.byref(csr), 2048, 4, 0, None, C.byref(h)) == abft.ENOTSUP
     assert L.abft_spmv(None, None, None, None, None, 1, None) == abft.EINVAL
+
+
+def test_pcg_dist_rejects_bad_args_without_gpu(L):
+    # include/abft.h: a NULL handle (or a handle without _begin) is EINVAL;
+    # nothing touches the device before the checks
+    from paper_conf_dsn_schollbkw16_b200 import abft
+    L_ = abft.lib()
+    assert L_.abft_pcg_dist_begin(None, None, None, None, None, None, 1e-6, 10, 1, None,
+                                  None) == abft.EINVAL
+    for phase in (abft.PCG_PHASE_INIT, abft.PCG_PHASE_CG1_DOT, 9):
+        assert L_.abft_pcg_dist_local(None, phase, 0, None, None) == abft.EINVAL
+        assert L_.abft_pcg_dist_combine(None, phase, 0, None, 2, None) == abft.EINVAL
+    assert L_.abft_pcg_dist_status(None, None, None, None) == abft.EINVAL
