@@ -344,10 +344,19 @@ class DistPcg:
                 # iter); kernels of a finished solve are no-ops and the host
                 # never replays after one, so reuse is exact.
                 if g is None:
+                    # capture_begin/end directly: torch.cuda.graph() would
+                    # also run gc.collect() + empty_cache() on every solve
                     import torch
                     g = torch.cuda.CUDAGraph()
-                    with torch.cuda.graph(g):
-                        batch(0, poll)
+                    cs = torch.cuda.Stream()
+                    cs.wait_stream(torch.cuda.current_stream())
+                    with torch.cuda.stream(cs):
+                        g.capture_begin()
+                        try:
+                            batch(0, poll)
+                        finally:
+                            g.capture_end()
+                    torch.cuda.current_stream().wait_stream(cs)
                 g.replay()
                 j += poll
             else:
