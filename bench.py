@@ -342,10 +342,10 @@ def run_pcg_dist(args):
     for lam in ((1e-8, 1e-6) if args.lam <= 0 else (args.lam,)):
         schemes += [(f"protected_lam{lam:g}", True, "pcg", lam),
                     (f"protected_cg1_lam{lam:g}", True, "cg1", lam)]
-    # CUDA-graph replay of 16-iteration batches, on request (ABFT_PCG_GRAPH=1;
-    # NCCL capture untested on this pool).  Measured at N = 1 it did not beat
-    # host sequencing (capture + instantiate per solve).
-    graph = os.environ.get("ABFT_PCG_GRAPH") == "1"
+    # CUDA-graph replay of 16-iteration batches, cached across solves on the
+    # same buffers: default at N = 1; at N > 1 on request (ABFT_PCG_GRAPH=1:
+    # NCCL capture is untested on this one-GPU pool).  DESIGN.md §8.
+    graph = os.environ.get("ABFT_PCG_GRAPH", "1" if world == 1 else "0") == "1"
     if graph:
         schemes += [("unprotected_eager", False, "pcg", -1.0), ("protected_eager", True, "pcg", -1.0)]
     for name, check, variant, lam in schemes:
@@ -356,8 +356,9 @@ def run_pcg_dist(args):
             if lam > 0 else None
         p = PL.DistPcg(d, check, variant, inj)
         times = []
-        for rep in range(max(1, args.pcg_reps) + 1):  # first: warm-up
-            x = x0.clone()
+        x = torch.empty_like(x0)  # one solution buffer: a captured graph is reused
+        for rep in range(max(1, args.pcg_reps) + 1):  # first: warm-up (and graph capture)
+            x.copy_(x0)
             barrier(world)
             torch.cuda.synchronize()
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -387,8 +388,9 @@ def run_pcg_dist(args):
                           "variants": "pcg = textbook (2 reductions + SpMV beta gather per "
                                       "iteration); cg1 = single reduction (Chronopoulos-Gear, "
                                       "1 reduction + SpMV beta gather, one extra SpMV)",
-                          "graph": "fault-free schemes replay a CUDA graph of 16 iterations "
-                                   "(*_eager: host-sequenced)" if graph else "none",
+                          "graph": "fault-free schemes replay a CUDA graph of 16 iterations, "
+                                   "captured in the warm-up solve and reused (*_eager: "
+                                   "host-sequenced)" if graph else "none",
                           "backend": os.environ.get("ABFT_DIST_BACKEND", "nccl") if world > 1
                           else "none", "results": res}), flush=True)
 

@@ -321,3 +321,33 @@ def test_dist_pcg_graph_replay(O, torch_cuda, variant, check):
         assert sts[0][1]["iters"] == ref.iters
         assert np.array_equal(hist.view(np.uint64), ref.res_hist.view(np.uint64))
         assert np.array_equal(x.view(np.uint64), ref.x.view(np.uint64))
+
+
+def test_dist_pcg_graph_reuse(O, torch_cuda):
+    """A second solve on the same buffers replays the cached graph and gives
+    the same bits (x reset to x0 between solves)."""
+    torch = torch_cuda
+    A = G.laplacian_3d_7pt(20)
+    b = O.spmv(A, G.uniform_vector(A.n, 43))
+    x0 = G.uniform_vector(A.n, 44)
+    ref = O.pcg_ranks(A, b, x0, [(0, A.n)], tol=1e-6)
+    (sh,) = make_shards(A, [(0, A.n)])
+    d = PL.DistSpmv(sh)
+    p = PL.DistPcg(d, True)
+
+    class Solo:
+        def gather_partials(self, part, out):
+            out.copy_(part)
+
+        def halo(self, s_, x_ext):
+            pass
+
+    bd = torch.from_numpy(b).cuda()
+    xd = torch.empty(A.n, dtype=torch.float64, device="cuda")
+    for rep in range(3):
+        xd.copy_(torch.from_numpy(x0))
+        state, st = p.solve(Solo(), bd, xd, A.n, tol=1e-6, graph=True)
+        torch.cuda.synchronize()
+        assert state == 1 and st["iters"] == ref.iters
+        assert np.array_equal(xd.cpu().numpy().view(np.uint64), ref.x.view(np.uint64))
+    assert p._graph is not None
