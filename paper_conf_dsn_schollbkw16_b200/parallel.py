@@ -388,8 +388,8 @@ class DistPcg:
         mi = self.begin(b, x, n_global, tol, max_iter, res_hist, diag)
         # the captured launches bake every pointer and the handle's argument
         # block: a later solve on the same buffers may replay the same graph
-        key = tuple(None if t is None else t.data_ptr() for t in (b, x, res_hist, diag)) + (
-            tol, mi, poll)
+        key = (tuple(None if t is None else t.data_ptr() for t in (b, x, res_hist, diag)) +
+               (tol, mi, poll)) if graph else None
         return self.run(spmv, reduce, self.local, self.status, mi, poll, graph, key)
 
 
