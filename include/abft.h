@@ -75,13 +75,20 @@ typedef struct abft_ctx *abft_handle_t;
  *        list_index[e] of target list_target[e] (0 = y row, 1 = t1 block,
  *        2 = t2 block) in round list_round[e] (0 = main pass, r >= 1 = r-th
  *        correction round).  The list arrays are HOST arrays, copied.
- *  RATE: every produced value is faulty with probability
- *        p = min(1, lambda * ops) (ops: 2*len(row) for y_i, 2*n_k for t1_k,
- *        rows-in-block for t2_k), decided by Philox4x32-10 with counter
- *        {index lo, index hi, call, round<<8 | target} and key {seed lo, seed
- *        hi}: faulty iff word0 < floor(p * 2^32); the burst starts at bit
- *        (word1 & 63) and its length is drawn from word2 through the table of
- *        abft_burst_table (R12/R13). */
+ *  RATE: the paper's Poisson process with rate lambda per arithmetic
+ *        operation (R13).  The call's operations are
+ *        numbered y first (2 per A entry, row order), then t1 (2 per C
+ *        entry, block order), then t2 (1 per row), and cut into chunks of
+ *        CH = abft_rate_chunk(lambda) operations.  Chunk c of round r draws
+ *        its event count from the Poisson(lambda * len) CDF table of
+ *        abft_poisson_table with Philox4x32-10 (key {seed lo, seed hi},
+ *        counter {c, 0, call, r<<8 | 0x80}) word 0; event e takes its offset
+ *        floor(w0 * len / 2^32) and its burst from counter {c, e, call,
+ *        r<<8 | 0x40}: start bit w1 & 63, length from w2 through the table of
+ *        abft_burst_table.  An event hits the element its operation produces
+ *        (row of y, block of t1 / t2); events on one element compose by XOR.
+ *        `targets` masks the targets that receive events.  The plan is built
+ *        on the device (5 short launches) by every call that injects. */
 enum { ABFT_INJ_NONE = 0, ABFT_INJ_LIST = 1, ABFT_INJ_RATE = 2 };
 enum { ABFT_TARGET_Y = 0, ABFT_TARGET_T1 = 1, ABFT_TARGET_T2 = 2 };
 typedef struct {
@@ -312,8 +319,10 @@ abft_status abft_pcg_dist_status(abft_handle_t h, int32_t *state, abft_pcg_stats
  * tau = K35 ||x||_2, K35 = ((n + 2N - 2) PW_i ||a_i||_2 + n ||c||_2) 2^-53.
  * A flag under ABFT_AUTOCORRECT recomputes ALL of y and re-checks, at most
  * max_rounds times (complete recomputation).  Square handles only
- * (ABFT_ENOTSUP for shards); list injection only (target 1 / 2 index 0 = t1 /
- * t2; rate mode: ABFT_ENOTSUP).
+ * (ABFT_ENOTSUP for shards).  List injection: target 0 = y row, target 1 / 2
+ * index 0 = t1 / t2 of the check.  Rate mode: the plan of R13 over the
+ * SpMV's y operations of round 0 only (the 3N operations of the check are not
+ * injected; R25).
  * abft_dense_encode: builds c and K35 on the device (owned by the handle;
  *   temporaries of ~17 B per nonzero during the call); synchronises.
  * abft_spmv_dense: the method's SpMV kernels with the check off, then one
@@ -332,6 +341,16 @@ abft_status abft_dense_checksum(abft_handle_t h, const double **c);
 
 abft_status abft_destroy(abft_handle_t h);
 
+/* Device-side health of a handle.  The finish / correction and dense-check
+ * kernels synchronise their CTAs with a software grid barrier that needs all
+ * CTAs (one per SM) co-resident; when other work holds SMs the barrier times
+ * out after about a second instead of hanging, and the calls that hit it
+ * leave incomplete results.  abft_health synchronises
+ * `stream`, sets *err = 1 if a barrier timed out since the last call (else
+ * 0) and then clears the error word and resets the barrier.  abft_pcg checks
+ * it before returning (ABFT_ECUDA on a timeout). */
+abft_status abft_health(abft_handle_t h, void *stream, int32_t *err);
+
 /* Plumbing for bindings: cudaMemcpyAsync(dst, src, bytes, cudaMemcpyDefault)
  * on `stream`, then synchronise it.  Used to read the device-resident results
  * above (flags, counts, C, K, beta) without a second CUDA binding. */
@@ -340,10 +359,16 @@ abft_status abft_memcpy(void *dst, const void *src, int64_t bytes, void *stream)
 /* Host helpers (no GPU needed). */
 const char *abft_status_string(abft_status st);
 const char *abft_last_cuda_error(void);
-/* The burst-length table the device injector uses: T[l] = floor(2^32 *
- * P(L <= l)), L = max(1, round(3 + sqrt(2) Z)) (R12),
- * computed on the host with the C library's erfc. */
+/* Fault-model tables (R13), host only:
+ * abft_burst_table: T[l] = floor(2^32 P(L <= l)) for the burst length
+ *   L = max(1, round(3 + sqrt(2) Z)), from the C library's erfc.
+ * abft_poisson_table: the Poisson(mu) event-count CDF table of rate mode
+ *   (floor(2^32 F(k)), last entry 2^32); returns its length (<= cap), 0 on a
+ *   bad argument.
+ * abft_rate_chunk: operations per chunk of rate mode for lambda. */
 void abft_burst_table(uint64_t T[65]);
+int32_t abft_poisson_table(double mu, uint64_t *T, int32_t cap);
+int64_t abft_rate_chunk(double lambda);
 /* Library version string. */
 const char *abft_version(void);
 

@@ -266,7 +266,7 @@ uint64_t or_fault_mask(const or_inject *inj, int32_t round, int32_t target, int6
   uint64_t m = 0;
   for (int64_t e = 0; e < inj->n_list; ++e)
     if (inj->list_round[e] == round && inj->list_target[e] == target &&
-        inj->list_index[e] == index)
+        inj->list_index[e] == index && (!inj->list_call || (uint64_t)inj->list_call[e] == inj->call))
       m ^= inj->list_mask[e];
   return m;
 }

@@ -48,6 +48,8 @@ typedef struct {
   const int32_t *list_target;
   const int64_t *list_index;
   const uint64_t *list_mask;
+  const int64_t *list_call; /* list mode, nullable: entry e applies only to SpMV call
+                               list_call[e] (matched against `call`); NULL = every call */
 } or_inject;
 
 /* --- canonical pairwise sum (R2) --- */

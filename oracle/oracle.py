@@ -41,7 +41,8 @@ class _Inj(C.Structure):
     _fields_ = [("mode", C.c_int32), ("seed", C.c_uint64), ("call", C.c_uint64),
                 ("lambda_", C.c_double), ("targets", C.c_uint32), ("n_list", C.c_int64),
                 ("list_round", C.c_void_p), ("list_target", C.c_void_p),
-                ("list_index", C.c_void_p), ("list_mask", C.c_void_p)]
+                ("list_index", C.c_void_p), ("list_mask", C.c_void_p),
+                ("list_call", C.c_void_p)]
 
 
 def lib():
@@ -128,6 +129,10 @@ class Inject:
             s.n_list = len(self.plan)
             s.list_round, s.list_target, s.list_index, s.list_mask = [
                 _p(a).value for a in self._keep]
+            call = getattr(self.plan, "call", None)
+            if call is not None:  # per-call list (entry e only in SpMV call[e])
+                self._keep_call = np.ascontiguousarray(call, np.int64)
+                s.list_call = _p(self._keep_call).value
         else:
             s.n_list = 0
         return s

@@ -30,7 +30,7 @@ SYMBOLS = [
     "abft_dense_encode", "abft_spmv_dense", "abft_dense_result", "abft_dense_checksum",
     "abft_spmv_host_pipelined", "abft_host_alloc", "abft_host_free",
     "abft_pcg_dist_begin", "abft_pcg_dist_local", "abft_pcg_dist_combine",
-    "abft_pcg_dist_status",
+    "abft_pcg_dist_status", "abft_poisson_table", "abft_rate_chunk", "abft_health",
 ]
 PCG_PHASE_INIT, PCG_PHASE_DOT, PCG_PHASE_UPDATE, PCG_PHASE_P = 0, 1, 2, 3
 PCG_PHASE_CG1_UPDATE, PCG_PHASE_CG1_DOT = 4, 5  # single-reduction variant
@@ -132,6 +132,10 @@ def lib():
         L.abft_status_string.argtypes = [st]
         L.abft_last_cuda_error.restype = C.c_char_p
         L.abft_burst_table.argtypes = [P]
+        L.abft_poisson_table.restype = i32
+        L.abft_poisson_table.argtypes = [d, P, i32]
+        L.abft_rate_chunk.restype = i64
+        L.abft_rate_chunk.argtypes = [d]
         L.abft_version.restype = C.c_char_p
         L.abft_info.restype = st
         L.abft_info.argtypes = [P, C.POINTER(Info)]
@@ -152,6 +156,8 @@ def lib():
         L.abft_dense_checksum.restype = st
         L.abft_dense_checksum.argtypes = [P, C.POINTER(P)]
         L.abft_finish.restype = st
+        L.abft_health.restype = st
+        L.abft_health.argtypes = [P, P, C.POINTER(i32)]
         L.abft_finish.argtypes = [P, P, P, P, i32, i32, P, P]
         _LIB = L
     return _LIB
@@ -172,10 +178,38 @@ def _ptr(t):
     return None if t is None else C.c_void_p(t.data_ptr())
 
 
+def _vec(t, min_len, what, optional=False):
+    """Device pointer of a float64 tensor the library reads or writes:
+    the C ABI only sees raw pointers, so dtype, device, contiguity and length
+    are checked here (ValueError instead of an out-of-bounds access)."""
+    if t is None:
+        if optional:
+            return None
+        raise ValueError(f"{what}: tensor required")
+    import torch
+    if not isinstance(t, torch.Tensor) or not t.is_cuda or t.dtype != torch.float64:
+        raise ValueError(f"{what}: expected a CUDA float64 tensor")
+    if not t.is_contiguous():
+        raise ValueError(f"{what}: tensor must be contiguous")
+    if t.numel() < min_len:
+        raise ValueError(f"{what}: {t.numel()} elements, need >= {min_len}")
+    return C.c_void_p(t.data_ptr())
+
+
 def burst_table() -> np.ndarray:
     t = np.zeros(65, dtype=np.uint64)
     lib().abft_burst_table(t.ctypes.data_as(C.c_void_p))
     return t
+
+
+def poisson_table(mu: float, cap: int = 1024) -> np.ndarray:
+    t = np.zeros(cap, dtype=np.uint64)
+    k = lib().abft_poisson_table(mu, t.ctypes.data_as(C.c_void_p), cap)
+    return t[:k].copy()
+
+
+def rate_chunk(lam: float) -> int:
+    return int(lib().abft_rate_chunk(lam))
 
 
 class Inject:
@@ -242,6 +276,7 @@ class Handle:
                  c_csr: bool = False):
         self.A = A
         self.n = A.n
+        self.n_cols = A.n_cols if A.n_cols > 0 else A.n
         self.block_size = block_size
         self.nb = (A.n + block_size - 1) // block_size
         self.max_rounds = max_rounds if max_rounds > 0 else 4
@@ -252,6 +287,12 @@ class Handle:
                                  ENCODE_C_CSR if c_csr else 0, _stream(stream), C.byref(h)),
                "abft_encode")
         self._h = h
+
+    def health(self, stream=None) -> int:
+        """1 if a grid barrier timed out since the last call (abft_health)."""
+        e = C.c_int32(0)
+        _check(lib().abft_health(self._h, _stream(stream), C.byref(e)), "abft_health")
+        return e.value
 
     def info(self) -> dict:
         inf = Info()
@@ -273,9 +314,11 @@ class Handle:
     def spmv(self, x, y=None, x_norm=None, inject: Inject | None = None, mode=CHECK, stream=None):
         import torch
         if y is None:
-            y = torch.empty_like(x)
+            y = torch.empty(self.n, dtype=torch.float64, device=x.device)
+        px, py = _vec(x, self.n_cols, "x"), _vec(y, self.n, "y")
+        pn = _vec(x_norm, 1, "x_norm", optional=True)
         inj = inject.struct() if inject is not None else None
-        _check(lib().abft_spmv(self._h, _ptr(x), _ptr(y), _ptr(x_norm),
+        _check(lib().abft_spmv(self._h, px, py, pn,
                                C.byref(inj) if inj is not None else None, mode, _stream(stream)),
                "abft_spmv")
         return y
@@ -283,7 +326,8 @@ class Handle:
     def beta_partial(self, out, stream=None):
         """Enqueue this shard's PW sum of x_i^2 (after a DEFER_FINISH spmv)
         into the device f64 tensor `out` (one element)."""
-        _check(lib().abft_beta_partial(self._h, _ptr(out), _stream(stream)), "abft_beta_partial")
+        _check(lib().abft_beta_partial(self._h, _vec(out, 1, "out"), _stream(stream)),
+               "abft_beta_partial")
         return out
 
     def finish(self, x, y, parts, rounds=None, inject: Inject | None = None, stream=None):
@@ -291,14 +335,16 @@ class Handle:
         the per-rank partials in rank order)."""
         inj = inject.struct() if inject is not None else None
         r = self.max_rounds if rounds is None else rounds
-        _check(lib().abft_finish(self._h, _ptr(x), _ptr(y), _ptr(parts), int(parts.numel()), r,
+        _check(lib().abft_finish(self._h, _vec(x, self.n_cols, "x"), _vec(y, self.n, "y"),
+                                 _vec(parts, 1, "parts"), int(parts.numel()), r,
                                  C.byref(inj) if inj is not None else None, _stream(stream)),
                "abft_finish")
         return y
 
     def correct(self, x, y, max_rounds=0, inject: Inject | None = None, stream=None):
         inj = inject.struct() if inject is not None else None
-        _check(lib().abft_correct(self._h, _ptr(x), _ptr(y), max_rounds,
+        _check(lib().abft_correct(self._h, _vec(x, self.n_cols, "x"), _vec(y, self.n, "y"),
+                                  max_rounds,
                                   C.byref(inj) if inj is not None else None, _stream(stream)),
                "abft_correct")
         return y
@@ -379,10 +425,10 @@ class Handle:
                    stream=None):
         import torch
         if y is None:
-            y = torch.empty_like(x)
+            y = torch.empty(self.n, dtype=torch.float64, device=x.device)
         inj = inject.struct() if inject is not None else None
         mode = (AUTOCORRECT if correct else 0) | (DENSE_BOUND35 if bound35 else 0)
-        _check(lib().abft_spmv_dense(self._h, _ptr(x), _ptr(y),
+        _check(lib().abft_spmv_dense(self._h, _vec(x, self.n_cols, "x"), _vec(y, self.n, "y"),
                                      C.byref(inj) if inj is not None else None, mode,
                                      _stream(stream)), "abft_spmv_dense")
         return y
@@ -412,9 +458,12 @@ class Handle:
         st = PcgStats()
         inj = inject.struct() if inject is not None else None
         mode = 2 if check == "checkpoint" else (1 if check else 0)
-        status = lib().abft_pcg(self._h, _ptr(b), _ptr(x), _ptr(diag), tol, max_iter,
+        mi = max_iter if max_iter > 0 else 10 * self.n
+        status = lib().abft_pcg(self._h, _vec(b, self.n, "b"), _vec(x, self.n, "x"),
+                                _vec(diag, self.n, "diag", optional=True), tol, max_iter,
                                 C.byref(inj) if inj is not None else None, mode,
-                                _ptr(res_hist), C.byref(st), _stream(stream))
+                                _vec(res_hist, mi + 1, "res_hist", optional=True), C.byref(st),
+                                _stream(stream))
         if status not in (OK, ENOCONV, EBREAKDOWN):
             _check(status, "abft_pcg")
         return status, st.as_dict()

@@ -41,14 +41,46 @@ abft_status cuda_fail(cudaError_t e, const char *where) {
     if (s_ != ABFT_OK) return s_;         \
   } while (0)
 
-void host_burst_table(uint64_t T[65]) {
-  T[0] = 0;
-  for (int l = 1; l < 64; ++l) {
-    const double p = 0.5 * std::erfc(-((double)l - 2.5) / 2.0);
-    T[l] = (uint64_t)std::floor(std::ldexp(p, 32));
+// Integer CDF tables of the fault model, written from DESIGN.md R13's
+// definitions (the oracle implements the same definitions separately):
+//  * burst length L = max(1, round(3 + sqrt(2) Z)): entry l of the table is
+//    floor(2^32 P(L <= l)) = floor(2^32 Phi((l - 2.5) / sqrt 2)), with
+//    Phi(t) = erfc(-t / sqrt 2) / 2, i.e. erfc((2.5 - l) / 2) / 2; entry 0 is
+//    0 and entry 64 is 2^32 (L <= 64 always).  Scaling by 1/2 and 2^32 is
+//    exact, so truncating the product is the floor of the definition.
+//  * Poisson(mu) event counts: term_0 = e^-mu, term_k = (term_{k-1} mu) / k,
+//    F_k = F_{k-1} + term_k (in this order of binary64 operations); entry k is
+//    floor(2^32 min(F_k, 1)); the table ends at the first entry >= 2^32 - 1
+//    (or at cap), whose value is replaced by 2^32.
+//  * chunk length CH = 2^e, e = 24 lowered while lambda 2^e > 4 (and e > 0).
+struct FaultTables {
+  static constexpr double kTwo32 = 4294967296.0;
+  static void burst(uint64_t out[65]) {
+    out[0] = 0;
+    for (int len = 1; len < 64; ++len)
+      out[len] = (uint64_t)(std::erfc((2.5 - (double)len) * 0.5) * 0.5 * kTwo32);
+    out[64] = (uint64_t)1 << 32;
   }
-  T[64] = (uint64_t)1 << 32;
-}
+  static int poisson(double mu, uint64_t *out, int cap) {
+    const uint64_t one = (uint64_t)1 << 32;
+    double term = std::exp(-mu), cum = term;
+    for (int k = 0;; ++k) {
+      const uint64_t v = cum >= 1.0 ? one : (uint64_t)(cum * kTwo32);
+      if (v + 1 >= one || k + 1 == cap) {
+        out[k] = one;
+        return k + 1;
+      }
+      out[k] = v;
+      term = term * mu / (double)(k + 1);
+      cum = cum + term;
+    }
+  }
+  static int64_t chunk(double lambda) {
+    int e = 24;
+    while (e > 0 && lambda * std::ldexp(1.0, e) > 4.0) --e;
+    return (int64_t)1 << e;
+  }
+};
 
 int g_init_device = -1;  // device the burst table / kernel attributes were set up on
 
@@ -217,30 +249,7 @@ abft_status ensure_list(abft_ctx *h, int64_t need) {
 
 // Rate mode (R13): expand a Poisson process over the call's
 // arithmetic operations into a sorted fault list on the device (no host
-// sync).  The chunking and the CDF tables are computed here exactly as the
-// oracle computes them.
-int64_t rate_chunk(double lambda) {
-  int64_t ch = (int64_t)1 << 24;
-  while (ch > 1 && lambda * (double)ch > 4.0) ch /= 2;
-  return ch;
-}
-
-int poisson_table(double mu, uint64_t *T, int cap) {
-  double p = std::exp(-mu), cdf = p;
-  int k = 0;
-  for (;;) {
-    const double c = cdf < 1.0 ? cdf : 1.0;
-    T[k] = (uint64_t)std::floor(std::ldexp(c, 32));
-    if (T[k] >= ((uint64_t)1 << 32) - 1 || k == cap - 1) {
-      T[k] = (uint64_t)1 << 32;
-      return k + 1;
-    }
-    ++k;
-    p = p * mu / (double)k;
-    cdf = cdf + p;
-  }
-}
-
+// sync); the chunking and the CDF tables come from FaultTables.
 abft_status gen_rate_plan(abft_ctx *h, const abft_inject_t *inj, uint64_t call, bool check,
                           cudaStream_t s, InjDev *d) {
   RatePlanArgs r;
@@ -252,7 +261,7 @@ abft_status gen_rate_plan(abft_ctx *h, const abft_inject_t *inj, uint64_t call, 
   r.t1_ops = check ? 2 * h->nnz_c : 0;
   r.ops = r.y_ops + r.t1_ops + (check ? h->n : 0);
   r.rounds = check ? h->max_rounds : 0;
-  r.ch = rate_chunk(inj->lambda);
+  r.ch = FaultTables::chunk(inj->lambda);
   r.nch = std::max<int64_t>(1, (r.ops + r.ch - 1) / r.ch);
   r.key0 = (uint32_t)inj->seed;
   r.key1 = (uint32_t)(inj->seed >> 32);
@@ -261,8 +270,8 @@ abft_status gen_rate_plan(abft_ctx *h, const abft_inject_t *inj, uint64_t call, 
   r.rp = h->rp;
   r.crp = h->c_rp;
   uint64_t tab[2 * kRateTab];
-  r.nf = poisson_table(inj->lambda * (double)r.ch, tab, kRateTab);
-  r.nl = poisson_table(inj->lambda * (double)(r.ops - (r.nch - 1) * r.ch), tab + kRateTab, kRateTab);
+  r.nf = FaultTables::poisson(inj->lambda * (double)r.ch, tab, kRateTab);
+  r.nl = FaultTables::poisson(inj->lambda * (double)(r.ops - (r.nch - 1) * r.ch), tab + kRateTab, kRateTab);
   const int64_t slots = (int64_t)(r.rounds + 1) * r.nch;
   if (slots > (1ll << 30)) return ABFT_EINVAL;
   if (slots > h->plan_slots) {
@@ -555,7 +564,7 @@ int cf_size(int cf) {
 abft_status init_device_once(int device) {
   if (g_init_device == device) return ABFT_OK;
   uint64_t T[65];
-  host_burst_table(T);
+  FaultTables::burst(T);
   CK(cudaMemcpyToSymbol(c_burst_T, T, sizeof T));
   int optin = 0;
   CK(cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, device));
@@ -941,7 +950,14 @@ const char *abft_status_string(abft_status st) {
   return "unknown status";
 }
 
-void abft_burst_table(uint64_t T[65]) { host_burst_table(T); }
+void abft_burst_table(uint64_t T[65]) { FaultTables::burst(T); }
+
+int32_t abft_poisson_table(double mu, uint64_t *T, int32_t cap) {
+  if (!T || cap <= 0 || !(mu >= 0.0)) return 0;
+  return FaultTables::poisson(mu, T, cap);
+}
+
+int64_t abft_rate_chunk(double lambda) { return FaultTables::chunk(lambda); }
 
 abft_status abft_destroy(abft_handle_t h) {
   if (!h) return ABFT_EINVAL;
@@ -1067,7 +1083,7 @@ abft_status abft_encode(const abft_csr_t *A, int32_t block_size, int32_t max_rou
       (st = dalloc(h, &h->cand_s, (size_t)h->nb)) ||
       (st = dalloc(h, &h->flags, (size_t)(h->max_rounds + 1) * h->nb)) ||
       (st = dalloc(h, &h->n_flags, (size_t)h->max_rounds + 1)) || (st = dalloc(h, &h->beta, 1)) ||
-      (st = dalloc(h, &h->beta_valid, 1)) || (st = dalloc(h, &h->gbar, 2)) ||
+      (st = dalloc(h, &h->beta_valid, 1)) || (st = dalloc(h, &h->gbar, 4)) ||
       (st = dalloc(h, &h->bnorm, 2)) ||
       (st = dalloc(h, &h->dbg_t1, (size_t)h->nb)) || (st = dalloc(h, &h->dbg_t2, (size_t)h->nb)))
     return fail(st);
@@ -1075,7 +1091,7 @@ abft_status abft_encode(const abft_csr_t *A, int32_t block_size, int32_t max_rou
       (e = cudaMemsetAsync(h->n_flags, 0, sizeof(int32_t) * (h->max_rounds + 1), s)) ||
       (e = cudaMemsetAsync(h->beta, 0, sizeof(double), s)) ||
       (e = cudaMemsetAsync(h->beta_valid, 0, sizeof(int32_t), s)) ||
-      (e = cudaMemsetAsync(h->gbar, 0, 2 * sizeof(unsigned), s)) || (e = cudaStreamSynchronize(s)))
+      (e = cudaMemsetAsync(h->gbar, 0, 4 * sizeof(unsigned), s)) || (e = cudaStreamSynchronize(s)))
     return fail(cuda_fail(e, "scratch init"));
   if ((st = plan_fused(h, s)) != ABFT_OK) return fail(st);
   *out = h;
@@ -1217,6 +1233,10 @@ abft_status abft_spmv_host_pipelined(abft_handle_t h, const double *const *x_hos
                                      int32_t *n_flagged_hosts, uint32_t mode, void *stream) {
   if (!h || !x_hosts || !y_hosts || nsteps < 0) return ABFT_EINVAL;
   if (nsteps == 0) return ABFT_OK;
+  // every buffer is checked before any copy is queued: an early return must
+  // not leave copies in flight that read or write caller memory
+  for (int32_t k = 0; k < nsteps; ++k)
+    if (!x_hosts[k] || !y_hosts[k]) return ABFT_EINVAL;
   cudaStream_t s = (cudaStream_t)stream;
   if (!h->s_in) {
     for (int q = 0; q < 2; ++q) {
@@ -1244,7 +1264,6 @@ abft_status abft_spmv_host_pipelined(abft_handle_t h, const double *const *x_hos
   CK(cudaStreamWaitEvent(h->s_out, start, 0));
   for (int32_t k = 0; k < nsteps; ++k) {
     const int sl = k & 1;
-    if (!x_hosts[k] || !y_hosts[k]) return ABFT_EINVAL;
     // x_k -> slot (after step k-2's compute read it)
     if (k >= 2) CK(cudaStreamWaitEvent(h->s_in, h->ev_c[sl], 0));
     CK(cudaMemcpyAsync(h->px[sl], x_hosts[k], sizeof(double) * h->n_cols, cudaMemcpyHostToDevice,
@@ -1292,6 +1311,20 @@ abft_status abft_info(abft_handle_t h, abft_info_t *info) {
   info->lean_runs = h->lean_runs ? 1 : 0;
   info->lean = h->lean ? 1 : 0;
   info->max_rounds = h->max_rounds;
+  return ABFT_OK;
+}
+
+abft_status abft_health(abft_handle_t h, void *stream, int32_t *err) {
+  if (!h || !err) return ABFT_EINVAL;
+  cudaStream_t s = (cudaStream_t)stream;
+  unsigned w[3] = {0, 0, 0};
+  CK(cudaMemcpyAsync(w, h->gbar, sizeof w, cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  *err = w[2] != 0u ? 1 : 0;
+  if (w[2] != 0u) {  // reset the poisoned barrier (arrival count is stale)
+    CK(cudaMemsetAsync(h->gbar, 0, 4 * sizeof(unsigned), s));
+    CK(cudaStreamSynchronize(s));
+  }
   return ABFT_OK;
 }
 

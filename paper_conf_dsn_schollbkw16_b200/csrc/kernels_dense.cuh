@@ -275,7 +275,7 @@ __global__ void __launch_bounds__(256) k_dense(const DenseArgs d) {
   for (int r = 0; r <= d.rounds; ++r) {
     if (r > 0) {
       dense_recompute<INJECT>(a, r);
-      grid_sync(a.gbar);
+      if (!grid_sync(a.gbar)) return;
     }
     for (int64_t ch = blockIdx.x; ch < nch; ch += gridDim.x) {
       double o[3];
@@ -283,7 +283,7 @@ __global__ void __launch_bounds__(256) k_dense(const DenseArgs d) {
       if (threadIdx.x == 0)
         for (int k = 0; k < 3; ++k) d.part[k * nch + ch] = o[k];
     }
-    grid_sync(a.gbar);
+    if (!grid_sync(a.gbar)) return;
     // every CTA finishes the totals itself (same bits everywhere)
     const double t2raw = cta_pw_array(d.part, nch, s_red);
     const double t1raw = cta_pw_array(d.part + nch, nch, s_red);
@@ -305,7 +305,7 @@ __global__ void __launch_bounds__(256) k_dense(const DenseArgs d) {
       d.flag_rounds[r] = flagged ? 1 : 0;
     }
     if (!flagged) break;
-    grid_sync(a.gbar);  // partials consumed before the next round rewrites them
+    if (!grid_sync(a.gbar)) return;  // partials consumed before the next round rewrites them
   }
 }
 

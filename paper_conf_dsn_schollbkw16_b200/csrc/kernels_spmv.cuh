@@ -1333,25 +1333,43 @@ __device__ __forceinline__ double big_block(const SpmvArgs &a, int64_t k, int ro
   return dsub(t1, t2);
 }
 
-// Software grid barrier (all CTAs co-resident: grid <= SM count).
-// bar[0] = arrivals, bar[1] = generation.
-__device__ __forceinline__ void grid_sync(unsigned *bar) {
+// Software grid barrier (all CTAs co-resident: grid <= SM count, one CTA per
+// SM, checked against the occupancy at encode).  bar[0] = arrivals, bar[1] =
+// generation, bar[2] = error word.  Co-residency is not guaranteed when other
+// work holds SMs (another process, MPS limits, kernels on other streams), so
+// the wait is bounded: after ~2^24 polls (about a second) the barrier sets
+// bar[2] = 1 and every CTA returns false; a set error word makes every later
+// barrier fail at once (the handle is poisoned until abft_health clears it),
+// so a co-residency failure is reported instead of hanging the device.
+__device__ __forceinline__ bool grid_sync(unsigned *bar) {
+  __shared__ int s_ok;
   __syncthreads();
   if (threadIdx.x == 0) {
-    const unsigned gen = *(volatile unsigned *)(bar + 1);
-    __threadfence();
-    if (atomicAdd(bar, 1u) == gridDim.x - 1) {
-      *(volatile unsigned *)bar = 0u;
+    int ok = *(volatile unsigned *)(bar + 2) == 0u;
+    if (ok) {
+      const unsigned gen = *(volatile unsigned *)(bar + 1);
       __threadfence();
-      atomicAdd(bar + 1, 1u);
-    } else {
-      while (*(volatile unsigned *)(bar + 1) == gen) __nanosleep(64);
+      if (atomicAdd(bar, 1u) == gridDim.x - 1) {
+        *(volatile unsigned *)bar = 0u;
+        __threadfence();
+        atomicAdd(bar + 1, 1u);
+      } else {
+        for (unsigned it = 0; *(volatile unsigned *)(bar + 1) == gen; ++it) {
+          if (it >= (1u << 24) || *(volatile unsigned *)(bar + 2) != 0u) {
+            atomicExch(bar + 2, 1u);
+            ok = 0;
+            break;
+          }
+          __nanosleep(64);
+        }
+      }
+      __threadfence();
     }
-    __threadfence();
+    s_ok = ok;
   }
   __syncthreads();
+  return s_ok != 0;
 }
-
 
 // Steps 4-5 after the fused pass, one launch (programmatic dependent launch:
 // its launch latency overlaps the fused kernels; griddepcontrol.wait orders
@@ -1397,7 +1415,7 @@ __global__ void __launch_bounds__(256) k_finish(const SpmvArgs a, int rounds) {
                                       min64(kBetaChunk, a.ngroups - c * kBetaChunk), s_red);
         if (threadIdx.x == 0) a.bpart[c] = v;
       }
-      grid_sync(a.gbar);
+      if (!grid_sync(a.gbar)) return;
       if (solo && blockIdx.x != 0) return;
       beta = __dsqrt_rn(cta_pw_array(a.bpart, nch, s_red));  // R10
     }
@@ -1405,8 +1423,8 @@ __global__ void __launch_bounds__(256) k_finish(const SpmvArgs a, int rounds) {
     if (threadIdx.x == 0) s_beta = beta;
     if (solo)
       __syncthreads();
-    else
-      grid_sync(a.gbar);  // n_flags zeroed, partials consumed
+    else if (!grid_sync(a.gbar))  // n_flags zeroed, partials consumed
+      return;
     beta = s_beta;
     for (int q = blockIdx.x * blockDim.x + threadIdx.x; q < nc; q += gridDim.x * blockDim.x) {
       const int32_t kk = __ldcg(a.cand + q);
@@ -1420,8 +1438,8 @@ __global__ void __launch_bounds__(256) k_finish(const SpmvArgs a, int rounds) {
     }
     if (solo)
       __syncthreads();
-    else
-      grid_sync(a.gbar);  // round 0's list complete; every CTA has read n_cand
+    else if (!grid_sync(a.gbar))  // round 0's list complete; every CTA has read n_cand
+      return;
     if (blockIdx.x == 0 && threadIdx.x == 0) *a.n_cand = 0;
   }
   if (rounds == 0 || __ldcg(a.n_flags) == 0) return;
@@ -1529,8 +1547,8 @@ __global__ void __launch_bounds__(256) k_finish(const SpmvArgs a, int rounds) {
     if (round < rounds) {
       if (solo)
         __syncthreads();
-      else
-        grid_sync(a.gbar);
+      else if (!grid_sync(a.gbar))
+        return;
     }
   }
 }

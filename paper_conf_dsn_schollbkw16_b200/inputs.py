@@ -302,13 +302,16 @@ def burst_mask(start_bit: int, length: int) -> int:
 class FaultPlan:
     """Explicit fault list: entry e XORs `mask[e]` into the value produced for
     element `index[e]` of `target[e]` (0 = y row, 1 = t1 block, 2 = t2 block)
-    in correction round `round[e]` (0 = the main pass)."""
+    in correction round `round[e]` (0 = the main pass).  `call` (optional):
+    entry e only applies to the `call[e]`-th SpMV of a solve (PCG); None =
+    every call."""
 
-    def __init__(self, round_, target, index, mask):
+    def __init__(self, round_, target, index, mask, call=None):
         self.round = np.ascontiguousarray(round_, dtype=np.int32)
         self.target = np.ascontiguousarray(target, dtype=np.int32)
         self.index = np.ascontiguousarray(index, dtype=np.int64)
         self.mask = np.ascontiguousarray(mask, dtype=np.uint64)
+        self.call = None if call is None else np.ascontiguousarray(call, dtype=np.int64)
 
     def __len__(self):
         return int(self.index.shape[0])
@@ -318,10 +321,13 @@ class FaultPlan:
         return FaultPlan([], [], [], [])
 
     def concat(self, other: "FaultPlan") -> "FaultPlan":
+        if (self.call is None) != (other.call is None):
+            raise ValueError("concat of a per-call plan with an all-calls plan")
         return FaultPlan(np.concatenate([self.round, other.round]),
                          np.concatenate([self.target, other.target]),
                          np.concatenate([self.index, other.index]),
-                         np.concatenate([self.mask, other.mask]))
+                         np.concatenate([self.mask, other.mask]),
+                         None if self.call is None else np.concatenate([self.call, other.call]))
 
 
 def single_fault_plan(n_elems: int, seed: int, target: int = TARGET_Y,

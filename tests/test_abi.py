@@ -68,6 +68,18 @@ def test_burst_table_matches_oracle(L, O):
     assert np.array_equal(abft.burst_table(), O.burst_table())
 
 
+def test_fault_tables_match_oracle(L, O):
+    # The Poisson CDF tables and the chunk rule of rate mode (R13)
+    # are written separately in the library and in the oracle; both follow
+    # the reading's definition, so the tables must agree entry for entry.
+    from paper_conf_dsn_schollbkw16_b200 import abft
+    for mu in (0.0, 1e-9, 1e-4, 0.01, 0.3, 1.0, 2.5, 4.0, 7.9):
+        assert np.array_equal(abft.poisson_table(mu, 32), O.poisson_table(mu, 32)), mu
+        assert np.array_equal(abft.poisson_table(mu, 1024), O.poisson_table(mu, 1024)), mu
+    for lam in (0.0, 1e-12, 1e-8, 2.4e-7, 1e-6, 1e-4, 0.01, 0.5, 1.0):
+        assert abft.rate_chunk(lam) == O.rate_chunk(lam), lam
+
+
 def test_encode_rejects_bad_args_without_gpu(L):
     import ctypes as C
     from paper_conf_dsn_schollbkw16_b200 import abft

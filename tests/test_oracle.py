@@ -211,6 +211,36 @@ class TestEncode:
         assert enc.n_k.tolist() == [2, 2, 2]
         assert enc.K[0] == ((2 + 2 * 2 - 2) * 18.0 + 2 * c0) * EPS
 
+    def test_c_value_is_pw_over_row_slots(self, O):
+        # R4*: c_kj = PW over the b_s row slots of block k, with ABSENT slots
+        # where a row lacks column j.  Column 0 of a 4-row block holds
+        # (1, absent, 1e16, -1e16): PW = 1 + (1e16 + -1e16) = 1.0; a left fold
+        # over the present rows gives (1 + 1e16) - 1e16 = 0.0.  Column 1 holds
+        # (1, 1e16, -1e16, 1): PW = (1 + 1e16) + (-1e16 + 1) = 1e16 - 1e16 = 0,
+        # a left fold gives ((1 + 1e16) - 1e16) + 1 = 1.0.
+        D = np.zeros((4, 4))
+        D[:, 0] = [1.0, 0.0, 1e16, -1e16]
+        D[:, 1] = [1.0, 1e16, -1e16, 1.0]
+        D[1, 2] = 1.0  # keeps row 1 non-empty
+        A = csr_from_dense(D)
+        enc = O.encode(A, 4)
+        assert enc.col.tolist() == [0, 1, 2]
+        assert enc.val.tolist() == [1.0, 0.0, 1.0]
+
+    def test_block_norm_sum_is_pw_over_row_slots(self, O):
+        # R7: S_k = PW over the b_s slots of ||a_i||.  diag(1, 2^53, 1, 1) with
+        # b_s = 4: S = (1 + 2^53) + (1 + 1) = 2^53 + 2 (1 + 2^53 rounds to
+        # 2^53, ties to even); a left fold gives 2^53.  ||c|| = sqrt((1 +
+        # 2^106) + (1 + 1)) = 2^53, n_k = 4, m = n_k + 2 b_s - 2 = 10:
+        # K = fl(fl(10 (2^53 + 2)) + 4 2^53) 2^-53 = (14 2^53 + 16) 2^-53
+        # = 14 + 2^-49 (10 (2^53 + 2) = 10 2^53 + 20 rounds to + 16 at ulp 16);
+        # with the left-fold S it would be exactly 14.
+        A = csr_from_dense(np.diag([1.0, 2.0 ** 53, 1.0, 1.0]))
+        enc = O.encode(A, 4)
+        assert enc.S[0] == 2.0 ** 53 + 2
+        assert enc.c_norm[0] == 2.0 ** 53
+        assert enc.K[0] == 14.0 + 2.0 ** -49
+
     def test_ragged_last_block(self, O):
         # R3 (Q3): the last block holds only the existing rows; b_s stays literal.
         A = G.laplacian_2d_5pt(5)  # N = 25, b_s = 8 -> last block has 1 row
@@ -526,6 +556,27 @@ class TestPcg:
         assert abs(r.iters - clean.iters) <= 3
         assert r.uncorrected_calls == 0
 
+    def test_corrected_fault_leaves_pcg_bits_unchanged(self, O):
+        # P:76 step 5: a fault the method flags is corrected by
+        # recomputing its block, which restores y bit for bit, so a protected
+        # PCG with one large fault in call 5 (a per-call list) has the
+        # fault-free residual history and solution; the unprotected solve
+        # with the same fault does not.
+        A = G.laplacian_3d_7pt(8)
+        enc = O.encode(A, 32)
+        b = O.spmv(A, G.uniform_vector(A.n, 43))
+        x0 = G.uniform_vector(A.n, 44)
+        ref = O.pcg(A, enc, b, x0, tol=1e-6)
+        plan = G.FaultPlan([0, 0], [0, 1], [100, 9],
+                           [np.uint64(1) << np.uint64(61), np.uint64(1) << np.uint64(60)],
+                           call=[5, 11])
+        r = O.pcg(A, enc, b, x0, tol=1e-6, inj=O.Inject.from_plan(plan))
+        assert r.status == 0 and r.flagged_blocks == 2 and r.uncorrected_calls == 0
+        assert np.array_equal(r.res_hist.view(np.uint64), ref.res_hist.view(np.uint64))
+        assert np.array_equal(r.x.view(np.uint64), ref.x.view(np.uint64))
+        u = O.pcg(A, enc, b, x0, tol=1e-6, inj=O.Inject.from_plan(plan), check=False)
+        assert not np.array_equal(u.res_hist[:8], ref.res_hist[:8])
+
     def test_unprotected_faulty_pcg_differs(self, O):
         A = G.laplacian_3d_7pt(8)
         enc = O.encode(A, 32)
@@ -680,6 +731,29 @@ class TestPcgCheckpoint:
         assert r.spmv_calls >= r.executed + 1
         if r.status == 0:  # converged: the recursive residual met the test
             assert r.res_hist[-1] <= 1e-6 * np.linalg.norm(b)
+
+    def test_detected_fault_rolls_back_to_fault_free_bits(self, O):
+        # after a detection the solver restores the last sample and
+        # re-executes from it.  A single fault in call 24 of the solve (the
+        # SpMV of iteration 24; |delta| far above ||p||) is detected, the
+        # state sampled after iteration 20 is restored, and iterations 21..24
+        # run again: 4 more executed iterations and SpMV calls than the
+        # fault-free solve.  The re-execution repeats the fault-free
+        # operations exactly, so the returned x and residual history are the
+        # fault-free run's bit for bit.
+        A = G.laplacian_3d_7pt(8)
+        den = O.dense_encode(A)
+        b = O.spmv(A, G.uniform_vector(A.n, 43))
+        x0 = G.uniform_vector(A.n, 44)
+        ref = O.pcg_cr(A, den, b, x0, tol=1e-6)
+        assert ref.rollbacks == 0 and ref.iters > 24
+        plan = G.FaultPlan([0], [0], [77], [np.uint64(1) << np.uint64(62)], call=[24])
+        r = O.pcg_cr(A, den, b, x0, tol=1e-6, inj=O.Inject.from_plan(plan))
+        assert r.status == 0 and r.rollbacks == 1
+        assert r.executed == ref.executed + 4 and r.spmv_calls == ref.spmv_calls + 4
+        assert r.iters == ref.iters
+        assert np.array_equal(r.res_hist.view(np.uint64), ref.res_hist.view(np.uint64))
+        assert np.array_equal(r.x.view(np.uint64), ref.x.view(np.uint64))
 
     def test_sample_every_iteration_loses_nothing(self, O):
         # ckpt_every = 1: a rollback restores the state of the iteration it
