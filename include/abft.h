@@ -138,7 +138,9 @@ abft_status abft_encode(const abft_csr_t *A, int32_t block_size, int32_t max_rou
  * kernel streams and its byte count, and how the groups of 32 rows split
  * between the staged fast path and the general path. */
 enum { ABFT_CFMT_CSR = 0, ABFT_CFMT_I8 = 1, ABFT_CFMT_I16 = 2, ABFT_CFMT_F32 = 3,
-       ABFT_CFMT_F64 = 4 };
+       ABFT_CFMT_F64 = 4,
+       /* position-map records (row-regular matrices) */
+       ABFT_CFMT_POS_I8 = 5, ABFT_CFMT_POS_I16 = 6, ABFT_CFMT_POS_F32 = 7, ABFT_CFMT_POS_F64 = 8 };
 typedef struct {
   int64_t n, nnz, nb, nnz_c;
   int32_t block_size, c_format;
@@ -149,6 +151,15 @@ typedef struct {
   int64_t irr_groups;       /* 32-row groups on the irregular-row path (k_irr) */
   int32_t lean_short;       /* k_lean SHORT instantiation (all its rows <= 8 entries) */
   int32_t lean_runs;        /* k_lean walks interleaved runs of groups (large matrices) */
+  int32_t stream;           /* warp-specialized kernel (position-map records) in use */
+  int32_t stream_g;         /* its groups per chunk (consumer warps per CTA) */
+  int32_t stream_stages;    /* its ring stages */
+  int32_t reserved0;
+  int64_t pos_exc_rows;     /* exception rows over all position-map records */
+  int64_t stream_plain_bytes;  /* bytes the warp-specialized kernel streams per call with the
+                                  check off (A values and columns, structure records, x, y),
+                                  0 if unused */
+  int64_t stream_check_bytes;  /* bytes the check adds (checksum records) */
 } abft_info_t;
 abft_status abft_info(abft_handle_t h, abft_info_t *info);
 

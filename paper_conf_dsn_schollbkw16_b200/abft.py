@@ -35,7 +35,8 @@ SYMBOLS = [
 PCG_PHASE_INIT, PCG_PHASE_DOT, PCG_PHASE_UPDATE, PCG_PHASE_P = 0, 1, 2, 3
 PCG_PHASE_CG1_UPDATE, PCG_PHASE_CG1_DOT = 4, 5  # single-reduction variant
 ENCODE_C_CSR = 1
-CFMT_NAMES = {0: "csr-f64", 1: "int8+u16", 2: "int16+u16", 3: "f32+u16", 4: "f64+u16"}
+CFMT_NAMES = {0: "csr-f64", 1: "int8+u16", 2: "int16+u16", 3: "f32+u16", 4: "f64+u16",
+              5: "int8+pos", 6: "int16+pos", 7: "f32+pos", 8: "f64+pos"}
 
 
 class AbftError(RuntimeError):
@@ -65,7 +66,10 @@ class Info(C.Structure):
                 ("block_size", C.c_int32), ("c_format", C.c_int32), ("c_bytes", C.c_int64),
                 ("groups", C.c_int64), ("general_groups", C.c_int64), ("lean", C.c_int32),
                 ("max_rounds", C.c_int32), ("irr_groups", C.c_int64), ("lean_short", C.c_int32),
-                ("lean_runs", C.c_int32)]
+                ("lean_runs", C.c_int32), ("stream", C.c_int32), ("stream_g", C.c_int32),
+                ("stream_stages", C.c_int32), ("reserved0", C.c_int32),
+                ("pos_exc_rows", C.c_int64), ("stream_plain_bytes", C.c_int64),
+                ("stream_check_bytes", C.c_int64)]
 
     def as_dict(self):
         d = {f: getattr(self, f) for f, _ in self._fields_}

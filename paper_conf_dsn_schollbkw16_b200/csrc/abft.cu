@@ -12,6 +12,7 @@
 #include "kernels_encode.cuh"
 #include "kernels_pcg.cuh"
 #include "kernels_spmv.cuh"
+#include "kernels_stream.cuh"
 #include "kernels_irr.cuh"
 #include "kernels_dense.cuh"
 #include "kernels_bigblock.cuh"
@@ -108,6 +109,20 @@ struct abft_ctx {
   int32_t *crp_c = nullptr;  // compact row starts (32-entry aligned)
   int64_t nnz_cpad = 0;      // compact slots incl. row padding
   StageCfg stage{};
+  // position-map records and the warp-specialized kernel (kernels_stream.cuh)
+  bool pos = false;            // C streamed as position-map records
+  int pos_cf = CF_F64;         // their value type
+  int32_t pos_S = 8;           // W slots per row
+  unsigned char *srec = nullptr;  // structure records (grec: checksum records)
+  uint32_t *soff = nullptr, *coff = nullptr;  // [ngroups + 1] record offsets (16-B units)
+  int64_t pos_sbytes = 0, pos_cbytes = 0;     // total record bytes
+  int64_t pos_exc = 0;         // exception rows over all records
+  bool stream = false;         // k_stream runs the eligible chunks
+  StreamCfg stc{};
+  int32_t *clist = nullptr;    // eligible chunks
+  int64_t n_clist = 0;
+  size_t stream_smem = 0;
+  int stream_grid = 1;
   bool lean = false;        // k_lean usable (b_s = 32, 16-B aligned A)
   bool lean_short = false;  // every k_lean group's rows <= 8 entries (SHORT instantiation)
   bool lean_runs = false;   // k_lean walks interleaved runs (RUNS instantiation)
@@ -187,6 +202,14 @@ abft_status dalloc(abft_ctx *h, T **p, size_t count) {
   return ABFT_OK;
 }
 
+template <typename T>
+abft_status upload(abft_ctx *h, T **dst, const std::vector<T> &v, cudaStream_t s) {
+  TRY(dalloc(h, dst, v.size()));
+  if (!v.empty())
+    CK(cudaMemcpyAsync(*dst, v.data(), v.size() * sizeof(T), cudaMemcpyHostToDevice, s));
+  return ABFT_OK;
+}
+
 bool aligned16(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
 
 SpmvArgs make_args(const abft_ctx *h, const double *x, double *y, const double *x_norm) {
@@ -234,6 +257,12 @@ SpmvArgs make_args(const abft_ctx *h, const double *x, double *y, const double *
   a.own_first = h->own_first;
   a.own_n = h->own_n;
   a.n_own = h->n_own;
+  a.srec = h->srec;
+  a.soff = h->soff;
+  a.coff = h->coff;
+  a.clist = h->clist;
+  a.n_clist = h->n_clist;
+  a.stc = h->stc;
   return a;
 }
 
@@ -397,6 +426,22 @@ void launch_lean(const abft_ctx *h, const SpmvArgs &a, cudaStream_t s) {
 }
 
 template <bool CHECK, bool INJECT>
+void launch_stream(const abft_ctx *h, const SpmvArgs &a, cudaStream_t s) {
+  const dim3 grid(h->stream_grid), block((h->stc.G + 1) * 32);
+  const size_t sm = h->stream_smem;
+#define STREAM(CF)                                                               \
+  (h->pos_S <= 8 ? k_stream<CHECK, INJECT, CF, true><<<grid, block, sm, s>>>(a) \
+                 : k_stream<CHECK, INJECT, CF, false><<<grid, block, sm, s>>>(a))
+  switch (h->pos_cf) {
+    case CF_I8: STREAM(CF_I8); break;
+    case CF_I16: STREAM(CF_I16); break;
+    case CF_F32: STREAM(CF_F32); break;
+    default: STREAM(CF_F64); break;
+  }
+#undef STREAM
+}
+
+template <bool CHECK, bool INJECT>
 void launch_irr(const abft_ctx *h, const SpmvArgs &a, cudaStream_t s) {
   const size_t smem = kIrrWarps * kIrrSmemPerWarp;
   const int64_t need = (h->n_ilist + kIrrWarps - 1) / kIrrWarps;
@@ -418,6 +463,16 @@ abft_status launch_fused_t(const abft_ctx *h, SpmvArgs a, cudaStream_t s) {
     const int64_t need = (h->nb + 3) / 4;
     k_bigblock<CHECK, INJECT><<<(unsigned)std::max<int64_t>(1, std::min<int64_t>((int64_t)h->num_sms * 16, need)),
                                 128, 0, s>>>(a);
+    CK(cudaGetLastError());
+    return ABFT_OK;
+  }
+  if (h->stream) {  // position-map records: the warp-specialized kernel + k_general
+    a.glist = h->glist;
+    a.n_glist = h->n_glist;
+    if (h->n_hub > 0) k_hub<<<general_grid(h, h->n_hub), kGenWarps * 32, 0, s>>>(a);
+    if (h->n_clist > 0) launch_stream<CHECK, INJECT>(h, a, s);
+    if (h->n_glist > 0)
+      k_general<CHECK, INJECT><<<general_grid(h, h->n_glist), kGenWarps * 32, 0, s>>>(a);
     CK(cudaGetLastError());
     return ABFT_OK;
   }
@@ -545,6 +600,16 @@ abft_status set_lean_attrs(int optin) {
   TRY(set_smem_attrs(k_lean<true, false, CF, 2, false, true>, optin));
   TRY(set_smem_attrs(k_lean<false, true, CF, 2, false, true>, optin));
   TRY(set_smem_attrs(k_lean<false, false, CF, 2, false, true>, optin));
+  if constexpr (CF != CF_CSR) {
+    TRY(set_smem_attrs(k_stream<true, true, CF, true>, optin));
+    TRY(set_smem_attrs(k_stream<true, false, CF, true>, optin));
+    TRY(set_smem_attrs(k_stream<false, true, CF, true>, optin));
+    TRY(set_smem_attrs(k_stream<false, false, CF, true>, optin));
+    TRY(set_smem_attrs(k_stream<true, true, CF, false>, optin));
+    TRY(set_smem_attrs(k_stream<true, false, CF, false>, optin));
+    TRY(set_smem_attrs(k_stream<false, true, CF, false>, optin));
+    TRY(set_smem_attrs(k_stream<false, false, CF, false>, optin));
+  }
   for (auto kern : {k_irr<true, true, CF>, k_irr<true, false, CF>, k_irr<false, true, CF>,
                     k_irr<false, false, CF>})
     CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -636,6 +701,199 @@ abft_status build_compact_c(abft_ctx *h, cudaStream_t s) {
   return ABFT_OK;
 }
 
+// Position-map records (kernels_stream.cuh) when the matrix
+// is row-regular: b_s = 32, rows of the full groups <= 32 entries, >= 90% of
+// the full groups eligible and on average <= 8 exception rows per record
+// (stencils: the x-boundary rows).  Otherwise the slot-map form (or CSR)
+// stays.  Synchronises the stream.
+abft_status scan_u32(abft_ctx *h, const uint32_t *in, uint32_t *out, int64_t n, cudaStream_t s) {
+  const int64_t nscan = (n + 1023) / 1024;
+  int32_t *totals = nullptr;
+  TRY(dalloc(h, &totals, (size_t)nscan));
+  const int32_t *i32 = reinterpret_cast<const int32_t *>(in);
+  int32_t *o32 = reinterpret_cast<int32_t *>(out);
+  k_scan_local<<<(unsigned)nscan, 1024, 0, s>>>(i32, o32, n, totals);
+  k_scan_totals<<<1, 1024, 0, s>>>(totals, nscan, o32 + n);
+  k_scan_add<<<(unsigned)nscan, 1024, 0, s>>>(o32, n, totals);
+  CK(cudaGetLastError());
+  return ABFT_OK;
+}
+
+abft_status build_pos_c(abft_ctx *h, cudaStream_t s) {
+  if (h->bs != 32 || h->nnz_c == 0 || h->n < 32 || getenv("ABFT_NO_POS")) return ABFT_OK;
+  if (!(aligned16(h->rp) && aligned16(h->ci) && aligned16(h->va))) return ABFT_OK;
+  int32_t *dev = nullptr;
+  unsigned long long *stats = nullptr;
+  TRY(dalloc(h, &dev, 2));
+  TRY(dalloc(h, &stats, 2));
+  CK(cudaMemsetAsync(dev, 0, 2 * sizeof(int32_t), s));
+  CK(cudaMemsetAsync(stats, 0, 2 * sizeof(unsigned long long), s));
+  const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((h->nb + 7) / 8, 65535));
+  k_cformat_scan<<<grid, 256, 0, s>>>(h->nb, h->c_rp, h->c_col, h->c_val, dev);
+  k_pos_maxlen<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>((h->n + 255) / 256, 4096)), 256, 0,
+                 s>>>(h->n, h->rp, dev + 1);
+  CK(cudaGetLastError());
+  int32_t hv[2] = {0, 0};
+  CK(cudaMemcpyAsync(hv, dev, sizeof hv, cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  const int props = hv[0];
+  const int cf = !(props & 1) ? CF_I8 : !(props & 2) ? CF_I16 : !(props & 4) ? CF_F32 : CF_F64;
+  // W slots: the longest row up to 32 (groups with longer rows are not eligible)
+  const int32_t S = std::max(8, (std::min(hv[1], 32) + 7) & ~7);
+  const int64_t ng = h->ngroups;
+  uint32_t *ssz = nullptr, *csz = nullptr;
+  TRY(dalloc(h, &ssz, (size_t)ng));
+  TRY(dalloc(h, &csz, (size_t)ng));
+  TRY(dalloc(h, &h->soff, (size_t)ng + 1));
+  TRY(dalloc(h, &h->coff, (size_t)ng + 1));
+#define POS(T, FILL, SR, CR)                                                                       \
+  k_pos_encode<T, FILL><<<grid, 256, 0, s>>>(h->n, ng, S, h->rp, h->ci, h->c_rp, h->c_col, h->c_val, \
+                                             h->K, ssz, csz, h->soff, h->coff, SR, CR, stats)
+  switch (cf) {
+    case CF_I8: POS(int8_t, false, nullptr, nullptr); break;
+    case CF_I16: POS(int16_t, false, nullptr, nullptr); break;
+    case CF_F32: POS(float, false, nullptr, nullptr); break;
+    default: POS(double, false, nullptr, nullptr); break;
+  }
+  TRY(scan_u32(h, ssz, h->soff, ng, s));
+  TRY(scan_u32(h, csz, h->coff, ng, s));
+  unsigned long long st[2] = {0, 0};
+  uint32_t tot[2] = {0, 0};
+  CK(cudaMemcpyAsync(st, stats, sizeof st, cudaMemcpyDeviceToHost, s));
+  CK(cudaMemcpyAsync(&tot[0], h->soff + ng, 4, cudaMemcpyDeviceToHost, s));
+  CK(cudaMemcpyAsync(&tot[1], h->coff + ng, 4, cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  const int64_t nfull = h->n / 32;
+  const bool accept = getenv("ABFT_FORCE_POS") ||
+                      ((int64_t)st[1] * 10 >= nfull * 9 && st[0] <= 8 * st[1] && st[1] > 0);
+  if (!accept || (int64_t)tot[0] >= ((int64_t)1 << 31) || (int64_t)tot[1] >= ((int64_t)1 << 31))
+    return ABFT_OK;
+  unsigned char *srec = nullptr, *crec = nullptr;
+  const size_t sb = (size_t)tot[0] * 16 + 64, cb = (size_t)tot[1] * 16 + 64;
+  TRY(dalloc(h, &srec, sb));
+  TRY(dalloc(h, &crec, cb));
+  CK(cudaMemsetAsync(srec, 0, sb, s));
+  CK(cudaMemsetAsync(crec, 0, cb, s));
+  switch (cf) {
+    case CF_I8: POS(int8_t, true, srec, crec); break;
+    case CF_I16: POS(int16_t, true, srec, crec); break;
+    case CF_F32: POS(float, true, srec, crec); break;
+    default: POS(double, true, srec, crec); break;
+  }
+#undef POS
+  CK(cudaGetLastError());
+  CK(cudaStreamSynchronize(s));
+  h->srec = srec;
+  h->grec = crec;
+  h->pos = true;
+  h->pos_cf = cf;
+  h->pos_S = S;
+  h->pos_sbytes = (int64_t)tot[0] * 16;
+  h->pos_cbytes = (int64_t)tot[1] * 16;
+  h->pos_exc = (int64_t)st[0];
+  return ABFT_OK;
+}
+
+// k_stream plan: chunks of G groups whose groups all have
+// records; ring stage capacities from the largest eligible chunk; G and the
+// stage count from the shared-memory budget of two CTAs per SM.  The other
+// groups go to k_general.  rp / crp: host copies.
+abft_status plan_stream(abft_ctx *h, const std::vector<int32_t> &rp, const std::vector<int32_t> &crp,
+                        std::vector<int32_t> &glist, cudaStream_t s) {
+  const int64_t ng = h->ngroups;
+  std::vector<uint32_t> soff((size_t)ng + 1), coff((size_t)ng + 1);
+  CK(cudaMemcpyAsync(soff.data(), h->soff, soff.size() * 4, cudaMemcpyDeviceToHost, s));
+  CK(cudaMemcpyAsync(coff.data(), h->coff, coff.size() * 4, cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  auto elig = [&](int64_t g) { return soff[(size_t)g + 1] > soff[(size_t)g]; };
+  StreamCfg best{};
+  int64_t best_score = -1;
+  std::vector<int32_t> best_list;
+  int forced_g = 0;
+  if (const char *e = getenv("ABFT_STREAM_G")) forced_g = atoi(e);
+  for (int G : {8, 4, 2}) {
+    if (forced_g && G != forced_g) continue;
+    const int64_t nch = (ng + G - 1) / G;
+    std::vector<int32_t> list;
+    int64_t capA = 0, capS = 0, capCR = 0, capC = 0;
+    for (int64_t q = 0; q < nch; ++q) {
+      const int64_t g0 = q * G, g1 = std::min<int64_t>(ng, g0 + G);
+      bool ok = true;
+      for (int64_t g = g0; g < g1 && ok; ++g) ok = elig(g);
+      if (!ok) continue;
+      list.push_back((int32_t)q);
+      const int64_t sa4 = rp[(size_t)g0 * 32] & ~3ll;
+      capA = std::max<int64_t>(capA, (int64_t)rp[(size_t)g1 * 32] + 3 - sa4);
+      capS = std::max<int64_t>(capS, (int64_t)(soff[(size_t)g1] - soff[(size_t)g0]) * 16);
+      capCR = std::max<int64_t>(capCR, (int64_t)(coff[(size_t)g1] - coff[(size_t)g0]) * 16);
+      for (int64_t g = g0; g < g1; ++g) capC = std::max<int64_t>(capC, crp[(size_t)g + 1] - crp[(size_t)g]);
+    }
+    if (list.empty()) continue;
+    StreamCfg c{};
+    c.G = G;
+    c.S = h->pos_S;
+    uint32_t o = stream_hdr_bytes(G);
+    c.off_srec = o;
+    o += align16((uint32_t)capS);
+    c.off_crec = o;
+    o += align16((uint32_t)capCR);
+    c.off_av = o;
+    o += align16((uint32_t)(capA + 12) * 8);  // + 8: unpredicated reads past a row
+    c.off_ac = o;
+    o += align16((uint32_t)(capA + 12) * 4);
+    c.stage_bytes = align16(o);
+    c.xs_bytes = align16((uint32_t)(((capC + 7) & ~7ll) + 32) * 8);  // + the trash slots
+    // ring stages: as many as fit two CTAs per SM (>= 2)
+    size_t budget = (size_t)std::min<size_t>(g_dyn_smem_limit, 113 * 1024);
+    if (const char *e = getenv("ABFT_STREAM_SMEM_KB"))  // tuning sweeps only
+      budget = std::min<size_t>(g_dyn_smem_limit, (size_t)atoi(e) * 1024);
+    const size_t fixed = 128 + (size_t)G * c.xs_bytes;
+    int NS = 0;
+    while (NS < 8 && fixed + (size_t)(NS + 1) * c.stage_bytes <= budget) ++NS;
+    if (const char *e = getenv("ABFT_STREAM_NS")) NS = std::min(NS, std::max(2, atoi(e)));
+    if (NS < 2) continue;
+    c.NS = NS;
+    c.ring_off = 128;
+    c.xs_off = 128 + (uint32_t)NS * c.stage_bytes;
+    // prefer more groups per chunk (fewer producer round trips) when >= 3 stages fit
+    const int64_t score = (int64_t)(NS >= 3 ? 1000 : 0) + G * 10 + NS;
+    if (score > best_score) {
+      best_score = score;
+      best = c;
+      best_list = list;
+    }
+  }
+  if (best_score < 0) return ABFT_OK;  // no chunk fits: k_general takes every group
+  h->stc = best;
+  h->stream_smem = best.xs_off + (size_t)best.G * best.xs_bytes;
+  std::vector<uint8_t> in((size_t)ng, 0);
+  for (int32_t q : best_list)
+    for (int64_t g = (int64_t)q * best.G; g < std::min<int64_t>(ng, (int64_t)(q + 1) * best.G); ++g)
+      in[(size_t)g] = 1;
+  for (int64_t g = 0; g < ng; ++g)
+    if (!in[(size_t)g]) glist.push_back((int32_t)g);
+  TRY(upload(h, &h->clist, best_list, s));
+  h->n_clist = (int64_t)best_list.size();
+  int per_sm = 0;
+#define OCC(CF)                                                                                   \
+  (h->pos_S <= 8 ? cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_stream<true, false, CF, true>, \
+                                                                 (best.G + 1) * 32, h->stream_smem)          \
+                 : cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_stream<true, false, CF, false>, \
+                                                                 (best.G + 1) * 32, h->stream_smem))
+  switch (h->pos_cf) {
+    case CF_I8: CK(OCC(CF_I8)); break;
+    case CF_I16: CK(OCC(CF_I16)); break;
+    case CF_F32: CK(OCC(CF_F32)); break;
+    default: CK(OCC(CF_F64)); break;
+  }
+#undef OCC
+  per_sm = std::max(per_sm, 1);
+  if (const char *e = getenv("ABFT_CTAS_PER_SM")) per_sm = std::max(1, std::min(per_sm, atoi(e)));
+  h->stream_grid = (int)std::max<int64_t>(1, std::min<int64_t>((int64_t)h->num_sms * per_sm, h->n_clist));
+  h->stream = true;
+  return ABFT_OK;
+}
+
 // Stage layout for capacities (capA, capC).
 uint32_t stage_layout(const abft_ctx *h, StageCfg &c) {
   uint32_t o = 0;
@@ -673,14 +931,6 @@ uint32_t stage_layout(const abft_ctx *h, StageCfg &c) {
     c.off_xg = c.off_av;
   }
   return align16(o);
-}
-
-template <typename T>
-abft_status upload(abft_ctx *h, T **dst, const std::vector<T> &v, cudaStream_t s) {
-  TRY(dalloc(h, dst, v.size()));
-  if (!v.empty())
-    CK(cudaMemcpyAsync(*dst, v.data(), v.size() * sizeof(T), cudaMemcpyHostToDevice, s));
-  return ABFT_OK;
 }
 
 // Encode-time plan of the fused pass ("Long rows"):
@@ -740,6 +990,24 @@ abft_status plan_fused(abft_ctx *h, cudaStream_t s) {
     TRY(upload(h, &h->own_n, on, s));
     h->n_hub = (int32_t)hbeg.size();
     h->n_own = (int32_t)own.size();
+  }
+  if (h->pos) {  // position-map records: k_stream + k_general
+    h->lean = false;
+    std::vector<uint8_t> lean_ok((size_t)h->ngroups, 0);
+    for (const auto &o : own) lean_ok[(size_t)(o.first >> 6)] |= 2;  // groups owning hub rows
+    std::vector<int32_t> gl, all;
+    TRY(plan_stream(h, rp, crp, gl, s));
+    for (int64_t g = 0; g < h->ngroups; ++g) all.push_back((int32_t)g);
+    if (!h->stream) gl = all;
+    TRY(upload(h, &h->lean_ok, lean_ok, s));
+    TRY(upload(h, &h->glist, gl, s));
+    TRY(upload(h, &h->glist_nl, all, s));
+    TRY(upload(h, &h->ilist, std::vector<int32_t>(), s));
+    h->n_glist = (int64_t)gl.size();
+    h->n_glist_nl = (int64_t)all.size();
+    h->n_ilist = 0;
+    CK(cudaStreamSynchronize(s));  // host vectors die at return
+    return ABFT_OK;
   }
   // k_lean candidates: (segment, C length) per group
   std::vector<uint8_t> lean_ok((size_t)h->ngroups, 0);
@@ -1074,7 +1342,10 @@ abft_status abft_encode(const abft_csr_t *A, int32_t block_size, int32_t max_rou
   if ((e = cudaMemsetAsync(h->c_col + h->nnz_c, 0, 8 * sizeof(int32_t), s)) ||
       (e = cudaMemsetAsync(h->c_val + h->nnz_c, 0, 8 * sizeof(double), s)))
     return fail(cuda_fail(e, "pad"));
-  if (!(flags & ABFT_ENCODE_C_CSR) && (st = build_compact_c(h, s)) != ABFT_OK) return fail(st);
+  if (!(flags & ABFT_ENCODE_C_CSR)) {
+    if ((st = build_pos_c(h, s)) != ABFT_OK) return fail(st);
+    if (!h->pos && (st = build_compact_c(h, s)) != ABFT_OK) return fail(st);
+  }
 
   // per-call scratch
   if ((st = dalloc(h, &h->gsum, (size_t)h->ngroups)) ||
@@ -1297,15 +1568,30 @@ abft_status abft_info(abft_handle_t h, abft_info_t *info) {
   info->nb = h->nb;
   info->nnz_c = h->nnz_c;
   info->block_size = h->bs;
-  info->c_format = h->cfmt;
-  if (h->cfmt == CF_CSR)
+  info->c_format = h->pos ? ABFT_CFMT_POS_I8 + (h->pos_cf - CF_I8) : h->cfmt;
+  info->stream = h->stream ? 1 : 0;
+  info->stream_g = h->stc.G;
+  info->stream_stages = h->stc.NS;
+  info->pos_exc_rows = h->pos_exc;
+  info->stream_plain_bytes = 0;
+  info->stream_check_bytes = 0;
+  if (h->pos) {
+    // k_stream streams A's values and columns, the structure records (row
+    // ends, position map; they replace row_ptr) and their offsets, x (read
+    // from HBM once, gathered from L2) and y; the check adds the checksum
+    // records (K, c_kj) and their offsets
+    info->stream_plain_bytes = 12 * h->nnz + h->pos_sbytes + 4 * (h->ngroups + 1) + 16 * h->n;
+    info->stream_check_bytes = h->pos_cbytes + 4 * (h->ngroups + 1);
+    info->c_bytes = info->stream_check_bytes;
+  }
+  else if (h->cfmt == CF_CSR)
     info->c_bytes = 12 * h->nnz_c + 4 * (h->nb + 1);
   else
     // values + A-slot map + compact row starts (the record headers re-encode
     // K and row_ptr, which the byte model counts once as K and A)
     info->c_bytes = (int64_t)(cf_size(h->cfmt) + 2) * h->nnz_cpad + 4 * (h->nb + 1);
   info->groups = h->ngroups;
-  info->general_groups = h->lean ? h->n_glist : h->n_glist_nl;
+  info->general_groups = (h->lean || h->stream) ? h->n_glist : h->n_glist_nl;
   info->irr_groups = h->n_ilist;
   info->lean_short = h->lean_short ? 1 : 0;
   info->lean_runs = h->lean_runs ? 1 : 0;

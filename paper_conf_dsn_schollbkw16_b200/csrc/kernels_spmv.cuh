@@ -45,7 +45,8 @@ template <> struct CType<CF_F32> { using T = float; };
 constexpr int kLeanWarps = 4;  // warps per CTA of k_lean (<= 4)
 // Timing experiments only (scripts/exp_libs.sh; results are NOT the method):
 // 1 = no C products, 2 = C neither staged nor multiplied, 3 = no butterflies,
-// 4 = no test, 5 = 1 + 3 + 4.  0 (the default) = the method.
+// 4 = no test, 5 = 1 + 3 + 4, 6 = k_stream without x gathers.  0 (the default)
+// = the method.
 #ifndef ABFT_EXP
 #define ABFT_EXP 0
 #endif
@@ -73,6 +74,21 @@ struct StageCfg {
   uint32_t bar_bytes;     // mbarrier region at the start of dynamic smem
   uint32_t off_rp, off_x, off_k, off_av, off_ac, off_cv, off_cc, off_cp, off_xg;
   int32_t colg;           // A columns read from global memory, not staged (COLG)
+};
+
+// k_stream (kernels_stream.cuh): producer / consumer ring configuration.
+constexpr int kStreamMaxG = 8;  // consumer warps per CTA (groups per chunk), at most
+struct StreamCfg {
+  int32_t G;             // groups per chunk = consumer warps per CTA
+  int32_t NS;            // ring stages
+  int32_t S;             // W slots per row of the structure records (multiple of 8)
+  uint32_t stage_bytes;  // bytes per stage
+  uint32_t off_srec;     // stage: structure records
+  uint32_t off_crec;     // stage: checksum records (CHECK)
+  uint32_t off_av, off_ac;  // stage: A values / columns (4-element grid from the chunk's first entry)
+  uint32_t ring_off;     // dynamic smem: ring start (after the barriers)
+  uint32_t xs_off;       // dynamic smem: per-consumer-warp C-position scratch
+  uint32_t xs_bytes;     // per warp
 };
 
 struct SpmvArgs {
@@ -126,6 +142,13 @@ struct SpmvArgs {
   int32_t n_own;
   StageCfg sc;
   InjDev inj;
+  // k_stream (position-map records, kernels_stream.cuh); grec = checksum records
+  const unsigned char *srec;  // structure records
+  const uint32_t *soff;     // [ngroups + 1] structure record offsets (16-B units)
+  const uint32_t *coff;     // [ngroups + 1] checksum record offsets (16-B units)
+  const int32_t *clist;     // eligible chunks
+  int64_t n_clist;
+  StreamCfg stc;
 };
 
 __device__ __forceinline__ bool skip_call(const SpmvArgs &a) {

@@ -229,10 +229,11 @@ def test_rate_mode_rmat_bs8(O, torch_cuda):
     c.run(G.uniform_vector(A.n, 1), rate=dict(seed=5, lam=1e-3, targets=0b111, call=7))
 
 
-def test_compact_formats_chosen(O, torch_cuda):
-    # the encoder picks the narrowest exact type
+def test_compact_formats_chosen(O, torch_cuda, monkeypatch):
+    # the encoder picks the narrowest exact type; row-
+    # regular matrices get position-map records (§6.9), the others the slot map
     from paper_conf_dsn_schollbkw16_b200 import encode
-    cases = [(G.laplacian_3d_7pt(16), "int8+u16"), (G.random_csr(500, 0.02, 1), "f64+u16"),
+    cases = [(G.laplacian_3d_7pt(16), "int8+pos"), (G.random_csr(500, 0.02, 1), "f64+u16"),
              (G.random_csr(300, 0.05, 2, integer=True, max_int=100), "int16+u16")]
     for A, fmt in cases:
         info = encode(A).info()
@@ -241,6 +242,10 @@ def test_compact_formats_chosen(O, torch_cuda):
     assert info["c_format_name"] == "csr-f64"
     A = G.laplacian_3d_7pt(16)
     info = encode(A).info()
+    assert info["general_groups"] == 0 and info["stream"] == 1
+    monkeypatch.setenv("ABFT_NO_POS", "1")
+    info = encode(A).info()
+    assert info["c_format_name"] == "int8+u16"
     assert info["general_groups"] == 0 and info["lean"] == 1
 
 
@@ -450,10 +455,12 @@ def test_lean_columns_from_global(O, torch_cuda, name, monkeypatch):
     # instead of staging them -- same bits, error-free and with faults
     monkeypatch.setenv("ABFT_COLG", "1")
     monkeypatch.setenv("ABFT_FORCE_COLG", "1")
+    monkeypatch.setenv("ABFT_NO_POS", "1")  # k_lean streams the slot-map records
     A = MATRICES[name]()
     c = Case(O, torch_cuda, A)
     monkeypatch.delenv("ABFT_FORCE_COLG")
     monkeypatch.delenv("ABFT_COLG")
+    monkeypatch.delenv("ABFT_NO_POS")
     c.check_encoding()
     ref = c.run(G.uniform_vector(A.n, 31))
     assert ref.flagged.size == 0
@@ -467,9 +474,11 @@ def test_lean_runs_large(O, torch_cuda, monkeypatch):
     # t2 / flags error-free, and with faults (the INJECT kernels walk
     # contiguous ranges) corrections
     monkeypatch.setenv("ABFT_FORCE_RUNS", "1")
+    monkeypatch.setenv("ABFT_NO_POS", "1")
     A = G.laplacian_3d_7pt(160)
     c = Case(O, torch_cuda, A)
     monkeypatch.delenv("ABFT_FORCE_RUNS")
+    monkeypatch.delenv("ABFT_NO_POS")
     info = c.h.info()
     assert info["lean_runs"] == 1 and info["lean_short"] == 1, info
     ref = c.run(G.uniform_vector(A.n, 34))
