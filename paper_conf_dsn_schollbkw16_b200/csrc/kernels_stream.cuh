@@ -419,6 +419,8 @@ struct ShortA {
   const unsigned char *st, *rec, *crec;
   int64_t g;
   int rs, len;
+  int ml;    // longest row of the group (uniform)
+  bool uni;  // every row of the group has ml entries (uniform)
   double xj[8];
   double xi;
 };
@@ -439,9 +441,15 @@ __device__ __forceinline__ void short_load(const SpmvArgs &a, const StreamCfg &c
   A.xi = CHECK ? ld_x(a.xr + g * 32 + lane) : 0.0;
   A.rs = rs;
   A.len = re - rs;
+  A.ml = warp_max_i(A.len);
+  A.uni = warp_min_i(A.len) == A.ml;
   const int32_t *ac = reinterpret_cast<const int32_t *>(st + c.off_ac) + rs;
 #pragma unroll
   for (int j = 0; j < 8; ++j) {
+    if (j == 7 && A.ml <= 7) {  // uniform: the 8th slot only when some row has 8 entries
+      A.xj[7] = 0.0;
+      break;
+    }
     if (ABFT_EXP == 6)  // timing experiment only: no x gathers (wrong results)
       A.xj[j] = (double)ac[j];
     else
@@ -457,12 +465,19 @@ __device__ __forceinline__ void short_finish(const SpmvArgs &a, const StreamCfg 
   const int64_t g = A.g, i = g * 32 + lane;
   const double *av = reinterpret_cast<const double *>(A.st + c.off_av) + A.rs;
   double v[8];
+  double yv;
+  if (A.uni && A.ml == 7) {  // every row 7 entries (7-pt interior): PW of 7 leaves
 #pragma unroll
-  for (int j = 0; j < 8; ++j) {
-    const double pr = dmul(av[j], A.xj[j]);
-    v[j] = j < A.len ? pr : kAbsent;  // absent leaves (R2): no branches
+    for (int j = 0; j < 7; ++j) v[j] = dmul(av[j], A.xj[j]);
+    yv = dadd(dadd(dadd(v[0], v[1]), dadd(v[2], v[3])), dadd(dadd(v[4], v[5]), v[6]));
+  } else {
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      const double pr = dmul(av[j], A.xj[j]);
+      v[j] = j < A.len ? pr : kAbsent;  // absent leaves (R2): no branches
+    }
+    yv = A.len > 0 ? tree<8>(v) : 0.0;  // PW of an empty row is +0.0 (R2)
   }
-  double yv = A.len > 0 ? tree<8>(v) : 0.0;  // PW of an empty row is +0.0 (R2)
   InjRange R{0, 0, 0, 0, 0, 0};
   if (INJECT) R = inj_range_group(a.inj, g, lane);
   if (INJECT && R.y0 < R.y1) yv = apply_mask(yv, list_mask_in(a.inj, R.y0, R.y1, list_key(0, 0, i)));
@@ -478,7 +493,8 @@ __device__ __forceinline__ void short_finish(const SpmvArgs &a, const StreamCfg 
   const int32_t W[8] = {w0.x, w0.y, w0.z, w0.w, w1.x, w1.y, w1.z, w1.w};
   // x_j -> C position W[j] + lane (slots past the row land in the trash)
 #pragma unroll
-  for (int j = 0; j < 8; ++j) sts_f64(xs + 8u * xs_phys(W[j] + lane), A.xj[j]);
+  for (int j = 0; j < 7; ++j) sts_f64(xs + 8u * xs_phys(W[j] + lane), A.xj[j]);
+  if (A.ml > 7) sts_f64(xs + 8u * xs_phys(W[7] + lane), A.xj[7]);
   const int npad = (-nC) & 7;  // positions nC .. roundup8(nC)-1 hold -0.0 (R2)
   if (lane < npad) sts_f64(xs + 8u * xs_phys(nC + lane), kAbsent);
   __syncwarp();
@@ -541,9 +557,11 @@ __global__ void __launch_bounds__((kStreamMaxG + 1) * 32, 2) k_stream(const Spmv
   // zero-fill the ring once: slots past a chunk's copy hold valid column
   // indices (0, or a previous chunk's) for the unpredicated SHORT gathers
   {
-    const uint32_t words = (uint32_t)NS * c.stage_bytes / 16u;
-    int4 *r4 = reinterpret_cast<int4 *>(ring);
-    for (uint32_t q = threadIdx.x; q < words; q += blockDim.x) r4[q] = make_int4(0, 0, 0, 0);
+    const uint32_t words = (c.stage_bytes - c.off_ac) / 16u;
+    for (int s = 0; s < NS; ++s) {
+      int4 *r4 = reinterpret_cast<int4 *>(ring + (size_t)s * c.stage_bytes + c.off_ac);
+      for (uint32_t q = threadIdx.x; q < words; q += blockDim.x) r4[q] = make_int4(0, 0, 0, 0);
+    }
   }
   if (threadIdx.x == 0) {
     for (int s = 0; s < NS; ++s) {
@@ -584,7 +602,7 @@ __global__ void __launch_bounds__((kStreamMaxG + 1) * 32, 2) k_stream(const Spmv
       t += gridDim.x;
       const int32_t qn = (q >= 0 && t < a.n_clist) ? __ldg(a.clist + t) : -1;
       if (wrapped)  // stage reuse: wait until its consumers released it
-        while (!mbar_try_wait(empty + s, eph)) __nanosleep(32);
+        mbar_wait_sleep(empty + s, eph);
       if (q < 0) {
         if (lane == 0) {
           hdr[3 * G + 3] = -1;
@@ -644,7 +662,7 @@ __global__ void __launch_bounds__((kStreamMaxG + 1) * 32, 2) k_stream(const Spmv
     // loads the next stage's group into one state and finishes the other
     const double *xg = a.x;
     ShortA sa, sb;
-    mbar_wait(full + s, fph);
+    mbar_wait_sleep(full + s, fph);
     {
       const int32_t *hdr = reinterpret_cast<const int32_t *>(ring + (size_t)s * c.stage_bytes);
       const int32_t g0 = hdr[3 * G + 3];
@@ -664,7 +682,7 @@ __global__ void __launch_bounds__((kStreamMaxG + 1) * 32, 2) k_stream(const Spmv
         fph1 ^= 1u;
       }
       const unsigned char *st1 = ring + (size_t)s1 * c.stage_bytes;
-      mbar_wait(full + s1, fph1);
+      mbar_wait_sleep(full + s1, fph1);
       const int32_t *hdr1 = reinterpret_cast<const int32_t *>(st1);
       const int32_t g0n = hdr1[3 * G + 3];
       nx.g = -1;
@@ -682,7 +700,7 @@ __global__ void __launch_bounds__((kStreamMaxG + 1) * 32, 2) k_stream(const Spmv
   } else {
     for (;;) {
       const unsigned char *st = ring + (size_t)s * c.stage_bytes;
-      mbar_wait(full + s, fph);
+      mbar_wait_sleep(full + s, fph);
       const int32_t *hdr = reinterpret_cast<const int32_t *>(st);
       const int32_t g0 = hdr[3 * G + 3];
       if (g0 < 0) break;
