@@ -297,16 +297,32 @@ def run_reference(args):
     print(json.dumps(line), flush=True)
 
 
+def nccl_dist(ranges, world, rank):
+    """abft_dist_t over an NCCL communicator the library owns; rank 0's
+    unique id travels over the torch.distributed group (plumbing only)."""
+    from paper_conf_dsn_schollbkw16_b200 import Dist, dist_unique_id
+    from paper_conf_dsn_schollbkw16_b200 import parallel as PL
+    nid = dist_unique_id() if rank == 0 else None
+    if world > 1:
+        import torch.distributed as dist
+        box = [nid]
+        dist.broadcast_object_list(box, src=0)
+        nid = box[0]
+    return Dist(rank, world, PL.ranges_array(ranges), nid)
+
+
 def run_pcg_dist(args):
     """configs[4] sharded: the 192^3 PCG split into 192/N-plane
-    slabs, one per rank (strong scaling: the total problem is fixed).  Every
-    SpMV is the distributed protected one (x halo over NCCL P2P + beta
-    partials all-gathered); every PCG reduction is an all-gather of 3 doubles
-    per rank finished in rank order on the device (abft_pcg_dist_*).  Fault
-    free; time-to-solution on the device (CUDA events, max over ranks) for the
-    method and for unprotected SpMVs on the same path."""
+    slabs, one per rank (strong scaling: the total problem is fixed).  The
+    whole solve is abft_dist_pcg: every SpMV is the library's distributed
+    protected SpMV (halo + beta partial in one NCCL group, interior blocks
+    overlapping it), every PCG reduction an NCCL all-gather of 3 doubles per
+    rank finished in rank order on the device.  Time-to-solution on the
+    device (CUDA events, max over ranks) for the method, unprotected SpMVs on
+    the same path, the single-reduction variant, and rate-mode faults."""
     import torch
 
+    from paper_conf_dsn_schollbkw16_b200 import Inject
     from paper_conf_dsn_schollbkw16_b200 import inputs as G
     from paper_conf_dsn_schollbkw16_b200 import parallel as PL
     world, rank, local = dist_init()
@@ -316,55 +332,34 @@ def run_pcg_dist(args):
     ranges = [(z0 * plane, z1 * plane) for z0, z1 in ranges_z]
     a, b_ = ranges[rank]
     rows = G.stencil_rows("7pt", n3, n3, n3, *ranges_z[rank])
-    sh = PL.make_shard(rows, a, b_, rank, world, ranges)
-    if world > 1:
-        comm = PL.TorchDistComm()
-        PL.plan_from_needs(sh, comm.gather_needs(sh))
-    d = PL.DistSpmv(sh, args.block_size, args.max_rounds)
+    d = nccl_dist(ranges, world, rank)
+    ds = PL.DistSpmv(d, rows, args.block_size, args.max_rounds)
     n_glob = n3 ** 3
     # b = A x* (x* seeded, R15/Q20) through the library's plain SpMV
-    d.own().copy_(torch.from_numpy(G.uniform_vector(sh.n, 43, start=a)))
-    class _Solo:  # world 1: no halo, partials need no exchange
-        def gather_partials(self, part, out):
-            out.copy_(part)
-
-        def halo(self, sh_, x_ext):
-            pass
-
-    c = comm if world > 1 else _Solo()
-    b = d.plain(c).clone()
-    x0 = torch.from_numpy(G.uniform_vector(sh.n, 44, start=a)).cuda()
+    xs = torch.from_numpy(G.uniform_vector(ds.sh.n, 43, start=a)).cuda()
+    b = ds.plain(x_own=xs).clone()
+    x0 = torch.from_numpy(G.uniform_vector(ds.sh.n, 44, start=a)).cuda()
     torch.cuda.synchronize()
     res = {}
-    from paper_conf_dsn_schollbkw16_b200 import Inject
     schemes = [("unprotected", False, "pcg", 0.0), ("protected", True, "pcg", 0.0),
                ("unprotected_cg1", False, "cg1", 0.0), ("protected_cg1", True, "cg1", 0.0)]
     for lam in ((1e-8, 1e-6) if args.lam <= 0 else (args.lam,)):
         schemes += [(f"protected_lam{lam:g}", True, "pcg", lam),
                     (f"protected_cg1_lam{lam:g}", True, "cg1", lam)]
-    # CUDA-graph replay of 16-iteration batches, cached across solves on the
-    # same buffers: default at N = 1; at N > 1 on request (ABFT_PCG_GRAPH=1:
-    # NCCL capture is untested on this one-GPU pool).  DESIGN.md §8.
-    graph = os.environ.get("ABFT_PCG_GRAPH", "1" if world == 1 else "0") == "1"
-    if graph:
-        schemes += [("unprotected_eager", False, "pcg", -1.0), ("protected_eager", True, "pcg", -1.0)]
     for name, check, variant, lam in schemes:
-        eager = lam < 0
-        lam = max(lam, 0.0)
         # rate-mode faults per arithmetic op in every rank's SpMVs
         inj = (lambda call, lam=lam: Inject.rate(seed=1000 * rank + 7, lam=lam, call=call)) \
             if lam > 0 else None
-        p = PL.DistPcg(d, check, variant, inj)
+        p = PL.DistPcg(ds, check, variant, inj)
         times = []
-        x = torch.empty_like(x0)  # one solution buffer: a captured graph is reused
-        for rep in range(max(1, args.pcg_reps) + 1):  # first: warm-up (and graph capture)
+        x = torch.empty_like(x0)
+        for rep in range(max(1, args.pcg_reps) + 1):  # first: warm-up
             x.copy_(x0)
             barrier(world)
             torch.cuda.synchronize()
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record()
-            state, st = p.solve(c, b, x, n_glob, tol=1e-6,
-                                graph=graph and lam == 0 and not eager)
+            state, st = p.solve(None, b, x, n_glob, tol=1e-6)
             e1.record()
             torch.cuda.synchronize()
             barrier(world)
@@ -377,55 +372,67 @@ def run_pcg_dist(args):
                      "uncorrected_calls_rank0": st["uncorrected_calls"]}
     for k, v in res.items():
         if k.startswith("protected"):
-            base = res["unprotected_cg1" if "cg1" in k else
-                       ("unprotected_eager" if "eager" in k else "unprotected")]["ms"]
+            base = res["unprotected_cg1" if "cg1" in k else "unprotected"]["ms"]
             v["overhead_pct"] = round((v["ms"] / base - 1) * 100, 2)
     if rank == 0:
         print(json.dumps({"metric": "PCG time-to-solution (ms), Jacobi, tol 1e-6, sharded",
                           "workload": f"3-D 7-point Laplacian {n3}^3 (BASELINE configs[4])",
                           "n": n_glob, "n_gpus": world, "scaling": "strong",
                           "parallelism": f"rowblock{world}",
-                          "variants": "pcg = textbook (2 reductions + SpMV beta gather per "
-                                      "iteration); cg1 = single reduction (Chronopoulos-Gear, "
-                                      "1 reduction + SpMV beta gather, one extra SpMV)",
-                          "graph": "fault-free schemes replay a CUDA graph of 16 iterations, "
-                                   "captured in the warm-up solve and reused (*_eager: "
-                                   "host-sequenced)" if graph else "none",
-                          "backend": os.environ.get("ABFT_DIST_BACKEND", "nccl") if world > 1
-                          else "none", "results": res}), flush=True)
+                          "api": "abft_dist_pcg (NCCL inside libabft.so)",
+                          "variants": "pcg = textbook (2 reductions + the SpMV's beta partial per "
+                                      "iteration); cg1 = single reduction (Chronopoulos-Gear)",
+                          "results": res}), flush=True)
+    if world > 1:
+        import torch.distributed as dist
+        dist.destroy_process_group()
 
 
 def run_ours_dist(args):
-    """N > 1: weak scaling.  Rank r owns planes [r*nz, (r+1)*nz) of a
-    (nz*N) x ny x nx grid of the workload's stencil (the configs[1] 128^3 slab
-    per rank); one step = halo exchange (NCCL P2P) + fused multiply+detect +
-    beta partial + all-gather (NCCL) + finish/correct."""
+    """N > 1 (or --strong): row-block shards through the library's NCCL path
+    (abft_dist_spmv: pack + one NCCL group carrying the halo and the beta
+    partials, interior blocks overlapping it, boundary blocks, finish).
+    Weak scaling (default): rank r owns planes [r*nz, (r+1)*nz) of a
+    (nz*N) x ny x nx grid of the workload's stencil (the single-GPU workload
+    per rank).  --strong: the workload's global grid (configs[3]: 27-pt
+    256^3) split into N z-slabs."""
     import torch
 
+    from paper_conf_dsn_schollbkw16_b200 import AUTOCORRECT, CHECK, NOCHECK
     from paper_conf_dsn_schollbkw16_b200 import inputs as G
     from paper_conf_dsn_schollbkw16_b200 import parallel as PL
     world, rank, local = dist_init()
     kind, nx = {"7pt128": ("7pt", 128), "27pt128": ("27pt", 128), "27pt256": ("27pt", 256),
                 "5pt64": ("5pt", 64)}[args.workload]
-    ny, nzl = (nx, nx) if kind != "5pt" else (nx, 1)
-    nz = nzl * world
+    ny = nx if kind != "5pt" else nx
+    if args.strong:
+        nz = nx if kind != "5pt" else 1
+        zr = [(nz * r // world, nz * (r + 1) // world) for r in range(world)]
+    else:
+        nzl = nx if kind != "5pt" else 1
+        nz = nzl * world
+        zr = [(r * nzl, (r + 1) * nzl) for r in range(world)]
     plane = nx * ny
-    ranges = [(r * nzl * plane, (r + 1) * nzl * plane) for r in range(world)]
+    ranges = [(z0 * plane, z1 * plane) for z0, z1 in zr]
     a, b = ranges[rank]
-    rows = G.stencil_rows(kind, nx, ny, nz, rank * nzl, (rank + 1) * nzl)
-    sh = PL.make_shard(rows, a, b, rank, world, ranges)
-    comm = PL.TorchDistComm()
-    PL.plan_from_needs(sh, comm.gather_needs(sh))
-    d = PL.DistSpmv(sh, args.block_size, args.max_rounds)
-    d.own().copy_(torch.from_numpy(G.uniform_vector(sh.n, 42, start=a)))
-    info = d.h.info()
+    rows = G.stencil_rows(kind, nx, ny, nz, *zr[rank])
+    d = nccl_dist(ranges, world, rank)
+    ds = PL.DistSpmv(d, rows, args.block_size, args.max_rounds)
+    h = ds.h
+    xo = torch.from_numpy(G.uniform_vector(ds.sh.n, 42, start=a)).cuda()
+    ds.set_own(xo)
+    info = h.info()
     torch.cuda.synchronize()
 
     def step():
-        d.spmv(comm)
+        h.dist_spmv(None, ds.y, mode=CHECK | AUTOCORRECT)
+
+    def plain():
+        h.dist_spmv(None, ds.y, mode=NOCHECK)
 
     for _ in range(max(args.warmup, 3)):
         step()
+        plain()
     torch.cuda.synchronize()
     clocks = ClockSampler(torch.cuda.current_device())
     clocks.start()
@@ -435,49 +442,59 @@ def run_ours_dist(args):
             step()
         torch.cuda.synchronize()
     ms = timed(step, args.steps, world)
+    ms_plain = timed(plain, args.steps, world)
     clk = clocks.stop()
-    # local bytes: A rows + own x + halo x + y + C + K
-    nbytes = (12 * sh.csr.nnz + 4 * (sh.n + 1) + 8 * sh.n_cols + 8 * sh.n + info["c_bytes"]
-              + 8 * info["nb"])
+    halo = h.n_cols - ds.sh.n
+    if info.get("stream"):
+        nb_plain = info["stream_plain_bytes"] + 8 * halo
+        nbytes = nb_plain + info["stream_check_bytes"]
+    else:
+        nb_plain = 12 * rows.nnz + 4 * (ds.sh.n + 1) + 8 * h.n_cols + 8 * ds.sh.n
+        nbytes = nb_plain + info["c_bytes"] + 8 * info["nb"]
     value = world * nbytes / (ms * 1e-3) / 1e9
     # end to end: host x slice in, host y slice out, per rank
-    xh = torch.from_numpy(G.uniform_vector(sh.n, 42, start=a)).pin_memory()
-    yh = torch.empty(sh.n, dtype=torch.float64).pin_memory()
+    xh = torch.from_numpy(G.uniform_vector(ds.sh.n, 42, start=a)).pin_memory()
+    yh = torch.empty(ds.sh.n, dtype=torch.float64).pin_memory()
     k_e2e = max(3, min(args.steps, 100))
     barrier(world)
     t0 = time.perf_counter()
     for _ in range(k_e2e):
-        d.own().copy_(xh, non_blocking=True)
-        step()
-        yh.copy_(d.y, non_blocking=True)
+        xd = xh.cuda(non_blocking=True)
+        h.dist_spmv(xd, ds.y, mode=CHECK | AUTOCORRECT)
+        yh.copy_(ds.y, non_blocking=True)
         torch.cuda.synchronize()
     dt_e2e = max_over_ranks((time.perf_counter() - t0) / k_e2e, world)
     peak, peak_src = load_peaks()
+    scaling = "strong" if args.strong else "weak"
     if rank == 0:
         print(json.dumps({
             "metric": METRIC, "value": round(value, 2), "unit": "GB/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms, 5),
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+            "higher_is_better": True, "scaling": scaling, "vs_baseline": None, "dtype": "f64",
             "data": "synthetic",
-            "config": {"workload": f"{kind} stencil {nx}x{ny}x{nzl} rows per GPU, "
-                                   f"global {nx}x{ny}x{nz}, row-block sharded",
-                       "rows_per_gpu": sh.n, "nnz_per_gpu": sh.csr.nnz,
+            "config": {"workload": f"{kind} stencil {nx}x{ny}x{nz}, row-block sharded into "
+                                   f"{world} z-slabs ({scaling} scaling)",
+                       "rows_per_gpu": ds.sh.n, "nnz_per_gpu": rows.nnz,
                        "parallelism": f"rowblock{world}", "c_format": info["c_format_name"],
                        "l2": "no flush: per-GPU working set > L2",
-                       "step": "halo (NCCL P2P) + k_lean (DEFER) + beta partial + all-gather "
-                               "(NCCL) + k_finish",
-                       "bytes_per_step_per_gpu": nbytes},
+                       "step": "abft_dist_spmv: k_dist_pack + NCCL group (halo send/recv + "
+                               "beta partial all-gather) || interior blocks; beta, boundary "
+                               "blocks, k_finish",
+                       "bytes_per_step_per_gpu": nbytes, "halo_doubles_per_gpu": halo},
+            "ft_overhead_pct": round((ms / ms_plain - 1) * 100, 2), "plain_ms": round(ms_plain, 5),
             "roofline": {"bound": "hbm", "kernel": "whole step", "achieved": round(value / world, 2),
                          "peak": peak, "unit": "GB/s", "frac": round(value / world / peak, 4),
                          "traffic": None, "peak_source": peak_src},
             "cpu_baseline": None,
             "e2e": {"value": round(world * nbytes / dt_e2e / 1e9, 3), "unit": "GB/s",
-                    "h2d_bytes_per_step": 8 * sh.n * world, "d2h_bytes_per_step": 8 * sh.n * world,
+                    "h2d_bytes_per_step": 8 * ds.sh.n * world,
+                    "d2h_bytes_per_step": 8 * ds.sh.n * world,
                     "ms_per_step": round(dt_e2e * 1e3, 4)},
-            "gpu_launches": args.steps * 5,
+            "gpu_launches": args.steps * 6,
             "clocks": clk}), flush=True)
-    import torch.distributed as dist
-    dist.destroy_process_group()
+    if world > 1:
+        import torch.distributed as dist
+        dist.destroy_process_group()
 
 
 def run_ours(args):
@@ -749,6 +766,9 @@ def main():
     ap.add_argument("--compare", action="store_true",
                     help="SURVEY §8(f)1: the method vs the dense check + complete recomputation")
     ap.add_argument("--pcg-n", type=int, default=192)
+    ap.add_argument("--strong", action="store_true",
+                    help="strong scaling through the sharded path: the workload's global grid "
+                         "(27pt256 = configs[3]) split over the ranks (also at N = 1)")
     ap.add_argument("--pcg-reps", type=int, default=3)
     ap.add_argument("--pcg-seeds", type=int, default=3, help="fault seeds per (scheme, lambda)")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
@@ -762,7 +782,7 @@ def main():
         run_pcg(args)
     elif args.compare:
         run_compare(args)
-    elif int(os.environ.get("WORLD_SIZE", "1")) > 1:
+    elif int(os.environ.get("WORLD_SIZE", "1")) > 1 or args.strong:
         run_ours_dist(args)
     else:
         run_ours(args)

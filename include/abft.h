@@ -45,7 +45,8 @@ typedef enum {
   ABFT_ENOTSUP = -4,       /* unsupported configuration (e.g. block_size > 1024) */
   ABFT_ENOCONV = -5,       /* PCG: not converged within max_iter */
   ABFT_EUNCORRECTED = -6,  /* blocks still flagged after max_rounds recomputations */
-  ABFT_EBREAKDOWN = -7     /* PCG: p.q <= 0 or NaN residual */
+  ABFT_EBREAKDOWN = -7,    /* PCG: p.q <= 0 or NaN residual */
+  ABFT_ENCCL = -8          /* NCCL error (multi-GPU; see abft_last_cuda_error) */
 } abft_status;
 
 /* CSR matrix, DEVICE arrays. row_ptr[n+1], col_idx[nnz], val[nnz].
@@ -320,6 +321,94 @@ abft_status abft_pcg_dist_combine(abft_handle_t h, int32_t phase, int64_t iter,
                                   const double *recv, int32_t world, void *stream);
 abft_status abft_pcg_dist_status(abft_handle_t h, int32_t *state, abft_pcg_stats_t *stats,
                                  void *stream);
+
+/* --- Multi-GPU: row-block shards inside the library (
+ * DESIGN.md §8) ---
+ * The paper runs one GPU; the split follows north_star: contiguous
+ * row ranges, one rank per GPU, one exchange per SpMV (the x halo) plus the
+ * all-gather of each rank's ||x||^2 partial (8 bytes per rank) that makes
+ * beta = sqrt(PW over the ranks, in rank order, of each rank's PW over its own
+ * rows) -- bit-identical to one GPU for equal power-of-two ranges (R28).
+ * Row blocks never straddle ranks (row boundaries multiples of block_size),
+ * so C, detection and correction stay rank-local.
+ *
+ * abft_dist_unique_id: a 128-byte NCCL unique id (host); rank 0 makes it and
+ *   the caller broadcasts it (torch.distributed, MPI, a file ...).
+ * abft_dist_create: ranges = host int64 [world + 1] row boundaries (ranges[0]
+ *   = 0, ranges[world] = n_global, non-decreasing); nccl_id = the 128-byte id
+ *   (host) -> an NCCL communicator over the `world` ranks (collective: every
+ *   rank calls it; the current device is this rank's GPU), or NULL -> no
+ *   communicator: the caller moves the exchange buffers itself
+ *   (abft_dist_begin / abft_dist_buffers / abft_dist_end; tests, other
+ *   transports).  The dist object must outlive its handles.
+ * abft_dist_encode: this rank's rows as CSR with GLOBAL column indices (n =
+ *   ranges[rank+1] - ranges[rank] rows, n_cols / x_offset ignored).  Builds
+ *   the local column order [halo below | own | halo above] (global order, so
+ *   every sum sees the single-GPU operands in the single-GPU order), a
+ *   handle-owned copy of the renumbered columns (row_ptr and values stay the
+ *   caller's and must outlive the handle), the halo plan (per peer: the
+ *   contiguous slice of the extended operand it fills, and the own entries
+ *   it needs), the checksum encoding of the local rows (as abft_encode), and
+ *   the split of the blocks into interior (no halo column) and boundary
+ *   ones.  With a communicator the ranks exchange their needs over NCCL
+ *   (collective); without one the caller reads abft_dist_needs and sets
+ *   abft_dist_set_send for every peer.  Synchronises.
+ * abft_dist_operand: device pointer to the handle's halo-extended operand
+ *   (n_cols doubles) and the offset of the own slice; a caller (the PCG) may
+ *   write its own x there directly.
+ * abft_dist_spmv (communicator only): one distributed protected SpMV of the
+ *   own x (device [n_own]; NULL = already in the operand's own slice) into
+ *   y (device [n_own]); mode / inj as abft_spmv (fault indices rank-local).
+ *   Enqueues on `stream`: the pack kernel (send buffer + x^2 partial), the
+ *   NCCL group (halo send/recv + partial all-gather) on the handle's comm
+ *   stream, the interior blocks meanwhile, then beta, the boundary blocks,
+ *   the finish and the corrections.  Asynchronous; collective.
+ * abft_dist_begin / abft_dist_end (either mode; abft_dist_spmv = begin +
+ *   exchange + end): begin copies x_own into the operand (unless NULL) and
+ *   packs the send buffers and the partial; the caller then delivers, for
+ *   every peer p, p's send buffer for this rank into this rank's receive
+ *   slice for p (abft_dist_buffers, device pointers, counts in doubles) and
+ *   all ranks' partials, in rank order, into a device array parts[world]
+ *   (abft_dist_partial); end runs the fused kernels, the finish and the
+ *   corrections with beta = sqrt(PW(parts)).
+ * abft_dist_pcg (communicator only): the distributed Jacobi-PCG of
+ *   abft_pcg_dist_* with every exchange (halo, beta, dot partials) inside
+ *   the library; b, x own rows (device), diag nullable, max_iter <= 0 -> 10 N
+ *   of the global matrix; inj->call counts this rank's SpMVs (rate mode: the
+ *   seed is the caller's, e.g. distinct per rank); variant 0 = textbook
+ *   PCG (two reductions per iteration), 1 = single reduction (R29).
+ *   Synchronises; every rank returns the same status.
+ * abft_halo_plan (host only, no GPU): the local column order of abft_dist_
+ *   encode for host arrays -- local_col [nnz], *n_below / *n_above, per peer
+ *   recv_start / recv_count [world], halo = the global index of every halo
+ *   column in operand order (capacity cap; NULL with cap 0 to count only). */
+typedef struct abft_dist *abft_dist_t;
+abft_status abft_dist_unique_id(void *nccl_id);
+abft_status abft_dist_create(int32_t rank, int32_t world, const int64_t *ranges,
+                             const void *nccl_id, abft_dist_t *out);
+abft_status abft_dist_destroy(abft_dist_t d);
+abft_status abft_dist_encode(abft_dist_t d, const abft_csr_t *A_rows, int32_t block_size,
+                             int32_t max_rounds, uint32_t flags, void *stream, abft_handle_t *out);
+abft_status abft_dist_needs(abft_handle_t h, int32_t peer, int64_t *count, int64_t *global_idx);
+abft_status abft_dist_set_send(abft_handle_t h, int32_t peer, const int64_t *global_idx,
+                               int64_t count);
+abft_status abft_dist_operand(abft_handle_t h, double **x_ext, int64_t *n_cols,
+                              int64_t *own_offset);
+abft_status abft_dist_spmv(abft_handle_t h, const double *x_own, double *y,
+                           const abft_inject_t *inj, uint32_t mode, void *stream);
+abft_status abft_dist_begin(abft_handle_t h, const double *x_own, void *stream);
+abft_status abft_dist_buffers(abft_handle_t h, int32_t peer, const double **send,
+                              int64_t *send_count, double **recv, int64_t *recv_count);
+abft_status abft_dist_partial(abft_handle_t h, const double **part);
+abft_status abft_dist_end(abft_handle_t h, double *y, const double *parts,
+                          const abft_inject_t *inj, uint32_t mode, void *stream);
+abft_status abft_dist_pcg(abft_handle_t h, const double *b, double *x, const double *diag,
+                          double tol, int64_t max_iter, const abft_inject_t *inj, int32_t check,
+                          int32_t variant, double *res_hist, abft_pcg_stats_t *stats,
+                          void *stream);
+abft_status abft_halo_plan(int32_t rank, int32_t world, const int64_t *ranges, const int32_t *col,
+                           int64_t nnz, int32_t *local_col, int64_t *n_below, int64_t *n_above,
+                           int64_t *recv_start, int64_t *recv_count, int64_t *halo, int64_t cap);
 
 /* --- Related-work baseline: DENSE CHECK [30, 31] + COMPLETE RECOMPUTATION ---
  * (eq. (1), P:148-152 [35]'s bound, P:240, P:250-252,

@@ -10,6 +10,28 @@ CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "libabft.so")
 ROOT = os.path.dirname(PKG)
 
+def nccl_dir() -> str:
+    """NCCL headers + library: the wheel torch itself loads (one libnccl.so.2
+    per process), else the system copy."""
+    try:
+        import nvidia
+        for base in list(nvidia.__path__):
+            d = os.path.join(base, "nccl")
+            if os.path.exists(os.path.join(d, "include", "nccl.h")):
+                return d
+    except Exception:  # noqa: BLE001
+        pass
+    return "/usr"
+
+
+def nccl_flags() -> list:
+    d = nccl_dir()
+    inc, lib = os.path.join(d, "include"), os.path.join(d, "lib")
+    if d == "/usr":
+        lib = "/usr/lib/x86_64-linux-gnu"
+    return ["-I" + inc, "-L" + lib, "-Xlinker", "-rpath," + lib, "-l:libnccl.so.2"]
+
+
 NVCC_FLAGS = [
     "-gencode", "arch=compute_100a,code=sm_100a",
     "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-ffp-contract=off",
@@ -44,7 +66,7 @@ def nvcc() -> str:
 def build(force: bool = False, verbose: bool = False) -> str:
     if not force and not needs_build():
         return LIB
-    cmd = [nvcc(), *NVCC_FLAGS, "-o", LIB + ".tmp", os.path.join(CSRC, "abft.cu")]
+    cmd = [nvcc(), *NVCC_FLAGS, "-o", LIB + ".tmp", os.path.join(CSRC, "abft.cu"), *nccl_flags()]
     if verbose:
         cmd.insert(1, "-Xptxas=-v")
     subprocess.check_call(cmd)

@@ -17,7 +17,8 @@ from . import _build
 
 _LIB = None
 
-OK, EINVAL, ECUDA, ENOMEM, ENOTSUP, ENOCONV, EUNCORRECTED, EBREAKDOWN = 0, -1, -2, -3, -4, -5, -6, -7
+OK, EINVAL, ECUDA, ENOMEM, ENOTSUP, ENOCONV, EUNCORRECTED, EBREAKDOWN, ENCCL = (
+    0, -1, -2, -3, -4, -5, -6, -7, -8)
 NOCHECK, CHECK, AUTOCORRECT, DEBUG_CHECKSUMS, DEFER_FINISH = 0, 1, 2, 4, 8
 DENSE_BOUND35 = 16  # abft_spmv_dense: tau = K35 ||x|| ([35]) instead of ||x|| ([30])
 INJ_NONE, INJ_LIST, INJ_RATE = 0, 1, 2
@@ -31,6 +32,10 @@ SYMBOLS = [
     "abft_spmv_host_pipelined", "abft_host_alloc", "abft_host_free",
     "abft_pcg_dist_begin", "abft_pcg_dist_local", "abft_pcg_dist_combine",
     "abft_pcg_dist_status", "abft_poisson_table", "abft_rate_chunk", "abft_health",
+    "abft_dist_unique_id", "abft_dist_create", "abft_dist_destroy", "abft_dist_encode",
+    "abft_dist_needs", "abft_dist_set_send", "abft_dist_operand", "abft_dist_spmv",
+    "abft_dist_begin", "abft_dist_buffers", "abft_dist_partial", "abft_dist_end", "abft_dist_pcg",
+    "abft_halo_plan",
 ]
 PCG_PHASE_INIT, PCG_PHASE_DOT, PCG_PHASE_UPDATE, PCG_PHASE_P = 0, 1, 2, 3
 PCG_PHASE_CG1_UPDATE, PCG_PHASE_CG1_DOT = 4, 5  # single-reduction variant
@@ -162,6 +167,35 @@ def lib():
         L.abft_finish.restype = st
         L.abft_health.restype = st
         L.abft_health.argtypes = [P, P, C.POINTER(i32)]
+        PI64 = C.POINTER(i64)
+        L.abft_dist_unique_id.restype = st
+        L.abft_dist_unique_id.argtypes = [P]
+        L.abft_dist_create.restype = st
+        L.abft_dist_create.argtypes = [i32, i32, P, P, C.POINTER(P)]
+        L.abft_dist_destroy.restype = st
+        L.abft_dist_destroy.argtypes = [P]
+        L.abft_dist_encode.restype = st
+        L.abft_dist_encode.argtypes = [P, P, i32, i32, u32, P, C.POINTER(P)]
+        L.abft_dist_needs.restype = st
+        L.abft_dist_needs.argtypes = [P, i32, PI64, P]
+        L.abft_dist_set_send.restype = st
+        L.abft_dist_set_send.argtypes = [P, i32, P, i64]
+        L.abft_dist_operand.restype = st
+        L.abft_dist_operand.argtypes = [P, C.POINTER(P), PI64, PI64]
+        L.abft_dist_spmv.restype = st
+        L.abft_dist_spmv.argtypes = [P, P, P, P, u32, P]
+        L.abft_dist_begin.restype = st
+        L.abft_dist_begin.argtypes = [P, P, P]
+        L.abft_dist_buffers.restype = st
+        L.abft_dist_buffers.argtypes = [P, i32, C.POINTER(P), PI64, C.POINTER(P), PI64]
+        L.abft_dist_partial.restype = st
+        L.abft_dist_partial.argtypes = [P, C.POINTER(P)]
+        L.abft_dist_end.restype = st
+        L.abft_dist_end.argtypes = [P, P, P, P, u32, P]
+        L.abft_dist_pcg.restype = st
+        L.abft_dist_pcg.argtypes = [P, P, P, P, d, i64, P, i32, i32, P, C.POINTER(PcgStats), P]
+        L.abft_halo_plan.restype = st
+        L.abft_halo_plan.argtypes = [i32, i32, P, P, i64, P, PI64, PI64, P, P, P, i64]
         L.abft_finish.argtypes = [P, P, P, P, i32, i32, P, P]
         _LIB = L
     return _LIB
@@ -277,13 +311,16 @@ class Handle:
     re-reads it in correction and PCG)."""
 
     def __init__(self, A: CsrDevice, block_size: int = 32, max_rounds: int = 4, stream=None,
-                 c_csr: bool = False):
+                 c_csr: bool = False, _raw=None):
         self.A = A
         self.n = A.n
         self.n_cols = A.n_cols if A.n_cols > 0 else A.n
         self.block_size = block_size
         self.nb = (A.n + block_size - 1) // block_size
         self.max_rounds = max_rounds if max_rounds > 0 else 4
+        if _raw is not None:  # a handle the library built (abft_dist_encode)
+            self._h = _raw
+            return
         csr = _Csr(A.n, A.nnz, A.row_ptr.data_ptr(), A.col.data_ptr() if A.nnz else 0,
                    A.val.data_ptr() if A.nnz else 0, A.n_cols, A.x_offset)
         h = C.c_void_p()
@@ -475,7 +512,9 @@ class Handle:
     # -- distributed PCG steps (abft_pcg_dist_*; parallel.DistPcg drives them)
     def pcg_dist_begin(self, b, x, pext, q, diag=None, tol=1e-6, max_iter=1, check=True,
                        res_hist=None, stream=None):
-        _check(lib().abft_pcg_dist_begin(self._h, _ptr(b), _ptr(x), _ptr(pext), _ptr(q),
+        # pext / q: tensors or raw device pointers (the library-owned operand)
+        rp = lambda t: C.c_void_p(t) if isinstance(t, int) else _ptr(t)  # noqa: E731
+        _check(lib().abft_pcg_dist_begin(self._h, _ptr(b), _ptr(x), rp(pext), rp(q),
                                          _ptr(diag), tol, max_iter, 1 if check else 0,
                                          _ptr(res_hist), _stream(stream)), "abft_pcg_dist_begin")
 
@@ -492,6 +531,159 @@ class Handle:
         _check(lib().abft_pcg_dist_status(self._h, C.byref(state), C.byref(st),
                                           _stream(stream)), "abft_pcg_dist_status")
         return state.value, st.as_dict()
+
+
+# ---------------------------------------------------------------------------
+# Multi-GPU row-block shards (include/abft.h "Multi-GPU"): the halo plan, the
+# pack, the NCCL exchange and the distributed PCG run in the library.
+# ---------------------------------------------------------------------------
+def dist_unique_id() -> bytes:
+    buf = (C.c_char * 128)()
+    _check(lib().abft_dist_unique_id(buf), "abft_dist_unique_id")
+    return bytes(buf)
+
+
+def halo_plan(rank: int, world: int, ranges, col):
+    """Host-only local column order of a shard (abft_halo_plan): returns
+    (local_col, n_below, n_above, recv_start[world], recv_count[world], halo)."""
+    rg = np.ascontiguousarray(ranges, dtype=np.int64)
+    col = np.ascontiguousarray(col, dtype=np.int32)
+    nb, na = C.c_int64(), C.c_int64()
+    rs = np.zeros(world, np.int64)
+    rc = np.zeros(world, np.int64)
+    local = np.zeros(max(col.size, 1), np.int32)
+    _check(lib().abft_halo_plan(rank, world, rg.ctypes.data, col.ctypes.data, col.size,
+                                local.ctypes.data, C.byref(nb), C.byref(na), rs.ctypes.data,
+                                rc.ctypes.data, None, 0), "abft_halo_plan")
+    halo = np.zeros(max(nb.value + na.value, 1), np.int64)
+    _check(lib().abft_halo_plan(rank, world, rg.ctypes.data, col.ctypes.data, col.size,
+                                local.ctypes.data, C.byref(nb), C.byref(na), rs.ctypes.data,
+                                rc.ctypes.data, halo.ctypes.data, halo.size), "abft_halo_plan")
+    return local[:col.size], nb.value, na.value, rs, rc, halo[:nb.value + na.value]
+
+
+class Dist:
+    """abft_dist_t: this rank's place in the row partition and (nccl_id given)
+    an NCCL communicator over the ranks."""
+
+    def __init__(self, rank: int, world: int, ranges, nccl_id: bytes | None = None):
+        self.rank, self.world = rank, world
+        self.ranges = np.ascontiguousarray(ranges, dtype=np.int64)
+        assert self.ranges.size == world + 1
+        d = C.c_void_p()
+        idbuf = None
+        if nccl_id is not None:
+            idbuf = (C.c_char * 128).from_buffer_copy(nccl_id)
+        _check(lib().abft_dist_create(rank, world, self.ranges.ctypes.data, idbuf, C.byref(d)),
+               "abft_dist_create")
+        self._d = d
+        self.nccl = nccl_id is not None
+
+    @property
+    def row0(self):
+        return int(self.ranges[self.rank])
+
+    @property
+    def row1(self):
+        return int(self.ranges[self.rank + 1])
+
+    def encode(self, rows: "CsrDevice", block_size: int = 32, max_rounds: int = 4,
+               c_csr: bool = False, stream=None) -> "DistHandle":
+        """rows: this rank's rows, GLOBAL column indices (device CSR)."""
+        csr = _Csr(rows.n, rows.nnz, rows.row_ptr.data_ptr(),
+                   rows.col.data_ptr() if rows.nnz else 0,
+                   rows.val.data_ptr() if rows.nnz else 0, 0, 0)
+        h = C.c_void_p()
+        _check(lib().abft_dist_encode(self._d, C.byref(csr), block_size, max_rounds,
+                                      ENCODE_C_CSR if c_csr else 0, _stream(stream), C.byref(h)),
+               "abft_dist_encode")
+        return DistHandle(self, rows, block_size, max_rounds, h)
+
+    def close(self):
+        if getattr(self, "_d", None) and self._d.value:
+            lib().abft_dist_destroy(self._d)
+            self._d = C.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+class DistHandle(Handle):
+    """A shard handle from abft_dist_encode.  Device pointers of the
+    library-owned operand / exchange buffers are plain ints."""
+
+    def __init__(self, dist: Dist, rows, block_size, max_rounds, raw):
+        super().__init__(rows, block_size, max_rounds, _raw=raw)
+        self.dist = dist  # the communicator outlives the handle
+        x, nc, off = C.c_void_p(), C.c_int64(), C.c_int64()
+        _check(lib().abft_dist_operand(self._h, C.byref(x), C.byref(nc), C.byref(off)),
+               "abft_dist_operand")
+        self.x_ext_ptr, self.n_cols, self.own_offset = x.value, nc.value, off.value
+
+    def own_ptr(self) -> int:
+        return self.x_ext_ptr + 8 * self.own_offset
+
+    def needs(self, peer: int) -> np.ndarray:
+        c = C.c_int64()
+        _check(lib().abft_dist_needs(self._h, peer, C.byref(c), None), "abft_dist_needs")
+        out = np.zeros(max(c.value, 1), np.int64)
+        _check(lib().abft_dist_needs(self._h, peer, C.byref(c), out.ctypes.data), "abft_dist_needs")
+        return out[:c.value]
+
+    def set_send(self, peer: int, idx) -> None:
+        idx = np.ascontiguousarray(idx, dtype=np.int64)
+        _check(lib().abft_dist_set_send(self._h, peer, idx.ctypes.data if idx.size else None,
+                                        idx.size), "abft_dist_set_send")
+
+    def buffers(self, peer: int):
+        """(send ptr, send count, recv ptr, recv count) for `peer` (device)."""
+        sp, sc, rp, rc = C.c_void_p(), C.c_int64(), C.c_void_p(), C.c_int64()
+        _check(lib().abft_dist_buffers(self._h, peer, C.byref(sp), C.byref(sc), C.byref(rp),
+                                       C.byref(rc)), "abft_dist_buffers")
+        return sp.value, sc.value, rp.value, rc.value
+
+    def partial_ptr(self) -> int:
+        p = C.c_void_p()
+        _check(lib().abft_dist_partial(self._h, C.byref(p)), "abft_dist_partial")
+        return p.value
+
+    def begin(self, x_own=None, stream=None):
+        _check(lib().abft_dist_begin(self._h, _vec(x_own, self.n, "x_own", optional=True),
+                                     _stream(stream)), "abft_dist_begin")
+
+    def end(self, y, parts, inject: Inject | None = None, mode=CHECK | AUTOCORRECT, stream=None):
+        inj = inject.struct() if inject is not None else None
+        _check(lib().abft_dist_end(self._h, _vec(y, self.n, "y"),
+                                   _vec(parts, self.dist.world, "parts"),
+                                   C.byref(inj) if inj is not None else None, mode,
+                                   _stream(stream)), "abft_dist_end")
+        return y
+
+    def dist_spmv(self, x_own, y, inject: Inject | None = None, mode=CHECK | AUTOCORRECT,
+                  stream=None):
+        inj = inject.struct() if inject is not None else None
+        _check(lib().abft_dist_spmv(self._h, _vec(x_own, self.n, "x_own", optional=True),
+                                    _vec(y, self.n, "y"),
+                                    C.byref(inj) if inj is not None else None, mode,
+                                    _stream(stream)), "abft_dist_spmv")
+        return y
+
+    def dist_pcg(self, b, x, diag=None, tol=1e-6, max_iter=0, inject: Inject | None = None,
+                 check=True, res_hist=None, stream=None, variant="pcg"):
+        st = PcgStats()
+        inj = inject.struct() if inject is not None else None
+        status = lib().abft_dist_pcg(self._h, _vec(b, self.n, "b"), _vec(x, self.n, "x"),
+                                     _vec(diag, self.n, "diag", optional=True), tol, max_iter,
+                                     C.byref(inj) if inj is not None else None, 1 if check else 0,
+                                     1 if variant == "cg1" else 0,
+                                     _vec(res_hist, 1, "res_hist", optional=True), C.byref(st),
+                                     _stream(stream))
+        if status not in (OK, ENOCONV, EBREAKDOWN):
+            _check(status, "abft_dist_pcg")
+        return status, st.as_dict()
 
 
 class PinnedArray:

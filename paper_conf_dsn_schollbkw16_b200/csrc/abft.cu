@@ -16,6 +16,7 @@
 #include "kernels_irr.cuh"
 #include "kernels_dense.cuh"
 #include "kernels_bigblock.cuh"
+#include "kernels_dist.cuh"
 
 #include <cub/device/device_radix_sort.cuh>
 
@@ -181,6 +182,25 @@ struct abft_ctx {
   int64_t ncta256 = 0;  // ceil(n / kPcgRows): PCG vector-kernel grid
   abft::PcgArgs pcg_dist{};  // distributed PCG (abft_pcg_dist_*): set by _begin
   bool pcg_dist_on = false;
+  // multi-GPU shard (abft_dist_encode, abft_dist_api.inc)
+  struct abft_dist *dist = nullptr;
+  int64_t row0 = 0, n_below = 0, n_above = 0;
+  std::vector<int64_t> recv_start, recv_count;  // per peer: slice of the operand it fills
+  std::vector<int64_t> send_off;                // per peer: slice of send_idx / send_buf ([world + 1])
+  std::vector<std::vector<int64_t>> send_host;  // per peer: global indices it needs (set or exchanged)
+  std::vector<int64_t> halo_global;             // global index of every halo column (operand order)
+  double *x_ext = nullptr;                      // halo-extended operand [n_cols]
+  int32_t *send_idx = nullptr;                  // own-local index per send slot
+  double *send_buf = nullptr;
+  int64_t n_send = 0;
+  double *d_chunk = nullptr, *d_part = nullptr, *d_parts = nullptr, *d_xnorm = nullptr;
+  unsigned *d_ticket = nullptr;
+  double *y_dist = nullptr;                     // PCG: q = A p
+  double *pcg_send = nullptr, *pcg_recv = nullptr;
+  cudaStream_t cs = nullptr;                    // NCCL stream
+  cudaEvent_t ev_pack = nullptr, ev_comm = nullptr;
+  int32_t *clist_int = nullptr, *clist_bnd = nullptr;  // k_stream chunks without / with halo columns
+  int64_t n_int = 0, n_bnd = 0;
   std::vector<void *> owned;
   int device = 0;
   int num_sms = 148;
@@ -426,8 +446,16 @@ void launch_lean(const abft_ctx *h, const SpmvArgs &a, cudaStream_t s) {
 }
 
 template <bool CHECK, bool INJECT>
-void launch_stream(const abft_ctx *h, const SpmvArgs &a, cudaStream_t s) {
-  const dim3 grid(h->stream_grid), block((h->stc.G + 1) * 32);
+void launch_stream(const abft_ctx *h, const SpmvArgs &a_in, cudaStream_t s,
+                   const int32_t *list = nullptr, int64_t n_list = -1) {
+  SpmvArgs a = a_in;
+  if (list) {  // a subset of the eligible chunks (multi-GPU interior / boundary)
+    a.clist = list;
+    a.n_clist = n_list;
+  }
+  if (a.n_clist <= 0) return;
+  const dim3 grid((unsigned)std::min<int64_t>(h->stream_grid, a.n_clist)),
+      block((h->stc.G + 1) * 32);
   const size_t sm = h->stream_smem;
 #define STREAM(CF)                                                               \
   (h->pos_S <= 8 ? k_stream<CHECK, INJECT, CF, true><<<grid, block, sm, s>>>(a) \
@@ -1214,6 +1242,7 @@ const char *abft_status_string(abft_status st) {
     case ABFT_ENOCONV: return "PCG did not converge";
     case ABFT_EUNCORRECTED: return "blocks remain flagged after correction";
     case ABFT_EBREAKDOWN: return "PCG breakdown";
+    case ABFT_ENCCL: return "NCCL error";
   }
   return "unknown status";
 }
@@ -1229,6 +1258,12 @@ int64_t abft_rate_chunk(double lambda) { return FaultTables::chunk(lambda); }
 
 abft_status abft_destroy(abft_handle_t h) {
   if (!h) return ABFT_EINVAL;
+  if (h->cs) {
+    cudaStreamSynchronize(h->cs);
+    cudaStreamDestroy(h->cs);
+  }
+  if (h->ev_pack) cudaEventDestroy(h->ev_pack);
+  if (h->ev_comm) cudaEventDestroy(h->ev_comm);
   if (h->s_in) {
     cudaStreamSynchronize(h->s_in);
     cudaStreamSynchronize(h->s_out);
@@ -1627,3 +1662,4 @@ abft_status abft_memcpy(void *dst, const void *src, int64_t bytes, void *stream)
 
 #include "abft_pcg_api.inc"
 #include "abft_dense_api.inc"
+#include "abft_dist_api.inc"

@@ -107,152 +107,202 @@ def halo_needs(sh: Shard) -> dict:
 
 
 # ---------------------------------------------------------------------------
-# Exchange backends (x_ext: the local extended vector, a torch tensor)
+# Distributed protected SpMV on top of the C ABI (include/abft.h "Multi-GPU"):
+# the library builds the shard's column order and halo plan, packs the send
+# buffers with the x^2 partial, and -- with an NCCL communicator -- does the
+# exchange itself (abft_dist_spmv, abft_dist_pcg).  Without a communicator
+# (tests: logical ranks on one GPU, or processes over gloo) the exchange
+# classes below move the library's buffers: abft_dist_begin -> copies ->
+# abft_dist_end.
 # ---------------------------------------------------------------------------
-class TorchDistComm:
-    """Halo exchange with torch.distributed point-to-point (NCCL on GPUs,
-    gloo on CPU) and the beta partials with all_gather_into_tensor."""
-
-    def __init__(self, group=None):
-        import torch.distributed as dist
-        self.dist = dist
-        self.group = group
-        self.rank = dist.get_rank(group)
-        self.world = dist.get_world_size(group)
-        self._idx = {}
-        # gloo carries CPU tensors only: stage device buffers through the host
-        self.stage = dist.get_backend(group) != "nccl"
-
-    def halo(self, sh: Shard, x_ext) -> None:
-        import torch
-        stage = self.stage and x_ext.is_cuda
-        ops, bufs, recvs = [], [], []
-        for q, idx in sorted(sh.send.items()):
-            key = (id(sh), q, x_ext.device)
-            if key not in self._idx:
-                self._idx[key] = torch.as_tensor(idx, device=x_ext.device)
-            buf = x_ext.index_select(0, self._idx[key])
-            if stage:
-                buf = buf.cpu()
-            bufs.append(buf)
-            ops.append(self.dist.P2POp(self.dist.isend, buf, q, self.group))
-        for q, (start, count) in sorted(sh.recv.items()):
-            dst = x_ext[start:start + count]
-            if stage:
-                tmp = torch.empty(count, dtype=x_ext.dtype)
-                recvs.append((dst, tmp))
-                dst = tmp
-            ops.append(self.dist.P2POp(self.dist.irecv, dst, q, self.group))
-        if ops:
-            for w in self.dist.batch_isend_irecv(ops):
-                w.wait()
-        for dst, tmp in recvs:
-            dst.copy_(tmp)
-
-    def gather_partials(self, partial, out) -> None:
-        if self.stage and partial.is_cuda:
-            o = out.cpu()
-            self.dist.all_gather_into_tensor(o, partial.cpu(), group=self.group)
-            out.copy_(o)
-        else:
-            self.dist.all_gather_into_tensor(out, partial, group=self.group)
-
-    def gather_needs(self, sh: Shard) -> dict:
-        """All-to-all of halo needs (once, at setup)."""
-        mine = halo_needs(sh)
-        allneeds = [None] * self.world
-        self.dist.all_gather_object(allneeds, mine, group=self.group)
-        return {q: allneeds[q][sh.rank] for q in range(self.world)
-                if q != sh.rank and sh.rank in allneeds[q]}
+def shard_rows(A: G.CSR, a: int, b: int) -> G.CSR:
+    """Rows [a, b) of A with their GLOBAL column indices."""
+    return G.CSR(A.row_ptr[a:b + 1] - A.row_ptr[a], A.col[A.row_ptr[a]:A.row_ptr[b]],
+                 A.val[A.row_ptr[a]:A.row_ptr[b]])
 
 
-class LocalComm:
-    """All shards in one process (logical shards on one GPU, tests): the halo
-    is copied from the owners' extended vectors."""
-
-    def __init__(self, shards, xs):
-        self.shards = {s.rank: s for s in shards}
-        self.xs = xs  # rank -> x_ext tensor
-        self._idx = {}  # device index lists, uploaded once (graph capture safe)
-
-    def halo(self, sh: Shard, x_ext) -> None:
-        import torch
-        for q, (start, count) in sh.recv.items():
-            src = self.xs[q]
-            key = (q, sh.rank, src.device)
-            if key not in self._idx:
-                self._idx[key] = torch.as_tensor(self.shards[q].send[sh.rank], device=src.device)
-            x_ext[start:start + count] = src.index_select(0, self._idx[key])
+def ranges_array(ranges) -> np.ndarray:
+    """[(a, b), ...] -> the [world + 1] boundary array abft_dist_create takes."""
+    return np.array([ranges[0][0]] + [b for _, b in ranges], dtype=np.int64)
 
 
-# ---------------------------------------------------------------------------
-# Distributed protected SpMV on top of the C ABI
-# ---------------------------------------------------------------------------
+@dataclass
+class ShardInfo:
+    rank: int
+    world: int
+    row0: int
+    row1: int
+
+    @property
+    def n(self) -> int:
+        return self.row1 - self.row0
+
+
 class DistSpmv:
-    """One rank's protected SpMV: halo exchange, fused multiply+detect on the
-    local shard (ABFT_DEFER_FINISH), beta partial, all-gather, finish."""
+    """One rank's shard: a DistHandle over its rows (global columns), the
+    result y and the gathered partials (external exchange)."""
 
-    def __init__(self, shard: Shard, block_size: int = 32, max_rounds: int = 4,
+    def __init__(self, dist, rows: G.CSR, block_size: int = 32, max_rounds: int = 4,
                  device="cuda"):
         import torch
 
-        from .abft import CsrDevice, Handle
-        self.sh = shard
-        A = CsrDevice(shard.n, torch.from_numpy(shard.csr.row_ptr).to(device),
-                      torch.from_numpy(shard.csr.col).to(device),
-                      torch.from_numpy(shard.csr.val).to(device),
-                      n_cols=shard.n_cols, x_offset=shard.x_offset)
-        self.h = Handle(A, block_size, max_rounds)
+        from .abft import CsrDevice
+        self.dist = dist
+        self.sh = ShardInfo(dist.rank, dist.world, dist.row0, dist.row1)
+        self.A = CsrDevice(rows.n, torch.from_numpy(np.ascontiguousarray(rows.row_ptr)).to(device),
+                           torch.from_numpy(np.ascontiguousarray(rows.col)).to(device),
+                           torch.from_numpy(np.ascontiguousarray(rows.val)).to(device))
+        self.h = dist.encode(self.A, block_size, max_rounds)
         self.max_rounds = max_rounds
-        self.x_ext = torch.zeros(shard.n_cols, dtype=torch.float64, device=device)
-        self.y = torch.empty(shard.n, dtype=torch.float64, device=device)
-        self.parts = torch.empty(shard.world, dtype=torch.float64, device=device)
+        self.y = torch.empty(rows.n, dtype=torch.float64, device=device)
+        self.parts = torch.zeros(dist.world, dtype=torch.float64, device=device)
 
-    def own(self):
-        s = self.sh
-        return self.x_ext[s.x_offset:s.x_offset + s.n]
+    def own_ptr(self) -> int:
+        return self.h.own_ptr()
 
-    def step1(self, comm, inject=None):
-        """Halo + fused pass (steps 1-3) + this rank's beta partial."""
+    def set_own(self, x_own) -> None:
+        """Write this rank's x into the operand's own slice."""
+        from .abft import lib
+        lib().abft_memcpy(self.own_ptr(), x_own.data_ptr(), 8 * self.sh.n, None)
+
+    def spmv(self, exchange=None, x_own=None, inject=None, mode=None):
+        """One distributed protected SpMV (all ranks call it): over the
+        library's NCCL communicator, or through `exchange` (external)."""
+        from .abft import AUTOCORRECT, CHECK
+        mode = CHECK | AUTOCORRECT if mode is None else mode
+        if self.dist.nccl:
+            return self.h.dist_spmv(x_own, self.y, inject, mode)
+        return exchange.spmv(self, x_own, inject, mode)
+
+    def plain(self, exchange=None, x_own=None):
+        from .abft import NOCHECK
+        return self.spmv(exchange, x_own, None, NOCHECK)
+
+
+class LocalExchange:
+    """Logical ranks in one process (tests on one GPU): the send lists come
+    from the other shards' needs; every SpMV runs begin on all ranks, moves
+    each send slice into its peer's receive slice and all partials into every
+    rank's parts array (rank order), then end on all ranks."""
+
+    def __init__(self, dss):
+        self.dss = {d.sh.rank: d for d in dss}
+        for r, d in self.dss.items():
+            for q, dq in self.dss.items():
+                if q != r:
+                    d.h.set_send(q, dq.h.needs(r))
+
+    def halo(self, x_owns=None):
+        """begin on every rank (x_owns: rank -> tensor or None) + the copies."""
         import torch
 
-        from .abft import CHECK, DEFER_FINISH
-        comm.halo(self.sh, self.x_ext)
-        self.h.spmv(self.x_ext, self.y, inject=inject, mode=CHECK | DEFER_FINISH)
-        if not hasattr(self, "_part"):
-            self._part = torch.empty(1, dtype=torch.float64, device=self.x_ext.device)
-        return self.h.beta_partial(self._part)
+        from .abft import lib
+        for r, d in self.dss.items():
+            d.h.begin(None if x_owns is None else x_owns.get(r))
+        torch.cuda.synchronize()
+        for r, d in self.dss.items():
+            for q, dq in self.dss.items():
+                if q == r:
+                    continue
+                sp, sc, _, _ = d.h.buffers(q)
+                _, _, rp, rc = dq.h.buffers(r)
+                assert sc == rc, (r, q, sc, rc)
+                if sc:
+                    lib().abft_memcpy(rp, sp, 8 * sc, None)
+        for r, d in self.dss.items():
+            for q, dq in self.dss.items():
+                lib().abft_memcpy(dq.parts.data_ptr() + 8 * r, d.h.partial_ptr(), 8, None)
 
-    def spmv(self, comm, inject=None, rounds=None):
-        """One distributed protected SpMV (all ranks call it)."""
-        part = self.step1(comm, inject)
-        comm.gather_partials(part, self.parts)
-        return self.step2(rounds, inject)
+    def spmv(self, ds, x_own, inject, mode):
+        raise RuntimeError("logical ranks step together: use spmv_all")
 
-    def step2(self, rounds=None, inject=None):
-        """Steps 4-5 with beta from all ranks' partials (self.parts)."""
-        self.h.finish(self.x_ext, self.y, self.parts, rounds, inject)
-        return self.y
+    def spmv_all(self, x_owns=None, injects=None, mode=None):
+        from .abft import AUTOCORRECT, CHECK
+        mode = CHECK | AUTOCORRECT if mode is None else mode
+        self.halo(x_owns)
+        for r, d in self.dss.items():
+            d.h.end(d.y, d.parts, None if injects is None else injects.get(r), mode)
+        return {r: d.y for r, d in self.dss.items()}
 
-    def plain(self, comm):
-        """Unprotected SpMV (same kernels, check off) over the extended x."""
-        from .abft import NOCHECK
-        comm.halo(self.sh, self.x_ext)
-        self.h.spmv(self.x_ext, self.y, mode=NOCHECK)
-        return self.y
+
+class TorchExchange:
+    """One process per rank over torch.distributed without the library's
+    communicator (tests: gloo, several processes sharing one GPU): the needs
+    are all-gathered once, each SpMV stages the library's send / receive
+    slices through host tensors."""
+
+    def __init__(self, ds: DistSpmv, group=None):
+        import torch.distributed as dist
+        self.dist, self.group = dist, group
+        self.rank, self.world = dist.get_rank(group), dist.get_world_size(group)
+        mine = {q: ds.h.needs(q).tolist() for q in range(self.world) if q != self.rank}
+        allneeds = [None] * self.world
+        dist.all_gather_object(allneeds, mine, group=group)
+        for q in range(self.world):
+            if q != self.rank:
+                ds.h.set_send(q, allneeds[q].get(self.rank, []))
+
+    def _d2h(self, ptr, count):
+        import torch
+
+        from .abft import lib
+        t = torch.empty(count, dtype=torch.float64)
+        if count:
+            lib().abft_memcpy(t.data_ptr(), ptr, 8 * count, None)
+        return t
+
+    def _h2d(self, ptr, t):
+        from .abft import lib
+        if t.numel():
+            lib().abft_memcpy(ptr, t.data_ptr(), 8 * t.numel(), None)
+
+    def gather(self, send_dev, recv_dev) -> None:
+        """All-gather a device vector (rank order) through the host."""
+        import torch
+        s = send_dev.cpu()
+        out = torch.empty(s.numel() * self.world, dtype=torch.float64)
+        self.dist.all_gather_into_tensor(out, s, group=self.group)
+        recv_dev.copy_(out.to(recv_dev.device))
+
+    def spmv(self, ds, x_own, inject, mode):
+        import torch
+        h = ds.h
+        h.begin(x_own)
+        torch.cuda.synchronize()
+        ops, recvs = [], []
+        for q in range(self.world):
+            if q == self.rank:
+                continue
+            sp, sc, rp, rc = h.buffers(q)
+            if sc:
+                ops.append(self.dist.P2POp(self.dist.isend, self._d2h(sp, sc), q, self.group))
+            if rc:
+                t = torch.empty(rc, dtype=torch.float64)
+                recvs.append((rp, t))
+                ops.append(self.dist.P2POp(self.dist.irecv, t, q, self.group))
+        if ops:
+            for w in self.dist.batch_isend_irecv(ops):
+                w.wait()
+        for rp, t in recvs:
+            self._h2d(rp, t)
+        part = self._d2h(h.partial_ptr(), 1)
+        out = torch.empty(self.world, dtype=torch.float64)
+        self.dist.all_gather_into_tensor(out, part, group=self.group)
+        ds.parts.copy_(out.to(ds.parts.device))
+        h.end(ds.y, ds.parts, inject, mode)
+        return ds.y
 
 
 # ---------------------------------------------------------------------------
 # Distributed Jacobi-PCG (SURVEY §8(e), P:294-300) on top of the C ABI
 # ---------------------------------------------------------------------------
 class DistPcg:
-    """One rank's share of the distributed PCG.  Vector kernels and scalar
-    updates run in libabft.so (abft_pcg_dist_*); this class only sequences
-    them around the two exchanges: the x halo of every SpMV (DistSpmv) and the
-    all-gather of the per-phase dot partials (3 doubles per rank), finished in
-    rank order on the device (R28).  Iterates like abft_pcg: the
-    device state word is read every `poll` iterations; every rank computes
-    identical scalars from identical partials, so all stop together."""
+    """One rank's share of the distributed PCG.  With the library's NCCL
+    communicator the whole solve is abft_dist_pcg (every exchange inside the
+    library).  Without one (tests) this class sequences the same device
+    phases (abft_pcg_dist_*) around an external exchange: the x halo of every
+    SpMV and the all-gather of the per-phase dot partials (3 doubles per
+    rank), finished in rank order on the device (R28)."""
 
     def __init__(self, ds: DistSpmv, check: bool = True, variant: str = "pcg", inject=None):
         import torch
@@ -261,8 +311,8 @@ class DistPcg:
         if inject is not None and not check:
             raise ValueError("fault injection needs the protected SpMV")
         self.ds, self.check, self.variant, self.inject = ds, check, variant, inject
-        self.calls, self._inj = 0, None
-        dev = ds.x_ext.device
+        self.calls = 0
+        dev = ds.y.device
         world = ds.sh.world
         self.send = torch.zeros(3, dtype=torch.float64, device=dev)
         self.recv = torch.zeros(3 * world, dtype=torch.float64, device=dev)
@@ -270,27 +320,19 @@ class DistPcg:
     def begin(self, b, x, n_global, tol=1e-6, max_iter=0, res_hist=None, diag=None):
         mi = max_iter if max_iter > 0 else 10 * n_global
         self.x, self.mi, self.calls = x, mi, 0
-        self.ds.h.pcg_dist_begin(b, x, self.ds.own(), self.ds.y, diag, tol, mi, self.check,
+        self.ds.h.pcg_dist_begin(b, x, self.ds.own_ptr(), self.ds.y, diag, tol, mi, self.check,
                                  res_hist)
-        self.ds.own().copy_(x)  # the first SpMV operand is x0
+        self.ds.set_own(x)  # the first SpMV operand is x0
         return mi
 
-    # -- the phases, each rank's half of one exchange --------------------------
-    def spmv_local(self, comm):
-        """Steps 1-3 of the SpMV (halo + fused pass); returns the beta partial
-        to gather (None for the unprotected baseline).  With `inject` set
-        (a function of the solve's SpMV call index -> Inject or None), the
-        call's faults go into the protected pass and its correction rounds."""
-        self._inj = self.inject(self.calls) if self.inject is not None else None
+    def next_inject(self):
+        inj = self.inject(self.calls) if self.inject is not None else None
         self.calls += 1
-        if not self.check:
-            self.ds.plain(comm)
-            return None
-        return self.ds.step1(comm, self._inj)
+        return inj
 
-    def spmv_finish(self):
-        if self.check:
-            self.ds.step2(None, self._inj)
+    def mode(self):
+        from .abft import AUTOCORRECT, CHECK, NOCHECK
+        return CHECK | AUTOCORRECT if self.check else NOCHECK
 
     def local(self, phase, it=0):
         from .abft import PCG_PHASE_P
@@ -303,16 +345,13 @@ class DistPcg:
     def status(self):
         return self.ds.h.pcg_dist_status()
 
-    # -- the iteration, over any exchange ------------------------------------
-    def run(self, spmv, reduce, local, status, mi, poll=16, graph=False, graph_key=None):
+    def run(self, spmv, reduce, local, status, mi, poll=16):
         """Sequence one solve (after begin).  spmv(): the distributed SpMV of
         the operand's own slice into ds.y; reduce(phases): run each
         (phase, it) local kernel, gather the send slots, combine the last
         phase; local(phase, it): a kernel without a reduction; status():
         (state, stats).  variant "pcg": standard (two reductions per
-        iteration); "cg1": single reduction (Chronopoulos-Gear, R29).
-        graph: capture `poll` iterations once and replay them (fault-free
-        solves; every call in an iteration must be capturable)."""
+        iteration); "cg1": single reduction (Chronopoulos-Gear, R29)."""
         from .abft import (PCG_PHASE_CG1_DOT, PCG_PHASE_CG1_UPDATE, PCG_PHASE_DOT,
                            PCG_PHASE_INIT, PCG_PHASE_P, PCG_PHASE_UPDATE)
         spmv()
@@ -320,81 +359,48 @@ class DistPcg:
         if self.variant == "cg1":
             spmv()  # w_0 = A u_0
             reduce([(PCG_PHASE_CG1_DOT, 0)])
-        def batch(j0, count):
-            for j in range(j0 + 1, j0 + count + 1):
-                if self.variant == "cg1":
-                    local(PCG_PHASE_CG1_UPDATE, j)
-                    spmv()  # w = A u
-                    reduce([(PCG_PHASE_CG1_DOT, j)])
-                else:
-                    spmv()  # q = A p (p sits in the operand's own slice)
-                    reduce([(PCG_PHASE_DOT, j)])
-                    reduce([(PCG_PHASE_UPDATE, j)])
-                    local(PCG_PHASE_P, j)
-
-        j, g = 0, None
-        if graph and graph_key is not None and getattr(self, "_graph", (None,))[0] == graph_key:
-            g = self._graph[1]  # same buffers and launch arguments: replay the cached graph
+        j = 0
         while True:
             state = status()
             if state[0] != 0 or j >= mi:
                 return state
-            if graph and mi - j >= poll:
-                # One CUDA graph of `poll` iterations, replayed until the
-                # device state leaves RUN.  The baked iteration indices
-                # 1..poll only pair each update with its p step (upd ==
-                # iter); kernels of a finished solve are no-ops and the host
-                # never replays after one, so reuse is exact.
-                if g is None:
-                    # capture_begin/end directly: torch.cuda.graph() would
-                    # also run gc.collect() + empty_cache() on every solve
-                    import torch
-                    g = torch.cuda.CUDAGraph()
-                    cs = torch.cuda.Stream()
-                    cs.wait_stream(torch.cuda.current_stream())
-                    with torch.cuda.stream(cs):
-                        g.capture_begin()
-                        try:
-                            batch(0, poll)
-                        finally:
-                            g.capture_end()
-                    torch.cuda.current_stream().wait_stream(cs)
-                    if graph_key is not None:
-                        self._graph = (graph_key, g)
-                g.replay()
-                j += poll
-            else:
-                n = min(poll, mi - j)
-                batch(j, n)
-                j += n
+            for it in range(j + 1, j + min(poll, mi - j) + 1):
+                if self.variant == "cg1":
+                    local(PCG_PHASE_CG1_UPDATE, it)
+                    spmv()  # w = A u
+                    reduce([(PCG_PHASE_CG1_DOT, it)])
+                else:
+                    spmv()  # q = A p (p sits in the operand's own slice)
+                    reduce([(PCG_PHASE_DOT, it)])
+                    reduce([(PCG_PHASE_UPDATE, it)])
+                    local(PCG_PHASE_P, it)
+            j += min(poll, mi - j)
 
-    # -- driver over torch.distributed (one process per GPU) -----------------
-    def solve(self, comm: TorchDistComm, b, x, n_global, tol=1e-6, max_iter=0, res_hist=None,
-              diag=None, poll=16, graph=False):
+    def solve(self, exchange, b, x, n_global, tol=1e-6, max_iter=0, res_hist=None, diag=None,
+              poll=16):
+        """One solve: abft_dist_pcg over the library's communicator, or the
+        phases over `exchange` (a TorchExchange)."""
+        if self.ds.dist.nccl:
+            inj = self.inject(0) if self.inject is not None else None
+            status, st = self.ds.h.dist_pcg(b, x, diag, tol, max_iter, inj, self.check, res_hist,
+                                            variant=self.variant)
+            return {0: 1, -5: 3, -7: 2}.get(status, status), st
+
         def spmv():
-            part = self.spmv_local(comm)
-            if part is not None:
-                comm.gather_partials(part, self.ds.parts)
-                self.spmv_finish()
+            exchange.spmv(self.ds, None, self.next_inject(), self.mode())
 
         def reduce(phases):
             for ph, it in phases:
                 self.local(ph, it)
-            comm.gather_partials(self.send, self.recv)
+            exchange.gather(self.send, self.recv)
             self.combine(*phases[-1])
 
-        if graph and self.inject is not None:
-            raise ValueError("graph replay needs a fault-free solve (per-call fault plans)")
         mi = self.begin(b, x, n_global, tol, max_iter, res_hist, diag)
-        # the captured launches bake every pointer and the handle's argument
-        # block: a later solve on the same buffers may replay the same graph
-        key = (tuple(None if t is None else t.data_ptr() for t in (b, x, res_hist, diag)) +
-               (tol, mi, poll)) if graph else None
-        return self.run(spmv, reduce, self.local, self.status, mi, poll, graph, key)
+        return self.run(spmv, reduce, self.local, self.status, mi, poll)
 
 
-def pcg_lockstep(pcgs, comm: LocalComm, bs, xs, n_global, tol=1e-6, max_iter=0, hists=None,
-                 poll=16, graph=False):
+def pcg_lockstep(pcgs, exchange: LocalExchange, bs, xs, n_global, tol=1e-6, max_iter=0,
+                 hists=None, poll=16):
     """Logical ranks in one process (tests): every phase runs on all ranks,
     then the partials are concatenated in rank order -- the exchange pattern
     of DistPcg.solve without a process group.  Rank 0's DistPcg.run sequences
@@ -403,12 +409,8 @@ def pcg_lockstep(pcgs, comm: LocalComm, bs, xs, n_global, tol=1e-6, max_iter=0, 
     hists = hists or [None] * len(pcgs)
 
     def spmv():
-        parts = [p.spmv_local(comm) for p in pcgs]
-        if parts[0] is not None:
-            allp = torch.cat(parts)
-            for p in pcgs:
-                p.ds.parts.copy_(allp)
-                p.spmv_finish()
+        injects = {p.ds.sh.rank: p.next_inject() for p in pcgs}
+        exchange.spmv_all(None, injects, pcgs[0].mode())
 
     def reduce(phases):
         for p in pcgs:
@@ -426,5 +428,5 @@ def pcg_lockstep(pcgs, comm: LocalComm, bs, xs, n_global, tol=1e-6, max_iter=0, 
     mi = 0
     for p, b, x, h in zip(pcgs, bs, xs, hists):
         mi = p.begin(b, x, n_global, tol, max_iter, h)
-    pcgs[0].run(spmv, reduce, local, pcgs[0].status, mi, poll, graph)
+    pcgs[0].run(spmv, reduce, local, pcgs[0].status, mi, poll)
     return [p.status() for p in pcgs]

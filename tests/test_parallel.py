@@ -6,6 +6,7 @@
 * 2 processes over gloo: the halo exchange and the partial all-gather.
 """
 import os
+import types
 
 import numpy as np
 import pytest
@@ -90,9 +91,31 @@ def test_shards_reproduce_global(O, name, world):
         assert O.pw(np.array(parts)) == O.pw(x * x)
 
 
+@pytest.mark.parametrize("world", [1, 2, 3, 4])
+@pytest.mark.parametrize("name", sorted(MATS))
+def test_library_halo_plan_matches_reference(name, world):
+    # abft_halo_plan (the host plan inside abft_dist_encode, C++) against the
+    # independent numpy reference make_shard: local columns, halo slices
+    from paper_conf_dsn_schollbkw16_b200 import halo_plan
+    A = MATS[name]()
+    ranges, shards = shard_all(A, world)
+    rg = PL.ranges_array(ranges)
+    for sh in shards:
+        rows = PL.shard_rows(A, sh.row0, sh.row1)
+        local, nb, na, rs, rc, halo = halo_plan(sh.rank, world, rg, rows.col)
+        assert np.array_equal(local, sh.csr.col)
+        assert nb == sh.x_offset and nb + sh.n + na == sh.n_cols
+        assert np.array_equal(halo, np.concatenate([sh.cols[:nb], sh.cols[nb + sh.n:]]))
+        for q in range(world):
+            start, count = sh.recv.get(q, (0, 0))
+            assert rc[q] == count and (count == 0 or rs[q] == start)
+
+
 def _gloo_worker(rank, world, port, q):
     import torch
     import torch.distributed as dist
+
+    from paper_conf_dsn_schollbkw16_b200 import halo_plan
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=world)
@@ -101,18 +124,43 @@ def _gloo_worker(rank, world, port, q):
         x = G.uniform_vector(A.n, 42)
         ranges = PL.block_partition(A.n, world)
         a, b = ranges[rank]
-        rows = G.CSR(A.row_ptr[a:b + 1] - A.row_ptr[a], A.col[A.row_ptr[a]:A.row_ptr[b]],
-                     A.val[A.row_ptr[a]:A.row_ptr[b]])
-        sh = PL.make_shard(rows, a, b, rank, world, ranges)
-        comm = PL.TorchDistComm()
-        PL.plan_from_needs(sh, comm.gather_needs(sh))
-        ext = torch.zeros(sh.n_cols, dtype=torch.float64)
-        ext[sh.x_offset:sh.x_offset + sh.n] = torch.from_numpy(x[a:b])
-        comm.halo(sh, ext)
-        ok = bool(np.array_equal(ext.numpy(), x[sh.cols]))
+        rows = PL.shard_rows(A, a, b)
+        # the library's host plan; needs exchanged over gloo (the protocol of
+        # abft_dist_needs / abft_dist_set_send), then the halo itself
+        local, nb, na, rs, rc, halo = halo_plan(rank, world, PL.ranges_array(ranges), rows.col)
+        hb = np.concatenate([halo[:nb], np.zeros(b - a, np.int64), halo[nb:]])
+        mine = {p: hb[rs[p]:rs[p] + rc[p]].tolist() for p in range(world) if p != rank and rc[p]}
+        allneeds = [None] * world
+        dist.all_gather_object(allneeds, mine)
+        ext = torch.zeros(nb + (b - a) + na, dtype=torch.float64)
+        ext[nb:nb + (b - a)] = torch.from_numpy(x[a:b])
+        ops, bufs = [], []
+        for p in range(world):
+            if p == rank:
+                continue
+            need = allneeds[p].get(rank, [])
+            if need:
+                buf = torch.from_numpy(x[np.asarray(need)] * 1.0)
+                assert np.all((np.asarray(need) >= a) & (np.asarray(need) < b))
+                bufs.append(buf)
+                ops.append(dist.P2POp(dist.isend, buf, p))
+            if rc[p]:
+                ops.append(dist.P2POp(dist.irecv, ext[rs[p]:rs[p] + rc[p]], p))
+        if ops:
+            for w in dist.batch_isend_irecv(ops):
+                w.wait()
+        cols = np.concatenate([halo[:nb], np.arange(a, b), halo[nb:]])
+        ok = bool(np.array_equal(ext.numpy(), x[cols]))
+        # the exchanged operand reproduces the global rows' products
+        y = np.array([np.sum(rows.val[rows.row_ptr[i]:rows.row_ptr[i + 1]] *
+                             ext.numpy()[local[rows.row_ptr[i]:rows.row_ptr[i + 1]]])
+                      for i in range(b - a)])
+        yg = np.array([np.sum(A.val[A.row_ptr[i]:A.row_ptr[i + 1]] *
+                              x[A.col[A.row_ptr[i]:A.row_ptr[i + 1]]]) for i in range(a, b)])
+        ok = ok and bool(np.array_equal(y, yg))
         part = torch.tensor([float(rank + 1)], dtype=torch.float64)
         out = torch.empty(world, dtype=torch.float64)
-        comm.gather_partials(part, out)
+        dist.all_gather_into_tensor(out, part)
         ok = ok and out.tolist() == [float(r + 1) for r in range(world)]
         q.put((rank, ok))
     finally:
@@ -229,12 +277,14 @@ class _FakeHandle:
 
 
 class _FakeDs:
-    """DistSpmv stand-in: the halo exchange is the real TorchDistComm; the
-    local product is the oracle's row sums over the extended x."""
+    """DistSpmv stand-in for DistPcg's external-exchange path: the operand is
+    a host tensor laid out like the library's ([halo below | own | halo
+    above], the numpy reference plan); the handle is the numpy test double."""
 
     def __init__(self, O, sh):
         import torch
         self.O, self.sh = O, sh
+        self.dist = types.SimpleNamespace(nccl=False)
         self.x_ext = torch.zeros(sh.n_cols, dtype=torch.float64)
         self.y = torch.zeros(sh.n, dtype=torch.float64)
         self.h = _FakeHandle(O)
@@ -244,16 +294,45 @@ class _FakeDs:
         on = c.col == rows + sh.x_offset
         self.h.diag[rows[on]] = c.val[on]
 
-    def own(self):
+    def own_ptr(self):
         return self.x_ext[self.sh.x_offset:self.sh.x_offset + self.sh.n]
 
-    def plain(self, comm):
-        comm.halo(self.sh, self.x_ext)
-        c, xe = self.sh.csr, self.x_ext.numpy()
-        self.y.numpy()[:] = [self.O.pw(c.val[c.row_ptr[i]:c.row_ptr[i + 1]] *
-                                       xe[c.col[c.row_ptr[i]:c.row_ptr[i + 1]]])
-                             for i in range(self.sh.n)]
-        return self.y
+    def set_own(self, x):
+        self.own_ptr().copy_(x)
+
+
+class _FakeExchange:
+    """The exchange DistPcg drives (spmv, gather) over gloo, with the halo of
+    the numpy reference plan and the oracle's row products."""
+
+    def __init__(self, O, sh):
+        import torch.distributed as dist
+        self.O, self.sh, self.dist = O, sh, dist
+        needs = {q: sh.cols[s:s + c].tolist() for q, (s, c) in sh.recv.items()}
+        allneeds = [None] * sh.world
+        dist.all_gather_object(allneeds, needs)
+        PL.plan_from_needs(sh, {q: allneeds[q][sh.rank] for q in range(sh.world)
+                                if q != sh.rank and sh.rank in allneeds[q]})
+
+    def spmv(self, ds, x_own, inject, mode):
+        import torch
+        dist, sh = self.dist, self.sh
+        ops = []
+        for q, idx in sorted(sh.send.items()):
+            ops.append(dist.P2POp(dist.isend, ds.x_ext[torch.as_tensor(idx)].clone(), q))
+        for q, (start, count) in sorted(sh.recv.items()):
+            ops.append(dist.P2POp(dist.irecv, ds.x_ext[start:start + count], q))
+        if ops:
+            for w in dist.batch_isend_irecv(ops):
+                w.wait()
+        c, xe = sh.csr, ds.x_ext.numpy()
+        ds.y.numpy()[:] = [self.O.pw(c.val[c.row_ptr[i]:c.row_ptr[i + 1]] *
+                                     xe[c.col[c.row_ptr[i]:c.row_ptr[i + 1]]])
+                           for i in range(sh.n)]
+        return ds.y
+
+    def gather(self, send, recv):
+        self.dist.all_gather_into_tensor(recv, send)
 
 
 def _gloo_pcg_worker(rank, world, port, variant, q):
@@ -270,15 +349,14 @@ def _gloo_pcg_worker(rank, world, port, variant, q):
         a, b_ = ranges[rank]
         rows = G.stencil_rows("7pt", 8, 8, 8, a // 64, b_ // 64)
         sh = PL.make_shard(rows, a, b_, rank, world, ranges)
-        comm = PL.TorchDistComm()
-        PL.plan_from_needs(sh, comm.gather_needs(sh))
+        ex = _FakeExchange(O, sh)
         ds = _FakeDs(O, sh)
         p = PL.DistPcg(ds, False, variant)
         bfull = O.spmv(A, G.uniform_vector(A.n, 43))
         b = torch.from_numpy(bfull[a:b_].copy())
         x = torch.from_numpy(G.uniform_vector(A.n, 44)[a:b_].copy())
         hist = []
-        state, st = p.solve(comm, b, x, A.n, tol=1e-6, res_hist=hist, poll=4)
+        state, st = p.solve(ex, b, x, A.n, tol=1e-6, res_hist=hist, poll=4)
         q.put((rank, state, st["iters"], st["spmv_calls"], x.numpy().tolist(), hist))
     finally:
         dist.destroy_process_group()
