@@ -172,6 +172,10 @@ struct abft_ctx {
   int32_t *pnf = nullptr;  // [pnf_cap] per-step round-0 flag counts
   int32_t pnf_cap = 0;
   cudaStream_t s_in = nullptr, s_out = nullptr;
+  // hub-row chunk sums (k_hub) on their own stream, concurrent with the
+  // group kernels that do not need them (k_lean / k_irr; opt-in)
+  cudaStream_t s_hub = nullptr;
+  cudaEvent_t ev_hub0 = nullptr, ev_hub1 = nullptr;
   cudaEvent_t ev_x[2] = {nullptr, nullptr}, ev_c[2] = {nullptr, nullptr}, ev_o[2] = {nullptr, nullptr};
   // PCG scratch
   double *pcg = nullptr;  // r, z, p, q, d : 5 n
@@ -511,10 +515,20 @@ abft_status launch_fused_t(const abft_ctx *h, SpmvArgs a, cudaStream_t s) {
   a.ilist = h->ilist;
   a.n_ilist = h->n_ilist;
   const int ggrid = ngen > 0 ? general_grid(h, ngen) : 0;
-  if (h->n_hub > 0)  // chunk sums of hub rows, read by the group kernels
+  // chunk sums of hub rows, read by k_general (the groups owning hub rows);
+  // with ABFT_HUB_STREAM on their own stream, overlapping k_lean / k_irr
+  const bool side = h->n_hub > 0 && h->s_hub;
+  if (side) {
+    CK(cudaEventRecord(h->ev_hub0, s));
+    CK(cudaStreamWaitEvent(h->s_hub, h->ev_hub0, 0));
+    k_hub<<<general_grid(h, h->n_hub), kGenWarps * 32, 0, h->s_hub>>>(a);
+    CK(cudaEventRecord(h->ev_hub1, h->s_hub));
+  } else if (h->n_hub > 0) {
     k_hub<<<general_grid(h, h->n_hub), kGenWarps * 32, 0, s>>>(a);
+  }
   if (lean) launch_lean<CHECK, INJECT>(h, a, s);
   if (h->n_ilist > 0) launch_irr<CHECK, INJECT>(h, a, s);
+  if (side) CK(cudaStreamWaitEvent(s, h->ev_hub1, 0));
   if (ggrid) k_general<CHECK, INJECT><<<ggrid, kGenWarps * 32, 0, s>>>(a);
   CK(cudaGetLastError());
   return ABFT_OK;
@@ -883,8 +897,10 @@ abft_status plan_stream(abft_ctx *h, const std::vector<int32_t> &rp, const std::
     c.NS = NS;
     c.ring_off = 128;
     c.xs_off = 128 + (uint32_t)NS * c.stage_bytes;
-    // prefer more groups per chunk (fewer producer round trips) when >= 3 stages fit
-    const int64_t score = (int64_t)(NS >= 3 ? 1000 : 0) + G * 10 + NS;
+    // the most consumer warps (groups per chunk) that still double-buffer,
+    // then the deepest ring (27-pt 128^3: G 4 x 2 stages 0.189 ms, G 2 x 4
+    // stages 0.354 ms)
+    const int64_t score = (int64_t)G * 100 + NS;
     if (score > best_score) {
       best_score = score;
       best = c;
@@ -1018,6 +1034,14 @@ abft_status plan_fused(abft_ctx *h, cudaStream_t s) {
     TRY(upload(h, &h->own_n, on, s));
     h->n_hub = (int32_t)hbeg.size();
     h->n_own = (int32_t)own.size();
+    // opt-in (ABFT_HUB_STREAM=1): measured slower on R-MAT scale 24 (4.67 ->
+    // 5.60 ms protected: the concurrent random gathers of k_hub and k_irr
+    // contend for DRAM and L2), so the default keeps one stream
+    if (h->n_hub > 0 && getenv("ABFT_HUB_STREAM")) {
+      CK(cudaStreamCreateWithFlags(&h->s_hub, cudaStreamNonBlocking));
+      CK(cudaEventCreateWithFlags(&h->ev_hub0, cudaEventDisableTiming));
+      CK(cudaEventCreateWithFlags(&h->ev_hub1, cudaEventDisableTiming));
+    }
   }
   if (h->pos) {  // position-map records: k_stream + k_general
     h->lean = false;
@@ -1262,6 +1286,12 @@ abft_status abft_destroy(abft_handle_t h) {
     cudaStreamSynchronize(h->cs);
     cudaStreamDestroy(h->cs);
   }
+  if (h->s_hub) {
+    cudaStreamSynchronize(h->s_hub);
+    cudaStreamDestroy(h->s_hub);
+  }
+  if (h->ev_hub0) cudaEventDestroy(h->ev_hub0);
+  if (h->ev_hub1) cudaEventDestroy(h->ev_hub1);
   if (h->ev_pack) cudaEventDestroy(h->ev_pack);
   if (h->ev_comm) cudaEventDestroy(h->ev_comm);
   if (h->s_in) {
