@@ -90,7 +90,7 @@ typedef struct abft_ctx *abft_handle_t;
  *        (row of y, block of t1 / t2); events on one element compose by XOR.
  *        `targets` masks the targets that receive events.  The plan is built
  *        on the device (5 short launches) by every call that injects. */
-enum { ABFT_INJ_NONE = 0, ABFT_INJ_LIST = 1, ABFT_INJ_RATE = 2 };
+enum { ABFT_INJ_NONE = 0, ABFT_INJ_LIST = 1, ABFT_INJ_RATE = 2, ABFT_INJ_RESIDENT = 3 };
 enum { ABFT_TARGET_Y = 0, ABFT_TARGET_T1 = 1, ABFT_TARGET_T2 = 2 };
 typedef struct {
   uint32_t mode;
@@ -104,6 +104,25 @@ typedef struct {
   const int64_t *list_index;   /* (host) */
   const uint64_t *list_mask;   /* (host) */
 } abft_inject_t;
+
+/* RESIDENT (mode 3): reuse the device fault list the handle's last injecting
+ * call (or abft_inject_prepare) built -- same faults, no plan generation: the
+ * method's cost under faults is then timed without the injector's.
+ * abft_inject_prepare: build the device list of `inj` (list upload, or the
+ *   rate plan of inj->call, for the op counts of `mode`: CHECK or not)
+ *   without running an SpMV; stream-ordered.
+ * abft_inject_list: device pointers to that list: keys ((round << 58) |
+ *   (target << 56) | index, ascending), XOR masks, its length (a device int32
+ *   for rate plans, else *n_host) and capacity; valid until the next
+ *   injecting call. */
+abft_status abft_inject_prepare(abft_handle_t h, const abft_inject_t *inj, uint32_t mode,
+                                void *stream);
+abft_status abft_inject_list(abft_handle_t h, const uint64_t **keys, const uint64_t **masks,
+                             const int32_t **n_dev, int32_t *n_host, int32_t *cap);
+/* Zero the masks of the resident list (keys kept): RESIDENT calls then do
+ * the injector's every lookup but change no value -- the harness control of
+ * an overhead measurement (bench.py --lam-sweep).  Stream-ordered. */
+abft_status abft_inject_clear_masks(abft_handle_t h, void *stream);
 
 /* abft_spmv mode bits */
 enum {

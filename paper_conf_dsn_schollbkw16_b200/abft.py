@@ -21,7 +21,7 @@ OK, EINVAL, ECUDA, ENOMEM, ENOTSUP, ENOCONV, EUNCORRECTED, EBREAKDOWN, ENCCL = (
     0, -1, -2, -3, -4, -5, -6, -7, -8)
 NOCHECK, CHECK, AUTOCORRECT, DEBUG_CHECKSUMS, DEFER_FINISH = 0, 1, 2, 4, 8
 DENSE_BOUND35 = 16  # abft_spmv_dense: tau = K35 ||x|| ([35]) instead of ||x|| ([30])
-INJ_NONE, INJ_LIST, INJ_RATE = 0, 1, 2
+INJ_NONE, INJ_LIST, INJ_RATE, INJ_RESIDENT = 0, 1, 2, 3
 
 SYMBOLS = [
     "abft_encode", "abft_spmv", "abft_correct", "abft_flags", "abft_beta",
@@ -35,7 +35,7 @@ SYMBOLS = [
     "abft_dist_unique_id", "abft_dist_create", "abft_dist_destroy", "abft_dist_encode",
     "abft_dist_needs", "abft_dist_set_send", "abft_dist_operand", "abft_dist_spmv",
     "abft_dist_begin", "abft_dist_buffers", "abft_dist_partial", "abft_dist_end", "abft_dist_pcg",
-    "abft_halo_plan",
+    "abft_halo_plan", "abft_inject_prepare", "abft_inject_list", "abft_inject_clear_masks",
 ]
 PCG_PHASE_INIT, PCG_PHASE_DOT, PCG_PHASE_UPDATE, PCG_PHASE_P = 0, 1, 2, 3
 PCG_PHASE_CG1_UPDATE, PCG_PHASE_CG1_DOT = 4, 5  # single-reduction variant
@@ -194,6 +194,13 @@ def lib():
         L.abft_dist_end.argtypes = [P, P, P, P, u32, P]
         L.abft_dist_pcg.restype = st
         L.abft_dist_pcg.argtypes = [P, P, P, P, d, i64, P, i32, i32, P, C.POINTER(PcgStats), P]
+        L.abft_inject_prepare.restype = st
+        L.abft_inject_prepare.argtypes = [P, P, u32, P]
+        L.abft_inject_list.restype = st
+        L.abft_inject_list.argtypes = [P, C.POINTER(P), C.POINTER(P), C.POINTER(P),
+                                       C.POINTER(i32), C.POINTER(i32)]
+        L.abft_inject_clear_masks.restype = st
+        L.abft_inject_clear_masks.argtypes = [P, P]
         L.abft_halo_plan.restype = st
         L.abft_halo_plan.argtypes = [i32, i32, P, P, i64, P, PI64, PI64, P, P, P, i64]
         L.abft_finish.argtypes = [P, P, P, P, i32, i32, P, P]
@@ -266,6 +273,11 @@ class Inject:
     def rate(seed, lam, targets=0b111, call=0):
         return Inject(mode=INJ_RATE, seed=seed, call=call, lam=lam, targets=targets)
 
+    @staticmethod
+    def resident():
+        """The device fault list the handle's last injecting call built."""
+        return Inject(mode=INJ_RESIDENT)
+
     def struct(self):
         s = _Inj()
         s.mode, s.seed, s.call, s.lambda_, s.targets = (self.mode, self.seed, self.call,
@@ -328,6 +340,30 @@ class Handle:
                                  ENCODE_C_CSR if c_csr else 0, _stream(stream), C.byref(h)),
                "abft_encode")
         self._h = h
+
+    def inject_prepare(self, inject: Inject, mode=CHECK, stream=None):
+        inj = inject.struct()
+        _check(lib().abft_inject_prepare(self._h, C.byref(inj), mode, _stream(stream)),
+               "abft_inject_prepare")
+
+    def inject_clear_masks(self, stream=None):
+        """Zero the resident list's masks (harness control: same lookups, no faults)."""
+        _check(lib().abft_inject_clear_masks(self._h, _stream(stream)), "abft_inject_clear_masks")
+
+    def inject_list(self, stream=None):
+        """The resident device fault list as host arrays (keys, masks):
+        decoded (round, target, index, mask)."""
+        k, m, nd = C.c_void_p(), C.c_void_p(), C.c_void_p()
+        nh, cap = C.c_int32(), C.c_int32()
+        _check(lib().abft_inject_list(self._h, C.byref(k), C.byref(m), C.byref(nd), C.byref(nh),
+                                      C.byref(cap)), "abft_inject_list")
+        n = nh.value
+        if nd.value:
+            n = min(int(self._d2h(nd, 1, np.int32, stream)[0]), cap.value)
+        keys = self._d2h(k, n, np.uint64, stream)
+        masks = self._d2h(m, n, np.uint64, stream)
+        return (keys >> np.uint64(58)).astype(np.int32), ((keys >> np.uint64(56)) & np.uint64(3)).astype(
+            np.int32), (keys & np.uint64((1 << 56) - 1)).astype(np.int64), masks
 
     def health(self, stream=None) -> int:
         """1 if a grid barrier timed out since the last call (abft_health)."""

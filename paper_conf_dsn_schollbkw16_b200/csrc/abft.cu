@@ -159,6 +159,10 @@ struct abft_ctx {
   int64_t inj_cap = 0;
   std::vector<uint64_t> list_keys_host, list_masks_host;  // last uploaded list plan
   bool list_cached = false;
+  uint32_t *inj_gbits = nullptr;  // [ceil(ngroups / 32)] group bitmap of the device list
+  int32_t *inj_gstart = nullptr;  // [3][ngroups] first entry of (target, group)
+  InjDev inj_last{};        // the device plan the last injecting call built (ABFT_INJ_RESIDENT)
+  bool inj_last_valid = false;
   // rate-mode plan scratch
   int32_t *plan_counts = nullptr, *plan_offs = nullptr, *plan_tot = nullptr, *plan_len = nullptr;
   uint64_t *plan_tab = nullptr;
@@ -303,8 +307,33 @@ abft_status ensure_list(abft_ctx *h, int64_t need) {
 // Rate mode (R13): expand a Poisson process over the call's
 // arithmetic operations into a sorted fault list on the device (no host
 // sync); the chunking and the CDF tables come from FaultTables.
+// The group bitmap of a device list just built (InjDev::gbits): groups
+// without round-0 entries skip the list search in the kernels.
+abft_status build_inj_bits(abft_ctx *h, InjDev *d, cudaStream_t s) {
+  d->gbits = nullptr;
+  if (d->mode == 0 || h->ngroups <= 0 || (d->n_list <= 0 && !d->n_list_dev)) return ABFT_OK;
+  const int64_t words = (h->ngroups + 31) / 32;
+  if (!h->inj_gbits) {
+    TRY(dalloc(h, &h->inj_gbits, (size_t)words));
+    TRY(dalloc(h, &h->inj_gstart, (size_t)(3 * h->ngroups)));
+    CK(cudaMemsetAsync(h->inj_gstart, 0xFF, (size_t)(3 * h->ngroups) * 4, s));
+  }
+  // gstart needs no reset: it is read only where this plan sets gbits, and
+  // this plan writes every such entry
+  CK(cudaMemsetAsync(h->inj_gbits, 0, (size_t)words * 4, s));
+  const int64_t cap = d->n_list_dev ? d->cap : d->n_list;
+  k_inj_bits<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>((cap + 255) / 256, 4 * h->num_sms)),
+               256, 0, s>>>(*d, h->bs, h->ngroups, h->inj_gbits, h->inj_gstart);
+  CK(cudaGetLastError());
+  d->gbits = h->inj_gbits;
+  d->gstart = h->inj_gstart;
+  d->ngroups = h->ngroups;
+  return ABFT_OK;
+}
+
 abft_status gen_rate_plan(abft_ctx *h, const abft_inject_t *inj, uint64_t call, bool check,
                           cudaStream_t s, InjDev *d) {
+  memset(d, 0, sizeof *d);
   RatePlanArgs r;
   memset(&r, 0, sizeof r);
   r.n = h->n;
@@ -370,13 +399,32 @@ abft_status gen_rate_plan(abft_ctx *h, const abft_inject_t *inj, uint64_t call, 
   d->cap = (int32_t)std::min<int64_t>(cap, INT32_MAX);
   d->keys = h->inj_keys;
   d->masks = h->inj_masks;
-  return ABFT_OK;
+  return build_inj_bits(h, d, s);
 }
 
 // Fill the device descriptor: upload a list-mode plan (sorted keys), or
 // generate the rate-mode plan of call inj->call.
+abft_status prepare_inject_impl(abft_ctx *h, const abft_inject_t *inj, bool check, cudaStream_t s,
+                                InjDev *d);
+
 abft_status prepare_inject(abft_ctx *h, const abft_inject_t *inj, bool check, cudaStream_t s,
                            InjDev *d) {
+  memset(d, 0, sizeof *d);
+  if (inj && inj->mode == ABFT_INJ_RESIDENT) {  // the plan already on the device
+    if (!h->inj_last_valid) return ABFT_EINVAL;
+    *d = h->inj_last;
+    return ABFT_OK;
+  }
+  TRY(prepare_inject_impl(h, inj, check, s, d));
+  if (d->mode != 0) {
+    h->inj_last = *d;
+    h->inj_last_valid = true;
+  }
+  return ABFT_OK;
+}
+
+abft_status prepare_inject_impl(abft_ctx *h, const abft_inject_t *inj, bool check, cudaStream_t s,
+                                InjDev *d) {
   memset(d, 0, sizeof *d);
   if (!inj || inj->mode == ABFT_INJ_NONE) return ABFT_OK;
   if (inj->mode == ABFT_INJ_RATE) {
@@ -419,7 +467,7 @@ abft_status prepare_inject(abft_ctx *h, const abft_inject_t *inj, bool check, cu
   }
   d->keys = h->inj_keys;
   d->masks = h->inj_masks;
-  return ABFT_OK;
+  return build_inj_bits(h, d, s);
 }
 
 int general_grid(const abft_ctx *h, int64_t groups) {  // kGenWarps warps per CTA
@@ -1662,6 +1710,35 @@ abft_status abft_info(abft_handle_t h, abft_info_t *info) {
   info->lean_runs = h->lean_runs ? 1 : 0;
   info->lean = h->lean ? 1 : 0;
   info->max_rounds = h->max_rounds;
+  return ABFT_OK;
+}
+
+abft_status abft_inject_prepare(abft_handle_t h, const abft_inject_t *inj, uint32_t mode,
+                                void *stream) {
+  if (!h || !inj || inj->mode == ABFT_INJ_RESIDENT) return ABFT_EINVAL;
+  const bool check = (mode & ABFT_CHECK) || (mode & ABFT_AUTOCORRECT);
+  InjDev d;
+  return prepare_inject(h, inj, check, (cudaStream_t)stream, &d);
+}
+
+abft_status abft_inject_list(abft_handle_t h, const uint64_t **keys, const uint64_t **masks,
+                             const int32_t **n_dev, int32_t *n_host, int32_t *cap) {
+  if (!h || !h->inj_last_valid) return ABFT_EINVAL;
+  if (keys) *keys = h->inj_last.keys;
+  if (masks) *masks = h->inj_last.masks;
+  if (n_dev) *n_dev = h->inj_last.n_list_dev;
+  if (n_host) *n_host = h->inj_last.n_list;
+  if (cap) *cap = h->inj_last.cap;
+  return ABFT_OK;
+}
+
+abft_status abft_inject_clear_masks(abft_handle_t h, void *stream) {
+  if (!h || !h->inj_last_valid) return ABFT_EINVAL;
+  const int64_t n = h->inj_last.n_list_dev ? h->inj_last.cap : h->inj_last.n_list;
+  if (n > 0)
+    CK(cudaMemsetAsync(const_cast<uint64_t *>(h->inj_last.masks), 0, (size_t)n * 8,
+                       (cudaStream_t)stream));
+  h->list_cached = false;  // the device list no longer matches the uploaded plan
   return ABFT_OK;
 }
 

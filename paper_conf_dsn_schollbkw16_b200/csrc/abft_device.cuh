@@ -110,6 +110,13 @@ struct InjDev {
   int32_t cap;       // capacity of a device-generated list
   const uint64_t *keys;   // sorted (round << 58) | (target << 56) | index
   const uint64_t *masks;
+  // bit g set <=> some round-0 entry touches 32-row group g (a y row of it,
+  // or the t1 / t2 of a block starting in it); null = search every group
+  const uint32_t *gbits;
+  // [3][ngroups] first list position of a round-0 entry of (target, group);
+  // read only for groups whose gbits bit is set (-1: no entry of that target)
+  const int32_t *gstart;
+  int64_t ngroups;
 };
 
 __device__ __forceinline__ void philox10(uint32_t c[4], uint32_t k0, uint32_t k1) {
@@ -138,6 +145,69 @@ __device__ __forceinline__ int list_len(const InjDev &inj) {
   return inj.n_list_dev ? min(*inj.n_list_dev, inj.cap) : inj.n_list;
 }
 
+// Whether group g may hold a round-0 fault (the kernels skip the list
+// search of every other group).
+__device__ __forceinline__ bool inj_group_hit(const InjDev &inj, int64_t g) {
+  return !inj.gbits || ((__ldg(inj.gbits + (g >> 5)) >> (g & 31)) & 1u);
+}
+
+// Build the group bitmap of a device list (round-0 entries only; the list
+// is sorted, so the round-0 entries come first).
+__device__ __forceinline__ int64_t inj_entry_group(uint64_t k, int32_t bs, int64_t ngroups,
+                                                    int &t) {
+  t = (int)((k >> 56) & 3u);
+  const int64_t idx = (int64_t)(k & ((1ull << 56) - 1));
+  if ((k >> 58) != 0) return ngroups;  // rounds >= 1: not the fused pass's
+  return t == 0 ? min(idx >> 5, ngroups) : idx < ((int64_t)1 << 40) ? min((idx * bs) >> 5, ngroups) : ngroups;
+}
+
+__global__ void k_inj_bits(const InjDev inj, int32_t bs, int64_t ngroups, uint32_t *gbits,
+                           int32_t *gstart) {
+  const int len = list_len(inj);
+  for (int e = blockIdx.x * blockDim.x + threadIdx.x; e < len; e += gridDim.x * blockDim.x) {
+    int t;
+    const int64_t g = inj_entry_group(inj.keys[e], bs, ngroups, t);
+    if (g >= ngroups) continue;
+    int tp = -1;
+    const int64_t gp = e > 0 ? inj_entry_group(inj.keys[e - 1], bs, ngroups, tp) : -1;
+    if (gp != g || tp != t) {  // first entry of (target, group): sorted list
+      gstart[(int64_t)t * ngroups + g] = e;
+      atomicOr(gbits + (g >> 5), 1u << (g & 31));
+    }
+  }
+}
+
+// The masks of a group with round-0 entries (gbits set): y row i (every
+// lane), t1 / t2 of block k (the stream kernel: bs = 32, k = g).  A few loads from the group's
+// first entry instead of binary searches; not inlined (rare path).
+struct InjMasks {
+  uint64_t y, t1, t2;
+};
+__device__ __noinline__ InjMasks inj_group_masks(const uint64_t *keys, const uint64_t *masks,
+                                                 const int32_t *n_dev, int n_list, int cap,
+                                                 const int32_t *gstart, int64_t ngroups,
+                                                 int64_t g, int64_t i, int64_t k) {
+  // a start left by an earlier plan (this plan has no entry of that target
+  // in g) points at an entry outside the range: the scans stop at once
+  const int len = n_dev ? min(*n_dev, cap) : n_list;
+  InjMasks m{0, 0, 0};
+  const uint64_t y0 = list_key(0, 0, g * 32), y1 = list_key(0, 0, g * 32 + 32);
+  for (int e = max(__ldg(gstart + g), 0); e < len; ++e) {
+    const uint64_t key = __ldg(keys + e);
+    if (key < y0 || key >= y1) break;
+    if (key == list_key(0, 0, i)) m.y ^= __ldg(masks + e);
+  }
+  for (int e = max(__ldg(gstart + ngroups + g), 0); e < len && __ldg(keys + e) == list_key(0, 1, k); ++e)
+    m.t1 ^= __ldg(masks + e);
+  for (int e = max(__ldg(gstart + 2 * ngroups + g), 0); e < len && __ldg(keys + e) == list_key(0, 2, k); ++e)
+    m.t2 ^= __ldg(masks + e);
+  return m;
+}
+__device__ __forceinline__ InjMasks inj_masks(const InjDev &inj, int64_t g, int64_t i) {
+  return inj_group_masks(inj.keys, inj.masks, inj.n_list_dev, inj.n_list, inj.cap, inj.gstart,
+                         inj.ngroups, g, i, g);
+}
+
 // First list position with key >= k.
 __device__ __forceinline__ int list_lower(const InjDev &inj, int len, uint64_t k) {
   int lo = 0, hi = len;
@@ -146,6 +216,27 @@ __device__ __forceinline__ int list_lower(const InjDev &inj, int len, uint64_t k
     if (__ldg(inj.keys + mid) < k) lo = mid + 1; else hi = mid;
   }
   return lo;
+}
+
+// XOR of the masks of every entry with key k (a search of its own; not
+// inlined, so the rare faulty groups do not cost the others registers).
+// (Arguments by value: a reference into the kernel's parameter block would
+// force a stack copy of the whole argument struct.)
+__device__ __noinline__ uint64_t list_mask_of_v(const uint64_t *keys, const uint64_t *masks,
+                                                const int32_t *n_dev, int n_list, int cap,
+                                                uint64_t k) {
+  const int len = n_dev ? min(*n_dev, cap) : n_list;
+  int lo = 0, hi = len;
+  while (lo < hi) {
+    const int mid = (lo + hi) >> 1;
+    if (__ldg(keys + mid) < k) lo = mid + 1; else hi = mid;
+  }
+  uint64_t m = 0;
+  for (int e = lo; e < len && __ldg(keys + e) == k; ++e) m ^= __ldg(masks + e);
+  return m;
+}
+__device__ __forceinline__ uint64_t list_mask_of(const InjDev &inj, uint64_t k) {
+  return list_mask_of_v(inj.keys, inj.masks, inj.n_list_dev, inj.n_list, inj.cap, k);
 }
 
 // XOR of the masks of entries [lo, hi) whose key equals k.

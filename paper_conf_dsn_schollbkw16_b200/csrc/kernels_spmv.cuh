@@ -1404,25 +1404,105 @@ __device__ __forceinline__ bool grid_sync(unsigned *bar) {
   return s_ok != 0;
 }
 
+// Step 5 for one flagged block k in round `round`: recompute
+// its rows and t1 / t2, re-check against tau_k = K_k beta.  Returns (warp-
+// uniform) whether the block still fails.  [olo, ohi): the hub rows of the
+// block's group whose chunk sums the CTA precomputed (solo hub rounds), or
+// empty.  A block's rounds depend on no other block: the kernel runs each
+// flagged block through all its rounds without grid barriers.
+template <bool INJECT>
+__device__ __forceinline__ bool fin_block(const SpmvArgs &a, int64_t k, int round, int lane,
+                                          double beta, int olo, int ohi) {
+  const int64_t n = a.n;
+  if (a.bs > 32) {  // big blocks: recompute the block's groups, re-verify
+    const double sv = big_block<true, INJECT>(a, k, round, lane, nullptr);
+    return __shfl_sync(kFull, !(fabs(sv) <= dmul(__ldg(a.K + k), beta)), 0);
+  }
+  const LdgSrc As{a.va, a.ci}, Cs{a.cval, a.ccol};
+  const int32_t cb = __ldg(a.crp + k), ce = __ldg(a.crp + k + 1);  // issued early
+  const int64_t i = (k << a.log2bs) + lane;
+  const bool valid = lane < a.bs && i < n;
+  int32_t rs = 0, len = 0;
+  if (valid) {
+    rs = __ldg(a.rp + i);
+    len = __ldg(a.rp + i + 1) - rs;
+  }
+  const int maxlen = warp_max_i(len);
+  double yv = 0.0;
+  if (maxlen <= 32) {
+    if (valid) yv = lane_dot_any(As, rs, len, maxlen, a.x);
+  } else {
+    for (int j = 0; j < a.bs; ++j) {
+      const int32_t rb = __shfl_sync(kFull, rs, j);
+      const int rl = __shfl_sync(kFull, len, j);
+      if ((k << a.log2bs) + j >= n) break;
+      double t;
+      const int e = rl > kHubLen ? own_find(a, olo, ohi, (int)(((k << a.log2bs) + j) & 31)) : -1;
+      if (e >= 0)
+        t = hub_sum(a, __ldg(a.own_first + e), __ldg(a.own_n + e));
+      else
+        t = warp_dot(As, rb, rl, a.x, lane);
+      if (lane == j) yv = t;
+    }
+  }
+  if (len == 0) yv = 0.0;
+  if (INJECT) {
+    const uint64_t m = group_y_mask(a.inj, round, k << a.log2bs, i, lane);
+    if (valid) yv = apply_mask(yv, m);
+  }
+  if (valid) a.y[i] = yv;
+  double t2 = bfly32(valid ? yv : kAbsent);
+  const int ec = ce - cb > kHubLen
+                     ? own_find(a, olo, ohi, 32 + (int)(k & ((32 >> a.log2bs) - 1))) : -1;
+  double t1 = ec >= 0 ? hub_sum(a, __ldg(a.own_first + ec), __ldg(a.own_n + ec))
+                      : warp_dot(Cs, cb, ce - cb, a.x, lane);
+  bool fail = false;
+  if (lane == 0) {
+    if (INJECT) {
+      t1 = apply_mask(t1, fault_mask(a.inj, round, 1, k, 2 * (int64_t)(ce - cb)));
+      t2 = apply_mask(t2, fault_mask(a.inj, round, 2, k, min64(a.bs, n - (k << a.log2bs))));
+    }
+    fail = !(fabs(dsub(t1, t2)) <= dmul(__ldg(a.K + k), beta));
+  }
+  return __shfl_sync(kFull, fail, 0);
+}
+
+// Rounds 1..rounds of one block flagged in round 0: a round's failure puts
+// the block on that round's list and runs the next round.
+template <bool INJECT>
+__device__ __forceinline__ void block_rounds(const SpmvArgs &a, int64_t k, int rounds, int lane,
+                                             double beta) {
+  for (int round = 1; round <= rounds; ++round) {
+    if (!fin_block<INJECT>(a, k, round, lane, beta, 0, 0)) return;
+    if (lane == 0) a.flags[(int64_t)round * a.nb + atomicAdd(a.n_flags + round, 1)] = (int32_t)k;
+  }
+}
+
 // Steps 4-5 after the fused pass, one launch (programmatic dependent launch:
 // its launch latency overlaps the fused kernels; griddepcontrol.wait orders
 // it after them).  One CTA per SM, software grid barrier.
 //  * CONFIRM: if the fused pass left candidates, beta = sqrt(PW(gsum))
-//    (aligned 1024-group partials reduced by all CTAs, then the partials by
-//    every CTA redundantly -- the same bits everywhere), and each candidate
-//    is flagged iff NOT(|s_k| <= K_k beta).  No candidates: flags
-//    are empty and the kernel returns at once.
-//  * rounds r = 1..R (step 5): recompute the rows of the blocks
-//    flagged in round r-1, recompute t1/t2, re-check; survivors form round
-//    r's list.  One warp per flagged block, grid-stride.
+//    (aligned 1024-group partials written by all CTAs; after one grid
+//    barrier every CTA reduces them -- the same bits everywhere), and each
+//    candidate is flagged iff NOT(|s_k| <= K_k beta).  No candidates:
+//    flags are empty and the kernel returns at once.
+//  * rounds r = 1..R (step 5): each block flagged in round 0 is
+//    recomputed (rows, t1, t2) and re-checked by one warp until it passes or
+//    R rounds are spent; round r's list holds the blocks failing round r.
+//    No barrier between rounds (a block's rounds depend on no other block).
+//    Matrices with hub rows and few candidates: CTA 0 alone runs the rounds
+//    round by round, each round's hub chunk sums spread over its warps.
 template <bool INJECT, bool CONFIRM>
 __global__ void __launch_bounds__(256) k_finish(const SpmvArgs a, int rounds) {
   __shared__ double s_red[256];
-  __shared__ double s_beta;
   asm volatile("griddepcontrol.wait;" ::: "memory");
   if (skip_call(a)) return;
   const int lane = threadIdx.x & 31;
-  bool solo = false;  // CTA 0 alone runs confirmation and rounds
+  const bool hub_m = a.n_own > 0 && a.bs <= 32;
+  bool hub_solo = false;
+  double beta;
+  int32_t nitems;
+  const int32_t *items;
   if (CONFIRM) {
     const int nc = __ldcg(a.n_cand);
     if (nc == 0) {
@@ -1435,64 +1515,60 @@ __global__ void __launch_bounds__(256) k_finish(const SpmvArgs a, int rounds) {
     }
     if (blockIdx.x == 0 && threadIdx.x == 0)
       for (int r = 0; r <= a.max_rounds; ++r) a.n_flags[r] = 0;
-    // few candidates (the usual faulty call): after the beta partials CTA 0
-    // alone confirms and corrects, with block barriers instead of grid ones
-    solo = nc <= kFewCand;
-    double beta;
-    if (a.x_norm) {
-      beta = __ldcg(a.x_norm);
-    } else {
-      const int64_t nch = (a.ngroups + kBetaChunk - 1) / kBetaChunk;
+    hub_solo = hub_m && nc <= kFewCand && rounds > 0;
+    const int64_t nch = (a.ngroups + kBetaChunk - 1) / kBetaChunk;
+    if (!a.x_norm)
       for (int64_t c = blockIdx.x; c < nch; c += gridDim.x) {
         const double v = cta_pw_array(a.gsum + c * kBetaChunk,
                                       min64(kBetaChunk, a.ngroups - c * kBetaChunk), s_red);
         if (threadIdx.x == 0) a.bpart[c] = v;
       }
-      if (!grid_sync(a.gbar)) return;
-      if (solo && blockIdx.x != 0) return;
-      beta = __dsqrt_rn(cta_pw_array(a.bpart, nch, s_red));  // R10
-    }
-    if (solo && blockIdx.x != 0) return;
-    if (threadIdx.x == 0) s_beta = beta;
-    if (solo)
-      __syncthreads();
-    else if (!grid_sync(a.gbar))  // n_flags zeroed, partials consumed
-      return;
-    beta = s_beta;
-    for (int q = blockIdx.x * blockDim.x + threadIdx.x; q < nc; q += gridDim.x * blockDim.x) {
-      const int32_t kk = __ldcg(a.cand + q);
-      const double sv = __ldcg(a.cand_s + q);
-      const double tau = dmul(__ldg(a.K + kk), beta);  // tau_k = K_k * beta
-      if (!(fabs(sv) <= tau)) a.flags[atomicAdd(a.n_flags, 1)] = kk;
-    }
+    // n_flags zeroed, partials written, n_cand read by every CTA
+    if (!grid_sync(a.gbar)) return;
+    if (hub_solo && blockIdx.x != 0) return;
+    beta = a.x_norm ? __ldcg(a.x_norm) : __dsqrt_rn(cta_pw_array(a.bpart, nch, s_red));  // R10
     if (blockIdx.x == 0 && threadIdx.x == 0) {
       *a.beta = beta;
       *a.beta_valid = 1;
+      *a.n_cand = 0;
     }
-    if (solo)
-      __syncthreads();
-    else if (!grid_sync(a.gbar))  // round 0's list complete; every CTA has read n_cand
-      return;
-    if (blockIdx.x == 0 && threadIdx.x == 0) *a.n_cand = 0;
+    // one warp per candidate: confirm, then (not hub_solo) its rounds
+    const int64_t gw = hub_solo ? (int64_t)(threadIdx.x >> 5)
+                                : ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = hub_solo ? (int64_t)(blockDim.x >> 5) : ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t q = gw; q < nc; q += nw) {
+      const int32_t kk = __ldcg(a.cand + q);
+      const double sv = __ldcg(a.cand_s + q);
+      if (fabs(sv) <= dmul(__ldg(a.K + kk), beta)) continue;  // tau_k = K_k * beta
+      if (lane == 0) a.flags[atomicAdd(a.n_flags, 1)] = kk;
+      if (!hub_solo) block_rounds<INJECT>(a, kk, rounds, lane, beta);
+    }
+    if (!hub_solo) return;
+    __syncthreads();  // round 0's list complete
+    nitems = __ldcg(a.n_flags);
+    items = a.flags;
+  } else {
+    beta = __ldcg(a.beta);
+    nitems = __ldcg(a.n_flags);
+    items = a.flags;
+    const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t q = gw; q < nitems; q += nw)
+      block_rounds<INJECT>(a, __ldcg(items + q), rounds, lane, beta);
+    return;
   }
-  if (rounds == 0 || __ldcg(a.n_flags) == 0) return;
-  const int64_t gw = solo ? (int64_t)(threadIdx.x >> 5)
-                          : ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  const int64_t nw = solo ? (int64_t)(blockDim.x >> 5) : ((int64_t)gridDim.x * blockDim.x) >> 5;
-  const double beta = __ldcg(a.beta);
-  const int64_t n = a.n;
+  // hub_solo: CTA 0, round by round
+  const int64_t gw = threadIdx.x >> 5, nw = blockDim.x >> 5;
   const LdgSrc As{a.va, a.ci}, Cs{a.cval, a.ccol};
   for (int round = 1; round <= rounds; ++round) {
-    const int32_t nprev = __ldcg(a.n_flags + round - 1);
-    if (nprev == 0) break;  // uniform: every CTA reads it after the barrier
+    const int32_t nprev = round == 1 ? nitems : __ldcg(a.n_flags + round - 1);
+    if (nprev == 0) break;
     const int32_t *prev = a.flags + (int64_t)(round - 1) * a.nb;
     int32_t *next = a.flags + (int64_t)round * a.nb;
-    // solo rounds on a matrix with hub rows (> kHubLen entries): first the
-    // flagged blocks' hub chunk sums, spread over the CTA's warps (a hub row
-    // of 40k entries is 40 chunks, not one warp's serial chain), then the
+    // the flagged blocks' hub chunk sums, spread over the CTA's warps (a hub
+    // row of 40k entries is 40 chunks, not one warp's serial chain), then the
     // blocks below combine them (hub_sum: aligned subtrees == PW)
-    const bool hubs = solo && a.n_own > 0 && a.bs <= 32;
-    if (hubs) {
+    {
       int item = 0;  // running chunk index over the flagged blocks (uniform)
       const int per_g = 32 >> a.log2bs;
       for (int q = 0; q < nprev; ++q) {
@@ -1521,68 +1597,12 @@ __global__ void __launch_bounds__(256) k_finish(const SpmvArgs a, int rounds) {
     }
     for (int64_t q = gw; q < nprev; q += nw) {
       const int64_t k = __ldcg(prev + q);
-      int olo = 0, ohi = 0;  // hub rows of the block's group (solo rounds)
-      if (hubs && (__ldg(a.lean_ok + ((k << a.log2bs) >> 5)) & 2))
-        own_range(a, (k << a.log2bs) >> 5, olo, ohi);
-      if (a.bs > 32) {  // big blocks: recompute the block's groups, re-verify
-        const double sv = big_block<true, INJECT>(a, k, round, lane, nullptr);
-        if (lane == 0 && !(fabs(sv) <= dmul(__ldg(a.K + k), beta)))
-          next[atomicAdd(a.n_flags + round, 1)] = (int32_t)k;
-        continue;
-      }
-      const int64_t i = (k << a.log2bs) + lane;
-      const bool valid = lane < a.bs && i < n;
-      int32_t rs = 0, len = 0;
-      if (valid) {
-        rs = __ldg(a.rp + i);
-        len = __ldg(a.rp + i + 1) - rs;
-      }
-      const int maxlen = warp_max_i(len);
-      double yv = 0.0;
-      if (maxlen <= 32) {
-        if (valid) yv = lane_dot_any(As, rs, len, maxlen, a.x);
-      } else {
-        for (int j = 0; j < a.bs; ++j) {
-          const int32_t rb = __shfl_sync(kFull, rs, j);
-          const int rl = __shfl_sync(kFull, len, j);
-          if ((k << a.log2bs) + j >= n) break;
-          double t;
-          const int e = rl > kHubLen ? own_find(a, olo, ohi, (int)(((k << a.log2bs) + j) & 31)) : -1;
-          if (e >= 0)
-            t = hub_sum(a, __ldg(a.own_first + e), __ldg(a.own_n + e));
-          else
-            t = warp_dot(As, rb, rl, a.x, lane);
-          if (lane == j) yv = t;
-        }
-      }
-      if (len == 0) yv = 0.0;
-      if (INJECT) {
-        const uint64_t m = group_y_mask(a.inj, round, k << a.log2bs, i, lane);
-        if (valid) yv = apply_mask(yv, m);
-      }
-      if (valid) a.y[i] = yv;
-      double t2 = bfly32(valid ? yv : kAbsent);
-      const int32_t cb = __ldg(a.crp + k), ce = __ldg(a.crp + k + 1);
-      const int ec = ce - cb > kHubLen
-                         ? own_find(a, olo, ohi, 32 + (int)(k & ((32 >> a.log2bs) - 1))) : -1;
-      double t1 = ec >= 0 ? hub_sum(a, __ldg(a.own_first + ec), __ldg(a.own_n + ec))
-                          : warp_dot(Cs, cb, ce - cb, a.x, lane);
-      if (lane == 0) {
-        if (INJECT) {
-          t1 = apply_mask(t1, fault_mask(a.inj, round, 1, k, 2 * (int64_t)(ce - cb)));
-          t2 = apply_mask(t2, fault_mask(a.inj, round, 2, k, min64(a.bs, n - (k << a.log2bs))));
-        }
-        const double sv = dsub(t1, t2);
-        if (!(fabs(sv) <= dmul(__ldg(a.K + k), beta)))
-          next[atomicAdd(a.n_flags + round, 1)] = (int32_t)k;
-      }
+      int olo = 0, ohi = 0;
+      if (__ldg(a.lean_ok + ((k << a.log2bs) >> 5)) & 2) own_range(a, (k << a.log2bs) >> 5, olo, ohi);
+      if (fin_block<INJECT>(a, k, round, lane, beta, olo, ohi) && lane == 0)
+        next[atomicAdd(a.n_flags + round, 1)] = (int32_t)k;
     }
-    if (round < rounds) {
-      if (solo)
-        __syncthreads();
-      else if (!grid_sync(a.gbar))
-        return;
-    }
+    __syncthreads();
   }
 }
 

@@ -228,30 +228,6 @@ __device__ __forceinline__ void cvals8(const unsigned char *p, double (&c)[8]) {
   for (int u = 0; u < 8; ++u) c[u] = (double)v[u];
 }
 
-// INJECT: fault-list ranges of group g (round 0): [y0, y1) rows, [k0, k1)
-// t1, [q0, q1) t2 -- six binary searches on lanes 0..5 at once.
-__device__ __forceinline__ InjRange inj_range_group(const InjDev &inj, int64_t g, int lane) {
-  InjRange R{0, 0, 0, 0, 0, 0};
-  int v = 0;
-  const int len = inj.mode == 1 ? list_len(inj) : 0;
-  if (len > 0 && lane < 6) {
-    const uint64_t k = lane == 0   ? list_key(0, 0, g * 32)
-                       : lane == 1 ? list_key(0, 0, g * 32 + 32)
-                       : lane == 2 ? list_key(0, 1, g)
-                       : lane == 3 ? list_key(0, 1, g + 1)
-                       : lane == 4 ? list_key(0, 2, g)
-                                   : list_key(0, 2, g + 1);
-    v = list_lower(inj, len, k);
-  }
-  R.y0 = __shfl_sync(kFull, v, 0);
-  R.y1 = __shfl_sync(kFull, v, 1);
-  R.k0 = __shfl_sync(kFull, v, 2);
-  R.k1 = __shfl_sync(kFull, v, 3);
-  R.q0 = __shfl_sync(kFull, v, 4);
-  R.q1 = __shfl_sync(kFull, v, 5);
-  return R;
-}
-
 // Consumer: group g from stage `st` (header hdr, warp w, scratch xs).
 template <bool CHECK, bool INJECT, int CF, bool SHORT>
 __device__ __forceinline__ void stream_group(const SpmvArgs &a, const StreamCfg &c, int64_t g,
@@ -271,8 +247,7 @@ __device__ __forceinline__ void stream_group(const SpmvArgs &a, const StreamCfg 
   const int re = a0 + ro[lane];
   const int rs = lane ? a0 + ro[lane - 1] : a0;
   const int len = re - rs;
-  InjRange R{0, 0, 0, 0, 0, 0};
-  if (INJECT) R = inj_range_group(a.inj, g, lane);
+  const bool hit = INJECT && inj_group_hit(a.inj, g);
 
   // C positions of this lane's row (CHECK): the regular row's bases, or
   // the lane's own block when it is an exception row
@@ -335,7 +310,11 @@ __device__ __forceinline__ void stream_group(const SpmvArgs &a, const StreamCfg 
     yv = dadd(s01, s23);
   }
   if (len == 0) yv = 0.0;  // PW of an empty row is +0.0 (R2)
-  if (INJECT && R.y0 < R.y1) yv = apply_mask(yv, list_mask_in(a.inj, R.y0, R.y1, list_key(0, 0, i)));
+  InjMasks M{0, 0, 0};
+  if (INJECT && hit) {
+    M = inj_masks(a.inj, g, i);
+    yv = apply_mask(yv, M.y);
+  }
   a.y[i] = yv;
   if (!CHECK) return;
 
@@ -394,9 +373,9 @@ __device__ __forceinline__ void stream_group(const SpmvArgs &a, const StreamCfg 
       if (t < nt) q[t] = bfly32(q[t]);
   }
   double t1 = (!SHORT && nC > 256) ? tree<4>(q) : q[0];  // nC > 0 (eligible groups)
-  if (INJECT && lane == 0) {
-    if (R.k0 < R.k1) t1 = apply_mask(t1, list_mask_in(a.inj, R.k0, R.k1, list_key(0, 1, g)));
-    if (R.q0 < R.q1) t2 = apply_mask(t2, list_mask_in(a.inj, R.q0, R.q1, list_key(0, 2, g)));
+  if (INJECT && hit) {
+    t1 = apply_mask(t1, M.t1);
+    t2 = apply_mask(t2, M.t2);
   }
   if (lane == 0) {
     if (a.dbg_t1) {
@@ -421,11 +400,12 @@ struct ShortA {
   int rs, len;
   int ml;    // longest row of the group (uniform)
   bool uni;  // every row of the group has ml entries (uniform)
+  bool hit;  // INJECT: the group may hold a round-0 fault (inj_group_hit)
   double xj[8];
   double xi;
 };
 
-template <bool CHECK>
+template <bool CHECK, bool INJECT>
 __device__ __forceinline__ void short_load(const SpmvArgs &a, const StreamCfg &c, const double *xg,
                                            int64_t g, int w, const unsigned char *st, int lane,
                                            ShortA &A) {
@@ -439,6 +419,7 @@ __device__ __forceinline__ void short_load(const SpmvArgs &a, const StreamCfg &c
   const int re = a0 + ro[lane];
   const int rs = lane ? a0 + ro[lane - 1] : a0;
   A.xi = CHECK ? ld_x(a.xr + g * 32 + lane) : 0.0;
+  A.hit = INJECT && inj_group_hit(a.inj, g);
   A.rs = rs;
   A.len = re - rs;
   A.ml = warp_max_i(A.len);
@@ -478,9 +459,11 @@ __device__ __forceinline__ void short_finish(const SpmvArgs &a, const StreamCfg 
     }
     yv = A.len > 0 ? tree<8>(v) : 0.0;  // PW of an empty row is +0.0 (R2)
   }
-  InjRange R{0, 0, 0, 0, 0, 0};
-  if (INJECT) R = inj_range_group(a.inj, g, lane);
-  if (INJECT && R.y0 < R.y1) yv = apply_mask(yv, list_mask_in(a.inj, R.y0, R.y1, list_key(0, 0, i)));
+  InjMasks M{0, 0, 0};
+  if (INJECT && A.hit) {
+    M = inj_masks(a.inj, g, i);
+    yv = apply_mask(yv, M.y);
+  }
   a.y[i] = yv;
   if (!CHECK) return;
   const unsigned char *rec = A.rec;
@@ -529,9 +512,9 @@ __device__ __forceinline__ void short_finish(const SpmvArgs &a, const StreamCfg 
     gs = __shfl_sync(kFull, vv, 2);
   }
   double t1 = q0;
-  if (INJECT && lane == 0) {
-    if (R.k0 < R.k1) t1 = apply_mask(t1, list_mask_in(a.inj, R.k0, R.k1, list_key(0, 1, g)));
-    if (R.q0 < R.q1) t2 = apply_mask(t2, list_mask_in(a.inj, R.q0, R.q1, list_key(0, 2, g)));
+  if (INJECT && A.hit) {
+    t1 = apply_mask(t1, M.t1);
+    t2 = apply_mask(t2, M.t2);
   }
   if (lane == 0) {
     if (a.dbg_t1) {
@@ -668,7 +651,7 @@ __global__ void __launch_bounds__((kStreamMaxG + 1) * 32, 2) k_stream(const Spmv
       const int32_t g0 = hdr[3 * G + 3];
       if (g0 < 0) return;
       if (warp < hdr[3 * G + 4])
-        short_load<CHECK>(a, c, xg, (int64_t)g0 + warp, warp, ring + (size_t)s * c.stage_bytes, lane, sa);
+        short_load<CHECK, INJECT>(a, c, xg, (int64_t)g0 + warp, warp, ring + (size_t)s * c.stage_bytes, lane, sa);
       else
         sa.g = -1;
     }
@@ -687,7 +670,7 @@ __global__ void __launch_bounds__((kStreamMaxG + 1) * 32, 2) k_stream(const Spmv
       const int32_t g0n = hdr1[3 * G + 3];
       nx.g = -1;
       if (g0n >= 0 && warp < hdr1[3 * G + 4])
-        short_load<CHECK>(a, c, xg, (int64_t)g0n + warp, warp, st1, lane, nx);
+        short_load<CHECK, INJECT>(a, c, xg, (int64_t)g0n + warp, warp, st1, lane, nx);
       if (cu.g >= 0) short_finish<CHECK, INJECT, CF>(a, c, cu, xs, lane);
       __syncwarp();
       if (lane == 0) mbar_arrive(empty + s);

@@ -554,3 +554,41 @@ def test_compact_c_with_huge_hub_row(O, torch_cuda):
     plan = G.FaultPlan([0, 0, 0], [0, 0, 1], [40001, 17, 40001 // 32], [1 << 62, 1 << 61, 1 << 60])
     ref = c.run(G.uniform_vector(n, 4), plan=plan)
     assert set([40001 // 32, 0]) <= set(ref.flagged.tolist())
+
+
+@pytest.mark.parametrize("lam", [1e-5, 1e-3])
+def test_resident_plan(O, torch_cuda, lam):
+    # ABFT_INJ_RESIDENT: the plan abft_inject_prepare builds is exactly the
+    # oracle's rate plan of that call (R13), and protected calls reusing it
+    # repeat the rate-mode call bit for bit (same faults, no plan generation).
+    from paper_conf_dsn_schollbkw16_b200 import AUTOCORRECT, CHECK, Inject, encode
+    A = MATRICES["lap3d_16"]()
+    enc = O.encode(A, 32)
+    h = encode(A)
+    x = G.uniform_vector(A.n, 21)
+    spec = dict(seed=31, lam=lam, targets=0b111, call=2)
+    ref = O.abft_spmv(A, enc, x, O.Inject.rate(**spec))
+    h.inject_prepare(Inject.rate(**spec), CHECK | AUTOCORRECT)
+    ro, ta, ix, mk = h.inject_list()
+    oro, ota, oix, omk = O.rate_plan(A, enc, O.Inject.rate(**spec))
+    def combined(*cols):  # equal (round, target, index) entries XOR together
+        comb = {}
+        for r, t, i, m in zip(*cols):
+            comb[(int(r), int(t), int(i))] = comb.get((int(r), int(t), int(i)), 0) ^ int(m)
+        return sorted(comb.items())
+    exp = combined(oro, ota, oix, omk)
+    assert combined(ro, ta, ix, mk) == exp and len(exp) > 0
+    assert np.all(np.diff(ro.astype(np.int64) * 4 + ta) >= 0)  # keys ascending
+    xd = torch_cuda.from_numpy(x).cuda()
+    for _ in range(2):
+        y = h.spmv(xd, inject=Inject.resident(), mode=CHECK | AUTOCORRECT)
+        torch_cuda.cuda.synchronize()
+        assert_bits_equal(y.cpu().numpy(), ref.y, "y (resident plan)")
+        for r in range(5):
+            assert np.array_equal(h.flags(r), ref.flags[r]), r
+    # harness control: same lookups, zeroed masks -> the fault-free result
+    h.inject_clear_masks()
+    y = h.spmv(xd, inject=Inject.resident(), mode=CHECK | AUTOCORRECT)
+    torch_cuda.cuda.synchronize()
+    assert_bits_equal(y.cpu().numpy(), O.spmv(A, x), "y (cleared masks)")
+    assert h.flags(0).size == 0
