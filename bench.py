@@ -238,6 +238,9 @@ def run_pcg(args):
             cap = 0 if (check != "checkpoint" or lam == 0 or clean_iters is None) else 10 * clean_iters
             reps = max(1, args.pcg_reps) if lam == 0 else max(1, args.pcg_seeds)
             times, ok, stt = [], 0, None
+            # untimed: first use of this (scheme, lambda) uploads the rate
+            # tables and may grow the device fault list
+            solve(check, lam, 1000, 20, 0 if name == "harness" else None)
             for rep in range(reps):
                 dt, status, st, rel, good = solve(check, lam, 7 + rep, cap,
                                                   0 if name == "harness" else None)

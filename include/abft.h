@@ -271,7 +271,9 @@ typedef struct {
 /* Jacobi-PCG (Saad Alg. 9.1) for SPD A: solves A x = b from the
  * initial guess in x (overwritten with the solution).  diag: nullable device
  * [n] (NULL -> the diagonal of A).  Stops when ||r||_2 <= tol * ||b||_2
- * (R16) or after max_iter iterations (<= 0 -> 10 N).
+ * (R16) or after max_iter iterations (<= 0 -> 10 N);
+ * check | ABFT_PCG_LITERAL_STOP: stops when r^T r < tol instead (P:296's
+ * "||r_k|| = r_k^T r_k < eps" read literally, R16*; not with check == 2).
  * check == 1 protects every SpMV (detect + correct); check == 0 runs the
  * unprotected baseline with the same kernels; check == 2 runs the related-work
  * CHECKPOINTING baseline: every SpMV checked by
@@ -285,6 +287,7 @@ typedef struct {
  * b, x, diag and res_hist must be 16-byte aligned (128-bit vector accesses;
  * ABFT_EINVAL otherwise).
  * Synchronises the stream.  Returns ABFT_OK, ABFT_ENOCONV or ABFT_EBREAKDOWN. */
+enum { ABFT_PCG_LITERAL_STOP = 0x100 };
 abft_status abft_pcg(abft_handle_t h, const double *b, double *x, const double *diag,
                      double tol, int64_t max_iter, const abft_inject_t *inj, int32_t check,
                      double *res_hist, abft_pcg_stats_t *stats, void *stream);

@@ -646,6 +646,9 @@ int or_pcg(const or_csr *A, int32_t bs, const int32_t *c_row_ptr, const int32_t 
            int32_t max_rounds, int32_t check, double *res_hist, int64_t *stats) {
   int64_t n = A->n, nb = (n + bs - 1) / bs;
   if (max_iter <= 0) max_iter = 10 * n;
+  /* P:296 read literally: stop when r^T r < eps (R16*); default: ||r|| <= eps ||b|| */
+  const int literal = (check & OR_PCG_LITERAL_STOP) != 0;
+  check &= ~OR_PCG_LITERAL_STOP;
   size_t vb = sizeof(double) * (size_t)(n > 0 ? n : 1);
   double *r = (double *)malloc(vb), *z = (double *)malloc(vb), *p = (double *)malloc(vb);
   double *q = (double *)malloc(vb), *tmp = (double *)malloc(vb), *d = (double *)malloc(vb);
@@ -698,10 +701,12 @@ int or_pcg(const or_csr *A, int32_t bs, const int32_t *c_row_ptr, const int32_t 
   double rho = dot_pw(r, z, n, tmp);
   double bnorm = sqrt(dot_pw(b, b, n, tmp));
   double thr = tol * bnorm;
-  double res = sqrt(dot_pw(r, r, n, tmp));
+  double rr = dot_pw(r, r, n, tmp);
+  double res = sqrt(rr);
   res_hist[0] = res;
   int64_t it = 0;
-  while (!(res <= thr) && it < max_iter) {
+#define PCG_DONE (literal ? (rr < tol) : (res <= thr))
+  while (!PCG_DONE && it < max_iter) {
     if (res != res) {
       rc = -7;
       break;
@@ -717,7 +722,8 @@ int or_pcg(const or_csr *A, int32_t bs, const int32_t *c_row_ptr, const int32_t 
     for (int64_t i = 0; i < n; ++i) r[i] = r[i] - alpha * q[i];
     for (int64_t i = 0; i < n; ++i) z[i] = r[i] / d[i];
     double rho_new = dot_pw(r, z, n, tmp);
-    res = sqrt(dot_pw(r, r, n, tmp));
+    rr = dot_pw(r, r, n, tmp);
+    res = sqrt(rr);
     ++it;
     res_hist[it] = res;
     double beta = rho_new / rho;
@@ -725,7 +731,8 @@ int or_pcg(const or_csr *A, int32_t bs, const int32_t *c_row_ptr, const int32_t 
     for (int64_t i = 0; i < n; ++i) p[i] = z[i] + beta * p[i];
   }
 #undef PROTECTED_SPMV
-  if (rc == 0 && !(res <= thr)) rc = -5;
+  if (rc == 0 && !PCG_DONE) rc = -5;
+#undef PCG_DONE
   stats[0] = it;
   stats[1] = calls;
   free(r);

@@ -106,7 +106,10 @@ int or_dense_spmv(const or_csr *A, const double *c, double k35, int32_t bound35,
 /* --- Jacobi-PCG with the protected SpMV (Saad Alg. 9.1) ---
  * res_hist [max_iter+1].  stats: [0] iters, [1] spmv calls, [2] flagged blocks
  * (round 0, summed), [3] recomputed blocks (summed over rounds), [4] uncorrected
- * calls.  Returns 0 converged, -5 not converged, -7 breakdown. */
+ * calls.  Returns 0 converged, -5 not converged, -7 breakdown.
+ * check: 0 plain SpMV, 1 protected; | OR_PCG_LITERAL_STOP: stop when
+ * r^T r < tol (P:296 read literally, R16*) instead of ||r|| <= tol ||b||. */
+#define OR_PCG_LITERAL_STOP 0x100
 int or_pcg(const or_csr *A, int32_t bs, const int32_t *c_row_ptr, const int32_t *c_col,
            const double *c_val, const double *K, const double *b, double *x,
            const double *diag, double tol, int64_t max_iter, const or_inject *inj,

@@ -334,7 +334,8 @@ class PcgResult:
 
 
 def pcg(A, enc: Encoded, b, x0, diag=None, tol=1e-6, max_iter=0, inj: Inject | None = None,
-        max_rounds=4, check=True) -> PcgResult:
+        max_rounds=4, check=True, literal_stop=False) -> PcgResult:
+    """or_pcg; literal_stop: stop when r^T r < tol (P:296 read literally)."""
     r = _CsrRef(A)
     b = np.ascontiguousarray(b, dtype=np.float64)
     x = np.array(x0, dtype=np.float64, copy=True)
@@ -345,7 +346,8 @@ def pcg(A, enc: Encoded, b, x0, diag=None, tol=1e-6, max_iter=0, inj: Inject | N
     ist = inj._struct() if inj is not None else None
     st = lib().or_pcg(r.ref(), enc.bs, _p(enc.row_ptr), _p(enc.col), _p(enc.val), _p(enc.K),
                       _p(b), _p(x), _p(d), tol, mi, C.byref(ist) if ist is not None else None,
-                      max_rounds, 1 if check else 0, _p(hist), _p(stats))
+                      max_rounds, (1 if check else 0) | (0x100 if literal_stop else 0),
+                      _p(hist), _p(stats))
     it = int(stats[0])
     return PcgResult(st, x, hist[: it + 1].copy(), it, int(stats[1]), int(stats[2]),
                      int(stats[3]), int(stats[4]))

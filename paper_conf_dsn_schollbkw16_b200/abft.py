@@ -22,6 +22,7 @@ OK, EINVAL, ECUDA, ENOMEM, ENOTSUP, ENOCONV, EUNCORRECTED, EBREAKDOWN, ENCCL = (
 NOCHECK, CHECK, AUTOCORRECT, DEBUG_CHECKSUMS, DEFER_FINISH = 0, 1, 2, 4, 8
 DENSE_BOUND35 = 16  # abft_spmv_dense: tau = K35 ||x|| ([35]) instead of ||x|| ([30])
 INJ_NONE, INJ_LIST, INJ_RATE, INJ_RESIDENT = 0, 1, 2, 3
+PCG_LITERAL_STOP = 0x100
 
 SYMBOLS = [
     "abft_encode", "abft_spmv", "abft_correct", "abft_flags", "abft_beta",
@@ -527,14 +528,16 @@ class Handle:
 
     # -- PCG ----------------------------------------------------------------
     def pcg(self, b, x, diag=None, tol=1e-6, max_iter=0, inject: Inject | None = None,
-            check=True, res_hist=None, stream=None):
+            check=True, res_hist=None, stream=None, literal_stop=False):
         # check: True = the method's protected SpMV, False = unprotected,
         # "checkpoint" = dense-check checkpoint-rollback baseline (
         # needs dense_encode(); stats: flagged_blocks = rollbacks,
-        # recomputed_blocks = discarded iterations)
+        # recomputed_blocks = discarded iterations).  literal_stop: stop when
+        # r^T r < tol (P:296 read literally) instead of ||r|| <= tol ||b||.
         st = PcgStats()
         inj = inject.struct() if inject is not None else None
-        mode = 2 if check == "checkpoint" else (1 if check else 0)
+        mode = (2 if check == "checkpoint" else (1 if check else 0)) | (
+            PCG_LITERAL_STOP if literal_stop else 0)
         mi = max_iter if max_iter > 0 else 10 * self.n
         status = lib().abft_pcg(self._h, _vec(b, self.n, "b"), _vec(x, self.n, "x"),
                                 _vec(diag, self.n, "diag", optional=True), tol, max_iter,

@@ -161,6 +161,7 @@ struct abft_ctx {
   bool list_cached = false;
   uint32_t *inj_gbits = nullptr;  // [ceil(ngroups / 32)] group bitmap of the device list
   int32_t *inj_gstart = nullptr;  // [3][ngroups] first entry of (target, group)
+  int32_t *op_ybkt = nullptr, *op_cbkt = nullptr;  // rate plans: op -> row / block buckets
   InjDev inj_last{};        // the device plan the last injecting call built (ABFT_INJ_RESIDENT)
   bool inj_last_valid = false;
   // rate-mode plan scratch
@@ -184,6 +185,12 @@ struct abft_ctx {
   // PCG scratch
   double *pcg = nullptr;  // r, z, p, q, d : 5 n
   double *pcg_part = nullptr;
+  double *pcg_pq = nullptr;  // [ngroups] p.q group partials of the fused SpMV epilogue
+  // abft_pcg's device-resident loop: the instantiated graph, the key of
+  // what it bakes in (PcgGraphKey), its capture stream
+  cudaGraphExec_t pcg_exec = nullptr;
+  alignas(8) unsigned char pcg_key[1024] = {};
+  cudaStream_t pcg_cap = nullptr;
   double *pcg_sc = nullptr;
   int32_t *pcg_state = nullptr;
   int64_t pcg_n = 0;
@@ -342,6 +349,16 @@ abft_status gen_rate_plan(abft_ctx *h, const abft_inject_t *inj, uint64_t call, 
   r.y_ops = 2 * h->nnz;
   r.t1_ops = check ? 2 * h->nnz_c : 0;
   r.ops = r.y_ops + r.t1_ops + (check ? h->n : 0);
+  if (!h->op_ybkt) {  // once per handle: the op -> row lookup buckets
+    const int64_t ny = ((2 * h->nnz) >> kOpBktShift) + 2, nc = ((2 * h->nnz_c) >> kOpBktShift) + 2;
+    TRY(dalloc(h, &h->op_ybkt, (size_t)ny));
+    TRY(dalloc(h, &h->op_cbkt, (size_t)nc));
+    k_op_buckets<<<(unsigned)((ny + 255) / 256), 256, 0, s>>>(h->rp, h->n, ny, h->op_ybkt);
+    k_op_buckets<<<(unsigned)((nc + 255) / 256), 256, 0, s>>>(h->c_rp, h->nb, nc, h->op_cbkt);
+    CK(cudaGetLastError());
+  }
+  r.ybkt = h->op_ybkt;
+  r.cbkt = h->op_cbkt;
   r.rounds = check ? h->max_rounds : 0;
   r.ch = FaultTables::chunk(inj->lambda);
   r.nch = std::max<int64_t>(1, (r.ops + r.ch - 1) / r.ch);
@@ -1330,6 +1347,11 @@ int64_t abft_rate_chunk(double lambda) { return FaultTables::chunk(lambda); }
 
 abft_status abft_destroy(abft_handle_t h) {
   if (!h) return ABFT_EINVAL;
+  if (h->pcg_exec) cudaGraphExecDestroy(h->pcg_exec);
+  if (h->pcg_cap) {
+    cudaStreamSynchronize(h->pcg_cap);
+    cudaStreamDestroy(h->pcg_cap);
+  }
   if (h->cs) {
     cudaStreamSynchronize(h->cs);
     cudaStreamDestroy(h->cs);

@@ -304,7 +304,37 @@ struct RatePlanArgs {
   const int32_t *offs;  // exclusive scan of counts
   uint64_t *keys, *masks;
   int64_t cap;          // capacity of keys/masks
+  // op -> row lookup: bkt[b] = the row (block) holding op b << kOpBktShift
+  // (largest i with 2 rp[i] <= op); the search then spans bkt[b]..bkt[b+1]
+  const int32_t *ybkt, *cbkt;
 };
+
+constexpr int kOpBktShift = 8;  // ops per bucket of the op -> row lookup (256)
+
+// bkt[b] = largest i in [0, n] with 2 rp[i] <= b << kOpBktShift, b in [0, nbkt)
+__global__ void k_op_buckets(const int32_t *__restrict__ rp, int64_t n, int64_t nbkt,
+                             int32_t *bkt) {
+  const int64_t b = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (b >= nbkt) return;
+  const int64_t p = b << kOpBktShift;
+  int64_t lo = 0, hi = n;
+  while (lo < hi) {
+    const int64_t mid = lo + (hi - lo + 1) / 2;
+    if (2 * (int64_t)rp[mid] <= p) lo = mid; else hi = mid - 1;
+  }
+  bkt[b] = (int32_t)lo;
+}
+
+// largest i in [bkt[p >> s], bkt[(p >> s) + 1]] with 2 rp[i] <= p
+__device__ __forceinline__ int64_t op_row(const int32_t *rp, const int32_t *bkt, int64_t p) {
+  const int64_t b = p >> kOpBktShift;
+  int64_t lo = __ldg(bkt + b), hi = __ldg(bkt + b + 1);
+  while (lo < hi) {
+    const int64_t mid = lo + (hi - lo + 1) / 2;
+    if (2 * (int64_t)__ldg(rp + mid) <= p) lo = mid; else hi = mid - 1;
+  }
+  return lo;
+}
 
 template <bool WRITE>
 __global__ void k_rate_plan(const RatePlanArgs a) {
@@ -342,22 +372,11 @@ __global__ void k_rate_plan(const RatePlanArgs a) {
     int tgt;
     int64_t idx;
     if (p < a.y_ops) {  // largest row i with 2 rp[i] <= p
-      int64_t lo = 0, hi = a.n;
-      while (lo < hi) {
-        const int64_t mid = lo + (hi - lo + 1) / 2;
-        if (2 * (int64_t)a.rp[mid] <= p) lo = mid; else hi = mid - 1;
-      }
       tgt = 0;
-      idx = lo;
-    } else if (p < a.y_ops + a.t1_ops) {
-      const int64_t qq = p - a.y_ops;
-      int64_t lo = 0, hi = a.nb;
-      while (lo < hi) {
-        const int64_t mid = lo + (hi - lo + 1) / 2;
-        if (2 * (int64_t)a.crp[mid] <= qq) lo = mid; else hi = mid - 1;
-      }
+      idx = op_row(a.rp, a.ybkt, p);
+    } else if (p < a.y_ops + a.t1_ops) {  // largest block k with 2 crp[k] <= p - y_ops
       tgt = 1;
-      idx = lo;
+      idx = op_row(a.crp, a.cbkt, p - a.y_ops);
     } else {
       tgt = 2;
       idx = (p - a.y_ops - a.t1_ops) / a.bs;

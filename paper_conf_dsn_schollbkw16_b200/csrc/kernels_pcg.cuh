@@ -30,6 +30,7 @@ struct PcgScalars {
   int64_t upd;               // host iteration index of the last executed update
   double ck_rho, ck_res;     // checkpoint mode: sampled scalars
   int64_t ck_it;
+  int64_t j;                 // device-resident loop: the next iteration's index (1-based)
 };
 
 struct PcgArgs {
@@ -59,7 +60,16 @@ struct PcgArgs {
   double *dsend;
   double *pext;
   double *s;  // single-reduction variant (cg1): s = A p, updated by recurrence
+  // stopping rule: 0 = ||r|| <= tol ||b|| (R16); 1 = r^T r < tol (P:296 read
+  // literally, R16*)
+  int32_t literal;
 };
+
+// The stopping test on res = ||r|| (R16) or RR = r^T r (R16*); thr is
+// tol ||b|| resp. tol.
+__device__ __forceinline__ bool pcg_done(const PcgArgs &a, double res, double RR, double thr) {
+  return a.literal ? (RR < thr) : (res <= thr);
+}
 
 // Eight consecutive doubles v[0..8) at p + 8t (or absent past n).
 __device__ __forceinline__ void ld8(double (&v)[8], const double *p, int64_t i0, int64_t n) {
@@ -102,6 +112,35 @@ __device__ __forceinline__ double cta_pw(double (&v)[8], int64_t i0, int64_t n, 
 #pragma unroll
   for (int q = 0; q < 8; ++q) w[q] = s_w[q];
   return tree<8>(w);
+}
+
+// Two chunk sums at once (one barrier pair): s_w holds 16 doubles.
+__device__ __forceinline__ void cta_pw2(double (&v)[8], double (&w)[8], int64_t i0, int64_t n,
+                                        double *s_w, double &out_v, double &out_w) {
+#pragma unroll
+  for (int u = 0; u < 8; ++u)
+    if (i0 + u >= n) v[u] = w[u] = kAbsent;
+  double t = tree<8>(v), q = tree<8>(w);
+#pragma unroll
+  for (int m = 1; m < 32; m <<= 1) {
+    t = dadd(t, __shfl_xor_sync(kFull, t, m));
+    q = dadd(q, __shfl_xor_sync(kFull, q, m));
+  }
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  __syncthreads();
+  if (lane == 0) {
+    s_w[warp] = t;
+    s_w[8 + warp] = q;
+  }
+  __syncthreads();
+  double a[8], b[8];
+#pragma unroll
+  for (int k = 0; k < 8; ++k) {
+    a[k] = s_w[k];
+    b[k] = s_w[8 + k];
+  }
+  out_v = tree<8>(a);
+  out_w = tree<8>(b);
 }
 
 // Last-CTA completion of PW over partials[0..ncta) (aligned chunk nodes):
@@ -181,10 +220,11 @@ __device__ __forceinline__ void init_scalars(const PcgArgs &a, double RZ, double
   pcg_stats(a, sc);  // the SpMV q = A x0
   sc->rho = RZ;
   sc->res = __dsqrt_rn(RR);
-  sc->thr = dmul(a.tol, __dsqrt_rn(BB));
+  sc->thr = a.literal ? a.tol : dmul(a.tol, __dsqrt_rn(BB));
   sc->it = 0;
   if (a.hist) a.hist[0] = sc->res;
-  sc->state = (sc->res <= sc->thr) ? PCG_CONVERGED : (sc->max_iter <= 0 ? PCG_MAXITER : PCG_RUN);
+  sc->state = pcg_done(a, sc->res, RR, sc->thr) ? PCG_CONVERGED
+                                                : (sc->max_iter <= 0 ? PCG_MAXITER : PCG_RUN);
   if (!(sc->res == sc->res)) sc->state = PCG_BREAKDOWN;
   if (a.cr) {
     sc->calls += 1;
@@ -215,7 +255,7 @@ __device__ __forceinline__ void update_scalars(const PcgArgs &a, int64_t iter, d
   sc->beta = __ddiv_rn(RZ, sc->rho);
   sc->rho = RZ;
   sc->upd = iter;
-  if (res <= sc->thr) sc->state = PCG_CONVERGED;
+  if (pcg_done(a, res, RR, sc->thr)) sc->state = PCG_CONVERGED;
   else if (!(res == res)) sc->state = PCG_BREAKDOWN;
   else if (sc->it >= sc->max_iter) sc->state = PCG_MAXITER;
 }
@@ -308,34 +348,56 @@ __global__ void __launch_bounds__(kPcgThreads) k_pcg_dot(const PcgArgs a) {
   }
 }
 
-// x += alpha p; r -= alpha q; z = r / d; rho' = PW(r.z); res = ||r||;
-// beta = rho'/rho; convergence test (R15, R16).
-__global__ void __launch_bounds__(kPcgThreads) k_pcg_update(const PcgArgs a, int64_t iter) {
+// pq = PW(p.q) from the SpMV's per-group partials (SpmvArgs::pq: aligned
+// 32-row nodes; a CTA's 2048 groups are an aligned node, the last CTA
+// completes the tree -- the same PW as k_pcg_dot over the n products).
+__global__ void __launch_bounds__(kPcgThreads) k_pcg_dotg(const PcgArgs a, const double *pqg,
+                                                          int64_t ngroups) {
   __shared__ double s_w[8];
+  __shared__ double s_red[kPcgThreads];
+  __shared__ int s_flag;
+  if (pcg_skip(a.sc)) return;
+  const int64_t i0 = (int64_t)blockIdx.x * kPcgRows + threadIdx.x * kPcgPer;
+  double v[8];
+  ld8(v, pqg, i0, ngroups);
+  const double PQc = cta_pw(v, i0, ngroups, s_w);
+  if (threadIdx.x == 0) a.part0[blockIdx.x] = PQc;
+  if (!last_cta(a.ticket, &s_flag)) return;
+  const double PQ = grid_pw(a.part0, gridDim.x, s_red);
+  if (threadIdx.x == 0) {
+    if (a.dsend)
+      a.dsend[0] = PQ;
+    else
+      dot_scalars(a, PQ);
+    *a.ticket = 0u;
+  }
+}
+
+// r -= alpha q; z = r / d; rho' = PW(r.z); res = ||r||; beta = rho'/rho;
+// convergence test (R15, R16).  x += alpha p moved to k_pcg_p, which reads
+// p anyway (one vector stream less per iteration; the same bits).
+__global__ void __launch_bounds__(kPcgThreads) k_pcg_update(const PcgArgs a, int64_t iter) {
+  __shared__ double s_w[16];
   __shared__ double s_red[kPcgThreads];
   __shared__ int s_flag;
   if (pcg_skip(a.sc)) return;
   const double alpha = a.sc->alpha;
   const int64_t i0 = (int64_t)blockIdx.x * kPcgRows + threadIdx.x * kPcgPer;
-  double xv[8], pv[8], rv[8], qv[8], dv[8], rz[8], rr[8];
-  ld8(xv, a.x, i0, a.n);
-  ld8(pv, a.p, i0, a.n);
+  double rv[8], qv[8], dv[8], rz[8], rr[8];
   ld8(rv, a.r, i0, a.n);
   ld8(qv, a.q, i0, a.n);
   ld8(dv, a.d, i0, a.n);
 #pragma unroll
   for (int u = 0; u < 8; ++u) {
-    xv[u] = dadd(xv[u], dmul(alpha, pv[u]));
     rv[u] = dsub(rv[u], dmul(alpha, qv[u]));
     dv[u] = __ddiv_rn(rv[u], dv[u]);  // z
     rz[u] = dmul(rv[u], dv[u]);
     rr[u] = dmul(rv[u], rv[u]);
   }
-  st8(a.x, xv, i0, a.n);
   st8(a.r, rv, i0, a.n);
   st8(a.z, dv, i0, a.n);
-  const double RZc = cta_pw(rz, i0, a.n, s_w);
-  const double RRc = cta_pw(rr, i0, a.n, s_w);
+  double RZc, RRc;
+  cta_pw2(rz, rr, i0, a.n, s_w, RZc, RRc);
   if (threadIdx.x == 0) {
     a.part0[blockIdx.x] = RZc;
     a.part1[blockIdx.x] = RRc;
@@ -348,30 +410,37 @@ __global__ void __launch_bounds__(kPcgThreads) k_pcg_update(const PcgArgs a, int
       a.dsend[0] = RZ;
       a.dsend[1] = RR;
     } else {
-      update_scalars(a, iter, RZ, RR);
+      update_scalars(a, iter >= 0 ? iter : a.sc->j, RZ, RR);
     }
     *a.ticket = 0u;
   }
 }
 
-// p = z + beta p.  Runs in the iteration that converged too (as the oracle);
-// skipped only when this iteration's update was skipped.
+// x += alpha p; p = z + beta p (old p for both).  Runs in the iteration
+// that converged too (as the oracle); skipped only when this iteration's
+// update was skipped.
 __global__ void __launch_bounds__(kPcgThreads) k_pcg_p(const PcgArgs a, int64_t iter) {
+  // iter < 0: the device-resident loop's counter (CUDA graph while node)
+  if (iter < 0) iter = *(volatile const int64_t *)&a.sc->j;
   if (*(volatile const int64_t *)&a.sc->upd != iter) return;  // this iteration did not execute
-  const double beta = a.sc->beta;
+  const double beta = a.sc->beta, alpha = a.sc->alpha;
   const int64_t i0 = (int64_t)blockIdx.x * kPcgRows + threadIdx.x * kPcgPer;
-  double zv[8], pv[8];
+  double zv[8], pv[8], xv[8];
   ld8(zv, a.z, i0, a.n);
   ld8(pv, a.p, i0, a.n);
+  ld8(xv, a.x, i0, a.n);
 #pragma unroll
-  for (int u = 0; u < 8; ++u) pv[u] = dadd(zv[u], dmul(beta, pv[u]));
+  for (int u = 0; u < 8; ++u) {
+    xv[u] = dadd(xv[u], dmul(alpha, pv[u]));
+    pv[u] = dadd(zv[u], dmul(beta, pv[u]));
+  }
+  st8(a.x, xv, i0, a.n);
   st8(a.p, pv, i0, a.n);
   st8_ext(a.pext, pv, i0, a.n);
   // checkpoint mode: sample (x, r, z, p, rho, it) every ckpt_every iterations
   const int64_t it = a.sc->it;
   if (a.cr && a.ckpt_every > 0 && it % a.ckpt_every == 0) {
-    double xv[8], rv[8];
-    ld8(xv, a.x, i0, a.n);
+    double rv[8];
     ld8(rv, a.r, i0, a.n);
     st8(a.ck, xv, i0, a.n);
     st8(a.ck + a.ns, rv, i0, a.n);
@@ -383,6 +452,16 @@ __global__ void __launch_bounds__(kPcgThreads) k_pcg_p(const PcgArgs a, int64_t 
       a.sc->ck_it = it;
     }
   }
+}
+
+// Device-resident loop (CUDA graph while node): the loop's condition --
+// the solve still runs and the next iteration is within max_iter (executed
+// iterations, as the host loop counts them); bump: advance the counter
+// first (end of an iteration's body).
+__global__ void k_pcg_cond(const PcgArgs a, cudaGraphConditionalHandle hnd, int bump) {
+  PcgScalars *sc = a.sc;
+  if (bump) sc->j += 1;
+  cudaGraphSetConditional(hnd, (sc->state == PCG_RUN && sc->j <= sc->max_iter) ? 1u : 0u);
 }
 
 // Checkpoint mode: after the dense check of this iteration's
@@ -523,7 +602,7 @@ __device__ __forceinline__ void cg1_scalars(const PcgArgs &a, int64_t iter, doub
   sc->res = res;
   if (a.hist) a.hist[sc->it] = res;
   sc->upd = iter;
-  if (res <= sc->thr) {
+  if (pcg_done(a, res, RR, sc->thr)) {
     sc->state = PCG_CONVERGED;
     return;
   }

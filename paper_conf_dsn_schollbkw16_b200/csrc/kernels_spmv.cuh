@@ -112,6 +112,10 @@ struct SpmvArgs {
   double *__restrict__ y;
   const double *x_norm;   // nullable device scalar
   double *gsum;           // [ngroups] x^2 subtree of each group
+  // nullable: [ngroups] PW over the group's rows of x_i y_i (PCG's p.q fused
+  // into the SpMV epilogue, a 32-row aligned node of the global PW tree;
+  // correction rounds rewrite it for the blocks they recompute, b_s = 32)
+  double *pq;
   double *bpart;          // [ceil(ngroups / 1024)] beta partials (k_finish)
   int32_t *n_cand;        // candidate count (reset by k_finish)
   int32_t *cand;          // [nb]
@@ -516,6 +520,10 @@ __device__ __forceinline__ void group_general(const SpmvArgs &a, int64_t g, int 
     if (valid) yv = apply_mask(yv, m);
   }
   if (valid) a.y[i] = yv;
+  if (a.pq) {
+    const double t = bfly32(valid ? dmul(xv, yv) : kAbsent);
+    if (lane == 0) a.pq[g] = t;
+  }
   if (!CHECK) return;
 
   // step 2: t2_k = w_k^T y_k over the b_s slots; absent past n.
@@ -1451,6 +1459,10 @@ __device__ __forceinline__ bool fin_block(const SpmvArgs &a, int64_t k, int roun
     if (valid) yv = apply_mask(yv, m);
   }
   if (valid) a.y[i] = yv;
+  if (a.pq) {  // b_s = 32: the block is the group
+    const double t = bfly32(valid ? dmul(__ldg(a.xr + i), yv) : kAbsent);
+    if (lane == 0) a.pq[k] = t;
+  }
   double t2 = bfly32(valid ? yv : kAbsent);
   const int ec = ce - cb > kHubLen
                      ? own_find(a, olo, ohi, 32 + (int)(k & ((32 >> a.log2bs) - 1))) : -1;

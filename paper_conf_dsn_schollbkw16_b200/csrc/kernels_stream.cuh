@@ -240,7 +240,7 @@ __device__ __forceinline__ void stream_group(const SpmvArgs &a, const StreamCfg 
   const int32_t *ac = reinterpret_cast<const int32_t *>(st + c.off_ac);
   const int64_t i = g * 32 + lane;
   double xi = 0.0;
-  if (CHECK) xi = ld_x(a.xr + i);  // own x_i for the x^2 subtree (L2; issued early)
+  if (CHECK || a.pq) xi = ld_x(a.xr + i);  // own x_i for the x^2 subtree (L2; issued early)
   const unsigned char *rec = st + c.off_srec + hdr[c.G + 1 + w];
   const unsigned char *crec = st + c.off_crec + hdr[2 * c.G + 2 + w];
   const uint16_t *ro = reinterpret_cast<const uint16_t *>(rec);
@@ -316,7 +316,13 @@ __device__ __forceinline__ void stream_group(const SpmvArgs &a, const StreamCfg 
     yv = apply_mask(yv, M.y);
   }
   a.y[i] = yv;
-  if (!CHECK) return;
+  if (!CHECK) {
+    if (a.pq) {
+      const double t = bfly32(dmul(xi, yv));
+      if (lane == 0) a.pq[g] = t;
+    }
+    return;
+  }
 
   // padding positions nC .. roundup8(nC) - 1 hold -0.0 (their c is 0: the
   // product is -0.0, the exact identity of the sum, R2)
@@ -355,8 +361,9 @@ __device__ __forceinline__ void stream_group(const SpmvArgs &a, const StreamCfg 
     // split the values over lane pairs; every value keeps PW's pairing);
     // afterwards lane 4m holds t2, 4m+1 t1 and 4m+2 the x^2 sum
     const bool b0 = lane & 1, b1 = lane & 2;
-    const double s0 = b0 ? t2 : q[0], s1 = b0 ? gs : kAbsent;
-    const double k0 = b0 ? q[0] : t2, k1 = b0 ? kAbsent : gs;
+    const double pq = a.pq ? dmul(xi, yv) : kAbsent;  // 4th value: x_i y_i (PCG p.q)
+    const double s0 = b0 ? t2 : q[0], s1 = b0 ? gs : pq;
+    const double k0 = b0 ? q[0] : t2, k1 = b0 ? pq : gs;
     const double r0 = dadd(k0, __shfl_xor_sync(kFull, s0, 1));
     const double r1 = dadd(k1, __shfl_xor_sync(kFull, s1, 1));
     double v = dadd(b1 ? r1 : r0, __shfl_xor_sync(kFull, b1 ? r0 : r1, 2));
@@ -365,9 +372,14 @@ __device__ __forceinline__ void stream_group(const SpmvArgs &a, const StreamCfg 
     t2 = v;
     q[0] = __shfl_sync(kFull, v, 1);
     gs = __shfl_sync(kFull, v, 2);
+    if (a.pq && lane == 3) a.pq[g] = v;
   } else {
     t2 = bfly32(t2);
     gs = bfly32(gs);
+    if (a.pq) {
+      const double t = bfly32(dmul(xi, yv));
+      if (lane == 0) a.pq[g] = t;
+    }
 #pragma unroll
     for (int t = 0; t < 4; ++t)
       if (t < nt) q[t] = bfly32(q[t]);
@@ -418,7 +430,7 @@ __device__ __forceinline__ void short_load(const SpmvArgs &a, const StreamCfg &c
   const uint16_t *ro = reinterpret_cast<const uint16_t *>(A.rec);
   const int re = a0 + ro[lane];
   const int rs = lane ? a0 + ro[lane - 1] : a0;
-  A.xi = CHECK ? ld_x(a.xr + g * 32 + lane) : 0.0;
+  A.xi = (CHECK || a.pq) ? ld_x(a.xr + g * 32 + lane) : 0.0;
   A.hit = INJECT && inj_group_hit(a.inj, g);
   A.rs = rs;
   A.len = re - rs;
@@ -465,7 +477,13 @@ __device__ __forceinline__ void short_finish(const SpmvArgs &a, const StreamCfg 
     yv = apply_mask(yv, M.y);
   }
   a.y[i] = yv;
-  if (!CHECK) return;
+  if (!CHECK) {
+    if (a.pq) {
+      const double t = bfly32(dmul(A.xi, yv));
+      if (lane == 0) a.pq[g] = t;
+    }
+    return;
+  }
   const unsigned char *rec = A.rec;
   const uint32_t mask = *reinterpret_cast<const uint32_t *>(rec + 68);
   const int nC = *reinterpret_cast<const uint16_t *>(rec + 64);
@@ -500,8 +518,9 @@ __device__ __forceinline__ void short_finish(const SpmvArgs &a, const StreamCfg 
   double t2 = yv, gs = dmul(A.xi, A.xi);
   {
     const bool b0 = lane & 1, b1 = lane & 2;
-    const double s0 = b0 ? t2 : q0, s1 = b0 ? gs : kAbsent;
-    const double k0 = b0 ? q0 : t2, k1 = b0 ? kAbsent : gs;
+    const double pq = a.pq ? dmul(A.xi, yv) : kAbsent;  // 4th value: x_i y_i (PCG p.q)
+    const double s0 = b0 ? t2 : q0, s1 = b0 ? gs : pq;
+    const double k0 = b0 ? q0 : t2, k1 = b0 ? pq : gs;
     const double r0 = dadd(k0, __shfl_xor_sync(kFull, s0, 1));
     const double r1 = dadd(k1, __shfl_xor_sync(kFull, s1, 1));
     double vv = dadd(b1 ? r1 : r0, __shfl_xor_sync(kFull, b1 ? r0 : r1, 2));
@@ -510,6 +529,7 @@ __device__ __forceinline__ void short_finish(const SpmvArgs &a, const StreamCfg 
     t2 = vv;
     q0 = __shfl_sync(kFull, vv, 1);
     gs = __shfl_sync(kFull, vv, 2);
+    if (a.pq && lane == 3) a.pq[g] = vv;
   }
   double t1 = q0;
   if (INJECT && A.hit) {

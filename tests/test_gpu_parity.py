@@ -326,21 +326,22 @@ def test_full_size_config1(O, torch_cuda):
 # --------------------------------------------------------------------------
 # PCG
 # --------------------------------------------------------------------------
-def _pcg_case(O, torch, A, inj_kw=None, check=True, max_iter=0):
+def _pcg_case(O, torch, A, inj_kw=None, check=True, max_iter=0, literal=False, bscale=1.0):
     from paper_conf_dsn_schollbkw16_b200 import encode
     enc = O.encode(A, 32)
     xs = G.uniform_vector(A.n, 43)
-    b = O.spmv(A, xs)
+    b = bscale * O.spmv(A, xs)
     x0 = G.uniform_vector(A.n, 44)
     oinj = O.Inject.rate(**inj_kw) if inj_kw else None
-    ref = O.pcg(A, enc, b, x0, tol=1e-6, inj=oinj, check=check, max_iter=max_iter)
+    ref = O.pcg(A, enc, b, x0, tol=1e-6, inj=oinj, check=check, max_iter=max_iter,
+                literal_stop=literal)
     h = encode(A, 32)
     bd = torch.from_numpy(b).cuda()
     xd = torch.from_numpy(x0.copy()).cuda()
     mi = max_iter if max_iter > 0 else 10 * A.n
     hist = torch.zeros(mi + 1, dtype=torch.float64, device="cuda")
     status, st = h.pcg(bd, xd, tol=1e-6, inject=gpu_inject(rate=inj_kw) if inj_kw else None,
-                       check=check, res_hist=hist, max_iter=max_iter)
+                       check=check, res_hist=hist, max_iter=max_iter, literal_stop=literal)
     torch.cuda.synchronize()
     return ref, status, st, xd.cpu().numpy(), hist.cpu().numpy()[: st["iters"] + 1]
 
@@ -359,6 +360,19 @@ def test_pcg_parity(O, torch_cuda, inj):
     assert_bits_equal(x, ref.x, "solution")
     if inj:
         assert st["flagged_blocks"] > 0
+
+
+@pytest.mark.parametrize("inj", [None, dict(seed=4, lam=1e-4, targets=0b111)])
+def test_pcg_literal_stop(O, torch_cuda, inj):
+    # P:296 read literally (r^T r < eps): bit-exact against the oracle's
+    # literal rule, and a different stopping iteration than the relative one
+    A = G.laplacian_3d_7pt(16)
+    ref, status, st, x, hist = _pcg_case(O, torch_cuda, A, inj, literal=True, bscale=40.0)
+    rel, *_ = _pcg_case(O, torch_cuda, A, inj, bscale=40.0)
+    assert status == ref.status == 0 and st["iters"] == ref.iters != rel.iters
+    assert st["flagged_blocks"] == ref.flagged_blocks
+    assert_bits_equal(hist, ref.res_hist, "literal-stop residual history")
+    assert_bits_equal(x, ref.x, "literal-stop solution")
 
 
 def test_pcg_odd_n(O, torch_cuda):

@@ -542,6 +542,29 @@ class TestPcg:
         spla.cg(S, b, x0=x0.copy(), rtol=1e-8, atol=0.0, callback=lambda xk: cnt.append(1))
         assert r.status == 0 and r.iters == len(cnt)
 
+    def test_literal_stop_matches_scipy_atol(self, O):
+        # P:296 read literally (R16*): stop when r^T r < eps, i.e. ||r|| <
+        # sqrt(eps) -- SciPy's CG with rtol = 0, atol = sqrt(eps) stops at
+        # the same iteration; the relative rule (R16) stops elsewhere here.
+        import scipy.sparse as sp
+        import scipy.sparse.linalg as spla
+        A = G.laplacian_3d_7pt(10)
+        enc = O.encode(A, 32)
+        b = 40.0 * O.spmv(A, G.uniform_vector(A.n, 43))
+        x0 = G.uniform_vector(A.n, 44)
+        eps = 1e-6
+        r = O.pcg(A, enc, b, x0, tol=eps, literal_stop=True)
+        rel = O.pcg(A, enc, b, x0, tol=eps)
+        assert r.status == 0 and r.iters != rel.iters
+        assert r.res_hist[-1] ** 2 < eps * (1 + 1e-9) and r.res_hist[-2] ** 2 >= eps * (1 - 1e-9)
+        S = sp.csr_matrix((A.val, A.col, A.row_ptr), shape=(A.n, A.n))
+        d = S.diagonal()
+        M = spla.LinearOperator(S.shape, matvec=lambda v: v / d)
+        cnt = []
+        spla.cg(S, b, x0=x0.copy(), rtol=0.0, atol=np.sqrt(eps), M=M,
+                callback=lambda xk: cnt.append(1), maxiter=10 * A.n)
+        assert r.iters == len(cnt)
+
     def test_faulty_pcg_still_converges(self, O):
         # With faults in the protected SpMV at a high rate the solver still
         # converges because flagged blocks are recomputed.
