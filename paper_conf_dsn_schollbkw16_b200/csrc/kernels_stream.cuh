@@ -281,14 +281,26 @@ __device__ __forceinline__ void stream_group(const SpmvArgs &a, const StreamCfg 
   } else {
     // rows of 9..32 entries: aligned 8-leaf subtrees one at a time,
     // tree<4>((q0 + q1) + (q2 + q3)) with absent = -0.0 (R2)
+    // software-pipelined: subtree t + 1's gathers are issued before subtree
+    // t is multiplied, so a row of 9..32 entries waits for L2 about once
+    // instead of once per subtree (27-pt: four dependent round trips)
     double s01 = kAbsent, s23 = kAbsent;
-#pragma unroll 1
-    for (int t = 0; t < 4 && len > 8 * t; ++t) {
+    double xn[8];
+#pragma unroll
+    for (int j = 0; j < 8; ++j)
+      if (j < len) xn[j] = ld_x(a.x + ac[rs + j]);
+#pragma unroll
+    for (int t = 0; t < 4; ++t) {
+      if (!(len > 8 * t)) break;
       const int lt = len - 8 * t;
       double xj[8];
 #pragma unroll
-      for (int j = 0; j < 8; ++j)
-        if (j < lt) xj[j] = ld_x(a.x + ac[rs + 8 * t + j]);
+      for (int j = 0; j < 8; ++j) xj[j] = xn[j];
+      if (t < 3) {
+#pragma unroll
+        for (int j = 0; j < 8; ++j)
+          if (j < lt - 8) xn[j] = ld_x(a.x + ac[rs + 8 * (t + 1) + j]);
+      }
       double v[8];
 #pragma unroll
       for (int j = 0; j < 8; ++j)
