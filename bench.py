@@ -54,6 +54,18 @@ def load_peaks():
         return 6650.0, "fallback (B200_PROFILING.md: 6.65 TB/s)"
 
 
+def fused_kernel_name(info) -> str:
+    """Name of the fused multiply+detect launch(es) the plan runs (abft_info)."""
+    if info.get("stream"):
+        k = f"k_stream<CHECK> (G={info.get('stream_g')}, {info.get('stream_stages')} stages)"
+        return k + (" + k_general<CHECK>" if info.get("general_groups") else "")
+    if info.get("lean"):
+        return ("k_lean<CHECK" + (", SHORT" if info.get("lean_short") else "")
+                + (", RUNS" if info.get("lean_runs") else "") + ">")
+    return ("fused pass: k_hub + k_irr<CHECK> + k_general<CHECK>"
+            if info.get("irr_groups") else "k_general<CHECK>")
+
+
 def algorithmic_bytes(n, nnz, nb, c_bytes, check=True):
     """A (CSR: 8+4 B per nnz + row_ptr), x read once, y written once; with
     the check: C in the format the kernel streams (c_bytes: CSR 12 B per entry
@@ -771,8 +783,8 @@ def run_ours(args):
                 "lambda": args.lam, "parallelism": f"replicas{world}" if world > 1 else "single",
                 "l2": "no flush: working set "
                       f"{nbytes / 1e6:.0f} MB per step > 126 MB L2 (A, C streamed evict-first)",
-                "step": "abft_spmv(CHECK|AUTOCORRECT): k_lean fused multiply+detect+finalize, "
-                        f"1 correction launch (PDL, up to {args.max_rounds} rounds)",
+                "step": f"abft_spmv(CHECK|AUTOCORRECT): {fused_kernel_name(info)} fused multiply+detect, then k_finish "
+                        f"(finalize + correction, PDL, up to {args.max_rounds} rounds)",
                 "bytes_per_step": nbytes,
             },
             "ft_overhead_pct": round((ms / ms_plain - 1) * 100, 2),
@@ -780,11 +792,7 @@ def run_ours(args):
             "plain_ms": round(ms_plain, 5),
             "paper_literal_csr_c": csr_c,
             "cusparse_plain": cusparse,
-            "roofline": {"bound": "hbm", "kernel": (("k_lean<CHECK" + (", SHORT" if info.get("lean_short") else "")
-                                     + (", RUNS" if info.get("lean_runs") else "") + ">")
-                                    if info.get("lean") else
-                                    ("fused pass: k_hub + k_irr<CHECK> + k_general<CHECK>"
-                                     if info.get("irr_groups") else "k_general<CHECK>")),
+            "roofline": {"bound": "hbm", "kernel": fused_kernel_name(info),
                          "achieved": round(fused_gbs, 2), "peak": peak, "unit": "GB/s",
                          "frac": round(fused_gbs / peak, 4), "traffic": traffic,
                          "peak_source": peak_src, "launch_ms": round(ms_fused, 5),
