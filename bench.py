@@ -66,6 +66,14 @@ def fused_kernel_name(info) -> str:
             if info.get("irr_groups") else "k_general<CHECK>")
 
 
+def fused_launches(info, check=True) -> int:
+    """Kernels one abft_spmv call launches (launch_fused + k_finish)."""
+    k = (1 if info.get("col_perm") else 0) + (1 if info.get("hub_chunks") else 0)
+    k += 1 if (info.get("stream") or info.get("lean")) else 0
+    k += (1 if info.get("irr_groups") else 0) + (1 if info.get("general_groups") else 0)
+    return k + (1 if check else 0)
+
+
 def algorithmic_bytes(n, nnz, nb, c_bytes, check=True):
     """A (CSR: 8+4 B per nnz + row_ptr), x read once, y written once; with
     the check: C in the format the kernel streams (c_bytes: CSR 12 B per entry
@@ -780,6 +788,7 @@ def run_ours(args):
             "config": {
                 "workload": desc, "n": n, "nnz": nnz, "nnz_c": nnz_c, "block_size": args.block_size,
                 "c_format": info["c_format_name"], "general_groups": info["general_groups"],
+                "col_perm": bool(info.get("col_perm")),
                 "lambda": args.lam, "parallelism": f"replicas{world}" if world > 1 else "single",
                 "l2": "no flush: working set "
                       f"{nbytes / 1e6:.0f} MB per step > 126 MB L2 (A, C streamed evict-first)",
@@ -803,7 +812,7 @@ def run_ours(args):
                     "api": "abft_spmv_host_pipelined (copies of step k overlap steps k-1/k+1)",
                     "sync_call": {"api": "abft_spmv_host", "ms_per_step": round(dt_e2e_sync * 1e3, 4),
                                   "value": round(world * nbytes / dt_e2e_sync / 1e9, 3)}},
-            "gpu_launches": args.steps * (2 + (1 if info["general_groups"] else 0)),
+            "gpu_launches": args.steps * fused_launches(info, check=True),
             "clocks": clk,
         }
         print(json.dumps(line), flush=True)

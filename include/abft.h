@@ -174,12 +174,15 @@ typedef struct {
   int32_t stream;           /* warp-specialized kernel (position-map records) in use */
   int32_t stream_g;         /* its groups per chunk (consumer warps per CTA) */
   int32_t stream_stages;    /* its ring stages */
-  int32_t reserved0;
+  int32_t col_perm;         /* irregular path gathers x through a popularity-ordered copy
+                               (renumbered column arrays, one scatter of x per call;
+                               DESIGN.md §6.10) */
   int64_t pos_exc_rows;     /* exception rows over all position-map records */
   int64_t stream_plain_bytes;  /* bytes the warp-specialized kernel streams per call with the
                                   check off (A values and columns, structure records, x, y),
                                   0 if unused */
   int64_t stream_check_bytes;  /* bytes the check adds (checksum records) */
+  int64_t hub_chunks;       /* aligned 1024-entry chunks of hub rows (k_hub items) */
 } abft_info_t;
 abft_status abft_info(abft_handle_t h, abft_info_t *info);
 

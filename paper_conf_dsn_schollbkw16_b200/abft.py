@@ -73,9 +73,9 @@ class Info(C.Structure):
                 ("groups", C.c_int64), ("general_groups", C.c_int64), ("lean", C.c_int32),
                 ("max_rounds", C.c_int32), ("irr_groups", C.c_int64), ("lean_short", C.c_int32),
                 ("lean_runs", C.c_int32), ("stream", C.c_int32), ("stream_g", C.c_int32),
-                ("stream_stages", C.c_int32), ("reserved0", C.c_int32),
+                ("stream_stages", C.c_int32), ("col_perm", C.c_int32),
                 ("pos_exc_rows", C.c_int64), ("stream_plain_bytes", C.c_int64),
-                ("stream_check_bytes", C.c_int64)]
+                ("stream_check_bytes", C.c_int64), ("hub_chunks", C.c_int64)]
 
     def as_dict(self):
         d = {f: getattr(self, f) for f, _ in self._fields_}

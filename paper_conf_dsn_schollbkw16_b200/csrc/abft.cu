@@ -17,6 +17,7 @@
 #include "kernels_dense.cuh"
 #include "kernels_bigblock.cuh"
 #include "kernels_dist.cuh"
+#include "kernels_perm.cuh"
 
 #include <cub/device/device_radix_sort.cuh>
 
@@ -215,6 +216,11 @@ struct abft_ctx {
   cudaStream_t cs = nullptr;                    // NCCL stream
   cudaEvent_t ev_pack = nullptr, ev_comm = nullptr;
   int32_t *clist_int = nullptr, *clist_bnd = nullptr;  // k_stream chunks without / with halo columns
+  // popularity-ordered x (kernels_perm.cuh): renumbered
+  // column arrays, the old -> new map, the per-call copy of x
+  bool cperm = false;
+  int32_t *cinv = nullptr, *ci_p = nullptr, *ccol_p = nullptr;
+  double *xp = nullptr;
   int64_t n_int = 0, n_bnd = 0;
   std::vector<void *> owned;
   int device = 0;
@@ -538,6 +544,8 @@ void launch_stream(const abft_ctx *h, const SpmvArgs &a_in, cudaStream_t s,
 #undef STREAM
 }
 
+abft_status colperm_args(const abft_ctx *h, SpmvArgs &a, bool fresh, cudaStream_t s);
+
 template <bool CHECK, bool INJECT>
 void launch_irr(const abft_ctx *h, const SpmvArgs &a, cudaStream_t s) {
   const size_t smem = kIrrWarps * kIrrSmemPerWarp;
@@ -599,7 +607,9 @@ abft_status launch_fused_t(const abft_ctx *h, SpmvArgs a, cudaStream_t s) {
   return ABFT_OK;
 }
 
-abft_status launch_fused(const abft_ctx *h, const SpmvArgs &a, bool check, cudaStream_t s) {
+abft_status launch_fused(const abft_ctx *h, const SpmvArgs &a_in, bool check, cudaStream_t s) {
+  SpmvArgs a = a_in;
+  TRY(colperm_args(h, a, true, s));
   const bool inj = a.inj.mode != 0;
   if (check) return inj ? launch_fused_t<true, true>(h, a, s) : launch_fused_t<true, false>(h, a, s);
   return inj ? launch_fused_t<false, true>(h, a, s) : launch_fused_t<false, false>(h, a, s);
@@ -608,8 +618,10 @@ abft_status launch_fused(const abft_ctx *h, const SpmvArgs &a, bool check, cudaS
 // Steps 4-5 in one launch (k_finish), as a programmatic dependent launch so
 // its launch latency overlaps the fused kernels (it waits on griddepcontrol).
 // confirm: turn the fused pass's candidates into round 0's flags first.
-abft_status launch_finish(const abft_ctx *h, const SpmvArgs &a, int rounds, bool confirm,
-                          cudaStream_t s) {
+abft_status launch_finish(const abft_ctx *h, const SpmvArgs &a_in, int rounds, bool confirm,
+                          cudaStream_t s, bool fresh_x = false) {
+  SpmvArgs a = a_in;
+  TRY(colperm_args(h, a, fresh_x, s));
   cudaLaunchConfig_t cfg;
   memset(&cfg, 0, sizeof cfg);
   cfg.gridDim = dim3((unsigned)h->correct_grid);
@@ -958,7 +970,7 @@ abft_status plan_stream(abft_ctx *h, const std::vector<int32_t> &rp, const std::
     int NS = 0;
     while (NS < 8 && fixed + (size_t)(NS + 1) * c.stage_bytes <= budget) ++NS;
     if (const char *e = getenv("ABFT_STREAM_NS")) NS = std::min(NS, std::max(2, atoi(e)));
-    if (NS < 2) continue;
+    if (NS < 2 || (ABFT_STREAM_DEPTH == 3 && h->pos_S <= 8 && NS < 3)) continue;
     c.NS = NS;
     c.ring_off = 128;
     c.xs_off = 128 + (uint32_t)NS * c.stage_bytes;
@@ -1040,6 +1052,67 @@ uint32_t stage_layout(const abft_ctx *h, StageCfg &c) {
     c.off_xg = c.off_av;
   }
   return align16(o);
+}
+
+// Popularity-ordered x: columns renumbered by descending
+// reference count (stable: ties keep column order); renumbered copies of A's
+// and C's column arrays.  Synchronises the stream.
+abft_status build_colperm(abft_ctx *h, cudaStream_t s) {
+  const int64_t n = h->n;
+  int32_t *cnt = nullptr, *cnt2 = nullptr, *idx = nullptr, *perm = nullptr;
+  TRY(dalloc(h, &cnt, (size_t)n));
+  TRY(dalloc(h, &cnt2, (size_t)n));
+  TRY(dalloc(h, &idx, (size_t)n));
+  TRY(dalloc(h, &perm, (size_t)n));
+  TRY(dalloc(h, &h->cinv, (size_t)n + 1));
+  TRY(dalloc(h, &h->ci_p, (size_t)h->nnz + 8));
+  TRY(dalloc(h, &h->ccol_p, (size_t)h->nnz_c + 8));
+  TRY(dalloc(h, &h->xp, (size_t)n + 2));
+  CK(cudaMemsetAsync(cnt, 0, (size_t)n * 4, s));
+  CK(cudaMemsetAsync(h->ci_p + h->nnz, 0, 8 * 4, s));
+  CK(cudaMemsetAsync(h->ccol_p + h->nnz_c, 0, 8 * 4, s));
+  const unsigned g = (unsigned)h->num_sms * 8;
+  k_col_hist<<<g, 256, 0, s>>>(h->nnz, h->ci, cnt);
+  k_iota<<<g, 256, 0, s>>>(n, idx);
+  CK(cudaGetLastError());
+  int bits = 1;
+  while (bits < 31 && ((int64_t)1 << bits) <= h->nnz) ++bits;
+  size_t tmp_bytes = 0;
+  CK(cub::DeviceRadixSort::SortPairsDescending(nullptr, tmp_bytes, cnt, cnt2, idx, perm, (int)n, 0,
+                                                bits, s));
+  void *tmp = nullptr;
+  CK(cudaMalloc(&tmp, std::max<size_t>(tmp_bytes, 1)));
+  const cudaError_t e = cub::DeviceRadixSort::SortPairsDescending(tmp, tmp_bytes, cnt, cnt2, idx, perm,
+                                                                  (int)n, 0, bits, s);
+  if (e != cudaSuccess) {
+    cudaFree(tmp);
+    return cuda_fail(e, "colperm sort");
+  }
+  k_perm_inv<<<g, 256, 0, s>>>(n, perm, h->cinv);
+  k_remap_cols<<<g, 256, 0, s>>>(h->nnz, h->ci, h->cinv, h->ci_p);
+  k_remap_cols<<<g, 256, 0, s>>>(h->nnz_c, h->c_col, h->cinv, h->ccol_p);
+  CK(cudaGetLastError());
+  CK(cudaStreamSynchronize(s));
+  cudaFree(tmp);
+  h->cperm = true;
+  return ABFT_OK;
+}
+
+// The column arrays and operand the fused / correction kernels gather
+// through: the popularity-ordered copies when the handle has them (x_j reads
+// only; a.xr, the own rows' x_i, stays the caller's x).  fresh: scatter x
+// into the copy first (every call that brings a new operand).
+abft_status colperm_args(const abft_ctx *h, SpmvArgs &a, bool fresh, cudaStream_t s) {
+  if (!h->cperm || !a.x) return ABFT_OK;
+  if (fresh) {
+    const int64_t blocks = std::min<int64_t>((h->n / 2 + 255) / 256 + 1, (int64_t)h->num_sms * 8);
+    k_xperm<<<(unsigned)blocks, 256, 0, s>>>(h->n, a.x, h->cinv, h->xp);
+    CK(cudaGetLastError());
+  }
+  a.x = h->xp;
+  a.ci = h->ci_p;
+  a.ccol = h->ccol_p;
+  return ABFT_OK;
 }
 
 // Encode-time plan of the fused pass ("Long rows"):
@@ -1500,6 +1573,15 @@ abft_status abft_encode(const abft_csr_t *A, int32_t block_size, int32_t max_rou
       (e = cudaMemsetAsync(h->gbar, 0, 4 * sizeof(unsigned), s)) || (e = cudaStreamSynchronize(s)))
     return fail(cuda_fail(e, "scratch init"));
   if ((st = plan_fused(h, s)) != ABFT_OK) return fail(st);
+  {
+    // popularity-ordered x for large irregular matrices (k_irr groups, no
+    // staged or position-map path); ABFT_COLPERM=0 / 1 forces it off / on
+    const char *cp = getenv("ABFT_COLPERM");
+    const bool eligible = !h->pos && !h->lean && h->bs == 32 && h->x_offset == 0 && h->n_cols == h->n &&
+                          h->nnz > 0;
+    const bool want = cp ? atoi(cp) != 0 : (h->n_ilist > 0 && h->n >= ((int64_t)1 << 20));
+    if (eligible && want && (st = build_colperm(h, s)) != ABFT_OK) return fail(st);
+  }
   *out = h;
   return ABFT_OK;
 }
@@ -1543,7 +1625,7 @@ abft_status abft_finish(abft_handle_t h, const double *x, double *y, const doubl
   CK(cudaGetLastError());
   SpmvArgs a = make_args(h, x, y, h->bnorm + 1);
   TRY(prepare_inject(h, inj, true, s, &a.inj));
-  return launch_finish(h, a, rounds, true, s);
+  return launch_finish(h, a, rounds, true, s, true);
 }
 
 abft_status abft_correct(abft_handle_t h, const double *x, double *y, int32_t max_rounds,
@@ -1556,7 +1638,7 @@ abft_status abft_correct(abft_handle_t h, const double *x, double *y, int32_t ma
   // rate mode: the plan of the preceding abft_spmv (same call) is still on
   // the device; regenerating it is deterministic, so do that for clarity
   TRY(prepare_inject(h, inj, true, s, &a.inj));
-  return launch_finish(h, a, max_rounds, false, s);
+  return launch_finish(h, a, max_rounds, false, s, true);
 }
 
 abft_status abft_flags(abft_handle_t h, int32_t round, const int32_t **flagged,
@@ -1707,6 +1789,8 @@ abft_status abft_info(abft_handle_t h, abft_info_t *info) {
   info->stream = h->stream ? 1 : 0;
   info->stream_g = h->stc.G;
   info->stream_stages = h->stc.NS;
+  info->col_perm = h->cperm ? 1 : 0;
+  info->hub_chunks = h->n_hub;
   info->pos_exc_rows = h->pos_exc;
   info->stream_plain_bytes = 0;
   info->stream_check_bytes = 0;

@@ -425,6 +425,7 @@ struct ShortA {
   int ml;    // longest row of the group (uniform)
   bool uni;  // every row of the group has ml entries (uniform)
   bool hit;  // INJECT: the group may hold a round-0 fault (inj_group_hit)
+  bool stg;  // came from a loaded (non-terminal) stage the warp must release (depth 3)
   double xj[8];
   double xi;
 };
@@ -559,8 +560,15 @@ __device__ __forceinline__ void short_finish(const SpmvArgs &a, const StreamCfg 
   __syncwarp();  // scratch reads done before the next group's stores
 }
 
+#ifndef ABFT_STREAM_DEPTH
+#define ABFT_STREAM_DEPTH 2  // SHORT consumers: groups whose gathers are in flight (2 or 3)
+#endif
+#ifndef ABFT_STREAM_MINB
+#define ABFT_STREAM_MINB 2  // resident CTAs per SM the register budget targets
+#endif
+
 template <bool CHECK, bool INJECT, int CF, bool SHORT>
-__global__ void __launch_bounds__((kStreamMaxG + 1) * 32, 2) k_stream(const SpmvArgs a) {
+__global__ void __launch_bounds__((kStreamMaxG + 1) * 32, ABFT_STREAM_MINB) k_stream(const SpmvArgs a) {
   extern __shared__ __align__(128) unsigned char smem[];
   if (skip_call(a)) return;
   const StreamCfg c = a.stc;
@@ -672,7 +680,48 @@ __global__ void __launch_bounds__((kStreamMaxG + 1) * 32, 2) k_stream(const Spmv
   const uint32_t xs = smem_u32(smem + c.xs_off + (size_t)warp * c.xs_bytes);
   int s = 0;
   uint32_t fph = 0;  // parity of the next completion of full[s]
-  if constexpr (SHORT) {
+  if constexpr (SHORT && ABFT_STREAM_DEPTH == 3) {
+    // three phase-A states in rotation: the gathers of the groups two and
+    // one stages ahead are in flight while a group is finished (needs NS >= 3)
+    const double *xg = a.x;
+    ShortA sa, sb, sc;
+    int ls = 0, fs = 0;  // next stage to load / to release
+    uint32_t lph = 0;    // parity of the next completion of full[ls]
+    bool done = false;
+    auto load_next = [&](ShortA &nx) {
+      nx.g = -1;
+      nx.stg = false;
+      if (done) return;
+      const unsigned char *st1 = ring + (size_t)ls * c.stage_bytes;
+      mbar_wait_sleep(full + ls, lph);
+      const int32_t *hdr1 = reinterpret_cast<const int32_t *>(st1);
+      const int32_t g0n = hdr1[3 * G + 3];
+      if (g0n < 0) {
+        done = true;
+        return;
+      }
+      nx.stg = true;
+      if (warp < hdr1[3 * G + 4])
+        short_load<CHECK, INJECT>(a, c, xg, (int64_t)g0n + warp, warp, st1, lane, nx);
+      if (++ls == NS) {
+        ls = 0;
+        lph ^= 1u;
+      }
+    };
+    auto step = [&](ShortA &cu, ShortA &nx) -> bool {
+      if (!cu.stg) return false;
+      load_next(nx);
+      if (cu.g >= 0) short_finish<CHECK, INJECT, CF>(a, c, cu, xs, lane);
+      __syncwarp();
+      if (lane == 0) mbar_arrive(empty + fs);
+      if (++fs == NS) fs = 0;
+      return true;
+    };
+    load_next(sa);
+    load_next(sb);
+    while (step(sa, sc) && step(sb, sa) && step(sc, sb)) {
+    }
+  } else if constexpr (SHORT) {
     // ping-pong between two phase-A states (no register copies): each step
     // loads the next stage's group into one state and finishes the other
     const double *xg = a.x;

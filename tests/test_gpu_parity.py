@@ -606,3 +606,32 @@ def test_resident_plan(O, torch_cuda, lam):
     torch_cuda.cuda.synchronize()
     assert_bits_equal(y.cpu().numpy(), O.spmv(A, x), "y (cleared masks)")
     assert h.flags(0).size == 0
+
+
+@pytest.mark.parametrize("c_csr", [False, True])
+@pytest.mark.parametrize("name", ["rmat11", "rmat11_natural", "hubs", "rand_empty", "rand_dense"])
+def test_popularity_ordered_x(O, torch_cuda, name, c_csr, monkeypatch):
+    # the irregular path gathers x through a copy ordered by
+    # column popularity (renumbered column arrays, one scatter of x per call)
+    # -- only where x_j is read from changes, so y, t1, t2, beta, the flags of
+    # every round and the corrected y stay bit-exact against the oracle
+    from paper_conf_dsn_schollbkw16_b200 import encode
+    monkeypatch.setenv("ABFT_COLPERM", "1")
+    A = MATRICES[name]()
+    info = encode(A, c_csr=c_csr).info()
+    if info["lean"] or info["stream"]:
+        pytest.skip("staged / position-map path: no reordering")
+    assert info["col_perm"] == 1, info
+    c = Case(O, torch_cuda, A, c_csr=c_csr)
+    assert c.h.info()["col_perm"] == 1
+    assert c.run(G.uniform_vector(A.n, 31)).flagged.size == 0
+    rl = np.diff(A.row_ptr)
+    rows = np.nonzero(rl > 0)[0]
+    r0, r1 = int(rows[0]), int(rows[-1])
+    plan = G.FaultPlan([0, 0, 0, 1], [0, 0, 1, 0], [r0, r1, r1 // 32, r1],
+                       [1 << 62, 1 << 58, 1 << 61, 1 << 62])
+    ref = c.run(G.uniform_vector(A.n, 32), plan=plan)
+    assert {r0 // 32, r1 // 32} <= set(ref.flagged.tolist())
+    c.run(G.uniform_vector(A.n, 33), rate=dict(seed=5, lam=1e-3, targets=0b111, call=1))
+    monkeypatch.setenv("ABFT_COLPERM", "0")
+    assert encode(A, c_csr=c_csr).info()["col_perm"] == 0
