@@ -36,6 +36,8 @@ WORKLOADS = {
     "27pt256": ("3-D 27-point stencil 256^3 FP64 ABFT-SpMV (BASELINE configs[3], 1 GPU)",
                 lambda G: G.stencil_3d_27pt(256)),
     "27pt128": ("3-D 27-point stencil 128^3 FP64 ABFT-SpMV", lambda G: G.stencil_3d_27pt(128)),
+    "7pt192": ("3-D 7-point Laplacian 192^3 FP64 ABFT-SpMV (the configs[4] PCG matrix)",
+               lambda G: G.laplacian_3d_7pt(192)),
     "rmat20": ("R-MAT scale 20, edge factor 16, permuted, FP64 ABFT-SpMV",
                lambda G: G.rmat(20, 16, 1)),
     "rmat22": ("R-MAT scale 22, edge factor 16, permuted, FP64 ABFT-SpMV",

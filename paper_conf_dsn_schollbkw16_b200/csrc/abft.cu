@@ -1105,7 +1105,7 @@ abft_status build_colperm(abft_ctx *h, cudaStream_t s) {
 abft_status colperm_args(const abft_ctx *h, SpmvArgs &a, bool fresh, cudaStream_t s) {
   if (!h->cperm || !a.x) return ABFT_OK;
   if (fresh) {
-    const int64_t blocks = std::min<int64_t>((h->n / 2 + 255) / 256 + 1, (int64_t)h->num_sms * 8);
+    const int64_t blocks = std::min<int64_t>((h->n / 8 + 255) / 256 + 1, (int64_t)h->num_sms * 8);
     k_xperm<<<(unsigned)blocks, 256, 0, s>>>(h->n, a.x, h->cinv, h->xp);
     CK(cudaGetLastError());
   }
@@ -1149,13 +1149,19 @@ abft_status plan_fused(abft_ctx *h, cudaStream_t s) {
     }
     own.push_back({key, {first, (int32_t)hbeg.size() - first}});
   };
-  for (int64_t i = 0; i < h->n && h->bs <= 32; ++i)  // b_s > 32: k_bigblock reduces any length
-    if (rp[i + 1] - rp[i] > kHubLen) add_hub(rp[i], rp[i + 1] - rp[i], false, (int32_t)((i / 32) * 64 + (i % 32)));
-  for (int64_t k = 0; k < h->nb && h->bs <= 32; ++k)
-    if (crp[k + 1] - crp[k] > kHubLen) {
-      const int64_t r = k * h->bs;
-      add_hub(crp[k], crp[k + 1] - crp[k], true, (int32_t)((r / 32) * 64 + 32 + (r % 32) / h->bs));
-    }
+  // items group by group: a group's hub A rows, then its hub C rows, so the
+  // C chunks (whose columns include the hub rows' columns) gather x while
+  // the A chunks' gathers still sit in L2
+  for (int64_t g = 0; g < h->ngroups && h->bs <= 32; ++g) {  // b_s > 32: k_bigblock reduces any length
+    const int64_t i1 = std::min<int64_t>(h->n, g * 32 + 32);
+    for (int64_t i = g * 32; i < i1; ++i)
+      if (rp[i + 1] - rp[i] > kHubLen) add_hub(rp[i], rp[i + 1] - rp[i], false, (int32_t)((i / 32) * 64 + (i % 32)));
+    for (int64_t k = (g * 32) / h->bs; k < h->nb && k * h->bs < i1; ++k)
+      if (crp[k + 1] - crp[k] > kHubLen) {
+        const int64_t r = k * h->bs;
+        add_hub(crp[k], crp[k + 1] - crp[k], true, (int32_t)((r / 32) * 64 + 32 + (r % 32) / h->bs));
+      }
+  }
   std::sort(own.begin(), own.end());
   {
     std::vector<int32_t> ok(own.size()), of(own.size()), on(own.size());

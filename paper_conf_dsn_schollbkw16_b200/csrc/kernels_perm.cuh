@@ -44,23 +44,38 @@ __global__ void k_remap_cols(int64_t m, const int32_t *__restrict__ in, const in
     out[e] = __ldg(inv + __ldg(in + e));
 }
 
-// Per call: xp[inv[j]] = x[j].  x and inv are read coalesced (two entries
-// per thread, 16-B / 8-B loads when x is 16-B aligned); the writes scatter,
-// and L2 merges the partial sectors before they reach DRAM.
+// Per call: xp[inv[j]] = x[j].  x and inv are read coalesced (four 16-B /
+// 8-B pairs per thread in flight before the first store, when x is 16-B
+// aligned); the writes scatter, and L2 merges the partial sectors before they
+// reach DRAM.
 __global__ void __launch_bounds__(256) k_xperm(int64_t n, const double *__restrict__ x,
                                                const int32_t *__restrict__ inv,
                                                double *__restrict__ xp) {
+  constexpr int U = 4;
   const bool vec = (reinterpret_cast<uintptr_t>(x) & 15u) == 0;
   const int64_t n2 = vec ? n / 2 : 0;
-  for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < n2;
-       t += (int64_t)gridDim.x * blockDim.x) {
-    const double2 v = __ldcs(reinterpret_cast<const double2 *>(x) + t);
-    const int2 k = __ldcs(reinterpret_cast<const int2 *>(inv) + t);
-    xp[k.x] = v.x;
-    xp[k.y] = v.y;
+  const int64_t nt = (int64_t)gridDim.x * blockDim.x;
+  const double2 *x2 = reinterpret_cast<const double2 *>(x);
+  const int2 *i2 = reinterpret_cast<const int2 *>(inv);
+  for (int64_t t0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t0 < n2; t0 += U * nt) {
+    double2 v[U];
+    int2 k[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const int64_t t = t0 + u * nt;
+      if (t < n2) {
+        v[u] = __ldcs(x2 + t);
+        k[u] = __ldcs(i2 + t);
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u)
+      if (t0 + u * nt < n2) {
+        xp[k[u].x] = v[u].x;
+        xp[k[u].y] = v[u].y;
+      }
   }
-  for (int64_t j = 2 * n2 + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < n;
-       j += (int64_t)gridDim.x * blockDim.x)
+  for (int64_t j = 2 * n2 + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < n; j += nt)
     xp[__ldg(inv + j)] = __ldg(x + j);
 }
 

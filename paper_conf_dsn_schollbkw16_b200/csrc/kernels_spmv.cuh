@@ -45,7 +45,8 @@ template <> struct CType<CF_F32> { using T = float; };
 constexpr int kLeanWarps = 4;  // warps per CTA of k_lean (<= 4)
 // Timing experiments only (scripts/exp_libs.sh; results are NOT the method):
 // 1 = no C products, 2 = C neither staged nor multiplied, 3 = no butterflies,
-// 4 = no test, 5 = 1 + 3 + 4, 6 = k_stream without x gathers.  0 (the default)
+// 4 = no test, 5 = 1 + 3 + 4, 6 = k_stream without x gathers, 7 = k_stream SHORT
+// without the C pass (no position stores, no t1 products).  0 (the default)
 // = the method.
 #ifndef ABFT_EXP
 #define ABFT_EXP 0
@@ -377,7 +378,13 @@ __device__ __noinline__ double warp_row_pw(const Src &s, int64_t b, int n,
 }
 
 // Chunk sums of hub items (one warp per item; items are independent).
-__global__ void __launch_bounds__(kGenWarps * 32) k_hub(const SpmvArgs a) {
+#ifndef ABFT_HUB_MINB
+#define ABFT_HUB_MINB 1  // resident CTAs per SM the register budget targets
+#endif
+#ifndef ABFT_HUB_U
+#define ABFT_HUB_U 16  // entries in flight per lane
+#endif
+__global__ void __launch_bounds__(kGenWarps * 32, ABFT_HUB_MINB) k_hub(const SpmvArgs a) {
   __shared__ double scr_all[kGenWarps][kScr];
   if (a.skip && *(volatile const int32_t *)a.skip != 0) return;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -392,12 +399,12 @@ __global__ void __launch_bounds__(kGenWarps * 32) k_hub(const SpmvArgs a) {
       struct { const double *v; const int32_t *c;
         __device__ double val(int64_t e) const { return ld_stream(v + e); }
         __device__ int32_t col(int64_t e) const { return ld_stream(c + e); } } Cs{a.cval, a.ccol};
-      r = warp_row_pw<16>(Cs, b, n, a.x, scr_all[warp], lane);
+      r = warp_row_pw<ABFT_HUB_U>(Cs, b, n, a.x, scr_all[warp], lane);
     } else {
       struct { const double *v; const int32_t *c;
         __device__ double val(int64_t e) const { return ld_stream(v + e); }
         __device__ int32_t col(int64_t e) const { return ld_stream(c + e); } } As{a.va, a.ci};
-      r = warp_row_pw<16>(As, b, n, a.x, scr_all[warp], lane);
+      r = warp_row_pw<ABFT_HUB_U>(As, b, n, a.x, scr_all[warp], lane);
     }
     if (lane == 0) a.hub_part[q] = r;
   }

@@ -505,14 +505,15 @@ __device__ __forceinline__ void short_finish(const SpmvArgs &a, const StreamCfg 
   const int4 w0 = *reinterpret_cast<const int4 *>(Wp);
   const int4 w1 = *reinterpret_cast<const int4 *>(Wp + 4);
   const int32_t W[8] = {w0.x, w0.y, w0.z, w0.w, w1.x, w1.y, w1.z, w1.w};
+  double q0 = kAbsent;
   // x_j -> C position W[j] + lane (slots past the row land in the trash)
+  if (ABFT_EXP != 7) {  // 7: timing experiment only, no C pass (wrong t1)
 #pragma unroll
   for (int j = 0; j < 7; ++j) sts_f64(xs + 8u * xs_phys(W[j] + lane), A.xj[j]);
   if (A.ml > 7) sts_f64(xs + 8u * xs_phys(W[7] + lane), A.xj[7]);
   const int npad = (-nC) & 7;  // positions nC .. roundup8(nC)-1 hold -0.0 (R2)
   if (lane < npad) sts_f64(xs + 8u * xs_phys(nC + lane), kAbsent);
   __syncwarp();
-  double q0 = kAbsent;
   const int j0 = lane * 8;
   if (j0 < nC) {
     double cv[8], u8[8];
@@ -527,6 +528,7 @@ __device__ __forceinline__ void short_finish(const SpmvArgs &a, const StreamCfg 
       u8[2 * u + 1] = dmul(cv[2 * u + 1], x1);
     }
     q0 = tree<8>(u8);
+  }
   }
   double t2 = yv, gs = dmul(A.xi, A.xi);
   {
@@ -567,8 +569,14 @@ __device__ __forceinline__ void short_finish(const SpmvArgs &a, const StreamCfg 
 #define ABFT_STREAM_MINB 2  // resident CTAs per SM the register budget targets
 #endif
 
+#ifdef ABFT_STREAM_MAXNREG
+#define ABFT_STREAM_BOUNDS __maxnreg__(ABFT_STREAM_MAXNREG)
+#else
+#define ABFT_STREAM_BOUNDS __launch_bounds__((kStreamMaxG + 1) * 32, ABFT_STREAM_MINB)
+#endif
+
 template <bool CHECK, bool INJECT, int CF, bool SHORT>
-__global__ void __launch_bounds__((kStreamMaxG + 1) * 32, ABFT_STREAM_MINB) k_stream(const SpmvArgs a) {
+__global__ void ABFT_STREAM_BOUNDS k_stream(const SpmvArgs a) {
   extern __shared__ __align__(128) unsigned char smem[];
   if (skip_call(a)) return;
   const StreamCfg c = a.stc;
