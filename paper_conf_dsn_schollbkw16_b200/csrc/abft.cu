@@ -5,6 +5,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <utility>
 #include <vector>
 
 #include "../../include/abft.h"
@@ -164,6 +165,13 @@ struct abft_ctx {
   int32_t *inj_gstart = nullptr;  // [3][ngroups] first entry of (target, group)
   int32_t *op_ybkt = nullptr, *op_cbkt = nullptr;  // rate plans: op -> row / block buckets
   InjDev inj_last{};        // the device plan the last injecting call built (ABFT_INJ_RESIDENT)
+  // the rate plan now in the device list: its key and descriptor (a call of
+  // abft_finish / abft_correct for the same SpMV call reuses it)
+  bool rate_valid = false, rate_check = false;
+  uint64_t rate_seed = 0, rate_call = 0;
+  double rate_lambda = 0.0;
+  uint32_t rate_targets = 0;
+  InjDev rate_dev{};
   bool inj_last_valid = false;
   // rate-mode plan scratch
   int32_t *plan_counts = nullptr, *plan_offs = nullptr, *plan_tot = nullptr, *plan_len = nullptr;
@@ -347,6 +355,12 @@ abft_status build_inj_bits(abft_ctx *h, InjDev *d, cudaStream_t s) {
 abft_status gen_rate_plan(abft_ctx *h, const abft_inject_t *inj, uint64_t call, bool check,
                           cudaStream_t s, InjDev *d) {
   memset(d, 0, sizeof *d);
+  if (h->rate_valid && h->rate_seed == inj->seed && h->rate_call == call &&
+      h->rate_lambda == inj->lambda && h->rate_targets == inj->targets && h->rate_check == check) {
+    *d = h->rate_dev;  // the same call's plan is still in the device list
+    return ABFT_OK;
+  }
+  h->rate_valid = false;
   RatePlanArgs r;
   memset(&r, 0, sizeof r);
   r.n = h->n;
@@ -422,7 +436,15 @@ abft_status gen_rate_plan(abft_ctx *h, const abft_inject_t *inj, uint64_t call, 
   d->cap = (int32_t)std::min<int64_t>(cap, INT32_MAX);
   d->keys = h->inj_keys;
   d->masks = h->inj_masks;
-  return build_inj_bits(h, d, s);
+  TRY(build_inj_bits(h, d, s));
+  h->rate_valid = true;
+  h->rate_seed = inj->seed;
+  h->rate_call = call;
+  h->rate_lambda = inj->lambda;
+  h->rate_targets = inj->targets;
+  h->rate_check = check;
+  h->rate_dev = *d;
+  return ABFT_OK;
 }
 
 // Fill the device descriptor: upload a list-mode plan (sorted keys), or
@@ -457,6 +479,7 @@ abft_status prepare_inject_impl(abft_ctx *h, const abft_inject_t *inj, bool chec
   }
   if (inj->mode != ABFT_INJ_LIST) return ABFT_EINVAL;
   if (inj->n_list < 0 || inj->n_list > (1 << 30)) return ABFT_EINVAL;
+  h->rate_valid = false;  // the list (and its group tables) replace the rate plan
   d->mode = 1;
   d->n_list = (int32_t)inj->n_list;
   if (inj->n_list == 0) return ABFT_OK;
@@ -520,6 +543,30 @@ void launch_lean(const abft_ctx *h, const SpmvArgs &a, cudaStream_t s) {
 #undef LEAN
 }
 
+// Kernel launch with programmatic dependent launch (the kernel calls
+// pdl_wait before touching anything its predecessor writes); ABFT_NO_PDL=1
+// launches plainly (A/B timing).
+bool pdl_on() {
+  static const bool on = getenv("ABFT_NO_PDL") == nullptr;
+  return on;
+}
+template <typename... KArgs, typename... Args>
+cudaError_t launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t s,
+                       Args &&...args) {
+  cudaLaunchConfig_t cfg;
+  memset(&cfg, 0, sizeof cfg);
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = pdl_on() ? 1 : 0;
+  return cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...);
+}
+
 template <bool CHECK, bool INJECT>
 void launch_stream(const abft_ctx *h, const SpmvArgs &a_in, cudaStream_t s,
                    const int32_t *list = nullptr, int64_t n_list = -1) {
@@ -532,9 +579,9 @@ void launch_stream(const abft_ctx *h, const SpmvArgs &a_in, cudaStream_t s,
   const dim3 grid((unsigned)std::min<int64_t>(h->stream_grid, a.n_clist)),
       block((h->stc.G + 1) * 32);
   const size_t sm = h->stream_smem;
-#define STREAM(CF)                                                               \
-  (h->pos_S <= 8 ? k_stream<CHECK, INJECT, CF, true><<<grid, block, sm, s>>>(a) \
-                 : k_stream<CHECK, INJECT, CF, false><<<grid, block, sm, s>>>(a))
+#define STREAM(CF)                                                                     \
+  (h->pos_S <= 8 ? launch_pdl(k_stream<CHECK, INJECT, CF, true>, grid, block, sm, s, a) \
+                 : launch_pdl(k_stream<CHECK, INJECT, CF, false>, grid, block, sm, s, a))
   switch (h->pos_cf) {
     case CF_I8: STREAM(CF_I8); break;
     case CF_I16: STREAM(CF_I16); break;
@@ -545,6 +592,8 @@ void launch_stream(const abft_ctx *h, const SpmvArgs &a_in, cudaStream_t s,
 }
 
 abft_status colperm_args(const abft_ctx *h, SpmvArgs &a, bool fresh, cudaStream_t s);
+
+
 
 template <bool CHECK, bool INJECT>
 void launch_irr(const abft_ctx *h, const SpmvArgs &a, cudaStream_t s) {
@@ -1851,6 +1900,7 @@ abft_status abft_inject_clear_masks(abft_handle_t h, void *stream) {
     CK(cudaMemsetAsync(const_cast<uint64_t *>(h->inj_last.masks), 0, (size_t)n * 8,
                        (cudaStream_t)stream));
   h->list_cached = false;  // the device list no longer matches the uploaded plan
+  h->rate_valid = false;
   return ABFT_OK;
 }
 

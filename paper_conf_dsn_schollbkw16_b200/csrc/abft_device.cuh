@@ -401,4 +401,13 @@ __device__ __forceinline__ double apply_mask(double v, uint64_t m) {
   return __longlong_as_double((long long)((uint64_t)__double_as_longlong(v) ^ m));
 }
 
+// Programmatic dependent launch (PDL): pdl_trigger lets the next kernel of
+// the stream start launching (its CTAs are scheduled once every CTA of this
+// grid has triggered or exited); pdl_wait blocks until the preceding grid has
+// COMPLETED and its memory is visible -- every kernel calls it before it
+// reads or writes anything a preceding kernel touches.  Both are no-ops
+// without the launch attribute.
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+
 }  // namespace abft

@@ -1514,7 +1514,8 @@ __device__ __forceinline__ void block_rounds(const SpmvArgs &a, int64_t k, int r
 template <bool INJECT, bool CONFIRM>
 __global__ void __launch_bounds__(256) k_finish(const SpmvArgs a, int rounds) {
   __shared__ double s_red[256];
-  asm volatile("griddepcontrol.wait;" ::: "memory");
+  pdl_trigger();
+  pdl_wait();
   if (skip_call(a)) return;
   const int lane = threadIdx.x & 31;
   const bool hub_m = a.n_own > 0 && a.bs <= 32;

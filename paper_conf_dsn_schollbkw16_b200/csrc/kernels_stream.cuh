@@ -578,7 +578,7 @@ __device__ __forceinline__ void short_finish(const SpmvArgs &a, const StreamCfg 
 template <bool CHECK, bool INJECT, int CF, bool SHORT>
 __global__ void ABFT_STREAM_BOUNDS k_stream(const SpmvArgs a) {
   extern __shared__ __align__(128) unsigned char smem[];
-  if (skip_call(a)) return;
+  pdl_trigger();  // the next kernel's CTAs may take SMs this grid leaves
   const StreamCfg c = a.stc;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int G = c.G, NS = c.NS;
@@ -603,6 +603,10 @@ __global__ void ABFT_STREAM_BOUNDS k_stream(const SpmvArgs a) {
   }
   fence_proxy_async_smem();  // the zero fill precedes the bulk writes into the ring
   __syncthreads();
+  // the prologue above overlaps the preceding kernel (PDL); everything below
+  // may read its results (x, the PCG state) or write what it reads (y, lists)
+  pdl_wait();
+  if (skip_call(a)) return;
   if (warp == G) {
     // ---------------- producer ----------------
     const uint64_t pol = policy_evict_first();
