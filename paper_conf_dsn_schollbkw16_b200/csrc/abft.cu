@@ -1904,6 +1904,19 @@ abft_status abft_inject_clear_masks(abft_handle_t h, void *stream) {
   return ABFT_OK;
 }
 
+// Timing experiment 8 only (not declared in abft.h): per-phase cycle sums of
+// the SHORT k_stream consumers since the last call; zeros in other builds.
+extern "C" abft_status abft_debug_phases(unsigned long long *out) {
+  if (!out) return ABFT_EINVAL;
+  memset(out, 0, 8 * sizeof(unsigned long long));
+#if ABFT_EXP == 8
+  CK(cudaMemcpyFromSymbol(out, abft::g_phase, 8 * sizeof(unsigned long long)));
+  const unsigned long long z[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+  CK(cudaMemcpyToSymbol(abft::g_phase, z, sizeof z));
+#endif
+  return ABFT_OK;
+}
+
 abft_status abft_health(abft_handle_t h, void *stream, int32_t *err) {
   if (!h || !err) return ABFT_EINVAL;
   cudaStream_t s = (cudaStream_t)stream;

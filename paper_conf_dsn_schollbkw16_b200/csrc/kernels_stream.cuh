@@ -228,6 +228,67 @@ __device__ __forceinline__ void cvals8(const unsigned char *p, double (&c)[8]) {
   for (int u = 0; u < 8; ++u) c[u] = (double)v[u];
 }
 
+// Scratch layout of the C positions.  Integer checksum types (int8 / int16):
+// LINEAR (position p at 8p), so a lane stores x_j at xs + 8 (W[j] + lane) with
+// one address add; the C pass's 128-bit reads stay conflict-free because lane
+// l reads its pairs in the order u ^ sw (sw = bits 1-2 of l) and takes the
+// c_kj pairs permuted the same way (a few integer ops on the packed values).
+// The 8-leaf tree then sees the pairs in the order P_{u ^ sw}: the level-1
+// pair sums are the same numbers (pairs are not split), and the two level-2
+// sums pair {P0, P1} and {P2, P3} in either order -- IEEE addition is
+// commutative, so the bits are those of PW (R8).  Float / double checksums
+// keep the XOR-swizzled layout (xs_phys) and natural-order values.
+template <int CF> struct XsLinear { static constexpr bool v = (CF == CF_I8 || CF == CF_I16); };
+template <int CF>
+__device__ __forceinline__ uint32_t xs_addr(uint32_t xs, int p) {
+  if constexpr (XsLinear<CF>::v) return xs + 8u * (uint32_t)p;
+  else return xs + 8u * xs_phys(p);
+}
+// c_kj pairs in the read order of the C pass: pair u of c = pair u ^ sw of the
+// record (linear layout); natural order otherwise.
+template <int CF>
+__device__ __forceinline__ void cvals8_read(const unsigned char *p, int sw, double (&c)[8]) {
+  using T = typename CType<CF>::T;
+  if constexpr (CF == CF_I8) {
+    uint2 w = *reinterpret_cast<const uint2 *>(p);   // pair q: word q >> 1, half q & 1
+    if (sw & 2) { const uint32_t t = w.x; w.x = w.y; w.y = t; }
+    const uint32_t sel = (sw & 1) ? 0x1032u : 0x3210u;
+    w.x = __byte_perm(w.x, 0u, sel);
+    w.y = __byte_perm(w.y, 0u, sel);
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      c[u] = (double)(int8_t)((w.x >> (8 * u)) & 0xff);
+      c[u + 4] = (double)(int8_t)((w.y >> (8 * u)) & 0xff);
+    }
+  } else if constexpr (CF == CF_I16) {
+    const uint4 w4 = *reinterpret_cast<const uint4 *>(p);  // pair q: word q
+    uint32_t w[4] = {w4.x, w4.y, w4.z, w4.w};
+    if (sw & 1) {
+      uint32_t t = w[0]; w[0] = w[1]; w[1] = t;
+      t = w[2]; w[2] = w[3]; w[3] = t;
+    }
+    if (sw & 2) {
+      uint32_t t = w[0]; w[0] = w[2]; w[2] = t;
+      t = w[1]; w[1] = w[3]; w[3] = t;
+    }
+#pragma unroll
+    for (int u = 0; u < 8; ++u) c[u] = (double)(int16_t)((w[u >> 1] >> (16 * (u & 1))) & 0xffff);
+  } else {
+    cvals8<T>(p, c);
+  }
+}
+
+#if ABFT_EXP == 8
+// timing experiment 8: per-phase SM clock cycles of the SHORT consumers
+// (summed over all consumer warps, lane 0), read by abft_debug_phases
+__device__ unsigned long long g_phase[8];
+#define PH_MARK(v) v = clock64()
+#define PH_ADD(k, t0, t1) ph[k] += (unsigned long long)((t1) - (t0))
+#else
+#define PH_MARK(v)
+#define PH_ADD(k, t0, t1)
+#endif
+
 // Consumer: group g from stage `st` (header hdr, warp w, scratch xs).
 template <bool CHECK, bool INJECT, int CF, bool SHORT>
 __device__ __forceinline__ void stream_group(const SpmvArgs &a, const StreamCfg &c, int64_t g,
@@ -276,7 +337,7 @@ __device__ __forceinline__ void stream_group(const SpmvArgs &a, const StreamCfg 
       const int32_t W[8] = {w0.x, w0.y, w0.z, w0.w, w1.x, w1.y, w1.z, w1.w};
 #pragma unroll
       for (int j = 0; j < 8; ++j)
-        if (j < len) sts_f64(xs + 8u * xs_phys(W[j] + lane), xj[j]);
+        if (j < len) sts_f64(xs_addr<CF>(xs, W[j] + lane), xj[j]);
     }
   } else {
     // rows of 9..32 entries: aligned 8-leaf subtrees one at a time,
@@ -316,7 +377,7 @@ __device__ __forceinline__ void stream_group(const SpmvArgs &a, const StreamCfg 
         const int32_t W[8] = {w0.x, w0.y, w0.z, w0.w, w1.x, w1.y, w1.z, w1.w};
 #pragma unroll
         for (int j = 0; j < 8; ++j)
-          if (j < lt) sts_f64(xs + 8u * xs_phys(W[j] + lane), xj[j]);
+          if (j < lt) sts_f64(xs_addr<CF>(xs, W[j] + lane), xj[j]);
       }
     }
     yv = dadd(s01, s23);
@@ -339,7 +400,7 @@ __device__ __forceinline__ void stream_group(const SpmvArgs &a, const StreamCfg 
   // padding positions nC .. roundup8(nC) - 1 hold -0.0 (their c is 0: the
   // product is -0.0, the exact identity of the sum, R2)
   const int npad = (-nC) & 7;
-  if (lane < npad) sts_f64(xs + 8u * xs_phys(nC + lane), kAbsent);
+  if (lane < npad) sts_f64(xs_addr<CF>(xs, nC + lane), kAbsent);
   __syncwarp();
   // t1_k = PW over C's row of fl(c_kj x_j) (R8): lane l owns positions
   // 256 t + 8 l .. + 7 -- an 8-leaf tree, then the butterfly; chunks of 256
@@ -354,7 +415,7 @@ __device__ __forceinline__ void stream_group(const SpmvArgs &a, const StreamCfg 
     const int j0 = t * 256 + lane * 8;
     if (j0 < nC) {
       double cv[8], v[8];
-      cvals8<CT>(cvb + (size_t)j0 * sizeof(CT), cv);
+      cvals8_read<CF>(cvb + (size_t)j0 * sizeof(CT), sw, cv);
       const uint32_t blk = xs + 8u * (uint32_t)j0;
 #pragma unroll
       for (int u = 0; u < 4; ++u) {
@@ -466,7 +527,9 @@ __device__ __forceinline__ void short_load(const SpmvArgs &a, const StreamCfg &c
 // Phase B: products and y, the C positions, t1, t2, x^2, the test.
 template <bool CHECK, bool INJECT, int CF>
 __device__ __forceinline__ void short_finish(const SpmvArgs &a, const StreamCfg &c, const ShortA &A,
-                                             uint32_t xs, int lane) {
+                                             uint32_t xs, int lane, unsigned long long *ph) {
+  long long f0 = 0, f1 = 0, f2 = 0, f3 = 0;
+  PH_MARK(f0);
   using CT = typename CType<CF>::T;
   const int64_t g = A.g, i = g * 32 + lane;
   const double *av = reinterpret_cast<const double *>(A.st + c.off_av) + A.rs;
@@ -490,6 +553,8 @@ __device__ __forceinline__ void short_finish(const SpmvArgs &a, const StreamCfg 
     yv = apply_mask(yv, M.y);
   }
   a.y[i] = yv;
+  PH_MARK(f1);
+  PH_ADD(3, f0, f1);
   if (!CHECK) {
     if (a.pq) {
       const double t = bfly32(dmul(A.xi, yv));
@@ -509,17 +574,17 @@ __device__ __forceinline__ void short_finish(const SpmvArgs &a, const StreamCfg 
   // x_j -> C position W[j] + lane (slots past the row land in the trash)
   if (ABFT_EXP != 7) {  // 7: timing experiment only, no C pass (wrong t1)
 #pragma unroll
-  for (int j = 0; j < 7; ++j) sts_f64(xs + 8u * xs_phys(W[j] + lane), A.xj[j]);
-  if (A.ml > 7) sts_f64(xs + 8u * xs_phys(W[7] + lane), A.xj[7]);
+  for (int j = 0; j < 7; ++j) sts_f64(xs_addr<CF>(xs, W[j] + lane), A.xj[j]);
+  if (A.ml > 7) sts_f64(xs_addr<CF>(xs, W[7] + lane), A.xj[7]);
   const int npad = (-nC) & 7;  // positions nC .. roundup8(nC)-1 hold -0.0 (R2)
-  if (lane < npad) sts_f64(xs + 8u * xs_phys(nC + lane), kAbsent);
+  if (lane < npad) sts_f64(xs_addr<CF>(xs, nC + lane), kAbsent);
   __syncwarp();
   const int j0 = lane * 8;
   if (j0 < nC) {
     double cv[8], u8[8];
-    cvals8<CT>(A.crec + 16 + (size_t)j0 * sizeof(CT), cv);
-    const uint32_t blk = xs + 8u * (uint32_t)j0;
     const int sw = (lane >> 1) & 3;
+    cvals8_read<CF>(A.crec + 16 + (size_t)j0 * sizeof(CT), sw, cv);
+    const uint32_t blk = xs + 8u * (uint32_t)j0;
 #pragma unroll
     for (int u = 0; u < 4; ++u) {
       double x0, x1;
@@ -530,6 +595,8 @@ __device__ __forceinline__ void short_finish(const SpmvArgs &a, const StreamCfg 
     q0 = tree<8>(u8);
   }
   }
+  PH_MARK(f2);
+  PH_ADD(4, f1, f2);
   double t2 = yv, gs = dmul(A.xi, A.xi);
   {
     const bool b0 = lane & 1, b1 = lane & 2;
@@ -560,6 +627,8 @@ __device__ __forceinline__ void short_finish(const SpmvArgs &a, const StreamCfg 
     test_block_lo(a, g, dsub(t1, t2), gs, *reinterpret_cast<const double *>(A.crec));  // steps 3-4
   }
   __syncwarp();  // scratch reads done before the next group's stores
+  PH_MARK(f3);
+  PH_ADD(5, f2, f3);
 }
 
 #ifndef ABFT_STREAM_DEPTH
@@ -697,6 +766,8 @@ __global__ void ABFT_STREAM_BOUNDS k_stream(const SpmvArgs a) {
     // one stages ahead are in flight while a group is finished (needs NS >= 3)
     const double *xg = a.x;
     ShortA sa, sb, sc;
+    unsigned long long ph[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    (void)ph;
     int ls = 0, fs = 0;  // next stage to load / to release
     uint32_t lph = 0;    // parity of the next completion of full[ls]
     bool done = false;
@@ -723,7 +794,7 @@ __global__ void ABFT_STREAM_BOUNDS k_stream(const SpmvArgs a) {
     auto step = [&](ShortA &cu, ShortA &nx) -> bool {
       if (!cu.stg) return false;
       load_next(nx);
-      if (cu.g >= 0) short_finish<CHECK, INJECT, CF>(a, c, cu, xs, lane);
+      if (cu.g >= 0) short_finish<CHECK, INJECT, CF>(a, c, cu, xs, lane, ph);
       __syncwarp();
       if (lane == 0) mbar_arrive(empty + fs);
       if (++fs == NS) fs = 0;
@@ -738,6 +809,8 @@ __global__ void ABFT_STREAM_BOUNDS k_stream(const SpmvArgs a) {
     // loads the next stage's group into one state and finishes the other
     const double *xg = a.x;
     ShortA sa, sb;
+    unsigned long long ph[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    (void)ph;
     mbar_wait_sleep(full + s, fph);
     {
       const int32_t *hdr = reinterpret_cast<const int32_t *>(ring + (size_t)s * c.stage_bytes);
@@ -751,6 +824,8 @@ __global__ void ABFT_STREAM_BOUNDS k_stream(const SpmvArgs a) {
     // one step: wait for the next stage, phase A of its group into `nx`,
     // phase B of `cu`, release the current stage; false at the end
     auto step = [&](ShortA &cu, ShortA &nx) -> bool {
+      long long t0 = 0, t1 = 0, t2 = 0, t3 = 0;
+      PH_MARK(t0);
       int s1 = s + 1;
       uint32_t fph1 = fph;
       if (s1 == NS) {
@@ -759,20 +834,31 @@ __global__ void ABFT_STREAM_BOUNDS k_stream(const SpmvArgs a) {
       }
       const unsigned char *st1 = ring + (size_t)s1 * c.stage_bytes;
       mbar_wait_sleep(full + s1, fph1);
+      PH_MARK(t1);
+      PH_ADD(0, t0, t1);
       const int32_t *hdr1 = reinterpret_cast<const int32_t *>(st1);
       const int32_t g0n = hdr1[3 * G + 3];
       nx.g = -1;
       if (g0n >= 0 && warp < hdr1[3 * G + 4])
         short_load<CHECK, INJECT>(a, c, xg, (int64_t)g0n + warp, warp, st1, lane, nx);
-      if (cu.g >= 0) short_finish<CHECK, INJECT, CF>(a, c, cu, xs, lane);
+      PH_MARK(t2);
+      PH_ADD(1, t1, t2);
+      if (cu.g >= 0) short_finish<CHECK, INJECT, CF>(a, c, cu, xs, lane, ph);
       __syncwarp();
       if (lane == 0) mbar_arrive(empty + s);
+      PH_MARK(t3);
+      PH_ADD(2, t2, t3);
+      ph[6] += 1;
       s = s1;
       fph = fph1;
       return g0n >= 0;
     };
     while (step(sa, sb) && step(sb, sa)) {
     }
+#if ABFT_EXP == 8
+    if (lane == 0)
+      for (int k = 0; k < 7; ++k) atomicAdd(&g_phase[k], ph[k]);
+#endif
   } else {
     for (;;) {
       const unsigned char *st = ring + (size_t)s * c.stage_bytes;
