@@ -1034,6 +1034,11 @@ abft_status plan_stream(abft_ctx *h, const std::vector<int32_t> &rp, const std::
     }
   }
   if (best_score < 0) return ABFT_OK;  // no chunk fits: k_general takes every group
+  // deferred butterflies pay off when the x gathers are slow (x beyond ~1/3
+  // of L2: 7-pt 192^3 0.156 -> 0.152 ms) and cost on a resident x (7-pt
+  // 128^3 0.0442 -> 0.0451 ms); ABFT_STREAM_DEFER=0/1 forces it
+  best.defer = h->n_cols * 8 > ((int64_t)40 << 20) ? 1 : 0;
+  if (const char *e = getenv("ABFT_STREAM_DEFER")) best.defer = atoi(e) != 0;
   h->stc = best;
   h->stream_smem = best.xs_off + (size_t)best.G * best.xs_bytes;
   std::vector<uint8_t> in((size_t)ng, 0);

@@ -90,6 +90,7 @@ struct StreamCfg {
   uint32_t ring_off;     // dynamic smem: ring start (after the barriers)
   uint32_t xs_off;       // dynamic smem: per-consumer-warp C-position scratch
   uint32_t xs_bytes;     // per warp
+  int32_t defer;         // SHORT consumers: a group's butterfly runs one step later
 };
 
 struct SpmvArgs {

@@ -285,8 +285,8 @@ __device__ unsigned long long g_phase[8];
 #define PH_MARK(v) v = clock64()
 #define PH_ADD(k, t0, t1) ph[k] += (unsigned long long)((t1) - (t0))
 #else
-#define PH_MARK(v)
-#define PH_ADD(k, t0, t1)
+#define PH_MARK(v) ((void)(v))
+#define PH_ADD(k, t0, t1) ((void)(t0), (void)(t1))
 #endif
 
 // Consumer: group g from stage `st` (header hdr, warp w, scratch xs).
@@ -525,10 +525,19 @@ __device__ __forceinline__ void short_load(const SpmvArgs &a, const StreamCfg &c
 }
 
 // Phase B: products and y, the C positions, t1, t2, x^2, the test.
+// A finished group's values between its C pass and its butterfly.
+struct ShortP {
+  int64_t g;
+  double t2, q0, gs, pq, K;
+  uint64_t mt1, mt2;
+  bool hit, on;
+};
+
 template <bool CHECK, bool INJECT, int CF>
 __device__ __forceinline__ void short_finish(const SpmvArgs &a, const StreamCfg &c, const ShortA &A,
-                                             uint32_t xs, int lane, unsigned long long *ph) {
-  long long f0 = 0, f1 = 0, f2 = 0, f3 = 0;
+                                             uint32_t xs, int lane, ShortP &P,
+                                             unsigned long long *ph) {
+  long long f0 = 0, f1 = 0, f2 = 0;
   PH_MARK(f0);
   using CT = typename CType<CF>::T;
   const int64_t g = A.g, i = g * 32 + lane;
@@ -597,10 +606,36 @@ __device__ __forceinline__ void short_finish(const SpmvArgs &a, const StreamCfg 
   }
   PH_MARK(f2);
   PH_ADD(4, f1, f2);
-  double t2 = yv, gs = dmul(A.xi, A.xi);
+  // hand the four values to the (possibly deferred) reduce-scatter + test
+  P.g = g;
+  P.t2 = yv;
+  P.q0 = q0;
+  P.gs = dmul(A.xi, A.xi);
+  P.pq = a.pq ? dmul(A.xi, yv) : kAbsent;  // 4th value: x_i y_i (PCG p.q)
+  P.K = *reinterpret_cast<const double *>(A.crec);
+  P.mt1 = M.t1;
+  P.mt2 = M.t2;
+  P.hit = INJECT && A.hit;
+  P.on = true;
+  __syncwarp();  // scratch reads done before the next group's stores
+}
+
+// Steps 2-4 of a finished group (ShortP): t2 (R9), t1 (R8), the x^2 subtree
+// and the p.q partial as ONE reduce-scatter butterfly (levels 1-2 split the
+// four values over lane pairs, each keeping PW's pairing), then the exact
+// pre-filter (R12) on lane 0.  Deferred (StreamCfg::defer): a warp runs it
+// for group g after issuing the next group's gathers and before it needs
+// them, so the shuffle chain overlaps their latency.
+template <bool INJECT>
+__device__ __forceinline__ void short_bfly(const SpmvArgs &a, ShortP &P, int lane,
+                                           unsigned long long *ph) {
+  long long f2 = 0, f3 = 0;
+  PH_MARK(f2);
+  const int64_t g = P.g;
+  double t2 = P.t2, q0 = P.q0, gs = P.gs;
   {
     const bool b0 = lane & 1, b1 = lane & 2;
-    const double pq = a.pq ? dmul(A.xi, yv) : kAbsent;  // 4th value: x_i y_i (PCG p.q)
+    const double pq = P.pq;
     const double s0 = b0 ? t2 : q0, s1 = b0 ? gs : pq;
     const double k0 = b0 ? q0 : t2, k1 = b0 ? pq : gs;
     const double r0 = dadd(k0, __shfl_xor_sync(kFull, s0, 1));
@@ -614,9 +649,9 @@ __device__ __forceinline__ void short_finish(const SpmvArgs &a, const StreamCfg 
     if (a.pq && lane == 3) a.pq[g] = vv;
   }
   double t1 = q0;
-  if (INJECT && A.hit) {
-    t1 = apply_mask(t1, M.t1);
-    t2 = apply_mask(t2, M.t2);
+  if (INJECT && P.hit) {
+    t1 = apply_mask(t1, P.mt1);
+    t2 = apply_mask(t2, P.mt2);
   }
   if (lane == 0) {
     if (a.dbg_t1) {
@@ -624,9 +659,9 @@ __device__ __forceinline__ void short_finish(const SpmvArgs &a, const StreamCfg 
       a.dbg_t2[g] = t2;
     }
     a.gsum[g] = gs;
-    test_block_lo(a, g, dsub(t1, t2), gs, *reinterpret_cast<const double *>(A.crec));  // steps 3-4
+    test_block_lo(a, g, dsub(t1, t2), gs, P.K);  // steps 3-4
   }
-  __syncwarp();  // scratch reads done before the next group's stores
+  P.on = false;
   PH_MARK(f3);
   PH_ADD(5, f2, f3);
 }
@@ -766,6 +801,8 @@ __global__ void ABFT_STREAM_BOUNDS k_stream(const SpmvArgs a) {
     // one stages ahead are in flight while a group is finished (needs NS >= 3)
     const double *xg = a.x;
     ShortA sa, sb, sc;
+    ShortP P;
+    P.on = false;
     unsigned long long ph[8] = {0, 0, 0, 0, 0, 0, 0, 0};
     (void)ph;
     int ls = 0, fs = 0;  // next stage to load / to release
@@ -794,7 +831,8 @@ __global__ void ABFT_STREAM_BOUNDS k_stream(const SpmvArgs a) {
     auto step = [&](ShortA &cu, ShortA &nx) -> bool {
       if (!cu.stg) return false;
       load_next(nx);
-      if (cu.g >= 0) short_finish<CHECK, INJECT, CF>(a, c, cu, xs, lane, ph);
+      if (cu.g >= 0) short_finish<CHECK, INJECT, CF>(a, c, cu, xs, lane, P, ph);
+      if (CHECK && P.on) short_bfly<INJECT>(a, P, lane, ph);
       __syncwarp();
       if (lane == 0) mbar_arrive(empty + fs);
       if (++fs == NS) fs = 0;
@@ -809,6 +847,8 @@ __global__ void ABFT_STREAM_BOUNDS k_stream(const SpmvArgs a) {
     // loads the next stage's group into one state and finishes the other
     const double *xg = a.x;
     ShortA sa, sb;
+    ShortP P;
+    P.on = false;
     unsigned long long ph[8] = {0, 0, 0, 0, 0, 0, 0, 0};
     (void)ph;
     mbar_wait_sleep(full + s, fph);
@@ -843,7 +883,9 @@ __global__ void ABFT_STREAM_BOUNDS k_stream(const SpmvArgs a) {
         short_load<CHECK, INJECT>(a, c, xg, (int64_t)g0n + warp, warp, st1, lane, nx);
       PH_MARK(t2);
       PH_ADD(1, t1, t2);
-      if (cu.g >= 0) short_finish<CHECK, INJECT, CF>(a, c, cu, xs, lane, ph);
+      if (CHECK && c.defer && P.on) short_bfly<INJECT>(a, P, lane, ph);
+      if (cu.g >= 0) short_finish<CHECK, INJECT, CF>(a, c, cu, xs, lane, P, ph);
+      if (CHECK && !c.defer && P.on) short_bfly<INJECT>(a, P, lane, ph);
       __syncwarp();
       if (lane == 0) mbar_arrive(empty + s);
       PH_MARK(t3);
@@ -855,6 +897,7 @@ __global__ void ABFT_STREAM_BOUNDS k_stream(const SpmvArgs a) {
     };
     while (step(sa, sb) && step(sb, sa)) {
     }
+    if (CHECK && P.on) short_bfly<INJECT>(a, P, lane, ph);
 #if ABFT_EXP == 8
     if (lane == 0)
       for (int k = 0; k < 7; ++k) atomicAdd(&g_phase[k], ph[k]);

@@ -154,12 +154,30 @@ def test_stream_exception_rows_counted(O, torch_cuda):
     assert info["pos_exc_rows"] == exp, (info, exp)
 
 
-def test_stream_pcg_parity(O, torch_cuda):
+@pytest.mark.parametrize("defer", [0, 1])
+def test_stream_pcg_parity(O, torch_cuda, defer, monkeypatch):
     # the PCG case study over the streamed SpMV, with rate faults
+    # (immediate and deferred butterflies: the fused p.q rides in it)
     from test_gpu_parity import _pcg_case
+    monkeypatch.setenv("ABFT_STREAM_DEFER", str(defer))
     A = G.laplacian_3d_7pt(32)
     for inj in (None, dict(seed=3, lam=1e-5, targets=0b111)):
         ref, status, st, x, hist = _pcg_case(O, torch_cuda, A, inj)
         assert st["iters"] == ref.iters and status == ref.status
         assert_bits_equal(hist, ref.res_hist, "residual history")
         assert_bits_equal(x, ref.x, "x")
+
+
+@pytest.mark.parametrize("defer", [0, 1])
+@pytest.mark.parametrize("name", ["lap3d_32", "lap2d_64", "rand_empty", "rand_int16"])
+def test_stream_deferred_butterfly(O, torch_cuda, name, defer, monkeypatch):
+    # StreamCfg::defer: a group's reduce-scatter + test runs
+    # one consumer step later, after the next group's gathers are issued --
+    # the same values, so flags, corrections and the PCG p.q stay bit-exact
+    A, c = make_case(O, torch_cuda, name, monkeypatch, ABFT_STREAM_DEFER=defer)
+    assert c.run(G.uniform_vector(A.n, 52)).flagged.size == 0
+    nb = c.enc.nb
+    plan = G.FaultPlan([0, 0, 0, 0], [0, 0, 1, 2], [3, A.n - 1, nb // 3, nb - 1],
+                       [1 << 62, 1 << 57, 1 << 61, 1 << 60])
+    assert c.run(G.uniform_vector(A.n, 53), plan=plan).flagged.size >= 3
+    c.run(G.uniform_vector(A.n, 54), rate=dict(seed=3, lam=1e-3, targets=0b111, call=2))
