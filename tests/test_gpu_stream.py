@@ -169,7 +169,7 @@ def test_stream_pcg_parity(O, torch_cuda, defer, monkeypatch):
 
 
 @pytest.mark.parametrize("defer", [0, 1])
-@pytest.mark.parametrize("name", ["lap3d_32", "lap2d_64", "rand_empty", "rand_int16"])
+@pytest.mark.parametrize("name", ["lap3d_32", "lap2d_64", "st27_32", "st27_11", "rand_empty", "rand_int16"])
 def test_stream_deferred_butterfly(O, torch_cuda, name, defer, monkeypatch):
     # StreamCfg::defer: a group's reduce-scatter + test runs
     # one consumer step later, after the next group's gathers are issued --
