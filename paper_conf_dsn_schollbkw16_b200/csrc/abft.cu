@@ -198,6 +198,10 @@ struct abft_ctx {
   // abft_pcg's device-resident loop: the instantiated graph, the key of
   // what it bakes in (PcgGraphKey), its capture stream
   cudaGraphExec_t pcg_exec = nullptr;
+  // abft_dist_pcg: kPcgBatch fault-free iterations as one graph, replayed
+  // until the device state leaves RUN; key = what it bakes in
+  cudaGraphExec_t dpcg_exec = nullptr;
+  alignas(8) unsigned char dpcg_key[64] = {};
   alignas(8) unsigned char pcg_key[1024] = {};
   cudaStream_t pcg_cap = nullptr;
   double *pcg_sc = nullptr;
@@ -1481,6 +1485,7 @@ int64_t abft_rate_chunk(double lambda) { return FaultTables::chunk(lambda); }
 abft_status abft_destroy(abft_handle_t h) {
   if (!h) return ABFT_EINVAL;
   if (h->pcg_exec) cudaGraphExecDestroy(h->pcg_exec);
+  if (h->dpcg_exec) cudaGraphExecDestroy(h->dpcg_exec);
   if (h->pcg_cap) {
     cudaStreamSynchronize(h->pcg_cap);
     cudaStreamDestroy(h->pcg_cap);
