@@ -584,8 +584,10 @@ void launch_stream(const abft_ctx *h, const SpmvArgs &a_in, cudaStream_t s,
       block((h->stc.G + 1) * 32);
   const size_t sm = h->stream_smem;
 #define STREAM(CF)                                                                     \
-  (h->pos_S <= 8 ? launch_pdl(k_stream<CHECK, INJECT, CF, true>, grid, block, sm, s, a) \
-                 : launch_pdl(k_stream<CHECK, INJECT, CF, false>, grid, block, sm, s, a))
+  (h->pos_S <= 8                                                                        \
+       ? (h->stc.defer ? launch_pdl(k_stream<CHECK, INJECT, CF, true, true>, grid, block, sm, s, a) \
+                       : launch_pdl(k_stream<CHECK, INJECT, CF, true, false>, grid, block, sm, s, a)) \
+       : launch_pdl(k_stream<CHECK, INJECT, CF, false>, grid, block, sm, s, a))
   switch (h->pos_cf) {
     case CF_I8: STREAM(CF_I8); break;
     case CF_I16: STREAM(CF_I16); break;
@@ -773,6 +775,10 @@ abft_status set_lean_attrs(int optin) {
   TRY(set_smem_attrs(k_lean<false, true, CF, 2, false, true>, optin));
   TRY(set_smem_attrs(k_lean<false, false, CF, 2, false, true>, optin));
   if constexpr (CF != CF_CSR) {
+    TRY(set_smem_attrs(k_stream<true, true, CF, true, true>, optin));
+    TRY(set_smem_attrs(k_stream<true, false, CF, true, true>, optin));
+    TRY(set_smem_attrs(k_stream<false, true, CF, true, true>, optin));
+    TRY(set_smem_attrs(k_stream<false, false, CF, true, true>, optin));
     TRY(set_smem_attrs(k_stream<true, true, CF, true>, optin));
     TRY(set_smem_attrs(k_stream<true, false, CF, true>, optin));
     TRY(set_smem_attrs(k_stream<false, true, CF, true>, optin));

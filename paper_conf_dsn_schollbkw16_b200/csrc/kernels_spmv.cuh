@@ -418,6 +418,18 @@ __device__ __noinline__ double hub_sum(const SpmvArgs &a, int32_t first, int32_t
   return acc.finish();
 }
 
+// The same PW with the whole warp: lanes load 32 consecutive chunk sums at a
+// time and the ascending xor butterfly reduces them (an aligned 32-chunk
+// subtree; absent slots past cnt), the subtrees join by the binary counter --
+// PW over the chunks again (R2: padding independence).  Warp-uniform.
+__device__ __forceinline__ double hub_sum_warp(const SpmvArgs &a, int32_t first, int32_t cnt,
+                                               int lane) {
+  PwSeq acc;
+  for (int32_t b = 0; b < cnt; b += 32)
+    acc.push(bfly32(lane < cnt - b ? __ldcg(a.hub_part + first + b + lane) : kAbsent));
+  return acc.finish();
+}
+
 // Range [lo, hi) of the group's entries in the sorted owner table.
 __device__ __forceinline__ void own_range(const SpmvArgs &a, int64_t g, int &lo, int &hi) {
   lo = hi = 0;
@@ -502,11 +514,14 @@ __device__ __forceinline__ void group_general(const SpmvArgs &a, int64_t g, int 
   if (a.lean_ok[g] & 2) own_range(a, g, olo, ohi);  // bit 1: the group owns hub rows
   bool hub = false;
   double yv = 0.0;
-  for (int e = olo; e < ohi; ++e) {
+  for (int e = olo; e < ohi; ++e) {  // warp-uniform
     const int32_t key = __ldg(a.own_key + e);
-    if ((key & 63) == lane) {  // A row 32g + lane (key & 32 == 0)
-      hub = true;
-      yv = hub_sum(a, __ldg(a.own_first + e), __ldg(a.own_n + e));
+    if (!(key & 32)) {  // A row 32g + (key & 31)
+      const double t = hub_sum_warp(a, __ldg(a.own_first + e), __ldg(a.own_n + e), lane);
+      if ((key & 31) == lane) {
+        hub = true;
+        yv = t;
+      }
     }
   }
   // row-length-adaptive y: rows <= 32 entries lane-private (an aligned tree of
@@ -551,11 +566,14 @@ __device__ __forceinline__ void group_general(const SpmvArgs &a, int64_t g, int 
   const int nkl = ce - cb;
   bool chub = false;
   double t1l = 0.0;
-  for (int e = olo; e < ohi; ++e) {
+  for (int e = olo; e < ohi; ++e) {  // warp-uniform
     const int32_t key = __ldg(a.own_key + e);
-    if ((key & 32) && (key & 31) == lane) {
-      chub = true;
-      t1l = hub_sum(a, __ldg(a.own_first + e), __ldg(a.own_n + e));
+    if (key & 32) {  // C row of block (key & 31) of the group
+      const double t = hub_sum_warp(a, __ldg(a.own_first + e), __ldg(a.own_n + e), lane);
+      if ((key & 31) == lane) {
+        chub = true;
+        t1l = t;
+      }
     }
   }
   const bool csmall = nblk > 1 && !chub && nkl <= 32;

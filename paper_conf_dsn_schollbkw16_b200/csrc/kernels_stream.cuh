@@ -679,7 +679,10 @@ __device__ __forceinline__ void short_bfly(const SpmvArgs &a, ShortP &P, int lan
 #define ABFT_STREAM_BOUNDS __launch_bounds__((kStreamMaxG + 1) * 32, ABFT_STREAM_MINB)
 #endif
 
-template <bool CHECK, bool INJECT, int CF, bool SHORT>
+// DEFER (SHORT only): a group's reduce-scatter + test one step later
+// (StreamCfg::defer picks the instantiation; a runtime branch cost 7-pt 128^3
+// 5% in registers and scheduling)
+template <bool CHECK, bool INJECT, int CF, bool SHORT, bool DEFER = false>
 __global__ void ABFT_STREAM_BOUNDS k_stream(const SpmvArgs a) {
   extern __shared__ __align__(128) unsigned char smem[];
   pdl_trigger();  // the next kernel's CTAs may take SMs this grid leaves
@@ -883,9 +886,9 @@ __global__ void ABFT_STREAM_BOUNDS k_stream(const SpmvArgs a) {
         short_load<CHECK, INJECT>(a, c, xg, (int64_t)g0n + warp, warp, st1, lane, nx);
       PH_MARK(t2);
       PH_ADD(1, t1, t2);
-      if (CHECK && c.defer && P.on) short_bfly<INJECT>(a, P, lane, ph);
+      if (CHECK && DEFER && P.on) short_bfly<INJECT>(a, P, lane, ph);
       if (cu.g >= 0) short_finish<CHECK, INJECT, CF>(a, c, cu, xs, lane, P, ph);
-      if (CHECK && !c.defer && P.on) short_bfly<INJECT>(a, P, lane, ph);
+      if (CHECK && !DEFER && P.on) short_bfly<INJECT>(a, P, lane, ph);
       __syncwarp();
       if (lane == 0) mbar_arrive(empty + s);
       PH_MARK(t3);
