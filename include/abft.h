@@ -209,7 +209,10 @@ abft_status abft_finish(abft_handle_t h, const double *x, double *y, const doubl
 
 /* Step 5 alone: rounds r = 1..max_rounds recompute the rows of
  * the blocks flagged in round r-1, recompute t1/t2 and re-check; blocks that
- * still fail form round r's list.  Uses beta of the last abft_spmv. */
+ * still fail form round r's list.  Uses beta of the last abft_spmv.  `inj`
+ * must describe the same call as that abft_spmv (rate mode: the same seed,
+ * lambda, targets and call index); the rate plan it built is reused from the
+ * device list when those match (abft_finish likewise), else rebuilt. */
 abft_status abft_correct(abft_handle_t h, const double *x, double *y, int32_t max_rounds,
                          const abft_inject_t *inj, void *stream);
 
