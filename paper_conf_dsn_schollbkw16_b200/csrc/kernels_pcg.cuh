@@ -144,32 +144,61 @@ __device__ __forceinline__ void cta_pw2(double (&v)[8], double (&w)[8], int64_t 
 }
 
 // Last-CTA completion of PW over partials[0..ncta) (aligned chunk nodes):
-// thread t reduces an aligned run of m <= 32 partials in registers (PwSeq
-// beyond), then a shared-memory tree over the threads.
-__device__ __forceinline__ double grid_pw(const double *partials, int ncta, double *s_red) {
+// thread t reduces an aligned run of m partials in registers (m <= 16; a
+// PwSeq beyond), the ascending xor butterfly joins the 32 runs of a warp and
+// an 8-leaf tree the 8 warps -- the PW tree over 256 m slots with absent
+// padding (R2).  Two arrays at once (their latency chains overlap); p1 may
+// be null.  All threads get the results.
+__device__ __forceinline__ void grid_pw2(const double *p0, const double *p1, int ncta, double *s_red,
+                                         double &o0, double &o1) {
   int m = 1;
   while (m * kPcgThreads < ncta) m <<= 1;
   const int b = threadIdx.x * m;
-  double t;
-  if (m <= 32) {
-    double v[32];
+  double t0, t1 = kAbsent;
+  if (m <= 16) {
+    double v0[16], v1[16];
 #pragma unroll
-    for (int q = 0; q < 32; ++q) v[q] = (q < m && b + q < ncta) ? __ldcg(partials + b + q) : kAbsent;
-    t = tree<32>(v);
+    for (int q = 0; q < 16; ++q) {
+      const bool in = q < m && b + q < ncta;
+      v0[q] = in ? __ldcg(p0 + b + q) : kAbsent;
+      v1[q] = (in && p1) ? __ldcg(p1 + b + q) : kAbsent;
+    }
+    t0 = tree<16>(v0);
+    t1 = tree<16>(v1);
   } else {
-    PwSeq acc;
-    for (int q = b; q < min(b + m, ncta); ++q) acc.push(__ldcg(partials + q));
-    t = acc.finish();
+    PwSeq a0, a1;
+    for (int q = b; q < min(b + m, ncta); ++q) {
+      a0.push(__ldcg(p0 + q));
+      if (p1) a1.push(__ldcg(p1 + q));
+    }
+    t0 = a0.finish();
+    if (p1) t1 = a1.finish();
+  }
+#pragma unroll
+  for (int sft = 1; sft < 32; sft <<= 1) {
+    t0 = dadd(t0, __shfl_xor_sync(kFull, t0, sft));
+    t1 = dadd(t1, __shfl_xor_sync(kFull, t1, sft));
+  }
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  __syncthreads();
+  if (lane == 0) {
+    s_red[warp] = t0;
+    s_red[8 + warp] = t1;
   }
   __syncthreads();
-  s_red[threadIdx.x] = t;
-  __syncthreads();
-  for (int s = 1; s < kPcgThreads; s <<= 1) {
-    if ((threadIdx.x & (2 * s - 1)) == 0)
-      s_red[threadIdx.x] = dadd(s_red[threadIdx.x], s_red[threadIdx.x + s]);
-    __syncthreads();
+  double w0[8], w1[8];
+#pragma unroll
+  for (int k = 0; k < 8; ++k) {
+    w0[k] = s_red[k];
+    w1[k] = s_red[8 + k];
   }
-  return s_red[0];
+  o0 = tree<8>(w0);
+  o1 = tree<8>(w1);
+}
+__device__ __forceinline__ double grid_pw(const double *partials, int ncta, double *s_red) {
+  double o0, o1;
+  grid_pw2(partials, nullptr, ncta, s_red, o0, o1);
+  return o0;
 }
 
 // Ticket: true in the last CTA to finish (after its partials are written).
@@ -308,9 +337,9 @@ __global__ void __launch_bounds__(kPcgThreads) k_pcg_init(const PcgArgs a) {
     a.part2[blockIdx.x] = BBc;
   }
   if (!last_cta(a.ticket, &s_flag)) return;
-  const double RZ = grid_pw(a.part0, gridDim.x, s_red);
-  const double RR = grid_pw(a.part1, gridDim.x, s_red);
-  const double BB = grid_pw(a.part2, gridDim.x, s_red);
+  double RZ, RR, BB, unused;
+  grid_pw2(a.part0, a.part1, gridDim.x, s_red, RZ, RR);
+  grid_pw2(a.part2, nullptr, gridDim.x, s_red, BB, unused);
   if (threadIdx.x == 0) {
     if (a.dsend) {
       a.dsend[0] = RZ;
@@ -390,7 +419,11 @@ __global__ void __launch_bounds__(kPcgThreads) k_pcg_update(const PcgArgs a, int
 #pragma unroll
   for (int u = 0; u < 8; ++u) {
     rv[u] = dsub(rv[u], dmul(alpha, qv[u]));
+#if ABFT_EXP == 9  // timing experiment only: no division (wrong z)
+    dv[u] = dmul(rv[u], dv[u]);
+#else
     dv[u] = __ddiv_rn(rv[u], dv[u]);  // z
+#endif
     rz[u] = dmul(rv[u], dv[u]);
     rr[u] = dmul(rv[u], rv[u]);
   }
@@ -403,8 +436,8 @@ __global__ void __launch_bounds__(kPcgThreads) k_pcg_update(const PcgArgs a, int
     a.part1[blockIdx.x] = RRc;
   }
   if (!last_cta(a.ticket, &s_flag)) return;
-  const double RZ = grid_pw(a.part0, gridDim.x, s_red);
-  const double RR = grid_pw(a.part1, gridDim.x, s_red);
+  double RZ, RR;
+  grid_pw2(a.part0, a.part1, gridDim.x, s_red, RZ, RR);
   if (threadIdx.x == 0) {
     if (a.dsend) {
       a.dsend[0] = RZ;
@@ -546,8 +579,8 @@ __global__ void __launch_bounds__(kPcgThreads, 2) k_cg1_update(const PcgArgs a) 
     a.part1[blockIdx.x] = RRc;
   }
   if (!last_cta(a.ticket, &s_flag)) return;
-  const double RU = grid_pw(a.part0, gridDim.x, s_red);
-  const double RR = grid_pw(a.part1, gridDim.x, s_red);
+  double RU, RR;
+  grid_pw2(a.part0, a.part1, gridDim.x, s_red, RU, RR);
   if (threadIdx.x == 0) {
     a.dsend[0] = RU;
     a.dsend[1] = RR;
