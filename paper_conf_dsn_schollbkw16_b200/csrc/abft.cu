@@ -270,6 +270,7 @@ SpmvArgs make_args(const abft_ctx *h, const double *x, double *y, const double *
   memset(&a, 0, sizeof a);
   a.n = h->n;
   a.nnz = h->nnz;
+  a.nnz_c = h->nnz_c;
   a.bs = h->bs;
   a.log2bs = h->log2bs;
   a.nb = h->nb;

@@ -96,6 +96,7 @@ struct StreamCfg {
 struct SpmvArgs {
   int64_t n;
   int64_t nnz;
+  int64_t nnz_c;     // entries of C (CSR arrays; k_hub's prefetch bound)
   int32_t bs;        // block size, power of two <= 1024 (> 32: kernels_bigblock.cuh)
   int32_t log2bs;
   int64_t nb;
@@ -391,7 +392,24 @@ __global__ void __launch_bounds__(kGenWarps * 32, ABFT_HUB_MINB) k_hub(const Spm
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  const bool pf = ((reinterpret_cast<uintptr_t>(a.va) | reinterpret_cast<uintptr_t>(a.ci) |
+                    reinterpret_cast<uintptr_t>(a.cval) | reinterpret_cast<uintptr_t>(a.ccol)) & 15u) == 0;
   for (int64_t q = gw; q < a.n_hub; q += nw) {
+    // the warp's next item: its values and columns on their way into L2
+    // while this one is reduced (the stream loads then wait for L2, not DRAM)
+    if (pf && lane == 0 && q + nw < a.n_hub) {
+      const uint32_t Ln = __ldg(a.hub_len + q + nw);
+      const int64_t bn = __ldg(a.hub_beg + q + nw);
+      const bool cn = Ln >> 31;
+      const int64_t lim = (cn ? a.nnz_c : a.nnz) & ~3ll;
+      const int64_t s4 = bn & ~3ll, e4 = min64((bn + (int64_t)(Ln & 0x7fffffffu) + 3) & ~3ll, lim);
+      if (e4 > s4) {
+        asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"((cn ? a.cval : a.va) + s4),
+                     "r"((uint32_t)(e4 - s4) * 8u) : "memory");
+        asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"((cn ? a.ccol : a.ci) + s4),
+                     "r"((uint32_t)(e4 - s4) * 4u) : "memory");
+      }
+    }
     const uint32_t L = __ldg(a.hub_len + q);
     const int64_t b = __ldg(a.hub_beg + q);
     const int n = (int)(L & 0x7fffffffu);
