@@ -1,0 +1,10 @@
+#!/bin/bash
+cd $GRAFT_REPO_ROOT; mkdir -p gpurun_out
+P=paper_conf_dsn_schollbkw16_b200
+timeout 900 python -m pytest tests/test_gpu_parity.py -q -x -k "popularity or irregular or hub or rmat or bench_workloads" > gpurun_out/hp_tests.log 2>&1; echo "rc=$?" >> gpurun_out/hp_tests.log
+rm -f gpurun_out/hp.log
+for rep in 1 2; do for lib in libabft_nopf.so libabft.so; do for w in rmat24 rmat22; do
+  echo -n "$lib $w: " >> gpurun_out/hp.log
+  ABFT_LIB=$PWD/$P/$lib timeout 300 python bench.py --no-cpu-baseline --steps 30 --workload $w 2>&1 | python -c "import sys,json; L=[l for l in sys.stdin if l.startswith('{')]; d=json.loads(L[-1]) if L else None; print(d and (d['value'], d['ms_per_step'], d['plain_ms'], d['roofline']['launch_ms'], d['ft_overhead_pct']))" >> gpurun_out/hp.log 2>&1
+done; done; done
+tail -2 gpurun_out/hp_tests.log; cat gpurun_out/hp.log
