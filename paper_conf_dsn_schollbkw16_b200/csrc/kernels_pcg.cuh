@@ -405,7 +405,10 @@ __global__ void __launch_bounds__(kPcgThreads) k_pcg_dotg(const PcgArgs a, const
 // r -= alpha q; z = r / d; rho' = PW(r.z); res = ||r||; beta = rho'/rho;
 // convergence test (R15, R16).  x += alpha p moved to k_pcg_p, which reads
 // p anyway (one vector stream less per iteration; the same bits).
-__global__ void __launch_bounds__(kPcgThreads) k_pcg_update(const PcgArgs a, int64_t iter) {
+#ifndef ABFT_PCG_UPD_MINB
+#define ABFT_PCG_UPD_MINB 4  // 64 registers, 4 CTAs per SM: 192^3 PCG 48.5 -> 46.9 ms (same box)
+#endif
+__global__ void __launch_bounds__(kPcgThreads, ABFT_PCG_UPD_MINB) k_pcg_update(const PcgArgs a, int64_t iter) {
   __shared__ double s_w[16];
   __shared__ double s_red[kPcgThreads];
   __shared__ int s_flag;
