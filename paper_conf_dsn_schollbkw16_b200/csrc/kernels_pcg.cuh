@@ -455,7 +455,10 @@ __global__ void __launch_bounds__(kPcgThreads, ABFT_PCG_UPD_MINB) k_pcg_update(c
 // x += alpha p; p = z + beta p (old p for both).  Runs in the iteration
 // that converged too (as the oracle); skipped only when this iteration's
 // update was skipped.
-__global__ void __launch_bounds__(kPcgThreads) k_pcg_p(const PcgArgs a, int64_t iter) {
+#ifndef ABFT_PCG_P_MINB
+#define ABFT_PCG_P_MINB 1
+#endif
+__global__ void __launch_bounds__(kPcgThreads, ABFT_PCG_P_MINB) k_pcg_p(const PcgArgs a, int64_t iter) {
   // iter < 0: the device-resident loop's counter (CUDA graph while node)
   if (iter < 0) iter = *(volatile const int64_t *)&a.sc->j;
   if (*(volatile const int64_t *)&a.sc->upd != iter) return;  // this iteration did not execute
