@@ -4,27 +4,30 @@
 //
 // Work unit: a GROUP of 32 consecutive rows (= 32/b_s row blocks).
 //
-// k_lean (b_s = 32, the paper's block size): a persistent grid; each warp owns
-// a contiguous range of groups and runs a software pipeline over them: one
-// lane issues TMA 1-D bulk copies (cp.async.bulk + mbarrier transaction
-// counts, L2 evict-first) of the next group's row pointers, x slice, A
-// segment (values + columns) and C segment into a shared-memory stage while
-// the warp computes the current group from the other stage.  Per group:
-//  * phase 1: every staged a_ij and c_kj becomes a product with the gathered
-//    x_j, in place (lane-strided, up to 16 x gathers in flight per lane: one
-//    L2 round trip per group);
-//  * y_i: lane l reduces row 32g+l from shared memory with an in-register PW
-//    tree of P = 2^ceil(log2 maxlen) leaves (rows > 32: the warp reduces it);
-//  * t2 = PW over the 32 slots of y (xor butterfly);
-//  * t1 = PW over C's row: butterfly per 32-chunk, tree over chunks (== PW);
-//  * s = t1 - t2 is compared with K_k * beta_g, beta_g = the norm of the
-//    group's own x slice -- an aligned node of the PW tree of ||x||^2, so
-//    beta_g <= beta exactly (monotone rounding, R12).  |s| <= K
-//    beta_g proves the block clean; anything else becomes a candidate;
-//  * the group's x^2 subtree goes to gsum[g].
-// k_general: every group k_lean cannot take (b_s < 32, the ragged last group,
-// segments beyond the staging capacity, unaligned operands) -- one warp per
-// group, operands read directly from global memory.
+// Which kernel runs a group (plan at encode, abft.cu plan_fused):
+//  * k_stream (kernels_stream.cuh): row-regular matrices --
+//    position-map records, a warp-specialized TMA ring; the default for
+//    every stencil;
+//  * k_lean (below): the slot-map compact-C records (ABFT_NO_POS, or when
+//    the position map cannot describe the matrix);
+//  * k_irr (kernels_irr.cuh): groups with rows of 33..1024 entries;
+//  * k_hub (below): aligned 1024-entry chunks of hub rows / hub C rows;
+//  * k_general (below): everything else (b_s < 32, the ragged last group,
+//    groups owning hub rows, unaligned operands) -- one warp per group,
+//    operands read directly from global memory.
+//
+// k_lean (b_s = 32): a persistent grid; each warp owns a contiguous range of
+// groups and pipelines them through per-warp shared-memory stages filled by
+// TMA 1-D bulk copies (cp.async.bulk + mbarrier transaction counts, L2
+// evict-first) of the group's record, x slice, A values and columns.  Per
+// group: lane l = row 32g + l computes y_i as an in-register PW tree of its
+// gathered products (rows <= 32 entries); each gathered x_j replaces a_ij in
+// the staged values, where the C pass finds it through the record's slot
+// map (t1 = PW over C's row); t2, t1 and the group's x^2 subtree share one
+// reduce-scatter butterfly; s = t1 - t2 is compared with K_k * beta_lo,
+// beta_lo <= beta exactly (an aligned node of the PW tree of ||x||^2,
+// rounded down; R12): |s| <= K beta_lo proves the block clean,
+// anything else becomes a candidate; the x^2 subtree goes to gsum[g].
 // k_finish (one PDL launch after them) confirms the candidates against
 // tau_k = K_k beta, beta = sqrt(PW(gsum)) computed by all SMs only when a
 // candidate exists (or taken from x_norm), writes the flagged-block list and
