@@ -58,6 +58,8 @@ def load_peaks():
 
 def fused_kernel_name(info) -> str:
     """Name of the fused multiply+detect launch(es) the plan runs (abft_info)."""
+    if info.get("block_size", 32) > 32:
+        return "k_bigblock<CHECK>"
     if info.get("stream"):
         k = f"k_stream<CHECK> (G={info.get('stream_g')}, {info.get('stream_stages')} stages)"
         return k + (" + k_general<CHECK>" if info.get("general_groups") else "")
