@@ -1030,7 +1030,7 @@ abft_status plan_stream(abft_ctx *h, const std::vector<int32_t> &rp, const std::
     int NS = 0;
     while (NS < 8 && fixed + (size_t)(NS + 1) * c.stage_bytes <= budget) ++NS;
     if (const char *e = getenv("ABFT_STREAM_NS")) NS = std::min(NS, std::max(2, atoi(e)));
-    if (NS < 2 || (ABFT_STREAM_DEPTH == 3 && h->pos_S <= 8 && NS < 3)) continue;
+    if (NS < 2) continue;
     c.NS = NS;
     c.ring_off = 128;
     c.xs_off = 128 + (uint32_t)NS * c.stage_bytes;

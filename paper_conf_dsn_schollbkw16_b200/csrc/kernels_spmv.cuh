@@ -48,8 +48,9 @@ template <> struct CType<CF_F32> { using T = float; };
 constexpr int kLeanWarps = 4;  // warps per CTA of k_lean (<= 4)
 // Timing experiments only (scripts/exp_libs.sh; results are NOT the method):
 // 1 = no C products, 2 = C neither staged nor multiplied, 3 = no butterflies,
-// 4 = no test, 5 = 1 + 3 + 4, 6 = k_stream without x gathers, 7 = k_stream SHORT
-// without the C pass (no position stores, no t1 products).  0 (the default)
+// 4 = no test, 5 = 1 + 3 + 4, 6 = k_stream without x gathers, 8 = k_stream
+// SHORT per-phase cycle counters (scripts/phase_probe.py), 9 = PCG update
+// without the division.  0 (the default)
 // = the method.
 #ifndef ABFT_EXP
 #define ABFT_EXP 0

@@ -486,7 +486,6 @@ struct ShortA {
   int ml;    // longest row of the group (uniform)
   bool uni;  // every row of the group has ml entries (uniform)
   bool hit;  // INJECT: the group may hold a round-0 fault (inj_group_hit)
-  bool stg;  // came from a loaded (non-terminal) stage the warp must release (depth 3)
   double xj[8];
   double xi;
 };
@@ -581,7 +580,6 @@ __device__ __forceinline__ void short_finish(const SpmvArgs &a, const StreamCfg 
   const int32_t W[8] = {w0.x, w0.y, w0.z, w0.w, w1.x, w1.y, w1.z, w1.w};
   double q0 = kAbsent;
   // x_j -> C position W[j] + lane (slots past the row land in the trash)
-  if (ABFT_EXP != 7) {  // 7: timing experiment only, no C pass (wrong t1)
 #pragma unroll
   for (int j = 0; j < 7; ++j) sts_f64(xs_addr<CF>(xs, W[j] + lane), A.xj[j]);
   if (A.ml > 7) sts_f64(xs_addr<CF>(xs, W[7] + lane), A.xj[7]);
@@ -602,7 +600,6 @@ __device__ __forceinline__ void short_finish(const SpmvArgs &a, const StreamCfg 
       u8[2 * u + 1] = dmul(cv[2 * u + 1], x1);
     }
     q0 = tree<8>(u8);
-  }
   }
   PH_MARK(f2);
   PH_ADD(4, f1, f2);
@@ -666,9 +663,6 @@ __device__ __forceinline__ void short_bfly(const SpmvArgs &a, ShortP &P, int lan
   PH_ADD(5, f2, f3);
 }
 
-#ifndef ABFT_STREAM_DEPTH
-#define ABFT_STREAM_DEPTH 2  // SHORT consumers: groups whose gathers are in flight (2 or 3)
-#endif
 #ifndef ABFT_STREAM_MINB
 #define ABFT_STREAM_MINB 2  // resident CTAs per SM the register budget targets
 #endif
@@ -799,53 +793,7 @@ __global__ void ABFT_STREAM_BOUNDS k_stream(const SpmvArgs a) {
   const uint32_t xs = smem_u32(smem + c.xs_off + (size_t)warp * c.xs_bytes);
   int s = 0;
   uint32_t fph = 0;  // parity of the next completion of full[s]
-  if constexpr (SHORT && ABFT_STREAM_DEPTH == 3) {
-    // three phase-A states in rotation: the gathers of the groups two and
-    // one stages ahead are in flight while a group is finished (needs NS >= 3)
-    const double *xg = a.x;
-    ShortA sa, sb, sc;
-    ShortP P;
-    P.on = false;
-    unsigned long long ph[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-    (void)ph;
-    int ls = 0, fs = 0;  // next stage to load / to release
-    uint32_t lph = 0;    // parity of the next completion of full[ls]
-    bool done = false;
-    auto load_next = [&](ShortA &nx) {
-      nx.g = -1;
-      nx.stg = false;
-      if (done) return;
-      const unsigned char *st1 = ring + (size_t)ls * c.stage_bytes;
-      mbar_wait_sleep(full + ls, lph);
-      const int32_t *hdr1 = reinterpret_cast<const int32_t *>(st1);
-      const int32_t g0n = hdr1[3 * G + 3];
-      if (g0n < 0) {
-        done = true;
-        return;
-      }
-      nx.stg = true;
-      if (warp < hdr1[3 * G + 4])
-        short_load<CHECK, INJECT>(a, c, xg, (int64_t)g0n + warp, warp, st1, lane, nx);
-      if (++ls == NS) {
-        ls = 0;
-        lph ^= 1u;
-      }
-    };
-    auto step = [&](ShortA &cu, ShortA &nx) -> bool {
-      if (!cu.stg) return false;
-      load_next(nx);
-      if (cu.g >= 0) short_finish<CHECK, INJECT, CF>(a, c, cu, xs, lane, P, ph);
-      if (CHECK && P.on) short_bfly<INJECT>(a, P, lane, ph);
-      __syncwarp();
-      if (lane == 0) mbar_arrive(empty + fs);
-      if (++fs == NS) fs = 0;
-      return true;
-    };
-    load_next(sa);
-    load_next(sb);
-    while (step(sa, sc) && step(sb, sa) && step(sc, sb)) {
-    }
-  } else if constexpr (SHORT) {
+  if constexpr (SHORT) {
     // ping-pong between two phase-A states (no register copies): each step
     // loads the next stage's group into one state and finishes the other
     const double *xg = a.x;
