@@ -627,7 +627,10 @@ __device__ __forceinline__ void group_general(const SpmvArgs &a, int64_t g, int 
 }
 
 template <bool CHECK, bool INJECT>
-__global__ void __launch_bounds__(kGenWarps * 32, 4) k_general(const SpmvArgs a) {
+#ifndef ABFT_GEN_MINB
+#define ABFT_GEN_MINB 4
+#endif
+__global__ void __launch_bounds__(kGenWarps * 32, ABFT_GEN_MINB) k_general(const SpmvArgs a) {
   __shared__ double scr_all[kGenWarps][kScr];
   if (skip_call(a)) return;
   const int lane = threadIdx.x & 31;
