@@ -392,3 +392,34 @@ def test_dist_pcg_processes(O, torch_cuda, tmp_path, world, variant):
         assert np.array_equal(np.load(tmp_path / f"h{r}.npy").view(np.uint64),
                               ref.res_hist.view(np.uint64))
     assert np.array_equal(x.view(np.uint64), ref.x.view(np.uint64))
+
+
+@pytest.mark.parametrize("eager", [False, True])
+@pytest.mark.parametrize("variant", ["pcg", "cg1"])
+def test_nccl_world1_pcg_graph_and_eager(O, torch_cuda, variant, eager, monkeypatch):
+    """abft_dist_pcg replays a captured 16-iteration graph for fault-free
+    solves (ABFT_DIST_PCG_EAGER=1: eager sequencing); both give the oracle's
+    bits, a second solve on the same buffers reuses the cached graph, and a
+    max_iter that is not a multiple of 16 stops exactly there."""
+    from paper_conf_dsn_schollbkw16_b200 import Dist, dist_unique_id
+    torch = torch_cuda
+    if eager:
+        monkeypatch.setenv("ABFT_DIST_PCG_EAGER", "1")
+    A = G.laplacian_3d_7pt(20)
+    d = Dist(0, 1, [0, A.n], dist_unique_id())
+    ds = PL.DistSpmv(d, PL.shard_rows(A, 0, A.n))
+    b = O.spmv(A, G.uniform_vector(A.n, 43))
+    x0 = G.uniform_vector(A.n, 44)
+    f = O.pcg_cg1_ranks if variant == "cg1" else O.pcg_ranks
+    for max_iter in (0, 0, 21):
+        pref = f(A, b, x0, [(0, A.n)], tol=1e-6, max_iter=max_iter)
+        xd = torch.from_numpy(x0.copy()).cuda()
+        hist = torch.zeros(10 * A.n + 1, dtype=torch.float64, device="cuda")
+        p = PL.DistPcg(ds, True, variant)
+        state, st = p.solve(None, torch.from_numpy(b).cuda(), xd, A.n, tol=1e-6,
+                            max_iter=max_iter, res_hist=hist)
+        assert st["iters"] == pref.iters, (max_iter, st["iters"], pref.iters)
+        assert state == (1 if max_iter == 0 else 3), state
+        assert np.array_equal(hist[: st["iters"] + 1].cpu().numpy().view(np.uint64),
+                              pref.res_hist.view(np.uint64))
+        assert np.array_equal(xd.cpu().numpy().view(np.uint64), pref.x.view(np.uint64))
