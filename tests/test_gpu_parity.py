@@ -635,3 +635,25 @@ def test_popularity_ordered_x(O, torch_cuda, name, c_csr, monkeypatch):
     c.run(G.uniform_vector(A.n, 33), rate=dict(seed=5, lam=1e-3, targets=0b111, call=1))
     monkeypatch.setenv("ABFT_COLPERM", "0")
     assert encode(A, c_csr=c_csr).info()["col_perm"] == 0
+
+
+def test_popularity_ordered_x_unaligned_operand(O, torch_cuda, monkeypatch):
+    # k_xperm's scalar path (x not 16-B aligned: a view one element into a
+    # buffer) gives the same bits as the oracle
+    from paper_conf_dsn_schollbkw16_b200 import CHECK, encode
+    monkeypatch.setenv("ABFT_COLPERM", "1")
+    torch = torch_cuda
+    A = MATRICES["rmat11"]()
+    h = encode(A)
+    assert h.info()["col_perm"] == 1
+    x = G.uniform_vector(A.n, 61)
+    enc = O.encode(A, 32)
+    ref = O.abft_spmv(A, enc, x, None, 4)
+    buf = torch.zeros(A.n + 1, dtype=torch.float64, device="cuda")
+    buf[1:] = torch.from_numpy(x).cuda()
+    xv = buf[1:]
+    assert xv.data_ptr() % 16 != 0
+    y = h.spmv(xv, mode=CHECK)
+    torch.cuda.synchronize()
+    assert_bits_equal(y.cpu().numpy(), ref.y_pre, "y")
+    assert np.array_equal(h.flags(0), ref.flags[0])
