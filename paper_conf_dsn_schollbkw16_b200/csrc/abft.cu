@@ -18,6 +18,7 @@
 #include "kernels_dense.cuh"
 #include "kernels_bigblock.cuh"
 #include "kernels_dist.cuh"
+#include "kernels_pcgfin.cuh"
 #include "kernels_perm.cuh"
 
 #include <cub/device/device_radix_sort.cuh>
@@ -195,6 +196,7 @@ struct abft_ctx {
   double *pcg = nullptr;  // r, z, p, q, d : 5 n
   double *pcg_part = nullptr;
   double *pcg_pq = nullptr;  // [ngroups] p.q group partials of the fused SpMV epilogue
+  abft::PcgArgs *pcg_args_dev = nullptr;  // device copy of the solve's PcgArgs (k_finish's p.q)
   // abft_pcg's device-resident loop: the instantiated graph, the key of
   // what it bakes in (PcgGraphKey), its capture stream
   cudaGraphExec_t pcg_exec = nullptr;

@@ -97,6 +97,8 @@ struct StreamCfg {
   int32_t defer;         // SHORT consumers: a group's butterfly runs one step later
 };
 
+struct PcgArgs;  // kernels_pcg.cuh
+
 struct SpmvArgs {
   int64_t n;
   int64_t nnz;
@@ -123,6 +125,9 @@ struct SpmvArgs {
   // into the SpMV epilogue, a 32-row aligned node of the global PW tree;
   // correction rounds rewrite it for the blocks they recompute, b_s = 32)
   double *pq;
+  // abft_pcg, protected: k_finish also completes PW over the p.q group
+  // partials and the PCG's alpha step (no separate k_pcg_dotg launch)
+  const PcgArgs *pcga;
   double *bpart;          // [ceil(ngroups / 1024)] beta partials (k_finish)
   int32_t *n_cand;        // candidate count (reset by k_finish)
   int32_t *cand;          // [nb]
@@ -1555,6 +1560,9 @@ __device__ __forceinline__ void block_rounds(const SpmvArgs &a, int64_t k, int r
 //    No barrier between rounds (a block's rounds depend on no other block).
 //    Matrices with hub rows and few candidates: CTA 0 alone runs the rounds
 //    round by round, each round's hub chunk sums spread over its warps.
+// kernels_pcgfin.cuh: the p.q completion k_finish runs for abft_pcg
+__device__ void pcg_fin_dot(const SpmvArgs &a, double *s_red, bool solo);
+
 template <bool INJECT, bool CONFIRM>
 __global__ void __launch_bounds__(256) k_finish(const SpmvArgs a, int rounds) {
   __shared__ double s_red[256];
@@ -1575,6 +1583,7 @@ __global__ void __launch_bounds__(256) k_finish(const SpmvArgs a, int rounds) {
         if (a.x_norm) *a.beta = __ldcg(a.x_norm);
         *a.beta_valid = a.x_norm ? 1 : 0;
       }
+      if (a.pcga) pcg_fin_dot(a, s_red, false);  // every CTA takes part (no barrier)
       return;
     }
     if (blockIdx.x == 0 && threadIdx.x == 0)
@@ -1607,7 +1616,11 @@ __global__ void __launch_bounds__(256) k_finish(const SpmvArgs a, int rounds) {
       if (lane == 0) a.flags[atomicAdd(a.n_flags, 1)] = kk;
       if (!hub_solo) block_rounds<INJECT>(a, kk, rounds, lane, beta);
     }
-    if (!hub_solo) return;
+    if (!hub_solo) {
+      // the corrections rewrote the p.q partials of their groups
+      if (a.pcga && grid_sync(a.gbar)) pcg_fin_dot(a, s_red, false);
+      return;
+    }
     __syncthreads();  // round 0's list complete
     nitems = __ldcg(a.n_flags);
     items = a.flags;
@@ -1668,6 +1681,7 @@ __global__ void __launch_bounds__(256) k_finish(const SpmvArgs a, int rounds) {
     }
     __syncthreads();
   }
+  if (a.pcga) pcg_fin_dot(a, s_red, true);  // CTA 0 alone (the others left after the barrier)
 }
 
 }  // namespace abft

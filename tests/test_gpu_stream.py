@@ -181,3 +181,48 @@ def test_stream_deferred_butterfly(O, torch_cuda, name, defer, monkeypatch):
                        [1 << 62, 1 << 57, 1 << 61, 1 << 60])
     assert c.run(G.uniform_vector(A.n, 53), plan=plan).flagged.size >= 3
     c.run(G.uniform_vector(A.n, 54), rate=dict(seed=3, lam=1e-3, targets=0b111, call=2))
+
+
+def _arrow_laplacian(n3=14):
+    # SPD: the 7-pt Laplacian plus an "arrow" -- row and column 0 dense with
+    # small entries (row 0 has n entries > 1024: a hub row on the general
+    # path) -- and a diagonal raised enough to stay diagonally dominant
+    L = G.laplacian_3d_7pt(n3)
+    n = L.n
+    rows = [np.arange(L.row_ptr[i], L.row_ptr[i + 1]) for i in range(n)]
+    cols, vals, rp = [], [], [0]
+    for i in range(n):
+        c = L.col[rows[i]].tolist()
+        v = L.val[rows[i]].tolist()
+        if i == 0:
+            lap = dict(zip(c, v))  # keep the Laplacian's own row-0 entries (symmetric)
+            c = list(range(n))
+            v = [lap.get(j, 1e-3) for j in range(n)]
+            v[0] = 6.0 + 1e-3 * n
+        elif 0 not in c:
+            c = [0] + c
+            v = [1e-3] + v
+        cols += c
+        vals += v
+        rp.append(len(cols))
+    return G.CSR(np.array(rp, np.int32), np.array(cols, np.int32), np.array(vals), "arrow")
+
+
+@pytest.mark.parametrize("inj", [None, dict(seed=5, lam=2e-6, targets=0b111)])
+def test_stream_pcg_with_hub_row(O, torch_cuda, inj, monkeypatch):
+    # position-map records with one hub row (> 1024 entries, k_hub + k_general)
+    # inside a PCG: few candidates per faulty SpMV take k_finish's CTA-0
+    # path, which also completes the p.q sum (kernels_pcgfin.cuh)
+    from test_gpu_parity import _pcg_case
+    from paper_conf_dsn_schollbkw16_b200 import encode
+    monkeypatch.setenv("ABFT_FORCE_POS", "1")  # the arrow column makes every row an exception
+    A = _arrow_laplacian()
+    info = encode(A).info()
+    assert info["stream"] == 1 and info["hub_chunks"] > 0, info
+    ref, status, st, x, hist = _pcg_case(O, torch_cuda, A, inj)
+    assert status == ref.status == 0
+    assert st["iters"] == ref.iters and st["flagged_blocks"] == ref.flagged_blocks
+    assert_bits_equal(hist, ref.res_hist, "residual history")
+    assert_bits_equal(x, ref.x, "x")
+    if inj:
+        assert ref.flagged_blocks > 0
