@@ -405,6 +405,9 @@ abft_status abft_pcg_dist_status(abft_handle_t h, int32_t *state, abft_pcg_stats
  *   of the global matrix; inj->call counts this rank's SpMVs (rate mode: the
  *   seed is the caller's, e.g. distinct per rank); variant 0 = textbook
  *   PCG (two reductions per iteration), 1 = single reduction (R29).
+ *   Fault-free solves replay a CUDA graph of 16 captured iterations (kernels,
+ *   NCCL calls, cross-stream events), cached per buffer set; faulty solves
+ *   are sequenced eagerly (ABFT_DIST_PCG_EAGER=1 forces eager sequencing).
  *   Synchronises; every rank returns the same status.
  * abft_halo_plan (host only, no GPU): the local column order of abft_dist_
  *   encode for host arrays -- local_col [nnz], *n_below / *n_above, per peer
