@@ -226,3 +226,36 @@ def test_stream_pcg_with_hub_row(O, torch_cuda, inj, monkeypatch):
     assert_bits_equal(x, ref.x, "x")
     if inj:
         assert ref.flagged_blocks > 0
+
+
+def test_stream_without_pdl_subprocess(torch_cuda):
+    # ABFT_NO_PDL=1 (plain launches instead of programmatic dependent launch;
+    # read once per process): the same bits as the oracle
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    code = (
+        "import numpy as np, torch\n"
+        "from oracle import oracle as O\n"
+        "from paper_conf_dsn_schollbkw16_b200 import CHECK, encode, inputs as G\n"
+        "A = G.laplacian_3d_7pt(24)\n"
+        "x = G.uniform_vector(A.n, 42)\n"
+        "plan = G.FaultPlan([0, 0], [0, 1], [100, 7], [1 << 62, 1 << 61])\n"
+        "ref = O.abft_spmv(A, O.encode(A, 32), x, O.Inject.from_plan(plan), 4)\n"
+        "from paper_conf_dsn_schollbkw16_b200 import Inject\n"
+        "h = encode(A, 32)\n"
+        "assert h.info()['stream'] == 1\n"
+        "xd = torch.from_numpy(x).cuda()\n"
+        "y = h.spmv(xd, inject=Inject.from_plan(plan), mode=CHECK)\n"
+        "torch.cuda.synchronize()\n"
+        "assert np.array_equal(y.cpu().numpy().view(np.uint64), ref.y_pre.view(np.uint64))\n"
+        "assert np.array_equal(h.flags(0), ref.flags[0])\n"
+        "h.correct(xd, y, 4, inject=Inject.from_plan(plan))\n"
+        "torch.cuda.synchronize()\n"
+        "assert np.array_equal(y.cpu().numpy().view(np.uint64), ref.y.view(np.uint64))\n"
+        "print('ok')\n")
+    env = dict(os.environ, ABFT_NO_PDL="1", PYTHONPATH=root)
+    r = subprocess.run([sys.executable, "-c", code], cwd=root, env=env, capture_output=True,
+                       text=True, timeout=600)
+    assert r.returncode == 0 and "ok" in r.stdout, r.stderr[-2000:]
