@@ -529,14 +529,16 @@ def test_config0_single_fault_sweep(O, torch_cuda):
     assert flagged_runs > 500
 
 
-@pytest.mark.parametrize("name", ["7pt128", "27pt128", "rmat20"])
+@pytest.mark.parametrize("name", ["7pt128", "27pt128", "rmat20", "7pt192"])
 def test_bench_workloads_full_size(O, torch_cuda, name):
     # the bench's own workloads at full size, in the launch configuration
     # bench.py times (7-pt 128^3 = configs[1]: k_lean SHORT; 27-pt 128^3: the
     # general k_lean; R-MAT scale 20: k_irr + k_hub + k_general), every output
     # against the oracle with faults in y, t1 and t2
+    # (7-pt 192^3, the PCG matrix: x > 40 MB, so the deferred-butterfly
+    # instantiation runs)
     A = {"7pt128": lambda: G.laplacian_3d_7pt(128), "27pt128": lambda: G.stencil_3d_27pt(128),
-         "rmat20": lambda: G.rmat(20, 16, 1)}[name]()
+         "rmat20": lambda: G.rmat(20, 16, 1), "7pt192": lambda: G.laplacian_3d_7pt(192)}[name]()
     c = Case(O, torch_cuda, A)
     ref = c.run(G.uniform_vector(A.n, 42))
     assert ref.flagged.size == 0
