@@ -659,3 +659,37 @@ def test_popularity_ordered_x_unaligned_operand(O, torch_cuda, monkeypatch):
     torch.cuda.synchronize()
     assert_bits_equal(y.cpu().numpy(), ref.y_pre, "y")
     assert np.array_equal(h.flags(0), ref.flags[0])
+
+
+@pytest.mark.parametrize("name", ["27pt256", "rmat24"])
+def test_full_size_properties(torch_cuda, name):
+    # configs[3] / configs[2] at full size in the bench's launch configuration
+    # (too large for the oracle within seconds): properties that hold at any
+    # size -- no flag on a fault-free call (the bound); every injected
+    # fault far above tau flagged and localized to its own block (y rows)
+    # or its block (t1 / t2); the correction restores the fault-free y bit
+    # for bit; the unprotected kernel computes the same y.
+    from paper_conf_dsn_schollbkw16_b200 import CHECK, Inject, encode
+    torch = torch_cuda
+    A = {"27pt256": lambda: G.stencil_3d_27pt(256), "rmat24": lambda: G.rmat(24, 16, 1)}[name]()
+    h = encode(A, 32)
+    x = torch.from_numpy(G.uniform_vector(A.n, 42)).cuda()
+    y0 = h.spmv(x, mode=CHECK)
+    torch.cuda.synchronize()
+    assert h.flags(0).size == 0
+    yp = h.spmv(x, mode=0)
+    torch.cuda.synchronize()
+    assert torch.equal(yp.view(torch.int64), y0.view(torch.int64))
+    nb = (A.n + 31) // 32
+    rows = [5, A.n // 3, A.n - 1]
+    blocks = [nb // 2 + 1, nb - 2]
+    plan = G.FaultPlan([0] * 5, [0, 0, 0, 1, 2], rows + blocks,
+                       [1 << 62, 1 << 62, 1 << 62, 1 << 62, 1 << 62])
+    y = h.spmv(x, inject=Inject.from_plan(plan), mode=CHECK)
+    torch.cuda.synchronize()
+    want = sorted({r // 32 for r in rows} | set(blocks))
+    assert sorted(h.flags(0).tolist()) == want
+    h.correct(x, y, 4, inject=Inject.from_plan(plan))
+    torch.cuda.synchronize()
+    assert h.flags(1).size == 0
+    assert torch.equal(y.view(torch.int64), y0.view(torch.int64))
